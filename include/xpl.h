@@ -1,0 +1,195 @@
+/* include/xpl.h -- the C-ABI of the B200-native XPlacer recording + diagnosis
+ * runtime (libxpl.so).
+ *
+ * Paper: P. Pirkelbauer, P.-H. Lin, T. Vanderbruggen, C. Liao, "XPlacer:
+ * Automatic Analysis of Data Access Patterns on Heterogeneous CPU/GPU
+ * Systems", IPDPS 2020.  "P:Lnnn" cites line nnn of the paper's text;
+ * "Dnn" cites a reading of DESIGN.md §3 (= SURVEY.md §8(c)).
+ *
+ * Conventions for every entry point:
+ *  - all functions return xpl_status; nothing throws across the ABI;
+ *  - pointers to user memory are only used as numbers: the library never
+ *    dereferences user data (only the address is looked up);
+ *  - "host" arguments are host pointers; the library copies what it needs
+ *    before returning, so the caller may reuse its buffers at once;
+ *  - one host thread per context; one context per process and GPU.  With
+ *    world > 1 every rank makes every call, in the same order;
+ *  - `stream` arguments are cudaStream_t values passed as void*.
+ */
+#ifndef XPL_H
+#define XPL_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  XPL_OK = 0,
+  XPL_ERR_INVALID_ARG = 1,    /* NULL pointer, zero size, unknown enum, cap too small */
+  XPL_ERR_OOM = 2,            /* shadow pool / table / staging capacity exhausted   */
+  XPL_ERR_OVERLAP = 3,        /* xpl_register_alloc intersects a live allocation     */
+  XPL_ERR_UNKNOWN_PTR = 4,    /* xpl_free of a pointer that is no live base          */
+  XPL_ERR_STATE = 5,          /* call not allowed now (e.g. diagnose in an epoch)    */
+  XPL_ERR_CUDA = 6,           /* a CUDA runtime call failed                           */
+  XPL_ERR_NCCL = 7,           /* a collective failed (world > 1)                      */
+  XPL_ERR_DEVICE_OVERFLOW = 8 /* a device-side capacity was exceeded                  */
+} xpl_status;
+
+/* How the memory was allocated; stored in the shadow memory table and
+ * used to gate the anti-pattern flags (D8). */
+typedef enum {
+  XPL_ALLOC_DEVICE = 0,  /* cudaMalloc               */
+  XPL_ALLOC_MANAGED = 1, /* cudaMallocManaged        */
+  XPL_ALLOC_HOST = 2     /* malloc/new/cudaMallocHost */
+} xpl_alloc_kind;
+
+/* traceR / traceW / traceRW (Table I).  RW = read, then write (D6). */
+typedef enum { XPL_ACC_R = 1, XPL_ACC_W = 2, XPL_ACC_RW = 3 } xpl_acc_kind;
+
+/* The cudaMemcpy / cudaMemset wrappers of `#pragma xpl replace`.
+ * H2D = a CPU write of dst, D2H = a CPU read of src; H2H = CPU read of src
+ * and write of dst; D2D and MEMSET_DEV = GPU accesses in their own epoch, or in the
+ * open one (D7, D19). */
+typedef enum {
+  XPL_COPY_H2D = 0,
+  XPL_COPY_D2H = 1,
+  XPL_COPY_H2H = 2,
+  XPL_COPY_D2D = 3,
+  XPL_MEMSET_DEV = 4
+} xpl_copy_dir;
+
+/* One host-side access as the host tracer saw it (16 bytes).  An access marks every
+ * 32-bit word overlapping [addr, addr+size) of the allocation holding `addr`,
+ * clipped to that allocation (D1, D2, D18). */
+typedef struct {
+  uint64_t addr;
+  uint32_t size; /* bytes, >= 1; any size (large sizes are ranges) */
+  uint32_t kind; /* xpl_acc_kind */
+} xpl_host_access;
+
+/* XplAllocData: names an allocation in the report. */
+typedef struct {
+  const void* addr;
+  const char* expr;
+  uint32_t elem_size;
+} xpl_name;
+
+typedef struct {
+  int device;            /* CUDA device ordinal                                   */
+  int rank, world;       /* world > 1 => address-range sharding over the ranks    */
+  void* nccl_comm;       /* ncclComm_t when world > 1, else NULL                  */
+  uint64_t pool_words;   /* shadow pool capacity in words (1 byte each)   */
+  uint64_t dirty_cap;    /* dirty-list capacity, in shadow u32s                    */
+  uint64_t staging_recs; /* host-record staging capacity (records)                */
+  uint32_t max_rows;     /* capacity of the allocation table                      */
+} xpl_config;
+
+/* Diagnosis parameters. */
+typedef struct {
+  uint32_t density_threshold_pct; /* default 50 ("e.g., 50%"); "<=" per Eq. P:L102 (D11) */
+  uint64_t block_words;           /* 0 = the whole allocation is one block (D12)           */
+  uint64_t min_run_words;         /* minimum transfer run, default 256 (D16); 0 acts as 1  */
+} xpl_diag_params;
+
+/* Report flags (the three anti-patterns of §III-A, plus "unused"). */
+#define XPL_PAT_ALTERNATING 1u  /* managed, CPU and GPU on one word, >= 1 a write */
+#define XPL_PAT_LOW_DENSITY 2u  /* device/managed block with <= threshold density  */
+#define XPL_PAT_UNNEEDED_H2D 4u /* device: CPU-written run the GPU never read     */
+#define XPL_PAT_UNNEEDED_D2H 8u /* device: CPU read back a run the GPU never updated       */
+#define XPL_PAT_UNUSED 16u      /* no access in the interval (Table II Backprop)   */
+
+/* One row of the diagnosis (Fig. 4).  Counts are numbers of words,
+ * each counted at most once per column. */
+typedef struct {
+  uint64_t id, base, bytes, words;
+  uint32_t kind, live, name_idx /* index into the xpl_name array, or 0xFFFFFFFF */, flags;
+  uint64_t w_c, w_g;                /* Fig. 4 "write counts C G"                   */
+  uint64_t r_cc, r_cg, r_gc, r_gg;  /* Fig. 4 "C>C C>G G>C G>G" (origin>reader)    */
+  uint64_t any_acc, gpu_acc, alternating;
+  uint64_t density_pct_any, density_pct_gpu; /* floor(100*accessed/words) (D10, D22) */
+  uint64_t low_density_blocks, low_density_words;
+  uint64_t h2d_unused_runs, h2d_unused_words;
+  uint64_t d2h_unneeded_runs, d2h_unneeded_words;
+  uint64_t ever_accessed; /* any access since registration */
+} xpl_alloc_report;
+
+typedef struct xpl_ctx xpl_ctx;
+struct xpl_dev_ctx; /* defined in xpl_device.cuh */
+
+/* Counters the runtime keeps about itself (not part of the paper's output). */
+typedef struct {
+  uint64_t epochs, folds, fold_full_scans, host_records, host_records_packed,
+      merge_segments, range_segments, diagnoses, dirty_max;
+} xpl_stats;
+
+/* Create a context on cfg->device.  *out is owned by the caller until
+ * xpl_finalize.  Zero fields of cfg take defaults (pool_words 2^28, dirty_cap
+ * 2^24, staging_recs 2^22, max_rows 4096).  Allocates the shadow pool in HBM. */
+xpl_status xpl_init(const xpl_config* cfg, xpl_ctx** out);
+xpl_status xpl_finalize(xpl_ctx* ctx);
+
+/* The allocation wrappers.  register: ceil(bytes/4) zeroed records
+ * (last writer = CPU, D3); OVERLAP if [ptr, ptr+bytes) intersects a live row;
+ * STATE inside an open GPU epoch.  free: UNKNOWN_PTR unless ptr is a live
+ * base; the row stops matching lookups now and is reported once more at the
+ * next diagnose before its shadow is recycled (D17). */
+xpl_status xpl_register_alloc(xpl_ctx* ctx, const void* ptr, size_t bytes, xpl_alloc_kind kind);
+xpl_status xpl_free(xpl_ctx* ctx, const void* ptr);
+
+/* GPU epoch delimiters around kernel launches (traceKernelLaunch).
+ * Epochs nest; the epoch is the outermost begin..end (D19).  begin orders
+ * `stream` after all pending runtime work; end orders the runtime after
+ * `stream` (and every stream that began inside the epoch) and enqueues the
+ * epoch close (fold).  Nothing synchronises the host.  end without an open
+ * epoch -> STATE. */
+xpl_status xpl_kernel_begin(xpl_ctx* ctx, void* stream);
+xpl_status xpl_kernel_end(xpl_ctx* ctx, void* stream);
+
+/* Host tracer batch (the !__CUDA_ARCH__ branch of traceR/traceW/traceRW).
+ * recs: host array of n records in program order.  Untracked addresses are
+ * ignored.  Inside an open GPU epoch the records are applied after
+ * the epoch closes (D20). */
+xpl_status xpl_record_host(xpl_ctx* ctx, const xpl_host_access* recs, size_t n);
+
+/* The transfer wrappers (D7).  dst/src are the cudaMemcpy arguments. */
+xpl_status xpl_record_copy(xpl_ctx* ctx, const void* dst, const void* src, size_t bytes,
+                           xpl_copy_dir dir);
+
+/* tracePrint: analyse every live row and every row freed since the
+ * last reset, write one report per row in id order into out[0..cap), set
+ * *n_out.  INVALID_ARG with *n_out = rows needed if cap is too small.  With
+ * reset != 0 the interval bits are cleared (the last writer is kept, D4) and
+ * freed rows are dropped.  STATE inside an open epoch.  Blocks until done.
+ * params NULL = defaults; names may be NULL when n_names == 0. */
+xpl_status xpl_diagnose(xpl_ctx* ctx, const xpl_diag_params* params, const xpl_name* names,
+                        size_t n_names, xpl_alloc_report* out, size_t cap, size_t* n_out,
+                        int reset);
+
+/* The device-side context the __device__ hooks of xpl_device.cuh use: copies
+ * it into *out (a host struct of device pointers; valid until xpl_finalize). */
+xpl_status xpl_get_device_ctx(xpl_ctx* ctx, struct xpl_dev_ctx* out);
+
+/* Per-word records of the live row whose base is `base`, words
+ * [word0, word0+n), copied into the host array out[n] (access maps, Fig. 5/7/8/10;
+ * also the sampled-parity hook of the tests).  Blocks until done. */
+xpl_status xpl_shadow_dump(xpl_ctx* ctx, const void* base, uint64_t word0, uint64_t n,
+                           uint8_t* out);
+
+/* Apply every staged host record now (normally done lazily at kernel_begin,
+ * diagnose and when staging fills up).  Asynchronous. */
+xpl_status xpl_flush(xpl_ctx* ctx);
+/* Wait for all runtime work enqueued so far. */
+xpl_status xpl_sync(xpl_ctx* ctx);
+/* The runtime's own stream (cudaStream_t as void*), e.g. for timing events. */
+xpl_status xpl_runtime_stream(xpl_ctx* ctx, void** stream);
+xpl_status xpl_get_stats(xpl_ctx* ctx, xpl_stats* out);
+
+const char* xpl_status_string(xpl_status s);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* XPL_H */

@@ -1,0 +1,828 @@
+// runtime.cu -- host side of the B200-native XPlacer runtime: the C-ABI of
+// include/xpl.h.  Owns the shadow memory table, the shadow pool,
+// the epoch state machine around kernel launches, host-record staging
+// with run-length coalescing (host tracer) and the diagnose driver
+// (tracePrint).  Every data-parallel step runs in kernels.cu or in the
+// inlined hooks of xpl_device.cuh; this file only orders and launches them.
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <string.h>
+
+#include <algorithm>
+#include <map>
+#include <new>
+#include <vector>
+
+#include "xpl_internal.h"
+
+using namespace xpl;
+
+#define CK(x)                                      \
+  do {                                             \
+    if ((x) != cudaSuccess) return XPL_ERR_CUDA;   \
+  } while (0)
+
+namespace {
+
+struct Row {
+  uint64_t id, base, bytes, words, off, span;  // span = pool words reserved
+  uint32_t kind;
+  bool live, dropped, ever;
+};
+
+// First-fit allocator of shadow-pool ranges (16-word granules so every row
+// starts on a 16-byte boundary for the vector loads of diagnose).
+struct PoolAlloc {
+  std::map<uint64_t, uint64_t> free_;  // off -> len
+  void init(uint64_t cap) { free_.clear(); free_[0] = cap; }
+  bool alloc(uint64_t n, uint64_t* off) {
+    for (auto it = free_.begin(); it != free_.end(); ++it) {
+      if (it->second >= n) {
+        *off = it->first;
+        const uint64_t rest = it->second - n, o = it->first + n;
+        free_.erase(it);
+        if (rest) free_[o] = rest;
+        return true;
+      }
+    }
+    return false;
+  }
+  void release(uint64_t off, uint64_t n) {
+    auto it = free_.emplace(off, n).first;
+    auto nx = std::next(it);
+    if (nx != free_.end() && it->first + it->second == nx->first) {
+      it->second += nx->second;
+      free_.erase(nx);
+    }
+    if (it != free_.begin()) {
+      auto pv = std::prev(it);
+      if (pv->first + pv->second == it->first) {
+        pv->second += it->second;
+        free_.erase(it);
+      }
+    }
+  }
+};
+
+template <class T>
+cudaError_t host_alloc(T** p, size_t n) {
+  return cudaMallocHost((void**)p, sizeof(T) * (n ? n : 1));
+}
+
+}  // namespace
+
+struct xpl_ctx {
+  xpl_config cfg;
+  cudaStream_t rs = nullptr;  // the runtime's stream
+
+  // shadow pool: 1 byte per word
+  uint8_t* d_pool = nullptr;
+  uint64_t pool_words = 0;
+  PoolAlloc pa;
+  uint32_t* d_first_w = nullptr;  // merge scratch, lazily allocated
+
+  // shadow memory table
+  std::vector<Row> rows;               // by id
+  std::map<uint64_t, uint64_t> live;   // base -> id
+  uint32_t n_dead = 0;
+  uint8_t* d_tab = nullptr;            // [u32 n | pad to 32 B | xpl_dev_row[max_rows]]
+  uint8_t* h_tab = nullptr;
+  bool table_dirty = true;
+  cudaEvent_t table_ev = nullptr;
+  const Row* cache = nullptr;          // last host lookup hit
+
+  // dirty list (epoch close)
+  uint32_t* d_dirty = nullptr;
+  uint32_t* d_misc = nullptr;          // [0] dirty_count, [1] fold done counter
+  unsigned long long* d_stats = nullptr;
+
+  // epochs (D19)
+  int depth = 0;
+  std::vector<cudaStream_t> epoch_streams;
+  std::vector<cudaEvent_t> ev_pool;
+  cudaEvent_t ev_begin = nullptr;
+
+  // host-record staging (8-byte packed records)
+  uint64_t* h_stage[2] = {nullptr, nullptr};
+  cudaEvent_t stage_ev[2] = {nullptr, nullptr};
+  int cur = 0;
+  size_t stage_n = 0, stage_cap = 0, stage_ranges = 0;
+  bool stage_has_r = false, stage_has_w = false;
+  uint64_t* d_stage = nullptr;
+  std::vector<uint64_t> deferred;      // host records inside an open epoch (D20)
+
+  // range descriptors
+  RangeDesc* h_ranges = nullptr;
+  RangeDesc* d_ranges = nullptr;
+  size_t ranges_cap = 0;
+  cudaEvent_t ranges_ev = nullptr;
+
+  // diagnose buffers (grown on demand)
+  DiagRow* h_drows = nullptr;
+  DiagRow* d_drows = nullptr;
+  size_t drows_cap = 0;
+  uint32_t* h_tile_row = nullptr;
+  uint32_t* d_tile_row = nullptr;
+  TileSum* d_tiles = nullptr;
+  size_t tiles_cap = 0;
+  uint32_t* d_blk = nullptr;
+  size_t blk_cap = 0;
+  unsigned long long* d_cnt = nullptr;
+  xpl_alloc_report* d_rep = nullptr;
+  xpl_alloc_report* h_rep = nullptr;
+
+  xpl_stats st;
+};
+
+namespace {
+
+// ---------------------------------------------------------------------------
+// host lookup: the live row holding addr; nullptr = untracked
+const Row* lookup(xpl_ctx* c, uint64_t addr) {
+  if (c->cache && addr >= c->cache->base && addr < c->cache->base + c->cache->bytes) return c->cache;
+  auto it = c->live.upper_bound(addr);
+  if (it == c->live.begin()) return nullptr;
+  --it;
+  const Row* r = &c->rows[it->second];
+  if (addr >= r->base + r->bytes) return nullptr;
+  c->cache = r;
+  return r;
+}
+
+// words [g0, g0+nw) of the access (addr, size), clipped (D1, D18)
+bool to_words(xpl_ctx* c, uint64_t addr, uint64_t size, uint64_t* g0, uint64_t* nw) {
+  if (size == 0) return false;
+  const Row* r = lookup(c, addr);
+  if (!r) return false;
+  const uint64_t w0 = (addr - r->base) >> 2;
+  uint64_t wl = (addr + size - 1 - r->base) >> 2;
+  if (wl > r->words - 1) wl = r->words - 1;
+  *g0 = r->off + w0;
+  *nw = wl - w0 + 1;
+  return true;
+}
+
+xpl_status flush(xpl_ctx* c);
+
+// Append one packed record to staging, coalescing with the previous one when
+// that is exact: same access kind and touching/overlapping words for R or W
+// (idempotent per word), adjacent disjoint words for RW.
+xpl_status stage_push(xpl_ctx* c, uint64_t g0, uint64_t nw, uint32_t acc) {
+  while (nw > kMaxRecWords) {  // split very long ranges (disjoint pieces)
+    xpl_status s = stage_push(c, g0, kMaxRecWords, acc);
+    if (s) return s;
+    g0 += kMaxRecWords;
+    nw -= kMaxRecWords;
+  }
+  c->st.host_records++;
+  if (c->stage_n) {
+    uint64_t& last = c->h_stage[c->cur][c->stage_n - 1];
+    const uint32_t la = rec_acc(last);
+    const uint64_t l0 = rec_g0(last), ln = rec_nw(last);
+    if (la == acc) {
+      uint64_t u0 = 0, u1 = 0;
+      bool ok = false;
+      if (acc != XPL_ACC_RW) {
+        if (g0 <= l0 + ln && g0 + nw >= l0) {
+          u0 = std::min(g0, l0);
+          u1 = std::max(g0 + nw, l0 + ln);
+          ok = true;
+        }
+      } else if (g0 == l0 + ln) {
+        u0 = l0;
+        u1 = g0 + nw;
+        ok = true;
+      }
+      if (ok && u1 - u0 <= kMaxRecWords) {
+        if (ln <= kRangeWords && u1 - u0 > kRangeWords) c->stage_ranges++;
+        last = pack_rec(u0, u1 - u0, acc);
+        return XPL_OK;
+      }
+    }
+  }
+  if (c->stage_n == c->stage_cap) {
+    xpl_status s = flush(c);
+    if (s) return s;
+  }
+  c->h_stage[c->cur][c->stage_n++] = pack_rec(g0, nw, acc);
+  c->st.host_records_packed++;
+  if (nw > kRangeWords) c->stage_ranges++;
+  if (acc & XPL_ACC_R) c->stage_has_r = true;
+  if (acc & XPL_ACC_W) c->stage_has_w = true;
+  return XPL_OK;
+}
+
+xpl_status ensure_ranges(xpl_ctx* c, size_t n) {
+  if (n <= c->ranges_cap) {
+    CK(cudaEventSynchronize(c->ranges_ev));
+    return XPL_OK;
+  }
+  CK(cudaStreamSynchronize(c->rs));
+  if (c->h_ranges) cudaFreeHost(c->h_ranges);
+  if (c->d_ranges) cudaFree(c->d_ranges);
+  size_t cap = std::max<size_t>(n, 1024);
+  CK(host_alloc(&c->h_ranges, cap));
+  CK(cudaMalloc(&c->d_ranges, sizeof(RangeDesc) * cap));
+  c->ranges_cap = cap;
+  return XPL_OK;
+}
+
+xpl_status ensure_first_w(xpl_ctx* c) {
+  if (c->d_first_w) return XPL_OK;
+  CK(cudaMalloc(&c->d_first_w, sizeof(uint32_t) * c->pool_words));
+  launch_fill_u32(c->rs, c->d_first_w, c->pool_words, 0xFFFFFFFFu);
+  return XPL_OK;
+}
+
+// Apply all staged host records on the runtime stream, in order: runs of short
+// records go through the 3-pass merge, runs of pairwise-disjoint long ranges
+// through range_apply.
+xpl_status flush(xpl_ctx* c) {
+  if (c->stage_n == 0) return XPL_OK;
+  const size_t n = c->stage_n;
+  uint64_t* h = c->h_stage[c->cur];
+  CK(cudaMemcpyAsync(c->d_stage, h, n * sizeof(uint64_t), cudaMemcpyHostToDevice, c->rs));
+  CK(cudaEventRecord(c->stage_ev[c->cur], c->rs));
+  if (c->stage_ranges == 0) {
+    xpl_status s = XPL_OK;
+    if (c->stage_has_r && c->stage_has_w) s = ensure_first_w(c);
+    if (s) return s;
+    launch_merge(c->rs, c->d_stage, (uint32_t)n, c->stage_has_r, c->stage_has_w, c->d_first_w,
+                 (uint32_t*)c->d_pool);
+    c->st.merge_segments++;
+  } else {
+    // Segment the batch.  Range descriptors of this flush go to h_ranges.
+    size_t n_long = 0;
+    for (size_t i = 0; i < n; ++i) n_long += rec_nw(h[i]) > kRangeWords;
+    xpl_status s = ensure_ranges(c, n_long);
+    if (s) return s;
+    size_t nr_total = 0;
+    struct Seg { size_t start, n; bool range, has_r, has_w; };
+    std::vector<Seg> segs;
+    std::map<uint64_t, uint64_t> iv;  // disjointness of the open range segment
+    for (size_t i = 0; i < n; ++i) {
+      const uint64_t r = h[i];
+      const uint64_t g0 = rec_g0(r), nw = rec_nw(r);
+      const uint32_t acc = rec_acc(r);
+      if (nw > kRangeWords) {
+        bool join = !segs.empty() && segs.back().range;
+        if (join) {
+          auto it = iv.lower_bound(g0);
+          if (it != iv.end() && it->first < g0 + nw) join = false;
+          if (join && it != iv.begin()) {
+            --it;
+            if (it->second > g0) join = false;
+          }
+        }
+        if (!join) {
+          segs.push_back({nr_total, 0, true, false, false});
+          iv.clear();
+        }
+        iv[g0] = g0 + nw;
+        RangeDesc& d = c->h_ranges[nr_total++];
+        d.g0 = g0;
+        d.nw = nw;
+        d.acc = acc;
+        d.side = 0;
+        segs.back().n++;
+      } else {
+        if (segs.empty() || segs.back().range) segs.push_back({i, 0, false, false, false});
+        Seg& sg = segs.back();
+        sg.n++;
+        if (acc & XPL_ACC_R) sg.has_r = true;
+        if (acc & XPL_ACC_W) sg.has_w = true;
+      }
+    }
+    // vbase per segment, then one upload of all descriptors
+    for (const Seg& sg : segs) {
+      if (!sg.range) continue;
+      uint64_t v = 0;
+      for (size_t i = sg.start; i < sg.start + sg.n; ++i) {
+        c->h_ranges[i].vbase = v;
+        v += ((c->h_ranges[i].g0 + c->h_ranges[i].nw - 1) >> 4) - (c->h_ranges[i].g0 >> 4) + 1;
+      }
+    }
+    CK(cudaMemcpyAsync(c->d_ranges, c->h_ranges, sizeof(RangeDesc) * nr_total,
+                       cudaMemcpyHostToDevice, c->rs));
+    CK(cudaEventRecord(c->ranges_ev, c->rs));
+    for (const Seg& sg : segs) {
+      if (sg.range) {
+        uint64_t nvec = c->h_ranges[sg.start + sg.n - 1].vbase +
+                        ((c->h_ranges[sg.start + sg.n - 1].g0 + c->h_ranges[sg.start + sg.n - 1].nw - 1) >> 4) -
+                        (c->h_ranges[sg.start + sg.n - 1].g0 >> 4) + 1;
+        launch_range(c->rs, c->d_ranges + sg.start, (uint32_t)sg.n, nvec, (uint32_t*)c->d_pool,
+                     c->d_dirty, c->d_misc, (uint32_t)c->cfg.dirty_cap);
+        c->st.range_segments++;
+      } else {
+        if (sg.has_r && sg.has_w) {
+          s = ensure_first_w(c);
+          if (s) return s;
+        }
+        launch_merge(c->rs, c->d_stage + sg.start, (uint32_t)sg.n, sg.has_r, sg.has_w,
+                     c->d_first_w, (uint32_t*)c->d_pool);
+        c->st.merge_segments++;
+      }
+    }
+  }
+  if (cudaGetLastError() != cudaSuccess) return XPL_ERR_CUDA;
+  c->cur ^= 1;
+  CK(cudaEventSynchronize(c->stage_ev[c->cur]));  // the other buffer's copy is done
+  c->stage_n = 0;
+  c->stage_ranges = 0;
+  c->stage_has_r = c->stage_has_w = false;
+  return XPL_OK;
+}
+
+xpl_status upload_table(xpl_ctx* c) {
+  if (!c->table_dirty) return XPL_OK;
+  CK(cudaEventSynchronize(c->table_ev));
+  uint32_t n = 0;
+  xpl_dev_row* hr = (xpl_dev_row*)(c->h_tab + 32);
+  for (auto& kv : c->live) {  // sorted by base
+    const Row& r = c->rows[kv.second];
+    hr[n].base = r.base;
+    hr[n].end = r.base + r.bytes;
+    hr[n].off = r.off;
+    hr[n].words = r.words;
+    ++n;
+  }
+  memcpy(c->h_tab, &n, sizeof n);
+  CK(cudaMemcpyAsync(c->d_tab, c->h_tab, 32 + sizeof(xpl_dev_row) * n, cudaMemcpyHostToDevice, c->rs));
+  CK(cudaEventRecord(c->table_ev, c->rs));
+  c->table_dirty = false;
+  return XPL_OK;
+}
+
+cudaEvent_t pool_event(xpl_ctx* c, size_t i) {
+  while (c->ev_pool.size() <= i) {
+    cudaEvent_t e;
+    cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+    c->ev_pool.push_back(e);
+  }
+  return c->ev_pool[i];
+}
+
+// GPU-side range accesses (D2D, memset; D7) inside the current epoch.
+xpl_status gpu_ranges(xpl_ctx* c, const RangeDesc* rd, size_t nr) {
+  if (!nr) return XPL_OK;
+  xpl_status s = ensure_ranges(c, nr);
+  if (s) return s;
+  memcpy(c->h_ranges, rd, sizeof(RangeDesc) * nr);
+  uint64_t v = 0;
+  for (size_t i = 0; i < nr; ++i) {
+    c->h_ranges[i].vbase = v;
+    v += ((c->h_ranges[i].g0 + c->h_ranges[i].nw - 1) >> 4) - (c->h_ranges[i].g0 >> 4) + 1;
+  }
+  CK(cudaMemcpyAsync(c->d_ranges, c->h_ranges, sizeof(RangeDesc) * nr, cudaMemcpyHostToDevice, c->rs));
+  CK(cudaEventRecord(c->ranges_ev, c->rs));
+  launch_range(c->rs, c->d_ranges, (uint32_t)nr, v, (uint32_t*)c->d_pool, c->d_dirty, c->d_misc,
+               (uint32_t)c->cfg.dirty_cap);
+  return cudaGetLastError() == cudaSuccess ? XPL_OK : XPL_ERR_CUDA;
+}
+
+void fold(xpl_ctx* c) {
+  launch_fold(c->rs, (uint32_t*)c->d_pool, c->pool_words / 4, c->d_dirty, c->d_misc,
+              (uint32_t)c->cfg.dirty_cap, c->d_misc + 1, c->d_stats);
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* xpl_status_string(xpl_status s) {
+  switch (s) {
+    case XPL_OK: return "ok";
+    case XPL_ERR_INVALID_ARG: return "invalid argument";
+    case XPL_ERR_OOM: return "out of memory (shadow pool, table or staging)";
+    case XPL_ERR_OVERLAP: return "allocation overlaps a live allocation";
+    case XPL_ERR_UNKNOWN_PTR: return "pointer is not the base of a live allocation";
+    case XPL_ERR_STATE: return "call not allowed in the current epoch state";
+    case XPL_ERR_CUDA: return "CUDA runtime error";
+    case XPL_ERR_NCCL: return "NCCL error";
+    case XPL_ERR_DEVICE_OVERFLOW: return "device-side capacity exceeded";
+  }
+  return "unknown status";
+}
+
+xpl_status xpl_init(const xpl_config* cfg, xpl_ctx** out) {
+  if (!cfg || !out) return XPL_ERR_INVALID_ARG;
+  if (cfg->world > 1) return XPL_ERR_INVALID_ARG;  // sharding: see DESIGN.md §8
+  xpl_ctx* c = new (std::nothrow) xpl_ctx();
+  if (!c) return XPL_ERR_OOM;
+  c->cfg = *cfg;
+  if (!c->cfg.pool_words) c->cfg.pool_words = 1ull << 28;
+  if (!c->cfg.dirty_cap) c->cfg.dirty_cap = 1ull << 24;
+  if (c->cfg.dirty_cap > 0xFFFFFFF0ull) c->cfg.dirty_cap = 0xFFFFFFF0ull;
+  if (!c->cfg.staging_recs) c->cfg.staging_recs = 1ull << 22;
+  if (!c->cfg.max_rows) c->cfg.max_rows = 4096;
+  c->pool_words = (c->cfg.pool_words + 15) & ~15ull;
+  if (c->pool_words / 4 > 0xFFFFFFFFull) { delete c; return XPL_ERR_INVALID_ARG; }
+#define CKI(x)                  \
+  do {                          \
+    if ((x) != cudaSuccess) {   \
+      xpl_finalize(c);          \
+      return XPL_ERR_CUDA;      \
+    }                           \
+  } while (0)
+  CKI(cudaSetDevice(cfg->device));
+  CKI(cudaStreamCreateWithFlags(&c->rs, cudaStreamNonBlocking));
+  CKI(cudaMalloc(&c->d_pool, c->pool_words));
+  CKI(cudaMemsetAsync(c->d_pool, 0, c->pool_words, c->rs));
+  c->pa.init(c->pool_words);
+  CKI(cudaMalloc(&c->d_tab, 32 + sizeof(xpl_dev_row) * c->cfg.max_rows));
+  CKI(cudaMemsetAsync(c->d_tab, 0, 32, c->rs));
+  CKI(host_alloc(&c->h_tab, 32 + sizeof(xpl_dev_row) * c->cfg.max_rows));
+  CKI(cudaMalloc(&c->d_dirty, sizeof(uint32_t) * c->cfg.dirty_cap));
+  CKI(cudaMalloc(&c->d_misc, 64));
+  CKI(cudaMemsetAsync(c->d_misc, 0, 64, c->rs));
+  CKI(cudaMalloc(&c->d_stats, 64));
+  CKI(cudaMemsetAsync(c->d_stats, 0, 64, c->rs));
+  c->stage_cap = c->cfg.staging_recs;
+  CKI(host_alloc(&c->h_stage[0], c->stage_cap));
+  CKI(host_alloc(&c->h_stage[1], c->stage_cap));
+  CKI(cudaMalloc(&c->d_stage, sizeof(uint64_t) * c->stage_cap));
+  CKI(cudaEventCreateWithFlags(&c->stage_ev[0], cudaEventDisableTiming));
+  CKI(cudaEventCreateWithFlags(&c->stage_ev[1], cudaEventDisableTiming));
+  CKI(cudaEventCreateWithFlags(&c->table_ev, cudaEventDisableTiming));
+  CKI(cudaEventCreateWithFlags(&c->ranges_ev, cudaEventDisableTiming));
+  CKI(cudaEventCreateWithFlags(&c->ev_begin, cudaEventDisableTiming));
+  CKI(cudaEventRecord(c->stage_ev[0], c->rs));
+  CKI(cudaEventRecord(c->stage_ev[1], c->rs));
+  CKI(cudaEventRecord(c->table_ev, c->rs));
+  CKI(cudaEventRecord(c->ranges_ev, c->rs));
+  xpl_status s = ensure_ranges(c, 1024);
+  if (s) { xpl_finalize(c); return s; }
+  CKI(cudaStreamSynchronize(c->rs));
+  memset(&c->st, 0, sizeof c->st);
+  *out = c;
+  return XPL_OK;
+#undef CKI
+}
+
+xpl_status xpl_finalize(xpl_ctx* c) {
+  if (!c) return XPL_ERR_INVALID_ARG;
+  if (c->rs) cudaStreamSynchronize(c->rs);
+  cudaFree(c->d_pool);
+  cudaFree(c->d_first_w);
+  cudaFree(c->d_tab);
+  cudaFreeHost(c->h_tab);
+  cudaFree(c->d_dirty);
+  cudaFree(c->d_misc);
+  cudaFree(c->d_stats);
+  cudaFreeHost(c->h_stage[0]);
+  cudaFreeHost(c->h_stage[1]);
+  cudaFree(c->d_stage);
+  cudaFreeHost(c->h_ranges);
+  cudaFree(c->d_ranges);
+  cudaFreeHost(c->h_drows);
+  cudaFree(c->d_drows);
+  cudaFreeHost(c->h_tile_row);
+  cudaFree(c->d_tile_row);
+  cudaFree(c->d_tiles);
+  cudaFree(c->d_blk);
+  cudaFree(c->d_cnt);
+  cudaFree(c->d_rep);
+  cudaFreeHost(c->h_rep);
+  for (cudaEvent_t e : c->ev_pool) cudaEventDestroy(e);
+  for (cudaEvent_t e : {c->stage_ev[0], c->stage_ev[1], c->table_ev, c->ranges_ev, c->ev_begin})
+    if (e) cudaEventDestroy(e);
+  if (c->rs) cudaStreamDestroy(c->rs);
+  delete c;
+  return XPL_OK;
+}
+
+xpl_status xpl_register_alloc(xpl_ctx* c, const void* ptr, size_t bytes, xpl_alloc_kind kind) {
+  if (!c || !ptr || bytes == 0 || (unsigned)kind > 2) return XPL_ERR_INVALID_ARG;
+  if (c->depth) return XPL_ERR_STATE;
+  const uint64_t p = (uint64_t)ptr;
+  auto it = c->live.lower_bound(p);
+  if (it != c->live.end() && it->first < p + bytes) return XPL_ERR_OVERLAP;
+  if (it != c->live.begin()) {
+    auto pv = std::prev(it);
+    const Row& r = c->rows[pv->second];
+    if (r.base + r.bytes > p) return XPL_ERR_OVERLAP;
+  }
+  if (c->live.size() >= c->cfg.max_rows) return XPL_ERR_OOM;
+  Row r;
+  r.id = c->rows.size();
+  r.base = p;
+  r.bytes = bytes;
+  r.words = (bytes + 3) / 4;
+  r.span = (r.words + 15) & ~15ull;
+  r.kind = kind;
+  r.live = true;
+  r.dropped = false;
+  r.ever = false;
+  if (!c->pa.alloc(r.span, &r.off)) return XPL_ERR_OOM;
+  CK(cudaMemsetAsync(c->d_pool + r.off, 0, r.span, c->rs));  // D3: last writer = CPU
+  const size_t cap_before = c->rows.capacity();
+  c->rows.push_back(r);
+  if (c->rows.capacity() != cap_before) c->cache = nullptr;
+  c->live[p] = r.id;
+  c->table_dirty = true;
+  c->cache = nullptr;
+  return XPL_OK;
+}
+
+xpl_status xpl_free(xpl_ctx* c, const void* ptr) {
+  if (!c) return XPL_ERR_INVALID_ARG;
+  if (c->depth) return XPL_ERR_STATE;
+  auto it = c->live.find((uint64_t)ptr);
+  if (it == c->live.end()) return XPL_ERR_UNKNOWN_PTR;
+  c->rows[it->second].live = false;  // shadow kept until the next diagnose
+  c->live.erase(it);
+  c->n_dead++;
+  c->table_dirty = true;
+  c->cache = nullptr;
+  return XPL_OK;
+}
+
+xpl_status xpl_kernel_begin(xpl_ctx* c, void* stream) {
+  if (!c) return XPL_ERR_INVALID_ARG;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (c->depth == 0) {
+    xpl_status st = flush(c);
+    if (st) return st;
+    st = upload_table(c);
+    if (st) return st;
+    CK(cudaEventRecord(c->ev_begin, c->rs));
+    c->epoch_streams.clear();
+    c->st.epochs++;
+  }
+  if (std::find(c->epoch_streams.begin(), c->epoch_streams.end(), s) == c->epoch_streams.end()) {
+    CK(cudaStreamWaitEvent(s, c->ev_begin, 0));
+    c->epoch_streams.push_back(s);
+  }
+  c->depth++;
+  return XPL_OK;
+}
+
+xpl_status xpl_kernel_end(xpl_ctx* c, void* stream) {
+  if (!c) return XPL_ERR_INVALID_ARG;
+  if (c->depth == 0) return XPL_ERR_STATE;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (std::find(c->epoch_streams.begin(), c->epoch_streams.end(), s) == c->epoch_streams.end())
+    c->epoch_streams.push_back(s);
+  if (--c->depth) return XPL_OK;
+  for (size_t i = 0; i < c->epoch_streams.size(); ++i) {
+    cudaEvent_t e = pool_event(c, i);
+    CK(cudaEventRecord(e, c->epoch_streams[i]));
+    CK(cudaStreamWaitEvent(c->rs, e, 0));
+  }
+  fold(c);
+  if (cudaGetLastError() != cudaSuccess) return XPL_ERR_CUDA;
+  std::vector<uint64_t> q;
+  q.swap(c->deferred);
+  for (uint64_t r : q) {
+    xpl_status st = stage_push(c, rec_g0(r), rec_nw(r), rec_acc(r));
+    if (st) return st;
+  }
+  return XPL_OK;
+}
+
+xpl_status xpl_record_host(xpl_ctx* c, const xpl_host_access* recs, size_t n) {
+  if (!c || (!recs && n)) return XPL_ERR_INVALID_ARG;
+  for (size_t i = 0; i < n; ++i) {
+    const uint32_t acc = recs[i].kind;
+    if (acc < 1 || acc > 3) return XPL_ERR_INVALID_ARG;
+    uint64_t g0, nw;
+    if (!to_words(c, recs[i].addr, recs[i].size, &g0, &nw)) continue;  // untracked
+    if (c->depth) {
+      while (nw > kMaxRecWords) {
+        c->deferred.push_back(pack_rec(g0, kMaxRecWords, acc));
+        g0 += kMaxRecWords;
+        nw -= kMaxRecWords;
+      }
+      c->deferred.push_back(pack_rec(g0, nw, acc));
+      continue;
+    }
+    xpl_status s = stage_push(c, g0, nw, acc);
+    if (s) return s;
+  }
+  return XPL_OK;
+}
+
+xpl_status xpl_record_copy(xpl_ctx* c, const void* dst, const void* src, size_t bytes,
+                           xpl_copy_dir dir) {
+  if (!c || (unsigned)dir > 4) return XPL_ERR_INVALID_ARG;
+  if (bytes == 0) return XPL_OK;
+  if (dir <= XPL_COPY_H2H) {  // CPU-side
+    xpl_host_access a[2];
+    size_t n = 0;
+    if (dir == XPL_COPY_H2D) a[n++] = {(uint64_t)dst, 0, XPL_ACC_W};
+    if (dir == XPL_COPY_D2H) a[n++] = {(uint64_t)src, 0, XPL_ACC_R};
+    if (dir == XPL_COPY_H2H) {
+      a[n++] = {(uint64_t)src, 0, XPL_ACC_R};
+      a[n++] = {(uint64_t)dst, 0, XPL_ACC_W};
+    }
+    for (size_t i = 0; i < n; ++i) {  // sizes may exceed 32 bits: split
+      uint64_t off = 0;
+      while (off < bytes) {
+        const uint64_t chunk = std::min<uint64_t>(bytes - off, 1ull << 30);
+        xpl_host_access r = {a[i].addr + off, (uint32_t)chunk, a[i].kind};
+        xpl_status s = xpl_record_host(c, &r, 1);
+        if (s) return s;
+        off += chunk;
+      }
+    }
+    return XPL_OK;
+  }
+  // GPU-side: D2D = GPU read src + GPU write dst; memset = GPU write dst (D7).
+  RangeDesc rd[2 * 64];
+  size_t nr = 0;
+  auto add = [&](uint64_t addr, uint32_t acc) {
+    uint64_t g0, nw;
+    if (!to_words(c, addr, bytes, &g0, &nw)) return;
+    while (nw && nr < 128) {
+      const uint64_t k = std::min<uint64_t>(nw, kMaxRecWords);
+      rd[nr++] = {g0, k, 0, acc, 1};
+      g0 += k;
+      nw -= k;
+    }
+  };
+  if (dir == XPL_COPY_D2D) add((uint64_t)src, XPL_ACC_R);
+  add((uint64_t)dst, XPL_ACC_W);
+  const bool own = c->depth == 0;
+  if (own) {
+    xpl_status s = flush(c);
+    if (s) return s;
+    c->st.epochs++;
+  }
+  xpl_status s = gpu_ranges(c, rd, nr);
+  if (s) return s;
+  if (own) fold(c);
+  return cudaGetLastError() == cudaSuccess ? XPL_OK : XPL_ERR_CUDA;
+}
+
+xpl_status xpl_flush(xpl_ctx* c) {
+  if (!c) return XPL_ERR_INVALID_ARG;
+  return flush(c);
+}
+
+xpl_status xpl_sync(xpl_ctx* c) {
+  if (!c) return XPL_ERR_INVALID_ARG;
+  CK(cudaStreamSynchronize(c->rs));
+  return XPL_OK;
+}
+
+xpl_status xpl_runtime_stream(xpl_ctx* c, void** s) {
+  if (!c || !s) return XPL_ERR_INVALID_ARG;
+  *s = (void*)c->rs;
+  return XPL_OK;
+}
+
+xpl_status xpl_get_device_ctx(xpl_ctx* c, struct xpl_dev_ctx* d) {
+  if (!c || !d) return XPL_ERR_INVALID_ARG;
+  d->rows = (const xpl_dev_row*)(c->d_tab + 32);
+  d->n_rows = (const unsigned int*)c->d_tab;
+  d->pool = (unsigned int*)c->d_pool;
+  d->dirty = c->d_dirty;
+  d->dirty_count = c->d_misc;
+  d->dirty_cap = (unsigned int)c->cfg.dirty_cap;
+  d->pad_ = 0;
+  return XPL_OK;
+}
+
+xpl_status xpl_get_stats(xpl_ctx* c, xpl_stats* o) {
+  if (!c || !o) return XPL_ERR_INVALID_ARG;
+  unsigned long long ds[8];
+  CK(cudaStreamSynchronize(c->rs));
+  CK(cudaMemcpy(ds, c->d_stats, sizeof ds, cudaMemcpyDeviceToHost));
+  *o = c->st;
+  o->dirty_max = ds[0];
+  o->fold_full_scans = ds[1];
+  o->folds = ds[2];
+  return XPL_OK;
+}
+
+xpl_status xpl_shadow_dump(xpl_ctx* c, const void* base, uint64_t word0, uint64_t n, uint8_t* out) {
+  if (!c || !out) return XPL_ERR_INVALID_ARG;
+  if (c->depth) return XPL_ERR_STATE;
+  auto it = c->live.find((uint64_t)base);
+  if (it == c->live.end()) return XPL_ERR_UNKNOWN_PTR;
+  const Row& r = c->rows[it->second];
+  if (word0 > r.words || n > r.words - word0) return XPL_ERR_INVALID_ARG;
+  xpl_status s = flush(c);
+  if (s) return s;
+  CK(cudaMemcpyAsync(out, c->d_pool + r.off + word0, n, cudaMemcpyDeviceToHost, c->rs));
+  CK(cudaStreamSynchronize(c->rs));
+  return XPL_OK;
+}
+
+xpl_status xpl_diagnose(xpl_ctx* c, const xpl_diag_params* params, const xpl_name* names,
+                        size_t n_names, xpl_alloc_report* out, size_t cap, size_t* n_out,
+                        int reset) {
+  if (!c || !n_out || (n_names && !names)) return XPL_ERR_INVALID_ARG;
+  if (c->depth) return XPL_ERR_STATE;
+  DiagParams p;
+  p.thr = params ? params->density_threshold_pct : 50;
+  p.block_words = params ? params->block_words : 0;
+  p.min_run = params ? params->min_run_words : 256;
+  if (p.min_run == 0) p.min_run = 1;
+  p.reset = reset ? 1 : 0;
+
+  std::vector<uint64_t> ids;  // live rows + rows freed since the last reset, id order (D23)
+  for (const Row& r : c->rows)
+    if (r.live || !r.dropped) ids.push_back(r.id);
+  *n_out = ids.size();
+  if (cap < ids.size() || (!out && ids.size())) return XPL_ERR_INVALID_ARG;
+
+  xpl_status s = flush(c);
+  if (s) return s;
+  const size_t nr = ids.size();
+  c->st.diagnoses++;
+  if (nr == 0) return XPL_OK;
+
+  // geometry
+  uint64_t ntiles = 0, nblocks = 0;
+  for (uint64_t id : ids) {
+    const Row& r = c->rows[id];
+    ntiles += (r.words + kTileWords - 1) / kTileWords;
+    if (p.block_words) nblocks += (r.words + p.block_words - 1) / p.block_words;
+  }
+  if (ntiles > 0x7FFFFFFFull) return XPL_ERR_OOM;
+  if (nr > c->drows_cap) {
+    cudaFreeHost(c->h_drows);
+    cudaFree(c->d_drows);
+    cudaFree(c->d_cnt);
+    cudaFree(c->d_rep);
+    cudaFreeHost(c->h_rep);
+    c->drows_cap = std::max<size_t>(nr, 256);
+    CK(host_alloc(&c->h_drows, c->drows_cap));
+    CK(cudaMalloc(&c->d_drows, sizeof(DiagRow) * c->drows_cap));
+    CK(cudaMalloc(&c->d_cnt, sizeof(unsigned long long) * C_NCNT * c->drows_cap));
+    CK(cudaMalloc(&c->d_rep, sizeof(xpl_alloc_report) * c->drows_cap));
+    CK(host_alloc(&c->h_rep, c->drows_cap));
+  }
+  if (ntiles > c->tiles_cap) {
+    cudaFreeHost(c->h_tile_row);
+    cudaFree(c->d_tile_row);
+    cudaFree(c->d_tiles);
+    c->tiles_cap = std::max<uint64_t>(ntiles, 1024);
+    CK(host_alloc(&c->h_tile_row, c->tiles_cap));
+    CK(cudaMalloc(&c->d_tile_row, sizeof(uint32_t) * c->tiles_cap));
+    CK(cudaMalloc(&c->d_tiles, sizeof(TileSum) * c->tiles_cap));
+  }
+  if (nblocks > c->blk_cap) {
+    cudaFree(c->d_blk);
+    c->blk_cap = std::max<uint64_t>(nblocks, 1024);
+    CK(cudaMalloc(&c->d_blk, sizeof(uint32_t) * c->blk_cap));
+  }
+  uint64_t t = 0, b = 0;
+  for (size_t i = 0; i < nr; ++i) {
+    const Row& r = c->rows[ids[i]];
+    DiagRow& d = c->h_drows[i];
+    d.off = r.off;
+    d.words = r.words;
+    d.tile0 = t;
+    d.ntiles = (r.words + kTileWords - 1) / kTileWords;
+    d.blk0 = b;
+    d.nblk = p.block_words ? (r.words + p.block_words - 1) / p.block_words : 0;
+    d.kind = r.kind;
+    d.pad = 0;
+    for (uint64_t k = 0; k < d.ntiles; ++k) c->h_tile_row[t + k] = (uint32_t)i;
+    t += d.ntiles;
+    b += d.nblk;
+  }
+  CK(cudaMemcpyAsync(c->d_drows, c->h_drows, sizeof(DiagRow) * nr, cudaMemcpyHostToDevice, c->rs));
+  CK(cudaMemcpyAsync(c->d_tile_row, c->h_tile_row, sizeof(uint32_t) * ntiles,
+                     cudaMemcpyHostToDevice, c->rs));
+  launch_diag(c->rs, c->d_drows, (uint32_t)nr, c->d_tile_row, ntiles, nblocks, p,
+              (uint32_t*)c->d_pool, c->d_cnt, c->d_tiles, c->d_blk, c->d_rep);
+  CK(cudaGetLastError());
+  CK(cudaMemcpyAsync(c->h_rep, c->d_rep, sizeof(xpl_alloc_report) * nr, cudaMemcpyDeviceToHost, c->rs));
+  CK(cudaStreamSynchronize(c->rs));
+
+  for (size_t i = 0; i < nr; ++i) {
+    Row& r = c->rows[ids[i]];
+    xpl_alloc_report o = c->h_rep[i];
+    o.id = r.id;
+    o.base = r.base;
+    o.bytes = r.bytes;
+    o.live = r.live ? 1 : 0;
+    o.name_idx = 0xFFFFFFFFu;
+    if (o.any_acc) r.ever = true;
+    o.ever_accessed = r.ever ? 1 : 0;
+    out[i] = o;
+  }
+  // names (XplAllocData): the first name inside a live row
+  c->cache = nullptr;
+  for (size_t j = 0; j < n_names; ++j) {
+    const Row* r = lookup(c, (uint64_t)names[j].addr);
+    if (!r) continue;
+    for (size_t i = 0; i < nr; ++i)
+      if (out[i].id == r->id && out[i].name_idx == 0xFFFFFFFFu) out[i].name_idx = (uint32_t)j;
+  }
+  if (reset) {  // drop freed rows and recycle their shadow (D17)
+    for (Row& r : c->rows) {
+      if (!r.live && !r.dropped) {
+        r.dropped = true;
+        c->pa.release(r.off, r.span);
+      }
+    }
+    c->n_dead = 0;
+  }
+  return XPL_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,37 @@
+// work_replay.cu -- an instrumented "user" kernel that replays a list of device
+// accesses through the public __device__ hooks (include/xpl_device.cuh).  It is
+// user code of libxpl, not part of it: it only sees xpl.h and xpl_device.cuh.
+// Used by the parity tests (any trace, any launch shape, any permutation) and
+// as the generic device-event source of the benchmarks.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "xpl.h"
+#include "xpl_device.cuh"
+
+namespace {
+
+__global__ void replay_kernel(const unsigned long long* __restrict__ addr,
+                              const unsigned int* __restrict__ size,
+                              const unsigned char* __restrict__ acc, unsigned long long n) {
+  for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (unsigned long long)gridDim.x * blockDim.x)
+    xpl_dev_record((const void*)addr[i], size[i], acc[i]);
+}
+
+}  // namespace
+
+extern "C" {
+
+// Bind this translation unit's hooks to ctx (xpl_device_bind).
+int xplw_bind(xpl_ctx* ctx) { return (int)xpl_device_bind(ctx); }
+
+// Launch the replay kernel on `stream` (between xpl_kernel_begin/_end).
+int xplw_replay(const unsigned long long* d_addr, const unsigned int* d_size,
+                const unsigned char* d_acc, unsigned long long n, int grid, int block,
+                void* stream) {
+  if (n == 0) return 0;
+  replay_kernel<<<grid, block, 0, (cudaStream_t)stream>>>(d_addr, d_size, d_acc, n);
+  return cudaGetLastError() == cudaSuccess ? 0 : (int)XPL_ERR_CUDA;
+}
+}

@@ -1,0 +1,89 @@
+// xpl_internal.h -- private declarations shared by runtime.cu and kernels.cu.
+// (CUDA path only; the oracle never sees this file.)
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "xpl.h"
+#include "xpl_device.cuh"
+
+namespace xpl {
+
+// Record byte (P:L243 + the pending bit): see include/xpl_device.cuh.
+constexpr uint32_t kL = 0x01, kP = 0x02, kWC = 0x04, kWG = 0x08, kRCC = 0x10, kRGC = 0x20,
+                   kRCG = 0x40, kRGG = 0x80;
+
+// Packed host record (8 B): bits [0,38) first pool word g0, [38,62) nwords-1,
+// [62,64) acc (R=1, W=2, RW=3).  The host runtime has already looked the address
+// up and clipped it to its allocation (D18).
+constexpr int kG0Bits = 38;
+constexpr uint64_t kG0Mask = (1ull << kG0Bits) - 1;
+constexpr uint64_t kMaxRecWords = 1ull << 24;
+__host__ __device__ inline uint64_t pack_rec(uint64_t g0, uint64_t nw, uint32_t acc) {
+  return g0 | ((nw - 1) << kG0Bits) | ((uint64_t)acc << 62);
+}
+__host__ __device__ inline uint64_t rec_g0(uint64_t r) { return r & kG0Mask; }
+__host__ __device__ inline uint64_t rec_nw(uint64_t r) { return ((r >> kG0Bits) & (kMaxRecWords - 1)) + 1; }
+__host__ __device__ inline uint32_t rec_acc(uint64_t r) { return (uint32_t)(r >> 62); }
+
+// Records of more than this many words are "ranges" and go through range_apply.
+constexpr uint64_t kRangeWords = 64;
+
+// A range for the vectorised range kernels (host transfers, D2D/memset).
+struct RangeDesc {
+  uint64_t g0, nw;     // first pool word, number of words
+  uint64_t vbase;      // prefix sum of the 16-word vectors the ranges touch
+  uint32_t acc, side;  // side 0 = CPU, 1 = GPU
+};
+
+// Diagnose geometry.
+constexpr uint32_t kTileWords = 32768;         // words per diagnose tile (one CTA)
+constexpr uint32_t kDiagThreads = 256;         // 8 warps x 32 lanes x 16 words x 8 iters
+constexpr uint32_t kDiagIters = 8;
+
+struct DiagRow {        // one row to analyse (live or dead-since-last-reset)
+  uint64_t off, words;  // pool offset (multiple of 16), words
+  uint64_t tile0;       // first tile index of this row
+  uint64_t ntiles;
+  uint64_t blk0;        // first block-counter index (block_words > 0)
+  uint64_t nblk;
+  uint32_t kind, pad;
+};
+
+// Per-row counters accumulated by the diagnose kernels (u64 each).
+enum Cnt {
+  C_WC, C_WG, C_RCC, C_RCG, C_RGC, C_RGG, C_ANY, C_GPU, C_ALT,
+  C_LDB, C_LDW, C_UR, C_UW, C_DR, C_DW, C_NCNT
+};
+
+// Run summary of a predicate over a contiguous word range (see kernels.cu).
+struct RunSum {
+  uint32_t len, pre, suf, cnt, sum;
+};
+struct TileSum {
+  RunSum u, d;  // u = wC & !rCG (unneeded H2D), d = rCC (unneeded D2H)
+};
+
+struct DiagParams {
+  uint32_t thr;
+  uint32_t reset;
+  uint64_t block_words;
+  uint64_t min_run;
+};
+
+// ---- launchers (kernels.cu) ----
+void launch_fold(cudaStream_t s, uint32_t* pool, uint64_t pool_u32, const uint32_t* dirty,
+                 uint32_t* dirty_count, uint32_t dirty_cap, uint32_t* done_ctr,
+                 unsigned long long* stats);
+void launch_merge(cudaStream_t s, const uint64_t* recs, uint32_t n, bool has_r, bool has_w,
+                  uint32_t* first_w, uint32_t* pool);
+void launch_range(cudaStream_t s, const RangeDesc* d_ranges, uint32_t nr, uint64_t nvec,
+                  uint32_t* pool, uint32_t* dirty, uint32_t* dirty_count, uint32_t dirty_cap);
+void launch_diag(cudaStream_t s, const DiagRow* rows, uint32_t nrows, const uint32_t* tile_row,
+                 uint64_t ntiles, uint64_t nblocks, const DiagParams& p, uint32_t* pool,
+                 unsigned long long* cnt, TileSum* tiles, uint32_t* blk_cnt,
+                 xpl_alloc_report* out);
+void launch_fill_u32(cudaStream_t s, uint32_t* p, uint64_t n, uint32_t v);
+
+}  // namespace xpl

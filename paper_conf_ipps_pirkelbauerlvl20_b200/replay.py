@@ -1,0 +1,103 @@
+"""Drive an event trace (xplgen.trace format) through the C-ABI.
+
+Host events go to xpl_record_host in program order, transfers to
+xpl_record_copy, device events are issued on the GPU by the instrumented
+replay kernel of libxplwork.so (each thread calls the xpl_read/xpl_write
+hooks), epochs are xpl_kernel_begin/_end around those launches, and DIAG is
+xpl_diagnose.  Returns the list of diagnose results (lists of row dicts) --
+the same shape as oracle.run_trace, so the tests compare them field by field.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+from .xpl import HOST_ACCESS_DTYPE, Context
+
+
+def _host_array(items):
+    a = np.zeros(len(items), dtype=HOST_ACCESS_DTYPE)
+    if items:
+        arr = np.array(items, dtype=np.uint64)
+        a["addr"], a["size"], a["kind"] = arr[:, 0], arr[:, 1], arr[:, 2]
+    return a
+
+
+def run_trace(ops, ctx: Context | None = None, grid=0, block=256, seed=None, host_split=None,
+              pool_words=1 << 24, stream=None):
+    """Replay `ops`.  seed: shuffle device events inside every epoch and split
+    host batches at random points (metamorphic variants); grid/block: launch
+    shape of the replay kernel (grid 0 = enough CTAs for one event each)."""
+    import torch
+
+    rng = np.random.default_rng(seed) if seed is not None else None
+    own = ctx is None
+    if own:
+        n_reg = sum(1 for op in ops if op[0] == "REG")
+        ctx = Context(pool_words=pool_words, max_rows=max(4096, n_reg + 16))
+    if stream is None:
+        stream = torch.cuda.current_stream().cuda_stream
+    results = []
+    host_items = []
+    dev = []  # (addr, size, acc) arrays of the open epoch, launched at flush points
+
+    def flush_host():
+        if not host_items:
+            return
+        arr = _host_array(host_items)
+        host_items.clear()
+        if rng is not None and host_split and arr.size > 1:
+            cuts = np.sort(rng.choice(np.arange(1, arr.size), size=min(host_split, arr.size - 1), replace=False))
+            for part in np.split(arr, cuts):
+                ctx.record_host(part)
+        else:
+            ctx.record_host(arr)
+
+    def flush_dev():
+        if not dev:
+            return
+        a = np.concatenate([d[0] for d in dev]).astype(np.uint64)
+        s = np.concatenate([d[1] for d in dev]).astype(np.uint32)
+        k = np.concatenate([d[2] for d in dev]).astype(np.uint8)
+        dev.clear()
+        if rng is not None:
+            p = rng.permutation(a.size)
+            a, s, k = a[p], s[p], k[p]
+        ta = torch.from_numpy(a.view(np.int64)).cuda()
+        ts = torch.from_numpy(s.view(np.int32)).cuda()
+        tk = torch.from_numpy(k).cuda()
+        ctx.replay(ta.data_ptr(), ts.data_ptr(), tk.data_ptr(), a.size, grid=grid, block=block, stream=stream)
+        torch.cuda.current_stream().synchronize()  # keep the temporaries alive until the launch ran
+
+    for op in ops:
+        t = op[0]
+        if t not in ("H", "HB"):
+            flush_host()
+        if t == "REG":
+            ctx.register(op[1], op[2], op[3])
+        elif t == "FREE":
+            ctx.free(op[1])
+        elif t == "KB":
+            flush_dev()
+            ctx.kernel_begin(stream)
+        elif t == "KE":
+            flush_dev()
+            ctx.kernel_end(stream)
+        elif t == "H":
+            host_items.append((op[1], op[2], op[3]))
+        elif t == "HB":
+            host_items.extend(zip(op[1].tolist(), op[2].tolist(), op[3].tolist()))
+        elif t == "D":
+            dev.append((np.array([op[1]], np.uint64), np.array([op[2]], np.uint32), np.array([op[3]], np.uint8)))
+        elif t == "DB":
+            dev.append((np.asarray(op[1], np.uint64), np.asarray(op[2], np.uint32), np.asarray(op[3], np.uint8)))
+        elif t == "X":
+            flush_dev()
+            ctx.record_copy(op[2], op[3], op[4], op[1])
+        elif t == "DIAG":
+            results.append(ctx.diagnose(op[1], op[2], op[3], bool(op[4]), op[5]))
+        else:
+            raise ValueError(op)
+    flush_host()
+    if own:
+        ctx.close()
+    return results

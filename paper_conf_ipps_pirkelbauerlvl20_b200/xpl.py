@@ -1,0 +1,212 @@
+"""ctypes binding of include/xpl.h (libxpl.so) and of the instrumented user
+kernels in libxplwork.so.  Marshalling only; names follow the C-ABI.
+
+Fails loudly (ImportError/OSError) if the shared libraries are missing: there
+is no fallback path.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+from . import LIB_PATH, WORK_PATH
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"{LIB_PATH} is not built: run __graft_entry__.build() (no CPU fallback exists)")
+
+_lib = C.CDLL(LIB_PATH, mode=C.RTLD_GLOBAL)
+_work = C.CDLL(WORK_PATH) if os.path.exists(WORK_PATH) else None
+
+u64, u32, i32, vp, sz = C.c_uint64, C.c_uint32, C.c_int, C.c_void_p, C.c_size_t
+
+XPL_OK = 0
+STATUS = {0: "XPL_OK", 1: "XPL_ERR_INVALID_ARG", 2: "XPL_ERR_OOM", 3: "XPL_ERR_OVERLAP",
+          4: "XPL_ERR_UNKNOWN_PTR", 5: "XPL_ERR_STATE", 6: "XPL_ERR_CUDA", 7: "XPL_ERR_NCCL",
+          8: "XPL_ERR_DEVICE_OVERFLOW"}
+ALLOC_DEVICE, ALLOC_MANAGED, ALLOC_HOST = 0, 1, 2
+ACC_R, ACC_W, ACC_RW = 1, 2, 3
+COPY_H2D, COPY_D2H, COPY_H2H, COPY_D2D, MEMSET_DEV = 0, 1, 2, 3, 4
+
+HOST_ACCESS_DTYPE = np.dtype([("addr", "<u8"), ("size", "<u4"), ("kind", "<u4")])
+
+
+class XplConfig(C.Structure):
+    _fields_ = [("device", i32), ("rank", i32), ("world", i32), ("nccl_comm", vp),
+                ("pool_words", u64), ("dirty_cap", u64), ("staging_recs", u64), ("max_rows", u32)]
+
+
+class XplDiagParams(C.Structure):
+    _fields_ = [("density_threshold_pct", u32), ("block_words", u64), ("min_run_words", u64)]
+
+
+class XplName(C.Structure):
+    _fields_ = [("addr", vp), ("expr", C.c_char_p), ("elem_size", u32)]
+
+
+REPORT_FIELDS = [
+    ("id", u64), ("base", u64), ("bytes", u64), ("words", u64),
+    ("kind", u32), ("live", u32), ("name_idx", u32), ("flags", u32),
+    ("w_c", u64), ("w_g", u64), ("r_cc", u64), ("r_cg", u64), ("r_gc", u64), ("r_gg", u64),
+    ("any_acc", u64), ("gpu_acc", u64), ("alternating", u64),
+    ("density_pct_any", u64), ("density_pct_gpu", u64),
+    ("low_density_blocks", u64), ("low_density_words", u64),
+    ("h2d_unused_runs", u64), ("h2d_unused_words", u64),
+    ("d2h_unneeded_runs", u64), ("d2h_unneeded_words", u64), ("ever_accessed", u64),
+]
+
+
+class XplAllocReport(C.Structure):
+    _fields_ = REPORT_FIELDS
+
+
+class XplStats(C.Structure):
+    _fields_ = [(n, u64) for n in ("epochs", "folds", "fold_full_scans", "host_records",
+                                   "host_records_packed", "merge_segments", "range_segments",
+                                   "diagnoses", "dirty_max")]
+
+
+class XplDevCtx(C.Structure):
+    _fields_ = [("rows", vp), ("n_rows", vp), ("pool", vp), ("dirty", vp), ("dirty_count", vp),
+                ("dirty_cap", u32), ("pad_", u32)]
+
+
+def _sig(name, args, res=i32, lib=_lib):
+    f = getattr(lib, name)
+    f.argtypes = args
+    f.restype = res
+    return f
+
+
+xpl_init = _sig("xpl_init", [C.POINTER(XplConfig), C.POINTER(vp)])
+xpl_finalize = _sig("xpl_finalize", [vp])
+xpl_register_alloc = _sig("xpl_register_alloc", [vp, vp, sz, i32])
+xpl_free = _sig("xpl_free", [vp, vp])
+xpl_kernel_begin = _sig("xpl_kernel_begin", [vp, vp])
+xpl_kernel_end = _sig("xpl_kernel_end", [vp, vp])
+xpl_record_host = _sig("xpl_record_host", [vp, vp, sz])
+xpl_record_copy = _sig("xpl_record_copy", [vp, vp, vp, sz, i32])
+xpl_diagnose = _sig("xpl_diagnose", [vp, C.POINTER(XplDiagParams), C.POINTER(XplName), sz,
+                                     C.POINTER(XplAllocReport), sz, C.POINTER(sz), i32])
+xpl_get_device_ctx = _sig("xpl_get_device_ctx", [vp, C.POINTER(XplDevCtx)])
+xpl_shadow_dump = _sig("xpl_shadow_dump", [vp, vp, u64, u64, vp])
+xpl_flush = _sig("xpl_flush", [vp])
+xpl_sync = _sig("xpl_sync", [vp])
+xpl_runtime_stream = _sig("xpl_runtime_stream", [vp, C.POINTER(vp)])
+xpl_get_stats = _sig("xpl_get_stats", [vp, C.POINTER(XplStats)])
+xpl_status_string = _sig("xpl_status_string", [i32], C.c_char_p)
+
+EXPORTED = ["xpl_init", "xpl_finalize", "xpl_register_alloc", "xpl_free", "xpl_kernel_begin",
+            "xpl_kernel_end", "xpl_record_host", "xpl_record_copy", "xpl_diagnose",
+            "xpl_get_device_ctx", "xpl_shadow_dump", "xpl_flush", "xpl_sync",
+            "xpl_runtime_stream", "xpl_get_stats", "xpl_status_string"]
+
+if _work is not None:
+    xplw_bind = _sig("xplw_bind", [vp], lib=_work)
+    xplw_replay = _sig("xplw_replay", [vp, vp, vp, u64, i32, i32, vp], lib=_work)
+
+
+class XplError(RuntimeError):
+    def __init__(self, fn, status):
+        super().__init__(f"{fn} -> {STATUS.get(status, status)}")
+        self.status = status
+
+
+def check(fn, status):
+    if status != XPL_OK:
+        raise XplError(fn, status)
+
+
+class Context:
+    """One xpl_ctx (one process, one GPU)."""
+
+    def __init__(self, device=0, pool_words=0, dirty_cap=0, staging_recs=0, max_rows=0):
+        cfg = XplConfig(device, 0, 1, None, pool_words, dirty_cap, staging_recs, max_rows)
+        h = vp()
+        check("xpl_init", xpl_init(C.byref(cfg), C.byref(h)))
+        self.h = h
+        if _work is not None:
+            check("xplw_bind", xplw_bind(self.h))
+
+    def close(self):
+        if self.h:
+            xpl_finalize(self.h)
+            self.h = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def register(self, ptr, nbytes, kind):
+        check("xpl_register_alloc", xpl_register_alloc(self.h, ptr, nbytes, kind))
+
+    def free(self, ptr):
+        check("xpl_free", xpl_free(self.h, ptr))
+
+    def kernel_begin(self, stream=0):
+        check("xpl_kernel_begin", xpl_kernel_begin(self.h, stream))
+
+    def kernel_end(self, stream=0):
+        check("xpl_kernel_end", xpl_kernel_end(self.h, stream))
+
+    def record_host(self, recs: np.ndarray):
+        recs = np.ascontiguousarray(recs, dtype=HOST_ACCESS_DTYPE)
+        check("xpl_record_host", xpl_record_host(self.h, recs.ctypes.data, recs.size))
+
+    def record_copy(self, dst, src, nbytes, direction):
+        check("xpl_record_copy", xpl_record_copy(self.h, dst, src, nbytes, direction))
+
+    def diagnose(self, thr=50, block_words=0, min_run=256, reset=True, names=()):
+        p = XplDiagParams(thr, block_words, min_run)
+        nn = len(names)
+        arr = (XplName * max(nn, 1))()
+        for i, a in enumerate(names):
+            arr[i].addr = a
+            arr[i].expr = b""
+            arr[i].elem_size = 0
+        cap = 64
+        while True:
+            out = (XplAllocReport * cap)()
+            n = sz(0)
+            st = xpl_diagnose(self.h, C.byref(p), arr if nn else None, nn, out, cap, C.byref(n),
+                              int(bool(reset)))
+            if st == 1 and n.value > cap:
+                cap = n.value
+                continue
+            check("xpl_diagnose", st)
+            return [{f: getattr(out[i], f) for f, _ in REPORT_FIELDS} for i in range(n.value)]
+
+    def shadow_dump(self, base, word0, n):
+        out = np.zeros(n, dtype=np.uint8)
+        check("xpl_shadow_dump", xpl_shadow_dump(self.h, base, word0, n, out.ctypes.data))
+        return out
+
+    def flush(self):
+        check("xpl_flush", xpl_flush(self.h))
+
+    def sync(self):
+        check("xpl_sync", xpl_sync(self.h))
+
+    def runtime_stream(self):
+        s = vp()
+        check("xpl_runtime_stream", xpl_runtime_stream(self.h, C.byref(s)))
+        return s.value or 0
+
+    def stats(self):
+        s = XplStats()
+        check("xpl_get_stats", xpl_get_stats(self.h, C.byref(s)))
+        return {f: getattr(s, f) for f, _ in XplStats._fields_}
+
+    def device_ctx(self):
+        d = XplDevCtx()
+        check("xpl_get_device_ctx", xpl_get_device_ctx(self.h, C.byref(d)))
+        return d
+
+    def replay(self, d_addr, d_size, d_acc, n, grid=0, block=256, stream=0):
+        """Launch the instrumented replay kernel (libxplwork) on device arrays."""
+        if grid <= 0:
+            grid = max(1, min((n + block - 1) // block, 148 * 8))
+        check("xplw_replay", xplw_replay(d_addr, d_size, d_acc, n, grid, block, stream))

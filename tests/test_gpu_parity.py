@@ -1,0 +1,184 @@
+"""GPU parity: the CUDA path, driven through the C-ABI, against the oracle on the
+same seeded traces -- element by element, every report field, bit-exact
+(all state is integer).  Run on a B200: pytest -m gpu."""
+import itertools
+import os
+
+import numpy as np
+import pytest
+
+from oracle import run_trace as oracle_run
+from xplgen.trace import (DEVICE, MANAGED, SEG_OPS, enumerated_trace, parse_text, random_trace,
+                          schedules)
+
+pytestmark = pytest.mark.gpu
+
+GOLDEN = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden")
+
+
+@pytest.fixture(scope="module")
+def gpu():
+    import torch
+    assert torch.cuda.is_available(), "GPU tests need a B200 (run under gpurun)"
+    from paper_conf_ipps_pirkelbauerlvl20_b200 import replay, xpl
+    return replay, xpl
+
+
+def compare(got, exp, what=""):
+    assert len(got) == len(exp), f"{what}: {len(got)} diagnoses vs {len(exp)}"
+    for k, (g, e) in enumerate(zip(got, exp)):
+        assert len(g) == len(e), f"{what} diag {k}: {len(g)} rows vs {len(e)}"
+        for gr, er in zip(g, e):
+            diff = {f: (gr[f], er[f]) for f in er if gr[f] != er[f]}
+            assert not diff, f"{what} diag {k} row {er['id']}: (gpu, oracle) {diff}"
+
+
+@pytest.mark.parametrize("name", sorted(f for f in os.listdir(GOLDEN) if f.endswith(".trace")))
+def test_golden(gpu, name):
+    replay, _ = gpu
+    ops = parse_text(open(os.path.join(GOLDEN, name)).read())
+    compare(replay.run_trace(ops), oracle_run(ops), name)
+
+
+@pytest.mark.parametrize("schedule", schedules(3), ids=lambda s: "".join(s[0]) + "".join("d" if x else "-" for x in s[1]))
+def test_bruteforce(gpu, schedule):
+    replay, _ = gpu
+    nseg = len(schedule[0])
+    if nseg <= 2:
+        asg = list(itertools.product(SEG_OPS, repeat=nseg))
+    else:
+        rng = np.random.default_rng(0x58504C00)
+        allasg = list(itertools.product(range(len(SEG_OPS)), repeat=3))
+        pick = rng.choice(len(allasg), size=20000, replace=False)
+        asg = [tuple(SEG_OPS[i] for i in allasg[p]) for p in pick]
+    for kind in (MANAGED, DEVICE):
+        ops = enumerated_trace(schedule, asg, kind=kind)
+        compare(replay.run_trace(ops, pool_words=1 << 26), oracle_run(ops), f"kind={kind}")
+
+
+@pytest.mark.parametrize("seed", range(24))
+def test_random(gpu, seed):
+    replay, _ = gpu
+    ops = random_trace(0x58504C00 + seed, n_allocs=6, n_steps=80, max_words=5000)
+    exp = oracle_run(ops)
+    compare(replay.run_trace(ops), exp, "plain")
+    # metamorphic: shuffled device events, other launch shapes, split host batches
+    compare(replay.run_trace(ops, seed=seed, grid=3, block=64, host_split=5), exp, "shuffled")
+    compare(replay.run_trace(ops, seed=seed + 1000, grid=1, block=32, host_split=1), exp, "1 warp")
+
+
+def big_trace(seed, words=(100_003, 32_768, 65_536 + 17, 1, 16, 31), n_events=400_000):
+    """Several tiles per allocation and ragged tails; dense and sparse accesses."""
+    rng = np.random.default_rng(seed)
+    ops, bases = [], []
+    b = 0x2000_0000
+    for i, w in enumerate(words):
+        ops.append(("REG", b, 4 * w - (i % 3), i % 3))
+        bases.append((b, 4 * w - (i % 3)))
+        b += ((4 * w + 65535) // 65536 + 1) * 65536
+    for epoch in range(6):
+        # host segment: a contiguous init of one array + random accesses
+        bb, nb = bases[epoch % len(bases)]
+        ops.append(("X", 0, bb, 0x7000_0000, nb // 2))
+        j = rng.integers(0, len(bases), size=20000)
+        off = rng.integers(0, 1 << 30, size=20000) % np.array([n for _, n in bases])[j]
+        addr = np.array([bases[x][0] for x in j], dtype=np.uint64) + off.astype(np.uint64)
+        ops.append(("HB", addr, rng.choice([1, 4, 8], size=addr.size).astype(np.uint32),
+                    rng.integers(1, 4, size=addr.size).astype(np.uint8)))
+        ops.append(("KB",))
+        j = rng.integers(0, len(bases), size=n_events)
+        off = rng.integers(0, 1 << 30, size=n_events) % np.array([n for _, n in bases])[j]
+        addr = np.array([bases[x][0] for x in j], dtype=np.uint64) + (off & ~3).astype(np.uint64)
+        ops.append(("DB", addr, np.full(addr.size, 4, np.uint32), rng.integers(1, 4, size=addr.size).astype(np.uint8)))
+        # a dense streaming kernel over one allocation
+        bb, nb = bases[(epoch + 1) % len(bases)]
+        a = bb + 4 * np.arange(nb // 4, dtype=np.uint64)
+        ops.append(("DB", a, np.full(a.size, 4, np.uint32), np.full(a.size, 1 + epoch % 3, np.uint8)))
+        ops.append(("KE",))
+        thr, blk, mr = [(50, 0, 256), (30, 1000, 16), (90, 64, 1), (50, 32768, 300), (10, 7, 3), (100, 0, 1)][epoch]
+        ops.append(("DIAG", thr, blk, mr, int(epoch % 2 == 0), ()))
+        if epoch == 3:
+            ops.append(("FREE", bases[0][0]))
+            ops.append(("REG", bases[0][0], 4 * 777, 0))
+            bases[0] = (bases[0][0], 4 * 777)
+    return ops
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_multi_tile(gpu, seed):
+    replay, _ = gpu
+    ops = big_trace(0x58504C00 + seed)
+    compare(replay.run_trace(ops, pool_words=1 << 24), oracle_run(ops), "big")
+
+
+def test_dirty_overflow_and_small_staging(gpu):
+    replay, xpl = gpu
+    ops = random_trace(0x58504C77, n_allocs=6, n_steps=60, max_words=5000)
+    exp = oracle_run(ops)
+    with xpl.Context(pool_words=1 << 22, dirty_cap=7, staging_recs=5) as ctx:
+        compare(replay.run_trace(ops, ctx=ctx), exp, "tiny capacities")
+        st = ctx.stats()
+        assert st["fold_full_scans"] > 0
+
+
+def test_shadow_dump_matches_oracle(gpu):
+    replay, xpl = gpu
+    from oracle import Oracle
+    ops = random_trace(0x58504C55, n_allocs=4, n_steps=40, max_words=3000)
+    ops = [o for o in ops if o[0] != "DIAG"]  # keep the interval bits
+    o = Oracle()
+    for op in ops:
+        o.op(op)
+    with xpl.Context(pool_words=1 << 22) as ctx:
+        replay.run_trace(ops, ctx=ctx)
+        live = {}
+        rid = 0
+        for op in ops:
+            if op[0] == "REG":
+                live[op[1]] = (rid, op[2])
+                rid += 1
+        for base, (rid, nb) in live.items():
+            try:
+                got = ctx.shadow_dump(base, 0, (nb + 3) // 4)
+            except xpl.XplError:
+                continue  # freed
+            exp = np.array([o.peek(rid, w) for w in range((nb + 3) // 4)], dtype=np.uint8)
+            assert np.array_equal(got & 0xFD, exp), base  # bit1 (P) is GPU-internal and 0 here
+
+
+def test_api_errors(gpu):
+    _, xpl = gpu
+    import torch
+    s = torch.cuda.current_stream().cuda_stream
+    with xpl.Context(pool_words=1 << 16, max_rows=4) as ctx:
+        assert ctx.diagnose() == []
+        ctx.register(0x1000, 64, 1)
+        with pytest.raises(xpl.XplError) as e:
+            ctx.register(0x1020, 64, 1)
+        assert e.value.status == 3
+        with pytest.raises(xpl.XplError) as e:
+            ctx.free(0x1004)
+        assert e.value.status == 4
+        with pytest.raises(xpl.XplError) as e:
+            ctx.kernel_end(s)
+        assert e.value.status == 5
+        ctx.kernel_begin(s)
+        with pytest.raises(xpl.XplError) as e:
+            ctx.diagnose()
+        assert e.value.status == 5
+        with pytest.raises(xpl.XplError) as e:
+            ctx.register(0x9000, 4, 0)
+        assert e.value.status == 5
+        ctx.kernel_end(s)
+        with pytest.raises(xpl.XplError) as e:
+            ctx.register(0x5000, 0, 0)
+        assert e.value.status == 1
+        for i in range(3):
+            ctx.register(0x10000 * (i + 2), 8, 0)
+        with pytest.raises(xpl.XplError) as e:  # table full
+            ctx.register(0x100000, 8, 0)
+        assert e.value.status == 2
+        with pytest.raises(xpl.XplError) as e:  # pool full
+            ctx.free(0x20000)
+            ctx.register(0x200000, 4 << 20, 0)
+        assert e.value.status == 2
