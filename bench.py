@@ -1,0 +1,303 @@
+#!/usr/bin/env python
+"""Benchmark of the B200-native XPlacer recording + diagnosis hot path.
+
+One STEP = one pass of the whole hot path over the
+configs[1] workload of BASELINE.json: the Rodinia-shaped instrumented programs
+(hotspot 1024x1024 x 20 iterations, backprop 640K x 16) run end to end through
+the C-ABI -- registration, host-tracer batches (merge), traced transfers
+(range apply), instrumented kernels (device hooks) in GPU epochs (fold), and a
+diagnose after every iteration and at the end (diagnose kernels), then frees.
+
+Metric (BASELINE.json): recorded accesses/s -- host tracer calls + device hook
+calls + transferred words -- per second of device time, whole job (all ranks).
+value: data of the apps resident in HBM (their cudaMemcpy not performed).
+e2e:   the same programs with their real host<->device copies (pinned host
+       buffers) inside the timed region.
+Also reported: the diagnose-kernel bandwidth, kernel-only and whole-program
+slowdown vs the uninstrumented twins, the roofline of the dominant runtime
+kernel (live CUDA-event timing on the runtime stream), and the oracle's rate
+on the host cores (cpu_baseline).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl xpl|reference]
+Under torchrun each rank runs its own instance (independent problems, weak
+scaling, no data-path collective); rank 0 prints one JSON line.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+HOT = (1024, 1024, 20)
+BACKPROP = (655360, 16)
+PARAMS = (50, 0, 256)  # threshold 50 %, whole-allocation blocks, min run 256 words
+WORKLOAD = "rodinia: hotspot 1024x1024x20 + backprop 640Kx16"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["xpl", "reference"], default="xpl")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    return ap.parse_args()
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+
+    def __init__(self, idx):
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--id={idx}", f"--query-gpu={q}", "--format=csv,noheader,nounits",
+                                       "-lms", "100"], stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        self.p.wait()
+        self.f.flush()
+        self.f.seek(0)
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in self.f.read().splitlines():
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                sm.append(float(parts[1]))
+                mx = float(parts[2])
+            except ValueError:
+                continue
+            for n, v in zip(names, parts[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        os.unlink(self.f.name)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def cpu_baseline(seconds_budget=20.0):
+    """The oracle as it stands, on a bounded sample of the same workload:
+    hotspot 1024x1024 (first iterations) replayed event by event."""
+    from oracle import Oracle
+    from xplgen import rodinia
+    rows, cols, _ = HOT
+    spec = rodinia.hotspot_spec(rows, cols)
+    addrs, _, _ = rodinia.layout(spec, 1 << 40, 1 << 44)
+    iters = 2
+    ops = rodinia.hotspot_trace(addrs, spec, rows, cols, iters, True, PARAMS)
+    n_acc = 2 * rows * cols + iters * rodinia.hotspot_accesses(rows, cols)
+    o = Oracle()
+    t0 = time.perf_counter()
+    for op in ops:
+        if op[0] == "X" and op[1] == 1:  # stop before the final transfer: sample = init + iterations
+            break
+        o.op(op)
+        if time.perf_counter() - t0 > seconds_budget * 3:
+            break
+    dt = time.perf_counter() - t0
+    o.close()
+    n_acc += 2 * rows * cols  # the two H2D transfers
+    return {"value": n_acc / dt, "unit": "accesses/s", "cores": 1, "kind": "oracle",
+            "sample": f"hotspot {rows}x{cols}: host init + 2 H2D + {iters} instrumented iterations "
+                      f"with a diagnose after each ({n_acc} accesses, {dt:.1f} s, 1 thread)"}
+
+
+def reference_main(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    steps = []
+    for _ in range(max(1, args.steps)):
+        steps.append(cpu_baseline(seconds_budget=5.0))
+    v = statistics.median(s["value"] for s in steps)
+    line = {"impl": "reference", "metric": "recorded accesses/s", "value": v, "unit": "accesses/s",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8",
+            "data": "synthetic", "config": {"workload": WORKLOAD + " (oracle sample)"},
+            "cpu_baseline": {"value": v, "unit": "accesses/s", "cores": 1, "kind": "oracle",
+                             "sample": steps[0]["sample"]},
+            "e2e": {"value": v, "unit": "accesses/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return reference_main(args)
+    import torch
+    import torch.distributed as dist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+
+    from paper_conf_ipps_pirkelbauerlvl20_b200 import apps, xpl
+    from xplgen import rodinia
+
+    ctx = xpl.Context(device=local, pool_words=1 << 28, max_rows=256)
+    rs = torch.cuda.ExternalStream(ctx.runtime_stream())
+    us = torch.cuda.Stream()
+    hs = rodinia.hotspot_spec(HOT[0], HOT[1])
+    bs = rodinia.backprop_spec(*BACKPROP)
+    ar_h, ar_b = apps.Arena(hs), apps.Arena(bs)
+    rodinia.fill_inputs("hotspot", ar_h.host_views(), 0x58504C01)
+    rodinia.fill_inputs("backprop", ar_b.host_views(), 0x58504C01)
+    flush_buf = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")  # > 126 MB L2
+
+    def step(c, do_copies, time_kernels=False):
+        counts = [0, 0, 0, 0, 0.0, 0.0]
+        for fn, ar, a in ((apps.hotspot, ar_h, HOT), (apps.backprop, ar_b, BACKPROP)):
+            run = apps.Run(c, us.cuda_stream, do_copies=do_copies, diag_each=True, params=PARAMS,
+                           time_kernels=time_kernels)
+            fn(run, ar, *a)
+            counts[0] += run.r.dev_accesses
+            counts[1] += run.r.host_accesses
+            counts[2] += run.r.copy_words
+            counts[3] += run.r.epochs
+            counts[4] += run.r.kernel_ms
+            counts[5] += run.r.host_ms
+        return counts
+
+    def timed(c, do_copies, steps, stream):
+        total, counts = 0.0, None
+        for _ in range(steps):
+            flush_buf.random_(0, 255)  # flush L2 between steps (untimed)
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            counts = step(c, do_copies)
+            e1.record(stream)
+            e1.synchronize()
+            us.synchronize()
+            total += e0.elapsed_time(e1)
+        return total, counts
+
+    for _ in range(args.warmup):
+        step(ctx, False)
+    torch.cuda.synchronize()
+
+    # --- value: device-timed, app data resident -------------------------------
+    st0 = ctx.stats()
+    ctx.profile(True)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clk = Clocks(local)
+    ms_total, counts = timed(ctx, False, args.steps, rs)
+    clocks = clk.stop()
+    prof = ctx.profile_read(reset=True)
+    ctx.profile(False)
+    st1 = ctx.stats()
+    per_step = counts[0] + counts[1] + counts[2]
+    ms_max = ms_total
+    if world > 1:
+        t = torch.tensor([ms_total], device="cuda", dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms_max = float(t.item())
+    value = per_step * args.steps * world / (ms_max / 1e3)
+    launches = (st1["kernel_launches"] - st0["kernel_launches"]) + counts[3] * args.steps
+
+    # --- e2e: with the programs' real copies -----------------------------------
+    for _ in range(1):
+        step(ctx, True)
+    st0 = ctx.stats()
+    if world > 1:
+        dist.barrier()
+    e2e_ms, _ = timed(ctx, True, args.steps, rs)
+    st1 = ctx.stats()
+    if world > 1:
+        t = torch.tensor([e2e_ms], device="cuda", dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_ms = float(t.item())
+    rec_bytes = 8 * (st1["host_records_packed"] - st0["host_records_packed"]) // args.steps
+    app_h2d = 4 * (2 * HOT[0] * HOT[1]) + 4 * ((BACKPROP[0] + 1) * (1 + 2 * (BACKPROP[1] + 1)) + BACKPROP[1] + 1)
+    app_d2h = 4 * HOT[0] * HOT[1] + 4 * ((BACKPROP[0] + 1) * (BACKPROP[1] + 2) + (BACKPROP[0] // 16) * BACKPROP[1])
+    n_diag_rows = 2 * (HOT[2] + 1) * 6  # upper bound of report rows per step
+    e2e = {"value": per_step * args.steps * world / (e2e_ms / 1e3), "unit": "accesses/s",
+           "h2d_bytes_per_step": rec_bytes + app_h2d,
+           "d2h_bytes_per_step": app_d2h + 208 * n_diag_rows}
+
+    # --- uninstrumented twins (slowdown, Table III context) ------------------
+    for _ in range(1):
+        step(None, False)
+    twin_ms, _ = timed(None, False, args.steps, us)
+
+    # --- breakdown (untimed pass with per-kernel events) ----------------------
+    bi = step(ctx, False, time_kernels=True)
+    bt = step(None, False, time_kernels=True)
+    torch.cuda.synchronize()
+
+    # --- roofline of the dominant runtime kernel -------------------------------
+    peak, peak_src = peaks()
+    dom = max(("diag_tile", "merge", "range", "fold"), key=lambda k: prof[k]["ms"])
+    d = prof[dom]
+    achieved = (d["bytes"] / d["launches"]) / (d["ms"] / d["launches"] / 1e3) / 1e9 if d["launches"] else 0.0
+    roof = {"kernel": dom, "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+            "frac": achieved / peak, "traffic": None, "peak_source": peak_src,
+            "algorithmic_bytes_per_launch": d["bytes"] / max(1, d["launches"]),
+            "avg_launch_ms": d["ms"] / max(1, d["launches"]),
+            "share_of_step": d["ms"] / ms_total}
+    dg = prof["diag_tile"]
+    line = {
+        "metric": "recorded accesses/s (host tracer + device hooks + transferred words)",
+        "value": value, "unit": "accesses/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": ms_max / args.steps, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+        "config": {"workload": WORKLOAD, "accesses_per_step": per_step, "device_accesses": counts[0],
+                   "host_accesses": counts[1], "transfer_words": counts[2], "epochs_per_step": counts[3],
+                   "diag_params": {"threshold_pct": PARAMS[0], "block_words": PARAMS[1], "min_run": PARAMS[2]},
+                   "l2": "flushed between steps (256 MB write, untimed)", "parallelism": f"replicas x{world}"},
+        "roofline": roof,
+        "diagnose_gbs": (dg["bytes"] / (dg["ms"] / 1e3) / 1e9) if dg["ms"] else None,
+        "runtime_kernels": {k: {"launches": v["launches"], "ms_per_step": v["ms"] / args.steps,
+                                "gbs": (v["bytes"] / (v["ms"] / 1e3) / 1e9) if v["ms"] else None}
+                            for k, v in prof.items()},
+        "breakdown_ms_per_step": {"instrumented_kernels": bi[4], "twin_kernels": bt[4],
+                                  "host_tracer": bi[5],
+                                  "runtime_kernels": sum(v["ms"] for k, v in prof.items() if k != "diagnose" and k != "diag_tile") / args.steps + prof["diagnose"]["ms"] / args.steps},
+        "slowdown": {"kernels_only": bi[4] / bt[4] if bt[4] else None,
+                     "whole_program": (ms_total / args.steps) / (twin_ms / args.steps),
+                     "twin_ms_per_step": twin_ms / args.steps,
+                     "paper_context": "Table III P:L431-443: 5x-20x, avg ~15x (Intel E5-2695 v4 + Pascal, CUDA 9.2)"},
+        "e2e": e2e, "gpu_launches": int(launches), "clocks": clocks,
+    }
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline()
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    ctx.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -122,7 +122,8 @@ struct xpl_dev_ctx; /* defined in xpl_device.cuh */
 /* Counters the runtime keeps about itself (not part of the paper's output). */
 typedef struct {
   uint64_t epochs, folds, fold_full_scans, host_records, host_records_packed,
-      merge_segments, range_segments, diagnoses, dirty_max;
+      merge_segments, range_segments, diagnoses, dirty_max,
+      kernel_launches; /* runtime kernels launched (not counting user kernels) */
 } xpl_stats;
 
 /* Create a context on cfg->device.  *out is owned by the caller until
@@ -153,6 +154,14 @@ xpl_status xpl_kernel_end(xpl_ctx* ctx, void* stream);
  * ignored.  Inside an open GPU epoch the records are applied after
  * the epoch closes (D20). */
 xpl_status xpl_record_host(xpl_ctx* ctx, const xpl_host_access* recs, size_t n);
+
+/* Coalesced host ranges (what xpl_host.h's inline tracer emits): each record
+ * stands for a run of consecutive accesses of one kind covering the bytes
+ * [addr, addr+size); every word of every live allocation overlapping it is
+ * accessed once, in program order with the other records.  Equal to
+ * xpl_record_host on the individual accesses whenever no individual access
+ * straddles two allocations.  Same ordering and epoch rules as xpl_record_host. */
+xpl_status xpl_record_host_ranges(xpl_ctx* ctx, const xpl_host_access* recs, size_t n);
 
 /* The transfer wrappers (D7).  dst/src are the cudaMemcpy arguments. */
 xpl_status xpl_record_copy(xpl_ctx* ctx, const void* dst, const void* src, size_t bytes,
@@ -186,6 +195,28 @@ xpl_status xpl_sync(xpl_ctx* ctx);
 /* The runtime's own stream (cudaStream_t as void*), e.g. for timing events. */
 xpl_status xpl_runtime_stream(xpl_ctx* ctx, void** stream);
 xpl_status xpl_get_stats(xpl_ctx* ctx, xpl_stats* out);
+
+/* Live kernel timing (for the roofline numbers of bench.py): with profiling on,
+ * every runtime kernel is bracketed by CUDA events on the runtime stream.
+ * xpl_profile_read waits for the runtime stream and returns, per kernel class,
+ * the launches, the summed event time and the ALGORITHMIC bytes moved
+ * (fold 12 B per dirty u32; merge 8 B per record + 2 B per word;
+ * range 2 B per word; diagnose 1 B per word + 1 B per word when resetting). */
+typedef enum {
+  XPL_K_FOLD = 0,
+  XPL_K_MERGE = 1,
+  XPL_K_RANGE = 2,
+  XPL_K_DIAG_TILE = 3, /* the one-pass shadow kernel of diagnose               */
+  XPL_K_DIAGNOSE = 4,  /* the whole diagnose call (all its kernels + copies)   */
+  XPL_K_NCLASS = 5
+} xpl_kernel_class;
+typedef struct {
+  uint64_t launches;
+  double ms;
+  uint64_t bytes;
+} xpl_kernel_time;
+xpl_status xpl_profile(xpl_ctx* ctx, int enable);
+xpl_status xpl_profile_read(xpl_ctx* ctx, xpl_kernel_time out[XPL_K_NCLASS], int reset);
 
 const char* xpl_status_string(xpl_status s);
 

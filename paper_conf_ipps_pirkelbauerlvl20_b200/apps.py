@@ -1,0 +1,113 @@
+"""Binding of the instrumented workload applications in libxplwork.so (xplw.h).
+
+Allocates each app's arrays (device arena in HBM via torch, host arena pinned),
+runs the native C++ program through ctypes and returns its reports.  The apps
+call the C-ABI themselves; this module only marshals.
+"""
+from __future__ import annotations
+
+import ctypes as C
+
+import numpy as np
+
+from . import xpl
+from .xpl import REPORT_FIELDS, XplAllocReport, XplDiagParams
+
+u64, u32, i32, vp, sz = C.c_uint64, C.c_uint32, C.c_int, C.c_void_p, C.c_size_t
+MAXA = 24
+
+
+class XplwArrays(C.Structure):
+    _fields_ = [("addr", u64 * MAXA), ("bytes", u64 * MAXA), ("kind", u32 * MAXA), ("n", i32)]
+
+
+class XplwRun(C.Structure):
+    _fields_ = [("ctx", vp), ("stream", vp), ("do_copies", i32), ("diag_each", i32),
+                ("params", XplDiagParams), ("out", vp), ("out_cap", sz), ("n_out", sz),
+                ("diag_rows", vp), ("diag_cap", sz), ("n_diag", sz), ("dev_accesses", u64),
+                ("host_accesses", u64), ("copy_words", u64), ("epochs", u64), ("status", i32),
+                ("time_kernels", i32), ("kernel_ms", C.c_double), ("host_ms", C.c_double)]
+
+
+_w = xpl._work
+_w.xplw_hotspot.argtypes = [C.POINTER(XplwRun), C.POINTER(XplwArrays), i32, i32, i32]
+_w.xplw_backprop.argtypes = [C.POINTER(XplwRun), C.POINTER(XplwArrays), i32, i32]
+for f in ("xplw_hotspot", "xplw_backprop"):
+    getattr(_w, f).restype = i32
+
+
+class Arena:
+    """Device + pinned-host memory for one app, laid out by xplgen.rodinia.layout."""
+
+    def __init__(self, spec):
+        import torch
+        from xplgen.rodinia import arena_sizes, layout
+        d, h = arena_sizes(spec)
+        self.dev = torch.empty(d + 4096, dtype=torch.uint8, device="cuda")
+        self.host = torch.empty(h + 4096, dtype=torch.uint8).pin_memory()
+        db = (self.dev.data_ptr() + 4095) // 4096 * 4096
+        hb = (self.host.data_ptr() + 4095) // 4096 * 4096
+        self.addrs, _, _ = layout(spec, db, hb)
+        self.spec = spec
+        self.arrays = XplwArrays()
+        for i, (a, s) in enumerate(zip(self.addrs, spec)):
+            self.arrays.addr[i] = a
+            self.arrays.bytes[i] = s[1]
+            self.arrays.kind[i] = s[2]
+        self.arrays.n = len(spec)
+
+    def host_views(self):
+        """numpy views of the host arrays (for seeding inputs)."""
+        base = self.host.data_ptr()
+        hv = self.host.numpy()
+        out = []
+        for a, s in zip(self.addrs, self.spec):
+            if s[3] == "host":
+                o = a - base
+                out.append(hv[o:o + s[1]])
+        return out
+
+
+class Run:
+    """One xplw_run: the context (or None = uninstrumented twin) and outputs."""
+
+    def __init__(self, ctx, stream, do_copies=False, diag_each=True, params=(50, 0, 256), out_cap=4096,
+                 time_kernels=False):
+        self.r = XplwRun()
+        self.r.time_kernels = int(time_kernels)
+        self.r.ctx = ctx.h if ctx is not None else None
+        self.r.stream = stream
+        self.r.do_copies = int(do_copies)
+        self.r.diag_each = int(diag_each)
+        self.r.params = XplDiagParams(*params)
+        self.out = (XplAllocReport * out_cap)()
+        self.rows = (u32 * 4096)()
+        self.r.out = C.cast(self.out, vp)
+        self.r.out_cap = out_cap
+        self.r.diag_rows = C.cast(self.rows, vp)
+        self.r.diag_cap = 4096
+
+    def reports(self):
+        """The diagnoses of the run, each a list of row dicts."""
+        res, k = [], 0
+        for d in range(self.r.n_diag):
+            n = self.rows[d]
+            res.append([{f: getattr(self.out[k + i], f) for f, _ in REPORT_FIELDS} for i in range(n)])
+            k += n
+        return res
+
+    def check(self):
+        if self.r.status:
+            raise xpl.XplError("workload", self.r.status)
+
+
+def hotspot(run: Run, arena: Arena, rows, cols, iters):
+    st = _w.xplw_hotspot(C.byref(run.r), C.byref(arena.arrays), rows, cols, iters)
+    run.check()
+    return st
+
+
+def backprop(run: Run, arena: Arena, n_in, hid):
+    st = _w.xplw_backprop(C.byref(run.r), C.byref(arena.arrays), n_in, hid)
+    run.check()
+    return st

@@ -63,6 +63,7 @@ __global__ void __launch_bounds__(256) fold_kernel(uint32_t* __restrict__ pool,
       if (n > stats[0]) stats[0] = n;
       if (n > cap) stats[1] += 1;
       stats[2] += 1;
+      stats[3] += n <= cap ? n : pool_u32;
       *dirty_count = 0;
       *done_ctr = 0;
       __threadfence();
@@ -668,10 +669,12 @@ void launch_range(cudaStream_t s, const RangeDesc* d_ranges, uint32_t nr, uint64
 void launch_diag(cudaStream_t s, const DiagRow* rows, uint32_t nrows, const uint32_t* tile_row,
                  uint64_t ntiles, uint64_t nblocks, const DiagParams& p, uint32_t* pool,
                  unsigned long long* cnt, TileSum* tiles, uint32_t* blk_cnt,
-                 xpl_alloc_report* out) {
+                 xpl_alloc_report* out, cudaEvent_t tile_ev0, cudaEvent_t tile_ev1) {
   cudaMemsetAsync(cnt, 0, sizeof(unsigned long long) * C_NCNT * nrows, s);
   if (p.block_words && nblocks) cudaMemsetAsync(blk_cnt, 0, sizeof(uint32_t) * nblocks, s);
+  if (tile_ev0) cudaEventRecord(tile_ev0, s);
   if (ntiles) diag_tile_kernel<<<(unsigned)ntiles, kDiagThreads, 0, s>>>(rows, tile_row, p, pool, cnt, tiles, blk_cnt);
+  if (tile_ev1) cudaEventRecord(tile_ev1, s);
   stitch_kernel<<<(nrows * 32 + 255) / 256, 256, 0, s>>>(rows, nrows, tiles, p.min_run, cnt);
   if (p.block_words && nblocks)
     block_eval_kernel<<<grid_for(nblocks, 256, 148 * 8), 256, 0, s>>>(rows, nrows, nblocks, blk_cnt,

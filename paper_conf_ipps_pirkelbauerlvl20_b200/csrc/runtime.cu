@@ -132,6 +132,18 @@ struct xpl_ctx {
   xpl_alloc_report* h_rep = nullptr;
 
   xpl_stats st;
+
+  // live kernel timing (xpl_profile)
+  struct ProfRec {
+    int cls;
+    cudaEvent_t a, b;
+    uint64_t bytes;
+  };
+  bool prof = false;
+  std::vector<ProfRec> prof_pending;
+  std::vector<cudaEvent_t> prof_free;
+  xpl_kernel_time prof_acc[XPL_K_NCLASS];
+  unsigned long long fold_entries_seen = 0;
 };
 
 namespace {
@@ -163,6 +175,36 @@ bool to_words(xpl_ctx* c, uint64_t addr, uint64_t size, uint64_t* g0, uint64_t* 
 }
 
 xpl_status flush(xpl_ctx* c);
+
+cudaEvent_t prof_event(xpl_ctx* c) {
+  if (!c->prof_free.empty()) {
+    cudaEvent_t e = c->prof_free.back();
+    c->prof_free.pop_back();
+    return e;
+  }
+  cudaEvent_t e = nullptr;
+  cudaEventCreate(&e);
+  return e;
+}
+
+// Bracket the next launches on the runtime stream (only when profiling).
+int prof_begin(xpl_ctx* c, int cls, uint64_t bytes, bool record = true) {
+  if (!c->prof) return -1;
+  xpl_ctx::ProfRec r{cls, prof_event(c), prof_event(c), bytes};
+  if (record) cudaEventRecord(r.a, c->rs);
+  c->prof_pending.push_back(r);
+  return (int)c->prof_pending.size() - 1;
+}
+void prof_end(xpl_ctx* c, int i) {
+  if (i >= 0) cudaEventRecord(c->prof_pending[i].b, c->rs);
+}
+
+uint64_t words_of(const uint64_t* h, size_t n) {
+  uint64_t w = 0;
+  for (size_t i = 0; i < n; ++i) w += rec_nw(h[i]);
+  return w;
+}
+
 
 // Append one packed record to staging, coalescing with the previous one when
 // that is exact: same access kind and touching/overlapping words for R or W
@@ -231,6 +273,7 @@ xpl_status ensure_first_w(xpl_ctx* c) {
   if (c->d_first_w) return XPL_OK;
   CK(cudaMalloc(&c->d_first_w, sizeof(uint32_t) * c->pool_words));
   launch_fill_u32(c->rs, c->d_first_w, c->pool_words, 0xFFFFFFFFu);
+  c->st.kernel_launches += 1;
   return XPL_OK;
 }
 
@@ -247,8 +290,11 @@ xpl_status flush(xpl_ctx* c) {
     xpl_status s = XPL_OK;
     if (c->stage_has_r && c->stage_has_w) s = ensure_first_w(c);
     if (s) return s;
+    const int pi = prof_begin(c, XPL_K_MERGE, c->prof ? 8 * n + 2 * words_of(h, n) : 0);
     launch_merge(c->rs, c->d_stage, (uint32_t)n, c->stage_has_r, c->stage_has_w, c->d_first_w,
                  (uint32_t*)c->d_pool);
+    c->st.kernel_launches += 1 + c->stage_has_w + (c->stage_has_r && c->stage_has_w);
+    prof_end(c, pi);
     c->st.merge_segments++;
   } else {
     // Segment the batch.  Range descriptors of this flush go to h_ranges.
@@ -310,16 +356,24 @@ xpl_status flush(xpl_ctx* c) {
         uint64_t nvec = c->h_ranges[sg.start + sg.n - 1].vbase +
                         ((c->h_ranges[sg.start + sg.n - 1].g0 + c->h_ranges[sg.start + sg.n - 1].nw - 1) >> 4) -
                         (c->h_ranges[sg.start + sg.n - 1].g0 >> 4) + 1;
+        uint64_t rw = 0;
+        for (size_t i = sg.start; i < sg.start + sg.n; ++i) rw += c->h_ranges[i].nw;
+        const int pi = prof_begin(c, XPL_K_RANGE, 2 * rw);
         launch_range(c->rs, c->d_ranges + sg.start, (uint32_t)sg.n, nvec, (uint32_t*)c->d_pool,
                      c->d_dirty, c->d_misc, (uint32_t)c->cfg.dirty_cap);
+        c->st.kernel_launches += 1;
+        prof_end(c, pi);
         c->st.range_segments++;
       } else {
         if (sg.has_r && sg.has_w) {
           s = ensure_first_w(c);
           if (s) return s;
         }
+        const int pi = prof_begin(c, XPL_K_MERGE, c->prof ? 8 * sg.n + 2 * words_of(h + sg.start, sg.n) : 0);
         launch_merge(c->rs, c->d_stage + sg.start, (uint32_t)sg.n, sg.has_r, sg.has_w,
                      c->d_first_w, (uint32_t*)c->d_pool);
+        c->st.kernel_launches += 1 + sg.has_w + (sg.has_r && sg.has_w);
+        prof_end(c, pi);
         c->st.merge_segments++;
       }
     }
@@ -375,15 +429,25 @@ xpl_status gpu_ranges(xpl_ctx* c, const RangeDesc* rd, size_t nr) {
   }
   CK(cudaMemcpyAsync(c->d_ranges, c->h_ranges, sizeof(RangeDesc) * nr, cudaMemcpyHostToDevice, c->rs));
   CK(cudaEventRecord(c->ranges_ev, c->rs));
+  uint64_t rw = 0;
+  for (size_t i = 0; i < nr; ++i) rw += rd[i].nw;
+  const int pi = prof_begin(c, XPL_K_RANGE, 2 * rw);
   launch_range(c->rs, c->d_ranges, (uint32_t)nr, v, (uint32_t*)c->d_pool, c->d_dirty, c->d_misc,
                (uint32_t)c->cfg.dirty_cap);
+  c->st.kernel_launches += 1;
+  prof_end(c, pi);
   return cudaGetLastError() == cudaSuccess ? XPL_OK : XPL_ERR_CUDA;
 }
 
 void fold(xpl_ctx* c) {
+  const int pi = prof_begin(c, XPL_K_FOLD, 0);
   launch_fold(c->rs, (uint32_t*)c->d_pool, c->pool_words / 4, c->d_dirty, c->d_misc,
               (uint32_t)c->cfg.dirty_cap, c->d_misc + 1, c->d_stats);
+  c->st.kernel_launches += 1;
+  prof_end(c, pi);
 }
+
+
 
 }  // namespace
 
@@ -484,6 +548,11 @@ xpl_status xpl_finalize(xpl_ctx* c) {
   cudaFree(c->d_rep);
   cudaFreeHost(c->h_rep);
   for (cudaEvent_t e : c->ev_pool) cudaEventDestroy(e);
+  for (cudaEvent_t e : c->prof_free) cudaEventDestroy(e);
+  for (auto& r : c->prof_pending) {
+    cudaEventDestroy(r.a);
+    cudaEventDestroy(r.b);
+  }
   for (cudaEvent_t e : {c->stage_ev[0], c->stage_ev[1], c->table_ev, c->ranges_ev, c->ev_begin})
     if (e) cudaEventDestroy(e);
   if (c->rs) cudaStreamDestroy(c->rs);
@@ -602,6 +671,43 @@ xpl_status xpl_record_host(xpl_ctx* c, const xpl_host_access* recs, size_t n) {
   return XPL_OK;
 }
 
+xpl_status xpl_record_host_ranges(xpl_ctx* c, const xpl_host_access* recs, size_t n) {
+  if (!c || (!recs && n)) return XPL_ERR_INVALID_ARG;
+  for (size_t i = 0; i < n; ++i) {
+    const uint32_t acc = recs[i].kind;
+    if (acc < 1 || acc > 3) return XPL_ERR_INVALID_ARG;
+    uint64_t a = recs[i].addr;
+    const uint64_t e = a + recs[i].size;
+    while (a < e) {
+      const Row* r = lookup(c, a);
+      if (!r) {  // skip to the next live allocation inside the range, if any
+        auto it = c->live.upper_bound(a);
+        if (it == c->live.end() || it->first >= e) break;
+        a = it->first;
+        continue;
+      }
+      const uint64_t re = r->base + r->bytes;
+      const uint64_t pe = e < re ? e : re;
+      uint64_t g0, nw;
+      if (to_words(c, a, pe - a, &g0, &nw)) {
+        if (c->depth) {
+          while (nw > kMaxRecWords) {
+            c->deferred.push_back(pack_rec(g0, kMaxRecWords, acc));
+            g0 += kMaxRecWords;
+            nw -= kMaxRecWords;
+          }
+          c->deferred.push_back(pack_rec(g0, nw, acc));
+        } else {
+          xpl_status s = stage_push(c, g0, nw, acc);
+          if (s) return s;
+        }
+      }
+      a = pe;
+    }
+  }
+  return XPL_OK;
+}
+
 xpl_status xpl_record_copy(xpl_ctx* c, const void* dst, const void* src, size_t bytes,
                            xpl_copy_dir dir) {
   if (!c || (unsigned)dir > 4) return XPL_ERR_INVALID_ARG;
@@ -692,6 +798,41 @@ xpl_status xpl_get_stats(xpl_ctx* c, xpl_stats* o) {
   o->dirty_max = ds[0];
   o->fold_full_scans = ds[1];
   o->folds = ds[2];
+  return XPL_OK;
+}
+
+xpl_status xpl_profile(xpl_ctx* c, int enable) {
+  if (!c) return XPL_ERR_INVALID_ARG;
+  if (enable && !c->prof) {
+    memset(c->prof_acc, 0, sizeof c->prof_acc);
+    CK(cudaStreamSynchronize(c->rs));
+    unsigned long long ds[8];
+    CK(cudaMemcpy(ds, c->d_stats, sizeof ds, cudaMemcpyDeviceToHost));
+    c->fold_entries_seen = ds[3];
+  }
+  c->prof = enable != 0;
+  return XPL_OK;
+}
+
+xpl_status xpl_profile_read(xpl_ctx* c, xpl_kernel_time* out, int reset) {
+  if (!c || !out) return XPL_ERR_INVALID_ARG;
+  CK(cudaStreamSynchronize(c->rs));
+  for (auto& r : c->prof_pending) {
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, r.a, r.b));
+    c->prof_acc[r.cls].launches += 1;
+    c->prof_acc[r.cls].ms += ms;
+    c->prof_acc[r.cls].bytes += r.bytes;
+    c->prof_free.push_back(r.a);
+    c->prof_free.push_back(r.b);
+  }
+  c->prof_pending.clear();
+  unsigned long long ds[8];
+  CK(cudaMemcpy(ds, c->d_stats, sizeof ds, cudaMemcpyDeviceToHost));
+  c->prof_acc[XPL_K_FOLD].bytes += 12ull * (ds[3] - c->fold_entries_seen);
+  c->fold_entries_seen = ds[3];
+  for (int k = 0; k < XPL_K_NCLASS; ++k) out[k] = c->prof_acc[k];
+  if (reset) memset(c->prof_acc, 0, sizeof c->prof_acc);
   return XPL_OK;
 }
 
@@ -787,10 +928,19 @@ xpl_status xpl_diagnose(xpl_ctx* c, const xpl_diag_params* params, const xpl_nam
   CK(cudaMemcpyAsync(c->d_drows, c->h_drows, sizeof(DiagRow) * nr, cudaMemcpyHostToDevice, c->rs));
   CK(cudaMemcpyAsync(c->d_tile_row, c->h_tile_row, sizeof(uint32_t) * ntiles,
                      cudaMemcpyHostToDevice, c->rs));
+  uint64_t total_words = 0;
+  for (size_t i = 0; i < nr; ++i) total_words += c->h_drows[i].words;
+  const uint64_t dbytes = total_words * (reset ? 2 : 1);
+  const int pall = prof_begin(c, XPL_K_DIAGNOSE, dbytes);
+  const int ptile = prof_begin(c, XPL_K_DIAG_TILE, dbytes, false);  // recorded by launch_diag
   launch_diag(c->rs, c->d_drows, (uint32_t)nr, c->d_tile_row, ntiles, nblocks, p,
-              (uint32_t*)c->d_pool, c->d_cnt, c->d_tiles, c->d_blk, c->d_rep);
+              (uint32_t*)c->d_pool, c->d_cnt, c->d_tiles, c->d_blk, c->d_rep,
+              ptile >= 0 ? c->prof_pending[ptile].a : nullptr,
+              ptile >= 0 ? c->prof_pending[ptile].b : nullptr);
   CK(cudaGetLastError());
+  c->st.kernel_launches += 3 + (p.block_words && nblocks ? 1 : 0);
   CK(cudaMemcpyAsync(c->h_rep, c->d_rep, sizeof(xpl_alloc_report) * nr, cudaMemcpyDeviceToHost, c->rs));
+  prof_end(c, pall);
   CK(cudaStreamSynchronize(c->rs));
 
   for (size_t i = 0; i < nr; ++i) {

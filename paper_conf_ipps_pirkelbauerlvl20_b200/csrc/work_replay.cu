@@ -23,8 +23,15 @@ __global__ void replay_kernel(const unsigned long long* __restrict__ addr,
 
 extern "C" {
 
-// Bind this translation unit's hooks to ctx (xpl_device_bind).
-int xplw_bind(xpl_ctx* ctx) { return (int)xpl_device_bind(ctx); }
+int xplw_bind_rodinia(xpl_ctx* ctx);
+
+// Bind the hooks of every instrumented translation unit of this library to ctx
+// (xpl_device_bind copies the device context into each TU's __constant__).
+int xplw_bind(xpl_ctx* ctx) {
+  int s = (int)xpl_device_bind(ctx);
+  if (!s) s = xplw_bind_rodinia(ctx);
+  return s;
+}
 
 // Launch the replay kernel on `stream` (between xpl_kernel_begin/_end).
 int xplw_replay(const unsigned long long* d_addr, const unsigned int* d_size,

@@ -83,7 +83,7 @@ void launch_range(cudaStream_t s, const RangeDesc* d_ranges, uint32_t nr, uint64
 void launch_diag(cudaStream_t s, const DiagRow* rows, uint32_t nrows, const uint32_t* tile_row,
                  uint64_t ntiles, uint64_t nblocks, const DiagParams& p, uint32_t* pool,
                  unsigned long long* cnt, TileSum* tiles, uint32_t* blk_cnt,
-                 xpl_alloc_report* out);
+                 xpl_alloc_report* out, cudaEvent_t tile_ev0, cudaEvent_t tile_ev1);
 void launch_fill_u32(cudaStream_t s, uint32_t* p, uint64_t n, uint32_t v);
 
 }  // namespace xpl

@@ -64,7 +64,7 @@ class XplAllocReport(C.Structure):
 class XplStats(C.Structure):
     _fields_ = [(n, u64) for n in ("epochs", "folds", "fold_full_scans", "host_records",
                                    "host_records_packed", "merge_segments", "range_segments",
-                                   "diagnoses", "dirty_max")]
+                                   "diagnoses", "dirty_max", "kernel_launches")]
 
 
 class XplDevCtx(C.Structure):
@@ -86,6 +86,7 @@ xpl_free = _sig("xpl_free", [vp, vp])
 xpl_kernel_begin = _sig("xpl_kernel_begin", [vp, vp])
 xpl_kernel_end = _sig("xpl_kernel_end", [vp, vp])
 xpl_record_host = _sig("xpl_record_host", [vp, vp, sz])
+xpl_record_host_ranges = _sig("xpl_record_host_ranges", [vp, vp, sz])
 xpl_record_copy = _sig("xpl_record_copy", [vp, vp, vp, sz, i32])
 xpl_diagnose = _sig("xpl_diagnose", [vp, C.POINTER(XplDiagParams), C.POINTER(XplName), sz,
                                      C.POINTER(XplAllocReport), sz, C.POINTER(sz), i32])
@@ -96,11 +97,21 @@ xpl_sync = _sig("xpl_sync", [vp])
 xpl_runtime_stream = _sig("xpl_runtime_stream", [vp, C.POINTER(vp)])
 xpl_get_stats = _sig("xpl_get_stats", [vp, C.POINTER(XplStats)])
 xpl_status_string = _sig("xpl_status_string", [i32], C.c_char_p)
+xpl_profile = _sig("xpl_profile", [vp, i32])
+
+
+class XplKernelTime(C.Structure):
+    _fields_ = [("launches", u64), ("ms", C.c_double), ("bytes", u64)]
+
+
+KERNEL_CLASSES = ["fold", "merge", "range", "diag_tile", "diagnose"]
+xpl_profile_read = _sig("xpl_profile_read", [vp, C.POINTER(XplKernelTime), i32])
 
 EXPORTED = ["xpl_init", "xpl_finalize", "xpl_register_alloc", "xpl_free", "xpl_kernel_begin",
-            "xpl_kernel_end", "xpl_record_host", "xpl_record_copy", "xpl_diagnose",
+            "xpl_kernel_end", "xpl_record_host", "xpl_record_host_ranges", "xpl_record_copy", "xpl_diagnose",
             "xpl_get_device_ctx", "xpl_shadow_dump", "xpl_flush", "xpl_sync",
-            "xpl_runtime_stream", "xpl_get_stats", "xpl_status_string"]
+            "xpl_runtime_stream", "xpl_get_stats", "xpl_status_string", "xpl_profile",
+            "xpl_profile_read"]
 
 if _work is not None:
     xplw_bind = _sig("xplw_bind", [vp], lib=_work)
@@ -156,6 +167,10 @@ class Context:
         recs = np.ascontiguousarray(recs, dtype=HOST_ACCESS_DTYPE)
         check("xpl_record_host", xpl_record_host(self.h, recs.ctypes.data, recs.size))
 
+    def record_host_ranges(self, recs: np.ndarray):
+        recs = np.ascontiguousarray(recs, dtype=HOST_ACCESS_DTYPE)
+        check("xpl_record_host_ranges", xpl_record_host_ranges(self.h, recs.ctypes.data, recs.size))
+
     def record_copy(self, dst, src, nbytes, direction):
         check("xpl_record_copy", xpl_record_copy(self.h, dst, src, nbytes, direction))
 
@@ -199,6 +214,15 @@ class Context:
         s = XplStats()
         check("xpl_get_stats", xpl_get_stats(self.h, C.byref(s)))
         return {f: getattr(s, f) for f, _ in XplStats._fields_}
+
+    def profile(self, enable=True):
+        check("xpl_profile", xpl_profile(self.h, int(bool(enable))))
+
+    def profile_read(self, reset=True):
+        arr = (XplKernelTime * len(KERNEL_CLASSES))()
+        check("xpl_profile_read", xpl_profile_read(self.h, arr, int(bool(reset))))
+        return {k: {"launches": arr[i].launches, "ms": arr[i].ms, "bytes": arr[i].bytes}
+                for i, k in enumerate(KERNEL_CLASSES)}
 
     def device_ctx(self):
         d = XplDevCtx()

@@ -182,3 +182,41 @@ def test_api_errors(gpu):
             ctx.free(0x20000)
             ctx.register(0x200000, 4 << 20, 0)
         assert e.value.status == 2
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_host_ranges(gpu, seed):
+    """xpl_record_host_ranges: byte ranges that may span several allocations and
+    the gaps between them == the same bytes as one-byte host accesses."""
+    replay, xpl = gpu
+    import torch
+    rng = np.random.default_rng(0x58504C10 + seed)
+    ops = []
+    bases = []
+    b = 0x3000_0000
+    for i in range(8):
+        n = int(rng.integers(1, 200))
+        ops.append(("REG", b, n, i % 3))
+        bases.append((b, n))
+        b += n + int(rng.integers(0, 3)) * 4  # adjacent allocations and small gaps
+    lo, hi = bases[0][0] - 16, b + 16
+    ranges = []
+    for _ in range(300):
+        a = int(rng.integers(lo, hi))
+        n = int(rng.integers(1, 64))
+        ranges.append((a, n, int(rng.integers(1, 3))))  # R or W (RW runs need word alignment)
+    # oracle: every byte as its own access, in order
+    for a, n, k in ranges:
+        ops.append(("HB", np.arange(a, a + n, dtype=np.uint64), np.ones(n, np.uint32), np.full(n, k, np.uint8)))
+    ops.append(("DIAG", 50, 0, 1, 1, ()))
+    exp = oracle_run(ops)
+    with xpl.Context(pool_words=1 << 20) as ctx:
+        for op in ops[:8]:
+            ctx.register(op[1], op[2], op[3])
+        rec = np.zeros(len(ranges), dtype=xpl.HOST_ACCESS_DTYPE)
+        rec["addr"] = [r[0] for r in ranges]
+        rec["size"] = [r[1] for r in ranges]
+        rec["kind"] = [r[2] for r in ranges]
+        ctx.record_host_ranges(rec)
+        got = [ctx.diagnose(50, 0, 1, True)]
+    compare(got, exp, "ranges")

@@ -1,0 +1,78 @@
+"""GPU parity of the instrumented Rodinia-shaped programs (configs[1]): the native
+app (csrc/work_rodinia.cu) runs through the C-ABI; its CPU twin (xplgen/rodinia.py)
+is replayed by the oracle at the SAME addresses; every report of every diagnose
+must match bit-exactly.  Sizes span several diagnose tiles with ragged tails."""
+import numpy as np
+import pytest
+
+from oracle import run_trace as oracle_run
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def env():
+    import torch
+    assert torch.cuda.is_available()
+    from paper_conf_ipps_pirkelbauerlvl20_b200 import apps, xpl
+    return torch, apps, xpl
+
+
+def compare(got, exp):
+    assert len(got) == len(exp), (len(got), len(exp))
+    for k, (g, e) in enumerate(zip(got, exp)):
+        assert len(g) == len(e), f"diag {k}: {len(g)} rows vs {len(e)}"
+        for gr, er in zip(g, e):
+            diff = {f: (gr[f], er[f]) for f in er if gr[f] != er[f]}
+            assert not diff, f"diag {k} row {er['id']}: (gpu, oracle) {diff}"
+
+
+@pytest.mark.parametrize("rows,cols,iters", [(8, 40, 3), (67, 130, 4), (256, 300, 3)])
+@pytest.mark.parametrize("params", [(50, 0, 256), (30, 1000, 8)])
+def test_hotspot(env, rows, cols, iters, params):
+    torch, apps, xpl = env
+    from xplgen import rodinia
+    spec = rodinia.hotspot_spec(rows, cols)
+    ar = apps.Arena(spec)
+    rodinia.fill_inputs("hotspot", ar.host_views(), 0x58504C01)
+    s = torch.cuda.Stream()
+    with xpl.Context(pool_words=1 << 24) as ctx:
+        run = apps.Run(ctx, s.cuda_stream, do_copies=True, diag_each=True, params=params)
+        apps.hotspot(run, ar, rows, cols, iters)
+        got = run.reports()
+        assert run.r.dev_accesses == iters * rodinia.hotspot_accesses(rows, cols)
+    exp = oracle_run(rodinia.hotspot_trace(ar.addrs, spec, rows, cols, iters, True, params))
+    compare(got, exp)
+
+
+@pytest.mark.parametrize("n_in", [64, 1024, 40960])
+def test_backprop(env, n_in):
+    torch, apps, xpl = env
+    from xplgen import rodinia
+    spec = rodinia.backprop_spec(n_in, 16)
+    ar = apps.Arena(spec)
+    rodinia.fill_inputs("backprop", ar.host_views(), 0x58504C01)
+    s = torch.cuda.Stream()
+    params = (50, 0, 256)
+    with xpl.Context(pool_words=1 << 25) as ctx:
+        run = apps.Run(ctx, s.cuda_stream, do_copies=bool(n_in % 2048), params=params)
+        apps.backprop(run, ar, n_in, 16)
+        got = run.reports()
+    exp = oracle_run(rodinia.backprop_trace(ar.addrs, spec, n_in, 16, params))
+    compare(got, exp)
+    # Table II: output_hidden_cuda unused; input_cuda copied back unmodified
+    rows = {r["id"]: r for r in got[-1]}
+    assert rows[6]["flags"] & 16
+    if n_in + 1 >= params[2]:
+        assert rows[5]["flags"] & 8
+
+
+def test_twin_runs_without_xpl(env):
+    torch, apps, xpl = env
+    from xplgen import rodinia
+    spec = rodinia.hotspot_spec(64, 64)
+    ar = apps.Arena(spec)
+    s = torch.cuda.Stream()
+    run = apps.Run(None, s.cuda_stream, do_copies=True)
+    apps.hotspot(run, ar, 64, 64, 2)
+    assert run.r.n_diag == 0 and run.r.status == 0
