@@ -128,6 +128,39 @@ def cpu_baseline(seconds_budget=20.0):
                       f"with a diagnose after each ({n_acc} accesses, {dt:.1f} s, 1 thread)"}
 
 
+def diag_at_scale(xpl, torch, words=1 << 31, reps=3):
+    """The diagnose pass over a cfg5-sized shadow (2^31 words = 2 GiB, SURVEY §8(d)
+    cfg5 ~2.2e9 words) with a mixed realistic content: CPU-written half (H2D),
+    GPU reads/writes in 4096-word blocks and random regions.  Timed live with
+    CUDA events on the runtime stream (xpl_profile)."""
+    ctx = xpl.Context(pool_words=words + (1 << 16), max_rows=16)
+    base = 1 << 44  # synthetic address range: hooks only use addresses
+    ctx.register(base, 4 * words, xpl.ALLOC_DEVICE)
+    ctx.record_copy(base, 0x1000, 2 * words, xpl.COPY_H2D)
+    s = torch.cuda.current_stream().cuda_stream
+    ctx.kernel_begin(s)
+    ctx.touch(base, words, 7, s)
+    ctx.kernel_end(s)
+    ctx.sync()
+    torch.cuda.synchronize()
+    ctx.profile(True)
+    for _ in range(reps):
+        ctx.diagnose(50, 0, 256, reset=False)
+    p0 = ctx.profile_read(reset=True)
+    ctx.diagnose(50, 0, 256, reset=True)
+    p1 = ctx.profile_read(reset=True)
+    ctx.profile(False)
+    ctx.close()
+    out = {}
+    for name, p in (("no_reset", p0), ("reset", p1)):
+        d = p["diag_tile"]
+        ms = d["ms"] / d["launches"]
+        out[name] = {"words": words, "ms": ms, "gbs": d["bytes"] / d["launches"] / (ms / 1e3) / 1e9,
+                     "bytes_per_launch": d["bytes"] / d["launches"],
+                     "whole_call_ms": p["diagnose"]["ms"] / p["diagnose"]["launches"]}
+    return out
+
+
 def reference_main(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
@@ -256,6 +289,9 @@ def main():
     bt = step(None, False, time_kernels=True)
     torch.cuda.synchronize()
 
+    # --- the diagnose pass at cfg5 scale ----------------------------------------
+    at_scale = diag_at_scale(xpl, torch)
+
     # --- roofline of the dominant runtime kernel -------------------------------
     peak, peak_src = peaks()
     dom = max(("diag_tile", "merge", "range", "fold"), key=lambda k: prof[k]["ms"])
@@ -277,7 +313,10 @@ def main():
                    "diag_params": {"threshold_pct": PARAMS[0], "block_words": PARAMS[1], "min_run": PARAMS[2]},
                    "l2": "flushed between steps (256 MB write, untimed)", "parallelism": f"replicas x{world}"},
         "roofline": roof,
-        "diagnose_gbs": (dg["bytes"] / (dg["ms"] / 1e3) / 1e9) if dg["ms"] else None,
+        "diagnose_gbs": at_scale["reset"]["gbs"],
+        "diagnose_at_scale": dict(at_scale, peak_gbs=peak, frac_reset=at_scale["reset"]["gbs"] / peak,
+                                  frac_no_reset=at_scale["no_reset"]["gbs"] / peak),
+        "diagnose_gbs_in_step": (dg["bytes"] / (dg["ms"] / 1e3) / 1e9) if dg["ms"] else None,
         "runtime_kernels": {k: {"launches": v["launches"], "ms_per_step": v["ms"] / args.steps,
                                 "gbs": (v["bytes"] / (v["ms"] / 1e3) / 1e9) if v["ms"] else None}
                             for k, v in prof.items()},

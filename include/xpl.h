@@ -82,7 +82,6 @@ typedef struct {
   int rank, world;       /* world > 1 => address-range sharding over the ranks    */
   void* nccl_comm;       /* ncclComm_t when world > 1, else NULL                  */
   uint64_t pool_words;   /* shadow pool capacity in words (1 byte each)   */
-  uint64_t dirty_cap;    /* dirty-list capacity, in shadow u32s                    */
   uint64_t staging_recs; /* host-record staging capacity (records)                */
   uint32_t max_rows;     /* capacity of the allocation table                      */
 } xpl_config;
@@ -121,14 +120,16 @@ struct xpl_dev_ctx; /* defined in xpl_device.cuh */
 
 /* Counters the runtime keeps about itself (not part of the paper's output). */
 typedef struct {
-  uint64_t epochs, folds, fold_full_scans, host_records, host_records_packed,
-      merge_segments, range_segments, diagnoses, dirty_max,
+  uint64_t epochs, folds, fold_chunks /* 128-word chunks folded */, host_records,
+      host_records_packed, merge_segments, range_segments, diagnoses,
+      fold_chunks_max /* largest single fold */,
       kernel_launches; /* runtime kernels launched (not counting user kernels) */
 } xpl_stats;
 
 /* Create a context on cfg->device.  *out is owned by the caller until
- * xpl_finalize.  Zero fields of cfg take defaults (pool_words 2^28, dirty_cap
- * 2^24, staging_recs 2^22, max_rows 4096).  Allocates the shadow pool in HBM. */
+ * xpl_finalize.  Zero fields of cfg take defaults (pool_words 2^28,
+ * staging_recs 2^22, max_rows 4096).  Allocates the shadow pool in HBM (plus
+ * 1/128 of it for the chunk maps of the epoch close). */
 xpl_status xpl_init(const xpl_config* cfg, xpl_ctx** out);
 xpl_status xpl_finalize(xpl_ctx* ctx);
 
@@ -200,7 +201,7 @@ xpl_status xpl_get_stats(xpl_ctx* ctx, xpl_stats* out);
  * every runtime kernel is bracketed by CUDA events on the runtime stream.
  * xpl_profile_read waits for the runtime stream and returns, per kernel class,
  * the launches, the summed event time and the ALGORITHMIC bytes moved
- * (fold 12 B per dirty u32; merge 8 B per record + 2 B per word;
+ * (fold 256 B per written 128-word chunk; merge 8 B per record + 2 B per word;
  * range 2 B per word; diagnose 1 B per word + 1 B per word when resetting). */
 typedef enum {
   XPL_K_FOLD = 0,

@@ -21,10 +21,12 @@
  *  3. warp aggregation: lanes that hit the same shadow u32 (4 records) are grouped
  *     with __match_any_sync, their bits OR-reduced, and one leader issues a single
  *     atomicOr -- and only if some bit is still missing (test before set);
- *  4. the first pending write in a shadow u32 appends its index to the dirty list,
- *     so closing the epoch costs O(words written), not O(shadow).
- * Device hooks never fail: a dirty-list overflow makes the epoch close scan the
- * whole pool instead (results are unchanged).
+ *  4. a write also marks its 128-word chunk (and 16K-word super-chunk) in two
+ *     byte maps with plain idempotent stores (test before store, no atomics),
+ *     so closing the epoch costs O(chunks written), not O(shadow).
+ * A single-word access (the common case: an aligned scalar) takes a short path
+ * with one ballot; multi-word accesses loop over the shadow u32s they cover.
+ * Device hooks never fail and never block.
  */
 #ifndef XPL_DEVICE_CUH
 #define XPL_DEVICE_CUH
@@ -43,13 +45,11 @@ struct xpl_dev_row {
 };
 
 struct xpl_dev_ctx {
-  const struct xpl_dev_row* rows; /* live rows, sorted by base      */
-  const unsigned int* n_rows;     /* number of live rows            */
-  unsigned int* pool;             /* shadow pool, 4 records per u32 */
-  unsigned int* dirty;            /* dirty list (u32 indices)       */
-  unsigned int* dirty_count;
-  unsigned int dirty_cap;
-  unsigned int pad_;
+  const struct xpl_dev_row* rows; /* live rows, sorted by base                   */
+  const unsigned int* n_rows;     /* number of live rows                         */
+  unsigned int* pool;             /* shadow pool, 4 records per u32              */
+  unsigned char* cmap;            /* 1 byte per 128-word chunk: GPU write pending */
+  unsigned char* smap;            /* 1 byte per 128 chunks (16K words)            */
 };
 
 #ifdef __CUDACC__
@@ -80,48 +80,81 @@ static __device__ __forceinline__ unsigned xpld_lane() {
   return l;
 }
 
+/* Mark the chunk (and super-chunk) of shadow u32 q as holding a pending GPU
+ * write: plain idempotent byte stores, tested first (a stale cached 0 only
+ * costs a redundant store).  Only first writes of a shadow u32 get here. */
+static __device__ __forceinline__ void xpld_mark(unsigned q) {
+  unsigned char* c = xpl_dctx.cmap + (q >> 5);
+  if (!*c) *c = 1;
+  unsigned char* s = xpl_dctx.smap + (q >> 12);
+  if (!*s) *s = 1;
+}
+
+/* OR the record bits m into shadow u32 q for the lanes in `needers` (lanes with
+ * bits still missing): lanes hitting the same u32 are grouped and one leader
+ * issues the atomic.  Only the lanes of `needers` may call it. */
+static __device__ __forceinline__ void xpld_commit(unsigned needers, unsigned q, unsigned m) {
+  const unsigned grp = __match_any_sync(needers, q);
+  const unsigned M = __reduce_or_sync(grp, m);
+  if (xpld_lane() == (unsigned)(__ffs(grp) - 1)) {
+    atomicOr(xpl_dctx.pool + q, M);  /* no return value needed: RED */
+    if (M & XPLD_P4) xpld_mark(q);
+  }
+}
+
+/* The record bits an access of kind acc sets on the 4 records of shadow u32 cur,
+ * restricted to the byte lanes of `bytes` (0xFF per record touched). */
+static __device__ __forceinline__ unsigned xpld_bits(unsigned cur, unsigned bytes, unsigned acc) {
+  unsigned m = 0;
+  if (acc & XPL_ACC_R) {
+    const unsigned l = cur & 0x01010101u;                  /* L per record        */
+    m = ((l << 7) | ((~l & 0x01010101u) << 6)) & bytes;    /* rGG if L else rCG   */
+  }
+  if (acc & XPL_ACC_W) m |= 0x0A0A0A0Au & bytes;           /* wG | P              */
+  return m;
+}
+
 /* Apply a GPU access to the shadow words [g0, g1] (global pool word indices;
- * empty when g0 > g1).  All lanes of the calling warp that are active must call it. */
+ * empty when g0 > g1).  All active lanes of the calling warp must call it. */
 static __device__ __forceinline__ void xpl_dev_apply(unsigned long long g0,
                                                      unsigned long long g1,
                                                      unsigned acc) {
   const unsigned active = __activemask();
-  const unsigned lane = xpld_lane();
+  const bool single = g0 >= g1; /* one word (g0 == g1) or none (g0 > g1) */
+  const unsigned singles = __ballot_sync(active, single);
+  if (single) { /* the short path */
+    const bool hit = g0 == g1;
+    const unsigned q = (unsigned)(g0 >> 2);
+    unsigned cur = 0, m = 0;
+    if (hit) {
+      cur = xpl_dctx.pool[q];
+      m = xpld_bits(cur, 0xFFu << (8 * (unsigned)(g0 & 3)), acc);
+    }
+    const bool need = hit && (cur & m) != m;
+    const unsigned needers = __ballot_sync(singles, need);
+    if (need) xpld_commit(needers, q, m);
+  }
+  if (singles == active) return;
+  /* multi-word accesses: one shadow u32 per iteration */
+  const bool multi = g0 < g1;
   unsigned long long q = g0 >> 2;
   const unsigned long long ql = g1 >> 2;
-  bool more = g0 <= g1;
+  bool more = multi;
   while (__any_sync(active, more)) {
-    unsigned m = 0, cur = 0;
+    unsigned cur = 0, m = 0;
     if (more) {
       cur = xpl_dctx.pool[q];
+      unsigned bytes = 0;
 #pragma unroll
       for (unsigned k = 0; k < 4; ++k) {
         const unsigned long long gw = q * 4 + k;
-        if (gw >= g0 && gw <= g1) {
-          unsigned b = 0;
-          if (acc & XPL_ACC_R) b = ((cur >> (8 * k)) & XPLD_L) ? XPLD_RGG : XPLD_RCG;
-          if (acc & XPL_ACC_W) b |= XPLD_WG | XPLD_P;
-          m |= b << (8 * k);
-        }
+        if (gw >= g0 && gw <= g1) bytes |= 0xFFu << (8 * k);
       }
+      m = xpld_bits(cur, bytes, acc);
     }
-    const bool need = more && ((cur & m) != m);
-    if (__any_sync(active, need)) {
-      const unsigned long long key = need ? q : ~0ull;
-      const unsigned grp = __match_any_sync(active, key);
-      const unsigned M = __reduce_or_sync(grp, m);
-      if (need && lane == (unsigned)(__ffs(grp) - 1)) {
-        if (M & XPLD_P4) {
-          const unsigned old = atomicOr(xpl_dctx.pool + q, M);
-          if ((old & XPLD_P4) == 0) {
-            const unsigned i = atomicAdd(xpl_dctx.dirty_count, 1u);
-            if (i < xpl_dctx.dirty_cap) xpl_dctx.dirty[i] = (unsigned)q;
-          }
-        } else {
-          atomicOr(xpl_dctx.pool + q, M);
-        }
-      }
-    }
+    const bool need = more && (cur & m) != m;
+    const unsigned needers = __ballot_sync(active, need);
+    if (need) xpld_commit(needers, (unsigned)q, m);
     more = more && q < ql;
     ++q;
   }

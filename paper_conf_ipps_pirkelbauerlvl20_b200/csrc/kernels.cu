@@ -2,7 +2,7 @@
 // inlined device hooks, which live in include/xpl_device.cuh).
 //
 //   fold          epoch close: pending GPU writes become "last writer = GPU"
-//                 (snapshot semantics D5), O(dirty u32s)
+//                 (snapshot semantics D5), O(chunks written)
 //   merge_*       ordered host-record batches (host tracer), 3 passes
 //   range_apply   transfers and other long ranges, 16 records / vector
 //   diag_*        tracePrint: counts, density blocks, transfer runs,
@@ -23,52 +23,52 @@ constexpr uint32_t kL4 = 0x01010101u;
 constexpr uint32_t kP4 = 0x02020202u;
 
 // ---------------------------------------------------------------------------
-// fold: for every shadow u32 in the dirty list, P -> L=1 and clear P.  If the
-// list overflowed during the epoch, scan the whole pool instead.  The last CTA
-// to finish resets the list for the next epoch (no host round trip).
+// fold (epoch close): every 128-word chunk a GPU write marked (cmap) gets
+// P -> L=1 and P cleared (snapshot semantics D5).  One CTA per 16K-word
+// super-chunk below the pool's high-water mark: a CTA-uniform check of the
+// super byte, then warp w checks chunks [16w, 16w+16) and folds the marked
+// ones four at a time (128 B coalesced each).  No list, no atomics; cost
+// O(super map + chunks written).
 __global__ void __launch_bounds__(256) fold_kernel(uint32_t* __restrict__ pool,
-                                                   uint64_t pool_u32,
-                                                   const uint32_t* __restrict__ dirty,
-                                                   uint32_t* dirty_count, uint32_t cap,
-                                                   uint32_t* done_ctr,
+                                                   uint8_t* __restrict__ cmap,
+                                                   uint8_t* __restrict__ smap, uint64_t n_super,
                                                    unsigned long long* stats) {
-  const uint32_t n = *((volatile uint32_t*)dirty_count);
-  const uint64_t tid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  if (n <= cap) {
-    for (uint64_t i = tid; i < n; i += stride) {
-      const uint32_t q = dirty[i];
-      const uint32_t v = pool[q];
-      const uint32_t p = v & kP4;
-      pool[q] = (v & ~kP4) | (p >> 1);
-    }
-  } else {
-    uint4* p4 = reinterpret_cast<uint4*>(pool);
-    for (uint64_t i = tid; i < pool_u32 / 4; i += stride) {
-      uint4 v = p4[i];
-      if ((v.x | v.y | v.z | v.w) & kP4) {
-        v.x = (v.x & ~kP4) | ((v.x & kP4) >> 1);
-        v.y = (v.y & ~kP4) | ((v.y & kP4) >> 1);
-        v.z = (v.z & ~kP4) | ((v.z & kP4) >> 1);
-        v.w = (v.w & ~kP4) | ((v.w & kP4) >> 1);
-        p4[i] = v;
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  __shared__ uint32_t s_go;
+  uint32_t folded = 0;
+  for (uint64_t sc = blockIdx.x; sc < n_super; sc += gridDim.x) {
+    if (threadIdx.x == 0) s_go = smap[sc];  // one read per CTA: a uniform decision
+    __syncthreads();
+    const bool go = s_go != 0;
+    __syncthreads();
+    if (!go) continue;
+    const uint64_t c0 = sc * 128 + warp * 16;
+    const bool m = lane < 16 && cmap[c0 + lane] != 0;
+    uint32_t marked = __ballot_sync(0xFFFFFFFFu, m);
+    folded += __popc(marked);
+    while (marked) {
+      uint64_t at[4];
+      uint32_t v[4];
+#pragma unroll
+      for (uint32_t k = 0; k < 4; ++k) {
+        if (marked) {
+          const uint32_t j = __ffs(marked) - 1;
+          marked &= marked - 1;
+          at[k] = (c0 + j) * 32 + lane;
+          v[k] = pool[at[k]];
+        } else {
+          at[k] = ~0ull;
+          v[k] = 0;
+        }
       }
+#pragma unroll
+      for (uint32_t k = 0; k < 4; ++k)
+        if (v[k] & kP4) pool[at[k]] = (v[k] & ~kP4) | ((v[k] & kP4) >> 1);
     }
+    if (m) cmap[c0 + lane] = 0;
+    if (threadIdx.x == 0) smap[sc] = 0;
   }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    __threadfence();
-    const uint32_t t = atomicAdd(done_ctr, 1u);
-    if (t == gridDim.x - 1) {
-      if (n > stats[0]) stats[0] = n;
-      if (n > cap) stats[1] += 1;
-      stats[2] += 1;
-      stats[3] += n <= cap ? n : pool_u32;
-      *dirty_count = 0;
-      *done_ctr = 0;
-      __threadfence();
-    }
-  }
+  if (lane == 0 && folded) atomicAdd(stats + 3, (unsigned long long)folded);
 }
 
 // ---------------------------------------------------------------------------
@@ -153,8 +153,7 @@ __device__ __forceinline__ uint32_t cpu_range_op(uint32_t v, uint32_t bm, uint32
 
 __global__ void __launch_bounds__(256) range_kernel(const RangeDesc* __restrict__ rd, uint32_t nr,
                                                     uint64_t nvec, uint32_t* pool,
-                                                    uint32_t* dirty, uint32_t* dirty_count,
-                                                    uint32_t dirty_cap) {
+                                                    uint8_t* cmap, uint8_t* smap) {
   for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < nvec;
        v += (uint64_t)gridDim.x * blockDim.x) {
     uint32_t lo = 0, hi = nr;  // last range with vbase <= v
@@ -216,10 +215,10 @@ __global__ void __launch_bounds__(256) range_kernel(const RangeDesc* __restrict_
         if (r.acc & XPL_ACC_W) m |= 0x0A0A0A0Au & bms[c];
         if ((in[c] & m) == m) continue;
         const uint32_t q = (uint32_t)(vi * 4 + c);
-        const uint32_t old = atomicOr(pool + q, m);
-        if ((m & kP4) && !(old & kP4)) {
-          const uint32_t i = atomicAdd(dirty_count, 1u);
-          if (i < dirty_cap) dirty[i] = q;
+        atomicOr(pool + q, m);
+        if (m & kP4) {
+          if (!cmap[q >> 5]) cmap[q >> 5] = 1;
+          if (!smap[q >> 12]) smap[q >> 12] = 1;
         }
       }
     }
@@ -261,7 +260,7 @@ __device__ __forceinline__ uint32_t pack4(uint32_t t) {  // bit0 of each byte ->
 
 // Warp summary of one predicate over the warp's 512 consecutive words; lane l
 // owns words [16l, 16l+16) as the 16-bit mask m.  Returns a warp-uniform RunSum.
-__device__ __forceinline__ RunSum warp_runs(uint32_t m, uint32_t lane, uint32_t min_run) {
+__device__ __noinline__ RunSum warp_runs(uint32_t m, uint32_t lane, uint32_t min_run) {
   const bool full = m == 0xFFFFu;
   const uint32_t pre = __ffs(~m) - 1;  // 16 when full
   const uint32_t x = ~m & 0xFFFFu;
@@ -310,7 +309,7 @@ __device__ __forceinline__ RunSum warp_runs(uint32_t m, uint32_t lane, uint32_t 
 }
 
 // Harley-Seal style vertical counter: bit j of plane k is bit k of the number of
-// ones seen at bit position j.  32 words per lane per tile -> 6 planes.
+// ones seen at bit position j.  32 words (u32) per lane per tile -> 6 planes.
 struct VCount {
   uint32_t p0 = 0, p1 = 0, p2 = 0, p3 = 0, p4 = 0, p5 = 0;
   __device__ __forceinline__ void add4(uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
@@ -345,154 +344,214 @@ __device__ __forceinline__ uint32_t derived_flags(uint32_t x) {
   return any | (gpu >> 1) | (alt >> 2);  // bit7 any, bit6 gpu, bit5 alternating
 }
 
-__global__ void __launch_bounds__(kDiagThreads) diag_tile_kernel(
+// Run summary updates of a warp's running summary A by one 512-word step that
+// is all zeros / all ones (the common cases; u32 arithmetic inside a tile).
+__device__ __forceinline__ void rs_append_zero(RunSum& a, uint32_t min_run) {
+  if (a.pre == a.len) {
+    a.pre = a.len;  // the leading run ends here
+  } else if (a.suf >= min_run && a.suf > 0) {
+    a.cnt += 1;
+    a.sum += a.suf;
+  }
+  a.suf = 0;
+  a.len += 512;
+}
+__device__ __forceinline__ void rs_append_full(RunSum& a) {
+  if (a.pre == a.len) a.pre += 512;
+  a.suf += 512;
+  a.len += 512;
+}
+__device__ __forceinline__ RunSum rs_combine32(const RunSum& a, const RunSum& b, uint32_t min_run) {
+  RunSum r;
+  const bool af = a.pre == a.len, bf = b.pre == b.len;
+  r.len = a.len + b.len;
+  r.pre = af ? a.len + b.pre : a.pre;
+  r.suf = bf ? b.len + a.suf : b.suf;
+  r.cnt = a.cnt + b.cnt;
+  r.sum = a.sum + b.sum;
+  if (!af && !bf) {
+    const uint32_t mid = a.suf + b.pre;
+    if (mid > 0 && mid >= min_run) {
+      r.cnt += 1;
+      r.sum += mid;
+    }
+  }
+  return r;
+}
+
+// The mixed (slow) case of one 512-word run step, out of line to keep the hot
+// loop small (instruction cache).
+__device__ __noinline__ RunSum run_step_mixed(RunSum a, const uint32_t* bits, uint32_t shift,
+                                              uint32_t lane, uint32_t min_run) {
+  const uint32_t m = pack4(bits[0] >> shift) | (pack4(bits[1] >> shift) << 4) |
+                     (pack4(bits[2] >> shift) << 8) | (pack4(bits[3] >> shift) << 12);
+  return rs_combine32(a, warp_runs(m, lane, min_run), min_run);
+}
+
+__device__ __noinline__ void block_counts(uint32_t f0, uint32_t f1, uint32_t f2, uint32_t f3,
+                                          uint64_t rw, uint64_t B, uint32_t* blk) {
+  const uint32_t g = ((f0 >> 6) & kL4) | (((f1 >> 6) & kL4) << 1) | (((f2 >> 6) & kL4) << 2) |
+                     (((f3 >> 6) & kL4) << 3);
+  uint32_t gm = 0;  // bit i = GPU-accessed flag of word rw + i
+#pragma unroll
+  for (uint32_t c = 0; c < 4; ++c)
+#pragma unroll
+    for (uint32_t k = 0; k < 4; ++k) gm |= ((g >> (8 * k + c)) & 1u) << (4 * c + k);
+  if (!gm) return;
+  uint64_t a = rw;
+  const uint64_t e = rw + 16;
+  while (a < e) {
+    const uint64_t k = a / B;
+    const uint64_t be = (k + 1) * B < e ? (k + 1) * B : e;
+    const uint32_t lo = (uint32_t)(a - rw), hi = (uint32_t)(be - rw);
+    const uint32_t seg = ((hi >= 32 ? 0xFFFFFFFFu : ((1u << hi) - 1u)) & ~((1u << lo) - 1u));
+    const uint32_t c = __popc(gm & seg);
+    if (c) atomicAdd(blk + k, c);
+    a = be;
+  }
+}
+
+struct TileAcc {
+  VCount raw, der;
+  RunSum wu = {0, 0, 0, 0, 0}, wd = {0, 0, 0, 0, 0};
+};
+
+// One 16-word lane step: TAIL = the warp's range may end inside the row.
+template <bool TAIL, bool RESET, bool BLOCKS>
+__device__ __forceinline__ void tile_step(TileAcc& A, uint4 y, uint4* dst, uint32_t w, uint32_t live,
+                                          uint32_t lane, uint32_t min_run, uint64_t rw0,
+                                          uint64_t B, uint32_t* blk) {
+  uint32_t x[4] = {y.x, y.y, y.z, y.w};
+  uint32_t keep[4] = {kL4, kL4, kL4, kL4};
+  if (TAIL && w + 16 > live) {  // mask the words past the row's end
+#pragma unroll
+    for (uint32_t c = 0; c < 4; ++c) {
+      uint32_t m = 0;
+#pragma unroll
+      for (uint32_t k = 0; k < 4; ++k)
+        if (w + c * 4 + k < live) m |= 0xFFu << (8 * k);
+      x[c] &= m;
+      keep[c] |= ~m;
+    }
+  }
+  A.raw.add4(x[0], x[1], x[2], x[3]);
+  const uint32_t f0 = derived_flags(x[0]), f1 = derived_flags(x[1]), f2 = derived_flags(x[2]),
+                 f3 = derived_flags(x[3]);
+  A.der.add4(f0, f1, f2, f3);
+  // transfer runs: u = wC & !rCG (bit 2), d = rCC (bit 4)
+  uint32_t uu[4], dd[4];
+#pragma unroll
+  for (uint32_t c = 0; c < 4; ++c) {
+    uu[c] = x[c] & ~(x[c] >> 4) & 0x04040404u;
+    dd[c] = x[c] & 0x10101010u;
+  }
+  if (__ballot_sync(0xFFFFFFFFu, (uu[0] | uu[1] | uu[2] | uu[3]) != 0) == 0)
+    rs_append_zero(A.wu, min_run);
+  else if (__all_sync(0xFFFFFFFFu, (uu[0] & uu[1] & uu[2] & uu[3]) == 0x04040404u))
+    rs_append_full(A.wu);
+  else
+    A.wu = run_step_mixed(A.wu, uu, 2, lane, min_run);
+  if (__ballot_sync(0xFFFFFFFFu, (dd[0] | dd[1] | dd[2] | dd[3]) != 0) == 0)
+    rs_append_zero(A.wd, min_run);
+  else if (__all_sync(0xFFFFFFFFu, (dd[0] & dd[1] & dd[2] & dd[3]) == 0x10101010u))
+    rs_append_full(A.wd);
+  else
+    A.wd = run_step_mixed(A.wd, dd, 4, lane, min_run);
+  if (BLOCKS && (!TAIL || w < live)) block_counts(f0, f1, f2, f3, rw0 + w, B, blk);
+  // fused reset (D4): keep L only, words of this row only
+  if (RESET && (!TAIL || w < live)) {
+    if (((y.x & ~keep[0]) | (y.y & ~keep[1]) | (y.z & ~keep[2]) | (y.w & ~keep[3])) != 0)
+      *dst = make_uint4(y.x & keep[0], y.y & keep[1], y.z & keep[2], y.w & keep[3]);
+  }
+}
+
+template <bool TAIL, bool RESET, bool BLOCKS>
+__device__ __forceinline__ void tile_loop(TileAcc& A, uint4* p4, uint32_t live, uint32_t lane,
+                                          uint32_t min_run, uint64_t rw0, uint64_t B, uint32_t* blk) {
+  // 2-step software pipeline: the next two 512-word steps are in flight while
+  // the current two are processed (a small loop body for the instruction cache)
+  auto ld = [&](uint32_t it) {
+    const uint32_t w = it * 512 + lane * 16;
+    return (it < kDiagIters && (!TAIL || w < live)) ? p4[it * 32 + lane] : make_uint4(0, 0, 0, 0);
+  };
+  uint4 a = ld(0), b = ld(1);
+#pragma unroll 1
+  for (uint32_t it = 0; it < kDiagIters; it += 2) {
+    const uint4 na = ld(it + 2), nb = ld(it + 3);
+    tile_step<TAIL, RESET, BLOCKS>(A, a, p4 + it * 32 + lane, it * 512 + lane * 16, live, lane,
+                                   min_run, rw0, B, blk);
+    tile_step<TAIL, RESET, BLOCKS>(A, b, p4 + (it + 1) * 32 + lane, (it + 1) * 512 + lane * 16,
+                                   live, lane, min_run, rw0, B, blk);
+    a = na;
+    b = nb;
+  }
+}
+
+// One CTA = one tile of kTileWords words of one row; warp w owns a contiguous
+// quarter (4096 words); per step lane l owns 16 words (one uint4 of records).
+// Counts: two Harley-Seal vertical counters (raw record bits; derived per-word
+// any/gpu/alternating flags) popcounted once per tile.  Runs: ballot fast paths
+// for all-zero/all-one 512-word steps, warp_runs() for mixed ones.  Reset fused.
+__global__ void __launch_bounds__(kDiagThreads, 6) diag_tile_kernel(
     const DiagRow* __restrict__ rows, const uint32_t* __restrict__ tile_row, DiagParams p,
     uint32_t* __restrict__ pool, unsigned long long* __restrict__ cnt, TileSum* __restrict__ tiles,
     uint32_t* __restrict__ blk_cnt) {
-  __shared__ uint32_t s_cnt[kDiagThreads / 32][9];
-  __shared__ RunSum s_u[kDiagThreads / 32], s_d[kDiagThreads / 32];
+  constexpr uint32_t kWarps = kDiagThreads / 32;
+  constexpr uint32_t kWarpWords = kTileWords / kWarps;
+  __shared__ uint32_t s_cnt[kWarps][9];
+  __shared__ RunSum s_u[kWarps], s_d[kWarps];
   const uint64_t t = blockIdx.x;
   const uint32_t ri = tile_row[t];
   const DiagRow row = rows[ri];
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const uint64_t tw0 = (t - row.tile0) * kTileWords;
-  const uint64_t ww0 = tw0 + (uint64_t)warp * (kTileWords / (kDiagThreads / 32));
+  const uint64_t ww0 = (t - row.tile0) * kTileWords + (uint64_t)warp * kWarpWords;  // row word
   const uint32_t min_run = (uint32_t)(p.min_run < 0xFFFFFFFFull ? p.min_run : 0xFFFFFFFFull);
-  uint4* p4 = reinterpret_cast<uint4*>(pool);
-
-  uint4 v[kDiagIters];
-#pragma unroll
-  for (uint32_t it = 0; it < kDiagIters; ++it) {
-    const uint64_t w = ww0 + it * 512 + lane * 16;
-    v[it] = w < row.words ? p4[(row.off + w) >> 4] : make_uint4(0, 0, 0, 0);
-  }
-
-  VCount raw, der;
-  RunSum wu = {0, 0, 0, 0, 0}, wd = {0, 0, 0, 0, 0};
-#pragma unroll
-  for (uint32_t it = 0; it < kDiagIters; ++it) {
-    const uint64_t w = ww0 + it * 512 + lane * 16;
-    uint32_t x[4] = {v[it].x, v[it].y, v[it].z, v[it].w};
-    uint32_t bm[4] = {0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu};
-    if (w + 16 > row.words) {  // tail of the row (or beyond it): mask the words
-#pragma unroll
-      for (uint32_t c = 0; c < 4; ++c) {
-        uint32_t m = 0;
-#pragma unroll
-        for (uint32_t k = 0; k < 4; ++k)
-          if (w + c * 4 + k < row.words) m |= 0xFFu << (8 * k);
-        bm[c] = m;
-        x[c] &= m;
-      }
-    }
-    raw.add4(x[0], x[1], x[2], x[3]);
-    const uint32_t f0 = derived_flags(x[0]), f1 = derived_flags(x[1]), f2 = derived_flags(x[2]),
-                   f3 = derived_flags(x[3]);
-    der.add4(f0, f1, f2, f3);
-
-    // transfer runs: u = wC & !rCG at bit 2, d = rCC at bit 4
-    uint32_t uu[4], dd[4];
-#pragma unroll
-    for (uint32_t c = 0; c < 4; ++c) {
-      uu[c] = x[c] & ~(x[c] >> 4) & 0x04040404u;
-      dd[c] = x[c] & 0x10101010u;
-    }
-    const uint32_t uor = uu[0] | uu[1] | uu[2] | uu[3];
-    const uint32_t uand = uu[0] & uu[1] & uu[2] & uu[3];
-    const uint32_t dor = dd[0] | dd[1] | dd[2] | dd[3];
-    const uint32_t dand = dd[0] & dd[1] & dd[2] & dd[3];
-    RunSum su, sd;
-    const unsigned any_u = __ballot_sync(0xFFFFFFFFu, uor != 0);
-    const unsigned full_u = __ballot_sync(0xFFFFFFFFu, uand == 0x04040404u);
-    if (any_u == 0) su = {512, 0, 0, 0, 0};
-    else if (full_u == 0xFFFFFFFFu) su = {512, 512, 512, 0, 0};
-    else {
-      const uint32_t m = pack4(uu[0] >> 2) | (pack4(uu[1] >> 2) << 4) | (pack4(uu[2] >> 2) << 8) |
-                         (pack4(uu[3] >> 2) << 12);
-      su = warp_runs(m, lane, min_run);
-    }
-    const unsigned any_d = __ballot_sync(0xFFFFFFFFu, dor != 0);
-    const unsigned full_d = __ballot_sync(0xFFFFFFFFu, dand == 0x10101010u);
-    if (any_d == 0) sd = {512, 0, 0, 0, 0};
-    else if (full_d == 0xFFFFFFFFu) sd = {512, 512, 512, 0, 0};
-    else {
-      const uint32_t m = pack4(dd[0] >> 4) | (pack4(dd[1] >> 4) << 4) | (pack4(dd[2] >> 4) << 8) |
-                         (pack4(dd[3] >> 4) << 12);
-      sd = warp_runs(m, lane, min_run);
-    }
-    wu = rs_combine(wu, su, min_run);
-    wd = rs_combine(wd, sd, min_run);
-
-    // density blocks when block_words > 0
-    if (p.block_words && w < row.words) {
-      const uint64_t B = p.block_words;
-      const uint32_t g = ((f0 >> 6) & kL4) | (((f1 >> 6) & kL4) << 1) |
-                         (((f2 >> 6) & kL4) << 2) | (((f3 >> 6) & kL4) << 3);
-      // bit (c + 8k) of g = gpu flag of word 4c + k; build the word-ordered 16-bit mask
-      uint32_t gm = 0;
-#pragma unroll
-      for (uint32_t c = 0; c < 4; ++c)
-#pragma unroll
-        for (uint32_t k = 0; k < 4; ++k) gm |= ((g >> (8 * k + c)) & 1u) << (4 * c + k);
-      if (gm) {
-        uint64_t a = w;
-        const uint64_t e = w + 16;
-        while (a < e) {
-          const uint64_t k = a / B;
-          const uint64_t be = (k + 1) * B < e ? (k + 1) * B : e;
-          const uint32_t lo = (uint32_t)(a - w), hi = (uint32_t)(be - w);
-          const uint32_t seg = ((hi >= 32 ? 0xFFFFFFFFu : ((1u << hi) - 1u)) & ~((1u << lo) - 1u));
-          const uint32_t c = __popc(gm & seg);
-          if (c) atomicAdd(blk_cnt + row.blk0 + k, c);
-          a = be;
-        }
-      }
-    }
-
-    // fused reset (D4): keep L only
-    if (p.reset && w < row.words) {
-      const uint32_t y[4] = {v[it].x, v[it].y, v[it].z, v[it].w};
-      uint32_t n[4];
-      bool ch = false;
-#pragma unroll
-      for (uint32_t c = 0; c < 4; ++c) {
-        n[c] = y[c] & (~bm[c] | kL4);
-        ch = ch || n[c] != y[c];
-      }
-      if (ch) p4[(row.off + w) >> 4] = make_uint4(n[0], n[1], n[2], n[3]);
-    }
+  const uint32_t live = row.words > ww0 ? (uint32_t)min(row.words - ww0, (uint64_t)kWarpWords) : 0u;
+  uint4* p4 = reinterpret_cast<uint4*>(pool) + ((row.off + ww0) >> 4);
+  uint32_t* blk = blk_cnt + row.blk0;
+  TileAcc A;
+  const bool tail = live < kWarpWords;
+  if (p.block_words) {  // rare: blocks need per-lane counter atomics
+    if (p.reset) tile_loop<true, true, true>(A, p4, live, lane, min_run, ww0, p.block_words, blk);
+    else tile_loop<true, false, true>(A, p4, live, lane, min_run, ww0, p.block_words, blk);
+  } else if (p.reset) {
+    if (tail) tile_loop<true, true, false>(A, p4, live, lane, min_run, ww0, 0, blk);
+    else tile_loop<false, true, false>(A, p4, live, lane, min_run, ww0, 0, blk);
+  } else {
+    if (tail) tile_loop<true, false, false>(A, p4, live, lane, min_run, ww0, 0, blk);
+    else tile_loop<false, false, false>(A, p4, live, lane, min_run, ww0, 0, blk);
   }
 
   // counters: 6 raw bit classes + any/gpu/alternating
   uint32_t c9[9];
-  c9[0] = raw.count(0x04040404u);  // wC
-  c9[1] = raw.count(0x08080808u);  // wG
-  c9[2] = raw.count(0x10101010u);  // rCC
-  c9[3] = raw.count(0x40404040u);  // rCG
-  c9[4] = raw.count(0x20202020u);  // rGC
-  c9[5] = raw.count(0x80808080u);  // rGG
-  c9[6] = der.count(0x80808080u);  // any
-  c9[7] = der.count(0x40404040u);  // gpu
-  c9[8] = der.count(0x20202020u);  // alternating
+  c9[0] = A.raw.count(0x04040404u);  // wC
+  c9[1] = A.raw.count(0x08080808u);  // wG
+  c9[2] = A.raw.count(0x10101010u);  // rCC
+  c9[3] = A.raw.count(0x40404040u);  // rCG
+  c9[4] = A.raw.count(0x20202020u);  // rGC
+  c9[5] = A.raw.count(0x80808080u);  // rGG
+  c9[6] = A.der.count(0x80808080u);  // any
+  c9[7] = A.der.count(0x40404040u);  // gpu
+  c9[8] = A.der.count(0x20202020u);  // alternating
 #pragma unroll
   for (int k = 0; k < 9; ++k) {
     const uint32_t s = __reduce_add_sync(0xFFFFFFFFu, c9[k]);
     if (lane == 0) s_cnt[warp][k] = s;
   }
   if (lane == 0) {
-    s_u[warp] = wu;
-    s_d[warp] = wd;
+    s_u[warp] = A.wu;
+    s_d[warp] = A.wd;
   }
   __syncthreads();
   if (threadIdx.x < 9) {
     uint32_t s = 0;
-    for (uint32_t w = 0; w < kDiagThreads / 32; ++w) s += s_cnt[w][threadIdx.x];
+    for (uint32_t w = 0; w < kWarps; ++w) s += s_cnt[w][threadIdx.x];
     if (s) atomicAdd(cnt + (uint64_t)ri * C_NCNT + threadIdx.x, (unsigned long long)s);
   } else if (threadIdx.x == 32) {
     RunSum a = s_u[0], b = s_d[0];
-    for (uint32_t w = 1; w < kDiagThreads / 32; ++w) {
-      a = rs_combine(a, s_u[w], min_run);
-      b = rs_combine(b, s_d[w], min_run);
+    for (uint32_t w = 1; w < kWarps; ++w) {
+      a = rs_combine32(a, s_u[w], min_run);
+      b = rs_combine32(b, s_d[w], min_run);
     }
     tiles[t].u = a;
     tiles[t].d = b;
@@ -512,50 +571,116 @@ __device__ __forceinline__ void run_final(const RunSum64& s, uint64_t min_run, u
   *words = w;
 }
 
-// One warp per row: ordered combine of the row's tile summaries.
-__global__ void stitch_kernel(const DiagRow* __restrict__ rows, uint32_t nrows,
-                              const TileSum* __restrict__ tiles, uint64_t min_run,
-                              unsigned long long* __restrict__ cnt) {
+struct RunPair {
+  RunSum64 u, d;
+};
+static_assert(sizeof(RunPair) == kRunPairBytes, "RunPair size");
+
+__device__ __forceinline__ RunSum64 shfl_down_rs(const RunSum64& a, uint32_t s) {
+  RunSum64 o;
+  o.len = __shfl_down_sync(0xFFFFFFFFu, a.len, s);
+  o.pre = __shfl_down_sync(0xFFFFFFFFu, a.pre, s);
+  o.suf = __shfl_down_sync(0xFFFFFFFFu, a.suf, s);
+  o.cnt = __shfl_down_sync(0xFFFFFFFFu, a.cnt, s);
+  o.sum = __shfl_down_sync(0xFFFFFFFFu, a.sum, s);
+  return o;
+}
+
+// Ordered warp reduction: lane 0 ends with combine(lane 0, ..., lane 31).
+__device__ __forceinline__ void warp_combine(RunSum64& a, RunSum64& b, uint32_t lane, uint64_t min_run) {
+  for (uint32_t s = 1; s < 32; s <<= 1) {
+    const RunSum64 oa = shfl_down_rs(a, s), ob = shfl_down_rs(b, s);
+    if ((lane & (2 * s - 1)) == 0 && lane + s < 32) {
+      a = rs_combine(a, oa, min_run);
+      b = rs_combine(b, ob, min_run);
+    }
+  }
+}
+
+// Stitch, level 1: one warp per segment of <= kSegTiles consecutive tiles of a
+// row; lanes combine contiguous sub-ranges, then an ordered warp reduction.
+__global__ void stitch_seg_kernel(const StitchSeg* __restrict__ segs, uint32_t nseg,
+                                  const TileSum* __restrict__ tiles, uint64_t min_run,
+                                  RunPair* __restrict__ out) {
   const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const uint32_t lane = threadIdx.x & 31;
-  if (gw >= nrows) return;
-  const DiagRow row = rows[gw];
-  const uint64_t per = (row.ntiles + 31) / 32;
-  const uint64_t t0 = row.tile0 + lane * per;
-  const uint64_t t1 = min(row.tile0 + row.ntiles, t0 + per);
+  if (gw >= nseg) return;
+  const StitchSeg sg = segs[gw];
+  const uint64_t per = (sg.n + 31) / 32;
+  const uint64_t t0 = sg.t0 + lane * per;
+  const uint64_t t1 = min(sg.t0 + sg.n, t0 + per);
   RunSum64 a = {0, 0, 0, 0, 0}, b = {0, 0, 0, 0, 0};
   for (uint64_t t = t0; t < t1; ++t) {
     const RunSum u = tiles[t].u, d = tiles[t].d;
     a = rs_combine(a, RunSum64{u.len, u.pre, u.suf, u.cnt, u.sum}, min_run);
     b = rs_combine(b, RunSum64{d.len, d.pre, d.suf, d.cnt, d.sum}, min_run);
   }
-  for (uint32_t s = 1; s < 32; s <<= 1) {
-    RunSum64 oa, ob;
-    oa.len = __shfl_down_sync(0xFFFFFFFFu, a.len, s);
-    oa.pre = __shfl_down_sync(0xFFFFFFFFu, a.pre, s);
-    oa.suf = __shfl_down_sync(0xFFFFFFFFu, a.suf, s);
-    oa.cnt = __shfl_down_sync(0xFFFFFFFFu, a.cnt, s);
-    oa.sum = __shfl_down_sync(0xFFFFFFFFu, a.sum, s);
-    ob.len = __shfl_down_sync(0xFFFFFFFFu, b.len, s);
-    ob.pre = __shfl_down_sync(0xFFFFFFFFu, b.pre, s);
-    ob.suf = __shfl_down_sync(0xFFFFFFFFu, b.suf, s);
-    ob.cnt = __shfl_down_sync(0xFFFFFFFFu, b.cnt, s);
-    ob.sum = __shfl_down_sync(0xFFFFFFFFu, b.sum, s);
-    if ((lane & (2 * s - 1)) == 0 && lane + s < 32) {
-      a = rs_combine(a, oa, min_run);
-      b = rs_combine(b, ob, min_run);
-    }
+  warp_combine(a, b, lane, min_run);
+  if (lane == 0) out[gw] = RunPair{a, b};
+}
+
+// Stitch, level 2 + finalize: one warp per row combines its segment summaries,
+// then lane 0 turns the counters into the report row (flags P:L84-114, D8).
+__global__ void stitch_row_finalize_kernel(const DiagRow* __restrict__ rows, uint32_t nrows,
+                                           const RunPair* __restrict__ segsum, DiagParams p,
+                                           unsigned long long* __restrict__ cnt,
+                                           xpl_alloc_report* __restrict__ out) {
+  const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint32_t lane = threadIdx.x & 31;
+  if (gw >= nrows) return;
+  const DiagRow r = rows[gw];
+  const uint64_t per = (r.nseg + 31) / 32;
+  const uint64_t s0 = r.seg0 + lane * per;
+  const uint64_t s1 = min(r.seg0 + r.nseg, s0 + per);
+  RunSum64 a = {0, 0, 0, 0, 0}, b = {0, 0, 0, 0, 0};
+  for (uint64_t s = s0; s < s1; ++s) {
+    a = rs_combine(a, segsum[s].u, p.min_run);
+    b = rs_combine(b, segsum[s].d, p.min_run);
   }
-  if (lane == 0) {
-    uint64_t r, w;
-    unsigned long long* c = cnt + (uint64_t)gw * C_NCNT;
-    run_final(a, min_run, &r, &w);
-    c[C_UR] = r;
-    c[C_UW] = w;
-    run_final(b, min_run, &r, &w);
-    c[C_DR] = r;
-    c[C_DW] = w;
+  warp_combine(a, b, lane, p.min_run);
+  if (lane != 0) return;
+  const unsigned long long* c = cnt + (uint64_t)gw * C_NCNT;
+  xpl_alloc_report o;
+  o.id = o.base = o.bytes = 0;
+  o.words = r.words;
+  o.kind = r.kind;
+  o.live = 0;
+  o.name_idx = 0xFFFFFFFFu;
+  o.w_c = c[C_WC];
+  o.w_g = c[C_WG];
+  o.r_cc = c[C_RCC];
+  o.r_cg = c[C_RCG];
+  o.r_gc = c[C_RGC];
+  o.r_gg = c[C_RGG];
+  o.any_acc = c[C_ANY];
+  o.gpu_acc = c[C_GPU];
+  o.alternating = c[C_ALT];
+  o.density_pct_any = o.any_acc * 100 / r.words;
+  o.density_pct_gpu = o.gpu_acc * 100 / r.words;
+  if (p.block_words == 0) {
+    const bool f = o.gpu_acc >= 1 && 100ull * o.gpu_acc <= (uint64_t)p.thr * r.words;
+    o.low_density_blocks = f ? 1 : 0;
+    o.low_density_words = f ? r.words : 0;
+  } else {
+    o.low_density_blocks = c[C_LDB];
+    o.low_density_words = c[C_LDW];
   }
+  uint64_t rr, ww;
+  run_final(a, p.min_run, &rr, &ww);
+  o.h2d_unused_runs = rr;
+  o.h2d_unused_words = ww;
+  run_final(b, p.min_run, &rr, &ww);
+  o.d2h_unneeded_runs = rr;
+  o.d2h_unneeded_words = ww;
+  o.ever_accessed = 0;
+  uint32_t f = 0;
+  if (r.kind == XPL_ALLOC_MANAGED && o.alternating > 0) f |= XPL_PAT_ALTERNATING;
+  if (r.kind != XPL_ALLOC_HOST && o.low_density_blocks > 0) f |= XPL_PAT_LOW_DENSITY;
+  if (r.kind == XPL_ALLOC_DEVICE && o.h2d_unused_runs > 0) f |= XPL_PAT_UNNEEDED_H2D;
+  if (r.kind == XPL_ALLOC_DEVICE && o.d2h_unneeded_runs > 0) f |= XPL_PAT_UNNEEDED_D2H;
+  if (o.any_acc == 0) f |= XPL_PAT_UNUSED;
+  o.flags = f;
+  out[gw] = o;
 }
 
 // Low-density blocks (Eq. P:L102, D11-D13): block flagged iff it has
@@ -583,53 +708,6 @@ __global__ void block_eval_kernel(const DiagRow* __restrict__ rows, uint32_t nro
   }
 }
 
-__global__ void finalize_kernel(const DiagRow* __restrict__ rows, uint32_t nrows, DiagParams p,
-                                const unsigned long long* __restrict__ cnt,
-                                xpl_alloc_report* __restrict__ out) {
-  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= nrows) return;
-  const DiagRow r = rows[i];
-  const unsigned long long* c = cnt + (uint64_t)i * C_NCNT;
-  xpl_alloc_report o;
-  o.id = o.base = o.bytes = 0;
-  o.words = r.words;
-  o.kind = r.kind;
-  o.live = 0;
-  o.name_idx = 0xFFFFFFFFu;
-  o.w_c = c[C_WC];
-  o.w_g = c[C_WG];
-  o.r_cc = c[C_RCC];
-  o.r_cg = c[C_RCG];
-  o.r_gc = c[C_RGC];
-  o.r_gg = c[C_RGG];
-  o.any_acc = c[C_ANY];
-  o.gpu_acc = c[C_GPU];
-  o.alternating = c[C_ALT];
-  o.density_pct_any = o.any_acc * 100 / r.words;
-  o.density_pct_gpu = o.gpu_acc * 100 / r.words;
-  if (p.block_words == 0) {
-    const bool f = o.gpu_acc >= 1 && 100ull * o.gpu_acc <= (uint64_t)p.thr * r.words;
-    o.low_density_blocks = f ? 1 : 0;
-    o.low_density_words = f ? r.words : 0;
-  } else {
-    o.low_density_blocks = c[C_LDB];
-    o.low_density_words = c[C_LDW];
-  }
-  o.h2d_unused_runs = c[C_UR];
-  o.h2d_unused_words = c[C_UW];
-  o.d2h_unneeded_runs = c[C_DR];
-  o.d2h_unneeded_words = c[C_DW];
-  o.ever_accessed = 0;
-  uint32_t f = 0;
-  if (r.kind == XPL_ALLOC_MANAGED && o.alternating > 0) f |= XPL_PAT_ALTERNATING;
-  if (r.kind != XPL_ALLOC_HOST && o.low_density_blocks > 0) f |= XPL_PAT_LOW_DENSITY;
-  if (r.kind == XPL_ALLOC_DEVICE && o.h2d_unused_runs > 0) f |= XPL_PAT_UNNEEDED_H2D;
-  if (r.kind == XPL_ALLOC_DEVICE && o.d2h_unneeded_runs > 0) f |= XPL_PAT_UNNEEDED_D2H;
-  if (o.any_acc == 0) f |= XPL_PAT_UNUSED;
-  o.flags = f;
-  out[i] = o;
-}
-
 __global__ void fill_u32_kernel(uint32_t* p, uint64_t n, uint32_t v) {
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
        i += (uint64_t)gridDim.x * blockDim.x)
@@ -645,10 +723,9 @@ int grid_for(uint64_t n, int threads, int max_ctas) {
 
 }  // namespace
 
-void launch_fold(cudaStream_t s, uint32_t* pool, uint64_t pool_u32, const uint32_t* dirty,
-                 uint32_t* dirty_count, uint32_t dirty_cap, uint32_t* done_ctr,
-                 unsigned long long* stats) {
-  fold_kernel<<<148, 256, 0, s>>>(pool, pool_u32, dirty, dirty_count, dirty_cap, done_ctr, stats);
+void launch_fold(cudaStream_t s, uint32_t* pool, uint8_t* cmap, uint8_t* smap,
+                 uint64_t n_super, unsigned long long* stats) {
+  if (n_super) fold_kernel<<<grid_for(n_super * 256, 256, 148 * 64), 256, 0, s>>>(pool, cmap, smap, n_super, stats);
 }
 
 void launch_merge(cudaStream_t s, const uint64_t* recs, uint32_t n, bool has_r, bool has_w,
@@ -661,25 +738,28 @@ void launch_merge(cudaStream_t s, const uint64_t* recs, uint32_t n, bool has_r, 
 }
 
 void launch_range(cudaStream_t s, const RangeDesc* d_ranges, uint32_t nr, uint64_t nvec,
-                  uint32_t* pool, uint32_t* dirty, uint32_t* dirty_count, uint32_t dirty_cap) {
+                  uint32_t* pool, uint8_t* cmap, uint8_t* smap) {
   const int g = grid_for(nvec, 256, 148 * 8);
-  range_kernel<<<g, 256, 0, s>>>(d_ranges, nr, nvec, pool, dirty, dirty_count, dirty_cap);
+  range_kernel<<<g, 256, 0, s>>>(d_ranges, nr, nvec, pool, cmap, smap);
 }
 
 void launch_diag(cudaStream_t s, const DiagRow* rows, uint32_t nrows, const uint32_t* tile_row,
-                 uint64_t ntiles, uint64_t nblocks, const DiagParams& p, uint32_t* pool,
-                 unsigned long long* cnt, TileSum* tiles, uint32_t* blk_cnt,
-                 xpl_alloc_report* out, cudaEvent_t tile_ev0, cudaEvent_t tile_ev1) {
+                 uint64_t ntiles, const StitchSeg* segs, uint32_t nseg, uint64_t nblocks,
+                 const DiagParams& p, uint32_t* pool, unsigned long long* cnt, TileSum* tiles,
+                 void* segsum, uint32_t* blk_cnt, xpl_alloc_report* out, cudaEvent_t tile_ev0,
+                 cudaEvent_t tile_ev1) {
   cudaMemsetAsync(cnt, 0, sizeof(unsigned long long) * C_NCNT * nrows, s);
   if (p.block_words && nblocks) cudaMemsetAsync(blk_cnt, 0, sizeof(uint32_t) * nblocks, s);
   if (tile_ev0) cudaEventRecord(tile_ev0, s);
   if (ntiles) diag_tile_kernel<<<(unsigned)ntiles, kDiagThreads, 0, s>>>(rows, tile_row, p, pool, cnt, tiles, blk_cnt);
   if (tile_ev1) cudaEventRecord(tile_ev1, s);
-  stitch_kernel<<<(nrows * 32 + 255) / 256, 256, 0, s>>>(rows, nrows, tiles, p.min_run, cnt);
   if (p.block_words && nblocks)
     block_eval_kernel<<<grid_for(nblocks, 256, 148 * 8), 256, 0, s>>>(rows, nrows, nblocks, blk_cnt,
                                                                     p.block_words, p.thr, cnt);
-  finalize_kernel<<<(nrows + 127) / 128, 128, 0, s>>>(rows, nrows, p, cnt, out);
+  stitch_seg_kernel<<<(nseg * 32 + 255) / 256, 256, 0, s>>>(segs, nseg, tiles, p.min_run,
+                                                             (RunPair*)segsum);
+  stitch_row_finalize_kernel<<<(nrows * 32 + 255) / 256, 256, 0, s>>>(rows, nrows, (const RunPair*)segsum,
+                                                                       p, cnt, out);
 }
 
 void launch_fill_u32(cudaStream_t s, uint32_t* p, uint64_t n, uint32_t v) {

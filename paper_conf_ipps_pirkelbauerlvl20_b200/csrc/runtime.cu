@@ -34,11 +34,13 @@ struct Row {
 // starts on a 16-byte boundary for the vector loads of diagnose).
 struct PoolAlloc {
   std::map<uint64_t, uint64_t> free_;  // off -> len
-  void init(uint64_t cap) { free_.clear(); free_[0] = cap; }
+  uint64_t hwm = 0;                    // high-water mark: no row ever extended past it
+  void init(uint64_t cap) { free_.clear(); free_[0] = cap; hwm = 0; }
   bool alloc(uint64_t n, uint64_t* off) {
     for (auto it = free_.begin(); it != free_.end(); ++it) {
       if (it->second >= n) {
         *off = it->first;
+        if (it->first + n > hwm) hwm = it->first + n;
         const uint64_t rest = it->second - n, o = it->first + n;
         free_.erase(it);
         if (rest) free_[o] = rest;
@@ -91,9 +93,10 @@ struct xpl_ctx {
   cudaEvent_t table_ev = nullptr;
   const Row* cache = nullptr;          // last host lookup hit
 
-  // dirty list (epoch close)
-  uint32_t* d_dirty = nullptr;
-  uint32_t* d_misc = nullptr;          // [0] dirty_count, [1] fold done counter
+  // epoch close: chunk maps (1 B per 128 words, 1 B per 16K words) + chunk list
+  uint8_t* d_cmap = nullptr;
+  uint8_t* d_smap = nullptr;
+  uint32_t* d_misc = nullptr;          // scratch counters
   unsigned long long* d_stats = nullptr;
 
   // epochs (D19)
@@ -127,6 +130,10 @@ struct xpl_ctx {
   size_t tiles_cap = 0;
   uint32_t* d_blk = nullptr;
   size_t blk_cap = 0;
+  StitchSeg* h_segs = nullptr;
+  StitchSeg* d_segs = nullptr;
+  void* d_segsum = nullptr;
+  size_t segs_cap = 0;
   unsigned long long* d_cnt = nullptr;
   xpl_alloc_report* d_rep = nullptr;
   xpl_alloc_report* h_rep = nullptr;
@@ -144,6 +151,7 @@ struct xpl_ctx {
   std::vector<cudaEvent_t> prof_free;
   xpl_kernel_time prof_acc[XPL_K_NCLASS];
   unsigned long long fold_entries_seen = 0;
+  uint64_t folds_host = 0;
 };
 
 namespace {
@@ -360,7 +368,7 @@ xpl_status flush(xpl_ctx* c) {
         for (size_t i = sg.start; i < sg.start + sg.n; ++i) rw += c->h_ranges[i].nw;
         const int pi = prof_begin(c, XPL_K_RANGE, 2 * rw);
         launch_range(c->rs, c->d_ranges + sg.start, (uint32_t)sg.n, nvec, (uint32_t*)c->d_pool,
-                     c->d_dirty, c->d_misc, (uint32_t)c->cfg.dirty_cap);
+                     c->d_cmap, c->d_smap);
         c->st.kernel_launches += 1;
         prof_end(c, pi);
         c->st.range_segments++;
@@ -432,8 +440,7 @@ xpl_status gpu_ranges(xpl_ctx* c, const RangeDesc* rd, size_t nr) {
   uint64_t rw = 0;
   for (size_t i = 0; i < nr; ++i) rw += rd[i].nw;
   const int pi = prof_begin(c, XPL_K_RANGE, 2 * rw);
-  launch_range(c->rs, c->d_ranges, (uint32_t)nr, v, (uint32_t*)c->d_pool, c->d_dirty, c->d_misc,
-               (uint32_t)c->cfg.dirty_cap);
+  launch_range(c->rs, c->d_ranges, (uint32_t)nr, v, (uint32_t*)c->d_pool, c->d_cmap, c->d_smap);
   c->st.kernel_launches += 1;
   prof_end(c, pi);
   return cudaGetLastError() == cudaSuccess ? XPL_OK : XPL_ERR_CUDA;
@@ -441,8 +448,10 @@ xpl_status gpu_ranges(xpl_ctx* c, const RangeDesc* rd, size_t nr) {
 
 void fold(xpl_ctx* c) {
   const int pi = prof_begin(c, XPL_K_FOLD, 0);
-  launch_fold(c->rs, (uint32_t*)c->d_pool, c->pool_words / 4, c->d_dirty, c->d_misc,
-              (uint32_t)c->cfg.dirty_cap, c->d_misc + 1, c->d_stats);
+  // only super-chunks below the pool's high-water mark can be marked
+  launch_fold(c->rs, (uint32_t*)c->d_pool, c->d_cmap, c->d_smap, (c->pa.hwm + 16383) / 16384,
+              c->d_stats);
+  c->folds_host++;
   c->st.kernel_launches += 1;
   prof_end(c, pi);
 }
@@ -475,11 +484,9 @@ xpl_status xpl_init(const xpl_config* cfg, xpl_ctx** out) {
   if (!c) return XPL_ERR_OOM;
   c->cfg = *cfg;
   if (!c->cfg.pool_words) c->cfg.pool_words = 1ull << 28;
-  if (!c->cfg.dirty_cap) c->cfg.dirty_cap = 1ull << 24;
-  if (c->cfg.dirty_cap > 0xFFFFFFF0ull) c->cfg.dirty_cap = 0xFFFFFFF0ull;
   if (!c->cfg.staging_recs) c->cfg.staging_recs = 1ull << 22;
   if (!c->cfg.max_rows) c->cfg.max_rows = 4096;
-  c->pool_words = (c->cfg.pool_words + 15) & ~15ull;
+  c->pool_words = (c->cfg.pool_words + 65535) & ~65535ull;  // whole 4-byte words of the super map
   if (c->pool_words / 4 > 0xFFFFFFFFull) { delete c; return XPL_ERR_INVALID_ARG; }
 #define CKI(x)                  \
   do {                          \
@@ -496,7 +503,10 @@ xpl_status xpl_init(const xpl_config* cfg, xpl_ctx** out) {
   CKI(cudaMalloc(&c->d_tab, 32 + sizeof(xpl_dev_row) * c->cfg.max_rows));
   CKI(cudaMemsetAsync(c->d_tab, 0, 32, c->rs));
   CKI(host_alloc(&c->h_tab, 32 + sizeof(xpl_dev_row) * c->cfg.max_rows));
-  CKI(cudaMalloc(&c->d_dirty, sizeof(uint32_t) * c->cfg.dirty_cap));
+  CKI(cudaMalloc(&c->d_cmap, c->pool_words / 128));
+  CKI(cudaMemsetAsync(c->d_cmap, 0, c->pool_words / 128, c->rs));
+  CKI(cudaMalloc(&c->d_smap, c->pool_words / 16384));
+  CKI(cudaMemsetAsync(c->d_smap, 0, c->pool_words / 16384, c->rs));
   CKI(cudaMalloc(&c->d_misc, 64));
   CKI(cudaMemsetAsync(c->d_misc, 0, 64, c->rs));
   CKI(cudaMalloc(&c->d_stats, 64));
@@ -530,7 +540,8 @@ xpl_status xpl_finalize(xpl_ctx* c) {
   cudaFree(c->d_first_w);
   cudaFree(c->d_tab);
   cudaFreeHost(c->h_tab);
-  cudaFree(c->d_dirty);
+  cudaFree(c->d_cmap);
+  cudaFree(c->d_smap);
   cudaFree(c->d_misc);
   cudaFree(c->d_stats);
   cudaFreeHost(c->h_stage[0]);
@@ -544,6 +555,9 @@ xpl_status xpl_finalize(xpl_ctx* c) {
   cudaFree(c->d_tile_row);
   cudaFree(c->d_tiles);
   cudaFree(c->d_blk);
+  cudaFreeHost(c->h_segs);
+  cudaFree(c->d_segs);
+  cudaFree(c->d_segsum);
   cudaFree(c->d_cnt);
   cudaFree(c->d_rep);
   cudaFreeHost(c->h_rep);
@@ -782,10 +796,8 @@ xpl_status xpl_get_device_ctx(xpl_ctx* c, struct xpl_dev_ctx* d) {
   d->rows = (const xpl_dev_row*)(c->d_tab + 32);
   d->n_rows = (const unsigned int*)c->d_tab;
   d->pool = (unsigned int*)c->d_pool;
-  d->dirty = c->d_dirty;
-  d->dirty_count = c->d_misc;
-  d->dirty_cap = (unsigned int)c->cfg.dirty_cap;
-  d->pad_ = 0;
+  d->cmap = c->d_cmap;
+  d->smap = c->d_smap;
   return XPL_OK;
 }
 
@@ -795,9 +807,9 @@ xpl_status xpl_get_stats(xpl_ctx* c, xpl_stats* o) {
   CK(cudaStreamSynchronize(c->rs));
   CK(cudaMemcpy(ds, c->d_stats, sizeof ds, cudaMemcpyDeviceToHost));
   *o = c->st;
-  o->dirty_max = ds[0];
-  o->fold_full_scans = ds[1];
-  o->folds = ds[2];
+  o->fold_chunks_max = 0;  // (not tracked by the one-kernel fold)
+  o->fold_chunks = ds[3];
+  o->folds = c->folds_host;
   return XPL_OK;
 }
 
@@ -829,7 +841,7 @@ xpl_status xpl_profile_read(xpl_ctx* c, xpl_kernel_time* out, int reset) {
   c->prof_pending.clear();
   unsigned long long ds[8];
   CK(cudaMemcpy(ds, c->d_stats, sizeof ds, cudaMemcpyDeviceToHost));
-  c->prof_acc[XPL_K_FOLD].bytes += 12ull * (ds[3] - c->fold_entries_seen);
+  c->prof_acc[XPL_K_FOLD].bytes += 256ull * (ds[3] - c->fold_entries_seen);  // 128 B read + 128 B written
   c->fold_entries_seen = ds[3];
   for (int k = 0; k < XPL_K_NCLASS; ++k) out[k] = c->prof_acc[k];
   if (reset) memset(c->prof_acc, 0, sizeof c->prof_acc);
@@ -875,10 +887,12 @@ xpl_status xpl_diagnose(xpl_ctx* c, const xpl_diag_params* params, const xpl_nam
   if (nr == 0) return XPL_OK;
 
   // geometry
-  uint64_t ntiles = 0, nblocks = 0;
+  uint64_t ntiles = 0, nblocks = 0, nseg = 0;
   for (uint64_t id : ids) {
     const Row& r = c->rows[id];
-    ntiles += (r.words + kTileWords - 1) / kTileWords;
+    const uint64_t nt = (r.words + kTileWords - 1) / kTileWords;
+    ntiles += nt;
+    nseg += (nt + kSegTiles - 1) / kSegTiles;
     if (p.block_words) nblocks += (r.words + p.block_words - 1) / p.block_words;
   }
   if (ntiles > 0x7FFFFFFFull) return XPL_ERR_OOM;
@@ -904,12 +918,21 @@ xpl_status xpl_diagnose(xpl_ctx* c, const xpl_diag_params* params, const xpl_nam
     CK(cudaMalloc(&c->d_tile_row, sizeof(uint32_t) * c->tiles_cap));
     CK(cudaMalloc(&c->d_tiles, sizeof(TileSum) * c->tiles_cap));
   }
+  if (nseg > c->segs_cap) {
+    cudaFreeHost(c->h_segs);
+    cudaFree(c->d_segs);
+    cudaFree(c->d_segsum);
+    c->segs_cap = std::max<uint64_t>(nseg, 1024);
+    CK(host_alloc(&c->h_segs, c->segs_cap));
+    CK(cudaMalloc(&c->d_segs, sizeof(StitchSeg) * c->segs_cap));
+    CK(cudaMalloc(&c->d_segsum, kRunPairBytes * c->segs_cap));
+  }
   if (nblocks > c->blk_cap) {
     cudaFree(c->d_blk);
     c->blk_cap = std::max<uint64_t>(nblocks, 1024);
     CK(cudaMalloc(&c->d_blk, sizeof(uint32_t) * c->blk_cap));
   }
-  uint64_t t = 0, b = 0;
+  uint64_t t = 0, b = 0, sgi = 0;
   for (size_t i = 0; i < nr; ++i) {
     const Row& r = c->rows[ids[i]];
     DiagRow& d = c->h_drows[i];
@@ -921,6 +944,13 @@ xpl_status xpl_diagnose(xpl_ctx* c, const xpl_diag_params* params, const xpl_nam
     d.nblk = p.block_words ? (r.words + p.block_words - 1) / p.block_words : 0;
     d.kind = r.kind;
     d.pad = 0;
+    d.seg0 = sgi;
+    d.nseg = (d.ntiles + kSegTiles - 1) / kSegTiles;
+    for (uint64_t k = 0; k < d.nseg; ++k) {
+      c->h_segs[sgi + k].t0 = t + k * kSegTiles;
+      c->h_segs[sgi + k].n = std::min<uint64_t>(kSegTiles, d.ntiles - k * kSegTiles);
+    }
+    sgi += d.nseg;
     for (uint64_t k = 0; k < d.ntiles; ++k) c->h_tile_row[t + k] = (uint32_t)i;
     t += d.ntiles;
     b += d.nblk;
@@ -928,13 +958,14 @@ xpl_status xpl_diagnose(xpl_ctx* c, const xpl_diag_params* params, const xpl_nam
   CK(cudaMemcpyAsync(c->d_drows, c->h_drows, sizeof(DiagRow) * nr, cudaMemcpyHostToDevice, c->rs));
   CK(cudaMemcpyAsync(c->d_tile_row, c->h_tile_row, sizeof(uint32_t) * ntiles,
                      cudaMemcpyHostToDevice, c->rs));
+  CK(cudaMemcpyAsync(c->d_segs, c->h_segs, sizeof(StitchSeg) * nseg, cudaMemcpyHostToDevice, c->rs));
   uint64_t total_words = 0;
   for (size_t i = 0; i < nr; ++i) total_words += c->h_drows[i].words;
   const uint64_t dbytes = total_words * (reset ? 2 : 1);
   const int pall = prof_begin(c, XPL_K_DIAGNOSE, dbytes);
   const int ptile = prof_begin(c, XPL_K_DIAG_TILE, dbytes, false);  // recorded by launch_diag
-  launch_diag(c->rs, c->d_drows, (uint32_t)nr, c->d_tile_row, ntiles, nblocks, p,
-              (uint32_t*)c->d_pool, c->d_cnt, c->d_tiles, c->d_blk, c->d_rep,
+  launch_diag(c->rs, c->d_drows, (uint32_t)nr, c->d_tile_row, ntiles, c->d_segs, (uint32_t)nseg,
+              nblocks, p, (uint32_t*)c->d_pool, c->d_cnt, c->d_tiles, c->d_segsum, c->d_blk, c->d_rep,
               ptile >= 0 ? c->prof_pending[ptile].a : nullptr,
               ptile >= 0 ? c->prof_pending[ptile].b : nullptr);
   CK(cudaGetLastError());

@@ -19,9 +19,48 @@ __global__ void replay_kernel(const unsigned long long* __restrict__ addr,
     xpl_dev_record((const void*)addr[i], size[i], acc[i]);
 }
 
+__device__ __forceinline__ unsigned hash32(unsigned x) {
+  x ^= x >> 16;
+  x *= 0x7feb352du;
+  x ^= x >> 15;
+  x *= 0x846ca68bu;
+  x ^= x >> 16;
+  return x;
+}
+
+// A synthetic instrumented kernel over n words at address `base` (no memory
+// behind it: hooks only use addresses).  Per 4096-word block one of: untouched,
+// all read, all written, or a per-word random R/W/RW mix -- long runs and
+// mixed regions, like a real shadow.
+__global__ void touch_kernel(unsigned long long base, unsigned long long n, unsigned seed) {
+  for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (unsigned long long)gridDim.x * blockDim.x) {
+    const unsigned hb = hash32((unsigned)(i >> 12) ^ seed);
+    unsigned acc = 0;
+    switch (hb & 3) {
+      case 1: acc = XPL_ACC_R; break;
+      case 2: acc = XPL_ACC_W; break;
+      case 3: {
+        const unsigned h = hash32((unsigned)i ^ (seed * 0x9E3779B9u));
+        acc = (h & 3);  // 0 = no access
+        break;
+      }
+      default: break;
+    }
+    if (acc) xpl_dev_record((const void*)(base + 4 * i), 4, acc);
+  }
+}
+
 }  // namespace
 
 extern "C" {
+
+// Launch the synthetic touch kernel (between xpl_kernel_begin/_end).
+int xplw_touch(unsigned long long base, unsigned long long n, unsigned seed, void* stream) {
+  touch_kernel<<<148 * 16, 256, 0, (cudaStream_t)stream>>>(base, n, seed);
+  return cudaGetLastError() == cudaSuccess ? 0 : (int)XPL_ERR_CUDA;
+}
+
 
 int xplw_bind_rodinia(xpl_ctx* ctx);
 

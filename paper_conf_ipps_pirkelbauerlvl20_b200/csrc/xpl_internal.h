@@ -38,8 +38,8 @@ struct RangeDesc {
 };
 
 // Diagnose geometry.
-constexpr uint32_t kTileWords = 32768;         // words per diagnose tile (one CTA)
-constexpr uint32_t kDiagThreads = 256;         // 8 warps x 32 lanes x 16 words x 8 iters
+constexpr uint32_t kTileWords = 16384;         // words per diagnose tile (one CTA)
+constexpr uint32_t kDiagThreads = 128;         // 4 warps x 32 lanes x 16 words x 8 iters
 constexpr uint32_t kDiagIters = 8;
 
 struct DiagRow {        // one row to analyse (live or dead-since-last-reset)
@@ -48,7 +48,14 @@ struct DiagRow {        // one row to analyse (live or dead-since-last-reset)
   uint64_t ntiles;
   uint64_t blk0;        // first block-counter index (block_words > 0)
   uint64_t nblk;
+  uint64_t seg0, nseg;  // its stitch segments
   uint32_t kind, pad;
+};
+
+// Stitch segment: <= kSegTiles consecutive tiles of one row.
+constexpr uint64_t kSegTiles = 1024;
+struct StitchSeg {
+  uint64_t t0, n;
 };
 
 // Per-row counters accumulated by the diagnose kernels (u64 each).
@@ -73,17 +80,18 @@ struct DiagParams {
 };
 
 // ---- launchers (kernels.cu) ----
-void launch_fold(cudaStream_t s, uint32_t* pool, uint64_t pool_u32, const uint32_t* dirty,
-                 uint32_t* dirty_count, uint32_t dirty_cap, uint32_t* done_ctr,
-                 unsigned long long* stats);
+void launch_fold(cudaStream_t s, uint32_t* pool, uint8_t* cmap, uint8_t* smap,
+                 uint64_t n_super, unsigned long long* stats);
 void launch_merge(cudaStream_t s, const uint64_t* recs, uint32_t n, bool has_r, bool has_w,
                   uint32_t* first_w, uint32_t* pool);
 void launch_range(cudaStream_t s, const RangeDesc* d_ranges, uint32_t nr, uint64_t nvec,
-                  uint32_t* pool, uint32_t* dirty, uint32_t* dirty_count, uint32_t dirty_cap);
+                  uint32_t* pool, uint8_t* cmap, uint8_t* smap);
 void launch_diag(cudaStream_t s, const DiagRow* rows, uint32_t nrows, const uint32_t* tile_row,
-                 uint64_t ntiles, uint64_t nblocks, const DiagParams& p, uint32_t* pool,
-                 unsigned long long* cnt, TileSum* tiles, uint32_t* blk_cnt,
-                 xpl_alloc_report* out, cudaEvent_t tile_ev0, cudaEvent_t tile_ev1);
+                 uint64_t ntiles, const StitchSeg* segs, uint32_t nseg, uint64_t nblocks,
+                 const DiagParams& p, uint32_t* pool, unsigned long long* cnt, TileSum* tiles,
+                 void* segsum, uint32_t* blk_cnt, xpl_alloc_report* out, cudaEvent_t tile_ev0,
+                 cudaEvent_t tile_ev1);
+constexpr size_t kRunPairBytes = 80;  // sizeof(RunPair) in kernels.cu
 void launch_fill_u32(cudaStream_t s, uint32_t* p, uint64_t n, uint32_t v);
 
 }  // namespace xpl

@@ -34,7 +34,7 @@ HOST_ACCESS_DTYPE = np.dtype([("addr", "<u8"), ("size", "<u4"), ("kind", "<u4")]
 
 class XplConfig(C.Structure):
     _fields_ = [("device", i32), ("rank", i32), ("world", i32), ("nccl_comm", vp),
-                ("pool_words", u64), ("dirty_cap", u64), ("staging_recs", u64), ("max_rows", u32)]
+                ("pool_words", u64), ("staging_recs", u64), ("max_rows", u32)]
 
 
 class XplDiagParams(C.Structure):
@@ -62,14 +62,13 @@ class XplAllocReport(C.Structure):
 
 
 class XplStats(C.Structure):
-    _fields_ = [(n, u64) for n in ("epochs", "folds", "fold_full_scans", "host_records",
+    _fields_ = [(n, u64) for n in ("epochs", "folds", "fold_chunks", "host_records",
                                    "host_records_packed", "merge_segments", "range_segments",
-                                   "diagnoses", "dirty_max", "kernel_launches")]
+                                   "diagnoses", "fold_chunks_max", "kernel_launches")]
 
 
 class XplDevCtx(C.Structure):
-    _fields_ = [("rows", vp), ("n_rows", vp), ("pool", vp), ("dirty", vp), ("dirty_count", vp),
-                ("dirty_cap", u32), ("pad_", u32)]
+    _fields_ = [("rows", vp), ("n_rows", vp), ("pool", vp), ("cmap", vp), ("smap", vp)]
 
 
 def _sig(name, args, res=i32, lib=_lib):
@@ -116,6 +115,7 @@ EXPORTED = ["xpl_init", "xpl_finalize", "xpl_register_alloc", "xpl_free", "xpl_k
 if _work is not None:
     xplw_bind = _sig("xplw_bind", [vp], lib=_work)
     xplw_replay = _sig("xplw_replay", [vp, vp, vp, u64, i32, i32, vp], lib=_work)
+    xplw_touch = _sig("xplw_touch", [u64, u64, u32, vp], lib=_work)
 
 
 class XplError(RuntimeError):
@@ -132,8 +132,8 @@ def check(fn, status):
 class Context:
     """One xpl_ctx (one process, one GPU)."""
 
-    def __init__(self, device=0, pool_words=0, dirty_cap=0, staging_recs=0, max_rows=0):
-        cfg = XplConfig(device, 0, 1, None, pool_words, dirty_cap, staging_recs, max_rows)
+    def __init__(self, device=0, pool_words=0, staging_recs=0, max_rows=0):
+        cfg = XplConfig(device, 0, 1, None, pool_words, staging_recs, max_rows)
         h = vp()
         check("xpl_init", xpl_init(C.byref(cfg), C.byref(h)))
         self.h = h
@@ -228,6 +228,10 @@ class Context:
         d = XplDevCtx()
         check("xpl_get_device_ctx", xpl_get_device_ctx(self.h, C.byref(d)))
         return d
+
+    def touch(self, base, nwords, seed=1, stream=0):
+        """Launch the synthetic instrumented touch kernel (libxplwork) over nwords at base."""
+        check("xplw_touch", xplw_touch(base, nwords, seed, stream))
 
     def replay(self, d_addr, d_size, d_acc, n, grid=0, block=256, stream=0):
         """Launch the instrumented replay kernel (libxplwork) on device arrays."""
