@@ -3,7 +3,8 @@
 
 One STEP = one pass of the whole hot path over the
 configs[1] workload of BASELINE.json: the Rodinia-shaped instrumented programs
-(hotspot 1024x1024 x 20 iterations, backprop 640K x 16) run end to end through
+(hotspot 1024x1024 x 20 iterations, backprop 640K x 16, bfs 1M nodes x 6, nw
+2048 x 2048) run end to end through
 the C-ABI -- registration, host-tracer batches (merge), traced transfers
 (range apply), instrumented kernels (device hooks) in GPU epochs (fold), and a
 diagnose after every iteration and at the end (diagnose kernels), then frees.
@@ -38,8 +39,10 @@ sys.path.insert(0, ROOT)
 
 HOT = (1024, 1024, 20)
 BACKPROP = (655360, 16)
+BFS = (1000000, 6)
+NW = (2048, 10)
 PARAMS = (50, 0, 256)  # threshold 50 %, whole-allocation blocks, min run 256 words
-WORKLOAD = "rodinia: hotspot 1024x1024x20 + backprop 640Kx16"
+WORKLOAD = "rodinia: hotspot 1024x1024x20 + backprop 640Kx16 + bfs 1Mx6 + nw 2048x2048"
 
 
 def parse():
@@ -196,22 +199,38 @@ def main():
     from paper_conf_ipps_pirkelbauerlvl20_b200 import apps, xpl
     from xplgen import rodinia
 
-    ctx = xpl.Context(device=local, pool_words=1 << 28, max_rows=256)
+    ctx = xpl.Context(device=local, pool_words=1 << 27, max_rows=256)
     rs = torch.cuda.ExternalStream(ctx.runtime_stream())
     us = torch.cuda.Stream()
     hs = rodinia.hotspot_spec(HOT[0], HOT[1])
     bs = rodinia.backprop_spec(*BACKPROP)
-    ar_h, ar_b = apps.Arena(hs), apps.Arena(bs)
+    fs = rodinia.bfs_spec(*BFS)
+    ns = rodinia.nw_spec(NW[0])
+    ar_h, ar_b, ar_f, ar_n = apps.Arena(hs), apps.Arena(bs), apps.Arena(fs), apps.Arena(ns)
     rodinia.fill_inputs("hotspot", ar_h.host_views(), 0x58504C01)
     rodinia.fill_inputs("backprop", ar_b.host_views(), 0x58504C01)
+    edges = rodinia.bfs_graph(BFS[0], BFS[1], 0x58504C02)
+    nw_in = rodinia.nw_inputs(NW[0], NW[1], 0x58504C03)
+    hook_ctr = torch.zeros(1, dtype=torch.int64, device="cuda")
     flush_buf = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")  # > 126 MB L2
+    levels = [0]
+
+    def prepare(do_copies):
+        """Untimed: the programs' inputs (bfs graph + resident device state, nw sequences)."""
+        apps.bfs_prepare(ar_f, BFS[0], BFS[1], edges, resident=not do_copies)
+        rodinia.nw_fill_host(ar_n.host_views(), ns, nw_in, NW[0])
+        hook_ctr.zero_()
 
     def step(c, do_copies, time_kernels=False):
         counts = [0, 0, 0, 0, 0.0, 0.0]
-        for fn, ar, a in ((apps.hotspot, ar_h, HOT), (apps.backprop, ar_b, BACKPROP)):
+        progs = ((apps.hotspot, ar_h, HOT), (apps.backprop, ar_b, BACKPROP),
+                 (apps.bfs, ar_f, BFS + (hook_ctr,)), (apps.nw, ar_n, NW + (nw_in["blosum"],)))
+        for fn, ar, a in progs:
             run = apps.Run(c, us.cuda_stream, do_copies=do_copies, diag_each=True, params=PARAMS,
                            time_kernels=time_kernels)
-            fn(run, ar, *a)
+            r = fn(run, ar, *a)
+            if fn is apps.bfs:
+                levels[0] = r
             counts[0] += run.r.dev_accesses
             counts[1] += run.r.host_accesses
             counts[2] += run.r.copy_words
@@ -223,6 +242,7 @@ def main():
     def timed(c, do_copies, steps, stream):
         total, counts = 0.0, None
         for _ in range(steps):
+            prepare(do_copies)
             flush_buf.random_(0, 255)  # flush L2 between steps (untimed)
             torch.cuda.synchronize()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -232,9 +252,13 @@ def main():
             e1.synchronize()
             us.synchronize()
             total += e0.elapsed_time(e1)
+            if c is not None:
+                counts[0] += int(hook_ctr.item())  # bfs hook calls (data dependent)
+                hook_ctr.zero_()
         return total, counts
 
     for _ in range(args.warmup):
+        prepare(False)
         step(ctx, False)
     torch.cuda.synchronize()
 
@@ -260,8 +284,8 @@ def main():
     launches = (st1["kernel_launches"] - st0["kernel_launches"]) + counts[3] * args.steps
 
     # --- e2e: with the programs' real copies -----------------------------------
-    for _ in range(1):
-        step(ctx, True)
+    prepare(True)
+    step(ctx, True)
     st0 = ctx.stats()
     if world > 1:
         dist.barrier()
@@ -272,20 +296,25 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_ms = float(t.item())
     rec_bytes = 8 * (st1["host_records_packed"] - st0["host_records_packed"]) // args.steps
-    app_h2d = 4 * (2 * HOT[0] * HOT[1]) + 4 * ((BACKPROP[0] + 1) * (1 + 2 * (BACKPROP[1] + 1)) + BACKPROP[1] + 1)
-    app_d2h = 4 * HOT[0] * HOT[1] + 4 * ((BACKPROP[0] + 1) * (BACKPROP[1] + 2) + (BACKPROP[0] // 16) * BACKPROP[1])
-    n_diag_rows = 2 * (HOT[2] + 1) * 6  # upper bound of report rows per step
+    nwc = (NW[0] + 1) ** 2
+    app_h2d = (4 * (2 * HOT[0] * HOT[1]) + 4 * ((BACKPROP[0] + 1) * (1 + 2 * (BACKPROP[1] + 1)) + BACKPROP[1] + 1)
+               + (8 + 4 * BFS[1] + 3 + 4) * BFS[0] + levels[0] + 2 * 4 * nwc)
+    app_d2h = (4 * HOT[0] * HOT[1] + 4 * ((BACKPROP[0] + 1) * (BACKPROP[1] + 2) + (BACKPROP[0] // 16) * BACKPROP[1])
+               + 4 * BFS[0] + levels[0] + 4 * nwc)
+    n_diag_rows = (HOT[2] + 1) * 6 + 11 + (levels[0] + 1) * 14 + 5  # report rows per step
     e2e = {"value": per_step * args.steps * world / (e2e_ms / 1e3), "unit": "accesses/s",
            "h2d_bytes_per_step": rec_bytes + app_h2d,
            "d2h_bytes_per_step": app_d2h + 208 * n_diag_rows}
 
     # --- uninstrumented twins (slowdown, Table III context) ------------------
-    for _ in range(1):
-        step(None, False)
+    prepare(False)
+    step(None, False)
     twin_ms, _ = timed(None, False, args.steps, us)
 
     # --- breakdown (untimed pass with per-kernel events) ----------------------
+    prepare(False)
     bi = step(ctx, False, time_kernels=True)
+    prepare(False)
     bt = step(None, False, time_kernels=True)
     torch.cuda.synchronize()
 

@@ -3,16 +3,25 @@
  * object the instrumented host code calls per access.
  *
  *     xpl_host_tracer tr(ctx);
- *     for (i...) tr.write(&a[i]);            // = traceW(a[i]) = ...
+ *     for (i...) tr.write(a[i]) = ...;       // = traceW(a[i]) = ...
  *     x = tr.read(b[i]);                     // = traceR(b[i])
  *     tr.flush();                            // before kernel launches / diagnose
  *
- * The tracer coalesces consecutive accesses of one kind to adjacent bytes into
- * one byte range in the caller's thread (R and W are idempotent per word;
- * RW only when every piece is word aligned, so no word sees RW twice) and
- * hands ranges to xpl_record_host_ranges.  For programs whose individual
- * accesses never straddle two allocations (every valid C/C++ object access)
- * this is exactly the per-access semantics of xpl_record_host.
+ * Coalescing, in the caller's thread: the tracer keeps up to kRuns open runs,
+ * each a byte range [beg, end) of one access kind.  Invariant: the open runs
+ * are pairwise disjoint at 32-bit-word granularity.  An access
+ *   - that lies inside an open run of its kind (R or W) is dropped: repeating
+ *     a read or a write of a word with no other access in between changes
+ *     nothing (the invariant guarantees there was none);
+ *   - that starts where an open run of its kind ends and overlaps no other
+ *     open run extends it (RW only with word-aligned pieces, so no word sees
+ *     RW twice);
+ *   - otherwise first closes every open run it overlaps (emitting them in
+ *     their order), then opens a new run (closing the oldest if all are used).
+ * Every word therefore sees its accesses in program order, so the emitted
+ * ranges (xpl_record_host_ranges) mean exactly what the individual accesses
+ * mean -- for programs whose individual accesses never straddle two
+ * allocations (every valid C/C++ object access; D28).
  */
 #ifndef XPL_HOST_H
 #define XPL_HOST_H
@@ -32,14 +41,15 @@ class xpl_host_tracer {
   xpl_host_tracer& operator=(const xpl_host_tracer&) = delete;
 
   /* One access of `size` bytes at p, kind = XPL_ACC_R / _W / _RW. */
-  inline void access(const void* p, uint32_t size, uint32_t kind) {
+  __attribute__((always_inline)) inline void access(const void* p, uint32_t size, uint32_t kind) {
     const uint64_t a = (uint64_t)p;
-    if (kind == kind_ && a == end_ && size <= kMaxRun - (end_ - beg_) &&
-        (kind != XPL_ACC_RW || ((a | size) & 3u) == 0)) {
-      end_ = a + size;
+    Run* r = cur_;
+    if (hit(r, a, size, kind)) return;  // the run used last
+    Run* n = r->next;                    // the run that followed it last time
+    if (n && hit(n, a, size, kind)) {
+      cur_ = n;
       return;
     }
-    if (kind == kind_ && kind != XPL_ACC_RW && a >= beg_ && a + size <= end_) return;  // repeat
     slow(a, size, kind);
   }
   template <class T>
@@ -59,33 +69,162 @@ class xpl_host_tracer {
   }
   /* Hand everything traced so far to the runtime (program order kept). */
   xpl_status flush() {
-    close_run();
-    xpl_status s = XPL_OK;
-    if (n_) s = xpl_record_host_ranges(ctx_, buf_, n_);
-    n_ = 0;
-    if (s != XPL_OK && status_ == XPL_OK) status_ = s;
+    for (;;) {  // close the open runs, oldest first
+      int o = -1;
+      for (int i = 0; i < kRuns; ++i)
+        if (run_[i].kind && (o < 0 || run_[i].seq < run_[o].seq)) o = i;
+      if (o < 0) break;
+      close(o);
+    }
+    drain();
     return status_;
   }
   xpl_status status() const { return status_; }
 
  private:
+  static const int kRuns = 8;
   static const uint64_t kMaxRun = 0xFFFFFFF0ull;
   static const size_t kBuf = 4096;
-  void close_run() {
-    if (kind_) buf_[n_++] = xpl_host_access{beg_, (uint32_t)(end_ - beg_), kind_};
-    kind_ = 0;
-    beg_ = end_ = 0;
+  struct Run {
+    uint64_t beg = 0, end = 0;  // bytes [beg, end)
+    uint64_t limit = 0;         // word-aligned start of the next open run above (or max)
+    uint64_t seq = 0;           // opening order
+    uint16_t kind = 0;          // 0 = slot free (16 bits: no aliasing with int/uint32 data)
+    uint16_t grew = 0;          // extended or repeated since opened
+    Run* next = nullptr;        // the run used after this one last time (a prediction)
+  };
+  /* The access joins run r (extension at its end, or a repeat inside it). */
+  static inline bool hit(Run* r, uint64_t a, uint32_t size, uint32_t kind) {
+    if (kind != r->kind) return false;
+    if (a == r->end) {
+      if (a + size > r->limit || a + size - r->beg > kMaxRun) return false;
+      if (kind == XPL_ACC_RW && ((a | size) & 3u)) return false;
+      r->end = a + size;
+      r->grew = 1;
+      return true;
+    }
+    if (kind != XPL_ACC_RW && a >= r->beg && a + size <= r->end) {  // repeat (R or W)
+      r->grew = 1;
+      return true;
+    }
+    return false;
   }
-  void slow(uint64_t a, uint32_t size, uint32_t kind) {
-    close_run();
-    if (n_ == kBuf) flush();
-    beg_ = a;
-    end_ = a + size;
-    kind_ = kind;
+  static uint64_t wlo(uint64_t a) { return a & ~3ull; }
+  static uint64_t whi(uint64_t e) { return (e + 3) & ~3ull; }
+
+  void drain() {
+    if (n_) {
+      const xpl_status s = xpl_record_host_ranges(ctx_, buf_, n_);
+      if (s != XPL_OK && status_ == XPL_OK) status_ = s;
+    }
+    n_ = 0;
   }
+  void close(int i) {
+    if (n_ == kBuf) drain();
+    buf_[n_++] = xpl_host_access{run_[i].beg, (uint32_t)(run_[i].end - run_[i].beg), run_[i].kind};
+    run_[i].kind = 0;
+    const uint64_t b = wlo(run_[i].beg);
+    for (int j = 0; j < kRuns; ++j) {
+      if (run_[j].next == &run_[i]) run_[j].next = nullptr;  // forget predictions into the slot
+      if (run_[j].kind && run_[j].limit == b) run_[j].limit = limit_of(j);  // it was the run above
+    }
+    run_[i].next = nullptr;
+  }
+  // word start of the closest open run above run i (the furthest i may grow)
+  uint64_t limit_of(int i) const {
+    uint64_t lim = ~0ull;
+    for (int j = 0; j < kRuns; ++j)
+      if (j != i && run_[j].kind && wlo(run_[j].beg) >= whi(run_[i].end) && wlo(run_[j].beg) < lim)
+        lim = wlo(run_[j].beg);
+    return lim;
+  }
+  bool overlaps(int i, uint64_t lo, uint64_t hi) const {  // word ranges intersect
+    return run_[i].kind && wlo(run_[i].beg) < hi && lo < whi(run_[i].end);
+  }
+  void touch(int k) {  // move mru_[k] to the front; learn the successor of the current run
+    const uint8_t i = mru_[k];
+    for (; k > 0; --k) mru_[k] = mru_[k - 1];
+    mru_[0] = i;
+    if (cur_ != &run_[i]) cur_->next = &run_[i];
+    cur_ = &run_[i];
+  }
+  __attribute__((noinline)) void slow(uint64_t a, uint32_t size, uint32_t kind) {
+    const uint64_t lo = wlo(a), hi = whi(a + size);
+    for (int k = 0; k < kRuns; ++k) {  // most recently used first: a run a starts in or right after
+      Run& r = run_[mru_[k]];
+      if (r.kind != kind || a < r.beg || a > r.end) continue;
+      if (kind != XPL_ACC_RW) {  // R / W: idempotent per word -> union
+        if (a + size <= r.end) {  // repeat inside the run (its words are no other run's)
+          r.grew = 1;
+          churn_ = 0;
+          touch(k);
+          return;
+        }
+        if (a + size <= r.limit && a + size - r.beg <= kMaxRun) {
+          r.end = a + size;
+          r.grew = 1;
+          churn_ = 0;
+          touch(k);
+          return;
+        }
+      } else if (a == r.end && ((a | size) & 3u) == 0 && a + size <= r.limit &&
+                 a + size - r.beg <= kMaxRun) {
+        r.end = a + size;
+        r.grew = 1;
+        churn_ = 0;
+        touch(k);
+        return;
+      }
+      break;
+    }
+    // close the runs this access overlaps (oldest first), then open a new one
+    for (;;) {
+      int o = -1;
+      for (int i = 0; i < kRuns; ++i)
+        if (overlaps(i, lo, hi) && (o < 0 || run_[i].seq < run_[o].seq)) o = i;
+      if (o < 0) break;
+      close(o);
+    }
+    // Scattered accesses (no run ever grows): emit them directly, re-trying
+    // runs every 64th access -- same records, without the slot churn.
+    if (churn_ >= 32 && (++tick_ & 63) != 0) {
+      if (n_ == kBuf) drain();
+      buf_[n_++] = xpl_host_access{a, size, kind};
+      return;
+    }
+    int slot = -1;
+    for (int i = 0; i < kRuns && slot < 0; ++i)
+      if (!run_[i].kind) slot = i;
+    if (slot < 0) {  // all used: close the oldest
+      slot = 0;
+      for (int i = 1; i < kRuns; ++i)
+        if (run_[i].seq < run_[slot].seq) slot = i;
+      churn_ = run_[slot].grew ? 0 : churn_ + 1;
+      close(slot);
+    }
+    Run& r = run_[slot];
+    r.beg = a;
+    r.end = a + size;
+    r.kind = (uint16_t)kind;
+    r.grew = 0;
+    r.seq = ++seq_;
+    r.limit = limit_of(slot);
+    for (int j = 0; j < kRuns; ++j)  // runs below the new one may now grow only up to it
+      if (j != slot && run_[j].kind && whi(run_[j].end) <= lo && run_[j].limit > lo) run_[j].limit = lo;
+    for (int k = 0; k < kRuns; ++k)
+      if (mru_[k] == slot) {
+        touch(k);
+        break;
+      }
+  }
+
   xpl_ctx* ctx_;
-  uint64_t beg_ = 0, end_ = 0;
-  uint32_t kind_ = 0;
+  Run run_[kRuns];
+  uint8_t mru_[kRuns] = {0, 1, 2, 3, 4, 5, 6, 7};  // run slots, most recently used first
+  Run* cur_ = &run_[0];                              // == &run_[mru_[0]]
+  uint64_t seq_ = 0;
+  uint32_t churn_ = 0;  // consecutive evictions of runs that never grew
+  uint32_t tick_ = 0;
   size_t n_ = 0;
   xpl_status status_ = XPL_OK;
   xpl_host_access buf_[kBuf];

@@ -32,7 +32,9 @@ class XplwRun(C.Structure):
 _w = xpl._work
 _w.xplw_hotspot.argtypes = [C.POINTER(XplwRun), C.POINTER(XplwArrays), i32, i32, i32]
 _w.xplw_backprop.argtypes = [C.POINTER(XplwRun), C.POINTER(XplwArrays), i32, i32]
-for f in ("xplw_hotspot", "xplw_backprop"):
+_w.xplw_bfs.argtypes = [C.POINTER(XplwRun), C.POINTER(XplwArrays), i32, i32, vp, C.POINTER(i32)]
+_w.xplw_nw.argtypes = [C.POINTER(XplwRun), C.POINTER(XplwArrays), i32, i32, vp]
+for f in ("xplw_hotspot", "xplw_backprop", "xplw_bfs", "xplw_nw"):
     getattr(_w, f).restype = i32
 
 
@@ -55,6 +57,17 @@ class Arena:
             self.arrays.bytes[i] = s[1]
             self.arrays.kind[i] = s[2]
         self.arrays.n = len(spec)
+
+    def view(self, name):
+        """numpy view (uint8) of one array by name (host) or torch view (device)."""
+        for a, sp in zip(self.addrs, self.spec):
+            if sp[0] == name:
+                if sp[3] == "host":
+                    o = a - self.host.data_ptr()
+                    return self.host.numpy()[o:o + sp[1]]
+                o = a - self.dev.data_ptr()
+                return self.dev[o:o + sp[1]]
+        raise KeyError(name)
 
     def host_views(self):
         """numpy views of the host arrays (for seeding inputs)."""
@@ -109,5 +122,31 @@ def hotspot(run: Run, arena: Arena, rows, cols, iters):
 
 def backprop(run: Run, arena: Arena, n_in, hid):
     st = _w.xplw_backprop(C.byref(run.r), C.byref(arena.arrays), n_in, hid)
+    run.check()
+    return st
+
+
+def bfs(run: Run, arena: Arena, n, deg, hook_counter):
+    """hook_counter: a torch int64 cuda tensor of 1 element (the kernels add to it)."""
+    lv = i32(0)
+    st = _w.xplw_bfs(C.byref(run.r), C.byref(arena.arrays), n, deg, hook_counter.data_ptr(), C.byref(lv))
+    run.check()
+    return lv.value
+
+
+def bfs_prepare(arena: Arena, n, deg, edges, resident: bool):
+    """Inputs of one bfs run: the graph in h_edges; for resident-data runs also the
+    device arrays as the program's H2D copies would have left them."""
+    import torch
+    from xplgen.rodinia import bfs_device_initial
+    arena.view("h_edges").view(np.int32)[:] = edges
+    if resident:
+        for name, arr in bfs_device_initial(n, deg, edges).items():
+            arena.view(name).copy_(torch.from_numpy(arr.view(np.uint8)), non_blocking=False)
+
+
+def nw(run: Run, arena: Arena, n, penalty, blosum):
+    """blosum: numpy int32 (24, 24), contiguous."""
+    st = _w.xplw_nw(C.byref(run.r), C.byref(arena.arrays), n, penalty, blosum.ctypes.data)
     run.check()
     return st

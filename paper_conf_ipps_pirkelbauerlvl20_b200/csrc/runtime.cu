@@ -114,6 +114,12 @@ struct xpl_ctx {
   uint64_t* d_stage = nullptr;
   std::vector<uint64_t> deferred;      // host records inside an open epoch (D20)
 
+  // merge pieces (records split to <= kPieceWords words)
+  uint64_t* h_pieces = nullptr;
+  uint64_t* d_pieces = nullptr;
+  size_t pieces_cap = 0;
+  cudaEvent_t pieces_ev = nullptr;
+
   // range descriptors
   RangeDesc* h_ranges = nullptr;
   RangeDesc* d_ranges = nullptr;
@@ -285,35 +291,51 @@ xpl_status ensure_first_w(xpl_ctx* c) {
   return XPL_OK;
 }
 
-// Apply all staged host records on the runtime stream, in order: runs of short
-// records go through the 3-pass merge, runs of pairwise-disjoint long ranges
-// through range_apply.
+// Apply all staged host records on the runtime stream, in order.  Records of
+// more than kRangeWords words cut the batch and go through range_apply (runs of
+// pairwise-disjoint ones share a launch); everything between them is one merge
+// segment, with records longer than kPieceWords split into consecutive pieces
+// (pieces of one record are disjoint, so program order is kept).
 xpl_status flush(xpl_ctx* c) {
   if (c->stage_n == 0) return XPL_OK;
   const size_t n = c->stage_n;
   uint64_t* h = c->h_stage[c->cur];
-  CK(cudaMemcpyAsync(c->d_stage, h, n * sizeof(uint64_t), cudaMemcpyHostToDevice, c->rs));
-  CK(cudaEventRecord(c->stage_ev[c->cur], c->rs));
-  if (c->stage_ranges == 0) {
+  size_t n_pieces = 0, n_long = 0;
+  for (size_t i = 0; i < n; ++i) {
+    const uint64_t nw = rec_nw(h[i]);
+    if (nw > kRangeWords) ++n_long;
+    else n_pieces += (nw + kPieceWords - 1) / kPieceWords;
+  }
+  if (n_long == 0 && n_pieces == n) {  // the common case: one merge segment as staged
+    CK(cudaMemcpyAsync(c->d_stage, h, n * sizeof(uint64_t), cudaMemcpyHostToDevice, c->rs));
+    CK(cudaEventRecord(c->stage_ev[c->cur], c->rs));
     xpl_status s = XPL_OK;
     if (c->stage_has_r && c->stage_has_w) s = ensure_first_w(c);
     if (s) return s;
     const int pi = prof_begin(c, XPL_K_MERGE, c->prof ? 8 * n + 2 * words_of(h, n) : 0);
     launch_merge(c->rs, c->d_stage, (uint32_t)n, c->stage_has_r, c->stage_has_w, c->d_first_w,
                  (uint32_t*)c->d_pool);
-    c->st.kernel_launches += 1 + c->stage_has_w + (c->stage_has_r && c->stage_has_w);
     prof_end(c, pi);
+    c->st.kernel_launches += 1 + c->stage_has_w + (c->stage_has_r && c->stage_has_w);
     c->st.merge_segments++;
   } else {
-    // Segment the batch.  Range descriptors of this flush go to h_ranges.
-    size_t n_long = 0;
-    for (size_t i = 0; i < n; ++i) n_long += rec_nw(h[i]) > kRangeWords;
+    // pieces go to a pinned buffer of their own, uploaded once
     xpl_status s = ensure_ranges(c, n_long);
     if (s) return s;
-    size_t nr_total = 0;
+    if (n_pieces > c->pieces_cap) {
+      CK(cudaStreamSynchronize(c->rs));
+      cudaFreeHost(c->h_pieces);
+      cudaFree(c->d_pieces);
+      c->pieces_cap = std::max<size_t>(n_pieces, 1 << 16);
+      CK(host_alloc(&c->h_pieces, c->pieces_cap));
+      CK(cudaMalloc(&c->d_pieces, sizeof(uint64_t) * c->pieces_cap));
+    } else {
+      CK(cudaEventSynchronize(c->pieces_ev));
+    }
     struct Seg { size_t start, n; bool range, has_r, has_w; };
     std::vector<Seg> segs;
     std::map<uint64_t, uint64_t> iv;  // disjointness of the open range segment
+    size_t nr_total = 0, np = 0;
     for (size_t i = 0; i < n; ++i) {
       const uint64_t r = h[i];
       const uint64_t g0 = rec_g0(r), nw = rec_nw(r);
@@ -340,15 +362,17 @@ xpl_status flush(xpl_ctx* c) {
         d.side = 0;
         segs.back().n++;
       } else {
-        if (segs.empty() || segs.back().range) segs.push_back({i, 0, false, false, false});
+        if (segs.empty() || segs.back().range) segs.push_back({np, 0, false, false, false});
         Seg& sg = segs.back();
-        sg.n++;
+        for (uint64_t o = 0; o < nw; o += kPieceWords) {
+          c->h_pieces[np++] = pack_rec(g0 + o, std::min<uint64_t>(kPieceWords, nw - o), acc);
+          sg.n++;
+        }
         if (acc & XPL_ACC_R) sg.has_r = true;
         if (acc & XPL_ACC_W) sg.has_w = true;
       }
     }
-    // vbase per segment, then one upload of all descriptors
-    for (const Seg& sg : segs) {
+    for (const Seg& sg : segs) {  // vbase per range segment
       if (!sg.range) continue;
       uint64_t v = 0;
       for (size_t i = sg.start; i < sg.start + sg.n; ++i) {
@@ -356,32 +380,35 @@ xpl_status flush(xpl_ctx* c) {
         v += ((c->h_ranges[i].g0 + c->h_ranges[i].nw - 1) >> 4) - (c->h_ranges[i].g0 >> 4) + 1;
       }
     }
-    CK(cudaMemcpyAsync(c->d_ranges, c->h_ranges, sizeof(RangeDesc) * nr_total,
-                       cudaMemcpyHostToDevice, c->rs));
+    if (np) CK(cudaMemcpyAsync(c->d_pieces, c->h_pieces, sizeof(uint64_t) * np, cudaMemcpyHostToDevice, c->rs));
+    CK(cudaEventRecord(c->pieces_ev, c->rs));
+    if (nr_total)
+      CK(cudaMemcpyAsync(c->d_ranges, c->h_ranges, sizeof(RangeDesc) * nr_total,
+                         cudaMemcpyHostToDevice, c->rs));
     CK(cudaEventRecord(c->ranges_ev, c->rs));
+    CK(cudaEventRecord(c->stage_ev[c->cur], c->rs));  // (staging itself was not uploaded)
     for (const Seg& sg : segs) {
       if (sg.range) {
-        uint64_t nvec = c->h_ranges[sg.start + sg.n - 1].vbase +
-                        ((c->h_ranges[sg.start + sg.n - 1].g0 + c->h_ranges[sg.start + sg.n - 1].nw - 1) >> 4) -
-                        (c->h_ranges[sg.start + sg.n - 1].g0 >> 4) + 1;
+        const RangeDesc& last = c->h_ranges[sg.start + sg.n - 1];
+        const uint64_t nvec = last.vbase + ((last.g0 + last.nw - 1) >> 4) - (last.g0 >> 4) + 1;
         uint64_t rw = 0;
         for (size_t i = sg.start; i < sg.start + sg.n; ++i) rw += c->h_ranges[i].nw;
         const int pi = prof_begin(c, XPL_K_RANGE, 2 * rw);
         launch_range(c->rs, c->d_ranges + sg.start, (uint32_t)sg.n, nvec, (uint32_t*)c->d_pool,
                      c->d_cmap, c->d_smap);
-        c->st.kernel_launches += 1;
         prof_end(c, pi);
+        c->st.kernel_launches += 1;
         c->st.range_segments++;
       } else {
         if (sg.has_r && sg.has_w) {
           s = ensure_first_w(c);
           if (s) return s;
         }
-        const int pi = prof_begin(c, XPL_K_MERGE, c->prof ? 8 * sg.n + 2 * words_of(h + sg.start, sg.n) : 0);
-        launch_merge(c->rs, c->d_stage + sg.start, (uint32_t)sg.n, sg.has_r, sg.has_w,
+        const int pi = prof_begin(c, XPL_K_MERGE, c->prof ? 8 * sg.n + 2 * words_of(c->h_pieces + sg.start, sg.n) : 0);
+        launch_merge(c->rs, c->d_pieces + sg.start, (uint32_t)sg.n, sg.has_r, sg.has_w,
                      c->d_first_w, (uint32_t*)c->d_pool);
-        c->st.kernel_launches += 1 + sg.has_w + (sg.has_r && sg.has_w);
         prof_end(c, pi);
+        c->st.kernel_launches += 1 + sg.has_w + (sg.has_r && sg.has_w);
         c->st.merge_segments++;
       }
     }
@@ -519,6 +546,8 @@ xpl_status xpl_init(const xpl_config* cfg, xpl_ctx** out) {
   CKI(cudaEventCreateWithFlags(&c->stage_ev[1], cudaEventDisableTiming));
   CKI(cudaEventCreateWithFlags(&c->table_ev, cudaEventDisableTiming));
   CKI(cudaEventCreateWithFlags(&c->ranges_ev, cudaEventDisableTiming));
+  CKI(cudaEventCreateWithFlags(&c->pieces_ev, cudaEventDisableTiming));
+  CKI(cudaEventRecord(c->pieces_ev, c->rs));
   CKI(cudaEventCreateWithFlags(&c->ev_begin, cudaEventDisableTiming));
   CKI(cudaEventRecord(c->stage_ev[0], c->rs));
   CKI(cudaEventRecord(c->stage_ev[1], c->rs));
@@ -567,7 +596,10 @@ xpl_status xpl_finalize(xpl_ctx* c) {
     cudaEventDestroy(r.a);
     cudaEventDestroy(r.b);
   }
-  for (cudaEvent_t e : {c->stage_ev[0], c->stage_ev[1], c->table_ev, c->ranges_ev, c->ev_begin})
+  cudaFreeHost(c->h_pieces);
+  cudaFree(c->d_pieces);
+  for (cudaEvent_t e : {c->stage_ev[0], c->stage_ev[1], c->table_ev, c->ranges_ev, c->ev_begin,
+                        c->pieces_ev})
     if (e) cudaEventDestroy(e);
   if (c->rs) cudaStreamDestroy(c->rs);
   delete c;

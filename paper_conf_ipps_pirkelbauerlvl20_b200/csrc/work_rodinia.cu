@@ -222,6 +222,117 @@ __global__ void __launch_bounds__(256) bp_adjust(const float* delta, const float
   }
 }
 
+
+// ---------------------------------------------------------------------------
+// bfs: Rodinia's two-kernel level-synchronous BFS (graph in CSR with uniform
+// degree).  Every hook call is counted per thread and added once per block.
+struct BfsNode {
+  int starting, no_of_edges;
+};
+
+template <bool I>
+__device__ __forceinline__ void count_hooks(unsigned long long* hc, unsigned c) {
+  if constexpr (I) {
+    __shared__ unsigned s_c;
+    if (threadIdx.x == 0) s_c = 0;
+    __syncthreads();
+    if (c) atomicAdd(&s_c, c);
+    __syncthreads();
+    if (threadIdx.x == 0 && s_c) atomicAdd(hc, (unsigned long long)s_c);
+  }
+}
+
+template <bool I>
+__global__ void __launch_bounds__(512) bfs_kernel1(BfsNode* nodes, int* edges, bool* mask,
+                                                   bool* updating, bool* visited, int* cost, int n,
+                                                   unsigned long long* hc) {
+  const int tid = blockIdx.x * blockDim.x + threadIdx.x;
+  unsigned c = 0;
+  if (tid < n) {
+    ++c;
+    if (RD<I>(mask[tid])) {
+      WR<I>(mask[tid]) = false;
+      c += 4;  // the write, the loop init and the first loop test (2 reads)
+      for (int i = RD<I>(nodes[tid].starting);
+           i < (RD<I>(nodes[tid].no_of_edges) + RD<I>(nodes[tid].starting)); i++) {
+        const int id = RD<I>(edges[i]);
+        c += 4;  // edges, visited, and the next loop test (2 reads)
+        if (!RD<I>(visited[id])) {
+          WR<I>(cost[id]) = RD<I>(cost[tid]) + 1;
+          WR<I>(updating[id]) = true;
+          c += 3;
+        }
+      }
+    }
+  }
+  count_hooks<I>(hc, c);
+}
+
+template <bool I>
+__global__ void __launch_bounds__(512) bfs_kernel2(bool* mask, bool* updating, bool* visited,
+                                                   bool* over, int n, unsigned long long* hc) {
+  const int tid = blockIdx.x * blockDim.x + threadIdx.x;
+  unsigned c = 0;
+  if (tid < n) {
+    ++c;
+    if (RD<I>(updating[tid])) {
+      WR<I>(mask[tid]) = true;
+      WR<I>(visited[tid]) = true;
+      WR<I>(*over) = true;
+      WR<I>(updating[tid]) = false;
+      c += 4;
+    }
+  }
+  count_hooks<I>(hc, c);
+}
+
+// ---------------------------------------------------------------------------
+// nw: Rodinia's Needleman-Wunsch, 16x16 tiles, one block-diagonal per launch.
+constexpr int NWB = 16;
+
+__host__ __device__ __forceinline__ int nw_max(int a, int b, int c) {
+  const int k = a <= b ? b : a;
+  return k <= c ? c : k;
+}
+
+template <bool I, bool UPPER>
+__global__ void __launch_bounds__(NWB) nw_kernel(int* ref, int* mat, int cols, int penalty, int i,
+                                                 int block_width) {
+  const int bx = blockIdx.x, tx = threadIdx.x;
+  const int b_index_x = UPPER ? bx : bx + block_width - i;
+  const int b_index_y = UPPER ? i - 1 - bx : block_width - bx - 1;
+  const int index = cols * NWB * b_index_y + NWB * b_index_x + tx + (cols + 1);
+  const int index_n = cols * NWB * b_index_y + NWB * b_index_x + tx + 1;
+  const int index_w = cols * NWB * b_index_y + NWB * b_index_x + cols;
+  const int index_nw = cols * NWB * b_index_y + NWB * b_index_x;
+  __shared__ int temp[NWB + 1][NWB + 1];
+  __shared__ int rf[NWB][NWB];
+  if (tx == 0) temp[tx][0] = RD<I>(mat[index_nw]);
+  for (int ty = 0; ty < NWB; ty++) rf[ty][tx] = RD<I>(ref[index + cols * ty]);
+  __syncthreads();
+  temp[tx + 1][0] = RD<I>(mat[index_w + cols * tx]);
+  __syncthreads();
+  temp[0][tx + 1] = RD<I>(mat[index_n]);
+  __syncthreads();
+  for (int m = 0; m < NWB; m++) {
+    if (tx <= m) {
+      const int t_x = tx + 1, t_y = m - tx + 1;
+      temp[t_y][t_x] = nw_max(temp[t_y - 1][t_x - 1] + rf[t_y - 1][t_x - 1],
+                              temp[t_y][t_x - 1] - penalty, temp[t_y - 1][t_x] - penalty);
+    }
+    __syncthreads();
+  }
+  for (int m = NWB - 2; m >= 0; m--) {
+    if (tx <= m) {
+      const int t_x = tx + NWB - m, t_y = NWB - tx;
+      temp[t_y][t_x] = nw_max(temp[t_y - 1][t_x - 1] + rf[t_y - 1][t_x - 1],
+                              temp[t_y][t_x - 1] - penalty, temp[t_y - 1][t_x] - penalty);
+    }
+    __syncthreads();
+  }
+  for (int ty = 0; ty < NWB; ty++) WR<I>(mat[index + ty * cols]) = temp[ty + 1][tx + 1];
+}
+
 }  // namespace
 
 extern "C" {
@@ -293,6 +404,196 @@ int xplw_backprop(xplw_run* run, const xplw_arrays* a, int in, int hid) {
   run->dev_accesses += (uint64_t)nblk * BP * BP * 5 + (uint64_t)BP * 4;
   app.copy(input_weights, input_hidden_cuda, nw * 4, XPL_COPY_D2H);
   app.copy(input_units, input_cuda, (in + 1) * 4, XPL_COPY_D2H);  // Table II: not modified
+  app.unreg(a);
+  app.diag();
+  return run->status;
+}
+
+
+int xplw_bfs(xplw_run* run, const xplw_arrays* a, int n, int deg, unsigned long long* hook_count,
+             int* levels) {
+  App app(run);
+  BfsNode* h_nodes = A<BfsNode>(a, 0);
+  int* h_edges = A<int>(a, 1);
+  bool *h_mask = A<bool>(a, 2), *h_updating = A<bool>(a, 3), *h_visited = A<bool>(a, 4);
+  int* h_cost = A<int>(a, 5);
+  bool* h_over = A<bool>(a, 6);
+  BfsNode* d_nodes = A<BfsNode>(a, 7);
+  int* d_edges = A<int>(a, 8);
+  bool *d_mask = A<bool>(a, 9), *d_updating = A<bool>(a, 10), *d_visited = A<bool>(a, 11);
+  int* d_cost = A<int>(a, 12);
+  bool* d_over = A<bool>(a, 13);
+  const uint64_t ne = (uint64_t)n * deg;
+  app.reg(a);
+  // read the graph "file": node records, masks, edges, costs (Rodinia bfs.cu order)
+  {
+    const auto t0 = std::chrono::steady_clock::now();
+    for (int i = 0; i < n; i++) {
+      if (app.tr) {
+        app.tr->write(h_nodes[i].starting) = i * deg;
+        app.tr->write(h_nodes[i].no_of_edges) = deg;
+        app.tr->write(h_mask[i]) = false;
+        app.tr->write(h_updating[i]) = false;
+        app.tr->write(h_visited[i]) = false;
+      } else {
+        h_nodes[i].starting = i * deg;
+        h_nodes[i].no_of_edges = deg;
+        h_mask[i] = h_updating[i] = h_visited[i] = false;
+      }
+    }
+    run->host_accesses += 5ull * n;
+    run->host_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  }
+  if (app.tr) {
+    app.tr->write(h_mask[0]) = true;
+    app.tr->write(h_visited[0]) = true;
+  } else {
+    h_mask[0] = h_visited[0] = true;
+  }
+  run->host_accesses += 2;
+  {  // the edge list is stored as read from the input; costs -1, source 0
+    const auto t0 = std::chrono::steady_clock::now();
+    for (uint64_t i = 0; i < ne; ++i) {
+      const int e = h_edges[i];  // (the input buffer; the traced store is the program's)
+      if (app.tr) app.tr->write(h_edges[i]) = e;
+    }
+    for (int i = 0; i < n; ++i) {
+      if (app.tr) app.tr->write(h_cost[i]) = -1;
+      else h_cost[i] = -1;
+    }
+    if (app.tr) app.tr->write(h_cost[0]) = 0;
+    else h_cost[0] = 0;
+    run->host_accesses += ne + n + 1;
+    run->host_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  }
+  app.copy(d_nodes, h_nodes, sizeof(BfsNode) * n, XPL_COPY_H2D);
+  app.copy(d_edges, h_edges, sizeof(int) * ne, XPL_COPY_H2D);
+  app.copy(d_mask, h_mask, n, XPL_COPY_H2D);
+  app.copy(d_updating, h_updating, n, XPL_COPY_H2D);
+  app.copy(d_visited, h_visited, n, XPL_COPY_H2D);
+  app.copy(d_cost, h_cost, sizeof(int) * n, XPL_COPY_H2D);
+  const int blocks = (n + 511) / 512;
+  int k = 0;
+  bool stop = false;
+  do {
+    if (app.tr) app.tr->write(*h_over) = false;
+    else *h_over = false;
+    run->host_accesses += 1;
+    app.copy(d_over, h_over, 1, XPL_COPY_H2D);
+    if (!run->do_copies)  // control data: the loop needs it even when bulk data is resident
+      app.ok_cuda(cudaMemcpyAsync(d_over, h_over, 1, cudaMemcpyHostToDevice, app.s));
+    app.begin();
+    if (app.on()) bfs_kernel1<true><<<blocks, 512, 0, app.s>>>(d_nodes, d_edges, d_mask, d_updating, d_visited, d_cost, n, hook_count);
+    else bfs_kernel1<false><<<blocks, 512, 0, app.s>>>(d_nodes, d_edges, d_mask, d_updating, d_visited, d_cost, n, hook_count);
+    app.end();
+    app.begin();
+    if (app.on()) bfs_kernel2<true><<<blocks, 512, 0, app.s>>>(d_mask, d_updating, d_visited, d_over, n, hook_count);
+    else bfs_kernel2<false><<<blocks, 512, 0, app.s>>>(d_mask, d_updating, d_visited, d_over, n, hook_count);
+    app.end();
+    app.copy(h_over, d_over, 1, XPL_COPY_D2H);
+    if (!run->do_copies) {  // the control flow needs the flag even with resident data
+      app.ok_cuda(cudaMemcpyAsync(h_over, d_over, 1, cudaMemcpyDeviceToHost, app.s));
+      app.ok_cuda(cudaStreamSynchronize(app.s));
+    }
+    stop = app.tr ? app.tr->read(*h_over) : *h_over;
+    run->host_accesses += 1;
+    ++k;
+    if (run->diag_each) app.diag();
+  } while (stop && k < n + 1 && !run->status);  // (a BFS has at most n levels)
+  *levels = k;
+  app.copy(h_cost, d_cost, sizeof(int) * n, XPL_COPY_D2H);
+  app.read_loop(h_cost, n);  // write the result file
+  app.unreg(a);
+  app.diag();
+  return run->status;
+}
+
+int xplw_nw(xplw_run* run, const xplw_arrays* a, int n, int penalty, const int* blosum) {
+  App app(run);
+  const int cols = n + 1, rows = n + 1;
+  int *in = A<int>(a, 0), *refh = A<int>(a, 1), *out = A<int>(a, 2);
+  int *ref_d = A<int>(a, 3), *mat_d = A<int>(a, 4);
+  app.reg(a);
+  // the sequences (row / column 0) are the input; the substitution matrix from them
+  {
+    const auto t0 = std::chrono::steady_clock::now();
+    if (app.tr) {
+      for (int i = 1; i < rows; i++)
+        for (int j = 1; j < cols; j++) {
+          const int x = app.tr->read(in[i * cols]), y = app.tr->read(in[j]);
+          app.tr->write(refh[i * cols + j]) = blosum[x * 24 + y];
+        }
+    } else {
+      for (int i = 1; i < rows; i++)
+        for (int j = 1; j < cols; j++) refh[i * cols + j] = blosum[in[i * cols] * 24 + in[j]];
+    }
+    run->host_accesses += 3ull * (rows - 1) * (cols - 1);
+    for (int i = 1; i < rows; i++) {
+      if (app.tr) app.tr->write(in[i * cols]) = -i * penalty;
+      else in[i * cols] = -i * penalty;
+    }
+    for (int j = 1; j < cols; j++) {
+      if (app.tr) app.tr->write(in[j]) = -j * penalty;
+      else in[j] = -j * penalty;
+    }
+    run->host_accesses += (uint64_t)(rows - 1) + (cols - 1);
+    run->host_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  }
+  app.copy(ref_d, refh, sizeof(int) * rows * cols, XPL_COPY_H2D);
+  app.copy(mat_d, in, sizeof(int) * rows * cols, XPL_COPY_H2D);
+  const int bw = (cols - 1) / NWB;
+  for (int i = 1; i <= bw; i++) {
+    app.begin();
+    if (app.on()) nw_kernel<true, true><<<i, NWB, 0, app.s>>>(ref_d, mat_d, cols, penalty, i, bw);
+    else nw_kernel<false, true><<<i, NWB, 0, app.s>>>(ref_d, mat_d, cols, penalty, i, bw);
+    app.end();
+    run->dev_accesses += (uint64_t)i * (1 + 2 * NWB * NWB + 2 * NWB);
+  }
+  for (int i = bw - 1; i >= 1; i--) {
+    app.begin();
+    if (app.on()) nw_kernel<true, false><<<i, NWB, 0, app.s>>>(ref_d, mat_d, cols, penalty, i, bw);
+    else nw_kernel<false, false><<<i, NWB, 0, app.s>>>(ref_d, mat_d, cols, penalty, i, bw);
+    app.end();
+    run->dev_accesses += (uint64_t)i * (1 + 2 * NWB * NWB + 2 * NWB);
+  }
+  app.copy(out, mat_d, sizeof(int) * rows * cols, XPL_COPY_D2H);
+  // traceback (Rodinia nw): from the bottom-right corner towards (0, 0)
+  {
+    const auto t0 = std::chrono::steady_clock::now();
+    const int LIMIT = -999;
+    auto R = [&](int* p) -> int {
+      run->host_accesses += 1;
+      return app.tr ? app.tr->read(*p) : *p;
+    };
+    app.sink += R(&out[(rows - 2) * cols + rows - 2]);  // the score printed first
+    for (int i = rows - 2, j = rows - 2; i >= 0 && j >= 0;) {
+      if (i == 0 && j == 0) break;
+      int nw, w, nn;
+      if (i > 0 && j > 0) {
+        nw = R(&out[(i - 1) * cols + j - 1]);
+        w = R(&out[i * cols + j - 1]);
+        nn = R(&out[(i - 1) * cols + j]);
+      } else if (i == 0) {
+        nw = nn = LIMIT;
+        w = R(&out[i * cols + j - 1]);
+      } else {
+        nw = w = LIMIT;
+        nn = R(&out[(i - 1) * cols + j]);
+      }
+      const int new_nw = nw + R(&refh[i * cols + j]);
+      const int new_w = w - penalty, new_n = nn - penalty;
+      int tb = nw_max(new_nw, new_w, new_n);
+      if (tb == new_nw) tb = nw;
+      if (tb == new_w) tb = w;
+      if (tb == new_n) tb = nn;
+      if (tb == nw) { i--; j--; continue; }
+      else if (tb == w) { j--; continue; }
+      else if (tb == nn) { i--; continue; }
+      else break;
+    }
+    app.flush();
+    run->host_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  }
   app.unreg(a);
   app.diag();
   return run->status;

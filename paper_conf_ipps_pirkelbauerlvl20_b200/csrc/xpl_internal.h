@@ -27,8 +27,11 @@ __host__ __device__ inline uint64_t rec_g0(uint64_t r) { return r & kG0Mask; }
 __host__ __device__ inline uint64_t rec_nw(uint64_t r) { return ((r >> kG0Bits) & (kMaxRecWords - 1)) + 1; }
 __host__ __device__ inline uint32_t rec_acc(uint64_t r) { return (uint32_t)(r >> 62); }
 
-// Records of more than this many words are "ranges" and go through range_apply.
-constexpr uint64_t kRangeWords = 64;
+// Records of more than kBigRange words are "ranges" and go through range_apply
+// (2 B/word, cutting the batch into segments); shorter ones are merged, split
+// into pieces of at most kPieceWords (one thread each, program order kept).
+constexpr uint64_t kRangeWords = 65536;  // (kBigRange)
+constexpr uint64_t kPieceWords = 256;
 
 // A range for the vectorised range kernels (host transfers, D2D/memset).
 struct RangeDesc {

@@ -61,6 +61,25 @@ int xplw_hotspot(xplw_run* run, const xplw_arrays* a, int rows, int cols, int it
  *         10 input_prev_weights_cuda (DEVICE). */
 int xplw_backprop(xplw_run* run, const xplw_arrays* a, int in, int hid);
 
+/* Rodinia bfs: n nodes with `deg` out-edges each (node i: edges [deg*i, deg*i+deg)),
+ * level-synchronous from node 0, two kernels per level, `over` flag round trip.
+ * arrays: 0 h_nodes, 1 h_edges, 2 h_mask, 3 h_updating, 4 h_visited, 5 h_cost,
+ *         6 h_over (HOST), 7 d_nodes, 8 d_edges, 9 d_mask, 10 d_updating,
+ *         11 d_visited, 12 d_cost, 13 d_over (DEVICE).  h_edges holds the graph
+ *         (input).  hook_count: device u64 the instrumented kernels add their
+ *         hook calls to (data-dependent).  Returns the number of levels in *levels. */
+int xplw_bfs(xplw_run* run, const xplw_arrays* a, int n, int deg, unsigned long long* hook_count,
+             int* levels);
+
+/* Rodinia nw (Needleman-Wunsch): (n+1) x (n+1) ints, 16 x 16 tiles, 2*(n/16)-1
+ * block-diagonal kernels, host traceback over the D2H result.
+ * arrays: 0 input_itemsets, 1 referrence, 2 output_itemsets (HOST), 3 referrence_cuda,
+ *         4 matrix_cuda (DEVICE).  blosum: 24 x 24 substitution scores (host, not
+ * traced).  input_itemsets row/column 0 hold the sequences (1..23) on entry;
+ * output_itemsets holds the expected DP result (the traceback reads it when
+ * do_copies == 0, i.e. when the D2H is not performed). */
+int xplw_nw(xplw_run* run, const xplw_arrays* a, int n, int penalty, const int* blosum);
+
 #ifdef __cplusplus
 }
 #endif

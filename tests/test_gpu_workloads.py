@@ -67,6 +67,49 @@ def test_backprop(env, n_in):
         assert rows[5]["flags"] & 8
 
 
+@pytest.mark.parametrize("n,resident", [(1000, False), (5000, True), (70000, False)])
+def test_bfs(env, n, resident):
+    torch, apps, xpl = env
+    from xplgen import rodinia
+    deg = 6
+    spec = rodinia.bfs_spec(n, deg)
+    ar = apps.Arena(spec)
+    edges = rodinia.bfs_graph(n, deg, 0x58504C02 + n)
+    apps.bfs_prepare(ar, n, deg, edges, resident)
+    s = torch.cuda.Stream()
+    params = (50, 0, 64)
+    hc = torch.zeros(1, dtype=torch.int64, device="cuda")
+    with xpl.Context(pool_words=1 << 24) as ctx:
+        run = apps.Run(ctx, s.cuda_stream, do_copies=not resident, diag_each=True, params=params)
+        levels = apps.bfs(run, ar, n, deg, hc)
+        got = run.reports()
+    ops, lv, hooks = rodinia.bfs_trace(ar.addrs, spec, n, deg, edges, True, params)
+    assert levels == lv
+    assert int(hc.item()) == hooks
+    compare(got, oracle_run(ops))
+
+
+@pytest.mark.parametrize("n,resident", [(64, False), (256, True), (512, False)])
+def test_nw(env, n, resident):
+    torch, apps, xpl = env
+    from xplgen import rodinia
+    spec = rodinia.nw_spec(n)
+    ar = apps.Arena(spec)
+    inp = rodinia.nw_inputs(n, 10, 0x58504C03 + n)
+    rodinia.nw_fill_host(ar.host_views(), spec, inp, n)
+    s = torch.cuda.Stream()
+    params = (50, 1024, 16)
+    with xpl.Context(pool_words=1 << 24) as ctx:
+        run = apps.Run(ctx, s.cuda_stream, do_copies=not resident, params=params)
+        apps.nw(run, ar, n, 10, inp["blosum"])
+        got = run.reports()
+        assert run.r.dev_accesses == rodinia.nw_accesses(n)
+    compare(got, oracle_run(rodinia.nw_trace(ar.addrs, spec, n, 10, inp, params)))
+    if not resident:  # the kernels computed the DP the twin expects
+        out = ar.view("output_itemsets").view(np.int32).reshape(n + 1, n + 1)
+        assert np.array_equal(out[1:, 1:], inp["dp"][1:, 1:])
+
+
 def test_twin_runs_without_xpl(env):
     torch, apps, xpl = env
     from xplgen import rodinia

@@ -159,3 +159,248 @@ def fill_inputs(name, host_arrays, seed):
     for t in host_arrays:
         a = t.numpy() if hasattr(t, "numpy") else t
         a.view(np.float32)[:] = rng.random(a.size // 4, dtype=np.float32)
+
+
+# ---------------------------------------------------------------------------
+# bfs (Rodinia shape; 1M nodes x out-degree 6 in the benchmark -- Rodinia's graph
+# size, not the paper's)
+def bfs_spec(n, deg):
+    return [("h_nodes", 8 * n, HOST, "host"), ("h_edges", 4 * n * deg, HOST, "host"),
+            ("h_mask", n, HOST, "host"), ("h_updating", n, HOST, "host"),
+            ("h_visited", n, HOST, "host"), ("h_cost", 4 * n, HOST, "host"), ("h_over", 1, HOST, "host"),
+            ("d_nodes", 8 * n, DEVICE, "dev"), ("d_edges", 4 * n * deg, DEVICE, "dev"),
+            ("d_mask", n, DEVICE, "dev"), ("d_updating", n, DEVICE, "dev"),
+            ("d_visited", n, DEVICE, "dev"), ("d_cost", 4 * n, DEVICE, "dev"), ("d_over", 1, DEVICE, "dev")]
+
+
+def bfs_graph(n, deg, seed):
+    """Uniformly random out-neighbours (seeded)."""
+    return np.random.default_rng(seed).integers(0, n, size=n * deg, dtype=np.int64).astype(np.int32)
+
+
+def bfs_device_initial(n, deg, edges):
+    """The device arrays right after the program's H2D copies (resident-data runs)."""
+    nodes = np.zeros(2 * n, np.int32)
+    nodes[0::2] = np.arange(n, dtype=np.int32) * deg
+    nodes[1::2] = deg
+    mask = np.zeros(n, np.uint8)
+    mask[0] = 1
+    visited = mask.copy()
+    cost = np.full(n, -1, np.int32)
+    cost[0] = 0
+    return {"d_nodes": nodes, "d_edges": edges, "d_mask": mask, "d_updating": np.zeros(n, np.uint8),
+            "d_visited": visited, "d_cost": cost}
+
+
+def bfs_trace(addrs, spec, n, deg, edges, diag_each, params):
+    """The CPU twin of xplw_bfs: returns (ops, levels, device hook calls)."""
+    A = dict(zip([s[0] for s in spec], addrs))
+    u64 = lambda x: np.asarray(x, dtype=np.uint64)
+    ops = [("REG", a, s[1], s[2]) for a, s in zip(addrs, spec)]
+    i = np.arange(n, dtype=np.uint64)
+    # per node: starting, no_of_edges, mask, updating, visited (program order)
+    a = np.stack([A["h_nodes"] + 8 * i, A["h_nodes"] + 8 * i + 4, A["h_mask"] + i,
+                  A["h_updating"] + i, A["h_visited"] + i], axis=1).reshape(-1)
+    sz = np.tile(np.array([4, 4, 1, 1, 1], np.uint32), n)
+    ops.append(batch("HB", a, sz, W))
+    ops.append(batch("HB", [A["h_mask"], A["h_visited"]], 1, W))
+    ops.append(batch("HB", A["h_edges"] + 4 * u64(np.arange(n * deg)), 4, W))
+    ops.append(batch("HB", A["h_cost"] + 4 * i, 4, W))
+    ops.append(batch("HB", [A["h_cost"]], 4, W))
+    for name, nb in (("nodes", 8 * n), ("edges", 4 * n * deg), ("mask", n), ("updating", n),
+                     ("visited", n), ("cost", 4 * n)):
+        ops.append(("X", H2D, A["d_" + name], A["h_" + name], nb))
+    mask = np.zeros(n, bool)
+    mask[0] = True
+    visited = mask.copy()
+    updating = np.zeros(n, bool)
+    e2 = edges.reshape(n, deg).astype(np.int64)
+    levels, hooks = 0, 0
+    while True:
+        ops.append(batch("HB", [A["h_over"]], 1, W))
+        ops.append(("X", H2D, A["d_over"], A["h_over"], 1))
+        # kernel 1
+        F = np.nonzero(mask)[0]
+        ids = e2[F]                                   # |F| x deg
+        unvis = ~visited[ids]
+        parent = np.repeat(F, deg).reshape(len(F), deg)
+        ev_a = [A["d_mask"] + i, A["d_mask"] + u64(F), A["d_nodes"] + 8 * u64(F),
+                A["d_nodes"] + 8 * u64(F) + 4,
+                A["d_edges"] + 4 * u64((F[:, None] * deg + np.arange(deg)).reshape(-1)),
+                A["d_visited"] + u64(ids.reshape(-1)), A["d_cost"] + 4 * u64(parent[unvis]),
+                A["d_cost"] + 4 * u64(ids[unvis]), A["d_updating"] + u64(ids[unvis])]
+        ev_s = [1, 1, 4, 4, 4, 1, 4, 4, 1]
+        ev_k = [R, W, R, R, R, R, R, W, W]
+        ops += [("KB",), ("DB", np.concatenate(ev_a).astype(np.uint64),
+                         np.concatenate([np.full(len(x), s, np.uint32) for x, s in zip(ev_a, ev_s)]),
+                         np.concatenate([np.full(len(x), k, np.uint8) for x, k in zip(ev_a, ev_k)])), ("KE",)]
+        hooks += n + len(F) * (4 + 4 * deg) + 3 * int(unvis.sum())
+        mask[F] = False
+        updating[ids[unvis]] = True
+        # kernel 2
+        U = np.nonzero(updating)[0]
+        ev_a = [A["d_updating"] + i, A["d_mask"] + u64(U), A["d_visited"] + u64(U),
+                np.full(len(U), A["d_over"], np.uint64), A["d_updating"] + u64(U)]
+        ev_k = [R, W, W, W, W]
+        ops += [("KB",), ("DB", np.concatenate(ev_a).astype(np.uint64),
+                         np.concatenate([np.ones(len(x), np.uint32) for x in ev_a]),
+                         np.concatenate([np.full(len(x), k, np.uint8) for x, k in zip(ev_a, ev_k)])), ("KE",)]
+        hooks += n + 4 * len(U)
+        mask[U] = True
+        visited[U] = True
+        updating[U] = False
+        ops.append(("X", D2H, A["h_over"], A["d_over"], 1))
+        ops.append(batch("HB", [A["h_over"]], 1, R))
+        levels += 1
+        if diag_each:
+            ops.append(("DIAG",) + params + (1, ()))
+        if len(U) == 0:
+            break
+    ops.append(("X", D2H, A["h_cost"], A["d_cost"], 4 * n))
+    ops.append(batch("HB", A["h_cost"] + 4 * i, 4, R))
+    ops += [("FREE", x) for x in addrs]
+    ops.append(("DIAG",) + params + (1, ()))
+    return ops, levels, hooks
+
+
+# ---------------------------------------------------------------------------
+# nw (Needleman-Wunsch, Rodinia shape; 2048 x 2048 in the benchmark)
+NWB = 16
+
+
+def nw_spec(n):
+    m = 4 * (n + 1) * (n + 1)
+    return [("input_itemsets", m, HOST, "host"), ("referrence", m, HOST, "host"),
+            ("output_itemsets", m, HOST, "host"), ("referrence_cuda", m, DEVICE, "dev"),
+            ("matrix_cuda", m, DEVICE, "dev")]
+
+
+def nw_inputs(n, penalty, seed):
+    """Sequences (1..23), a symmetric 24x24 substitution table, and the exact DP
+    result the kernels compute (for the traceback of resident-data runs)."""
+    rng = np.random.default_rng(seed)
+    cols = n + 1
+    a = rng.integers(1, 24, size=n).astype(np.int32)   # column 0, rows 1..n
+    b = rng.integers(1, 24, size=n).astype(np.int32)   # row 0, cols 1..n
+    t = rng.integers(-4, 12, size=(24, 24)).astype(np.int32)
+    blosum = np.triu(t) + np.triu(t, 1).T
+    ref = np.zeros((cols, cols), np.int64)
+    ref[1:, 1:] = blosum[a[:, None], b[None, :]]
+    M = np.zeros((cols, cols), np.int64)
+    M[:, 0] = -np.arange(cols) * penalty
+    M[0, :] = -np.arange(cols) * penalty
+    for d in range(2, 2 * n + 1):  # anti-diagonals i + j = d
+        i = np.arange(max(1, d - n), min(n, d - 1) + 1)
+        j = d - i
+        M[i, j] = np.maximum(np.maximum(M[i - 1, j - 1] + ref[i, j], M[i, j - 1] - penalty), M[i - 1, j] - penalty)
+    return {"a": a, "b": b, "blosum": blosum.astype(np.int32), "ref": ref.astype(np.int32),
+            "dp": M.astype(np.int32)}
+
+
+def nw_traceback(dp, ref, n, penalty):
+    """The host traceback of Rodinia nw: the (array, index) reads in order."""
+    cols = n + 1
+    rows = n + 1
+    LIMIT = -999
+    reads = [("out", (rows - 2) * cols + rows - 2)]
+    i = j = rows - 2
+    while i >= 0 and j >= 0:
+        if i == 0 and j == 0:
+            break
+        if i > 0 and j > 0:
+            nw, w, nn = dp[i - 1, j - 1], dp[i, j - 1], dp[i - 1, j]
+            reads += [("out", (i - 1) * cols + j - 1), ("out", i * cols + j - 1), ("out", (i - 1) * cols + j)]
+        elif i == 0:
+            nw = nn = LIMIT
+            w = dp[i, j - 1]
+            reads.append(("out", i * cols + j - 1))
+        else:
+            nw = w = LIMIT
+            nn = dp[i - 1, j]
+            reads.append(("out", (i - 1) * cols + j))
+        new_nw = nw + ref[i, j]
+        reads.append(("ref", i * cols + j))
+        new_w, new_n = w - penalty, nn - penalty
+        tb = max(new_nw, new_w, new_n)
+        if tb == new_nw:
+            tb = nw
+        if tb == new_w:
+            tb = w
+        if tb == new_n:
+            tb = nn
+        if tb == nw:
+            i -= 1
+            j -= 1
+        elif tb == w:
+            j -= 1
+        elif tb == nn:
+            i -= 1
+        else:
+            break
+    return reads
+
+
+def nw_accesses(n):
+    bw = n // NWB
+    return sum(i for i in range(1, bw + 1)) * 545 + sum(i for i in range(1, bw)) * 545
+
+
+def nw_trace(addrs, spec, n, penalty, inp, params):
+    A = dict(zip([s[0] for s in spec], addrs))
+    cols = n + 1
+    u64 = lambda x: np.asarray(x, dtype=np.uint64)
+    ops = [("REG", a, s[1], s[2]) for a, s in zip(addrs, spec)]
+    ii = np.repeat(np.arange(1, cols, dtype=np.int64), n)
+    jj = np.tile(np.arange(1, cols, dtype=np.int64), n)
+    a = np.stack([A["input_itemsets"] + 4 * u64(ii * cols), A["input_itemsets"] + 4 * u64(jj),
+                  A["referrence"] + 4 * u64(ii * cols + jj)], axis=1).reshape(-1)
+    k = np.tile(np.array([R, R, W], np.uint8), n * n)
+    ops.append(("HB", a.astype(np.uint64), np.full(a.size, 4, np.uint32), k))
+    ops.append(batch("HB", A["input_itemsets"] + 4 * u64(np.arange(1, cols) * cols), 4, W))
+    ops.append(batch("HB", A["input_itemsets"] + 4 * u64(np.arange(1, cols)), 4, W))
+    ops.append(("X", H2D, A["referrence_cuda"], A["referrence"], 4 * cols * cols))
+    ops.append(("X", H2D, A["matrix_cuda"], A["input_itemsets"], 4 * cols * cols))
+    bw = n // NWB
+    tx = np.arange(NWB, dtype=np.int64)
+    ty = np.arange(NWB, dtype=np.int64)
+
+    def tiles(bx, by):
+        index = cols * NWB * by + NWB * bx + (cols + 1)
+        index_n = cols * NWB * by + NWB * bx + 1
+        index_w = cols * NWB * by + NWB * bx + cols
+        index_nw = cols * NWB * by + NWB * bx
+        grid = (ty[:, None] * cols + tx[None, :]).reshape(-1)
+        rd = np.concatenate([A["matrix_cuda"] + 4 * u64(index_nw[:, None]),
+                             A["referrence_cuda"] + 4 * u64(index[:, None] + grid[None, :]),
+                             A["matrix_cuda"] + 4 * u64(index_w[:, None] + cols * tx[None, :]),
+                             A["matrix_cuda"] + 4 * u64(index_n[:, None] + tx[None, :])], axis=1).reshape(-1)
+        wr = (A["matrix_cuda"] + 4 * u64(index[:, None] + grid[None, :])).reshape(-1)
+        return ("DB", np.concatenate([rd, wr]).astype(np.uint64), np.full(rd.size + wr.size, 4, np.uint32),
+                np.concatenate([np.full(rd.size, R, np.uint8), np.full(wr.size, W, np.uint8)]))
+
+    for i in range(1, bw + 1):
+        bx = np.arange(i, dtype=np.int64)
+        ops += [("KB",), tiles(bx, i - 1 - bx), ("KE",)]
+    for i in range(bw - 1, 0, -1):
+        bx = np.arange(i, dtype=np.int64)
+        ops += [("KB",), tiles(bx + bw - i, bw - bx - 1), ("KE",)]
+    ops.append(("X", D2H, A["output_itemsets"], A["matrix_cuda"], 4 * cols * cols))
+    tb = nw_traceback(inp["dp"], inp["ref"], n, penalty)
+    base = {"out": A["output_itemsets"], "ref": A["referrence"]}
+    ops.append(batch("HB", [base[w] + 4 * x for w, x in tb], 4, R))
+    ops += [("FREE", x) for x in addrs]
+    ops.append(("DIAG",) + params + (1, ()))
+    return ops
+
+
+def nw_fill_host(arena_views, spec, inp, n):
+    """Reset the program's host inputs before a run: sequences in row/col 0 of
+    input_itemsets, the DP result in output_itemsets (resident-data runs)."""
+    cols = n + 1
+    names = [s[0] for s in spec if s[3] == "host"]
+    v = dict(zip(names, arena_views))
+    inn = v["input_itemsets"].view(np.int32).reshape(cols, cols)
+    inn[:] = 0
+    inn[1:, 0] = inp["a"]
+    inn[0, 1:] = inp["b"]
+    v["output_itemsets"].view(np.int32).reshape(cols, cols)[:] = inp["dp"]
