@@ -34,7 +34,11 @@ _w.xplw_hotspot.argtypes = [C.POINTER(XplwRun), C.POINTER(XplwArrays), i32, i32,
 _w.xplw_backprop.argtypes = [C.POINTER(XplwRun), C.POINTER(XplwArrays), i32, i32]
 _w.xplw_bfs.argtypes = [C.POINTER(XplwRun), C.POINTER(XplwArrays), i32, i32, vp, C.POINTER(i32)]
 _w.xplw_nw.argtypes = [C.POINTER(XplwRun), C.POINTER(XplwArrays), i32, i32, vp]
-for f in ("xplw_hotspot", "xplw_backprop", "xplw_bfs", "xplw_nw"):
+_w.xplw_sw.argtypes = [C.POINTER(XplwRun), C.POINTER(XplwArrays), i32, i32, i32, i32, i32, C.POINTER(i32)]
+_w.xplw_alloc_managed.argtypes = [u64]
+_w.xplw_alloc_managed.restype = vp
+_w.xplw_free_managed.argtypes = [vp]
+for f in ("xplw_hotspot", "xplw_backprop", "xplw_bfs", "xplw_nw", "xplw_sw", "xplw_free_managed"):
     getattr(_w, f).restype = i32
 
 
@@ -44,12 +48,20 @@ class Arena:
     def __init__(self, spec):
         import torch
         from xplgen.rodinia import arena_sizes, layout
-        d, h = arena_sizes(spec)
-        self.dev = torch.empty(d + 4096, dtype=torch.uint8, device="cuda")
-        self.host = torch.empty(h + 4096, dtype=torch.uint8).pin_memory()
+        sz = arena_sizes(spec)
+        self.dev = torch.empty(sz["dev"] + 4096, dtype=torch.uint8, device="cuda")
+        self.host = torch.empty(sz["host"] + 4096, dtype=torch.uint8).pin_memory()
+        self.managed = None
+        self.managed_bytes = sz["managed"]
+        mb = 0
+        if sz["managed"]:
+            self.managed = _w.xplw_alloc_managed(sz["managed"] + 4096)
+            if not self.managed:
+                raise MemoryError("cudaMallocManaged failed")
+            mb = (self.managed + 4095) // 4096 * 4096
         db = (self.dev.data_ptr() + 4095) // 4096 * 4096
         hb = (self.host.data_ptr() + 4095) // 4096 * 4096
-        self.addrs, _, _ = layout(spec, db, hb)
+        self.addrs, _, _ = layout(spec, db, hb, mb)
         self.spec = spec
         self.arrays = XplwArrays()
         for i, (a, s) in enumerate(zip(self.addrs, spec)):
@@ -58,10 +70,17 @@ class Arena:
             self.arrays.kind[i] = s[2]
         self.arrays.n = len(spec)
 
+    def __del__(self):
+        if getattr(self, "managed", None):
+            _w.xplw_free_managed(self.managed)
+            self.managed = None
+
     def view(self, name):
-        """numpy view (uint8) of one array by name (host) or torch view (device)."""
+        """numpy view (uint8) of one array by name (host, managed) or torch view (device)."""
         for a, sp in zip(self.addrs, self.spec):
             if sp[0] == name:
+                if sp[3] == "managed":
+                    return np.ctypeslib.as_array((C.c_uint8 * sp[1]).from_address(a))
                 if sp[3] == "host":
                     o = a - self.host.data_ptr()
                     return self.host.numpy()[o:o + sp[1]]
@@ -150,3 +169,17 @@ def nw(run: Run, arena: Arena, n, penalty, blosum):
     st = _w.xplw_nw(C.byref(run.r), C.byref(arena.arrays), n, penalty, blosum.ctypes.data)
     run.check()
     return st
+
+
+def sw(run: Run, arena: Arena, n, m, per_diagonal, tb_every, diag_every, inp):
+    """Smith-Waterman (managed arrays a, b, H); inp = xplgen.sw.sw_inputs().
+    Returns the traceback length."""
+    import torch
+    arena.view("a").view(np.int32)[:] = inp["a"]
+    arena.view("b").view(np.int32)[:] = inp["b"]
+    torch.cuda.synchronize()
+    tb = i32(0)
+    _w.xplw_sw(C.byref(run.r), C.byref(arena.arrays), n, m, int(per_diagonal), tb_every, diag_every,
+               C.byref(tb))
+    run.check()
+    return tb.value

@@ -80,6 +80,21 @@ int xplw_bfs(xplw_run* run, const xplw_arrays* a, int n, int deg, unsigned long 
  * do_copies == 0, i.e. when the D2H is not performed). */
 int xplw_nw(xplw_run* run, const xplw_arrays* a, int n, int penalty, const int* blosum);
 
+/* Smith-Waterman (Fig. 7/8 P:L341-349; cfg1 SW-128 and cfg3 SW-16K of SURVEY §8(d)):
+ * managed a[n], b[m], H[(n+1) x (m+1)] ints; the CPU writes a, b and zero-fills H;
+ * GPU epochs fill H (score +3 match / -3 mismatch, gap 2, floor 0):
+ *   per_diagonal = 0: ONE launch of one CTA (n <= 1024 threads) sweeping all
+ *                     anti-diagonals with __syncthreads (cfg1);
+ *   per_diagonal = 1: one launch per anti-diagonal d = 2 .. n+m (cfg3); every
+ *                     `tb_every` diagonals a host segment reads the finished diagonal,
+ *                     every `diag_every` diagonals a diagnose (0 = never);
+ * then the CPU scans H for the maximum and traces back from it; with
+ * per_diagonal = 0 a final GPU epoch re-zeroes the interior (the next query).
+ * arrays: 0 a, 1 b, 2 H (MANAGED).  a, b hold the sequences (0..3) on entry.
+ * Returns the traceback length in *tb_len. */
+int xplw_sw(xplw_run* run, const xplw_arrays* a, int n, int m, int per_diagonal, int tb_every,
+            int diag_every, int* tb_len);
+
 #ifdef __cplusplus
 }
 #endif

@@ -110,6 +110,35 @@ def test_nw(env, n, resident):
         assert np.array_equal(out[1:, 1:], inp["dp"][1:, 1:])
 
 
+@pytest.mark.parametrize("n,m,per_diag,tb_every,diag_every", [
+    (128, 128, False, 0, 0),      # cfg1 SW-128: one cooperative launch, 4 epochs
+    (40, 70, True, 16, 32),       # cfg3 shape: per-diagonal launches, traceback + diagnose points
+    (300, 257, True, 64, 128)])
+def test_smith_waterman(env, n, m, per_diag, tb_every, diag_every):
+    torch, apps, xpl = env
+    from xplgen import sw
+    spec = sw.sw_spec(n, m)
+    ar = apps.Arena(spec)
+    inp = sw.sw_inputs(n, m, 0x58504C04 + n)
+    s = torch.cuda.Stream()
+    params = (50, 0, 8)
+    with xpl.Context(pool_words=1 << 22) as ctx:
+        run = apps.Run(ctx, s.cuda_stream, params=params)
+        tb = apps.sw(run, ar, n, m, per_diag, tb_every, diag_every, inp)
+        got = run.reports()
+        assert run.r.dev_accesses == sw.sw_accesses(n, m, per_diag)
+    H = sw.sw_dp(inp["a"], inp["b"])
+    assert tb == sw.sw_traceback(H, inp["a"], inp["b"])[3]
+    if per_diag:  # (the single-launch program re-zeroes H at the end)
+        assert np.array_equal(ar.view("H").view(np.int32).reshape(n + 1, m + 1), H)
+    compare(got, oracle_run(sw.sw_trace(ar.addrs, spec, n, m, per_diag, tb_every, diag_every, inp, params)))
+    if not per_diag:
+        # cfg1 under the snapshot reading (D5): one launch sees only the pre-epoch
+        # (CPU) values, so no read of H is G>G although the wavefront reads its own output
+        h = got[-1][2]
+        assert h["w_g"] == n * m and h["r_gg"] == 0 and h["r_cg"] == (n + 1) * (m + 1) - 1
+
+
 def test_twin_runs_without_xpl(env):
     torch, apps, xpl = env
     from xplgen import rodinia

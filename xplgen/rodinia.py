@@ -18,21 +18,22 @@ from .trace import D2H, DEVICE, H2D, HOST, R, RW, W, batch
 ALIGN = 256
 
 
-def layout(spec, dev_base, host_base):
-    """Place the arrays of `spec` [(name, nbytes, kind, where)] in two arenas;
-    returns (addrs, total_dev_bytes, total_host_bytes)."""
-    off = {"dev": 0, "host": 0}
+def layout(spec, dev_base, host_base, managed_base=0):
+    """Place the arrays of `spec` [(name, nbytes, kind, where)] in their arenas
+    (where = "dev" | "host" | "managed"); returns (addrs, dev_bytes, host_bytes)."""
+    off = {"dev": 0, "host": 0, "managed": 0}
+    base = {"dev": dev_base, "host": host_base, "managed": managed_base}
     addrs = []
     for name, nbytes, kind, where in spec:
-        base = dev_base if where == "dev" else host_base
-        addrs.append(base + off[where])
+        addrs.append(base[where] + off[where])
         off[where] += (nbytes + ALIGN - 1) // ALIGN * ALIGN + ALIGN
+    layout.last_sizes = dict(off)
     return addrs, off["dev"], off["host"]
 
 
 def arena_sizes(spec):
-    _, d, h = layout(spec, 0, 0)
-    return d, h
+    layout(spec, 0, 0, 0)
+    return layout.last_sizes
 
 
 # ---------------------------------------------------------------------------
