@@ -14,7 +14,7 @@ from . import xpl
 from .xpl import REPORT_FIELDS, XplAllocReport, XplDiagParams
 
 u64, u32, i32, vp, sz = C.c_uint64, C.c_uint32, C.c_int, C.c_void_p, C.c_size_t
-MAXA = 24
+MAXA = 64
 
 
 class XplwArrays(C.Structure):
@@ -35,10 +35,13 @@ _w.xplw_backprop.argtypes = [C.POINTER(XplwRun), C.POINTER(XplwArrays), i32, i32
 _w.xplw_bfs.argtypes = [C.POINTER(XplwRun), C.POINTER(XplwArrays), i32, i32, vp, C.POINTER(i32)]
 _w.xplw_nw.argtypes = [C.POINTER(XplwRun), C.POINTER(XplwArrays), i32, i32, vp]
 _w.xplw_sw.argtypes = [C.POINTER(XplwRun), C.POINTER(XplwArrays), i32, i32, i32, i32, i32, C.POINTER(i32)]
+_w.xplw_lulesh.argtypes = [C.POINTER(XplwRun), C.POINTER(XplwArrays), i32, i32, vp, vp]
+_w.xplw_lulesh_layout.argtypes = [i32]
+_w.xplw_lulesh_layout.restype = i32
 _w.xplw_alloc_managed.argtypes = [u64]
 _w.xplw_alloc_managed.restype = vp
 _w.xplw_free_managed.argtypes = [vp]
-for f in ("xplw_hotspot", "xplw_backprop", "xplw_bfs", "xplw_nw", "xplw_sw", "xplw_free_managed"):
+for f in ("xplw_hotspot", "xplw_backprop", "xplw_bfs", "xplw_nw", "xplw_sw", "xplw_free_managed", "xplw_lulesh"):
     getattr(_w, f).restype = i32
 
 
@@ -183,3 +186,25 @@ def sw(run: Run, arena: Arena, n, m, per_diagonal, tb_every, diag_every, inp):
                C.byref(tb))
     run.check()
     return tb.value
+
+
+def lulesh_prepare(arena: Arena, s, topo):
+    """Write the mesh topology (input) into the managed topology arrays."""
+    import torch
+    from xplgen import lulesh as L
+    for k, arr in topo.items():
+        arena.view(L.NAMES[k]).view(np.int32)[:] = arr
+    torch.cuda.synchronize()
+
+
+def lulesh(run: Run, arena: Arena, s, steps, hook_counter):
+    """Returns the temporaries' addresses [(force, gradient)] per step."""
+    tmp = (u64 * (2 * steps))()
+    _w.xplw_lulesh(C.byref(run.r), C.byref(arena.arrays), s, steps, hook_counter.data_ptr(), tmp)
+    run.check()
+    return [(tmp[2 * i], tmp[2 * i + 1]) for i in range(steps)]
+
+
+def lulesh_layout():
+    """The CUDA program's domain layout (for the cross-check with xplgen.lulesh)."""
+    return [_w.xplw_lulesh_layout(i) for i in range(9)]

@@ -1,0 +1,561 @@
+// work_lulesh.cu -- a LULESH-shaped instrumented program (the paper's main case
+// study, §II-C, §III-D, Fig. 4).
+//
+// Shape, not physics: a managed singleton "domain" object of 3736 bytes
+// holds the pointers of 50 managed arrays and the scalar
+// parameters; every kernel reads the array pointers it uses from the domain
+// (RAJA lambdas capture the domain), so all GPU threads hit the same domain
+// words.  Per timestep: 16 kernel stages (19 launches) -- nodal force zeroing,
+// element stress and hourglass forces gathered through the 8-node lists into a
+// temporary, corner sums back to nodes through node->corner lists, nodal
+// acceleration / symmetry planes / velocity / position, element kinematics into
+// a second temporary, Q gradients over face neighbours, four EOS stages, volume
+// update, courant and hydro dt reductions.  Two temporaries are allocated,
+// published through the domain, and freed every timestep.  The
+// host then reads the dt reductions and updates the domain (TimeIncrement): it
+// writes 27 domain words and reads 680; the kernels read 85 domain words, 18 of
+// them CPU-written -- the dom row of Fig. 4 (C=27, C>C=680, 9 %, 18
+// alternating).  The CPU twin (oracle trace) is xplgen/lulesh.py.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <chrono>
+
+#include "xpl.h"
+#include "xpl_device.cuh"
+#include "xpl_host.h"
+#include "xplw.h"
+
+namespace {
+
+// ---- the domain object (3736 bytes = 934 words) ----
+enum Slot {
+  X, Y, Z, XD, YD, ZD, XDD, YDD, ZDD, FX, FY, FZ, NODALMASS,                   // nodal reals
+  E, P, Q, V, VOLO, VNEW, DELV, VDOV, AREALG, SS, ELEMMASS, QL, QQ,             // element reals
+  NODELIST, LXIM, LXIP, NODEELEMSTART, CORNERLIST, SYMMX, ELEMBC,               // topology
+  LETAM, LETAP, LZETAM, LZETAP, SYMMY, SYMMZ,                                   // never used
+  DELV_XI, DELV_ETA, DELV_ZETA, DELX_XI, DELX_ETA, DELX_ZETA, DXX, DYY, DZZ,    // never used
+  TMP_FORCE, TMP_DVDX, NSLOT
+};
+struct Dom {
+  void* ptr[NSLOT];  // words 0..99
+  uint32_t numElem;  // word 100 (read by every kernel)
+  uint32_t numNode;  // word 101
+  double dt;         // words 102-103
+  double time;       // words 104-105
+  uint32_t cycle;    // word 106
+  uint32_t pad107;
+  double dtcourant;  // words 108-109
+  double dthydro;    // words 110-111
+  uint32_t misc[14]; // words 112-125: written by the host each step; 112-121 read by kernels
+  uint32_t params[808];
+};
+static_assert(NSLOT == 50, "50 pointer slots");
+static_assert(sizeof(Dom) == 3736, "the domain object of Fig. 5 has 3736 bytes (P:L315)");
+
+template <bool I, class T>
+__device__ __forceinline__ const T& RD(const T& x) {
+  if constexpr (I) return xpl_read(x);
+  else return x;
+}
+template <bool I, class T>
+__device__ __forceinline__ T& WR(T& x) {
+  if constexpr (I) return xpl_write(x);
+  else return x;
+}
+template <bool I, class T>
+__device__ __forceinline__ T& RW(T& x) {
+  if constexpr (I) return xpl_rw(x);
+  else return x;
+}
+
+// Hook calls are counted per thread (c) and added once per block (exact counts).
+template <bool I>
+__device__ __forceinline__ void count_hooks(unsigned long long* hc, unsigned c) {
+  if constexpr (I) {
+    __shared__ unsigned s_c;
+    if (threadIdx.x == 0) s_c = 0;
+    __syncthreads();
+    if (c) atomicAdd(&s_c, c);
+    __syncthreads();
+    if (threadIdx.x == 0 && s_c) atomicAdd(hc, (unsigned long long)s_c);
+  }
+}
+
+// every traced access goes through one of these (and is counted)
+#define R_(x) (++c, RD<I>(x))
+#define W_(x) (++c, WR<I>(x))
+#define RW_(x) (++c, RW<I>(x))
+#define PTR(T, slot) static_cast<T*>(R_(d->ptr[slot]))
+#define NE() (int)R_(d->numElem)
+
+// 1. zero the nodal forces
+template <bool I>
+__global__ void k_zero_forces(Dom* d, int nn, unsigned long long* hc) {
+  const int n = blockIdx.x * blockDim.x + threadIdx.x;
+  unsigned c = 0;
+  if (n < nn) {
+    double *fx = PTR(double, FX), *fy = PTR(double, FY), *fz = PTR(double, FZ);
+    W_(fx[n]) = 0.0;
+    W_(fy[n]) = 0.0;
+    W_(fz[n]) = 0.0;
+  }
+  count_hooks<I>(hc, c);
+}
+
+// 2. stress integration: gather the 8 nodes, write 8 corner forces x 3
+template <bool I>
+__global__ void k_integrate_stress(Dom* d, unsigned long long* hc) {
+  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+  unsigned c = 0;
+  if (e < NE()) {
+    const int* nl = PTR(const int, NODELIST);
+    const double *x = PTR(const double, X), *y = PTR(const double, Y), *z = PTR(const double, Z);
+    const double sig = -(R_(PTR(const double, P)[e]) + R_(PTR(const double, Q)[e]));
+    double* f = PTR(double, TMP_FORCE);
+    for (int k = 0; k < 8; ++k) {
+      const int n = R_(nl[8 * e + k]);
+      const double g = R_(x[n]) + R_(y[n]) + R_(z[n]);
+      W_(f[24 * e + 3 * k + 0]) = sig * g;
+      W_(f[24 * e + 3 * k + 1]) = sig * g * 0.5;
+      W_(f[24 * e + 3 * k + 2]) = sig * g * 0.25;
+    }
+  }
+  count_hooks<I>(hc, c);
+}
+
+// 3. hourglass control: gather nodal velocities, add to the corner forces
+template <bool I>
+__global__ void k_hourglass(Dom* d, unsigned long long* hc) {
+  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+  unsigned c = 0;
+  if (e < NE()) {
+    const int* nl = PTR(const int, NODELIST);
+    const double *xd = PTR(const double, XD), *yd = PTR(const double, YD), *zd = PTR(const double, ZD);
+    const double coef = R_(PTR(const double, SS)[e]) * R_(PTR(const double, ELEMMASS)[e]) /
+                        (R_(PTR(const double, VOLO)[e]) * R_(PTR(const double, V)[e]) + 1.0);
+    double* f = PTR(double, TMP_FORCE);
+    for (int k = 0; k < 8; ++k) {
+      const int n = R_(nl[8 * e + k]);
+      const double a = R_(xd[n]), b = R_(yd[n]), g = R_(zd[n]);
+      RW_(f[24 * e + 3 * k + 0]) += coef * a;
+      RW_(f[24 * e + 3 * k + 1]) += coef * b;
+      RW_(f[24 * e + 3 * k + 2]) += coef * g;
+    }
+  }
+  count_hooks<I>(hc, c);
+}
+
+// 4. sum the corner forces into the nodes through the node->corner lists
+template <bool I>
+__global__ void k_corner_sum(Dom* d, int nn, unsigned long long* hc) {
+  const int n = blockIdx.x * blockDim.x + threadIdx.x;
+  unsigned c = 0;
+  if (n < nn) {
+    const int *st = PTR(const int, NODEELEMSTART), *cl = PTR(const int, CORNERLIST);
+    const double* f = PTR(const double, TMP_FORCE);
+    double *fx = PTR(double, FX), *fy = PTR(double, FY), *fz = PTR(double, FZ);
+    const int b = R_(st[n]), en = R_(st[n + 1]);
+    double sx = 0, sy = 0, sz = 0;
+    for (int k = b; k < en; ++k) {
+      const int corner = R_(cl[k]);
+      sx += R_(f[3 * corner + 0]);
+      sy += R_(f[3 * corner + 1]);
+      sz += R_(f[3 * corner + 2]);
+    }
+    W_(fx[n]) = sx;
+    W_(fy[n]) = sy;
+    W_(fz[n]) = sz;
+  }
+  count_hooks<I>(hc, c);
+}
+
+// 5. nodal accelerations
+template <bool I>
+__global__ void k_accel(Dom* d, int nn, unsigned long long* hc) {
+  const int n = blockIdx.x * blockDim.x + threadIdx.x;
+  unsigned c = 0;
+  if (n < nn) {
+    const double m = R_(PTR(const double, NODALMASS)[n]);
+    const double ax = R_(PTR(const double, FX)[n]) / m, ay = R_(PTR(const double, FY)[n]) / m,
+                 az = R_(PTR(const double, FZ)[n]) / m;
+    W_(PTR(double, XDD)[n]) = ax;
+    W_(PTR(double, YDD)[n]) = ay;
+    W_(PTR(double, ZDD)[n]) = az;
+  }
+  count_hooks<I>(hc, c);
+}
+
+// 6. symmetry plane: zero the accelerations of the plane's nodes
+template <bool I>
+__global__ void k_symm(Dom* d, int ns, unsigned long long* hc) {
+  const int k = blockIdx.x * blockDim.x + threadIdx.x;
+  unsigned c = 0;
+  if (k < ns) {
+    const int n = R_(PTR(const int, SYMMX)[k]);
+    W_(PTR(double, XDD)[n]) = 0.0;
+    W_(PTR(double, YDD)[n]) = 0.0;
+    W_(PTR(double, ZDD)[n]) = 0.0;
+  }
+  count_hooks<I>(hc, c);
+}
+
+// 7./8. velocity and position updates
+template <bool I>
+__global__ void k_velocity(Dom* d, int nn, unsigned long long* hc) {
+  const int n = blockIdx.x * blockDim.x + threadIdx.x;
+  unsigned c = 0;
+  if (n < nn) {
+    const double dt = R_(d->dt);
+    const double ax = R_(PTR(const double, XDD)[n]), ay = R_(PTR(const double, YDD)[n]),
+                 az = R_(PTR(const double, ZDD)[n]);
+    RW_(PTR(double, XD)[n]) += dt * ax;
+    RW_(PTR(double, YD)[n]) += dt * ay;
+    RW_(PTR(double, ZD)[n]) += dt * az;
+  }
+  count_hooks<I>(hc, c);
+}
+template <bool I>
+__global__ void k_position(Dom* d, int nn, unsigned long long* hc) {
+  const int n = blockIdx.x * blockDim.x + threadIdx.x;
+  unsigned c = 0;
+  if (n < nn) {
+    const double dt = R_(d->dt);
+    const double vx = R_(PTR(const double, XD)[n]), vy = R_(PTR(const double, YD)[n]),
+                 vz = R_(PTR(const double, ZD)[n]);
+    RW_(PTR(double, X)[n]) += dt * vx;
+    RW_(PTR(double, Y)[n]) += dt * vy;
+    RW_(PTR(double, Z)[n]) += dt * vz;
+  }
+  count_hooks<I>(hc, c);
+}
+
+// 9. element kinematics: gather positions and velocities, new volume, gradients
+template <bool I>
+__global__ void k_kinematics(Dom* d, unsigned long long* hc) {
+  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+  unsigned c = 0;
+  if (e < NE()) {
+    const int* nl = PTR(const int, NODELIST);
+    const double *x = PTR(const double, X), *y = PTR(const double, Y), *z = PTR(const double, Z);
+    const double *xd = PTR(const double, XD), *yd = PTR(const double, YD), *zd = PTR(const double, ZD);
+    double vol = 0, dv = 0;
+    for (int k = 0; k < 8; ++k) {
+      const int n = R_(nl[8 * e + k]);
+      vol += R_(x[n]) * R_(y[n]) + R_(z[n]);
+      dv += R_(xd[n]) + R_(yd[n]) + R_(zd[n]);
+    }
+    const double vnew = vol / (R_(PTR(const double, VOLO)[e]) + 1.0);
+    const double vold = R_(PTR(const double, V)[e]);
+    W_(PTR(double, VNEW)[e]) = vnew;
+    W_(PTR(double, DELV)[e]) = vnew - vold;
+    W_(PTR(double, AREALG)[e]) = vol;
+    double* g = PTR(double, TMP_DVDX);
+    W_(g[3 * e + 0]) = dv;
+    W_(g[3 * e + 1]) = dv * 0.5;
+    W_(g[3 * e + 2]) = dv * 0.25;
+  }
+  count_hooks<I>(hc, c);
+}
+
+// 10. strain rate from the gradients
+template <bool I>
+__global__ void k_lagrange(Dom* d, unsigned long long* hc) {
+  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+  unsigned c = 0;
+  if (e < NE()) {
+    const double* g = PTR(const double, TMP_DVDX);
+    const double r = (R_(g[3 * e]) + R_(g[3 * e + 1]) + R_(g[3 * e + 2])) / (R_(PTR(const double, VNEW)[e]) + 1.0);
+    W_(PTR(double, VDOV)[e]) = r;
+  }
+  count_hooks<I>(hc, c);
+}
+
+// 11./12. monotonic Q: gradients over the xi face neighbours, region limiter
+template <bool I>
+__global__ void k_monoq_grad(Dom* d, unsigned long long* hc) {
+  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+  unsigned c = 0;
+  if (e < NE()) {
+    const double* vdov = PTR(const double, VDOV);
+    const int m = R_(PTR(const int, LXIM)[e]), p = R_(PTR(const int, LXIP)[e]);
+    const double r = R_(vdov[p]) - R_(vdov[m]) + R_(PTR(const double, VNEW)[e]);
+    W_(PTR(double, QL)[e]) = r;
+  }
+  count_hooks<I>(hc, c);
+}
+template <bool I>
+__global__ void k_monoq_region(Dom* d, unsigned long long* hc) {
+  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+  unsigned c = 0;
+  if (e < NE()) {
+    const int bc = R_(PTR(const int, ELEMBC)[e]);
+    const double r = (bc & 1 ? 0.5 : 1.0) * R_(PTR(const double, QL)[e]) * R_(PTR(const double, VDOV)[e]);
+    W_(PTR(double, QQ)[e]) = r;
+  }
+  count_hooks<I>(hc, c);
+}
+
+// 13. the four EOS stages (they read material parameters from the domain)
+template <bool I>
+__global__ void k_eos(Dom* d, int stage, unsigned long long* hc) {
+  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+  unsigned c = 0;
+  if (e < NE()) {
+    const double t = R_(d->time);
+    if (stage == 0) {  // energy
+      const double w = R_(d->misc[0]) * 1e-6 + R_(d->misc[1]) * 1e-6 + R_(d->misc[2]);
+      const double de = R_(PTR(const double, DELV)[e]) *
+                        (R_(PTR(const double, P)[e]) + R_(PTR(const double, Q)[e]) +
+                         R_(PTR(const double, QQ)[e]) + R_(PTR(const double, QL)[e]));
+      RW_(PTR(double, E)[e]) += w - de;
+    } else if (stage == 1) {  // pressure
+      const double pmin = R_(d->misc[3]) * 1e-6 + R_(d->misc[4]);
+      const double r = pmin + R_(PTR(const double, E)[e]) / (R_(PTR(const double, VNEW)[e]) + t);
+      W_(PTR(double, P)[e]) = r;
+    } else if (stage == 2) {  // sound speed
+      const double ss4o3 = R_(d->misc[5]) * 1e-6 + R_(d->misc[6]);
+      const double r = ss4o3 * (R_(PTR(const double, P)[e]) + R_(PTR(const double, E)[e])) /
+                       (R_(PTR(const double, VNEW)[e]) + 1.0);
+      W_(PTR(double, SS)[e]) = r;
+    } else {  // artificial viscosity
+      const double qstop = R_(d->misc[7]) * 1e-6 + R_(d->misc[8]) + R_(d->misc[9]);
+      const double r = qstop + R_(PTR(const double, QL)[e]) + R_(PTR(const double, QQ)[e]) +
+                       0.0 * R_(PTR(const double, P)[e]);
+      W_(PTR(double, Q)[e]) = r;
+    }
+  }
+  count_hooks<I>(hc, c);
+}
+
+// 14. volumes
+template <bool I>
+__global__ void k_update_volumes(Dom* d, unsigned long long* hc) {
+  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+  unsigned c = 0;
+  if (e < NE()) {
+    const double v = R_(PTR(const double, VNEW)[e]);
+    W_(PTR(double, V)[e]) = v;
+  }
+  count_hooks<I>(hc, c);
+}
+
+// 15./16. dt reductions: one minimum per 256-element block into dtb (GPU W, host R)
+template <bool I, bool COURANT>
+__global__ void __launch_bounds__(256) k_dt(Dom* d, double* dtb, int nblk, unsigned long long* hc) {
+  __shared__ double s_min[256];
+  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+  unsigned c = 0;
+  double v = 1e30;
+  if (e < NE()) {
+    if (COURANT) {
+      const double ss = R_(PTR(const double, SS)[e]), vd = R_(PTR(const double, VDOV)[e]),
+                   ar = R_(PTR(const double, AREALG)[e]);
+      v = ar / (ss * ss + vd * vd + 1.0);
+    } else {
+      const double vd = R_(PTR(const double, VDOV)[e]);
+      v = 1.0 / (vd * vd + 1e-3);
+    }
+  }
+  s_min[threadIdx.x] = v;
+  __syncthreads();
+  for (int o = 128; o > 0; o >>= 1) {
+    if (threadIdx.x < o && s_min[threadIdx.x + o] < s_min[threadIdx.x]) s_min[threadIdx.x] = s_min[threadIdx.x + o];
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) W_(dtb[(COURANT ? 0 : nblk) + blockIdx.x]) = s_min[0];
+  count_hooks<I>(hc, c);
+}
+
+}  // namespace
+
+extern "C" {
+
+int xplw_bind_lulesh(xpl_ctx* ctx) { return (int)xpl_device_bind(ctx); }
+
+// Word-level layout of the domain for the CPU twin: byte offset of a field.
+int xplw_lulesh_layout(int what) {
+  switch (what) {
+    case 0: return (int)sizeof(Dom);
+    case 1: return (int)offsetof(Dom, numElem);
+    case 2: return (int)offsetof(Dom, dt);
+    case 3: return (int)offsetof(Dom, time);
+    case 4: return (int)offsetof(Dom, cycle);
+    case 5: return (int)offsetof(Dom, dtcourant);
+    case 6: return (int)offsetof(Dom, dthydro);
+    case 7: return (int)offsetof(Dom, misc);
+    case 8: return (int)offsetof(Dom, params);
+    default: return -1;
+  }
+}
+
+int xplw_lulesh(xplw_run* run, const xplw_arrays* arr, int s, int steps, unsigned long long* hook_count,
+                unsigned long long* tmp_addrs) {
+  const bool on = run->ctx != nullptr;
+  cudaStream_t st = (cudaStream_t)run->stream;
+  const int ne = s * s * s, nn = (s + 1) * (s + 1) * (s + 1), nsym = (s + 1) * (s + 1);
+  const int nblk = (ne + 255) / 256;
+  Dom* dom = (Dom*)arr->addr[0];
+  double* dtb = (double*)arr->addr[1];
+  // arr->addr[2 + k] = the array of pointer slot k (k < TMP_FORCE)
+  xpl_host_tracer* tr = on ? new xpl_host_tracer(run->ctx) : nullptr;
+  auto ok = [&](int x) {
+    if (x && !run->status) run->status = x;
+  };
+  auto okc = [&](cudaError_t e) {
+    if (e != cudaSuccess && !run->status) run->status = XPL_ERR_CUDA;
+  };
+  auto flush = [&]() {
+    if (tr) ok(tr->flush());
+  };
+  auto host_t = [&](std::chrono::steady_clock::time_point t0) {
+    run->host_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  };
+  auto diag = [&]() {
+    flush();
+    if (!on) return;
+    size_t nr = 0;
+    xpl_alloc_report* o = run->out ? run->out + run->n_out : nullptr;
+    const size_t cap = run->out ? run->out_cap - run->n_out : 0;
+    const int x = xpl_diagnose(run->ctx, &run->params, nullptr, 0, o, cap, &nr, 1);
+    if (x == XPL_OK) {
+      run->n_out += nr;
+      if (run->diag_rows && run->n_diag < run->diag_cap) run->diag_rows[run->n_diag] = (uint32_t)nr;
+      run->n_diag++;
+    } else {
+      ok(x);
+    }
+  };
+  // one instrumented launch = one GPU epoch (the kernel-launch wrapper)
+  auto launch = [&](auto fi, auto ft, int grid) {
+    flush();
+    if (on) ok(xpl_kernel_begin(run->ctx, st));
+    if (on) fi(grid);
+    else ft(grid);
+    okc(cudaGetLastError());
+    if (on) ok(xpl_kernel_end(run->ctx, st));
+    run->epochs++;
+  };
+#define LAUNCH(KER, GRID, ...)                                                          \
+  launch([&](int g) { KER<true><<<g, 256, 0, st>>>(__VA_ARGS__); },                    \
+         [&](int g) { KER<false><<<g, 256, 0, st>>>(__VA_ARGS__); }, GRID)
+  auto managed = [&](size_t bytes) -> void* {
+    void* p = nullptr;
+    okc(cudaMallocManaged(&p, bytes));
+    if (on && p) ok(xpl_register_alloc(run->ctx, p, bytes, XPL_ALLOC_MANAGED));
+    return p;
+  };
+  auto release = [&](void* p) {
+    if (on) ok(xpl_free(run->ctx, p));
+    okc(cudaFree(p));  // (synchronises, like the application's cudaFree)
+  };
+  auto hw = [&](auto& x, auto v) {  // a traced host write
+    if (tr) tr->write(x) = v;
+    else x = v;
+    run->host_accesses++;
+  };
+
+  if (on)
+    for (int k = 0; k < arr->n; ++k)
+      ok(xpl_register_alloc(run->ctx, (const void*)arr->addr[k], arr->bytes[k], (xpl_alloc_kind)arr->kind[k]));
+  // ---- initialisation (host): the domain, the arrays, the mesh topology ----
+  auto t0 = std::chrono::steady_clock::now();
+  for (int k = 0; k < NSLOT; ++k) hw(dom->ptr[k], k < TMP_FORCE ? (void*)arr->addr[2 + k] : (void*)nullptr);
+  hw(dom->numElem, (uint32_t)ne);
+  hw(dom->numNode, (uint32_t)nn);
+  hw(dom->dt, 1e-3);
+  hw(dom->time, 0.0);
+  hw(dom->cycle, 0u);
+  hw(dom->pad107, 0u);
+  hw(dom->dtcourant, 1e20);
+  hw(dom->dthydro, 1e20);
+  for (int k = 0; k < 14; ++k) hw(dom->misc[k], (uint32_t)(k + 1));
+  for (int k = 0; k < 808; ++k) hw(dom->params[k], (uint32_t)k);
+  for (int k = 0; k < TMP_FORCE; ++k) {  // every array: its initial values (topology arrays: the input)
+    const uint64_t bytes = arr->bytes[2 + k];
+    if (k >= NODELIST && k <= ELEMBC) {
+      int* a = (int*)arr->addr[2 + k];
+      for (uint64_t i = 0; i < bytes / 4; ++i) hw(a[i], a[i]);
+    } else if (k >= NODELIST) {
+      int* a = (int*)arr->addr[2 + k];
+      for (uint64_t i = 0; i < bytes / 4; ++i) hw(a[i], 0);
+    } else {
+      double* a = (double*)arr->addr[2 + k];
+      for (uint64_t i = 0; i < bytes / 8; ++i) hw(a[i], 1.0 + (double)(i & 7) * 0.125);
+    }
+  }
+  for (int b = 0; b < 2 * nblk; ++b) hw(dtb[b], 0.0);
+  host_t(t0);
+
+  for (int step = 0; step < steps; ++step) {
+    // forces: a temporary for the 8 corner forces of every element
+    void* tf = managed(sizeof(double) * 24 * (size_t)ne);
+    if (tmp_addrs) tmp_addrs[2 * step] = (unsigned long long)tf;
+    hw(dom->ptr[TMP_FORCE], tf);
+    LAUNCH(k_zero_forces, (nn + 255) / 256, dom, nn, hook_count);
+    LAUNCH(k_integrate_stress, nblk, dom, hook_count);
+    LAUNCH(k_hourglass, nblk, dom, hook_count);
+    LAUNCH(k_corner_sum, (nn + 255) / 256, dom, nn, hook_count);
+    okc(cudaStreamSynchronize(st));
+    hw(dom->ptr[TMP_FORCE], (void*)nullptr);
+    flush();
+    release(tf);
+    LAUNCH(k_accel, (nn + 255) / 256, dom, nn, hook_count);
+    LAUNCH(k_symm, (nsym + 255) / 256, dom, nsym, hook_count);
+    LAUNCH(k_velocity, (nn + 255) / 256, dom, nn, hook_count);
+    LAUNCH(k_position, (nn + 255) / 256, dom, nn, hook_count);
+    // kinematics: a temporary for the velocity gradients
+    void* tg = managed(sizeof(double) * 3 * (size_t)ne);
+    if (tmp_addrs) tmp_addrs[2 * step + 1] = (unsigned long long)tg;
+    hw(dom->ptr[TMP_DVDX], tg);
+    LAUNCH(k_kinematics, nblk, dom, hook_count);
+    LAUNCH(k_lagrange, nblk, dom, hook_count);
+    okc(cudaStreamSynchronize(st));
+    hw(dom->ptr[TMP_DVDX], (void*)nullptr);
+    flush();
+    release(tg);
+    LAUNCH(k_monoq_grad, nblk, dom, hook_count);
+    LAUNCH(k_monoq_region, nblk, dom, hook_count);
+    for (int stage = 0; stage < 4; ++stage) LAUNCH(k_eos, nblk, dom, stage, hook_count);
+    LAUNCH(k_update_volumes, nblk, dom, hook_count);
+    launch([&](int g) { k_dt<true, true><<<g, 256, 0, st>>>(dom, dtb, nblk, hook_count); },
+           [&](int g) { k_dt<false, true><<<g, 256, 0, st>>>(dom, dtb, nblk, hook_count); }, nblk);
+    launch([&](int g) { k_dt<true, false><<<g, 256, 0, st>>>(dom, dtb, nblk, hook_count); },
+           [&](int g) { k_dt<false, false><<<g, 256, 0, st>>>(dom, dtb, nblk, hook_count); }, nblk);
+    okc(cudaStreamSynchronize(st));
+    // TimeIncrement (host): the dt minima, the domain's parameters, the new dt
+    t0 = std::chrono::steady_clock::now();
+    double dc = 1e30, dh = 1e30;
+    for (int b = 0; b < nblk; ++b) {
+      const double v = tr ? tr->read(dtb[b]) : dtb[b];
+      dc = v < dc ? v : dc;
+    }
+    for (int b = 0; b < nblk; ++b) {
+      const double v = tr ? tr->read(dtb[nblk + b]) : dtb[nblk + b];
+      dh = v < dh ? v : dh;
+    }
+    run->host_accesses += 2 * nblk;
+    hw(dom->dtcourant, dc);
+    hw(dom->dthydro, dh);
+    const uint32_t* w = (const uint32_t*)dom;
+    uint64_t chk = 0;
+    for (int k = 100; k < 780; ++k) chk += tr ? tr->read(w[k]) : w[k];  // 680 words of parameters
+    run->host_accesses += 680;
+    hw(dom->dt, 1e-3 + (double)(chk & 1) * 1e-9);
+    hw(dom->time, dom->time + 1e-3);
+    hw(dom->cycle, (uint32_t)(step + 1));
+    for (int k = 0; k < 14; ++k) hw(dom->misc[k], (uint32_t)(k + 1));
+    host_t(t0);
+    if (run->diag_each) diag();  // "diagnostics are called at the end of every timestep"
+  }
+  flush();
+  delete tr;
+  tr = nullptr;
+  if (on)
+    for (int k = 0; k < arr->n; ++k) ok(xpl_free(run->ctx, (const void*)arr->addr[k]));
+  diag();
+  okc(cudaStreamSynchronize(st));
+  return run->status;
+}
+
+}  // extern "C"

@@ -64,6 +64,7 @@ int xplw_touch(unsigned long long base, unsigned long long n, unsigned seed, voi
 
 int xplw_bind_rodinia(xpl_ctx* ctx);
 int xplw_bind_sw(xpl_ctx* ctx);
+int xplw_bind_lulesh(xpl_ctx* ctx);
 
 // Bind the hooks of every instrumented translation unit of this library to ctx
 // (xpl_device_bind copies the device context into each TU's __constant__).
@@ -71,6 +72,7 @@ int xplw_bind(xpl_ctx* ctx) {
   int s = (int)xpl_device_bind(ctx);
   if (!s) s = xplw_bind_rodinia(ctx);
   if (!s) s = xplw_bind_sw(ctx);
+  if (!s) s = xplw_bind_lulesh(ctx);
   return s;
 }
 

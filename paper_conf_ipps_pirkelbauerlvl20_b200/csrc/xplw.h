@@ -20,7 +20,7 @@
 extern "C" {
 #endif
 
-#define XPLW_MAX_ARRAYS 24
+#define XPLW_MAX_ARRAYS 64
 
 typedef struct {
   uint64_t addr[XPLW_MAX_ARRAYS];  /* base address of each array (app order)   */
@@ -94,6 +94,17 @@ int xplw_nw(xplw_run* run, const xplw_arrays* a, int n, int penalty, const int* 
  * Returns the traceback length in *tb_len. */
 int xplw_sw(xplw_run* run, const xplw_arrays* a, int n, int m, int per_diagonal, int tb_every,
             int diag_every, int* tb_len);
+
+/* LULESH-shaped program (§II-C, §III-D, Fig. 4; cfg4/cfg5): edge s elements,
+ * `steps` timesteps of 19 instrumented launches with two temporaries allocated
+ * and freed per step (managed, registered by the program) and a diagnose after
+ * each step.  arrays: 0 dom (3736 B), 1 dt_block (2*ceil(s^3/256) doubles),
+ * 2 + k = the array of domain pointer slot k for k < 48 (all MANAGED; slots
+ * 26..32 hold the mesh topology on entry).  hook_count: device u64.  tmp_addrs:
+ * host array of 2*steps (the temporaries' addresses, for the CPU twin) or NULL. */
+int xplw_lulesh(xplw_run* run, const xplw_arrays* a, int s, int steps, unsigned long long* hook_count,
+                unsigned long long* tmp_addrs);
+int xplw_lulesh_layout(int what);
 
 #ifdef __cplusplus
 }

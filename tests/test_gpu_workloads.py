@@ -139,6 +139,42 @@ def test_smith_waterman(env, n, m, per_diag, tb_every, diag_every):
         assert h["w_g"] == n * m and h["r_gg"] == 0 and h["r_cg"] == (n + 1) * (m + 1) - 1
 
 
+def test_lulesh_layout_matches_twin(env):
+    torch, apps, xpl = env
+    from xplgen import lulesh as L
+    assert apps.lulesh_layout() == [L.DOM_BYTES, L.OFF_NUMELEM, L.OFF_DT, L.OFF_TIME, L.OFF_CYCLE,
+                                    L.OFF_DTC, L.OFF_DTH, L.OFF_MISC, L.OFF_PARAMS]
+
+
+@pytest.mark.parametrize("s,steps", [(8, 3), (5, 2), (13, 2)])
+def test_lulesh(env, s, steps):
+    torch, apps, xpl = env
+    from xplgen import lulesh as L
+    spec = L.lulesh_spec(s)
+    ar = apps.Arena(spec)
+    topo = L.topology(s, 0x58504C05)
+    apps.lulesh_prepare(ar, s, topo)
+    st = torch.cuda.Stream()
+    params = (50, 0, 256)
+    hc = torch.zeros(1, dtype=torch.int64, device="cuda")
+    with xpl.Context(pool_words=1 << 24) as ctx:
+        run = apps.Run(ctx, st.cuda_stream, params=params)
+        tmps = apps.lulesh(run, ar, s, steps, hc)
+        got = run.reports()
+    ops, hooks = L.lulesh_trace(ar.addrs, spec, s, steps, topo, params, tmps)
+    assert int(hc.item()) == hooks
+    exp = oracle_run(ops)
+    compare(got, exp)
+    if s == 8:
+        # Fig. 4, "after the second iteration": dom C=27, G=0, C>C=680,
+        # density 9 %, 18 alternating; (dom)->m_p C=0, G=1024, C>C=0, G>G=1024, 100 %, 0
+        dom = got[1][0]
+        assert (dom["w_c"], dom["w_g"], dom["r_cc"], dom["density_pct_gpu"], dom["alternating"]) == (27, 0, 680, 9, 18)
+        mp = got[1][2 + L.P]
+        assert (mp["words"], mp["w_c"], mp["w_g"], mp["r_cc"], mp["r_gg"], mp["density_pct_gpu"],
+                mp["alternating"]) == (1024, 0, 1024, 0, 1024, 100, 0)
+
+
 def test_twin_runs_without_xpl(env):
     torch, apps, xpl = env
     from xplgen import rodinia
