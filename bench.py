@@ -52,6 +52,7 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["xpl", "reference"], default="xpl")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-other-configs", action="store_true")
     return ap.parse_args()
 
 
@@ -161,6 +162,78 @@ def diag_at_scale(xpl, torch, words=1 << 31, reps=3):
         out[name] = {"words": words, "ms": ms, "gbs": d["bytes"] / d["launches"] / (ms / 1e3) / 1e9,
                      "bytes_per_launch": d["bytes"] / d["launches"],
                      "whole_call_ms": p["diagnose"]["ms"] / p["diagnose"]["launches"]}
+    return out
+
+
+def other_configs(xpl, apps, torch, lulesh_steps=100):
+    """The other BASELINE.json configs, each run once instrumented and once as the
+    uninstrumented twin, device-timed: cfg1 SW-128 (one cooperative launch, 4
+    epochs), cfg3 SW-16K (32,767 per-diagonal epochs, host traceback segments and
+    diagnoses every 1,024 diagonals), cfg4 LULESH-shaped 100^3 x 100 timesteps."""
+    from xplgen import lulesh as L
+    from xplgen import sw
+    out = {}
+    us = torch.cuda.Stream()
+
+    def timed_run(ctx, fn):
+        s = torch.cuda.ExternalStream(ctx.runtime_stream()) if ctx is not None else us
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        run = fn(ctx)
+        e1.record(s)
+        e1.synchronize()
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1), run
+
+    for name, (n, m, per_diag, tb, dg, pool) in {
+            "cfg1_sw128": (128, 128, False, 0, 0, 1 << 20),
+            "cfg3_sw16k": (16384, 16384, True, 1024, 1024, 1 << 29)}.items():
+        spec = sw.sw_spec(n, m)
+        ar = apps.Arena(spec)
+        inp = sw.sw_inputs(n, m, 0x58504C04)
+        res = {}
+        with xpl.Context(pool_words=pool, max_rows=16) as ctx:
+            for c in (ctx, None):
+                def fn(c):
+                    run = apps.Run(c, us.cuda_stream, params=PARAMS)
+                    apps.sw(run, ar, n, m, per_diag, tb, dg, inp)
+                    return run
+                ms, run = timed_run(c, fn)
+                res["instr" if c is not None else "twin"] = (ms, run.r.dev_accesses + run.r.host_accesses,
+                                                            run.r.epochs, run.r.n_diag)
+        acc = res["instr"][1]
+        out[name] = {"workload": f"Smith-Waterman {n}x{m}, managed, "
+                                 f"{'per-diagonal launches' if per_diag else 'one cooperative launch'}",
+                     "ms": res["instr"][0], "accesses": acc, "accesses_per_s": acc / (res["instr"][0] / 1e3),
+                     "epochs": res["instr"][2], "diagnoses": res["instr"][3], "twin_ms": res["twin"][0],
+                     "slowdown": res["instr"][0] / res["twin"][0]}
+        del ar
+    s_edge = 100
+    spec = L.lulesh_spec(s_edge)
+    ar = apps.Arena(spec)
+    topo = L.topology(s_edge, 0x58504C05)
+    hc = torch.zeros(1, dtype=torch.int64, device="cuda")
+    res = {}
+    with xpl.Context(pool_words=1 << 28, max_rows=64) as ctx:
+        for c in (ctx, None):
+            apps.lulesh_prepare(ar, s_edge, topo)
+            hc.zero_()
+
+            def fn(c):
+                run = apps.Run(c, us.cuda_stream, params=PARAMS, out_cap=64 * (lulesh_steps + 1))
+                apps.lulesh(run, ar, s_edge, lulesh_steps, hc)
+                return run
+            ms, run = timed_run(c, fn)
+            res["instr" if c is not None else "twin"] = (ms, int(hc.item()) + run.r.host_accesses,
+                                                        run.r.epochs, run.r.n_diag, run.r.host_ms)
+    acc = res["instr"][1]
+    out["cfg4_lulesh100"] = {"workload": f"LULESH-shaped {s_edge}^3 x {lulesh_steps} timesteps, 50 managed "
+                                         "allocations + 2 temporaries/step, 19 launches/step",
+                             "ms": res["instr"][0], "accesses": acc,
+                             "accesses_per_s": acc / (res["instr"][0] / 1e3), "epochs": res["instr"][2],
+                             "diagnoses": res["instr"][3], "host_ms": res["instr"][4],
+                             "twin_ms": res["twin"][0], "slowdown": res["instr"][0] / res["twin"][0]}
     return out
 
 
@@ -318,8 +391,9 @@ def main():
     bt = step(None, False, time_kernels=True)
     torch.cuda.synchronize()
 
-    # --- the diagnose pass at cfg5 scale ----------------------------------------
+    # --- the diagnose pass at cfg5 scale; the other configs -------------------
     at_scale = diag_at_scale(xpl, torch)
+    others = other_configs(xpl, apps, torch) if not args.no_other_configs else None
 
     # --- roofline of the dominant runtime kernel -------------------------------
     peak, peak_src = peaks()
@@ -357,6 +431,7 @@ def main():
                      "twin_ms_per_step": twin_ms / args.steps,
                      "paper_context": "Table III P:L431-443: 5x-20x, avg ~15x (Intel E5-2695 v4 + Pascal, CUDA 9.2)"},
         "e2e": e2e, "gpu_launches": int(launches), "clocks": clocks,
+        "other_configs": others,
     }
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline()
