@@ -178,6 +178,44 @@ xpl_status xpl_diagnose(xpl_ctx* ctx, const xpl_diag_params* params, const xpl_n
                         size_t n_names, xpl_alloc_report* out, size_t cap, size_t* n_out,
                         int reset);
 
+/* ---- Address-range sharding: one logical allocation split into
+ * pieces held by different contexts (ranks).  A piece is the contiguous range of
+ * logical words [word_offset, word_offset + ceil(bytes/4)) of the logical
+ * allocation `logical_id` (logical size logical_bytes); its address range
+ * [ptr, ptr+bytes) is registered like xpl_register_alloc.  Pieces of one logical
+ * allocation must tile [0, ceil(logical_bytes/4)) exactly. */
+xpl_status xpl_register_alloc_piece(xpl_ctx* ctx, const void* ptr, size_t bytes,
+                                    xpl_alloc_kind kind, uint64_t logical_id,
+                                    uint64_t word_offset, uint64_t logical_bytes);
+
+/* One piece's share of a diagnosis: exchanged between ranks (all-gather of the
+ * raw bytes) and combined by xpl_combine_partials.  Run summaries are the run
+ * monoid (len, pre, suf, cnt, sum) of DESIGN.md §5; `blk_*` are the density
+ * blocks cut by the piece's ends (block_words > 0): global block index, GPU
+ * words in the piece, piece words in the block. */
+typedef struct {
+  uint64_t logical_id, word_offset, words, logical_words, logical_bytes, base;
+  uint32_t kind, live, name_idx, pad;
+  uint64_t cnt[9]; /* w_c w_g r_cc r_cg r_gc r_gg any gpu alternating */
+  uint64_t u_run[5], d_run[5];
+  uint64_t low_density_blocks, low_density_words; /* blocks wholly inside the piece */
+  uint64_t blk_first, blk_first_g, blk_first_s, blk_last, blk_last_g, blk_last_s;
+  uint64_t ever_accessed;
+} xpl_partial;
+
+/* xpl_diagnose, but every row is returned as a partial (out[0..cap), *n_out);
+ * rows registered with xpl_register_alloc are single pieces of themselves. */
+xpl_status xpl_diagnose_partials(xpl_ctx* ctx, const xpl_diag_params* params,
+                                 const xpl_name* names, size_t n_names, xpl_partial* out,
+                                 size_t cap, size_t* n_out, int reset);
+
+/* Combine the partials of all ranks (host only, no GPU needed): one report per
+ * logical allocation, in logical id order -- byte-identical to the report of
+ * the unsharded allocation.  INVALID_ARG if the pieces do not tile their
+ * logical allocation; *n_out = reports needed if cap is too small. */
+xpl_status xpl_combine_partials(const xpl_partial* parts, size_t n, const xpl_diag_params* params,
+                                xpl_alloc_report* out, size_t cap, size_t* n_out);
+
 /* The device-side context the __device__ hooks of xpl_device.cuh use: copies
  * it into *out (a host struct of device pointers; valid until xpl_finalize). */
 xpl_status xpl_get_device_ctx(xpl_ctx* ctx, struct xpl_dev_ctx* out);

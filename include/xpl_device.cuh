@@ -160,31 +160,45 @@ static __device__ __forceinline__ void xpl_dev_apply(unsigned long long g0,
   }
 }
 
-/* Lookup + apply.  size in bytes; acc = XPL_ACC_R / _W / _RW. */
+/* Lookup + apply.  size in bytes; acc = XPL_ACC_R / _W / _RW.
+ * A per-warp cache of the last row found (in shared memory, 32 slots per
+ * block, validated against the row on every use, so stale or uninitialised
+ * slots only cost the full search) skips the binary search when consecutive
+ * accesses of a warp hit the same allocation -- the common case. */
 static __device__ __forceinline__ void xpl_dev_record(const void* p, unsigned size,
                                                       unsigned acc) {
 #ifndef XPL_OFF
+  __shared__ unsigned xpl_row_cache[32];
   const unsigned long long a = (unsigned long long)p;
   const xpl_dev_row* rows = xpl_dctx.rows;
-  unsigned lo = 0, hi = __ldg(xpl_dctx.n_rows);
-  while (lo < hi) {
-    const unsigned mid = (lo + hi) >> 1;
-    if (__ldg(&rows[mid].base) <= a) lo = mid + 1;
-    else hi = mid;
+  const unsigned n = __ldg(xpl_dctx.n_rows);
+  const unsigned slot = ((threadIdx.z * blockDim.y + threadIdx.y) * blockDim.x + threadIdx.x) >> 5 & 31;
+  unsigned ri = xpl_row_cache[slot];
+  bool hit = ri < n && __ldg(&rows[ri].base) <= a && a < __ldg(&rows[ri].end);
+  if (!hit) {
+    unsigned lo = 0, hi = n;
+    while (lo < hi) {
+      const unsigned mid = (lo + hi) >> 1;
+      if (__ldg(&rows[mid].base) <= a) lo = mid + 1;
+      else hi = mid;
+    }
+    if (lo > 0 && a < __ldg(&rows[lo - 1].end)) {
+      ri = lo - 1;
+      hit = true;
+      xpl_row_cache[slot] = ri;  /* benign race: any lane's row is a valid entry */
+    }
   }
   unsigned long long g0 = 1, g1 = 0;
-  if (lo > 0 && size > 0) {
-    const xpl_dev_row* r = rows + (lo - 1);
+  if (hit && size > 0) {
+    const xpl_dev_row* r = rows + ri;
     const unsigned long long base = __ldg(&r->base);
-    if (a < __ldg(&r->end)) {
-      const unsigned long long w0 = (a - base) >> 2;
-      unsigned long long wl = (a + size - 1 - base) >> 2;
-      const unsigned long long wmax = __ldg(&r->words) - 1;
-      if (wl > wmax) wl = wmax;
-      const unsigned long long off = __ldg(&r->off);
-      g0 = off + w0;
-      g1 = off + wl;
-    }
+    const unsigned long long w0 = (a - base) >> 2;
+    unsigned long long wl = (a + size - 1 - base) >> 2;
+    const unsigned long long wmax = __ldg(&r->words) - 1;
+    if (wl > wmax) wl = wmax;
+    const unsigned long long off = __ldg(&r->off);
+    g0 = off + w0;
+    g1 = off + wl;
   }
   xpl_dev_apply(g0, g1, acc);
 #else

@@ -388,8 +388,50 @@ __device__ __noinline__ RunSum run_step_mixed(RunSum a, const uint32_t* bits, ui
   return rs_combine32(a, warp_runs(m, lane, min_run), min_run);
 }
 
+// rw = logical word of the lane's first word; blk = counters of this row, the
+// first one being logical block goff / B.
+// The step holding the row's end: the exact summary of its first n words (no
+// padding words, so a run reaching the row end stays open -- what a piece of a
+// sharded allocation needs).  Streams the 32 lane masks; rare (once per row).
+__device__ __noinline__ RunSum run_step_exact(RunSum a, const uint32_t* bits, uint32_t shift,
+                                              uint32_t n, uint32_t min_run) {
+  const uint32_t m = pack4(bits[0] >> shift) | (pack4(bits[1] >> shift) << 4) |
+                     (pack4(bits[2] >> shift) << 8) | (pack4(bits[3] >> shift) << 12);
+  uint32_t pre = 0, run = 0, cnt = 0, sum = 0;
+  bool seen_zero = false;
+  for (uint32_t l = 0; l < 32; ++l) {
+    const uint32_t ml = __shfl_sync(0xFFFFFFFFu, m, l);
+    for (uint32_t k = 0; k < 16; ++k) {
+      if (l * 16 + k >= n) break;
+      if ((ml >> k) & 1u) {
+        ++run;
+      } else {
+        if (!seen_zero) {
+          pre = run;
+          seen_zero = true;
+        } else if (run >= min_run && run > 0) {
+          ++cnt;
+          sum += run;
+        }
+        run = 0;
+      }
+    }
+  }
+  RunSum b;
+  b.len = n;
+  if (!seen_zero) {
+    b.pre = b.suf = n;
+  } else {
+    b.pre = pre;
+    b.suf = run;
+  }
+  b.cnt = cnt;
+  b.sum = sum;
+  return rs_combine32(a, b, min_run);
+}
+
 __device__ __noinline__ void block_counts(uint32_t f0, uint32_t f1, uint32_t f2, uint32_t f3,
-                                          uint64_t rw, uint64_t B, uint32_t* blk) {
+                                          uint64_t rw, uint64_t B, uint32_t* blk, uint64_t kb0) {
   const uint32_t g = ((f0 >> 6) & kL4) | (((f1 >> 6) & kL4) << 1) | (((f2 >> 6) & kL4) << 2) |
                      (((f3 >> 6) & kL4) << 3);
   uint32_t gm = 0;  // bit i = GPU-accessed flag of word rw + i
@@ -406,7 +448,7 @@ __device__ __noinline__ void block_counts(uint32_t f0, uint32_t f1, uint32_t f2,
     const uint32_t lo = (uint32_t)(a - rw), hi = (uint32_t)(be - rw);
     const uint32_t seg = ((hi >= 32 ? 0xFFFFFFFFu : ((1u << hi) - 1u)) & ~((1u << lo) - 1u));
     const uint32_t c = __popc(gm & seg);
-    if (c) atomicAdd(blk + k, c);
+    if (c) atomicAdd(blk + (k - kb0), c);
     a = be;
   }
 }
@@ -420,7 +462,7 @@ struct TileAcc {
 template <bool TAIL, bool RESET, bool BLOCKS>
 __device__ __forceinline__ void tile_step(TileAcc& A, uint4 y, uint4* dst, uint32_t w, uint32_t live,
                                           uint32_t lane, uint32_t min_run, uint64_t rw0,
-                                          uint64_t B, uint32_t* blk) {
+                                          uint64_t B, uint32_t* blk, uint64_t kb0) {
   uint32_t x[4] = {y.x, y.y, y.z, y.w};
   uint32_t keep[4] = {kL4, kL4, kL4, kL4};
   if (TAIL && w + 16 > live) {  // mask the words past the row's end
@@ -445,6 +487,13 @@ __device__ __forceinline__ void tile_step(TileAcc& A, uint4 y, uint4* dst, uint3
     uu[c] = x[c] & ~(x[c] >> 4) & 0x04040404u;
     dd[c] = x[c] & 0x10101010u;
   }
+  const uint32_t step0 = w - lane * 16;  // first (warp-relative) word of this 512-word step
+  if (TAIL && step0 + 512 > live) {      // the row ends in (or before) this step
+    if (step0 < live) {
+      A.wu = run_step_exact(A.wu, uu, 2, live - step0, min_run);
+      A.wd = run_step_exact(A.wd, dd, 4, live - step0, min_run);
+    }
+  } else {
   if (__ballot_sync(0xFFFFFFFFu, (uu[0] | uu[1] | uu[2] | uu[3]) != 0) == 0)
     rs_append_zero(A.wu, min_run);
   else if (__all_sync(0xFFFFFFFFu, (uu[0] & uu[1] & uu[2] & uu[3]) == 0x04040404u))
@@ -457,7 +506,8 @@ __device__ __forceinline__ void tile_step(TileAcc& A, uint4 y, uint4* dst, uint3
     rs_append_full(A.wd);
   else
     A.wd = run_step_mixed(A.wd, dd, 4, lane, min_run);
-  if (BLOCKS && (!TAIL || w < live)) block_counts(f0, f1, f2, f3, rw0 + w, B, blk);
+  }
+  if (BLOCKS && (!TAIL || w < live)) block_counts(f0, f1, f2, f3, rw0 + w, B, blk, kb0);
   // fused reset (D4): keep L only, words of this row only
   if (RESET && (!TAIL || w < live)) {
     if (((y.x & ~keep[0]) | (y.y & ~keep[1]) | (y.z & ~keep[2]) | (y.w & ~keep[3])) != 0)
@@ -467,7 +517,8 @@ __device__ __forceinline__ void tile_step(TileAcc& A, uint4 y, uint4* dst, uint3
 
 template <bool TAIL, bool RESET, bool BLOCKS>
 __device__ __forceinline__ void tile_loop(TileAcc& A, uint4* p4, uint32_t live, uint32_t lane,
-                                          uint32_t min_run, uint64_t rw0, uint64_t B, uint32_t* blk) {
+                                          uint32_t min_run, uint64_t rw0, uint64_t B, uint32_t* blk,
+                                          uint64_t kb0 = 0) {
   // 2-step software pipeline: the next two 512-word steps are in flight while
   // the current two are processed (a small loop body for the instruction cache)
   auto ld = [&](uint32_t it) {
@@ -479,9 +530,9 @@ __device__ __forceinline__ void tile_loop(TileAcc& A, uint4* p4, uint32_t live, 
   for (uint32_t it = 0; it < kDiagIters; it += 2) {
     const uint4 na = ld(it + 2), nb = ld(it + 3);
     tile_step<TAIL, RESET, BLOCKS>(A, a, p4 + it * 32 + lane, it * 512 + lane * 16, live, lane,
-                                   min_run, rw0, B, blk);
+                                   min_run, rw0, B, blk, kb0);
     tile_step<TAIL, RESET, BLOCKS>(A, b, p4 + (it + 1) * 32 + lane, (it + 1) * 512 + lane * 16,
-                                   live, lane, min_run, rw0, B, blk);
+                                   live, lane, min_run, rw0, B, blk, kb0);
     a = na;
     b = nb;
   }
@@ -511,9 +562,10 @@ __global__ void __launch_bounds__(kDiagThreads, 6) diag_tile_kernel(
   uint32_t* blk = blk_cnt + row.blk0;
   TileAcc A;
   const bool tail = live < kWarpWords;
-  if (p.block_words) {  // rare: blocks need per-lane counter atomics
-    if (p.reset) tile_loop<true, true, true>(A, p4, live, lane, min_run, ww0, p.block_words, blk);
-    else tile_loop<true, false, true>(A, p4, live, lane, min_run, ww0, p.block_words, blk);
+  if (p.block_words) {  // rare: blocks need per-lane counter atomics (logical block index)
+    const uint64_t kb0 = row.goff / p.block_words;
+    if (p.reset) tile_loop<true, true, true>(A, p4, live, lane, min_run, row.goff + ww0, p.block_words, blk, kb0);
+    else tile_loop<true, false, true>(A, p4, live, lane, min_run, row.goff + ww0, p.block_words, blk, kb0);
   } else if (p.reset) {
     if (tail) tile_loop<true, true, false>(A, p4, live, lane, min_run, ww0, 0, blk);
     else tile_loop<false, true, false>(A, p4, live, lane, min_run, ww0, 0, blk);
@@ -624,7 +676,9 @@ __global__ void stitch_seg_kernel(const StitchSeg* __restrict__ segs, uint32_t n
 __global__ void stitch_row_finalize_kernel(const DiagRow* __restrict__ rows, uint32_t nrows,
                                            const RunPair* __restrict__ segsum, DiagParams p,
                                            unsigned long long* __restrict__ cnt,
-                                           xpl_alloc_report* __restrict__ out) {
+                                           xpl_alloc_report* __restrict__ out,
+                                           RowPartial* __restrict__ parts,
+                                           const uint32_t* __restrict__ blk_cnt) {
   const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const uint32_t lane = threadIdx.x & 31;
   if (gw >= nrows) return;
@@ -639,6 +693,13 @@ __global__ void stitch_row_finalize_kernel(const DiagRow* __restrict__ rows, uin
   }
   warp_combine(a, b, lane, p.min_run);
   if (lane != 0) return;
+  if (parts) {
+    RowPartial& q = parts[gw];
+    q.u[0] = a.len; q.u[1] = a.pre; q.u[2] = a.suf; q.u[3] = a.cnt; q.u[4] = a.sum;
+    q.d[0] = b.len; q.d[1] = b.pre; q.d[2] = b.suf; q.d[3] = b.cnt; q.d[4] = b.sum;
+    q.blk_first_g = (p.block_words && r.nblk) ? blk_cnt[r.blk0] : 0;
+    q.blk_last_g = (p.block_words && r.nblk) ? blk_cnt[r.blk0 + r.nblk - 1] : 0;
+  }
   const unsigned long long* c = cnt + (uint64_t)gw * C_NCNT;
   xpl_alloc_report o;
   o.id = o.base = o.bytes = 0;
@@ -699,8 +760,9 @@ __global__ void block_eval_kernel(const DiagRow* __restrict__ rows, uint32_t nro
       else hi = mid;
     }
     const DiagRow r = rows[lo];
-    const uint64_t k = j - r.blk0;
-    const uint64_t s = min(B, r.words - k * B);
+    const uint64_t k = r.goff / B + (j - r.blk0);  // logical block
+    const uint64_t s = min(B, r.lwords - k * B);   // its size in the logical allocation
+    if (k * B < r.goff || k * B + s > r.goff + r.words) continue;  // cut by the piece: combined later
     if (100ull * g <= (uint64_t)thr * s) {
       atomicAdd(cnt + (uint64_t)lo * C_NCNT + C_LDB, 1ull);
       atomicAdd(cnt + (uint64_t)lo * C_NCNT + C_LDW, (unsigned long long)s);
@@ -746,8 +808,8 @@ void launch_range(cudaStream_t s, const RangeDesc* d_ranges, uint32_t nr, uint64
 void launch_diag(cudaStream_t s, const DiagRow* rows, uint32_t nrows, const uint32_t* tile_row,
                  uint64_t ntiles, const StitchSeg* segs, uint32_t nseg, uint64_t nblocks,
                  const DiagParams& p, uint32_t* pool, unsigned long long* cnt, TileSum* tiles,
-                 void* segsum, uint32_t* blk_cnt, xpl_alloc_report* out, cudaEvent_t tile_ev0,
-                 cudaEvent_t tile_ev1) {
+                 void* segsum, uint32_t* blk_cnt, xpl_alloc_report* out, RowPartial* parts,
+                 cudaEvent_t tile_ev0, cudaEvent_t tile_ev1) {
   cudaMemsetAsync(cnt, 0, sizeof(unsigned long long) * C_NCNT * nrows, s);
   if (p.block_words && nblocks) cudaMemsetAsync(blk_cnt, 0, sizeof(uint32_t) * nblocks, s);
   if (tile_ev0) cudaEventRecord(tile_ev0, s);
@@ -759,7 +821,7 @@ void launch_diag(cudaStream_t s, const DiagRow* rows, uint32_t nrows, const uint
   stitch_seg_kernel<<<(nseg * 32 + 255) / 256, 256, 0, s>>>(segs, nseg, tiles, p.min_run,
                                                              (RunPair*)segsum);
   stitch_row_finalize_kernel<<<(nrows * 32 + 255) / 256, 256, 0, s>>>(rows, nrows, (const RunPair*)segsum,
-                                                                       p, cnt, out);
+                                                                       p, cnt, out, parts, blk_cnt);
 }
 
 void launch_fill_u32(cudaStream_t s, uint32_t* p, uint64_t n, uint32_t v) {

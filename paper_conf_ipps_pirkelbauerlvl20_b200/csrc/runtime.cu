@@ -26,6 +26,7 @@ namespace {
 
 struct Row {
   uint64_t id, base, bytes, words, off, span;  // span = pool words reserved
+  uint64_t logical_id, goff, lbytes;           // sharded pieces (else id, 0, bytes)
   uint32_t kind;
   bool live, dropped, ever;
 };
@@ -143,6 +144,9 @@ struct xpl_ctx {
   unsigned long long* d_cnt = nullptr;
   xpl_alloc_report* d_rep = nullptr;
   xpl_alloc_report* h_rep = nullptr;
+  RowPartial* d_rpart = nullptr;
+  RowPartial* h_rpart = nullptr;
+  unsigned long long* h_cnt = nullptr;
 
   xpl_stats st;
 
@@ -590,6 +594,9 @@ xpl_status xpl_finalize(xpl_ctx* c) {
   cudaFree(c->d_cnt);
   cudaFree(c->d_rep);
   cudaFreeHost(c->h_rep);
+  cudaFree(c->d_rpart);
+  cudaFreeHost(c->h_rpart);
+  cudaFreeHost(c->h_cnt);
   for (cudaEvent_t e : c->ev_pool) cudaEventDestroy(e);
   for (cudaEvent_t e : c->prof_free) cudaEventDestroy(e);
   for (auto& r : c->prof_pending) {
@@ -606,8 +613,10 @@ xpl_status xpl_finalize(xpl_ctx* c) {
   return XPL_OK;
 }
 
-xpl_status xpl_register_alloc(xpl_ctx* c, const void* ptr, size_t bytes, xpl_alloc_kind kind) {
+static xpl_status register_row(xpl_ctx* c, const void* ptr, size_t bytes, xpl_alloc_kind kind,
+                               bool piece, uint64_t logical_id, uint64_t goff, uint64_t lbytes) {
   if (!c || !ptr || bytes == 0 || (unsigned)kind > 2) return XPL_ERR_INVALID_ARG;
+  if (piece && (lbytes == 0 || goff + (bytes + 3) / 4 > (lbytes + 3) / 4)) return XPL_ERR_INVALID_ARG;
   if (c->depth) return XPL_ERR_STATE;
   const uint64_t p = (uint64_t)ptr;
   auto it = c->live.lower_bound(p);
@@ -628,6 +637,9 @@ xpl_status xpl_register_alloc(xpl_ctx* c, const void* ptr, size_t bytes, xpl_all
   r.live = true;
   r.dropped = false;
   r.ever = false;
+  r.logical_id = piece ? logical_id : r.id;
+  r.goff = piece ? goff : 0;
+  r.lbytes = piece ? lbytes : bytes;
   if (!c->pa.alloc(r.span, &r.off)) return XPL_ERR_OOM;
   CK(cudaMemsetAsync(c->d_pool + r.off, 0, r.span, c->rs));  // D3: last writer = CPU
   const size_t cap_before = c->rows.capacity();
@@ -637,6 +649,15 @@ xpl_status xpl_register_alloc(xpl_ctx* c, const void* ptr, size_t bytes, xpl_all
   c->table_dirty = true;
   c->cache = nullptr;
   return XPL_OK;
+}
+
+xpl_status xpl_register_alloc(xpl_ctx* c, const void* ptr, size_t bytes, xpl_alloc_kind kind) {
+  return register_row(c, ptr, bytes, kind, false, 0, 0, 0);
+}
+
+xpl_status xpl_register_alloc_piece(xpl_ctx* c, const void* ptr, size_t bytes, xpl_alloc_kind kind,
+                                    uint64_t logical_id, uint64_t word_offset, uint64_t logical_bytes) {
+  return register_row(c, ptr, bytes, kind, true, logical_id, word_offset, logical_bytes);
 }
 
 xpl_status xpl_free(xpl_ctx* c, const void* ptr) {
@@ -894,9 +915,11 @@ xpl_status xpl_shadow_dump(xpl_ctx* c, const void* base, uint64_t word0, uint64_
   return XPL_OK;
 }
 
-xpl_status xpl_diagnose(xpl_ctx* c, const xpl_diag_params* params, const xpl_name* names,
-                        size_t n_names, xpl_alloc_report* out, size_t cap, size_t* n_out,
-                        int reset) {
+// The diagnosis of every live row and every row freed since the last reset
+// (tracePrint).  Fills `out` (reports) or `pout` (sharding partials).
+static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const xpl_name* names,
+                                size_t n_names, xpl_alloc_report* out, xpl_partial* pout, size_t cap,
+                                size_t* n_out, int reset) {
   if (!c || !n_out || (n_names && !names)) return XPL_ERR_INVALID_ARG;
   if (c->depth) return XPL_ERR_STATE;
   DiagParams p;
@@ -905,12 +928,13 @@ xpl_status xpl_diagnose(xpl_ctx* c, const xpl_diag_params* params, const xpl_nam
   p.min_run = params ? params->min_run_words : 256;
   if (p.min_run == 0) p.min_run = 1;
   p.reset = reset ? 1 : 0;
+  const uint64_t B = p.block_words;
 
   std::vector<uint64_t> ids;  // live rows + rows freed since the last reset, id order (D23)
   for (const Row& r : c->rows)
     if (r.live || !r.dropped) ids.push_back(r.id);
   *n_out = ids.size();
-  if (cap < ids.size() || (!out && ids.size())) return XPL_ERR_INVALID_ARG;
+  if (cap < ids.size() || (!out && !pout && ids.size())) return XPL_ERR_INVALID_ARG;
 
   xpl_status s = flush(c);
   if (s) return s;
@@ -918,6 +942,9 @@ xpl_status xpl_diagnose(xpl_ctx* c, const xpl_diag_params* params, const xpl_nam
   c->st.diagnoses++;
   if (nr == 0) return XPL_OK;
 
+  auto row_blocks = [&](const Row& r) -> uint64_t {  // logical blocks the row touches
+    return B ? (r.goff + r.words - 1) / B - r.goff / B + 1 : 0;
+  };
   // geometry
   uint64_t ntiles = 0, nblocks = 0, nseg = 0;
   for (uint64_t id : ids) {
@@ -925,7 +952,7 @@ xpl_status xpl_diagnose(xpl_ctx* c, const xpl_diag_params* params, const xpl_nam
     const uint64_t nt = (r.words + kTileWords - 1) / kTileWords;
     ntiles += nt;
     nseg += (nt + kSegTiles - 1) / kSegTiles;
-    if (p.block_words) nblocks += (r.words + p.block_words - 1) / p.block_words;
+    nblocks += row_blocks(r);
   }
   if (ntiles > 0x7FFFFFFFull) return XPL_ERR_OOM;
   if (nr > c->drows_cap) {
@@ -934,12 +961,18 @@ xpl_status xpl_diagnose(xpl_ctx* c, const xpl_diag_params* params, const xpl_nam
     cudaFree(c->d_cnt);
     cudaFree(c->d_rep);
     cudaFreeHost(c->h_rep);
+    cudaFree(c->d_rpart);
+    cudaFreeHost(c->h_rpart);
+    cudaFreeHost(c->h_cnt);
     c->drows_cap = std::max<size_t>(nr, 256);
     CK(host_alloc(&c->h_drows, c->drows_cap));
     CK(cudaMalloc(&c->d_drows, sizeof(DiagRow) * c->drows_cap));
     CK(cudaMalloc(&c->d_cnt, sizeof(unsigned long long) * C_NCNT * c->drows_cap));
     CK(cudaMalloc(&c->d_rep, sizeof(xpl_alloc_report) * c->drows_cap));
     CK(host_alloc(&c->h_rep, c->drows_cap));
+    CK(cudaMalloc(&c->d_rpart, sizeof(RowPartial) * c->drows_cap));
+    CK(host_alloc(&c->h_rpart, c->drows_cap));
+    CK(host_alloc(&c->h_cnt, C_NCNT * c->drows_cap));
   }
   if (ntiles > c->tiles_cap) {
     cudaFreeHost(c->h_tile_row);
@@ -973,7 +1006,9 @@ xpl_status xpl_diagnose(xpl_ctx* c, const xpl_diag_params* params, const xpl_nam
     d.tile0 = t;
     d.ntiles = (r.words + kTileWords - 1) / kTileWords;
     d.blk0 = b;
-    d.nblk = p.block_words ? (r.words + p.block_words - 1) / p.block_words : 0;
+    d.nblk = row_blocks(r);
+    d.goff = r.goff;
+    d.lwords = (r.lbytes + 3) / 4;
     d.kind = r.kind;
     d.pad = 0;
     d.seg0 = sgi;
@@ -998,33 +1033,88 @@ xpl_status xpl_diagnose(xpl_ctx* c, const xpl_diag_params* params, const xpl_nam
   const int ptile = prof_begin(c, XPL_K_DIAG_TILE, dbytes, false);  // recorded by launch_diag
   launch_diag(c->rs, c->d_drows, (uint32_t)nr, c->d_tile_row, ntiles, c->d_segs, (uint32_t)nseg,
               nblocks, p, (uint32_t*)c->d_pool, c->d_cnt, c->d_tiles, c->d_segsum, c->d_blk, c->d_rep,
-              ptile >= 0 ? c->prof_pending[ptile].a : nullptr,
+              pout ? c->d_rpart : nullptr, ptile >= 0 ? c->prof_pending[ptile].a : nullptr,
               ptile >= 0 ? c->prof_pending[ptile].b : nullptr);
   CK(cudaGetLastError());
-  c->st.kernel_launches += 3 + (p.block_words && nblocks ? 1 : 0);
+  c->st.kernel_launches += 3 + (B && nblocks ? 1 : 0);
   CK(cudaMemcpyAsync(c->h_rep, c->d_rep, sizeof(xpl_alloc_report) * nr, cudaMemcpyDeviceToHost, c->rs));
+  if (pout) {
+    CK(cudaMemcpyAsync(c->h_rpart, c->d_rpart, sizeof(RowPartial) * nr, cudaMemcpyDeviceToHost, c->rs));
+    CK(cudaMemcpyAsync(c->h_cnt, c->d_cnt, sizeof(unsigned long long) * C_NCNT * nr,
+                       cudaMemcpyDeviceToHost, c->rs));
+  }
   prof_end(c, pall);
   CK(cudaStreamSynchronize(c->rs));
 
-  for (size_t i = 0; i < nr; ++i) {
-    Row& r = c->rows[ids[i]];
-    xpl_alloc_report o = c->h_rep[i];
-    o.id = r.id;
-    o.base = r.base;
-    o.bytes = r.bytes;
-    o.live = r.live ? 1 : 0;
-    o.name_idx = 0xFFFFFFFFu;
-    if (o.any_acc) r.ever = true;
-    o.ever_accessed = r.ever ? 1 : 0;
-    out[i] = o;
-  }
-  // names (XplAllocData): the first name inside a live row
-  c->cache = nullptr;
+  std::vector<uint32_t> name_of(nr, 0xFFFFFFFFu);
+  c->cache = nullptr;  // names (XplAllocData): the first name inside a live row
   for (size_t j = 0; j < n_names; ++j) {
     const Row* r = lookup(c, (uint64_t)names[j].addr);
     if (!r) continue;
     for (size_t i = 0; i < nr; ++i)
-      if (out[i].id == r->id && out[i].name_idx == 0xFFFFFFFFu) out[i].name_idx = (uint32_t)j;
+      if (ids[i] == r->id && name_of[i] == 0xFFFFFFFFu) name_of[i] = (uint32_t)j;
+  }
+  for (size_t i = 0; i < nr; ++i) {
+    Row& r = c->rows[ids[i]];
+    const xpl_alloc_report& h = c->h_rep[i];
+    if (h.any_acc) r.ever = true;
+    if (out) {
+      xpl_alloc_report o = h;
+      o.id = r.id;
+      o.base = r.base;
+      o.bytes = r.bytes;
+      o.live = r.live ? 1 : 0;
+      o.name_idx = name_of[i];
+      o.ever_accessed = r.ever ? 1 : 0;
+      out[i] = o;
+    }
+    if (pout) {
+      const DiagRow& d = c->h_drows[i];
+      const RowPartial& q = c->h_rpart[i];
+      const unsigned long long* cn = c->h_cnt + (uint64_t)C_NCNT * i;
+      xpl_partial o;
+      memset(&o, 0, sizeof o);
+      o.logical_id = r.logical_id;
+      o.word_offset = r.goff;
+      o.words = r.words;
+      o.logical_words = d.lwords;
+      o.logical_bytes = r.lbytes;
+      o.base = r.base;
+      o.kind = r.kind;
+      o.live = r.live ? 1 : 0;
+      o.name_idx = name_of[i];
+      for (int k = 0; k < 9; ++k) o.cnt[k] = cn[k];
+      for (int k = 0; k < 5; ++k) {
+        o.u_run[k] = q.u[k];
+        o.d_run[k] = q.d[k];
+      }
+      o.low_density_blocks = B ? cn[C_LDB] : 0;
+      o.low_density_words = B ? cn[C_LDW] : 0;
+      o.blk_first = o.blk_last = ~0ull;
+      if (B) {  // the blocks cut by the piece's ends are combined across pieces
+        const uint64_t k0 = r.goff / B, k1 = (r.goff + r.words - 1) / B;
+        auto cut = [&](uint64_t k) {
+          const uint64_t lo = k * B, hi = std::min(lo + B, d.lwords);
+          return lo < r.goff || hi > r.goff + r.words;
+        };
+        auto in_piece = [&](uint64_t k) {
+          const uint64_t lo = std::max(k * B, r.goff), hi = std::min(std::min(k * B + B, d.lwords), r.goff + r.words);
+          return hi - lo;
+        };
+        if (cut(k0)) {
+          o.blk_first = k0;
+          o.blk_first_g = q.blk_first_g;
+          o.blk_first_s = in_piece(k0);
+        }
+        if (k1 != k0 && cut(k1)) {
+          o.blk_last = k1;
+          o.blk_last_g = q.blk_last_g;
+          o.blk_last_s = in_piece(k1);
+        }
+      }
+      o.ever_accessed = r.ever ? 1 : 0;
+      pout[i] = o;
+    }
   }
   if (reset) {  // drop freed rows and recycle their shadow (D17)
     for (Row& r : c->rows) {
@@ -1036,6 +1126,18 @@ xpl_status xpl_diagnose(xpl_ctx* c, const xpl_diag_params* params, const xpl_nam
     c->n_dead = 0;
   }
   return XPL_OK;
+}
+
+xpl_status xpl_diagnose(xpl_ctx* c, const xpl_diag_params* params, const xpl_name* names,
+                        size_t n_names, xpl_alloc_report* out, size_t cap, size_t* n_out,
+                        int reset) {
+  return diagnose_impl(c, params, names, n_names, out, nullptr, cap, n_out, reset);
+}
+
+xpl_status xpl_diagnose_partials(xpl_ctx* c, const xpl_diag_params* params, const xpl_name* names,
+                                 size_t n_names, xpl_partial* out, size_t cap, size_t* n_out,
+                                 int reset) {
+  return diagnose_impl(c, params, names, n_names, nullptr, out, cap, n_out, reset);
 }
 
 }  // extern "C"

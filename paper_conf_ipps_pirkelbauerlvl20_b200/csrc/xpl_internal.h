@@ -52,7 +52,15 @@ struct DiagRow {        // one row to analyse (live or dead-since-last-reset)
   uint64_t blk0;        // first block-counter index (block_words > 0)
   uint64_t nblk;
   uint64_t seg0, nseg;  // its stitch segments
+  uint64_t goff;        // first logical word (pieces of a sharded allocation; else 0)
+  uint64_t lwords;      // logical words (== words unless sharded)
   uint32_t kind, pad;
+};
+
+// What a row contributes to a sharded diagnosis besides its counters.
+struct RowPartial {
+  uint64_t u[5], d[5];             // run summaries (len, pre, suf, cnt, sum)
+  uint64_t blk_first_g, blk_last_g;  // GPU words of the first / last block of the row
 };
 
 // Stitch segment: <= kSegTiles consecutive tiles of one row.
@@ -92,8 +100,8 @@ void launch_range(cudaStream_t s, const RangeDesc* d_ranges, uint32_t nr, uint64
 void launch_diag(cudaStream_t s, const DiagRow* rows, uint32_t nrows, const uint32_t* tile_row,
                  uint64_t ntiles, const StitchSeg* segs, uint32_t nseg, uint64_t nblocks,
                  const DiagParams& p, uint32_t* pool, unsigned long long* cnt, TileSum* tiles,
-                 void* segsum, uint32_t* blk_cnt, xpl_alloc_report* out, cudaEvent_t tile_ev0,
-                 cudaEvent_t tile_ev1);
+                 void* segsum, uint32_t* blk_cnt, xpl_alloc_report* out, RowPartial* parts,
+                 cudaEvent_t tile_ev0, cudaEvent_t tile_ev1);
 constexpr size_t kRunPairBytes = 80;  // sizeof(RunPair) in kernels.cu
 void launch_fill_u32(cudaStream_t s, uint32_t* p, uint64_t n, uint32_t v);
 

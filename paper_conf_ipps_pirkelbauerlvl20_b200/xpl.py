@@ -61,6 +61,15 @@ class XplAllocReport(C.Structure):
     _fields_ = REPORT_FIELDS
 
 
+class XplPartial(C.Structure):
+    _fields_ = [("logical_id", u64), ("word_offset", u64), ("words", u64), ("logical_words", u64),
+                ("logical_bytes", u64), ("base", u64), ("kind", u32), ("live", u32), ("name_idx", u32),
+                ("pad", u32), ("cnt", u64 * 9), ("u_run", u64 * 5), ("d_run", u64 * 5),
+                ("low_density_blocks", u64), ("low_density_words", u64), ("blk_first", u64),
+                ("blk_first_g", u64), ("blk_first_s", u64), ("blk_last", u64), ("blk_last_g", u64),
+                ("blk_last_s", u64), ("ever_accessed", u64)]
+
+
 class XplStats(C.Structure):
     _fields_ = [(n, u64) for n in ("epochs", "folds", "fold_chunks", "host_records",
                                    "host_records_packed", "merge_segments", "range_segments",
@@ -89,6 +98,11 @@ xpl_record_host_ranges = _sig("xpl_record_host_ranges", [vp, vp, sz])
 xpl_record_copy = _sig("xpl_record_copy", [vp, vp, vp, sz, i32])
 xpl_diagnose = _sig("xpl_diagnose", [vp, C.POINTER(XplDiagParams), C.POINTER(XplName), sz,
                                      C.POINTER(XplAllocReport), sz, C.POINTER(sz), i32])
+xpl_register_alloc_piece = _sig("xpl_register_alloc_piece", [vp, vp, sz, i32, u64, u64, u64])
+xpl_diagnose_partials = _sig("xpl_diagnose_partials", [vp, C.POINTER(XplDiagParams), C.POINTER(XplName), sz,
+                                                       C.POINTER(XplPartial), sz, C.POINTER(sz), i32])
+xpl_combine_partials = _sig("xpl_combine_partials", [C.POINTER(XplPartial), sz, C.POINTER(XplDiagParams),
+                                                     C.POINTER(XplAllocReport), sz, C.POINTER(sz)])
 xpl_get_device_ctx = _sig("xpl_get_device_ctx", [vp, C.POINTER(XplDevCtx)])
 xpl_shadow_dump = _sig("xpl_shadow_dump", [vp, vp, u64, u64, vp])
 xpl_flush = _sig("xpl_flush", [vp])
@@ -110,7 +124,7 @@ EXPORTED = ["xpl_init", "xpl_finalize", "xpl_register_alloc", "xpl_free", "xpl_k
             "xpl_kernel_end", "xpl_record_host", "xpl_record_host_ranges", "xpl_record_copy", "xpl_diagnose",
             "xpl_get_device_ctx", "xpl_shadow_dump", "xpl_flush", "xpl_sync",
             "xpl_runtime_stream", "xpl_get_stats", "xpl_status_string", "xpl_profile",
-            "xpl_profile_read"]
+            "xpl_profile_read", "xpl_register_alloc_piece", "xpl_diagnose_partials", "xpl_combine_partials"]
 
 if _work is not None:
     xplw_bind = _sig("xplw_bind", [vp], lib=_work)
@@ -139,6 +153,10 @@ class Context:
         self.h = h
         if _work is not None:
             check("xplw_bind", xplw_bind(self.h))
+
+    def bind(self):
+        """Point the instrumented kernels of libxplwork at this context."""
+        check("xplw_bind", xplw_bind(self.h))
 
     def close(self):
         if self.h:
@@ -194,6 +212,24 @@ class Context:
             check("xpl_diagnose", st)
             return [{f: getattr(out[i], f) for f, _ in REPORT_FIELDS} for i in range(n.value)]
 
+    def register_piece(self, ptr, nbytes, kind, logical_id, word_offset, logical_bytes):
+        check("xpl_register_alloc_piece",
+              xpl_register_alloc_piece(self.h, ptr, nbytes, kind, logical_id, word_offset, logical_bytes))
+
+    def diagnose_partials(self, thr=50, block_words=0, min_run=256, reset=True):
+        """This context's partials as raw bytes (what ranks exchange)."""
+        p = XplDiagParams(thr, block_words, min_run)
+        cap = 64
+        while True:
+            out = (XplPartial * cap)()
+            n = sz(0)
+            st = xpl_diagnose_partials(self.h, C.byref(p), None, 0, out, cap, C.byref(n), int(bool(reset)))
+            if st == 1 and n.value > cap:
+                cap = n.value
+                continue
+            check("xpl_diagnose_partials", st)
+            return bytes(memoryview(out).cast("B")[:n.value * C.sizeof(XplPartial)])
+
     def shadow_dump(self, base, word0, n):
         out = np.zeros(n, dtype=np.uint8)
         check("xpl_shadow_dump", xpl_shadow_dump(self.h, base, word0, n, out.ctypes.data))
@@ -238,3 +274,22 @@ class Context:
         if grid <= 0:
             grid = max(1, min((n + block - 1) // block, 148 * 8))
         check("xplw_replay", xplw_replay(d_addr, d_size, d_acc, n, grid, block, stream))
+
+
+def combine_partials(blobs, thr=50, block_words=0, min_run=256):
+    """Combine the partials of all ranks (list of byte blobs) into reports (host only)."""
+    raw = b"".join(blobs)
+    n = len(raw) // C.sizeof(XplPartial)
+    arr = (XplPartial * max(n, 1)).from_buffer_copy(raw if n else bytes(C.sizeof(XplPartial)))
+    p = XplDiagParams(thr, block_words, min_run)
+    cap = max(n, 1)
+    out = (XplAllocReport * cap)()
+    m = sz(0)
+    check("xpl_combine_partials", xpl_combine_partials(arr, n, C.byref(p), out, cap, C.byref(m)))
+    return [{f: getattr(out[i], f) for f, _ in REPORT_FIELDS} for i in range(m.value)]
+
+
+def partials_from_bytes(blob):
+    n = len(blob) // C.sizeof(XplPartial)
+    arr = (XplPartial * max(n, 1)).from_buffer_copy(blob if n else bytes(C.sizeof(XplPartial)))
+    return [arr[i] for i in range(n)]
