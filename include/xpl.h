@@ -216,6 +216,19 @@ xpl_status xpl_diagnose_partials(xpl_ctx* ctx, const xpl_diag_params* params,
 xpl_status xpl_combine_partials(const xpl_partial* parts, size_t n, const xpl_diag_params* params,
                                 xpl_alloc_report* out, size_t cap, size_t* n_out);
 
+/* tracePrint's output: format reports as the textual summary of
+ * Fig. 4 -- per allocation its name, write counts C G, read counts
+ * C>C C>G G>C G>G, access density, alternating elements and the anti-pattern
+ * findings -- or (csv != 0) as comma-separated raw counts with a header line.
+ * names/n_names: the XplAllocData list the reports' name_idx refer to (may be
+ * NULL); unnamed rows print as "alloc <id>".  only_named != 0 prints named rows
+ * only ("checking N named allocations").  Writes at most cap bytes including the
+ * terminating NUL into buf and sets *needed to the full length + 1; INVALID_ARG
+ * if it did not fit (the caller retries with a larger buffer). */
+xpl_status xpl_format_reports(const xpl_alloc_report* reps, size_t n, const xpl_name* names,
+                              size_t n_names, int csv, int only_named, char* buf, size_t cap,
+                              size_t* needed);
+
 /* The device-side context the __device__ hooks of xpl_device.cuh use: copies
  * it into *out (a host struct of device pointers; valid until xpl_finalize). */
 xpl_status xpl_get_device_ctx(xpl_ctx* ctx, struct xpl_dev_ctx* out);

@@ -103,6 +103,8 @@ xpl_diagnose_partials = _sig("xpl_diagnose_partials", [vp, C.POINTER(XplDiagPara
                                                        C.POINTER(XplPartial), sz, C.POINTER(sz), i32])
 xpl_combine_partials = _sig("xpl_combine_partials", [C.POINTER(XplPartial), sz, C.POINTER(XplDiagParams),
                                                      C.POINTER(XplAllocReport), sz, C.POINTER(sz)])
+xpl_format_reports = _sig("xpl_format_reports", [C.POINTER(XplAllocReport), sz, C.POINTER(XplName), sz, i32,
+                                                 i32, C.c_char_p, sz, C.POINTER(sz)])
 xpl_get_device_ctx = _sig("xpl_get_device_ctx", [vp, C.POINTER(XplDevCtx)])
 xpl_shadow_dump = _sig("xpl_shadow_dump", [vp, vp, u64, u64, vp])
 xpl_flush = _sig("xpl_flush", [vp])
@@ -124,7 +126,8 @@ EXPORTED = ["xpl_init", "xpl_finalize", "xpl_register_alloc", "xpl_free", "xpl_k
             "xpl_kernel_end", "xpl_record_host", "xpl_record_host_ranges", "xpl_record_copy", "xpl_diagnose",
             "xpl_get_device_ctx", "xpl_shadow_dump", "xpl_flush", "xpl_sync",
             "xpl_runtime_stream", "xpl_get_stats", "xpl_status_string", "xpl_profile",
-            "xpl_profile_read", "xpl_register_alloc_piece", "xpl_diagnose_partials", "xpl_combine_partials"]
+            "xpl_profile_read", "xpl_register_alloc_piece", "xpl_diagnose_partials", "xpl_combine_partials",
+            "xpl_format_reports"]
 
 if _work is not None:
     xplw_bind = _sig("xplw_bind", [vp], lib=_work)
@@ -293,3 +296,30 @@ def partials_from_bytes(blob):
     n = len(blob) // C.sizeof(XplPartial)
     arr = (XplPartial * max(n, 1)).from_buffer_copy(blob if n else bytes(C.sizeof(XplPartial)))
     return [arr[i] for i in range(n)]
+
+
+def format_reports(reports, names=(), csv=False, only_named=False):
+    """tracePrint's text (Fig. 4 layout) or CSV for report dicts; names: list of
+    (addr, expr) pairs the reports' name_idx refer to."""
+    n = len(reports)
+    arr = (XplAllocReport * max(n, 1))()
+    for i, r in enumerate(reports):
+        for f, _ in REPORT_FIELDS:
+            setattr(arr[i], f, r[f])
+    nm = (XplName * max(len(names), 1))()
+    keep = []
+    for i, (a, e) in enumerate(names):
+        b = e.encode()
+        keep.append(b)
+        nm[i].addr, nm[i].expr, nm[i].elem_size = a, b, 0
+    need = sz(0)
+    cap = 4096
+    while True:
+        buf = C.create_string_buffer(cap)
+        st = xpl_format_reports(arr, n, nm if names else None, len(names), int(csv), int(only_named),
+                                buf, cap, C.byref(need))
+        if st == 1 and need.value > cap:
+            cap = need.value
+            continue
+        check("xpl_format_reports", st)
+        return buf.value.decode()
