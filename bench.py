@@ -132,6 +132,66 @@ def cpu_baseline(seconds_budget=20.0):
                       f"with a diagnose after each ({n_acc} accesses, {dt:.1f} s, 1 thread)"}
 
 
+def diag_sharded(xpl, torch, dist, rank, world, words=1 << 31, reps=3, check_1gpu=True):
+    """Address-range sharding of the cfg5-sized shadow over the ranks:
+    rank r holds words [r*W/N, (r+1)*W/N) of one logical allocation, records its
+    part (H2D of the logical first half + the instrumented touch kernel with the
+    logical pattern), diagnoses into partials; the partials are all-gathered and
+    combined on every rank.  Timed: partial diagnose + exchange + combine, max over
+    ranks.  Rank 0 also diagnoses the unsharded allocation and checks the combined
+    report is byte-identical (shard-count invariance)."""
+    import time
+    chunk = -(-words // world)
+    goff = rank * chunk
+    n = max(0, min(words, goff + chunk) - goff)
+    base = 1 << 44
+    ctx = xpl.Context(pool_words=n + (1 << 16), max_rows=16)
+    s = torch.cuda.current_stream().cuda_stream
+    ctx.register_piece(base + 4 * goff, 4 * n, xpl.ALLOC_DEVICE, 0, goff, 4 * words)
+    h0, h1 = goff, min(goff + n, words // 2)
+    if h1 > h0:
+        ctx.record_copy(base + 4 * h0, 0x1000, 4 * (h1 - h0), xpl.COPY_H2D)
+    ctx.kernel_begin(s)
+    ctx.touch(base + 4 * goff, n, 7, s, goff)
+    ctx.kernel_end(s)
+    ctx.sync()
+    ms = []
+    got = None
+    for _ in range(reps):
+        dist.barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        blob = ctx.diagnose_partials(50, 0, 256, reset=False)
+        blobs = [None] * world
+        dist.all_gather_object(blobs, blob)
+        got = xpl.combine_partials(blobs, 50, 0, 256)
+        ms.append((time.perf_counter() - t0) * 1e3)
+    ctx.close()
+    dt = _allmax(torch, dist, min(ms))
+    out = {"words": words, "ranks": world, "ms": dt, "gbs": words / (dt / 1e3) / 1e9,
+           "note": "reset=0 (1 B/word); wall-clock of partial diagnose + all_gather + combine, max over ranks"}
+    if rank == 0 and check_1gpu:
+        ref = xpl.Context(pool_words=words + (1 << 16), max_rows=16)
+        ref.register(base, 4 * words, xpl.ALLOC_DEVICE)
+        ref.record_copy(base, 0x1000, 2 * words, xpl.COPY_H2D)
+        ref.kernel_begin(s)
+        ref.touch(base, words, 7, s, 0)
+        ref.kernel_end(s)
+        exp = ref.diagnose(50, 0, 256, reset=False)
+        ref.close()
+        out["identical_to_unsharded"] = exp == got
+    return out
+
+
+def _allmax(torch, dist, x):
+    if not dist.is_available() or not dist.is_initialized():
+        return x
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([x], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
 def diag_at_scale(xpl, torch, words=1 << 31, reps=3):
     """The diagnose pass over a cfg5-sized shadow (2^31 words = 2 GiB, SURVEY §8(d)
     cfg5 ~2.2e9 words) with a mixed realistic content: CPU-written half (H2D),
@@ -143,7 +203,7 @@ def diag_at_scale(xpl, torch, words=1 << 31, reps=3):
     ctx.record_copy(base, 0x1000, 2 * words, xpl.COPY_H2D)
     s = torch.cuda.current_stream().cuda_stream
     ctx.kernel_begin(s)
-    ctx.touch(base, words, 7, s)
+    ctx.touch(base, words, 7, s, 0)
     ctx.kernel_end(s)
     ctx.sync()
     torch.cuda.synchronize()
@@ -264,10 +324,14 @@ def main():
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0")) % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
+    backend = os.environ.get("XPL_DIST_BACKEND", "nccl")  # gloo: test the N>1 logic on one GPU
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
 
     from paper_conf_ipps_pirkelbauerlvl20_b200 import apps, xpl
     from xplgen import rodinia
@@ -348,11 +412,7 @@ def main():
     ctx.profile(False)
     st1 = ctx.stats()
     per_step = counts[0] + counts[1] + counts[2]
-    ms_max = ms_total
-    if world > 1:
-        t = torch.tensor([ms_total], device="cuda", dtype=torch.float64)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms_max = float(t.item())
+    ms_max = _allmax(torch, dist, ms_total)
     value = per_step * args.steps * world / (ms_max / 1e3)
     launches = (st1["kernel_launches"] - st0["kernel_launches"]) + counts[3] * args.steps
 
@@ -364,10 +424,7 @@ def main():
         dist.barrier()
     e2e_ms, _ = timed(ctx, True, args.steps, rs)
     st1 = ctx.stats()
-    if world > 1:
-        t = torch.tensor([e2e_ms], device="cuda", dtype=torch.float64)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        e2e_ms = float(t.item())
+    e2e_ms = _allmax(torch, dist, e2e_ms)
     rec_bytes = 8 * (st1["host_records_packed"] - st0["host_records_packed"]) // args.steps
     nwc = (NW[0] + 1) ** 2
     app_h2d = (4 * (2 * HOT[0] * HOT[1]) + 4 * ((BACKPROP[0] + 1) * (1 + 2 * (BACKPROP[1] + 1)) + BACKPROP[1] + 1)
@@ -393,6 +450,12 @@ def main():
 
     # --- the diagnose pass at cfg5 scale; the other configs -------------------
     at_scale = diag_at_scale(xpl, torch)
+    sharded = None
+    if world > 1:
+        try:
+            sharded = diag_sharded(xpl, torch, dist, rank, world)
+        except Exception as ex:  # keep the primary line even if this extra fails
+            sharded = {"error": repr(ex)}
     others = other_configs(xpl, apps, torch) if not args.no_other_configs else None
 
     # --- roofline of the dominant runtime kernel -------------------------------
@@ -432,6 +495,7 @@ def main():
                      "paper_context": "Table III P:L431-443: 5x-20x, avg ~15x (Intel E5-2695 v4 + Pascal, CUDA 9.2)"},
         "e2e": e2e, "gpu_launches": int(launches), "clocks": clocks,
         "other_configs": others,
+        "diagnose_sharded": sharded,
     }
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline()

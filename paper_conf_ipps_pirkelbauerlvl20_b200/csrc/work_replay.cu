@@ -32,9 +32,11 @@ __device__ __forceinline__ unsigned hash32(unsigned x) {
 // behind it: hooks only use addresses).  Per 4096-word block one of: untouched,
 // all read, all written, or a per-word random R/W/RW mix -- long runs and
 // mixed regions, like a real shadow.
-__global__ void touch_kernel(unsigned long long base, unsigned long long n, unsigned seed) {
-  for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
-       i += (unsigned long long)gridDim.x * blockDim.x) {
+__global__ void touch_kernel(unsigned long long base, unsigned long long n, unsigned seed,
+                             unsigned long long i0) {
+  for (unsigned long long j = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; j < n;
+       j += (unsigned long long)gridDim.x * blockDim.x) {
+    const unsigned long long i = i0 + j;  // the pattern is a function of the logical word
     const unsigned hb = hash32((unsigned)(i >> 12) ^ seed);
     unsigned acc = 0;
     switch (hb & 3) {
@@ -47,7 +49,7 @@ __global__ void touch_kernel(unsigned long long base, unsigned long long n, unsi
       }
       default: break;
     }
-    if (acc) xpl_dev_record((const void*)(base + 4 * i), 4, acc);
+    if (acc) xpl_dev_record((const void*)(base + 4 * j), 4, acc);
   }
 }
 
@@ -55,9 +57,11 @@ __global__ void touch_kernel(unsigned long long base, unsigned long long n, unsi
 
 extern "C" {
 
-// Launch the synthetic touch kernel (between xpl_kernel_begin/_end).
-int xplw_touch(unsigned long long base, unsigned long long n, unsigned seed, void* stream) {
-  touch_kernel<<<148 * 16, 256, 0, (cudaStream_t)stream>>>(base, n, seed);
+// Launch the synthetic touch kernel (between xpl_kernel_begin/_end) over the n
+// words at base, which are logical words i0 .. i0+n-1 of the pattern.
+int xplw_touch(unsigned long long base, unsigned long long n, unsigned seed, void* stream,
+               unsigned long long i0) {
+  touch_kernel<<<148 * 16, 256, 0, (cudaStream_t)stream>>>(base, n, seed, i0);
   return cudaGetLastError() == cudaSuccess ? 0 : (int)XPL_ERR_CUDA;
 }
 

@@ -132,7 +132,7 @@ EXPORTED = ["xpl_init", "xpl_finalize", "xpl_register_alloc", "xpl_free", "xpl_k
 if _work is not None:
     xplw_bind = _sig("xplw_bind", [vp], lib=_work)
     xplw_replay = _sig("xplw_replay", [vp, vp, vp, u64, i32, i32, vp], lib=_work)
-    xplw_touch = _sig("xplw_touch", [u64, u64, u32, vp], lib=_work)
+    xplw_touch = _sig("xplw_touch", [u64, u64, u32, vp, u64], lib=_work)
 
 
 class XplError(RuntimeError):
@@ -268,9 +268,10 @@ class Context:
         check("xpl_get_device_ctx", xpl_get_device_ctx(self.h, C.byref(d)))
         return d
 
-    def touch(self, base, nwords, seed=1, stream=0):
-        """Launch the synthetic instrumented touch kernel (libxplwork) over nwords at base."""
-        check("xplw_touch", xplw_touch(base, nwords, seed, stream))
+    def touch(self, base, nwords, seed=1, stream=0, i0=0):
+        """Launch the synthetic instrumented touch kernel (libxplwork) over nwords at
+        base = logical words i0 .. i0+nwords-1 of its access pattern."""
+        check("xplw_touch", xplw_touch(base, nwords, seed, stream, i0))
 
     def replay(self, d_addr, d_size, d_acc, n, grid=0, block=256, stream=0):
         """Launch the instrumented replay kernel (libxplwork) on device arrays."""
