@@ -22,6 +22,18 @@
  * ranges (xpl_record_host_ranges) mean exactly what the individual accesses
  * mean -- for programs whose individual accesses never straddle two
  * allocations (every valid C/C++ object access; D28).
+ *
+ * Site hints.  An instrumenting tool knows the static access site; giving each
+ * site a local `xpl_host_site` (the run slot that site hit last) lets the fast
+ * path go straight to that run instead of through the shared "current run"
+ * prediction, so interleaved streams (a[i], b[i], c[i] in one loop body) do
+ * not form a dependency chain through the tracer's state:
+ *
+ *     xpl_host_site sa, sb;
+ *     for (i...) tr.write(a[i], sa) = tr.read(b[i], sb);
+ *
+ * A hint is only a starting point: whatever run it names is checked like any
+ * other, so a stale hint costs a slow-path call, never a wrong record.
  */
 #ifndef XPL_HOST_H
 #define XPL_HOST_H
@@ -32,6 +44,11 @@
 #include "xpl.h"
 
 #ifdef __cplusplus
+
+/* Per-access-site hint (a local of the instrumented code; see above). */
+struct xpl_host_site {
+  uint32_t slot = 0;
+};
 
 class xpl_host_tracer {
  public:
@@ -51,6 +68,28 @@ class xpl_host_tracer {
       return;
     }
     slow(a, size, kind);
+  }
+  /* The same access with a site hint: try the run the site used last. */
+  __attribute__((always_inline)) inline void access(const void* p, uint32_t size, uint32_t kind,
+                                                    xpl_host_site& s) {
+    const uint64_t a = (uint64_t)p;
+    if (hit(&run_[s.slot], a, size, kind)) return;
+    s.slot = slow(a, size, kind);
+  }
+  template <class T>
+  inline const T& read(const T& x, xpl_host_site& s) {
+    access(&x, sizeof(T), XPL_ACC_R, s);
+    return x;
+  }
+  template <class T>
+  inline T& write(T& x, xpl_host_site& s) {
+    access(&x, sizeof(T), XPL_ACC_W, s);
+    return x;
+  }
+  template <class T>
+  inline T& rw(T& x, xpl_host_site& s) {
+    access(&x, sizeof(T), XPL_ACC_RW, s);
+    return x;
   }
   template <class T>
   inline const T& read(const T& x) {
@@ -87,20 +126,21 @@ class xpl_host_tracer {
   static const size_t kBuf = 4096;
   struct Run {
     uint64_t beg = 0, end = 0;  // bytes [beg, end)
+    uint64_t end0 = 0;          // end when opened
     uint64_t limit = 0;         // word-aligned start of the next open run above (or max)
+    uint64_t cap = 0;           // min(limit, beg + kMaxRun): the run may grow up to here
     uint64_t seq = 0;           // opening order
     uint16_t kind = 0;          // 0 = slot free (16 bits: no aliasing with int/uint32 data)
-    uint16_t grew = 0;          // extended or repeated since opened
+    uint16_t grew = 0;          // repeated since opened (extension: end != end0)
     Run* next = nullptr;        // the run used after this one last time (a prediction)
   };
   /* The access joins run r (extension at its end, or a repeat inside it). */
   static inline bool hit(Run* r, uint64_t a, uint32_t size, uint32_t kind) {
     if (kind != r->kind) return false;
     if (a == r->end) {
-      if (a + size > r->limit || a + size - r->beg > kMaxRun) return false;
+      if (a + size > r->cap) return false;
       if (kind == XPL_ACC_RW && ((a | size) & 3u)) return false;
-      r->end = a + size;
-      r->grew = 1;
+      r->end = a + size;  // (growth is seen at close: end != end0)
       return true;
     }
     if (kind != XPL_ACC_RW && a >= r->beg && a + size <= r->end) {  // repeat (R or W)
@@ -119,6 +159,10 @@ class xpl_host_tracer {
     }
     n_ = 0;
   }
+  static void set_limit(Run& r, uint64_t lim) {
+    r.limit = lim;
+    r.cap = lim < r.beg + kMaxRun ? lim : r.beg + kMaxRun;
+  }
   void close(int i) {
     if (n_ == kBuf) drain();
     buf_[n_++] = xpl_host_access{run_[i].beg, (uint32_t)(run_[i].end - run_[i].beg), run_[i].kind};
@@ -126,7 +170,7 @@ class xpl_host_tracer {
     const uint64_t b = wlo(run_[i].beg);
     for (int j = 0; j < kRuns; ++j) {
       if (run_[j].next == &run_[i]) run_[j].next = nullptr;  // forget predictions into the slot
-      if (run_[j].kind && run_[j].limit == b) run_[j].limit = limit_of(j);  // it was the run above
+      if (run_[j].kind && run_[j].limit == b) set_limit(run_[j], limit_of(j));  // it was the run above
     }
     run_[i].next = nullptr;
   }
@@ -148,32 +192,31 @@ class xpl_host_tracer {
     if (cur_ != &run_[i]) cur_->next = &run_[i];
     cur_ = &run_[i];
   }
-  __attribute__((noinline)) void slow(uint64_t a, uint32_t size, uint32_t kind) {
+  /* Returns the slot that now holds the access (kRuns: emitted directly). */
+  __attribute__((noinline)) uint32_t slow(uint64_t a, uint32_t size, uint32_t kind) {
     const uint64_t lo = wlo(a), hi = whi(a + size);
     for (int k = 0; k < kRuns; ++k) {  // most recently used first: a run a starts in or right after
-      Run& r = run_[mru_[k]];
+      const uint32_t i = mru_[k];
+      Run& r = run_[i];
       if (r.kind != kind || a < r.beg || a > r.end) continue;
       if (kind != XPL_ACC_RW) {  // R / W: idempotent per word -> union
         if (a + size <= r.end) {  // repeat inside the run (its words are no other run's)
           r.grew = 1;
           churn_ = 0;
           touch(k);
-          return;
+          return i;
         }
-        if (a + size <= r.limit && a + size - r.beg <= kMaxRun) {
+        if (a + size <= r.cap) {
           r.end = a + size;
-          r.grew = 1;
           churn_ = 0;
           touch(k);
-          return;
+          return i;
         }
-      } else if (a == r.end && ((a | size) & 3u) == 0 && a + size <= r.limit &&
-                 a + size - r.beg <= kMaxRun) {
+      } else if (a == r.end && ((a | size) & 3u) == 0 && a + size <= r.cap) {
         r.end = a + size;
-        r.grew = 1;
         churn_ = 0;
         touch(k);
-        return;
+        return i;
       }
       break;
     }
@@ -190,7 +233,7 @@ class xpl_host_tracer {
     if (churn_ >= 32 && (++tick_ & 63) != 0) {
       if (n_ == kBuf) drain();
       buf_[n_++] = xpl_host_access{a, size, kind};
-      return;
+      return kRuns;
     }
     int slot = -1;
     for (int i = 0; i < kRuns && slot < 0; ++i)
@@ -199,27 +242,28 @@ class xpl_host_tracer {
       slot = 0;
       for (int i = 1; i < kRuns; ++i)
         if (run_[i].seq < run_[slot].seq) slot = i;
-      churn_ = run_[slot].grew ? 0 : churn_ + 1;
+      churn_ = (run_[slot].grew || run_[slot].end != run_[slot].end0) ? 0 : churn_ + 1;
       close(slot);
     }
     Run& r = run_[slot];
     r.beg = a;
-    r.end = a + size;
+    r.end = r.end0 = a + size;
     r.kind = (uint16_t)kind;
     r.grew = 0;
     r.seq = ++seq_;
-    r.limit = limit_of(slot);
+    set_limit(r, limit_of(slot));
     for (int j = 0; j < kRuns; ++j)  // runs below the new one may now grow only up to it
-      if (j != slot && run_[j].kind && whi(run_[j].end) <= lo && run_[j].limit > lo) run_[j].limit = lo;
+      if (j != slot && run_[j].kind && whi(run_[j].end) <= lo && run_[j].limit > lo) set_limit(run_[j], lo);
     for (int k = 0; k < kRuns; ++k)
       if (mru_[k] == slot) {
         touch(k);
         break;
       }
+    return (uint32_t)slot;
   }
 
   xpl_ctx* ctx_;
-  Run run_[kRuns];
+  Run run_[kRuns + 1];  // run_[kRuns]: never open (the hint of a directly emitted access)
   uint8_t mru_[kRuns] = {0, 1, 2, 3, 4, 5, 6, 7};  // run slots, most recently used first
   Run* cur_ = &run_[0];                              // == &run_[mru_[0]]
   uint64_t seq_ = 0;

@@ -81,8 +81,9 @@ struct App {
   template <class T>
   void write_loop(T* p, uint64_t n) {
     const auto t0 = std::chrono::steady_clock::now();
+    xpl_host_site st;  // one per static access site (xpl_host.h)
     if (tr)
-      for (uint64_t i = 0; i < n; ++i) tr->write(p[i]) = (T)(i & 1023) * (T)0.001;
+      for (uint64_t i = 0; i < n; ++i) tr->write(p[i], st) = (T)(i & 1023) * (T)0.001;
     else
       for (uint64_t i = 0; i < n; ++i) p[i] = (T)(i & 1023) * (T)0.001;
     run->host_accesses += n;
@@ -93,8 +94,9 @@ struct App {
   T read_loop(const T* p, uint64_t n, uint64_t stride = 1, uint64_t off = 0) {
     const auto t0 = std::chrono::steady_clock::now();
     T acc = 0;
+    xpl_host_site st;
     if (tr)
-      for (uint64_t i = 0; i < n; ++i) acc += tr->read(p[i * stride + off]);
+      for (uint64_t i = 0; i < n; ++i) acc += tr->read(p[i * stride + off], st);
     else
       for (uint64_t i = 0; i < n; ++i) acc += p[i * stride + off];
     run->host_accesses += n;
@@ -428,13 +430,14 @@ int xplw_bfs(xplw_run* run, const xplw_arrays* a, int n, int deg, unsigned long 
   // read the graph "file": node records, masks, edges, costs (Rodinia bfs.cu order)
   {
     const auto t0 = std::chrono::steady_clock::now();
+    xpl_host_site s0, s1, s2, s3, s4;
     for (int i = 0; i < n; i++) {
       if (app.tr) {
-        app.tr->write(h_nodes[i].starting) = i * deg;
-        app.tr->write(h_nodes[i].no_of_edges) = deg;
-        app.tr->write(h_mask[i]) = false;
-        app.tr->write(h_updating[i]) = false;
-        app.tr->write(h_visited[i]) = false;
+        app.tr->write(h_nodes[i].starting, s0) = i * deg;
+        app.tr->write(h_nodes[i].no_of_edges, s1) = deg;
+        app.tr->write(h_mask[i], s2) = false;
+        app.tr->write(h_updating[i], s3) = false;
+        app.tr->write(h_visited[i], s4) = false;
       } else {
         h_nodes[i].starting = i * deg;
         h_nodes[i].no_of_edges = deg;
@@ -453,12 +456,13 @@ int xplw_bfs(xplw_run* run, const xplw_arrays* a, int n, int deg, unsigned long 
   run->host_accesses += 2;
   {  // the edge list is stored as read from the input; costs -1, source 0
     const auto t0 = std::chrono::steady_clock::now();
+    xpl_host_site s0, s1;
     for (uint64_t i = 0; i < ne; ++i) {
       const int e = h_edges[i];  // (the input buffer; the traced store is the program's)
-      if (app.tr) app.tr->write(h_edges[i]) = e;
+      if (app.tr) app.tr->write(h_edges[i], s0) = e;
     }
     for (int i = 0; i < n; ++i) {
-      if (app.tr) app.tr->write(h_cost[i]) = -1;
+      if (app.tr) app.tr->write(h_cost[i], s1) = -1;
       else h_cost[i] = -1;
     }
     if (app.tr) app.tr->write(h_cost[0]) = 0;
@@ -517,11 +521,12 @@ int xplw_nw(xplw_run* run, const xplw_arrays* a, int n, int penalty, const int* 
   // the sequences (row / column 0) are the input; the substitution matrix from them
   {
     const auto t0 = std::chrono::steady_clock::now();
+    xpl_host_site s0, s1, s2, s3, s4;
     if (app.tr) {
       for (int i = 1; i < rows; i++)
         for (int j = 1; j < cols; j++) {
-          const int x = app.tr->read(in[i * cols]), y = app.tr->read(in[j]);
-          app.tr->write(refh[i * cols + j]) = blosum[x * 24 + y];
+          const int x = app.tr->read(in[i * cols], s0), y = app.tr->read(in[j], s1);
+          app.tr->write(refh[i * cols + j], s2) = blosum[x * 24 + y];
         }
     } else {
       for (int i = 1; i < rows; i++)
@@ -529,11 +534,11 @@ int xplw_nw(xplw_run* run, const xplw_arrays* a, int n, int penalty, const int* 
     }
     run->host_accesses += 3ull * (rows - 1) * (cols - 1);
     for (int i = 1; i < rows; i++) {
-      if (app.tr) app.tr->write(in[i * cols]) = -i * penalty;
+      if (app.tr) app.tr->write(in[i * cols], s3) = -i * penalty;
       else in[i * cols] = -i * penalty;
     }
     for (int j = 1; j < cols; j++) {
-      if (app.tr) app.tr->write(in[j]) = -j * penalty;
+      if (app.tr) app.tr->write(in[j], s4) = -j * penalty;
       else in[j] = -j * penalty;
     }
     run->host_accesses += (uint64_t)(rows - 1) + (cols - 1);
@@ -561,26 +566,27 @@ int xplw_nw(xplw_run* run, const xplw_arrays* a, int n, int penalty, const int* 
   {
     const auto t0 = std::chrono::steady_clock::now();
     const int LIMIT = -999;
-    auto R = [&](int* p) -> int {
+    xpl_host_site s_nw, s_w, s_n, s_ref;  // the traceback's read sites
+    auto R = [&](int* p, xpl_host_site& st) -> int {
       run->host_accesses += 1;
-      return app.tr ? app.tr->read(*p) : *p;
+      return app.tr ? app.tr->read(*p, st) : *p;
     };
-    app.sink += R(&out[(rows - 2) * cols + rows - 2]);  // the score printed first
+    app.sink += R(&out[(rows - 2) * cols + rows - 2], s_nw);  // the score printed first
     for (int i = rows - 2, j = rows - 2; i >= 0 && j >= 0;) {
       if (i == 0 && j == 0) break;
       int nw, w, nn;
       if (i > 0 && j > 0) {
-        nw = R(&out[(i - 1) * cols + j - 1]);
-        w = R(&out[i * cols + j - 1]);
-        nn = R(&out[(i - 1) * cols + j]);
+        nw = R(&out[(i - 1) * cols + j - 1], s_nw);
+        w = R(&out[i * cols + j - 1], s_w);
+        nn = R(&out[(i - 1) * cols + j], s_n);
       } else if (i == 0) {
         nw = nn = LIMIT;
-        w = R(&out[i * cols + j - 1]);
+        w = R(&out[i * cols + j - 1], s_w);
       } else {
         nw = w = LIMIT;
-        nn = R(&out[(i - 1) * cols + j]);
+        nn = R(&out[(i - 1) * cols + j], s_n);
       }
-      const int new_nw = nw + R(&refh[i * cols + j]);
+      const int new_nw = nw + R(&refh[i * cols + j], s_ref);
       const int new_w = w - penalty, new_n = nn - penalty;
       int tb = nw_max(new_nw, new_w, new_n);
       if (tb == new_nw) tb = nw;

@@ -33,6 +33,7 @@ int main() {
       int nstreams = 1 + rng() % 6;
       std::vector<uint64_t> pos(nstreams), base(nstreams);
       std::vector<int> kind(nstreams), sz(nstreams);
+      std::vector<xpl_host_site> site(nstreams);
       for (int s = 0; s < nstreams; ++s) {
         base[s] = 0x1000 + (rng() % 8) * 64 + (rng() % 3);  // arrays may overlap / be adjacent
         pos[s] = base[s];
@@ -46,7 +47,16 @@ int main() {
         const bool scatter = (trial % 3 == 2) && (rng() % 2 == 0);  // scattered mode
         uint64_t a = scatter ? 0x1000 + rng() % 4096 : (rng() % 10 == 0) ? base[s] + (rng() % 64) : pos[s];
         int k = (rng() % 15 == 0) ? 1 + rng() % 3 : kind[s];
-        tr.access((void*)a, sz[s], k);
+        // trial % 4: 0 no hint (current-run prediction), 1 one site per stream,
+        // 2 one site shared by all streams, 3 per-stream sites scrambled now and then
+        const int mode = trial % 4;
+        if (mode == 0) {
+          tr.access((void*)a, sz[s], k);
+        } else {
+          xpl_host_site& h = site[mode == 2 ? 0 : s];
+          if (mode == 3 && rng() % 7 == 0) h.slot = rng() % 9;  // stale / foreign / never-open slot
+          tr.access((void*)a, sz[s], k, h);
+        }
         add(want, a, sz[s], k);
         pos[s] = a + sz[s];
       }
