@@ -19,8 +19,9 @@
  *                (snapshot semantics, D5);
  *       write -> wG and P ("GPU write pending"; the epoch close turns P into L=1);
  *  3. warp aggregation: lanes that hit the same shadow u32 (4 records) are grouped
- *     with __match_any_sync, their bits OR-reduced, and one leader issues a single
- *     atomicOr -- and only if some bit is still missing (test before set);
+ *     with __match_any_sync, their bits combined (per-byte-lane ballots), and one
+ *     leader issues a single atomicOr -- and only if some bit is still missing
+ *     (test before set);
  *  4. a write also marks its 128-word chunk (and 16K-word super-chunk) in two
  *     byte maps with plain idempotent stores (test before store, no atomics),
  *     so closing the epoch costs O(chunks written), not O(shadow).
@@ -82,40 +83,80 @@ static __device__ __forceinline__ unsigned xpld_lane() {
 
 /* Mark the chunk (and super-chunk) of shadow u32 q as holding a pending GPU
  * write: plain idempotent byte stores, tested first (a stale cached 0 only
- * costs a redundant store).  Only first writes of a shadow u32 get here. */
+ * costs a redundant store).  Both bytes are loaded before either store, so
+ * the two loads overlap.  Only first writes of a shadow u32 get here. */
 static __device__ __forceinline__ void xpld_mark(unsigned q) {
   unsigned char* c = xpl_dctx.cmap + (q >> 5);
-  if (!*c) *c = 1;
   unsigned char* s = xpl_dctx.smap + (q >> 12);
-  if (!*s) *s = 1;
+  const unsigned cv = *c, sv = *s;
+  if (!cv) *c = 1;
+  if (!sv) *s = 1;
 }
 
-/* OR the record bits m into shadow u32 q for the lanes in `needers` (lanes with
- * bits still missing): lanes hitting the same u32 are grouped and one leader
- * issues the atomic.  Only the lanes of `needers` may call it. */
-static __device__ __forceinline__ void xpld_commit(unsigned needers, unsigned q, unsigned m) {
-  const unsigned grp = __match_any_sync(needers, q);
-  const unsigned M = __reduce_or_sync(grp, m);
-  if (xpld_lane() == (unsigned)(__ffs(grp) - 1)) {
-    atomicOr(xpl_dctx.pool + q, M);  /* no return value needed: RED */
-    if (M & XPLD_P4) xpld_mark(q);
-  }
+/* The record bits a read of the byte lanes rb and a write of the byte lanes wb
+ * (0xFF per record) set on the 4 records of shadow u32 cur. */
+static __device__ __forceinline__ unsigned xpld_bits2(unsigned cur, unsigned rb, unsigned wb) {
+  const unsigned l = cur & 0x01010101u;                           /* L per record      */
+  return (((l << 7) | ((~l & 0x01010101u) << 6)) & rb)            /* rGG if L else rCG */
+         | (0x0A0A0A0Au & wb);                                    /* wG | P            */
 }
 
 /* The record bits an access of kind acc sets on the 4 records of shadow u32 cur,
  * restricted to the byte lanes of `bytes` (0xFF per record touched). */
 static __device__ __forceinline__ unsigned xpld_bits(unsigned cur, unsigned bytes, unsigned acc) {
-  unsigned m = 0;
-  if (acc & XPL_ACC_R) {
-    const unsigned l = cur & 0x01010101u;                  /* L per record        */
-    m = ((l << 7) | ((~l & 0x01010101u) << 6)) & bytes;    /* rGG if L else rCG   */
+  return xpld_bits2(cur, (acc & XPL_ACC_R) ? bytes : 0u, (acc & XPL_ACC_W) ? bytes : 0u);
+}
+
+/* Commit the access of every lane of `needers` (lanes with bits still missing):
+ * lanes hitting the same shadow u32 q are grouped (__match_any_sync) and one
+ * leader issues a single atomicOr with the group's bits.  The group's bits are
+ * formed from warp ballots (which byte lanes the group reads / writes), not
+ * from a reduction over the group's own lane mask: that mask differs between
+ * groups, and a reduction under a non-uniform mask serialises over the groups.
+ * Any lane's `cur` gives the group's L bits (L is frozen for the epoch).
+ * K = the access kind when it is the same for every lane (the hook's call site
+ * fixes it), 0 when each lane brings its own (acc).  SINGLE: every lane touches
+ * one byte lane, bytes == 0xFF << 8*b, so two ballots of b's bits name the
+ * group's byte lanes.  Only the lanes of `needers` may call it. */
+template <unsigned K, bool SINGLE>
+static __device__ __forceinline__ void xpld_commit(unsigned needers, unsigned q, unsigned cur,
+                                                   unsigned bytes, unsigned acc) {
+  const unsigned grp = __match_any_sync(needers, q);
+  unsigned rb = 0, wb = 0;
+  if (K != 0 && SINGLE) {
+    const unsigned b = (unsigned)(__ffs(bytes) - 1) >> 3;
+    const unsigned b0 = __ballot_sync(needers, b & 1) & grp, b1 = __ballot_sync(needers, b & 2) & grp;
+    const unsigned n0 = grp & ~b0, n1 = grp & ~b1;
+    const unsigned u = ((n0 & n1) ? 0x000000FFu : 0u) | ((b0 & n1) ? 0x0000FF00u : 0u) |
+                       ((n0 & b1) ? 0x00FF0000u : 0u) | ((b0 & b1) ? 0xFF000000u : 0u);
+    rb = (K & XPL_ACC_R) ? u : 0u;
+    wb = (K & XPL_ACC_W) ? u : 0u;
+  } else {
+#pragma unroll
+    for (unsigned k = 0; k < 4; ++k) {
+      const unsigned sel = 0xFFu << (8 * k);
+      const bool has = (bytes & sel) != 0;
+      if (K != 0) {
+        if (__ballot_sync(needers, has) & grp) {
+          if (K & XPL_ACC_R) rb |= sel;
+          if (K & XPL_ACC_W) wb |= sel;
+        }
+      } else {
+        if (__ballot_sync(needers, has && (acc & XPL_ACC_R)) & grp) rb |= sel;
+        if (__ballot_sync(needers, has && (acc & XPL_ACC_W)) & grp) wb |= sel;
+      }
+    }
   }
-  if (acc & XPL_ACC_W) m |= 0x0A0A0A0Au & bytes;           /* wG | P              */
-  return m;
+  if (xpld_lane() == (unsigned)(__ffs(grp) - 1)) {
+    atomicOr(xpl_dctx.pool + q, xpld_bits2(cur, rb, wb)); /* no return value needed: RED */
+    if (wb) xpld_mark(q);
+  }
 }
 
 /* Apply a GPU access to the shadow words [g0, g1] (global pool word indices;
- * empty when g0 > g1).  All active lanes of the calling warp must call it. */
+ * empty when g0 > g1).  All active lanes of the calling warp must call it.
+ * K: the access kind if uniform over the warp (a compile-time call site), else 0. */
+template <unsigned K>
 static __device__ __forceinline__ void xpl_dev_apply(unsigned long long g0,
                                                      unsigned long long g1,
                                                      unsigned acc) {
@@ -125,14 +166,15 @@ static __device__ __forceinline__ void xpl_dev_apply(unsigned long long g0,
   if (single) { /* the short path */
     const bool hit = g0 == g1;
     const unsigned q = (unsigned)(g0 >> 2);
+    const unsigned bytes = 0xFFu << (8 * (unsigned)(g0 & 3));
     unsigned cur = 0, m = 0;
     if (hit) {
       cur = xpl_dctx.pool[q];
-      m = xpld_bits(cur, 0xFFu << (8 * (unsigned)(g0 & 3)), acc);
+      m = xpld_bits(cur, bytes, acc);
     }
     const bool need = hit && (cur & m) != m;
     const unsigned needers = __ballot_sync(singles, need);
-    if (need) xpld_commit(needers, q, m);
+    if (need) xpld_commit<K, true>(needers, q, cur, bytes, acc);
   }
   if (singles == active) return;
   /* multi-word accesses: one shadow u32 per iteration */
@@ -141,10 +183,9 @@ static __device__ __forceinline__ void xpl_dev_apply(unsigned long long g0,
   const unsigned long long ql = g1 >> 2;
   bool more = multi;
   while (__any_sync(active, more)) {
-    unsigned cur = 0, m = 0;
+    unsigned cur = 0, m = 0, bytes = 0;
     if (more) {
       cur = xpl_dctx.pool[q];
-      unsigned bytes = 0;
 #pragma unroll
       for (unsigned k = 0; k < 4; ++k) {
         const unsigned long long gw = q * 4 + k;
@@ -154,7 +195,7 @@ static __device__ __forceinline__ void xpl_dev_apply(unsigned long long g0,
     }
     const bool need = more && (cur & m) != m;
     const unsigned needers = __ballot_sync(active, need);
-    if (need) xpld_commit(needers, (unsigned)q, m);
+    if (need) xpld_commit<K, false>(needers, (unsigned)q, cur, bytes, acc);
     more = more && q < ql;
     ++q;
   }
@@ -165,16 +206,26 @@ static __device__ __forceinline__ void xpl_dev_apply(unsigned long long g0,
  * block, validated against the row on every use, so stale or uninitialised
  * slots only cost the full search) skips the binary search when consecutive
  * accesses of a warp hit the same allocation -- the common case. */
-static __device__ __forceinline__ void xpl_dev_record(const void* p, unsigned size,
-                                                      unsigned acc) {
+/* The per-warp row cache (one per block, shared by every hook of the kernel). */
+static __device__ __forceinline__ unsigned* xpld_row_cache() {
+  __shared__ unsigned c[32];
+  return c;
+}
+
+template <unsigned K>
+static __device__ __forceinline__ void xpl_dev_record_k(const void* p, unsigned size,
+                                                        unsigned acc) {
 #ifndef XPL_OFF
-  __shared__ unsigned xpl_row_cache[32];
+  unsigned* const xpl_row_cache = xpld_row_cache();
   const unsigned long long a = (unsigned long long)p;
   const xpl_dev_row* rows = xpl_dctx.rows;
   const unsigned n = __ldg(xpl_dctx.n_rows);
   const unsigned slot = ((threadIdx.z * blockDim.y + threadIdx.y) * blockDim.x + threadIdx.x) >> 5 & 31;
   unsigned ri = xpl_row_cache[slot];
-  bool hit = ri < n && __ldg(&rows[ri].base) <= a && a < __ldg(&rows[ri].end);
+  const unsigned rc = ri < n ? ri : 0; /* (n == 0: nothing matches below) */
+  ulonglong2 be = __ldg(reinterpret_cast<const ulonglong2*>(rows + rc));     /* base, end  */
+  ulonglong2 ow = __ldg(reinterpret_cast<const ulonglong2*>(rows + rc) + 1); /* off, words */
+  bool hit = ri < n && be.x <= a && a < be.y;
   if (!hit) {
     unsigned lo = 0, hi = n;
     while (lo < hi) {
@@ -186,40 +237,45 @@ static __device__ __forceinline__ void xpl_dev_record(const void* p, unsigned si
       ri = lo - 1;
       hit = true;
       xpl_row_cache[slot] = ri;  /* benign race: any lane's row is a valid entry */
+      be = __ldg(reinterpret_cast<const ulonglong2*>(rows + ri));
+      ow = __ldg(reinterpret_cast<const ulonglong2*>(rows + ri) + 1);
     }
   }
   unsigned long long g0 = 1, g1 = 0;
   if (hit && size > 0) {
-    const xpl_dev_row* r = rows + ri;
-    const unsigned long long base = __ldg(&r->base);
+    const unsigned long long base = be.x;
     const unsigned long long w0 = (a - base) >> 2;
     unsigned long long wl = (a + size - 1 - base) >> 2;
-    const unsigned long long wmax = __ldg(&r->words) - 1;
+    const unsigned long long wmax = ow.y - 1;
     if (wl > wmax) wl = wmax;
-    const unsigned long long off = __ldg(&r->off);
-    g0 = off + w0;
-    g1 = off + wl;
+    g0 = ow.x + w0;
+    g1 = ow.x + wl;
   }
-  xpl_dev_apply(g0, g1, acc);
+  xpl_dev_apply<K>(g0, g1, K ? K : acc);
 #else
   (void)p; (void)size; (void)acc;
 #endif
 }
 
+/* Generic form: acc may differ from lane to lane. */
+static __device__ __forceinline__ void xpl_dev_record(const void* p, unsigned size, unsigned acc) {
+  xpl_dev_record_k<0>(p, size, acc);
+}
+
 /* traceR / traceW / traceRW: take the element, return it (Table I). */
 template <class T>
 static __device__ __forceinline__ const T& xpl_read(const T& x) {
-  xpl_dev_record(&x, sizeof(T), XPL_ACC_R);
+  xpl_dev_record_k<XPL_ACC_R>(&x, sizeof(T), XPL_ACC_R);
   return x;
 }
 template <class T>
 static __device__ __forceinline__ T& xpl_write(T& x) {
-  xpl_dev_record(&x, sizeof(T), XPL_ACC_W);
+  xpl_dev_record_k<XPL_ACC_W>(&x, sizeof(T), XPL_ACC_W);
   return x;
 }
 template <class T>
 static __device__ __forceinline__ T& xpl_rw(T& x) {
-  xpl_dev_record(&x, sizeof(T), XPL_ACC_RW);
+  xpl_dev_record_k<XPL_ACC_RW>(&x, sizeof(T), XPL_ACC_RW);
   return x;
 }
 

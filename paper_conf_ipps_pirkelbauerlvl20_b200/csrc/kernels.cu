@@ -24,49 +24,67 @@ constexpr uint32_t kP4 = 0x02020202u;
 
 // ---------------------------------------------------------------------------
 // fold (epoch close): every 128-word chunk a GPU write marked (cmap) gets
-// P -> L=1 and P cleared (snapshot semantics D5).  One CTA per 16K-word
-// super-chunk below the pool's high-water mark: a CTA-uniform check of the
-// super byte, then warp w checks chunks [16w, 16w+16) and folds the marked
-// ones four at a time (128 B coalesced each).  No list, no atomics; cost
-// O(super map + chunks written).
-__global__ void __launch_bounds__(256) fold_kernel(uint32_t* __restrict__ pool,
-                                                   uint8_t* __restrict__ cmap,
-                                                   uint8_t* __restrict__ smap, uint64_t n_super,
-                                                   unsigned long long* stats) {
+// P -> L=1 and P cleared (snapshot semantics D5).  A one-wave grid:
+// CTA b owns the super-chunks b, b+G, b+2G, ... (16K words each, below the
+// pool's high-water mark).  It first reads all its super bytes at once (one
+// byte per thread per round) and lists the marked ones in shared memory, so
+// an epoch that wrote little costs one launch and one read of the super map;
+// then, per listed super-chunk, warp w checks chunks [16w, 16w+16) and folds
+// the marked ones four at a time (128 B coalesced each).  Consecutive
+// super-chunks go to different CTAs, so a dense epoch spreads over the grid.
+// No global list, no atomics; cost O(super map + chunks written).
+constexpr int kFoldThreads = 256;
+
+__global__ void __launch_bounds__(kFoldThreads) fold_kernel(uint32_t* __restrict__ pool,
+                                                            uint8_t* __restrict__ cmap,
+                                                            uint8_t* __restrict__ smap,
+                                                            uint64_t n_super,
+                                                            unsigned long long* stats) {
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  __shared__ uint32_t s_go;
+  __shared__ uint64_t s_list[kFoldThreads];
+  __shared__ uint32_t s_n;
   uint32_t folded = 0;
-  for (uint64_t sc = blockIdx.x; sc < n_super; sc += gridDim.x) {
-    if (threadIdx.x == 0) s_go = smap[sc];  // one read per CTA: a uniform decision
+  const uint64_t G = gridDim.x;
+  const uint64_t mine = n_super > blockIdx.x ? (n_super - blockIdx.x + G - 1) / G : 0;
+  for (uint64_t r0 = 0; r0 < mine; r0 += kFoldThreads) {
+    if (threadIdx.x == 0) s_n = 0;
     __syncthreads();
-    const bool go = s_go != 0;
-    __syncthreads();
-    if (!go) continue;
-    const uint64_t c0 = sc * 128 + warp * 16;
-    const bool m = lane < 16 && cmap[c0 + lane] != 0;
-    uint32_t marked = __ballot_sync(0xFFFFFFFFu, m);
-    folded += __popc(marked);
-    while (marked) {
-      uint64_t at[4];
-      uint32_t v[4];
-#pragma unroll
-      for (uint32_t k = 0; k < 4; ++k) {
-        if (marked) {
-          const uint32_t j = __ffs(marked) - 1;
-          marked &= marked - 1;
-          at[k] = (c0 + j) * 32 + lane;
-          v[k] = pool[at[k]];
-        } else {
-          at[k] = ~0ull;
-          v[k] = 0;
-        }
-      }
-#pragma unroll
-      for (uint32_t k = 0; k < 4; ++k)
-        if (v[k] & kP4) pool[at[k]] = (v[k] & ~kP4) | ((v[k] & kP4) >> 1);
+    const uint64_t it = r0 + threadIdx.x;
+    if (it < mine) {
+      const uint64_t sc = blockIdx.x + it * G;
+      if (smap[sc]) s_list[atomicAdd(&s_n, 1u)] = sc;
     }
-    if (m) cmap[c0 + lane] = 0;
-    if (threadIdx.x == 0) smap[sc] = 0;
+    __syncthreads();
+    const uint32_t n = s_n;
+    for (uint32_t k = 0; k < n; ++k) {
+      const uint64_t sc = s_list[k];
+      const uint64_t c0 = sc * 128 + warp * 16;
+      const bool m = lane < 16 && cmap[c0 + lane] != 0;
+      uint32_t marked = __ballot_sync(0xFFFFFFFFu, m);
+      folded += __popc(marked);
+      while (marked) {
+        uint64_t at[4];
+        uint32_t v[4];
+#pragma unroll
+        for (uint32_t j4 = 0; j4 < 4; ++j4) {
+          if (marked) {
+            const uint32_t j = __ffs(marked) - 1;
+            marked &= marked - 1;
+            at[j4] = (c0 + j) * 32 + lane;
+            v[j4] = pool[at[j4]];
+          } else {
+            at[j4] = ~0ull;
+            v[j4] = 0;
+          }
+        }
+#pragma unroll
+        for (uint32_t j4 = 0; j4 < 4; ++j4)
+          if (v[j4] & kP4) pool[at[j4]] = (v[j4] & ~kP4) | ((v[j4] & kP4) >> 1);
+      }
+      if (m) cmap[c0 + lane] = 0;
+      if (threadIdx.x == 0) smap[sc] = 0;
+    }
+    __syncthreads();  // s_list / s_n are rewritten by the next round
   }
   if (lane == 0 && folded) atomicAdd(stats + 3, (unsigned long long)folded);
 }
@@ -787,7 +805,10 @@ int grid_for(uint64_t n, int threads, int max_ctas) {
 
 void launch_fold(cudaStream_t s, uint32_t* pool, uint8_t* cmap, uint8_t* smap,
                  uint64_t n_super, unsigned long long* stats) {
-  if (n_super) fold_kernel<<<grid_for(n_super * 256, 256, 148 * 64), 256, 0, s>>>(pool, cmap, smap, n_super, stats);
+  if (n_super) {
+    const uint64_t g = n_super < 148 * 4 ? n_super : 148 * 4;  // one wave
+    fold_kernel<<<(unsigned)g, kFoldThreads, 0, s>>>(pool, cmap, smap, n_super, stats);
+  }
 }
 
 void launch_merge(cudaStream_t s, const uint64_t* recs, uint32_t n, bool has_r, bool has_w,
