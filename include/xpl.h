@@ -70,6 +70,18 @@ typedef struct {
   uint32_t kind; /* xpl_acc_kind */
 } xpl_host_access;
 
+/* A strided sequence of host accesses (what xpl_host.h emits for scattered
+ * accesses with a constant stride, e.g. a column walk): `count` accesses, the
+ * j-th covering [addr + j*stride, addr + j*stride + size), in order j = 0, 1, ...
+ * (32 bytes).  count == 1 is one xpl_record_host_ranges record. */
+typedef struct {
+  uint64_t addr;
+  uint32_t size;  /* bytes, >= 1 */
+  uint32_t kind;  /* xpl_acc_kind */
+  int64_t stride; /* bytes between consecutive accesses (any sign, 0 = repeats) */
+  uint64_t count; /* >= 1 */
+} xpl_host_strided;
+
 /* XplAllocData: names an allocation in the report. */
 typedef struct {
   const void* addr;
@@ -163,6 +175,13 @@ xpl_status xpl_record_host(xpl_ctx* ctx, const xpl_host_access* recs, size_t n);
  * xpl_record_host on the individual accesses whenever no individual access
  * straddles two allocations.  Same ordering and epoch rules as xpl_record_host. */
 xpl_status xpl_record_host_ranges(xpl_ctx* ctx, const xpl_host_access* recs, size_t n);
+
+/* Strided host ranges: record i stands for recs[i].count ranges records
+ * (addr + j*stride, size, kind), j = 0 .. count-1, in that order; the records
+ * are in program order with each other.  Exactly xpl_record_host_ranges on the
+ * expanded list (same ordering and epoch rules).  INVALID_ARG on kind outside
+ * 1..3, size 0 or count 0. */
+xpl_status xpl_record_host_strided(xpl_ctx* ctx, const xpl_host_strided* recs, size_t n);
 
 /* The transfer wrappers (D7).  dst/src are the cudaMemcpy arguments. */
 xpl_status xpl_record_copy(xpl_ctx* ctx, const void* dst, const void* src, size_t bytes,

@@ -154,7 +154,7 @@ class xpl_host_tracer {
 
   void drain() {
     if (n_) {
-      const xpl_status s = xpl_record_host_ranges(ctx_, buf_, n_);
+      const xpl_status s = xpl_record_host_strided(ctx_, buf_, n_);
       if (s != XPL_OK && status_ == XPL_OK) status_ = s;
     }
     n_ = 0;
@@ -165,7 +165,7 @@ class xpl_host_tracer {
   }
   void close(int i) {
     if (n_ == kBuf) drain();
-    buf_[n_++] = xpl_host_access{run_[i].beg, (uint32_t)(run_[i].end - run_[i].beg), run_[i].kind};
+    buf_[n_++] = xpl_host_strided{run_[i].beg, (uint32_t)(run_[i].end - run_[i].beg), run_[i].kind, 0, 1};
     run_[i].kind = 0;
     const uint64_t b = wlo(run_[i].beg);
     for (int j = 0; j < kRuns; ++j) {
@@ -229,10 +229,26 @@ class xpl_host_tracer {
       close(o);
     }
     // Scattered accesses (no run ever grows): emit them directly, re-trying
-    // runs every 64th access -- same records, without the slot churn.
+    // runs every 64th access -- same records, without the slot churn.  An
+    // emitted access that continues the arithmetic progression of the record
+    // emitted last (same kind and size, nothing emitted in between) joins it.
     if (churn_ >= 32 && (++tick_ & 63) != 0) {
+      if (n_) {
+        xpl_host_strided& l = buf_[n_ - 1];
+        if (l.kind == kind && l.size == size) {
+          if (l.count == 1) {
+            l.stride = (int64_t)(a - l.addr);
+            l.count = 2;
+            return kRuns;
+          }
+          if (a == l.addr + (uint64_t)l.stride * l.count) {
+            ++l.count;
+            return kRuns;
+          }
+        }
+      }
       if (n_ == kBuf) drain();
-      buf_[n_++] = xpl_host_access{a, size, kind};
+      buf_[n_++] = xpl_host_strided{a, size, kind, 0, 1};
       return kRuns;
     }
     int slot = -1;
@@ -271,7 +287,7 @@ class xpl_host_tracer {
   uint32_t tick_ = 0;
   size_t n_ = 0;
   xpl_status status_ = XPL_OK;
-  xpl_host_access buf_[kBuf];
+  xpl_host_strided buf_[kBuf];
 };
 
 #endif /* __cplusplus */

@@ -775,6 +775,47 @@ xpl_status xpl_record_host_ranges(xpl_ctx* c, const xpl_host_access* recs, size_
   return XPL_OK;
 }
 
+xpl_status xpl_record_host_strided(xpl_ctx* c, const xpl_host_strided* recs, size_t n) {
+  if (!c || (!recs && n)) return XPL_ERR_INVALID_ARG;
+  for (size_t i = 0; i < n; ++i) {
+    const xpl_host_strided& q = recs[i];
+    if (q.kind < 1 || q.kind > 3 || q.size == 0 || q.count == 0) return XPL_ERR_INVALID_ARG;
+    if (q.count == 1) {
+      const xpl_host_access one = {q.addr, q.size, q.kind};
+      xpl_status s = xpl_record_host_ranges(c, &one, 1);
+      if (s) return s;
+      continue;
+    }
+    // the lowest and highest element: if both lie inside one live row, so do all
+    const uint64_t last = q.addr + (uint64_t)q.stride * (q.count - 1);
+    const uint64_t lo = q.stride >= 0 ? q.addr : last, hi = q.stride >= 0 ? last : q.addr;
+    const Row* r = lookup(c, lo);
+    if (r && hi + q.size <= r->base + r->bytes && hi + q.size > hi) {
+      uint64_t a = q.addr;
+      for (uint64_t j = 0; j < q.count; ++j, a += (uint64_t)q.stride) {
+        const uint64_t w0 = (a - r->base) >> 2, wl = (a + q.size - 1 - r->base) >> 2;
+        uint64_t g0 = r->off + w0, nw = wl - w0 + 1;
+        if (c->depth) {
+          for (; nw > kMaxRecWords; g0 += kMaxRecWords, nw -= kMaxRecWords)
+            c->deferred.push_back(pack_rec(g0, kMaxRecWords, q.kind));
+          c->deferred.push_back(pack_rec(g0, nw, q.kind));
+        } else {
+          xpl_status s = stage_push(c, g0, nw, q.kind);
+          if (s) return s;
+        }
+      }
+      continue;
+    }
+    uint64_t a = q.addr;  // elements in several rows (or untracked): one by one
+    for (uint64_t j = 0; j < q.count; ++j, a += (uint64_t)q.stride) {
+      const xpl_host_access one = {a, q.size, q.kind};
+      xpl_status s = xpl_record_host_ranges(c, &one, 1);
+      if (s) return s;
+    }
+  }
+  return XPL_OK;
+}
+
 xpl_status xpl_record_copy(xpl_ctx* c, const void* dst, const void* src, size_t bytes,
                            xpl_copy_dir dir) {
   if (!c || (unsigned)dir > 4) return XPL_ERR_INVALID_ARG;

@@ -78,8 +78,10 @@ struct App {
     if (tr) ok(tr->flush());
   }
   // for (i < n) p[i] = f(i)   -- a traced host write loop doing the real stores
+  // (noinline: the loops get their own register allocation instead of sharing
+  // the program's large driver function; the same for the twin)
   template <class T>
-  void write_loop(T* p, uint64_t n) {
+  __attribute__((noinline)) void write_loop(T* p, uint64_t n) {
     const auto t0 = std::chrono::steady_clock::now();
     xpl_host_site st;  // one per static access site (xpl_host.h)
     if (tr)
@@ -91,7 +93,7 @@ struct App {
   }
   // s += p[i * stride + off] for i < n  -- a traced host read loop
   template <class T>
-  T read_loop(const T* p, uint64_t n, uint64_t stride = 1, uint64_t off = 0) {
+  __attribute__((noinline)) T read_loop(const T* p, uint64_t n, uint64_t stride = 1, uint64_t off = 0) {
     const auto t0 = std::chrono::steady_clock::now();
     T acc = 0;
     xpl_host_site st;
@@ -335,6 +337,65 @@ __global__ void __launch_bounds__(NWB) nw_kernel(int* ref, int* mat, int cols, i
   for (int ty = 0; ty < NWB; ty++) WR<I>(mat[index + ty * cols]) = temp[ty + 1][tx + 1];
 }
 
+// ---------------------------------------------------------------------------
+// Host loops of the programs, as separate functions (their own register
+// allocation; tr == nullptr is the uninstrumented twin).  Each static access
+// site has its own xpl_host_site (xpl_host.h).
+__attribute__((noinline)) void bfs_read_nodes(xpl_host_tracer* tr, BfsNode* h_nodes, bool* h_mask,
+                                              bool* h_updating, bool* h_visited, int n, int deg) {
+  if (tr) {
+    xpl_host_site s0, s1, s2, s3, s4;
+    for (int i = 0; i < n; i++) {
+      tr->write(h_nodes[i].starting, s0) = i * deg;
+      tr->write(h_nodes[i].no_of_edges, s1) = deg;
+      tr->write(h_mask[i], s2) = false;
+      tr->write(h_updating[i], s3) = false;
+      tr->write(h_visited[i], s4) = false;
+    }
+  } else {
+    for (int i = 0; i < n; i++) {
+      h_nodes[i].starting = i * deg;
+      h_nodes[i].no_of_edges = deg;
+      h_mask[i] = h_updating[i] = h_visited[i] = false;
+    }
+  }
+}
+
+// the edge list is stored as read from the input; costs -1
+__attribute__((noinline)) void bfs_read_edges(xpl_host_tracer* tr, int* h_edges, uint64_t ne,
+                                              int* h_cost, int n) {
+  if (tr) {
+    xpl_host_site s0, s1;
+    for (uint64_t i = 0; i < ne; ++i) {
+      const int e = h_edges[i];  // (the input buffer; the traced store is the program's)
+      tr->write(h_edges[i], s0) = e;
+    }
+    for (int i = 0; i < n; ++i) tr->write(h_cost[i], s1) = -1;
+  } else {
+    for (int i = 0; i < n; ++i) h_cost[i] = -1;
+  }
+}
+
+// the substitution matrix from the sequences (row / column 0), then the gap row and column
+__attribute__((noinline)) void nw_fill_reference(xpl_host_tracer* tr, int* in, int* refh,
+                                                 const int* blosum, int rows, int cols, int penalty) {
+  if (tr) {
+    xpl_host_site s0, s1, s2, s3, s4;
+    for (int i = 1; i < rows; i++)
+      for (int j = 1; j < cols; j++) {
+        const int x = tr->read(in[i * cols], s0), y = tr->read(in[j], s1);
+        tr->write(refh[i * cols + j], s2) = blosum[x * 24 + y];
+      }
+    for (int i = 1; i < rows; i++) tr->write(in[i * cols], s3) = -i * penalty;
+    for (int j = 1; j < cols; j++) tr->write(in[j], s4) = -j * penalty;
+  } else {
+    for (int i = 1; i < rows; i++)
+      for (int j = 1; j < cols; j++) refh[i * cols + j] = blosum[in[i * cols] * 24 + in[j]];
+    for (int i = 1; i < rows; i++) in[i * cols] = -i * penalty;
+    for (int j = 1; j < cols; j++) in[j] = -j * penalty;
+  }
+}
+
 }  // namespace
 
 extern "C" {
@@ -430,20 +491,7 @@ int xplw_bfs(xplw_run* run, const xplw_arrays* a, int n, int deg, unsigned long 
   // read the graph "file": node records, masks, edges, costs (Rodinia bfs.cu order)
   {
     const auto t0 = std::chrono::steady_clock::now();
-    xpl_host_site s0, s1, s2, s3, s4;
-    for (int i = 0; i < n; i++) {
-      if (app.tr) {
-        app.tr->write(h_nodes[i].starting, s0) = i * deg;
-        app.tr->write(h_nodes[i].no_of_edges, s1) = deg;
-        app.tr->write(h_mask[i], s2) = false;
-        app.tr->write(h_updating[i], s3) = false;
-        app.tr->write(h_visited[i], s4) = false;
-      } else {
-        h_nodes[i].starting = i * deg;
-        h_nodes[i].no_of_edges = deg;
-        h_mask[i] = h_updating[i] = h_visited[i] = false;
-      }
-    }
+    bfs_read_nodes(app.tr, h_nodes, h_mask, h_updating, h_visited, n, deg);
     run->host_accesses += 5ull * n;
     run->host_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
   }
@@ -456,15 +504,7 @@ int xplw_bfs(xplw_run* run, const xplw_arrays* a, int n, int deg, unsigned long 
   run->host_accesses += 2;
   {  // the edge list is stored as read from the input; costs -1, source 0
     const auto t0 = std::chrono::steady_clock::now();
-    xpl_host_site s0, s1;
-    for (uint64_t i = 0; i < ne; ++i) {
-      const int e = h_edges[i];  // (the input buffer; the traced store is the program's)
-      if (app.tr) app.tr->write(h_edges[i], s0) = e;
-    }
-    for (int i = 0; i < n; ++i) {
-      if (app.tr) app.tr->write(h_cost[i], s1) = -1;
-      else h_cost[i] = -1;
-    }
+    bfs_read_edges(app.tr, h_edges, ne, h_cost, n);
     if (app.tr) app.tr->write(h_cost[0]) = 0;
     else h_cost[0] = 0;
     run->host_accesses += ne + n + 1;
@@ -521,26 +561,8 @@ int xplw_nw(xplw_run* run, const xplw_arrays* a, int n, int penalty, const int* 
   // the sequences (row / column 0) are the input; the substitution matrix from them
   {
     const auto t0 = std::chrono::steady_clock::now();
-    xpl_host_site s0, s1, s2, s3, s4;
-    if (app.tr) {
-      for (int i = 1; i < rows; i++)
-        for (int j = 1; j < cols; j++) {
-          const int x = app.tr->read(in[i * cols], s0), y = app.tr->read(in[j], s1);
-          app.tr->write(refh[i * cols + j], s2) = blosum[x * 24 + y];
-        }
-    } else {
-      for (int i = 1; i < rows; i++)
-        for (int j = 1; j < cols; j++) refh[i * cols + j] = blosum[in[i * cols] * 24 + in[j]];
-    }
+    nw_fill_reference(app.tr, in, refh, blosum, rows, cols, penalty);
     run->host_accesses += 3ull * (rows - 1) * (cols - 1);
-    for (int i = 1; i < rows; i++) {
-      if (app.tr) app.tr->write(in[i * cols], s3) = -i * penalty;
-      else in[i * cols] = -i * penalty;
-    }
-    for (int j = 1; j < cols; j++) {
-      if (app.tr) app.tr->write(in[j], s4) = -j * penalty;
-      else in[j] = -j * penalty;
-    }
     run->host_accesses += (uint64_t)(rows - 1) + (cols - 1);
     run->host_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
   }

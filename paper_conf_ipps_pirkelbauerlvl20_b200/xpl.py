@@ -30,6 +30,8 @@ ACC_R, ACC_W, ACC_RW = 1, 2, 3
 COPY_H2D, COPY_D2H, COPY_H2H, COPY_D2D, MEMSET_DEV = 0, 1, 2, 3, 4
 
 HOST_ACCESS_DTYPE = np.dtype([("addr", "<u8"), ("size", "<u4"), ("kind", "<u4")])
+HOST_STRIDED_DTYPE = np.dtype([("addr", "<u8"), ("size", "<u4"), ("kind", "<u4"), ("stride", "<i8"),
+                               ("count", "<u8")])
 
 
 class XplConfig(C.Structure):
@@ -95,6 +97,7 @@ xpl_kernel_begin = _sig("xpl_kernel_begin", [vp, vp])
 xpl_kernel_end = _sig("xpl_kernel_end", [vp, vp])
 xpl_record_host = _sig("xpl_record_host", [vp, vp, sz])
 xpl_record_host_ranges = _sig("xpl_record_host_ranges", [vp, vp, sz])
+xpl_record_host_strided = _sig("xpl_record_host_strided", [vp, vp, sz])
 xpl_record_copy = _sig("xpl_record_copy", [vp, vp, vp, sz, i32])
 xpl_diagnose = _sig("xpl_diagnose", [vp, C.POINTER(XplDiagParams), C.POINTER(XplName), sz,
                                      C.POINTER(XplAllocReport), sz, C.POINTER(sz), i32])
@@ -123,7 +126,7 @@ KERNEL_CLASSES = ["fold", "merge", "range", "diag_tile", "diagnose"]
 xpl_profile_read = _sig("xpl_profile_read", [vp, C.POINTER(XplKernelTime), i32])
 
 EXPORTED = ["xpl_init", "xpl_finalize", "xpl_register_alloc", "xpl_free", "xpl_kernel_begin",
-            "xpl_kernel_end", "xpl_record_host", "xpl_record_host_ranges", "xpl_record_copy", "xpl_diagnose",
+            "xpl_kernel_end", "xpl_record_host", "xpl_record_host_ranges", "xpl_record_host_strided", "xpl_record_copy", "xpl_diagnose",
             "xpl_get_device_ctx", "xpl_shadow_dump", "xpl_flush", "xpl_sync",
             "xpl_runtime_stream", "xpl_get_stats", "xpl_status_string", "xpl_profile",
             "xpl_profile_read", "xpl_register_alloc_piece", "xpl_diagnose_partials", "xpl_combine_partials",
@@ -191,6 +194,11 @@ class Context:
     def record_host_ranges(self, recs: np.ndarray):
         recs = np.ascontiguousarray(recs, dtype=HOST_ACCESS_DTYPE)
         check("xpl_record_host_ranges", xpl_record_host_ranges(self.h, recs.ctypes.data, recs.size))
+
+    def record_host_strided(self, recs: np.ndarray):
+        """recs: HOST_STRIDED_DTYPE records (addr, size, kind, stride, count)."""
+        recs = np.ascontiguousarray(recs, dtype=HOST_STRIDED_DTYPE)
+        check("xpl_record_host_strided", xpl_record_host_strided(self.h, recs.ctypes.data, recs.size))
 
     def record_copy(self, dst, src, nbytes, direction):
         check("xpl_record_copy", xpl_record_copy(self.h, dst, src, nbytes, direction))

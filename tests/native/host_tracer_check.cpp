@@ -9,8 +9,13 @@
 #include <random>
 #include "xpl.h"
 static std::vector<xpl_host_access> got;
-extern "C" xpl_status xpl_record_host_ranges(xpl_ctx*, const xpl_host_access* r, size_t n) {
-  for (size_t i = 0; i < n; ++i) got.push_back(r[i]);
+static size_t n_strided = 0;
+extern "C" xpl_status xpl_record_host_strided(xpl_ctx*, const xpl_host_strided* r, size_t n) {
+  for (size_t i = 0; i < n; ++i) {
+    if (r[i].count > 1) ++n_strided;
+    for (uint64_t j = 0; j < r[i].count; ++j)
+      got.push_back(xpl_host_access{r[i].addr + (uint64_t)r[i].stride * j, r[i].size, r[i].kind});
+  }
   return XPL_OK;
 }
 #include "xpl_host.h"
@@ -45,7 +50,10 @@ int main() {
       for (int i = 0; i < n; ++i) {
         int s = rng() % nstreams;
         const bool scatter = (trial % 3 == 2) && (rng() % 2 == 0);  // scattered mode
-        uint64_t a = scatter ? 0x1000 + rng() % 4096 : (rng() % 10 == 0) ? base[s] + (rng() % 64) : pos[s];
+        // trial % 5 == 4: column walks (strided) mixed in
+        const bool walk = (trial % 5 == 4) && (rng() % 4 != 0);
+        uint64_t a = walk ? base[s] + ((uint64_t)(i / nstreams) * (16 + 8 * s)) % 8192
+                   : scatter ? 0x1000 + rng() % 4096 : (rng() % 10 == 0) ? base[s] + (rng() % 64) : pos[s];
         int k = (rng() % 15 == 0) ? 1 + rng() % 3 : kind[s];
         // trial % 4: 0 no hint (current-run prediction), 1 one site per stream,
         // 2 one site shared by all streams, 3 per-stream sites scrambled now and then
@@ -65,6 +73,7 @@ int main() {
     for (auto& r : got) add(have, r.addr, r.size, r.kind);
     if (want != have) { printf("MISMATCH trial %d\n", trial); return 1; }
   }
-  printf("tracer ok, last trial %zu records\n", got.size());
+  printf("tracer ok, last trial %zu records, %zu strided records overall\n", got.size(), n_strided);
+  if (n_strided == 0) { printf("no strided record was ever formed\n"); return 1; }
   return 0;
 }

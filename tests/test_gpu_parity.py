@@ -220,3 +220,64 @@ def test_host_ranges(gpu, seed):
         ctx.record_host_ranges(rec)
         got = [ctx.diagnose(50, 0, 1, True)]
     compare(got, exp, "ranges")
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_host_strided(gpu, seed):
+    """xpl_record_host_strided: strided sequences (positive, negative and zero
+    strides; elements in one allocation, spanning several, or untracked;
+    some recorded inside an open GPU epoch, so deferred) == every element as
+    its own one-byte-per-byte host access, in order."""
+    replay, xpl = gpu
+    import torch
+    rng = np.random.default_rng(0x58504C20 + seed)
+    ops, bases = [], []
+    b = 0x3100_0000
+    for i in range(6):
+        n = int(rng.integers(64, 4000))
+        ops.append(("REG", b, n, i % 3))
+        bases.append((b, n))
+        b += n + int(rng.integers(0, 3)) * 4
+    lo, hi = bases[0][0] - 64, b + 64
+    recs, expanded = [], []
+    for _ in range(200):
+        size = int(rng.choice([1, 2, 4, 8, 12]))
+        kind = int(rng.integers(1, 4))
+        if kind == 3:
+            size = 4 * int(rng.integers(1, 3))
+        stride = int(rng.choice([0, 4, 8, 16, 64, -4, -64, 100, 4 * int(rng.integers(1, 300))]))
+        count = int(rng.integers(1, 80))
+        a = int(rng.integers(lo, hi))
+        if kind == 3:
+            a &= ~3
+        recs.append((a, size, kind, stride, count))
+        expanded += [(a + j * stride, size, kind) for j in range(count)]
+    split = len(recs) // 2  # the second half inside a GPU epoch (D20: applied at its close)
+    n_first = sum(r[4] for r in recs[:split])
+
+    def host_ops(part):
+        out = []
+        for a, n, k in part:
+            if k == 3:  # RW of a word-aligned range: per word R then W (one access per word)
+                out.append(("HB", np.arange(a, a + n, 4, dtype=np.uint64), np.full(n // 4, 4, np.uint32),
+                            np.full(n // 4, 3, np.uint8)))
+            else:
+                out.append(("HB", np.arange(a, a + n, dtype=np.uint64), np.ones(n, np.uint32), np.full(n, k, np.uint8)))
+        return out
+
+    ops += host_ops(expanded[:n_first]) + [("KB",)] + host_ops(expanded[n_first:]) + [("KE",)]
+    ops.append(("DIAG", 50, 0, 1, 1, ()))
+    exp = oracle_run(ops)
+    with xpl.Context(pool_words=1 << 20) as ctx:
+        for op in ops[:6]:
+            ctx.register(op[1], op[2], op[3])
+        rec = np.zeros(len(recs), dtype=xpl.HOST_STRIDED_DTYPE)
+        for f, k in zip(("addr", "size", "kind", "stride", "count"), range(5)):
+            rec[f] = [r[k] for r in recs]
+        ctx.record_host_strided(rec[:split])
+        s = torch.cuda.current_stream().cuda_stream
+        ctx.kernel_begin(s)
+        ctx.record_host_strided(rec[split:])
+        ctx.kernel_end(s)
+        got = [ctx.diagnose(50, 0, 1, True)]
+    compare(got, exp, "strided")
