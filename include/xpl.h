@@ -263,7 +263,14 @@ xpl_status xpl_shadow_dump(xpl_ctx* ctx, const void* base, uint64_t word0, uint6
 xpl_status xpl_flush(xpl_ctx* ctx);
 /* Wait for all runtime work enqueued so far. */
 xpl_status xpl_sync(xpl_ctx* ctx);
-/* The runtime's own stream (cudaStream_t as void*), e.g. for timing events. */
+/* Make `stream` (cudaStream_t as void*) wait on the device for every runtime
+ * operation enqueued so far (host merges, transfers' shadow updates, the last
+ * epoch's fold).  Runtime work runs on the runtime's own stream, or on the
+ * stream of the last single-stream epoch (its fold directly follows that
+ * epoch's kernels there).  No host blocking.  XPL_ERR_STATE inside an epoch. */
+xpl_status xpl_join(xpl_ctx* ctx, void* stream);
+/* The runtime's own stream (cudaStream_t as void*).  To order work or timing
+ * events after the runtime's work, use xpl_join on the stream first. */
 xpl_status xpl_runtime_stream(xpl_ctx* ctx, void** stream);
 xpl_status xpl_get_stats(xpl_ctx* ctx, xpl_stats* out);
 

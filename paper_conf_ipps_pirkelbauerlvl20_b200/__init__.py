@@ -8,8 +8,9 @@ There is no CPU fallback: importing `xpl` without the built library raises.
 import os
 
 PKG_DIR = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(PKG_DIR, "libxpl.so")
-WORK_PATH = os.path.join(PKG_DIR, "libxplwork.so")
+# (XPL_LIB_PATH: an alternative build of the same library, for A/B tuning runs)
+LIB_PATH = os.environ.get("XPL_LIB_PATH") or os.path.join(PKG_DIR, "libxpl.so")
+WORK_PATH = os.environ.get("XPL_WORK_PATH") or os.path.join(PKG_DIR, "libxplwork.so")
 
 
 def build(verbose=False):

@@ -32,7 +32,10 @@ constexpr uint32_t kP4 = 0x02020202u;
 // then, per listed super-chunk, warp w checks chunks [16w, 16w+16) and folds
 // the marked ones four at a time (128 B coalesced each).  Consecutive
 // super-chunks go to different CTAs, so a dense epoch spreads over the grid.
-// No global list, no atomics; cost O(super map + chunks written).
+// No global list, no atomics; cost O(super map + chunks written).  Launched
+// with programmatic stream serialization when it directly follows the epoch's
+// kernels on their stream: griddepcontrol.wait holds it until they are
+// complete, while its own launch overlaps their tail.
 constexpr int kFoldThreads = 256;
 
 __global__ void __launch_bounds__(kFoldThreads) fold_kernel(uint32_t* __restrict__ pool,
@@ -40,6 +43,7 @@ __global__ void __launch_bounds__(kFoldThreads) fold_kernel(uint32_t* __restrict
                                                             uint8_t* __restrict__ smap,
                                                             uint64_t n_super,
                                                             unsigned long long* stats) {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   __shared__ uint64_t s_list[kFoldThreads];
   __shared__ uint32_t s_n;
@@ -327,9 +331,10 @@ __device__ __noinline__ RunSum warp_runs(uint32_t m, uint32_t lane, uint32_t min
 }
 
 // Harley-Seal style vertical counter: bit j of plane k is bit k of the number of
-// ones seen at bit position j.  32 words (u32) per lane per tile -> 6 planes.
+// ones seen at bit position j.  Up to 4 x kDiagIters = 128 u32 per lane per tile
+// -> 8 planes (counts up to 255).
 struct VCount {
-  uint32_t p0 = 0, p1 = 0, p2 = 0, p3 = 0, p4 = 0, p5 = 0;
+  uint32_t p0 = 0, p1 = 0, p2 = 0, p3 = 0, p4 = 0, p5 = 0, p6 = 0, p7 = 0;
   __device__ __forceinline__ void add4(uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
     // two full adders into (p0, carries), then carries into p1, ripple up
     uint32_t u = p0 ^ a ^ b;
@@ -344,13 +349,17 @@ struct VCount {
     uint32_t t = p2 & c4; p2 ^= c4;
     uint32_t t2 = p3 & t; p3 ^= t;
     uint32_t t3 = p4 & t2; p4 ^= t2;
-    p5 ^= t3;
+    uint32_t t4 = p5 & t3; p5 ^= t3;
+    uint32_t t5 = p6 & t4; p6 ^= t4;
+    p7 ^= t5;
   }
   __device__ __forceinline__ uint32_t count(uint32_t mask) const {
     return __popc(p0 & mask) + 2 * __popc(p1 & mask) + 4 * __popc(p2 & mask) +
-           8 * __popc(p3 & mask) + 16 * __popc(p4 & mask) + 32 * __popc(p5 & mask);
+           8 * __popc(p3 & mask) + 16 * __popc(p4 & mask) + 32 * __popc(p5 & mask) +
+           64 * __popc(p6 & mask) + 128 * __popc(p7 & mask);
   }
 };
+static_assert(4 * kDiagIters <= 255, "vertical counter planes");
 
 // Per-byte flags, 0x80 in each byte where the predicate holds.
 __device__ __forceinline__ uint32_t derived_flags(uint32_t x) {
@@ -364,20 +373,18 @@ __device__ __forceinline__ uint32_t derived_flags(uint32_t x) {
 
 // Run summary updates of a warp's running summary A by one 512-word step that
 // is all zeros / all ones (the common cases; u32 arithmetic inside a tile).
-__device__ __forceinline__ void rs_append_zero(RunSum& a, uint32_t min_run) {
-  if (a.pre == a.len) {
-    a.pre = a.len;  // the leading run ends here
-  } else if (a.suf >= min_run && a.suf > 0) {
+__device__ __forceinline__ void rs_append_zero(RunSum& a, uint32_t min_run, uint32_t n = 512) {
+  if (a.pre != a.len && a.suf >= min_run && a.suf > 0) {  // an inner run ends here
     a.cnt += 1;
     a.sum += a.suf;
-  }
+  }  // (pre == len: the leading run ends here and stays the prefix)
   a.suf = 0;
-  a.len += 512;
+  a.len += n;
 }
-__device__ __forceinline__ void rs_append_full(RunSum& a) {
-  if (a.pre == a.len) a.pre += 512;
-  a.suf += 512;
-  a.len += 512;
+__device__ __forceinline__ void rs_append_full(RunSum& a, uint32_t n = 512) {
+  if (a.pre == a.len) a.pre += n;
+  a.suf += n;
+  a.len += n;
 }
 __device__ __forceinline__ RunSum rs_combine32(const RunSum& a, const RunSum& b, uint32_t min_run) {
   RunSum r;
@@ -474,6 +481,34 @@ __device__ __noinline__ void block_counts(uint32_t f0, uint32_t f1, uint32_t f2,
 struct TileAcc {
   VCount raw, der;
   RunSum wu = {0, 0, 0, 0, 0}, wd = {0, 0, 0, 0, 0};
+  // uniform 512-word steps (every record byte equal): counted by byte value,
+  // warp-uniform -- ub = the byte of the current stretch, un = its steps; the
+  // stretches already closed are added to the warp's counters in shared memory
+  uint32_t ub = 0, un = 0;
+  uint32_t* uc = nullptr;  // this warp's 9 counters (shared memory)
+  // Close the current stretch: its counts (lane 0, shared memory) and its run
+  // steps (warp-uniform; must precede any other step's run update).
+  __device__ __forceinline__ void close_uniform(uint32_t lane, uint32_t min_run) {
+    if (!un) return;
+    const uint32_t b = ub, n = un * 512;
+    if (lane == 0) {
+      const bool cpu = (b & 0x34u) != 0, gpu = (b & 0xC8u) != 0, wr = (b & 0x0Cu) != 0;
+      uc[0] += (b >> 2 & 1u) * n;  // wC
+      uc[1] += (b >> 3 & 1u) * n;  // wG
+      uc[2] += (b >> 4 & 1u) * n;  // rCC
+      uc[3] += (b >> 6 & 1u) * n;  // rCG
+      uc[4] += (b >> 5 & 1u) * n;  // rGC
+      uc[5] += (b >> 7 & 1u) * n;  // rGG
+      uc[6] += (cpu || gpu) ? n : 0u;
+      uc[7] += gpu ? n : 0u;
+      uc[8] += (cpu && gpu && wr) ? n : 0u;
+    }
+    if ((b & 0x44u) == 0x04u) rs_append_full(wu, n);  // u = wC & !rCG
+    else rs_append_zero(wu, min_run, n);
+    if (b & 0x10u) rs_append_full(wd, n);  // d = rCC
+    else rs_append_zero(wd, min_run, n);
+    un = 0;
+  }
 };
 
 // One 16-word lane step: TAIL = the warp's range may end inside the row.
@@ -481,6 +516,28 @@ template <bool TAIL, bool RESET, bool BLOCKS>
 __device__ __forceinline__ void tile_step(TileAcc& A, uint4 y, uint4* dst, uint32_t w, uint32_t live,
                                           uint32_t lane, uint32_t min_run, uint64_t rw0,
                                           uint64_t B, uint32_t* blk, uint64_t kb0) {
+  if (!BLOCKS) {
+    // Fast path: the warp's 512 words all hold the same record byte (long
+    // stretches of one access pattern are the common case of a real shadow).
+    const uint32_t u = y.x;
+    const bool lu = y.y == u && y.z == u && y.w == u && __byte_perm(u, 0, 0) == u &&
+                    (!TAIL || w - lane * 16 + 512 <= live);
+    const uint32_t u0 = __shfl_sync(0xFFFFFFFFu, u, 0);
+    if (__all_sync(0xFFFFFFFFu, lu && u == u0)) {
+      const uint32_t b = u0 & 0xFFu;
+      if (b != A.ub) {
+        A.close_uniform(lane, min_run);
+        A.ub = b;
+      }
+      A.un += 1;
+      if (RESET && (b & 0xFEu)) {
+        const uint32_t k = u0 & kL4;
+        *dst = make_uint4(k, k, k, k);
+      }
+      return;
+    }
+  }
+  A.close_uniform(lane, min_run);  // (a pending stretch precedes this step)
   uint32_t x[4] = {y.x, y.y, y.z, y.w};
   uint32_t keep[4] = {kL4, kL4, kL4, kL4};
   if (TAIL && w + 16 > live) {  // mask the words past the row's end
@@ -533,63 +590,131 @@ __device__ __forceinline__ void tile_step(TileAcc& A, uint4 y, uint4* dst, uint3
   }
 }
 
+// ---- 1D TMA (cp.async.bulk) staging of the shadow, one mbarrier per stage ----
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  uint32_t ok = 0;
+  do {
+    asm volatile(
+        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+        : "=r"(ok)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+  } while (!ok);
+}
+
+// The warp's staging ring: kDiagStages slots of kStageSteps 512-word steps each
+// (kStageSteps x 512 B of records), filled by 1D bulk copies (TMA) that lane 0
+// issues a whole ring ahead; each slot's mbarrier counts the bytes in.  No
+// register staging, so the prefetch depth (8 KB per warp) does not cost
+// registers (occupancy), and the wait + refill is paid once per kStageSteps.
+constexpr uint32_t kStageSteps = 4;
+constexpr uint32_t kDiagStages = 4;
+struct WarpRing {
+  uint4 buf[kDiagStages][kStageSteps * 32];
+  uint64_t bar[kDiagStages];
+};
+constexpr size_t kDiagSmem = (kDiagThreads / 32) * sizeof(WarpRing);
+
 template <bool TAIL, bool RESET, bool BLOCKS>
-__device__ __forceinline__ void tile_loop(TileAcc& A, uint4* p4, uint32_t live, uint32_t lane,
-                                          uint32_t min_run, uint64_t rw0, uint64_t B, uint32_t* blk,
-                                          uint64_t kb0 = 0) {
-  // 2-step software pipeline: the next two 512-word steps are in flight while
-  // the current two are processed (a small loop body for the instruction cache)
-  auto ld = [&](uint32_t it) {
-    const uint32_t w = it * 512 + lane * 16;
-    return (it < kDiagIters && (!TAIL || w < live)) ? p4[it * 32 + lane] : make_uint4(0, 0, 0, 0);
+__device__ __forceinline__ void tile_loop(TileAcc& A, WarpRing& R, uint4* p4, uint32_t live,
+                                          uint32_t lane, uint32_t min_run, uint64_t rw0, uint64_t B,
+                                          uint32_t* blk, uint64_t kb0 = 0) {
+  const uint32_t n = TAIL ? (live + 511) / 512 : kDiagIters;  // steps holding row words
+  const uint32_t ns = (n + kStageSteps - 1) / kStageSteps;     // stages
+  // bytes of stage j: whole 16-word vectors up to the row's end (the row's
+  // shadow span is a multiple of 16 words, so they are all inside it)
+  auto issue = [&](uint32_t j) {
+    const uint32_t words = TAIL ? min(kStageSteps * 512u, live - j * kStageSteps * 512) : kStageSteps * 512u;
+    bulk_load(R.buf[j % kDiagStages], p4 + j * kStageSteps * 32, ((words + 15) & ~15u),
+              &R.bar[j % kDiagStages]);
   };
-  uint4 a = ld(0), b = ld(1);
+  if (lane == 0)
+    for (uint32_t j = 0; j < ns && j < kDiagStages; ++j) issue(j);
 #pragma unroll 1
-  for (uint32_t it = 0; it < kDiagIters; it += 2) {
-    const uint4 na = ld(it + 2), nb = ld(it + 3);
-    tile_step<TAIL, RESET, BLOCKS>(A, a, p4 + it * 32 + lane, it * 512 + lane * 16, live, lane,
-                                   min_run, rw0, B, blk, kb0);
-    tile_step<TAIL, RESET, BLOCKS>(A, b, p4 + (it + 1) * 32 + lane, (it + 1) * 512 + lane * 16,
-                                   live, lane, min_run, rw0, B, blk, kb0);
-    a = na;
-    b = nb;
+  for (uint32_t j = 0; j < ns; ++j) {
+    const uint32_t st = j % kDiagStages;
+    mbar_wait(&R.bar[st], (j / kDiagStages) & 1u);
+#pragma unroll 1
+    for (uint32_t k = 0; k < kStageSteps; ++k) {
+      const uint32_t it = j * kStageSteps + k;
+      if (TAIL && it >= n) break;
+      const uint32_t w = it * 512 + lane * 16;
+      uint4 y = R.buf[st][k * 32 + lane];
+      if (TAIL && w >= live) y = make_uint4(0, 0, 0, 0);  // (bytes not copied this round)
+      tile_step<TAIL, RESET, BLOCKS>(A, y, p4 + it * 32 + lane, w, live, lane, min_run, rw0, B, blk, kb0);
+    }
+    __syncwarp();
+    if (lane == 0 && j + kDiagStages < ns) {
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // our reads before the refill
+      issue(j + kDiagStages);
+    }
   }
 }
 
-// One CTA = one tile of kTileWords words of one row; warp w owns a contiguous
-// quarter (4096 words); per step lane l owns 16 words (one uint4 of records).
-// Counts: two Harley-Seal vertical counters (raw record bits; derived per-word
-// any/gpu/alternating flags) popcounted once per tile.  Runs: ballot fast paths
-// for all-zero/all-one 512-word steps, warp_runs() for mixed ones.  Reset fused.
-__global__ void __launch_bounds__(kDiagThreads, 6) diag_tile_kernel(
-    const DiagRow* __restrict__ rows, const uint32_t* __restrict__ tile_row, DiagParams p,
-    uint32_t* __restrict__ pool, unsigned long long* __restrict__ cnt, TileSum* __restrict__ tiles,
+// One warp = one tile of kTileWords words of one row (no CTA-wide barrier: the
+// warps of a CTA are independent, so a warp on a cheap uniform stretch never
+// waits for one on a mixed stretch); per step lane l owns 16 words (one uint4
+// of records).  Counts: two Harley-Seal vertical counters (raw record bits;
+// derived per-word any/gpu/alternating flags) popcounted once per tile, plus
+// the uniform-step counts.  Runs: ballot fast paths for all-zero/all-one
+// 512-word steps, warp_runs() for mixed ones.  Reset fused.  The tile's counts
+// and run summaries go to tiles[t]; the stitch adds and combines them in order.
+#ifndef XPL_DIAG_MINB
+#define XPL_DIAG_MINB 3  // CTAs per SM the register budget is sized for
+#endif
+__global__ void __launch_bounds__(kDiagThreads, XPL_DIAG_MINB) diag_tile_kernel(
+    const DiagRow* __restrict__ rows, const uint32_t* __restrict__ tile_row, uint64_t ntiles,
+    DiagParams p, uint32_t* __restrict__ pool, TileSum* __restrict__ tiles,
     uint32_t* __restrict__ blk_cnt) {
   constexpr uint32_t kWarps = kDiagThreads / 32;
-  constexpr uint32_t kWarpWords = kTileWords / kWarps;
-  __shared__ uint32_t s_cnt[kWarps][9];
-  __shared__ RunSum s_u[kWarps], s_d[kWarps];
-  const uint64_t t = blockIdx.x;
+  __shared__ uint32_t s_uc[kWarps][9];
+  extern __shared__ __align__(128) unsigned char s_dyn[];
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint64_t t = (uint64_t)blockIdx.x * kWarps + warp;
+  if (t >= ntiles) return;
+  WarpRing& R = reinterpret_cast<WarpRing*>(s_dyn)[warp];
+  if (lane == 0) {
+    for (uint32_t k = 0; k < kDiagStages; ++k) mbar_init(&R.bar[k], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncwarp();
   const uint32_t ri = tile_row[t];
   const DiagRow row = rows[ri];
-  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const uint64_t ww0 = (t - row.tile0) * kTileWords + (uint64_t)warp * kWarpWords;  // row word
+  const uint64_t ww0 = (t - row.tile0) * kTileWords;  // row word
   const uint32_t min_run = (uint32_t)(p.min_run < 0xFFFFFFFFull ? p.min_run : 0xFFFFFFFFull);
-  const uint32_t live = row.words > ww0 ? (uint32_t)min(row.words - ww0, (uint64_t)kWarpWords) : 0u;
+  const uint32_t live = (uint32_t)min(row.words - ww0, (uint64_t)kTileWords);
   uint4* p4 = reinterpret_cast<uint4*>(pool) + ((row.off + ww0) >> 4);
   uint32_t* blk = blk_cnt + row.blk0;
   TileAcc A;
-  const bool tail = live < kWarpWords;
+  if (lane < 9) s_uc[warp][lane] = 0;
+  __syncwarp();
+  A.uc = s_uc[warp];
+  const bool tail = live < kTileWords;
   if (p.block_words) {  // rare: blocks need per-lane counter atomics (logical block index)
     const uint64_t kb0 = row.goff / p.block_words;
-    if (p.reset) tile_loop<true, true, true>(A, p4, live, lane, min_run, row.goff + ww0, p.block_words, blk, kb0);
-    else tile_loop<true, false, true>(A, p4, live, lane, min_run, row.goff + ww0, p.block_words, blk, kb0);
+    if (p.reset) tile_loop<true, true, true>(A, R, p4, live, lane, min_run, row.goff + ww0, p.block_words, blk, kb0);
+    else tile_loop<true, false, true>(A, R, p4, live, lane, min_run, row.goff + ww0, p.block_words, blk, kb0);
   } else if (p.reset) {
-    if (tail) tile_loop<true, true, false>(A, p4, live, lane, min_run, ww0, 0, blk);
-    else tile_loop<false, true, false>(A, p4, live, lane, min_run, ww0, 0, blk);
+    if (tail) tile_loop<true, true, false>(A, R, p4, live, lane, min_run, ww0, 0, blk);
+    else tile_loop<false, true, false>(A, R, p4, live, lane, min_run, ww0, 0, blk);
   } else {
-    if (tail) tile_loop<true, false, false>(A, p4, live, lane, min_run, ww0, 0, blk);
-    else tile_loop<false, false, false>(A, p4, live, lane, min_run, ww0, 0, blk);
+    if (tail) tile_loop<true, false, false>(A, R, p4, live, lane, min_run, ww0, 0, blk);
+    else tile_loop<false, false, false>(A, R, p4, live, lane, min_run, ww0, 0, blk);
   }
 
   // counters: 6 raw bit classes + any/gpu/alternating
@@ -603,28 +728,17 @@ __global__ void __launch_bounds__(kDiagThreads, 6) diag_tile_kernel(
   c9[6] = A.der.count(0x80808080u);  // any
   c9[7] = A.der.count(0x40404040u);  // gpu
   c9[8] = A.der.count(0x20202020u);  // alternating
+  A.close_uniform(lane, min_run);
+  __syncwarp();
+  TileSum* ts = tiles + t;
 #pragma unroll
   for (int k = 0; k < 9; ++k) {
     const uint32_t s = __reduce_add_sync(0xFFFFFFFFu, c9[k]);
-    if (lane == 0) s_cnt[warp][k] = s;
+    if (lane == k) ts->cnt[k] = s + A.uc[k];
   }
   if (lane == 0) {
-    s_u[warp] = A.wu;
-    s_d[warp] = A.wd;
-  }
-  __syncthreads();
-  if (threadIdx.x < 9) {
-    uint32_t s = 0;
-    for (uint32_t w = 0; w < kWarps; ++w) s += s_cnt[w][threadIdx.x];
-    if (s) atomicAdd(cnt + (uint64_t)ri * C_NCNT + threadIdx.x, (unsigned long long)s);
-  } else if (threadIdx.x == 32) {
-    RunSum a = s_u[0], b = s_d[0];
-    for (uint32_t w = 1; w < kWarps; ++w) {
-      a = rs_combine32(a, s_u[w], min_run);
-      b = rs_combine32(b, s_d[w], min_run);
-    }
-    tiles[t].u = a;
-    tiles[t].d = b;
+    ts->u = A.wu;
+    ts->d = A.wd;
   }
 }
 
@@ -671,7 +785,7 @@ __device__ __forceinline__ void warp_combine(RunSum64& a, RunSum64& b, uint32_t 
 // row; lanes combine contiguous sub-ranges, then an ordered warp reduction.
 __global__ void stitch_seg_kernel(const StitchSeg* __restrict__ segs, uint32_t nseg,
                                   const TileSum* __restrict__ tiles, uint64_t min_run,
-                                  RunPair* __restrict__ out) {
+                                  RunPair* __restrict__ out, unsigned long long* __restrict__ cnt) {
   const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const uint32_t lane = threadIdx.x & 31;
   if (gw >= nseg) return;
@@ -680,13 +794,22 @@ __global__ void stitch_seg_kernel(const StitchSeg* __restrict__ segs, uint32_t n
   const uint64_t t0 = sg.t0 + lane * per;
   const uint64_t t1 = min(sg.t0 + sg.n, t0 + per);
   RunSum64 a = {0, 0, 0, 0, 0}, b = {0, 0, 0, 0, 0};
+  uint64_t c9[9] = {0, 0, 0, 0, 0, 0, 0, 0, 0};
   for (uint64_t t = t0; t < t1; ++t) {
     const RunSum u = tiles[t].u, d = tiles[t].d;
     a = rs_combine(a, RunSum64{u.len, u.pre, u.suf, u.cnt, u.sum}, min_run);
     b = rs_combine(b, RunSum64{d.len, d.pre, d.suf, d.cnt, d.sum}, min_run);
+#pragma unroll
+    for (int k = 0; k < 9; ++k) c9[k] += tiles[t].cnt[k];
   }
   warp_combine(a, b, lane, min_run);
   if (lane == 0) out[gw] = RunPair{a, b};
+#pragma unroll
+  for (int k = 0; k < 9; ++k) {
+    uint64_t v = c9[k];
+    for (uint32_t o = 16; o; o >>= 1) v += __shfl_down_sync(0xFFFFFFFFu, v, o);
+    if (lane == 0 && v) atomicAdd(cnt + (uint64_t)sg.row * C_NCNT + k, (unsigned long long)v);
+  }
 }
 
 // Stitch, level 2 + finalize: one warp per row combines its segment summaries,
@@ -803,12 +926,19 @@ int grid_for(uint64_t n, int threads, int max_ctas) {
 
 }  // namespace
 
-void launch_fold(cudaStream_t s, uint32_t* pool, uint8_t* cmap, uint8_t* smap,
+void launch_fold(cudaStream_t s, bool pdl, uint32_t* pool, uint8_t* cmap, uint8_t* smap,
                  uint64_t n_super, unsigned long long* stats) {
-  if (n_super) {
-    const uint64_t g = n_super < 148 * 4 ? n_super : 148 * 4;  // one wave
-    fold_kernel<<<(unsigned)g, kFoldThreads, 0, s>>>(pool, cmap, smap, n_super, stats);
-  }
+  if (!n_super) return;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(n_super < 148 * 4 ? n_super : 148 * 4));  // one wave
+  cfg.blockDim = dim3(kFoldThreads);
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl ? 1 : 0;
+  cudaLaunchKernelEx(&cfg, fold_kernel, pool, cmap, smap, n_super, stats);
 }
 
 void launch_merge(cudaStream_t s, const uint64_t* recs, uint32_t n, bool has_r, bool has_w,
@@ -834,13 +964,18 @@ void launch_diag(cudaStream_t s, const DiagRow* rows, uint32_t nrows, const uint
   cudaMemsetAsync(cnt, 0, sizeof(unsigned long long) * C_NCNT * nrows, s);
   if (p.block_words && nblocks) cudaMemsetAsync(blk_cnt, 0, sizeof(uint32_t) * nblocks, s);
   if (tile_ev0) cudaEventRecord(tile_ev0, s);
-  if (ntiles) diag_tile_kernel<<<(unsigned)ntiles, kDiagThreads, 0, s>>>(rows, tile_row, p, pool, cnt, tiles, blk_cnt);
+  constexpr uint32_t kWarps = kDiagThreads / 32;
+  // (per device; cheap next to a diagnose)
+  cudaFuncSetAttribute(diag_tile_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kDiagSmem);
+  if (ntiles)
+    diag_tile_kernel<<<(unsigned)((ntiles + kWarps - 1) / kWarps), kDiagThreads, kDiagSmem, s>>>(
+        rows, tile_row, ntiles, p, pool, tiles, blk_cnt);
   if (tile_ev1) cudaEventRecord(tile_ev1, s);
   if (p.block_words && nblocks)
     block_eval_kernel<<<grid_for(nblocks, 256, 148 * 8), 256, 0, s>>>(rows, nrows, nblocks, blk_cnt,
                                                                     p.block_words, p.thr, cnt);
   stitch_seg_kernel<<<(nseg * 32 + 255) / 256, 256, 0, s>>>(segs, nseg, tiles, p.min_run,
-                                                             (RunPair*)segsum);
+                                                             (RunPair*)segsum, cnt);
   stitch_row_finalize_kernel<<<(nrows * 32 + 255) / 256, 256, 0, s>>>(rows, nrows, (const RunPair*)segsum,
                                                                        p, cnt, out, parts, blk_cnt);
 }

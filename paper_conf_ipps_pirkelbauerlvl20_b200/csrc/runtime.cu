@@ -76,7 +76,12 @@ cudaError_t host_alloc(T** p, size_t n) {
 
 struct xpl_ctx {
   xpl_config cfg;
-  cudaStream_t rs = nullptr;  // the runtime's stream
+  cudaStream_t rs = nullptr;  // the runtime's own stream
+  // The stream the runtime's latest work is on: rs, or the stream of the last
+  // single-stream epoch (its fold was enqueued right behind the epoch's kernels,
+  // so the next epoch on that stream needs no cross-stream event).  Every
+  // runtime enqueue goes to cs; switching streams always goes through an event.
+  cudaStream_t cs = nullptr;
 
   // shadow pool: 1 byte per word
   uint8_t* d_pool = nullptr;
@@ -95,16 +100,19 @@ struct xpl_ctx {
   const Row* cache = nullptr;          // last host lookup hit
 
   // epoch close: chunk maps (1 B per 128 words, 1 B per 16K words) + chunk list
-  uint8_t* d_cmap = nullptr;
-  uint8_t* d_smap = nullptr;
+  uint8_t* d_cmap = nullptr;           // 1 byte per 128-word chunk: GPU write pending
+  uint8_t* d_smap = nullptr;           // 1 byte per 16K-word super-chunk
   uint32_t* d_misc = nullptr;          // scratch counters
   unsigned long long* d_stats = nullptr;
 
   // epochs (D19)
   int depth = 0;
-  std::vector<cudaStream_t> epoch_streams;
+  std::vector<cudaStream_t> epoch_streams;  // streams that joined the open epoch
   std::vector<cudaEvent_t> ev_pool;
   cudaEvent_t ev_begin = nullptr;
+  bool ev_begin_valid = false;       // ev_begin recorded on cs for this epoch
+  bool cs_in_epoch = false;          // runtime work (D2D / memset) enqueued inside the epoch
+  cudaEvent_t ev_join = nullptr;
 
   // host-record staging (8-byte packed records)
   uint64_t* h_stage[2] = {nullptr, nullptr};
@@ -209,12 +217,12 @@ cudaEvent_t prof_event(xpl_ctx* c) {
 int prof_begin(xpl_ctx* c, int cls, uint64_t bytes, bool record = true) {
   if (!c->prof) return -1;
   xpl_ctx::ProfRec r{cls, prof_event(c), prof_event(c), bytes};
-  if (record) cudaEventRecord(r.a, c->rs);
+  if (record) cudaEventRecord(r.a, c->cs);
   c->prof_pending.push_back(r);
   return (int)c->prof_pending.size() - 1;
 }
 void prof_end(xpl_ctx* c, int i) {
-  if (i >= 0) cudaEventRecord(c->prof_pending[i].b, c->rs);
+  if (i >= 0) cudaEventRecord(c->prof_pending[i].b, c->cs);
 }
 
 uint64_t words_of(const uint64_t* h, size_t n) {
@@ -277,7 +285,7 @@ xpl_status ensure_ranges(xpl_ctx* c, size_t n) {
     CK(cudaEventSynchronize(c->ranges_ev));
     return XPL_OK;
   }
-  CK(cudaStreamSynchronize(c->rs));
+  CK(cudaStreamSynchronize(c->cs));
   if (c->h_ranges) cudaFreeHost(c->h_ranges);
   if (c->d_ranges) cudaFree(c->d_ranges);
   size_t cap = std::max<size_t>(n, 1024);
@@ -290,7 +298,7 @@ xpl_status ensure_ranges(xpl_ctx* c, size_t n) {
 xpl_status ensure_first_w(xpl_ctx* c) {
   if (c->d_first_w) return XPL_OK;
   CK(cudaMalloc(&c->d_first_w, sizeof(uint32_t) * c->pool_words));
-  launch_fill_u32(c->rs, c->d_first_w, c->pool_words, 0xFFFFFFFFu);
+  launch_fill_u32(c->cs, c->d_first_w, c->pool_words, 0xFFFFFFFFu);
   c->st.kernel_launches += 1;
   return XPL_OK;
 }
@@ -311,13 +319,13 @@ xpl_status flush(xpl_ctx* c) {
     else n_pieces += (nw + kPieceWords - 1) / kPieceWords;
   }
   if (n_long == 0 && n_pieces == n) {  // the common case: one merge segment as staged
-    CK(cudaMemcpyAsync(c->d_stage, h, n * sizeof(uint64_t), cudaMemcpyHostToDevice, c->rs));
-    CK(cudaEventRecord(c->stage_ev[c->cur], c->rs));
+    CK(cudaMemcpyAsync(c->d_stage, h, n * sizeof(uint64_t), cudaMemcpyHostToDevice, c->cs));
+    CK(cudaEventRecord(c->stage_ev[c->cur], c->cs));
     xpl_status s = XPL_OK;
     if (c->stage_has_r && c->stage_has_w) s = ensure_first_w(c);
     if (s) return s;
     const int pi = prof_begin(c, XPL_K_MERGE, c->prof ? 8 * n + 2 * words_of(h, n) : 0);
-    launch_merge(c->rs, c->d_stage, (uint32_t)n, c->stage_has_r, c->stage_has_w, c->d_first_w,
+    launch_merge(c->cs, c->d_stage, (uint32_t)n, c->stage_has_r, c->stage_has_w, c->d_first_w,
                  (uint32_t*)c->d_pool);
     prof_end(c, pi);
     c->st.kernel_launches += 1 + c->stage_has_w + (c->stage_has_r && c->stage_has_w);
@@ -327,7 +335,7 @@ xpl_status flush(xpl_ctx* c) {
     xpl_status s = ensure_ranges(c, n_long);
     if (s) return s;
     if (n_pieces > c->pieces_cap) {
-      CK(cudaStreamSynchronize(c->rs));
+      CK(cudaStreamSynchronize(c->cs));
       cudaFreeHost(c->h_pieces);
       cudaFree(c->d_pieces);
       c->pieces_cap = std::max<size_t>(n_pieces, 1 << 16);
@@ -384,13 +392,13 @@ xpl_status flush(xpl_ctx* c) {
         v += ((c->h_ranges[i].g0 + c->h_ranges[i].nw - 1) >> 4) - (c->h_ranges[i].g0 >> 4) + 1;
       }
     }
-    if (np) CK(cudaMemcpyAsync(c->d_pieces, c->h_pieces, sizeof(uint64_t) * np, cudaMemcpyHostToDevice, c->rs));
-    CK(cudaEventRecord(c->pieces_ev, c->rs));
+    if (np) CK(cudaMemcpyAsync(c->d_pieces, c->h_pieces, sizeof(uint64_t) * np, cudaMemcpyHostToDevice, c->cs));
+    CK(cudaEventRecord(c->pieces_ev, c->cs));
     if (nr_total)
       CK(cudaMemcpyAsync(c->d_ranges, c->h_ranges, sizeof(RangeDesc) * nr_total,
-                         cudaMemcpyHostToDevice, c->rs));
-    CK(cudaEventRecord(c->ranges_ev, c->rs));
-    CK(cudaEventRecord(c->stage_ev[c->cur], c->rs));  // (staging itself was not uploaded)
+                         cudaMemcpyHostToDevice, c->cs));
+    CK(cudaEventRecord(c->ranges_ev, c->cs));
+    CK(cudaEventRecord(c->stage_ev[c->cur], c->cs));  // (staging itself was not uploaded)
     for (const Seg& sg : segs) {
       if (sg.range) {
         const RangeDesc& last = c->h_ranges[sg.start + sg.n - 1];
@@ -398,7 +406,7 @@ xpl_status flush(xpl_ctx* c) {
         uint64_t rw = 0;
         for (size_t i = sg.start; i < sg.start + sg.n; ++i) rw += c->h_ranges[i].nw;
         const int pi = prof_begin(c, XPL_K_RANGE, 2 * rw);
-        launch_range(c->rs, c->d_ranges + sg.start, (uint32_t)sg.n, nvec, (uint32_t*)c->d_pool,
+        launch_range(c->cs, c->d_ranges + sg.start, (uint32_t)sg.n, nvec, (uint32_t*)c->d_pool,
                      c->d_cmap, c->d_smap);
         prof_end(c, pi);
         c->st.kernel_launches += 1;
@@ -409,7 +417,7 @@ xpl_status flush(xpl_ctx* c) {
           if (s) return s;
         }
         const int pi = prof_begin(c, XPL_K_MERGE, c->prof ? 8 * sg.n + 2 * words_of(c->h_pieces + sg.start, sg.n) : 0);
-        launch_merge(c->rs, c->d_pieces + sg.start, (uint32_t)sg.n, sg.has_r, sg.has_w,
+        launch_merge(c->cs, c->d_pieces + sg.start, (uint32_t)sg.n, sg.has_r, sg.has_w,
                      c->d_first_w, (uint32_t*)c->d_pool);
         prof_end(c, pi);
         c->st.kernel_launches += 1 + sg.has_w + (sg.has_r && sg.has_w);
@@ -440,8 +448,8 @@ xpl_status upload_table(xpl_ctx* c) {
     ++n;
   }
   memcpy(c->h_tab, &n, sizeof n);
-  CK(cudaMemcpyAsync(c->d_tab, c->h_tab, 32 + sizeof(xpl_dev_row) * n, cudaMemcpyHostToDevice, c->rs));
-  CK(cudaEventRecord(c->table_ev, c->rs));
+  CK(cudaMemcpyAsync(c->d_tab, c->h_tab, 32 + sizeof(xpl_dev_row) * n, cudaMemcpyHostToDevice, c->cs));
+  CK(cudaEventRecord(c->table_ev, c->cs));
   c->table_dirty = false;
   return XPL_OK;
 }
@@ -466,28 +474,37 @@ xpl_status gpu_ranges(xpl_ctx* c, const RangeDesc* rd, size_t nr) {
     c->h_ranges[i].vbase = v;
     v += ((c->h_ranges[i].g0 + c->h_ranges[i].nw - 1) >> 4) - (c->h_ranges[i].g0 >> 4) + 1;
   }
-  CK(cudaMemcpyAsync(c->d_ranges, c->h_ranges, sizeof(RangeDesc) * nr, cudaMemcpyHostToDevice, c->rs));
-  CK(cudaEventRecord(c->ranges_ev, c->rs));
+  CK(cudaMemcpyAsync(c->d_ranges, c->h_ranges, sizeof(RangeDesc) * nr, cudaMemcpyHostToDevice, c->cs));
+  CK(cudaEventRecord(c->ranges_ev, c->cs));
   uint64_t rw = 0;
   for (size_t i = 0; i < nr; ++i) rw += rd[i].nw;
   const int pi = prof_begin(c, XPL_K_RANGE, 2 * rw);
-  launch_range(c->rs, c->d_ranges, (uint32_t)nr, v, (uint32_t*)c->d_pool, c->d_cmap, c->d_smap);
+  launch_range(c->cs, c->d_ranges, (uint32_t)nr, v, (uint32_t*)c->d_pool, c->d_cmap, c->d_smap);
+  if (c->depth) c->cs_in_epoch = true;
   c->st.kernel_launches += 1;
   prof_end(c, pi);
   return cudaGetLastError() == cudaSuccess ? XPL_OK : XPL_ERR_CUDA;
 }
 
-void fold(xpl_ctx* c) {
+// Epoch close (D5): the fold on cs.  pdl = it directly follows the
+// epoch's kernels on the same stream (programmatic stream serialization).
+void fold(xpl_ctx* c, bool pdl) {
   const int pi = prof_begin(c, XPL_K_FOLD, 0);
-  // only super-chunks below the pool's high-water mark can be marked
-  launch_fold(c->rs, (uint32_t*)c->d_pool, c->d_cmap, c->d_smap, (c->pa.hwm + 16383) / 16384,
-              c->d_stats);
+  // only super-chunks below the pool's high-water mark can be flagged
+  launch_fold(c->cs, pdl && pi < 0, (uint32_t*)c->d_pool, c->d_cmap, c->d_smap,
+              (c->pa.hwm + 16383) / 16384, c->d_stats);
   c->folds_host++;
   c->st.kernel_launches += 1;
   prof_end(c, pi);
 }
 
-
+// Make stream s wait for every runtime enqueue so far (no-op when s is cs).
+xpl_status join(xpl_ctx* c, cudaStream_t s) {
+  if (s == c->cs) return XPL_OK;
+  CK(cudaEventRecord(c->ev_join, c->cs));
+  CK(cudaStreamWaitEvent(s, c->ev_join, 0));
+  return XPL_OK;
+}
 
 }  // namespace
 
@@ -528,20 +545,21 @@ xpl_status xpl_init(const xpl_config* cfg, xpl_ctx** out) {
   } while (0)
   CKI(cudaSetDevice(cfg->device));
   CKI(cudaStreamCreateWithFlags(&c->rs, cudaStreamNonBlocking));
+  c->cs = c->rs;
   CKI(cudaMalloc(&c->d_pool, c->pool_words));
-  CKI(cudaMemsetAsync(c->d_pool, 0, c->pool_words, c->rs));
+  CKI(cudaMemsetAsync(c->d_pool, 0, c->pool_words, c->cs));
   c->pa.init(c->pool_words);
   CKI(cudaMalloc(&c->d_tab, 32 + sizeof(xpl_dev_row) * c->cfg.max_rows));
-  CKI(cudaMemsetAsync(c->d_tab, 0, 32, c->rs));
+  CKI(cudaMemsetAsync(c->d_tab, 0, 32, c->cs));
   CKI(host_alloc(&c->h_tab, 32 + sizeof(xpl_dev_row) * c->cfg.max_rows));
   CKI(cudaMalloc(&c->d_cmap, c->pool_words / 128));
-  CKI(cudaMemsetAsync(c->d_cmap, 0, c->pool_words / 128, c->rs));
+  CKI(cudaMemsetAsync(c->d_cmap, 0, c->pool_words / 128, c->cs));
   CKI(cudaMalloc(&c->d_smap, c->pool_words / 16384));
-  CKI(cudaMemsetAsync(c->d_smap, 0, c->pool_words / 16384, c->rs));
+  CKI(cudaMemsetAsync(c->d_smap, 0, c->pool_words / 16384, c->cs));
   CKI(cudaMalloc(&c->d_misc, 64));
-  CKI(cudaMemsetAsync(c->d_misc, 0, 64, c->rs));
+  CKI(cudaMemsetAsync(c->d_misc, 0, 64, c->cs));
   CKI(cudaMalloc(&c->d_stats, 64));
-  CKI(cudaMemsetAsync(c->d_stats, 0, 64, c->rs));
+  CKI(cudaMemsetAsync(c->d_stats, 0, 64, c->cs));
   c->stage_cap = c->cfg.staging_recs;
   CKI(host_alloc(&c->h_stage[0], c->stage_cap));
   CKI(host_alloc(&c->h_stage[1], c->stage_cap));
@@ -551,15 +569,16 @@ xpl_status xpl_init(const xpl_config* cfg, xpl_ctx** out) {
   CKI(cudaEventCreateWithFlags(&c->table_ev, cudaEventDisableTiming));
   CKI(cudaEventCreateWithFlags(&c->ranges_ev, cudaEventDisableTiming));
   CKI(cudaEventCreateWithFlags(&c->pieces_ev, cudaEventDisableTiming));
-  CKI(cudaEventRecord(c->pieces_ev, c->rs));
+  CKI(cudaEventRecord(c->pieces_ev, c->cs));
   CKI(cudaEventCreateWithFlags(&c->ev_begin, cudaEventDisableTiming));
-  CKI(cudaEventRecord(c->stage_ev[0], c->rs));
-  CKI(cudaEventRecord(c->stage_ev[1], c->rs));
-  CKI(cudaEventRecord(c->table_ev, c->rs));
-  CKI(cudaEventRecord(c->ranges_ev, c->rs));
+  CKI(cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming));
+  CKI(cudaEventRecord(c->stage_ev[0], c->cs));
+  CKI(cudaEventRecord(c->stage_ev[1], c->cs));
+  CKI(cudaEventRecord(c->table_ev, c->cs));
+  CKI(cudaEventRecord(c->ranges_ev, c->cs));
   xpl_status s = ensure_ranges(c, 1024);
   if (s) { xpl_finalize(c); return s; }
-  CKI(cudaStreamSynchronize(c->rs));
+  CKI(cudaStreamSynchronize(c->cs));
   memset(&c->st, 0, sizeof c->st);
   *out = c;
   return XPL_OK;
@@ -568,6 +587,7 @@ xpl_status xpl_init(const xpl_config* cfg, xpl_ctx** out) {
 
 xpl_status xpl_finalize(xpl_ctx* c) {
   if (!c) return XPL_ERR_INVALID_ARG;
+  if (c->cs) cudaStreamSynchronize(c->cs);
   if (c->rs) cudaStreamSynchronize(c->rs);
   cudaFree(c->d_pool);
   cudaFree(c->d_first_w);
@@ -606,7 +626,7 @@ xpl_status xpl_finalize(xpl_ctx* c) {
   cudaFreeHost(c->h_pieces);
   cudaFree(c->d_pieces);
   for (cudaEvent_t e : {c->stage_ev[0], c->stage_ev[1], c->table_ev, c->ranges_ev, c->ev_begin,
-                        c->pieces_ev})
+                        c->pieces_ev, c->ev_join})
     if (e) cudaEventDestroy(e);
   if (c->rs) cudaStreamDestroy(c->rs);
   delete c;
@@ -641,7 +661,7 @@ static xpl_status register_row(xpl_ctx* c, const void* ptr, size_t bytes, xpl_al
   r.goff = piece ? goff : 0;
   r.lbytes = piece ? lbytes : bytes;
   if (!c->pa.alloc(r.span, &r.off)) return XPL_ERR_OOM;
-  CK(cudaMemsetAsync(c->d_pool + r.off, 0, r.span, c->rs));  // D3: last writer = CPU
+  CK(cudaMemsetAsync(c->d_pool + r.off, 0, r.span, c->cs));  // D3: last writer = CPU
   const size_t cap_before = c->rows.capacity();
   c->rows.push_back(r);
   if (c->rows.capacity() != cap_before) c->cache = nullptr;
@@ -673,6 +693,11 @@ xpl_status xpl_free(xpl_ctx* c, const void* ptr) {
   return XPL_OK;
 }
 
+// Epochs (D19).  The runtime's pending work (host merges, table
+// upload) sits on cs; a stream joining the epoch waits for it through ev_begin,
+// unless it is cs itself.  At the close, a single-stream epoch gets its fold
+// enqueued right behind its kernels on that stream (which becomes cs); several
+// streams are joined on rs first.
 xpl_status xpl_kernel_begin(xpl_ctx* c, void* stream) {
   if (!c) return XPL_ERR_INVALID_ARG;
   cudaStream_t s = (cudaStream_t)stream;
@@ -681,12 +706,19 @@ xpl_status xpl_kernel_begin(xpl_ctx* c, void* stream) {
     if (st) return st;
     st = upload_table(c);
     if (st) return st;
-    CK(cudaEventRecord(c->ev_begin, c->rs));
+    c->ev_begin_valid = false;
+    c->cs_in_epoch = false;
     c->epoch_streams.clear();
     c->st.epochs++;
   }
   if (std::find(c->epoch_streams.begin(), c->epoch_streams.end(), s) == c->epoch_streams.end()) {
-    CK(cudaStreamWaitEvent(s, c->ev_begin, 0));
+    if (s != c->cs) {
+      if (!c->ev_begin_valid) {
+        CK(cudaEventRecord(c->ev_begin, c->cs));
+        c->ev_begin_valid = true;
+      }
+      CK(cudaStreamWaitEvent(s, c->ev_begin, 0));
+    }
     c->epoch_streams.push_back(s);
   }
   c->depth++;
@@ -697,15 +729,34 @@ xpl_status xpl_kernel_end(xpl_ctx* c, void* stream) {
   if (!c) return XPL_ERR_INVALID_ARG;
   if (c->depth == 0) return XPL_ERR_STATE;
   cudaStream_t s = (cudaStream_t)stream;
-  if (std::find(c->epoch_streams.begin(), c->epoch_streams.end(), s) == c->epoch_streams.end())
+  if (std::find(c->epoch_streams.begin(), c->epoch_streams.end(), s) == c->epoch_streams.end()) {
+    if (s != c->cs && !c->ev_begin_valid) {  // (ended on a stream that never began)
+      CK(cudaEventRecord(c->ev_begin, c->cs));
+      c->ev_begin_valid = true;
+    }
+    if (s != c->cs) CK(cudaStreamWaitEvent(s, c->ev_begin, 0));
     c->epoch_streams.push_back(s);
-  if (--c->depth) return XPL_OK;
-  for (size_t i = 0; i < c->epoch_streams.size(); ++i) {
-    cudaEvent_t e = pool_event(c, i);
-    CK(cudaEventRecord(e, c->epoch_streams[i]));
-    CK(cudaStreamWaitEvent(c->rs, e, 0));
   }
-  fold(c);
+  if (--c->depth) return XPL_OK;
+  // the stream the fold goes on, and everything of the epoch that must precede it
+  const bool single = c->epoch_streams.size() == 1;
+  cudaStream_t t = single ? c->epoch_streams[0] : c->rs;
+  std::vector<cudaStream_t> wait = c->epoch_streams;
+  // cs: only in-epoch D2D / memset work is not yet ordered before the epoch's
+  // streams (everything earlier was, through ev_begin)
+  if (c->cs_in_epoch) wait.push_back(c->cs);
+  size_t k = 0;
+  bool crossed = false;
+  for (size_t i = 0; i < wait.size(); ++i) {
+    const cudaStream_t x = wait[i];
+    if (x == t || std::find(wait.begin(), wait.begin() + i, x) != wait.begin() + i) continue;
+    cudaEvent_t e = pool_event(c, k++);
+    CK(cudaEventRecord(e, x));
+    CK(cudaStreamWaitEvent(t, e, 0));
+    crossed = true;
+  }
+  c->cs = t;
+  fold(c, !crossed);
   if (cudaGetLastError() != cudaSuccess) return XPL_ERR_CUDA;
   std::vector<uint64_t> q;
   q.swap(c->deferred);
@@ -864,7 +915,7 @@ xpl_status xpl_record_copy(xpl_ctx* c, const void* dst, const void* src, size_t 
   }
   xpl_status s = gpu_ranges(c, rd, nr);
   if (s) return s;
-  if (own) fold(c);
+  if (own) fold(c, false);
   return cudaGetLastError() == cudaSuccess ? XPL_OK : XPL_ERR_CUDA;
 }
 
@@ -875,8 +926,15 @@ xpl_status xpl_flush(xpl_ctx* c) {
 
 xpl_status xpl_sync(xpl_ctx* c) {
   if (!c) return XPL_ERR_INVALID_ARG;
-  CK(cudaStreamSynchronize(c->rs));
+  CK(cudaStreamSynchronize(c->cs));
+  if (c->cs != c->rs) CK(cudaStreamSynchronize(c->rs));
   return XPL_OK;
+}
+
+xpl_status xpl_join(xpl_ctx* c, void* stream) {
+  if (!c) return XPL_ERR_INVALID_ARG;
+  if (c->depth) return XPL_ERR_STATE;
+  return join(c, (cudaStream_t)stream);
 }
 
 xpl_status xpl_runtime_stream(xpl_ctx* c, void** s) {
@@ -898,7 +956,7 @@ xpl_status xpl_get_device_ctx(xpl_ctx* c, struct xpl_dev_ctx* d) {
 xpl_status xpl_get_stats(xpl_ctx* c, xpl_stats* o) {
   if (!c || !o) return XPL_ERR_INVALID_ARG;
   unsigned long long ds[8];
-  CK(cudaStreamSynchronize(c->rs));
+  CK(cudaStreamSynchronize(c->cs));
   CK(cudaMemcpy(ds, c->d_stats, sizeof ds, cudaMemcpyDeviceToHost));
   *o = c->st;
   o->fold_chunks_max = 0;  // (not tracked by the one-kernel fold)
@@ -911,7 +969,7 @@ xpl_status xpl_profile(xpl_ctx* c, int enable) {
   if (!c) return XPL_ERR_INVALID_ARG;
   if (enable && !c->prof) {
     memset(c->prof_acc, 0, sizeof c->prof_acc);
-    CK(cudaStreamSynchronize(c->rs));
+    CK(cudaStreamSynchronize(c->cs));
     unsigned long long ds[8];
     CK(cudaMemcpy(ds, c->d_stats, sizeof ds, cudaMemcpyDeviceToHost));
     c->fold_entries_seen = ds[3];
@@ -922,7 +980,7 @@ xpl_status xpl_profile(xpl_ctx* c, int enable) {
 
 xpl_status xpl_profile_read(xpl_ctx* c, xpl_kernel_time* out, int reset) {
   if (!c || !out) return XPL_ERR_INVALID_ARG;
-  CK(cudaStreamSynchronize(c->rs));
+  CK(cudaStreamSynchronize(c->cs));
   for (auto& r : c->prof_pending) {
     float ms = 0.f;
     CK(cudaEventElapsedTime(&ms, r.a, r.b));
@@ -951,8 +1009,8 @@ xpl_status xpl_shadow_dump(xpl_ctx* c, const void* base, uint64_t word0, uint64_
   if (word0 > r.words || n > r.words - word0) return XPL_ERR_INVALID_ARG;
   xpl_status s = flush(c);
   if (s) return s;
-  CK(cudaMemcpyAsync(out, c->d_pool + r.off + word0, n, cudaMemcpyDeviceToHost, c->rs));
-  CK(cudaStreamSynchronize(c->rs));
+  CK(cudaMemcpyAsync(out, c->d_pool + r.off + word0, n, cudaMemcpyDeviceToHost, c->cs));
+  CK(cudaStreamSynchronize(c->cs));
   return XPL_OK;
 }
 
@@ -1057,35 +1115,36 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
     for (uint64_t k = 0; k < d.nseg; ++k) {
       c->h_segs[sgi + k].t0 = t + k * kSegTiles;
       c->h_segs[sgi + k].n = std::min<uint64_t>(kSegTiles, d.ntiles - k * kSegTiles);
+      c->h_segs[sgi + k].row = i;
     }
     sgi += d.nseg;
     for (uint64_t k = 0; k < d.ntiles; ++k) c->h_tile_row[t + k] = (uint32_t)i;
     t += d.ntiles;
     b += d.nblk;
   }
-  CK(cudaMemcpyAsync(c->d_drows, c->h_drows, sizeof(DiagRow) * nr, cudaMemcpyHostToDevice, c->rs));
+  CK(cudaMemcpyAsync(c->d_drows, c->h_drows, sizeof(DiagRow) * nr, cudaMemcpyHostToDevice, c->cs));
   CK(cudaMemcpyAsync(c->d_tile_row, c->h_tile_row, sizeof(uint32_t) * ntiles,
-                     cudaMemcpyHostToDevice, c->rs));
-  CK(cudaMemcpyAsync(c->d_segs, c->h_segs, sizeof(StitchSeg) * nseg, cudaMemcpyHostToDevice, c->rs));
+                     cudaMemcpyHostToDevice, c->cs));
+  CK(cudaMemcpyAsync(c->d_segs, c->h_segs, sizeof(StitchSeg) * nseg, cudaMemcpyHostToDevice, c->cs));
   uint64_t total_words = 0;
   for (size_t i = 0; i < nr; ++i) total_words += c->h_drows[i].words;
   const uint64_t dbytes = total_words * (reset ? 2 : 1);
   const int pall = prof_begin(c, XPL_K_DIAGNOSE, dbytes);
   const int ptile = prof_begin(c, XPL_K_DIAG_TILE, dbytes, false);  // recorded by launch_diag
-  launch_diag(c->rs, c->d_drows, (uint32_t)nr, c->d_tile_row, ntiles, c->d_segs, (uint32_t)nseg,
+  launch_diag(c->cs, c->d_drows, (uint32_t)nr, c->d_tile_row, ntiles, c->d_segs, (uint32_t)nseg,
               nblocks, p, (uint32_t*)c->d_pool, c->d_cnt, c->d_tiles, c->d_segsum, c->d_blk, c->d_rep,
               pout ? c->d_rpart : nullptr, ptile >= 0 ? c->prof_pending[ptile].a : nullptr,
               ptile >= 0 ? c->prof_pending[ptile].b : nullptr);
   CK(cudaGetLastError());
   c->st.kernel_launches += 3 + (B && nblocks ? 1 : 0);
-  CK(cudaMemcpyAsync(c->h_rep, c->d_rep, sizeof(xpl_alloc_report) * nr, cudaMemcpyDeviceToHost, c->rs));
+  CK(cudaMemcpyAsync(c->h_rep, c->d_rep, sizeof(xpl_alloc_report) * nr, cudaMemcpyDeviceToHost, c->cs));
   if (pout) {
-    CK(cudaMemcpyAsync(c->h_rpart, c->d_rpart, sizeof(RowPartial) * nr, cudaMemcpyDeviceToHost, c->rs));
+    CK(cudaMemcpyAsync(c->h_rpart, c->d_rpart, sizeof(RowPartial) * nr, cudaMemcpyDeviceToHost, c->cs));
     CK(cudaMemcpyAsync(c->h_cnt, c->d_cnt, sizeof(unsigned long long) * C_NCNT * nr,
-                       cudaMemcpyDeviceToHost, c->rs));
+                       cudaMemcpyDeviceToHost, c->cs));
   }
   prof_end(c, pall);
-  CK(cudaStreamSynchronize(c->rs));
+  CK(cudaStreamSynchronize(c->cs));
 
   std::vector<uint32_t> name_of(nr, 0xFFFFFFFFu);
   c->cache = nullptr;  // names (XplAllocData): the first name inside a live row

@@ -41,9 +41,9 @@ struct RangeDesc {
 };
 
 // Diagnose geometry.
-constexpr uint32_t kTileWords = 16384;         // words per diagnose tile (one CTA)
-constexpr uint32_t kDiagThreads = 128;         // 4 warps x 32 lanes x 16 words x 8 iters
-constexpr uint32_t kDiagIters = 8;
+constexpr uint32_t kTileWords = 16384;         // words per diagnose tile (one warp)
+constexpr uint32_t kDiagIters = 32;            // 512-word steps per tile (32 lanes x 16 words)
+constexpr uint32_t kDiagThreads = 256;         // 8 independent warps (tiles) per CTA
 
 struct DiagRow {        // one row to analyse (live or dead-since-last-reset)
   uint64_t off, words;  // pool offset (multiple of 16), words
@@ -64,9 +64,10 @@ struct RowPartial {
 };
 
 // Stitch segment: <= kSegTiles consecutive tiles of one row.
-constexpr uint64_t kSegTiles = 1024;
+constexpr uint64_t kSegTiles = 128;
 struct StitchSeg {
   uint64_t t0, n;
+  uint64_t row;  // the row (report index) the segment belongs to
 };
 
 // Per-row counters accumulated by the diagnose kernels (u64 each).
@@ -80,7 +81,9 @@ struct RunSum {
   uint32_t len, pre, suf, cnt, sum;
 };
 struct TileSum {
-  RunSum u, d;  // u = wC & !rCG (unneeded H2D), d = rCC (unneeded D2H)
+  RunSum u, d;      // u = wC & !rCG (unneeded H2D), d = rCC (unneeded D2H)
+  uint32_t cnt[9];  // wC wG rCC rCG rGC rGG any gpu alternating (C_WC .. C_ALT)
+  uint32_t pad;
 };
 
 struct DiagParams {
@@ -91,7 +94,7 @@ struct DiagParams {
 };
 
 // ---- launchers (kernels.cu) ----
-void launch_fold(cudaStream_t s, uint32_t* pool, uint8_t* cmap, uint8_t* smap,
+void launch_fold(cudaStream_t s, bool pdl, uint32_t* pool, uint8_t* cmap, uint8_t* smap,
                  uint64_t n_super, unsigned long long* stats);
 void launch_merge(cudaStream_t s, const uint64_t* recs, uint32_t n, bool has_r, bool has_w,
                   uint32_t* first_w, uint32_t* pool);

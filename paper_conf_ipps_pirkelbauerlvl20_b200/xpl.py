@@ -112,6 +112,7 @@ xpl_get_device_ctx = _sig("xpl_get_device_ctx", [vp, C.POINTER(XplDevCtx)])
 xpl_shadow_dump = _sig("xpl_shadow_dump", [vp, vp, u64, u64, vp])
 xpl_flush = _sig("xpl_flush", [vp])
 xpl_sync = _sig("xpl_sync", [vp])
+xpl_join = _sig("xpl_join", [vp, vp])
 xpl_runtime_stream = _sig("xpl_runtime_stream", [vp, C.POINTER(vp)])
 xpl_get_stats = _sig("xpl_get_stats", [vp, C.POINTER(XplStats)])
 xpl_status_string = _sig("xpl_status_string", [i32], C.c_char_p)
@@ -127,7 +128,7 @@ xpl_profile_read = _sig("xpl_profile_read", [vp, C.POINTER(XplKernelTime), i32])
 
 EXPORTED = ["xpl_init", "xpl_finalize", "xpl_register_alloc", "xpl_free", "xpl_kernel_begin",
             "xpl_kernel_end", "xpl_record_host", "xpl_record_host_ranges", "xpl_record_host_strided", "xpl_record_copy", "xpl_diagnose",
-            "xpl_get_device_ctx", "xpl_shadow_dump", "xpl_flush", "xpl_sync",
+            "xpl_get_device_ctx", "xpl_shadow_dump", "xpl_flush", "xpl_sync", "xpl_join",
             "xpl_runtime_stream", "xpl_get_stats", "xpl_status_string", "xpl_profile",
             "xpl_profile_read", "xpl_register_alloc_piece", "xpl_diagnose_partials", "xpl_combine_partials",
             "xpl_format_reports"]
@@ -251,6 +252,10 @@ class Context:
 
     def sync(self):
         check("xpl_sync", xpl_sync(self.h))
+
+    def join(self, stream):
+        """Make `stream` wait (on the device) for all runtime work enqueued so far."""
+        check("xpl_join", xpl_join(self.h, stream))
 
     def runtime_stream(self):
         s = vp()

@@ -8,7 +8,7 @@ import numpy as np
 import pytest
 
 from oracle import run_trace as oracle_run
-from xplgen.trace import (DEVICE, MANAGED, SEG_OPS, enumerated_trace, parse_text, random_trace,
+from xplgen.trace import (DEVICE, MANAGED, RW, SEG_OPS, R, W, enumerated_trace, parse_text, random_trace,
                           schedules)
 
 pytestmark = pytest.mark.gpu
@@ -281,3 +281,48 @@ def test_host_strided(gpu, seed):
         ctx.kernel_end(s)
         got = [ctx.diagnose(50, 0, 1, True)]
     compare(got, exp, "strided")
+
+
+def stretch_trace(seed, words=(300_000, 70_001, 16_384 * 3)):
+    """Long stretches of identical record bytes (the diagnose kernel's uniform
+    512-word fast path) with ragged, unaligned stretch ends, so steps are uniform,
+    mixed, and uniform with a different byte than the step before; every access
+    recipe is applied to a whole stretch (transfers + dense device batches)."""
+    rng = np.random.default_rng(seed)
+    ops, allocs = [], []
+    b = 0x3000_0000
+    for i, w in enumerate(words):
+        ops.append(("REG", b, 4 * w, (DEVICE, MANAGED, DEVICE)[i]))
+        allocs.append((b, w))
+        b += ((4 * w + 65535) // 65536 + 1) * 65536
+    recipes = ["HW", "GR", "HR", "GW", "GRW", "HW GR", "GW HR", "HW HR GR GW", "GR HW", ""]
+    for rnd in range(3):
+        for base, w in allocs:
+            cuts = np.sort(rng.choice(np.arange(1, w), size=min(w - 1, 40), replace=False))
+            cuts = np.concatenate([[0], cuts, [w]])
+            # bias some cuts onto 512-word boundaries
+            cuts = np.where(rng.random(cuts.size) < 0.5, (cuts // 512) * 512, cuts)
+            cuts = np.unique(np.clip(cuts, 0, w))
+            for s, e in zip(cuts[:-1], cuts[1:]):
+                if e <= s:
+                    continue
+                a0, nb = base + 4 * int(s), 4 * int(e - s)
+                for step in recipes[int(rng.integers(0, len(recipes)))].split():
+                    if step == "HW":
+                        ops.append(("X", 0, a0, 0x7000_0000, nb))
+                    elif step == "HR":
+                        ops.append(("X", 1, 0x7000_0000, a0, nb))
+                    else:
+                        acc = {"GR": R, "GW": W, "GRW": RW}[step]
+                        a = a0 + 4 * np.arange(nb // 4, dtype=np.uint64)
+                        ops += [("KB",), ("DB", a, np.full(a.size, 4, np.uint32), np.full(a.size, acc, np.uint8)), ("KE",)]
+        for params, reset in (((50, 0, 256), 0), ((50, 0, 1), 0), ((30, 0, 5000), rnd % 2)):
+            ops.append(("DIAG", *params, reset, ()))
+    return ops
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_uniform_stretches(gpu, seed):
+    replay, _ = gpu
+    ops = stretch_trace(0x58504C40 + seed)
+    compare(replay.run_trace(ops, pool_words=1 << 22), oracle_run(ops), "stretches")
