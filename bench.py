@@ -43,6 +43,7 @@ BFS = (1000000, 6)
 NW = (2048, 10)
 PARAMS = (50, 0, 256)  # threshold 50 %, whole-allocation blocks, min run 256 words
 WORKLOAD = "rodinia: hotspot 1024x1024x20 + backprop 640Kx16 + bfs 1Mx6 + nw 2048x2048"
+METRIC = "recorded accesses/s (host tracer + device hooks + transferred words)"
 
 
 def parse():
@@ -53,6 +54,8 @@ def parse():
     ap.add_argument("--impl", choices=["xpl", "reference"], default="xpl")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-other-configs", action="store_true")
+    ap.add_argument("--step-only", action="store_true",
+                    help="warm-up + timed steps only, no JSON line (for ncu captures of the step's kernels)")
     return ap.parse_args()
 
 
@@ -105,9 +108,11 @@ class Clocks:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
-def cpu_baseline(seconds_budget=20.0):
+def cpu_baseline(seconds_budget=None):
     """The oracle as it stands, on a bounded sample of the same workload:
-    hotspot 1024x1024 (first iterations) replayed event by event."""
+    hotspot 1024x1024 (first iterations) replayed event by event (~8-15 s on one
+    core).  seconds_budget: stop early (untimed warm-up only -- the count would
+    then not match the work done)."""
     from oracle import Oracle
     from xplgen import rodinia
     rows, cols, _ = HOT
@@ -122,7 +127,7 @@ def cpu_baseline(seconds_budget=20.0):
         if op[0] == "X" and op[1] == 1:  # stop before the final transfer: sample = init + iterations
             break
         o.op(op)
-        if time.perf_counter() - t0 > seconds_budget * 3:
+        if seconds_budget is not None and time.perf_counter() - t0 > seconds_budget:
             break
     dt = time.perf_counter() - t0
     o.close()
@@ -323,14 +328,16 @@ def reference_main(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
+    for _ in range(args.warmup):  # untimed warm-up samples (short)
+        cpu_baseline(seconds_budget=1.0)
     steps = []
     for _ in range(max(1, args.steps)):
-        steps.append(cpu_baseline(seconds_budget=5.0))
+        steps.append(cpu_baseline())
     v = statistics.median(s["value"] for s in steps)
-    line = {"impl": "reference", "metric": "recorded accesses/s", "value": v, "unit": "accesses/s",
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "accesses/s",
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8",
-            "data": "synthetic", "config": {"workload": WORKLOAD + " (oracle sample)"},
+            "data": "synthetic", "config": {"workload": WORKLOAD},
             "cpu_baseline": {"value": v, "unit": "accesses/s", "cores": 1, "kind": "oracle",
                              "sample": steps[0]["sample"]},
             "e2e": {"value": v, "unit": "accesses/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -438,6 +445,9 @@ def main():
     per_step = counts[0] + counts[1] + counts[2]
     ms_max = _allmax(torch, dist, ms_total)
     value = per_step * args.steps * world / (ms_max / 1e3)
+    if args.step_only:
+        ctx.close()
+        return
     launches = (st1["kernel_launches"] - st0["kernel_launches"]) + counts[3] * args.steps
 
     # --- e2e: with the programs' real copies -----------------------------------
@@ -487,14 +497,20 @@ def main():
     dom = max(("diag_tile", "merge", "range", "fold"), key=lambda k: prof[k]["ms"])
     d = prof[dom]
     achieved = (d["bytes"] / d["launches"]) / (d["ms"] / d["launches"] / 1e3) / 1e9 if d["launches"] else 0.0
+    traffic = None  # DRAM bytes per launch of that kernel from an ncu capture (profiles/traffic.json)
+    try:
+        tj = json.load(open(os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles", "traffic.json")))
+        traffic = tj[dom]["bytes_per_launch"] if dom in tj else None
+    except (OSError, ValueError, KeyError):
+        pass
     roof = {"kernel": dom, "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-            "frac": achieved / peak, "traffic": None, "peak_source": peak_src,
+            "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
             "algorithmic_bytes_per_launch": d["bytes"] / max(1, d["launches"]),
             "avg_launch_ms": d["ms"] / max(1, d["launches"]),
             "share_of_step": d["ms"] / ms_total}
     dg = prof["diag_tile"]
     line = {
-        "metric": "recorded accesses/s (host tracer + device hooks + transferred words)",
+        "metric": METRIC,
         "value": value, "unit": "accesses/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": ms_max / args.steps, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u8", "data": "synthetic",

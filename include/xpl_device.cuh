@@ -21,7 +21,8 @@
  *  3. warp aggregation: lanes that hit the same shadow u32 (4 records) are grouped
  *     with __match_any_sync, their bits combined (per-byte-lane ballots), and one
  *     leader issues a single atomicOr -- and only if some bit is still missing
- *     (test before set);
+ *     (test before set; write-only call sites skip the test: their bits do not
+ *     depend on the record, so they need no shadow load at all);
  *  4. a write also marks its 128-word chunk (and 16K-word super-chunk) in two
  *     byte maps with plain idempotent stores (test before store, no atomics),
  *     so closing the epoch costs O(chunks written), not O(shadow).
@@ -169,10 +170,12 @@ static __device__ __forceinline__ void xpl_dev_apply(unsigned long long g0,
     const unsigned bytes = 0xFFu << (8 * (unsigned)(g0 & 3));
     unsigned cur = 0, m = 0;
     if (hit) {
-      cur = xpl_dctx.pool[q];
+      /* a write's bits (wG | P) do not depend on L: write-only call sites skip
+       * the shadow load (and its latency) and always commit */
+      cur = K == XPL_ACC_W ? 0u : xpl_dctx.pool[q];
       m = xpld_bits(cur, bytes, acc);
     }
-    const bool need = hit && (cur & m) != m;
+    const bool need = hit && (K == XPL_ACC_W || (cur & m) != m);
     const unsigned needers = __ballot_sync(singles, need);
     if (need) xpld_commit<K, true>(needers, q, cur, bytes, acc);
   }
@@ -185,7 +188,7 @@ static __device__ __forceinline__ void xpl_dev_apply(unsigned long long g0,
   while (__any_sync(active, more)) {
     unsigned cur = 0, m = 0, bytes = 0;
     if (more) {
-      cur = xpl_dctx.pool[q];
+      cur = K == XPL_ACC_W ? 0u : xpl_dctx.pool[q];
 #pragma unroll
       for (unsigned k = 0; k < 4; ++k) {
         const unsigned long long gw = q * 4 + k;
@@ -193,7 +196,7 @@ static __device__ __forceinline__ void xpl_dev_apply(unsigned long long g0,
       }
       m = xpld_bits(cur, bytes, acc);
     }
-    const bool need = more && (cur & m) != m;
+    const bool need = more && (K == XPL_ACC_W || (cur & m) != m);
     const unsigned needers = __ballot_sync(active, need);
     if (need) xpld_commit<K, false>(needers, (unsigned)q, cur, bytes, acc);
     more = more && q < ql;

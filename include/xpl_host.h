@@ -34,15 +34,6 @@
  *
  * A hint is only a starting point: whatever run it names is checked like any
  * other, so a stale hint costs a slow-path call, never a wrong record.
- *
- * Owned runs.  A site that extended a run at its end becomes the run's owner
- * and keeps the run's end, cap and kind in its own fields (locals of the
- * instrumented loop, so the compiler keeps them in registers).  While it owns
- * the run, an access at the site's cached end is a compare and one store (the
- * new end, never re-loaded on this path): no load -> store -> load chain
- * through the tracer's state per access.  Every other change of a run (another
- * site or the general path extending it, a close, a new cap) clears the run's
- * owner, and the owner re-checks `run->owner == this` on every access.
  */
 #ifndef XPL_HOST_H
 #define XPL_HOST_H
@@ -54,15 +45,9 @@
 
 #ifdef __cplusplus
 
-/* Per-access-site hint (a local of the instrumented code; see above).  Passed
- * by value to the tracer's out-of-line path and returned, so its address never
- * escapes and the compiler can keep it in registers across a loop. */
+/* Per-access-site hint (a local of the instrumented code; see above). */
 struct xpl_host_site {
-  uint64_t end = 0, cap = 0; /* owned run: its end and cap (valid while run->owner == id) */
-  void* run = nullptr;       /* the run this site owns (or owned)                      */
-  uint32_t kind = 0;         /* owned run: its kind                                     */
-  uint32_t slot = 0;         /* the run slot the site used last                        */
-  uint32_t id = 0;           /* the site's owner token (0: none assigned yet)          */
+  uint32_t slot = 0;
 };
 
 class xpl_host_tracer {
@@ -84,20 +69,12 @@ class xpl_host_tracer {
     }
     slow(a, size, kind);
   }
-  /* The same access with a site hint: extend the run the site owns, else try
-   * the run the site used last, else the slow path; then try to own the run. */
+  /* The same access with a site hint: try the run the site used last. */
   __attribute__((always_inline)) inline void access(const void* p, uint32_t size, uint32_t kind,
                                                     xpl_host_site& s) {
     const uint64_t a = (uint64_t)p;
-    Run* o = static_cast<Run*>(s.run);
-    if (a == s.end && kind == s.kind && a + size <= s.cap && o && o->owner == s.id &&
-        (kind != XPL_ACC_RW || ((a | size) & 3u) == 0)) {
-      s.end = a + size;
-      o->end = s.end;
-      return;
-    }
-    if (site_hit(&run_[s.slot < (uint32_t)kRuns ? s.slot : (uint32_t)kRuns], a, size, kind, s)) return;
-    s = site_access(a, size, kind, s);
+    if (hit(&run_[s.slot], a, size, kind)) return;
+    s.slot = slow(a, size, kind);
   }
   template <class T>
   inline const T& read(const T& x, xpl_host_site& s) {
@@ -156,47 +133,7 @@ class xpl_host_tracer {
     uint16_t kind = 0;          // 0 = slot free (16 bits: no aliasing with int/uint32 data)
     uint16_t grew = 0;          // repeated since opened (extension: end != end0)
     Run* next = nullptr;        // the run used after this one last time (a prediction)
-    uint32_t owner = 0;         // id of the site caching end/cap/kind (0: none; see above)
   };
-  /* Site s takes over run r (whose end its access just became). */
-  inline void own(Run* r, xpl_host_site& s) {
-    if (!s.id) s.id = ++site_ids_;
-    Run* o = static_cast<Run*>(s.run);
-    if (o && o != r && o->owner == s.id) o->owner = 0;
-    r->owner = s.id;
-    s.run = r;
-    s.end = r->end;
-    s.cap = r->cap;
-    s.kind = r->kind;
-  }
-  /* hit() for a site: an extension hands the run to the site unless another
-   * site owns it (then nobody does: interleaved streams on one run, e.g. the
-   * fields of a struct array, stay on this path instead of trading it). */
-  inline bool site_hit(Run* r, uint64_t a, uint32_t size, uint32_t kind, xpl_host_site& s) {
-    if (kind != r->kind) return false;
-    if (a == r->end) {
-      if (a + size > r->cap) return false;
-      if (kind == XPL_ACC_RW && ((a | size) & 3u)) return false;
-      r->end = a + size;
-      if (r->owner == 0 || r->owner == s.id) own(r, s);
-      else r->owner = 0;
-      return true;
-    }
-    if (kind != XPL_ACC_RW && a >= r->beg && a + size <= r->end) {  // repeat (R or W)
-      r->grew = 1;
-      return true;
-    }
-    return false;
-  }
-  /* The slow path of a site access; the site takes over the run its access
-   * ended (a new run, or one extended there) unless another site owns it. */
-  __attribute__((noinline)) xpl_host_site site_access(uint64_t a, uint32_t size, uint32_t kind,
-                                                      xpl_host_site s) {
-    s.slot = slow(a, size, kind);
-    Run* r = &run_[s.slot];
-    if (r->kind && r->end == a + size && (r->owner == 0 || r->owner == s.id)) own(r, s);
-    return s;
-  }
   /* The access joins run r (extension at its end, or a repeat inside it). */
   static inline bool hit(Run* r, uint64_t a, uint32_t size, uint32_t kind) {
     if (kind != r->kind) return false;
@@ -204,7 +141,6 @@ class xpl_host_tracer {
       if (a + size > r->cap) return false;
       if (kind == XPL_ACC_RW && ((a | size) & 3u)) return false;
       r->end = a + size;  // (growth is seen at close: end != end0)
-      r->owner = 0;  // its owner's cached end is stale now
       return true;
     }
     if (kind != XPL_ACC_RW && a >= r->beg && a + size <= r->end) {  // repeat (R or W)
@@ -226,13 +162,11 @@ class xpl_host_tracer {
   static void set_limit(Run& r, uint64_t lim) {
     r.limit = lim;
     r.cap = lim < r.beg + kMaxRun ? lim : r.beg + kMaxRun;
-    r.owner = 0;  // its owner's cached cap is stale now
   }
   void close(int i) {
     if (n_ == kBuf) drain();
     buf_[n_++] = xpl_host_strided{run_[i].beg, (uint32_t)(run_[i].end - run_[i].beg), run_[i].kind, 0, 1};
     run_[i].kind = 0;
-    run_[i].owner = 0;
     const uint64_t b = wlo(run_[i].beg);
     for (int j = 0; j < kRuns; ++j) {
       if (run_[j].next == &run_[i]) run_[j].next = nullptr;  // forget predictions into the slot
@@ -274,14 +208,12 @@ class xpl_host_tracer {
         }
         if (a + size <= r.cap) {
           r.end = a + size;
-          r.owner = 0;
           churn_ = 0;
           touch(k);
           return i;
         }
       } else if (a == r.end && ((a | size) & 3u) == 0 && a + size <= r.cap) {
         r.end = a + size;
-        r.owner = 0;
         churn_ = 0;
         touch(k);
         return i;
@@ -332,7 +264,6 @@ class xpl_host_tracer {
     Run& r = run_[slot];
     r.beg = a;
     r.end = r.end0 = a + size;
-    r.owner = 0;
     r.kind = (uint16_t)kind;
     r.grew = 0;
     r.seq = ++seq_;
@@ -353,7 +284,6 @@ class xpl_host_tracer {
   Run* cur_ = &run_[0];                              // == &run_[mru_[0]]
   uint64_t seq_ = 0;
   uint32_t churn_ = 0;  // consecutive evictions of runs that never grew
-  uint32_t site_ids_ = 0;  // owner tokens handed out (wraps after 4G sites: ids are only compared)
   uint32_t tick_ = 0;
   size_t n_ = 0;
   xpl_status status_ = XPL_OK;

@@ -634,7 +634,7 @@ template <bool TAIL, bool RESET, bool BLOCKS>
 __device__ __forceinline__ void tile_loop(TileAcc& A, WarpRing& R, uint4* p4, uint32_t live,
                                           uint32_t lane, uint32_t min_run, uint64_t rw0, uint64_t B,
                                           uint32_t* blk, uint64_t kb0 = 0) {
-  const uint32_t n = TAIL ? (live + 511) / 512 : kDiagIters;  // steps holding row words
+  const uint32_t n = (live + 511) / 512;  // steps holding row words (live = the tile size unless TAIL)
   const uint32_t ns = (n + kStageSteps - 1) / kStageSteps;     // stages
   // bytes of stage j: whole 16-word vectors up to the row's end (the row's
   // shadow span is a multiple of 16 words, so they are all inside it)
@@ -666,7 +666,7 @@ __device__ __forceinline__ void tile_loop(TileAcc& A, WarpRing& R, uint4* p4, ui
   }
 }
 
-// One warp = one tile of kTileWords words of one row (no CTA-wide barrier: the
+// One warp = one tile of p.tile_words words of one row (no CTA-wide barrier: the
 // warps of a CTA are independent, so a warp on a cheap uniform stretch never
 // waits for one on a mixed stretch); per step lane l owns 16 words (one uint4
 // of records).  Counts: two Harley-Seal vertical counters (raw record bits;
@@ -695,16 +695,17 @@ __global__ void __launch_bounds__(kDiagThreads, XPL_DIAG_MINB) diag_tile_kernel(
   __syncwarp();
   const uint32_t ri = tile_row[t];
   const DiagRow row = rows[ri];
-  const uint64_t ww0 = (t - row.tile0) * kTileWords;  // row word
+  const uint32_t tw = p.tile_words;
+  const uint64_t ww0 = (t - row.tile0) * tw;  // row word
   const uint32_t min_run = (uint32_t)(p.min_run < 0xFFFFFFFFull ? p.min_run : 0xFFFFFFFFull);
-  const uint32_t live = (uint32_t)min(row.words - ww0, (uint64_t)kTileWords);
+  const uint32_t live = (uint32_t)min(row.words - ww0, (uint64_t)tw);
   uint4* p4 = reinterpret_cast<uint4*>(pool) + ((row.off + ww0) >> 4);
   uint32_t* blk = blk_cnt + row.blk0;
   TileAcc A;
   if (lane < 9) s_uc[warp][lane] = 0;
   __syncwarp();
   A.uc = s_uc[warp];
-  const bool tail = live < kTileWords;
+  const bool tail = live < tw;
   if (p.block_words) {  // rare: blocks need per-lane counter atomics (logical block index)
     const uint64_t kb0 = row.goff / p.block_words;
     if (p.reset) tile_loop<true, true, true>(A, R, p4, live, lane, min_run, row.goff + ww0, p.block_words, blk, kb0);

@@ -6,6 +6,7 @@
 // inlined hooks of xpl_device.cuh; this file only orders and launches them.
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <algorithm>
@@ -1044,11 +1045,23 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
   auto row_blocks = [&](const Row& r) -> uint64_t {  // logical blocks the row touches
     return B ? (r.goff + r.words - 1) / B - r.goff / B + 1 : 0;
   };
-  // geometry
+  // geometry: the tile size is halved (down to kMinTileWords) while the call
+  // would not fill every SM with several warps -- small diagnoses get more,
+  // shorter warps instead of a partial wave of long ones
+  uint64_t total_words = 0;
+  for (uint64_t id : ids) total_words += c->rows[id].words;
+  uint32_t tw = kTileWords;
+  while (tw > kMinTileWords && total_words / tw < 148ull * 24) tw >>= 1;
+  if (const char* e = getenv("XPL_DIAG_TILE_WORDS")) {  // test knob: force a tile size
+    const unsigned long v = strtoul(e, nullptr, 10);
+    if (v >= kMinTileWords && v <= kTileWords && (v & (v - 1)) == 0) tw = (uint32_t)v;
+  }
+  p.tile_words = tw;
+  p.pad = 0;
   uint64_t ntiles = 0, nblocks = 0, nseg = 0;
   for (uint64_t id : ids) {
     const Row& r = c->rows[id];
-    const uint64_t nt = (r.words + kTileWords - 1) / kTileWords;
+    const uint64_t nt = (r.words + tw - 1) / tw;
     ntiles += nt;
     nseg += (nt + kSegTiles - 1) / kSegTiles;
     nblocks += row_blocks(r);
@@ -1103,7 +1116,7 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
     d.off = r.off;
     d.words = r.words;
     d.tile0 = t;
-    d.ntiles = (r.words + kTileWords - 1) / kTileWords;
+    d.ntiles = (r.words + tw - 1) / tw;
     d.blk0 = b;
     d.nblk = row_blocks(r);
     d.goff = r.goff;
@@ -1126,8 +1139,6 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
   CK(cudaMemcpyAsync(c->d_tile_row, c->h_tile_row, sizeof(uint32_t) * ntiles,
                      cudaMemcpyHostToDevice, c->cs));
   CK(cudaMemcpyAsync(c->d_segs, c->h_segs, sizeof(StitchSeg) * nseg, cudaMemcpyHostToDevice, c->cs));
-  uint64_t total_words = 0;
-  for (size_t i = 0; i < nr; ++i) total_words += c->h_drows[i].words;
   const uint64_t dbytes = total_words * (reset ? 2 : 1);
   const int pall = prof_begin(c, XPL_K_DIAGNOSE, dbytes);
   const int ptile = prof_begin(c, XPL_K_DIAG_TILE, dbytes, false);  // recorded by launch_diag

@@ -41,8 +41,9 @@ struct RangeDesc {
 };
 
 // Diagnose geometry.
-constexpr uint32_t kTileWords = 16384;         // words per diagnose tile (one warp)
-constexpr uint32_t kDiagIters = 32;            // 512-word steps per tile (32 lanes x 16 words)
+constexpr uint32_t kTileWords = 16384;         // max words per diagnose tile (one warp)
+constexpr uint32_t kMinTileWords = 2048;       // min: small diagnoses use smaller tiles (more warps)
+constexpr uint32_t kDiagIters = kTileWords / 512;  // max 512-word steps per tile (32 lanes x 16 words)
 constexpr uint32_t kDiagThreads = 256;         // 8 independent warps (tiles) per CTA
 
 struct DiagRow {        // one row to analyse (live or dead-since-last-reset)
@@ -91,6 +92,8 @@ struct DiagParams {
   uint32_t reset;
   uint64_t block_words;
   uint64_t min_run;
+  uint32_t tile_words;  // this call's tile size (power of two in [kMinTileWords, kTileWords])
+  uint32_t pad;
 };
 
 // ---- launchers (kernels.cu) ----

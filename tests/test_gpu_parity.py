@@ -326,3 +326,14 @@ def test_uniform_stretches(gpu, seed):
     replay, _ = gpu
     ops = stretch_trace(0x58504C40 + seed)
     compare(replay.run_trace(ops, pool_words=1 << 22), oracle_run(ops), "stretches")
+
+
+@pytest.mark.parametrize("tile", ["2048", "4096", "16384"])
+def test_tile_size_invariance(gpu, tile, monkeypatch):
+    """The diagnose kernel's tile size (chosen per call from the call's size) must
+    not change any report: the stretch and multi-tile traces under a forced tile
+    size equal the oracle (which has no tiles)."""
+    replay, _ = gpu
+    monkeypatch.setenv("XPL_DIAG_TILE_WORDS", tile)
+    for ops in (stretch_trace(0x58504C50), big_trace(0x58504C51)):
+        compare(replay.run_trace(ops, pool_words=1 << 24), oracle_run(ops), f"tile={tile}")

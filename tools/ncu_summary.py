@@ -4,6 +4,7 @@ kernel, aggregated; shares of the step) and key metrics of `--set full` captures
 
   python tools/ncu_summary.py launches gpurun_out/launches.csv > profiles/rN_launches.txt
   python tools/ncu_summary.py full gpurun_out/prof.ncu-rep > profiles/rN_ncu_<kernel>.txt
+  python tools/ncu_summary.py traffic gpurun_out/traffic.csv   (-> profiles/traffic.json)
 """
 import collections
 import csv
@@ -63,5 +64,39 @@ def full(path):
                 print(f"{k:62s} {r[idx[k]]} {units[idx[k]]}")
 
 
+BYTES = {"byte": 1.0, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "KB": 1e3, "MB": 1e6, "GB": 1e9}
+
+
+def traffic(path, out_json="profiles/traffic.json"):
+    """Per-kernel DRAM traffic per launch (dram__bytes_read.sum + dram__bytes_write.sum,
+    averaged over every captured launch) from an ncu --metrics CSV log; merged into
+    profiles/traffic.json, which bench.py reports as roofline.traffic."""
+    import json
+    import os
+    rows = list(csv.reader(open(path)))
+    hdr, data = None, []
+    for r in rows:
+        if r and r[0] == "ID":
+            hdr = r
+            continue
+        if hdr and len(r) == len(hdr):
+            data.append(dict(zip(hdr, r)))
+    per = collections.defaultdict(dict)
+    for d in data:
+        if d["Metric Name"] in ("dram__bytes_read.sum", "dram__bytes_write.sum"):
+            v = float(d["Metric Value"].replace(",", "")) * BYTES.get(d["Metric Unit"], 1.0)
+            per[(d["Kernel Name"].split("(")[0], d["ID"])][d["Metric Name"]] = v
+    agg = collections.defaultdict(lambda: [0, 0.0])
+    for (k, _), m in per.items():
+        agg[k][0] += 1
+        agg[k][1] += sum(m.values())
+    cur = json.load(open(out_json)) if os.path.exists(out_json) else {}
+    for k, (n, b) in agg.items():
+        short = k.split("::")[-1].replace("_kernel", "")
+        cur[short] = {"bytes_per_launch": b / n, "launches": n, "source": os.path.basename(path)}
+        print(f"{short:24s} {n:6d} launches  {b / n:14.1f} B/launch")
+    json.dump(cur, open(out_json, "w"), indent=1, sort_keys=True)
+
+
 if __name__ == "__main__":
-    {"launches": launches, "full": full}[sys.argv[1]](sys.argv[2])
+    {"launches": launches, "full": full, "traffic": traffic}[sys.argv[1]](sys.argv[2])
