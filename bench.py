@@ -250,11 +250,14 @@ def diag_at_scale(xpl, torch, words=1 << 31, reps=3):
     return out
 
 
-def other_configs(xpl, apps, torch, lulesh_steps=100):
+def other_configs(xpl, apps, torch, lulesh_steps=100, lulesh250_steps=10):
     """The other BASELINE.json configs, each run once instrumented and once as the
     uninstrumented twin, device-timed: cfg1 SW-128 (one cooperative launch, 4
     epochs), cfg3 SW-16K (32,767 per-diagonal epochs, host traceback segments and
-    diagnoses every 1,024 diagonals), cfg4 LULESH-shaped 100^3 x 100 timesteps."""
+    diagnoses every 1,024 diagonals), cfg4 LULESH-shaped 100^3 x 100 timesteps,
+    cfg5 LULESH-shaped 250^3 (1.47e9 + 0.84e9 shadow words per timestep) on one
+    GPU for 10 timesteps (the 100-timestep run is 10x this; its shadow fits one
+    B200)."""
     from xplgen import lulesh as L
     from xplgen import sw
     out = {}
@@ -274,8 +277,9 @@ def other_configs(xpl, apps, torch, lulesh_steps=100):
         return e0.elapsed_time(e1), run
 
     for name, (n, m, per_diag, tb, dg, pool) in {
-            "cfg1_sw128": (128, 128, False, 0, 0, 1 << 20),
-            "cfg3_sw16k": (16384, 16384, True, 1024, 1024, 1 << 29)}.items():
+            "cfg1_sw128": (128, 128, 0, 0, 0, 1 << 20),
+            "cfg1_sw128_split": (128, 128, 2, 0, 0, 1 << 20),
+            "cfg3_sw16k": (16384, 16384, 1, 1024, 1024, 1 << 29)}.items():
         spec = sw.sw_spec(n, m)
         ar = apps.Arena(spec)
         inp = sw.sw_inputs(n, m, 0x58504C04)
@@ -291,36 +295,41 @@ def other_configs(xpl, apps, torch, lulesh_steps=100):
                                                             run.r.epochs, run.r.n_diag)
         acc = res["instr"][1]
         out[name] = {"workload": f"Smith-Waterman {n}x{m}, managed, "
-                                 f"{'per-diagonal launches' if per_diag else 'one cooperative launch'}",
+                                 + ["one launch", "per-diagonal launches",
+                                    "one cooperative launch, device-side epoch split per diagonal"][per_diag],
                      "ms": res["instr"][0], "accesses": acc, "accesses_per_s": acc / (res["instr"][0] / 1e3),
                      "epochs": res["instr"][2], "diagnoses": res["instr"][3], "twin_ms": res["twin"][0],
                      "slowdown": res["instr"][0] / res["twin"][0]}
         del ar
-    s_edge = 100
-    spec = L.lulesh_spec(s_edge)
-    ar = apps.Arena(spec)
-    topo = L.topology(s_edge, 0x58504C05)
-    hc = torch.zeros(1, dtype=torch.int64, device="cuda")
-    res = {}
-    with xpl.Context(pool_words=1 << 28, max_rows=64) as ctx:
-        for c in (ctx, None):
-            apps.lulesh_prepare(ar, s_edge, topo)
-            hc.zero_()
+    for name, s_edge, steps, pool in (("cfg4_lulesh100", 100, lulesh_steps, 1 << 28),
+                                      ("cfg5_lulesh250", 250, lulesh250_steps, 2_500_000_000)):
+        if not steps:
+            continue
+        spec = L.lulesh_spec(s_edge)
+        ar = apps.Arena(spec)
+        topo = L.topology(s_edge, 0x58504C05)
+        hc = torch.zeros(1, dtype=torch.int64, device="cuda")
+        res = {}
+        with xpl.Context(pool_words=pool, max_rows=64) as ctx:
+            for c in (ctx, None):
+                apps.lulesh_prepare(ar, s_edge, topo)
+                hc.zero_()
 
-            def fn(c):
-                run = apps.Run(c, us.cuda_stream, params=PARAMS, out_cap=64 * (lulesh_steps + 1))
-                apps.lulesh(run, ar, s_edge, lulesh_steps, hc)
-                return run
-            ms, run = timed_run(c, fn)
-            res["instr" if c is not None else "twin"] = (ms, int(hc.item()) + run.r.host_accesses,
-                                                        run.r.epochs, run.r.n_diag, run.r.host_ms)
-    acc = res["instr"][1]
-    out["cfg4_lulesh100"] = {"workload": f"LULESH-shaped {s_edge}^3 x {lulesh_steps} timesteps, 50 managed "
-                                         "allocations + 2 temporaries/step, 19 launches/step",
-                             "ms": res["instr"][0], "accesses": acc,
-                             "accesses_per_s": acc / (res["instr"][0] / 1e3), "epochs": res["instr"][2],
-                             "diagnoses": res["instr"][3], "host_ms": res["instr"][4],
-                             "twin_ms": res["twin"][0], "slowdown": res["instr"][0] / res["twin"][0]}
+                def fn(c):
+                    run = apps.Run(c, us.cuda_stream, params=PARAMS, out_cap=64 * (steps + 1))
+                    apps.lulesh(run, ar, s_edge, steps, hc)
+                    return run
+                ms, run = timed_run(c, fn)
+                res["instr" if c is not None else "twin"] = (ms, int(hc.item()) + run.r.host_accesses,
+                                                            run.r.epochs, run.r.n_diag, run.r.host_ms)
+        del ar, topo
+        acc = res["instr"][1]
+        out[name] = {"workload": f"LULESH-shaped {s_edge}^3 x {steps} timesteps, 50 managed "
+                                 "allocations + 2 temporaries/step, 19 launches/step",
+                     "ms": res["instr"][0], "accesses": acc,
+                     "accesses_per_s": acc / (res["instr"][0] / 1e3), "epochs": res["instr"][2],
+                     "diagnoses": res["instr"][3], "host_ms": res["instr"][4],
+                     "twin_ms": res["twin"][0], "slowdown": res["instr"][0] / res["twin"][0]}
     return out
 
 

@@ -52,9 +52,12 @@ struct xpl_dev_ctx {
   unsigned int* pool;             /* shadow pool, 4 records per u32              */
   unsigned char* cmap;            /* 1 byte per 128-word chunk: GPU write pending */
   unsigned char* smap;            /* 1 byte per 128 chunks (16K words)            */
+  const unsigned long long* n_super; /* super-chunks below the pool's high-water mark */
 };
 
 #ifdef __CUDACC__
+
+#include <cooperative_groups.h>
 
 /* Translation-unit-local copy of the device context (set by xpl_device_bind). */
 static __constant__ xpl_dev_ctx xpl_dctx;
@@ -280,6 +283,49 @@ template <class T>
 static __device__ __forceinline__ T& xpl_rw(T& x) {
   xpl_dev_record_k<XPL_ACC_RW>(&x, sizeof(T), XPL_ACC_RW);
   return x;
+}
+
+/* Device-side epoch boundary (the paper's per-iteration
+ * view of a wavefront, Fig. 8).  Inside ONE cooperative launch
+ * (cudaLaunchCooperativeKernel), every thread of the grid calls it at the same
+ * point: it closes the epoch the kernel's accesses so far belong to and opens a
+ * new one, exactly like xpl_kernel_end + xpl_kernel_begin between two launches
+ * (trace: KE KB).  Steps: grid barrier (all hooks of the segment have landed),
+ * the fold of that segment's pending writes (P -> L, D5) spread over the warps
+ * of the grid, grid barrier (reads of the next segment see the new L).  The
+ * barrier's release/acquire at gpu scope orders the plain shadow loads of the
+ * hooks after the fold.  Must not be called from a non-cooperative launch (the
+ * grid barrier would deadlock or fault); a no-op under -DXPL_OFF except for the
+ * barrier itself, which keeps the twin's control flow. */
+static __device__ __forceinline__ void xpl_grid_epoch() {
+  cooperative_groups::grid_group g = cooperative_groups::this_grid();
+  g.sync();
+#ifndef XPL_OFF
+  const unsigned lane = xpld_lane();
+  const unsigned long long nthreads = (unsigned long long)gridDim.x * gridDim.y * gridDim.z *
+                                      blockDim.x * blockDim.y * blockDim.z;
+  const unsigned long long nwarps = (nthreads + 31) / 32;
+  const unsigned long long gw = g.thread_rank() / 32;
+  const unsigned long long n_super = __ldcg(xpl_dctx.n_super);
+  for (unsigned long long sc = gw; sc < n_super; sc += nwarps) {
+    if (!__ldcg(xpl_dctx.smap + sc)) continue; /* (uniform over the warp) */
+    for (unsigned c0 = 0; c0 < 128; c0 += 32) {
+      const unsigned long long ch = sc * 128 + c0 + lane;
+      const bool m = __ldcg(xpl_dctx.cmap + ch) != 0;
+      unsigned marked = __ballot_sync(0xFFFFFFFFu, m);
+      while (marked) {
+        const unsigned j = __ffs(marked) - 1;
+        marked &= marked - 1;
+        unsigned* w = xpl_dctx.pool + (sc * 128 + c0 + j) * 32 + lane;
+        const unsigned v = __ldcg(w);
+        if (v & XPLD_P4) *w = (v & ~XPLD_P4) | ((v & XPLD_P4) >> 1); /* P -> L */
+      }
+      if (m) xpl_dctx.cmap[ch] = 0;
+    }
+    if (lane == 0) xpl_dctx.smap[sc] = 0;
+  }
+  g.sync();
+#endif
 }
 
 #endif /* __CUDACC__ */

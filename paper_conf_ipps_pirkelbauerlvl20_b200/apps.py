@@ -26,7 +26,8 @@ class XplwRun(C.Structure):
                 ("params", XplDiagParams), ("out", vp), ("out_cap", sz), ("n_out", sz),
                 ("diag_rows", vp), ("diag_cap", sz), ("n_diag", sz), ("dev_accesses", u64),
                 ("host_accesses", u64), ("copy_words", u64), ("epochs", u64), ("status", i32),
-                ("time_kernels", i32), ("kernel_ms", C.c_double), ("host_ms", C.c_double)]
+                ("time_kernels", i32), ("kernel_ms", C.c_double), ("host_ms", C.c_double),
+                ("diag_no_reset", i32), ("keep_allocs", i32)]
 
 
 _w = xpl._work
@@ -107,8 +108,10 @@ class Run:
     """One xplw_run: the context (or None = uninstrumented twin) and outputs."""
 
     def __init__(self, ctx, stream, do_copies=False, diag_each=True, params=(50, 0, 256), out_cap=4096,
-                 time_kernels=False):
+                 time_kernels=False, diag_reset=True, keep_allocs=False):
         self.r = XplwRun()
+        self.r.diag_no_reset = int(not diag_reset)
+        self.r.keep_allocs = int(keep_allocs)
         self.r.time_kernels = int(time_kernels)
         self.r.ctx = ctx.h if ctx is not None else None
         self.r.stream = stream

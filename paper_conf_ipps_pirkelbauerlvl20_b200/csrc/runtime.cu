@@ -449,6 +449,8 @@ xpl_status upload_table(xpl_ctx* c) {
     ++n;
   }
   memcpy(c->h_tab, &n, sizeof n);
+  const unsigned long long n_super = (c->pa.hwm + 16383) / 16384;  // for xpl_grid_epoch
+  memcpy(c->h_tab + 8, &n_super, sizeof n_super);
   CK(cudaMemcpyAsync(c->d_tab, c->h_tab, 32 + sizeof(xpl_dev_row) * n, cudaMemcpyHostToDevice, c->cs));
   CK(cudaEventRecord(c->table_ev, c->cs));
   c->table_dirty = false;
@@ -951,6 +953,7 @@ xpl_status xpl_get_device_ctx(xpl_ctx* c, struct xpl_dev_ctx* d) {
   d->pool = (unsigned int*)c->d_pool;
   d->cmap = c->d_cmap;
   d->smap = c->d_smap;
+  d->n_super = (const unsigned long long*)(c->d_tab + 8);
   return XPL_OK;
 }
 

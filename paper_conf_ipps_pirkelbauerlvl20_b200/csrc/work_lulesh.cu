@@ -417,7 +417,7 @@ int xplw_lulesh(xplw_run* run, const xplw_arrays* arr, int s, int steps, unsigne
     size_t nr = 0;
     xpl_alloc_report* o = run->out ? run->out + run->n_out : nullptr;
     const size_t cap = run->out ? run->out_cap - run->n_out : 0;
-    const int x = xpl_diagnose(run->ctx, &run->params, nullptr, 0, o, cap, &nr, 1);
+    const int x = xpl_diagnose(run->ctx, &run->params, nullptr, 0, o, cap, &nr, run->diag_no_reset ? 0 : 1);
     if (x == XPL_OK) {
       run->n_out += nr;
       if (run->diag_rows && run->n_diag < run->diag_cap) run->diag_rows[run->n_diag] = (uint32_t)nr;
@@ -551,6 +551,11 @@ int xplw_lulesh(xplw_run* run, const xplw_arrays* arr, int s, int steps, unsigne
   flush();
   delete tr;
   tr = nullptr;
+  if (run->keep_allocs) {
+    if (on) ok(xpl_sync(run->ctx));
+    okc(cudaStreamSynchronize(st));
+    return run->status;
+  }
   if (on)
     for (int k = 0; k < arr->n; ++k) ok(xpl_free(run->ctx, (const void*)arr->addr[k]));
   diag();

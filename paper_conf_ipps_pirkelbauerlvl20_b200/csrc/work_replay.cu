@@ -19,6 +19,21 @@ __global__ void replay_kernel(const unsigned long long* __restrict__ addr,
     xpl_dev_record((const void*)addr[i], size[i], acc[i]);
 }
 
+// The same replay as ONE cooperative launch over several epochs: segment k is
+// events [seg[k], seg[k+1]); a device-side epoch split (xpl_grid_epoch,
+// NEXT-2) separates consecutive segments.  Equal to one launch per segment.
+__global__ void replay_split_kernel(const unsigned long long* __restrict__ addr,
+                                    const unsigned int* __restrict__ size,
+                                    const unsigned char* __restrict__ acc,
+                                    const unsigned long long* __restrict__ seg, int nseg) {
+  for (int k = 0; k < nseg; ++k) {
+    if (k) xpl_grid_epoch();
+    for (unsigned long long i = seg[k] + (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x;
+         i < seg[k + 1]; i += (unsigned long long)gridDim.x * blockDim.x)
+      xpl_dev_record((const void*)addr[i], size[i], acc[i]);
+  }
+}
+
 __device__ __forceinline__ unsigned hash32(unsigned x) {
   x ^= x >> 16;
   x *= 0x7feb352du;
@@ -87,5 +102,23 @@ int xplw_replay(const unsigned long long* d_addr, const unsigned int* d_size,
   if (n == 0) return 0;
   replay_kernel<<<grid, block, 0, (cudaStream_t)stream>>>(d_addr, d_size, d_acc, n);
   return cudaGetLastError() == cudaSuccess ? 0 : (int)XPL_ERR_CUDA;
+}
+
+// One cooperative launch replaying nseg epochs (between one xpl_kernel_begin/_end);
+// d_seg: nseg+1 event offsets (device).  grid is capped at the co-resident limit.
+int xplw_replay_split(const unsigned long long* d_addr, const unsigned int* d_size,
+                      const unsigned char* d_acc, const unsigned long long* d_seg, int nseg,
+                      int grid, int block, void* stream) {
+  if (nseg <= 0) return 0;
+  int dev = 0, sms = 0, per_sm = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, replay_split_kernel, block, 0);
+  const int cap = sms * per_sm;
+  if (grid <= 0 || grid > cap) grid = cap;
+  void* args[] = {&d_addr, &d_size, &d_acc, &d_seg, &nseg};
+  const cudaError_t e = cudaLaunchCooperativeKernel((const void*)replay_split_kernel, dim3(grid), dim3(block),
+                                                    args, 0, (cudaStream_t)stream);
+  return e == cudaSuccess ? 0 : (int)XPL_ERR_CUDA;
 }
 }

@@ -49,6 +49,24 @@ __global__ void sw_wavefront(const int* a, const int* b, int* H, int n, int m) {
   }
 }
 
+// cfg1 with device-side epoch splits (NEXT-2): the same single launch, but each
+// anti-diagonal is its own epoch (xpl_grid_epoch; launched cooperatively), so
+// the wavefront's reads of the previous diagonal see the GPU as the last writer
+// -- the paper's per-iteration view (Fig. 8).
+template <bool I>
+__global__ void sw_wavefront_split(const int* a, const int* b, int* H, int n, int m) {
+  const int ld = m + 1, i = threadIdx.x + 1;
+  for (int d = 2; d <= n + m; ++d) {
+    const int j = d - i;
+    if (i <= n && j >= 1 && j <= m) sw_cell<I>(a, b, H, ld, i, j);
+    if constexpr (I) {
+      if (d < n + m) xpl_grid_epoch();  // (the last diagonal's epoch closes at xpl_kernel_end)
+    } else {
+      __syncthreads();
+    }
+  }
+}
+
 // cfg3: one launch per anti-diagonal d, thread per cell.
 template <bool I>
 __global__ void __launch_bounds__(256) sw_diagonal(const int* a, const int* b, int* H, int n, int m,
@@ -139,7 +157,17 @@ int xplw_sw(xplw_run* run, const xplw_arrays* arr, int n, int m, int per_diagona
   run->host_accesses += n + m + hn;
   host_ms(t0);
   // the GPU fills H
-  if (!per_diagonal) {
+  if (per_diagonal == 2) {  // one cooperative launch, one epoch per anti-diagonal
+    begin();
+    if (on) {
+      void* args[] = {&a, &b, &H, &n, &m};
+      okc(cudaLaunchCooperativeKernel((const void*)sw_wavefront_split<true>, dim3(1), dim3(n), args, 0, s));
+    } else {
+      sw_wavefront_split<false><<<1, n, 0, s>>>(a, b, H, n, m);
+    }
+    end();
+    run->dev_accesses += 6ull * n * m;
+  } else if (!per_diagonal) {
     begin();
     if (on) sw_wavefront<true><<<1, n, 0, s>>>(a, b, H, n, m);
     else sw_wavefront<false><<<1, n, 0, s>>>(a, b, H, n, m);
@@ -200,7 +228,7 @@ int xplw_sw(xplw_run* run, const xplw_arrays* arr, int n, int m, int per_diagona
   }
   *tb_len = len;
   host_ms(t0);
-  if (!per_diagonal) {  // E3: the GPU re-zeroes the interior for the next query
+  if (per_diagonal != 1) {  // E3: the GPU re-zeroes the interior for the next query
     begin();
     if (on) sw_rezero<true><<<(n * m + 255) / 256, 256, 0, s>>>(H, n, m);
     else sw_rezero<false><<<(n * m + 255) / 256, 256, 0, s>>>(H, n, m);

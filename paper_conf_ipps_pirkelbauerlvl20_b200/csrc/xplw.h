@@ -47,6 +47,9 @@ typedef struct {
   int time_kernels;       /* 1 = time the app's kernels with CUDA events          */
   double kernel_ms;       /* sum of the app's kernel times (time_kernels)         */
   double host_ms;         /* host wall time spent in traced host loops + tracer   */
+  int diag_no_reset;      /* 1 = diagnoses keep the interval bits (D25)            */
+  int keep_allocs;        /* 1 = leave the arrays registered at the end (no final  *
+                           *     frees + diagnose), for shadow dumps (LULESH)      */
 } xplw_run;
 
 /* Rodinia hotspot: rows x cols temperatures, `iters` 5-point stencil steps.

@@ -22,12 +22,60 @@ def _host_array(items):
     return a
 
 
+def _group_splits(ops):
+    """Fold every maximal chain of >= 2 consecutive top-level epochs
+    (KB dev* KE KB dev* KE ...) into one ("SPLIT", [segments]) op: one cooperative
+    launch with a device-side epoch split between segments (NEXT-2)."""
+    out, i, depth = [], 0, 0
+    while i < len(ops):
+        if ops[i][0] == "KB" and depth == 0:
+            segs, j = [], i
+            while j < len(ops) and ops[j][0] == "KB":
+                k = j + 1
+                while k < len(ops) and ops[k][0] in ("D", "DB"):
+                    k += 1
+                if k >= len(ops) or ops[k][0] != "KE":
+                    break
+                segs.append(ops[j + 1:k])
+                j = k + 1
+            if len(segs) >= 2:
+                out.append(("SPLIT", segs))
+                i = j
+                continue
+        if ops[i][0] == "KB":
+            depth += 1
+        elif ops[i][0] == "KE":
+            depth -= 1
+        out.append(ops[i])
+        i += 1
+    return out
+
+
+def _dev_arrays(evs):
+    a, s, k = [], [], []
+    for op in evs:
+        if op[0] == "D":
+            a.append(np.array([op[1]], np.uint64)), s.append(np.array([op[2]], np.uint32))
+            k.append(np.array([op[3]], np.uint8))
+        else:
+            a.append(np.asarray(op[1], np.uint64)), s.append(np.asarray(op[2], np.uint32))
+            k.append(np.asarray(op[3], np.uint8))
+    if not a:
+        return np.zeros(0, np.uint64), np.zeros(0, np.uint32), np.zeros(0, np.uint8)
+    return np.concatenate(a), np.concatenate(s), np.concatenate(k)
+
+
 def run_trace(ops, ctx: Context | None = None, grid=0, block=256, seed=None, host_split=None,
-              pool_words=1 << 24, stream=None):
+              pool_words=1 << 24, stream=None, split_epochs=False):
     """Replay `ops`.  seed: shuffle device events inside every epoch and split
     host batches at random points (metamorphic variants); grid/block: launch
-    shape of the replay kernel (grid 0 = enough CTAs for one event each)."""
+    shape of the replay kernel (grid 0 = enough CTAs for one event each);
+    split_epochs: chains of consecutive epochs run as one cooperative launch
+    with device-side epoch splits (xpl_grid_epoch) -- must give the same reports."""
     import torch
+
+    if split_epochs:
+        ops = _group_splits(ops)
 
     rng = np.random.default_rng(seed) if seed is not None else None
     own = ctx is None
@@ -90,6 +138,25 @@ def run_trace(ops, ctx: Context | None = None, grid=0, block=256, seed=None, hos
             dev.append((np.array([op[1]], np.uint64), np.array([op[2]], np.uint32), np.array([op[3]], np.uint8)))
         elif t == "DB":
             dev.append((np.asarray(op[1], np.uint64), np.asarray(op[2], np.uint32), np.asarray(op[3], np.uint8)))
+        elif t == "SPLIT":
+            flush_dev()
+            parts = [_dev_arrays(seg) for seg in op[1]]
+            if rng is not None:
+                parts = [tuple(x[p] for x in pt) for pt in parts for p in [rng.permutation(pt[0].size)]]
+            off = np.zeros(len(parts) + 1, np.uint64)
+            off[1:] = np.cumsum([pt[0].size for pt in parts])
+            a = np.concatenate([pt[0] for pt in parts])
+            sz = np.concatenate([pt[1] for pt in parts])
+            kk = np.concatenate([pt[2] for pt in parts])
+            ta = torch.from_numpy(a.view(np.int64)).cuda()
+            ts = torch.from_numpy(sz.view(np.int32)).cuda()
+            tk = torch.from_numpy(kk).cuda()
+            to = torch.from_numpy(off.view(np.int64)).cuda()
+            ctx.kernel_begin(stream)
+            ctx.replay_split(ta.data_ptr(), ts.data_ptr(), tk.data_ptr(), to.data_ptr(), len(parts),
+                             grid=grid, block=block, stream=stream)
+            ctx.kernel_end(stream)
+            torch.cuda.current_stream().synchronize()
         elif t == "X":
             flush_dev()
             ctx.record_copy(op[2], op[3], op[4], op[1])

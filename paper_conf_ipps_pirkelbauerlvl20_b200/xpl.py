@@ -136,6 +136,7 @@ EXPORTED = ["xpl_init", "xpl_finalize", "xpl_register_alloc", "xpl_free", "xpl_k
 if _work is not None:
     xplw_bind = _sig("xplw_bind", [vp], lib=_work)
     xplw_replay = _sig("xplw_replay", [vp, vp, vp, u64, i32, i32, vp], lib=_work)
+    xplw_replay_split = _sig("xplw_replay_split", [vp, vp, vp, vp, i32, i32, i32, vp], lib=_work)
     xplw_touch = _sig("xplw_touch", [u64, u64, u32, vp, u64], lib=_work)
 
 
@@ -291,6 +292,11 @@ class Context:
         if grid <= 0:
             grid = max(1, min((n + block - 1) // block, 148 * 8))
         check("xplw_replay", xplw_replay(d_addr, d_size, d_acc, n, grid, block, stream))
+
+    def replay_split(self, d_addr, d_size, d_acc, d_seg, nseg, grid=0, block=256, stream=0):
+        """One cooperative launch of the replay kernel over nseg epochs separated by
+        device-side epoch splits (xpl_grid_epoch); d_seg = nseg+1 event offsets."""
+        check("xplw_replay_split", xplw_replay_split(d_addr, d_size, d_acc, d_seg, nseg, grid, block, stream))
 
 
 def combine_partials(blobs, thr=50, block_words=0, min_run=256):

@@ -8,7 +8,7 @@ import numpy as np
 import pytest
 
 from oracle import run_trace as oracle_run
-from xplgen.trace import (DEVICE, MANAGED, RW, SEG_OPS, R, W, enumerated_trace, parse_text, random_trace,
+from xplgen.trace import (epoch_chain_trace, DEVICE, MANAGED, RW, SEG_OPS, R, W, enumerated_trace, parse_text, random_trace,
                           schedules)
 
 pytestmark = pytest.mark.gpu
@@ -337,3 +337,23 @@ def test_tile_size_invariance(gpu, tile, monkeypatch):
     monkeypatch.setenv("XPL_DIAG_TILE_WORDS", tile)
     for ops in (stretch_trace(0x58504C50), big_trace(0x58504C51)):
         compare(replay.run_trace(ops, pool_words=1 << 24), oracle_run(ops), f"tile={tile}")
+
+
+@pytest.mark.parametrize("seed", range(6))
+@pytest.mark.parametrize("grid,block", [(1, 128), (0, 256), (3, 96)])
+def test_device_epoch_split(gpu, seed, grid, block):
+    """NEXT-2: chains of epochs replayed as ONE cooperative launch with a
+    device-side epoch split (xpl_grid_epoch) between them give the oracle's
+    reports (= one launch per epoch), for one CTA, the full co-resident grid
+    and odd shapes, with the events of each segment shuffled."""
+    replay, _ = gpu
+    ops = epoch_chain_trace(0x58504C20 + seed)
+    exp = oracle_run(ops)
+    assert replay.run_trace(ops, grid=grid, block=block, seed=seed, split_epochs=True) == exp
+
+
+def test_device_epoch_split_random_traces(gpu):
+    replay, _ = gpu
+    for seed in range(4):
+        ops = random_trace(0x58504C30 + seed, n_allocs=5, n_steps=80, max_words=4000, p_device=0.9)
+        assert replay.run_trace(ops, split_epochs=True) == oracle_run(ops)

@@ -111,9 +111,11 @@ def test_nw(env, n, resident):
 
 
 @pytest.mark.parametrize("n,m,per_diag,tb_every,diag_every", [
-    (128, 128, False, 0, 0),      # cfg1 SW-128: one cooperative launch, 4 epochs
-    (40, 70, True, 16, 32),       # cfg3 shape: per-diagonal launches, traceback + diagnose points
-    (300, 257, True, 64, 128)])
+    (128, 128, 0, 0, 0),          # cfg1 SW-128: one launch, 4 epochs
+    (128, 128, 2, 0, 0),          # cfg1 with a device-side epoch split per anti-diagonal (NEXT-2)
+    (37, 90, 2, 0, 0),
+    (40, 70, 1, 16, 32),       # cfg3 shape: per-diagonal launches, traceback + diagnose points
+    (300, 257, 1, 64, 128)])
 def test_smith_waterman(env, n, m, per_diag, tb_every, diag_every):
     torch, apps, xpl = env
     from xplgen import sw
@@ -129,9 +131,14 @@ def test_smith_waterman(env, n, m, per_diag, tb_every, diag_every):
         assert run.r.dev_accesses == sw.sw_accesses(n, m, per_diag)
     H = sw.sw_dp(inp["a"], inp["b"])
     assert tb == sw.sw_traceback(H, inp["a"], inp["b"])[3]
-    if per_diag:  # (the single-launch program re-zeroes H at the end)
+    if per_diag == 1:  # (the single-launch programs re-zero H at the end)
         assert np.array_equal(ar.view("H").view(np.int32).reshape(n + 1, m + 1), H)
     compare(got, oracle_run(sw.sw_trace(ar.addrs, spec, n, m, per_diag, tb_every, diag_every, inp, params)))
+    if per_diag == 2:
+        # split epochs: the wavefront reads its own earlier diagonals as G>G; only
+        # the CPU's boundary zeros (row 0 and column 0) are C>G (Fig. 7)
+        h = got[-1][2]
+        assert h["w_g"] == n * m and h["r_cg"] == n + m + 1 and h["r_gg"] > 0
     if not per_diag:
         # cfg1 under the snapshot reading (D5): one launch sees only the pre-epoch
         # (CPU) values, so no read of H is G>G although the wavefront reads its own output

@@ -49,3 +49,35 @@ def test_sampled_three_segments(schedule):
 @pytest.mark.parametrize("seed", range(40))
 def test_random_traces(seed):
     compare(random_trace(0x58504C00 + seed, n_allocs=5, n_steps=50, max_words=64))
+
+
+def test_lulesh_sampled_twin_equals_full_twin():
+    """The sampled LULESH twin (cfg5 full-size parity: only the events of chosen
+    word windows, repeats inside an epoch dropped, temporaries left out) leaves
+    every sampled word -- and every word of dom and dt_block, whose rows it
+    reproduces exactly -- with the record the full trace gives."""
+    from oracle import Oracle
+    from xplgen import lulesh as L
+    from xplgen.rodinia import layout
+    s = 5
+    spec = L.lulesh_spec(s)
+    addrs, _, _ = layout(spec, 1 << 40, 1 << 44, 1 << 36)
+    topo = L.topology(s, 0x58504C05)
+    tmps = [((1 << 50) + (2 * i << 30), (1 << 50) + ((2 * i + 1) << 30)) for i in range(3)]
+    win = {k: [(0, 7), (31, 45), (L.slot_bytes(s, k) // 4 - 5, L.slot_bytes(s, k) // 4)] for k in range(0, 48, 2)}
+    full, _ = L.lulesh_trace(addrs, spec, s, 3, topo, (50, 0, 256), tmps, reset=0, final=False)
+    samp, hooks = L.lulesh_trace(addrs, spec, s, 3, topo, (50, 0, 256), tmps, windows=win, reset=0, final=False)
+    assert hooks is None
+    assert sum(len(op[1]) for op in samp if op[0] in ("DB", "HB")) < \
+        sum(len(op[1]) for op in full if op[0] in ("DB", "HB")) // 5
+    o1, o2 = Oracle(), Oracle()
+    d1 = [r for r in map(o1.op, full) if r is not None]
+    d2 = [r for r in map(o2.op, samp) if r is not None]
+    for a, b in zip(d1, d2):
+        assert a[0] == b[0] and a[1] == b[1]  # dom, dt_block: complete rows
+    for k, ws in win.items():
+        for w0, w1 in ws:
+            for w in range(w0, w1):
+                assert o1.peek(2 + k, w) == o2.peek(2 + k, w), (k, w)
+    for w in range(L.DOM_BYTES // 4):
+        assert o1.peek(0, w) == o2.peek(0, w)

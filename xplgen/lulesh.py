@@ -92,16 +92,50 @@ class _Ev:
         return (t, np.concatenate(self.a), np.concatenate(self.s), np.concatenate(self.k))
 
 
-def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs):
+def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs, windows=None, reset=1, final=True):
     """The CPU twin of xplw_lulesh: returns (ops, device hook calls).
     tmp_addrs[step] = (force temporary, gradient temporary) base addresses, as
-    the program's cudaMallocManaged returned them."""
+    the program's cudaMallocManaged returned them.
+
+    Sampled form (the cfg5 full-size parity, where the whole trace does not fit):
+    windows = {k: [(w0, w1), ...]} word windows of array slot k (0..47); then
+    only the events of those words are emitted, plus every event of `dom` and
+    `dt_block` -- a word's record depends only on the events that touch it --
+    and events of one address repeated inside one GPU epoch are emitted once
+    (their multiplicity does not matter, D5/D21).  The temporaries are left out
+    (their REG/FREE stay, so ids match); hooks is then None.  reset: the
+    diagnoses' reset flag; final=False: no final frees + diagnose (the
+    program's keep_allocs)."""
     ne, nn, nsym, nblk = sizes(s)
     dom, dtb = addrs[0], addrs[1]
     A = [addrs[2 + k] for k in range(48)]
     u = lambda x: np.asarray(x, dtype=np.uint64)
     ops = [("REG", a, sp[1], sp[2]) for a, sp in zip(addrs, spec)]
-    hooks = 0
+    hooks = 0 if windows is None else None
+    sampled = windows is not None
+    if sampled:
+        tab = {}
+        for k in range(48):
+            es = 8 if k <= QQ else 4
+            t = np.zeros(slot_bytes(s, k) // es, bool)
+            for w0, w1 in windows.get(k, ()):
+                t[(4 * w0) // es:-(-(4 * w1) // es)] = True
+            tab[k] = t
+
+    def D(k, idx):  # a double of slot k
+        idx = np.asarray(idx).reshape(-1)
+        return A[k] + 8 * u(idx[tab[k][idx]] if sampled else idx)
+
+    def I4(k, idx):  # an int of slot k
+        idx = np.asarray(idx).reshape(-1)
+        return A[k] + 4 * u(idx[tab[k][idx]] if sampled else idx)
+
+    def rep(addr, n):  # one address read by n threads of a kernel
+        return addr * np.ones(min(n, 1) if sampled else n, np.uint64)
+
+    def TMP(fn):  # events of a temporary (not sampled)
+        return np.zeros(0, np.uint64) if sampled else fn()
+
     # ---- host initialisation ----
     h = _Ev()
     h.add(dom + 8 * u(np.arange(NSLOT)), 8, W)
@@ -113,13 +147,13 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs):
     for k in range(48):
         nb = slot_bytes(s, k)
         if k <= QQ:
-            h.add(A[k] + 8 * u(np.arange(nb // 8)), 8, W)
+            h.add(D(k, np.arange(nb // 8)), 8, W)
         else:  # int arrays, and the never-used ones zero-filled as 4-byte words
-            h.add(A[k] + 4 * u(np.arange(nb // 4)), 4, W)
+            h.add(I4(k, np.arange(nb // 4)), 4, W)
     h.add(dtb + 8 * u(np.arange(2 * nblk)), 8, W)
     ops.append(h.op("HB"))
 
-    ptr = lambda k, n: (dom + 8 * k) * np.ones(n, np.uint64)
+    ptr = lambda k, n: rep(dom + 8 * k, n)
     e = np.arange(ne)
     nidx = np.arange(nn)
     nl = topo[NODELIST].reshape(ne, 8).astype(np.int64)
@@ -130,9 +164,7 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs):
     grid_e = nblk * 256
     grid_n = (nn + 255) // 256 * 256
     grid_s = (nsym + 255) // 256 * 256
-    numelem = lambda g: (dom + OFF_NUMELEM) * np.ones(g, np.uint64)
-    D = lambda k, idx: A[k] + 8 * u(idx)   # a double of slot k
-    I4 = lambda k, idx: A[k] + 4 * u(idx)  # an int of slot k
+    numelem = lambda g: rep(dom + OFF_NUMELEM, g)
 
     for step in range(steps):
         tf, tg = tmp_addrs[step]
@@ -157,7 +189,7 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs):
         ev.add(I4(NODELIST, 8 * e[:, None] + np.arange(8)), 4, R)
         for k in (X, Y, Z):
             ev.add(D(k, nl), 8, R)
-        ev.add(tf + 8 * u(np.arange(24 * ne)), 8, W)
+        ev.add(TMP(lambda: tf + 8 * u(np.arange(24 * ne))), 8, W)
         kernels.append(ev)
         # 3 hourglass
         ev = _Ev()
@@ -171,7 +203,7 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs):
         ev.add(I4(NODELIST, 8 * e[:, None] + np.arange(8)), 4, R)
         for k in (XD, YD, ZD):
             ev.add(D(k, nl), 8, R)
-        ev.add(tf + 8 * u(np.arange(24 * ne)), 8, RW)
+        ev.add(TMP(lambda: tf + 8 * u(np.arange(24 * ne))), 8, RW)
         kernels.append(ev)
         # 4 corner sums
         ev = _Ev()
@@ -180,13 +212,14 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs):
         ev.add(I4(NODEELEMSTART, nidx), 4, R)
         ev.add(I4(NODEELEMSTART, nidx + 1), 4, R)
         ev.add(I4(CORNERLIST, np.arange(len(cl))), 4, R)
-        ev.add(tf + 8 * u(3 * cl[:, None] + np.arange(3)), 8, R)
+        ev.add(TMP(lambda: tf + 8 * u(3 * cl[:, None] + np.arange(3))), 8, R)
         for k in (FX, FY, FZ):
             ev.add(D(k, nidx), 8, W)
         kernels.append(ev)
         for ev in kernels:
             ops += [("KB",), ev.op("DB"), ("KE",)]
-            hooks += ev.op("DB")[1].size
+            if hooks is not None:
+                hooks += ev.op("DB")[1].size
         ops.append(("H", dom + 8 * TMP_FORCE, 8, W))
         ops.append(("FREE", tf))
         kernels = []
@@ -210,7 +243,7 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs):
         # 7 velocity, 8 position
         for src, dst in (((XDD, YDD, ZDD), (XD, YD, ZD)), ((XD, YD, ZD), (X, Y, Z))):
             ev = _Ev()
-            ev.add((dom + OFF_DT) * np.ones(nn, np.uint64), 8, R)
+            ev.add(rep(dom + OFF_DT, nn), 8, R)
             for k in src:
                 ev.add(ptr(k, nn), 8, R)
                 ev.add(D(k, nidx), 8, R)
@@ -220,7 +253,8 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs):
             kernels.append(ev)
         for ev in kernels:
             ops += [("KB",), ev.op("DB"), ("KE",)]
-            hooks += ev.op("DB")[1].size
+            if hooks is not None:
+                hooks += ev.op("DB")[1].size
         ops.append(("REG", tg, 8 * 3 * ne, MANAGED))
         ops.append(("H", dom + 8 * TMP_DVDX, 8, W))
         kernels = []
@@ -239,13 +273,13 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs):
             ev.add(ptr(k, ne), 8, R)
             ev.add(D(k, e), 8, W)
         ev.add(ptr(TMP_DVDX, ne), 8, R)
-        ev.add(tg + 8 * u(np.arange(3 * ne)), 8, W)
+        ev.add(TMP(lambda: tg + 8 * u(np.arange(3 * ne))), 8, W)
         kernels.append(ev)
         # 10 lagrange
         ev = _Ev()
         ev.add(numelem(grid_e), 4, R)
         ev.add(ptr(TMP_DVDX, ne), 8, R)
-        ev.add(tg + 8 * u(np.arange(3 * ne)), 8, R)
+        ev.add(TMP(lambda: tg + 8 * u(np.arange(3 * ne))), 8, R)
         ev.add(ptr(VNEW, ne), 8, R)
         ev.add(D(VNEW, e), 8, R)
         ev.add(ptr(VDOV, ne), 8, R)
@@ -253,7 +287,8 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs):
         kernels.append(ev)
         for ev in kernels:
             ops += [("KB",), ev.op("DB"), ("KE",)]
-            hooks += ev.op("DB")[1].size
+            if hooks is not None:
+                hooks += ev.op("DB")[1].size
         ops.append(("H", dom + 8 * TMP_DVDX, 8, W))
         ops.append(("FREE", tg))
         kernels = []
@@ -281,13 +316,13 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs):
         ev.add(D(QQ, e), 8, W)
         kernels.append(ev)
         # 13 EOS stages
-        misc = lambda i: (dom + OFF_MISC + 4 * i) * np.ones(ne, np.uint64)
+        misc = lambda i: rep(dom + OFF_MISC + 4 * i, ne)
         stages = [((0, 1, 2), (DELV, P, Q, QQ, QL), (E,), RW), ((3, 4), (E, VNEW), (P,), W),
                   ((5, 6), (P, E, VNEW), (SS,), W), ((7, 8, 9), (QL, QQ, P), (Q,), W)]
         for ms, ins, outs, kind in stages:
             ev = _Ev()
             ev.add(numelem(grid_e), 4, R)
-            ev.add((dom + OFF_TIME) * np.ones(ne, np.uint64), 8, R)
+            ev.add(rep(dom + OFF_TIME, ne), 8, R)
             for i in ms:
                 ev.add(misc(i), 4, R)
             for k in ins:
@@ -316,7 +351,8 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs):
             kernels.append(ev)
         for ev in kernels:
             ops += [("KB",), ev.op("DB"), ("KE",)]
-            hooks += ev.op("DB")[1].size
+            if hooks is not None:
+                hooks += ev.op("DB")[1].size
         # TimeIncrement (host)
         h = _Ev()
         h.add(dtb + 8 * u(np.arange(2 * nblk)), 8, R)
@@ -328,7 +364,8 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs):
         h.add([dom + OFF_CYCLE], 4, W)
         h.add(dom + OFF_MISC + 4 * u(np.arange(14)), 4, W)
         ops.append(h.op("HB"))
-        ops.append(("DIAG",) + params + (1, ()))
-    ops += [("FREE", a) for a in addrs]
-    ops.append(("DIAG",) + params + (1, ()))
+        ops.append(("DIAG",) + params + (reset, ()))
+    if final:
+        ops += [("FREE", a) for a in addrs]
+        ops.append(("DIAG",) + params + (reset, ()))
     return ops, hooks

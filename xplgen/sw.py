@@ -88,6 +88,12 @@ def sw_trace(addrs, spec, n, m, per_diagonal, tb_every, diag_every, inp, params)
         ii = np.repeat(np.arange(1, n + 1, dtype=np.int64), m)
         jj = np.tile(np.arange(1, m + 1, dtype=np.int64), n)
         ops += [("KB",), cell_events(ii, jj), ("KE",)]
+    elif per_diagonal == 2:
+        # one launch with a device-side epoch split after every anti-diagonal:
+        # the same event sequence as one launch per diagonal (KE KB at a split)
+        for d in range(2, n + m + 1):
+            i, j = _diag_cells(n, m, d)
+            ops += [("KB",), cell_events(i, j), ("KE",)]
     else:
         for d in range(2, n + m + 1):
             i, j = _diag_cells(n, m, d)
@@ -100,7 +106,7 @@ def sw_trace(addrs, spec, n, m, per_diagonal, tb_every, diag_every, inp, params)
     ops.append(batch("HB", Hh + 4 * u64(np.arange((n + 1) * (m + 1))), 4, R))
     rh, ra, rb, _ = sw_traceback(H, inp["a"], inp["b"])
     ops.append(batch("HB", np.concatenate([Hh + 4 * u64(rh), A + 4 * u64(ra), B + 4 * u64(rb)]), 4, R))
-    if not per_diagonal:
+    if per_diagonal != 1:
         ii = np.repeat(np.arange(1, n + 1, dtype=np.int64), m)
         jj = np.tile(np.arange(1, m + 1, dtype=np.int64), n)
         ops += [("KB",), batch("DB", Hh + 4 * u64(ii * ld + jj), 4, W), ("KE",)]
@@ -110,4 +116,6 @@ def sw_trace(addrs, spec, n, m, per_diagonal, tb_every, diag_every, inp, params)
 
 
 def sw_accesses(n, m, per_diagonal):
-    return 6 * n * m + (0 if per_diagonal else n * m)
+    """per_diagonal: 0 = one launch, 1 = one launch per anti-diagonal, 2 = one
+    launch with a device-side epoch split per anti-diagonal."""
+    return 6 * n * m + (0 if per_diagonal == 1 else n * m)

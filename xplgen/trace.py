@@ -221,3 +221,36 @@ def random_trace(seed, n_allocs=6, n_steps=60, max_words=300, p_device=0.5):
             ops.append(("DIAG", thr, blk, mr, int(rng.random() < 0.8), names))
     ops.append(("DIAG", 50, 0, 4, 1, ()))
     return ops
+
+
+def epoch_chain_trace(seed, n_allocs=4, n_chains=3, chain_len=6, max_words=20000, n_ev=3000):
+    """Chains of back-to-back GPU epochs (nothing between them: the shape a
+    single-launch wavefront with device-side epoch splits produces, NEXT-2),
+    each chain preceded by a host segment and followed by a diagnose.  Device
+    events hit a few hot words often (so reads of earlier segments' writes
+    recur) and random words of every allocation, multi-word and unaligned."""
+    rng = np.random.default_rng(seed)
+    ops, allocs, base = [], [], 0x200000
+    for _ in range(n_allocs):
+        nb = int(rng.integers(4, max_words * 4))
+        ops.append(("REG", base, nb, int(rng.integers(0, 3))))
+        allocs.append((base, nb))
+        base += ((nb + 4095) // 4096 + 1) * 4096
+
+    def accesses(n):
+        k = rng.integers(0, len(allocs), size=n)
+        b = np.array([allocs[i][0] for i in k], np.uint64)
+        nb = np.array([allocs[i][1] for i in k], np.int64)
+        hot = rng.random(n) < 0.3
+        off = np.where(hot, 4 * rng.integers(0, 64, size=n), rng.integers(0, nb))
+        size = rng.choice(np.array([1, 2, 4, 8, 16], np.uint32), size=n, p=[0.05, 0.05, 0.6, 0.2, 0.1])
+        return b + off.astype(np.uint64), size.astype(np.uint32), rng.integers(1, 4, size=n).astype(np.uint8)
+
+    for _ in range(n_chains):
+        ops.append(("HB",) + accesses(int(rng.integers(1, 500))))
+        for _ in range(chain_len):
+            ops += [("KB",), ("DB",) + accesses(int(rng.integers(1, n_ev))), ("KE",)]
+        ops.append(("DIAG", int(rng.choice([10, 50, 100])), int(rng.choice([0, 64, 1000])),
+                    int(rng.choice([1, 4, 256])), int(rng.random() < 0.7), ()))
+    ops.append(("DIAG", 50, 0, 4, 1, ()))
+    return ops
