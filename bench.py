@@ -203,6 +203,30 @@ def _allmax(torch, dist, x):
     return float(t.item())
 
 
+def atomic_peaks(xpl, torch, reps=3):
+    """The recording roofline's denominator: 32-bit atomic OR
+    throughput of this B200 from the in-repo microbenchmark, one op per distinct
+    u32, coalesced: RED (what a hook's commit issues) and ATOM over 1 GiB (HBM
+    backed) and over 32 MiB (L2 resident), plus the same-u32-per-warp case."""
+    out = {}
+    buf = torch.zeros(1 << 28, dtype=torch.int32, device="cuda")
+    st = torch.cuda.current_stream()
+    for name, n, mode in (("red_hbm", 1 << 28, 0), ("atom_hbm", 1 << 28, 1), ("red_l2", 1 << 23, 0),
+                          ("red_same_word", 1 << 28, 2)):
+        xpl.atomic_bench(buf.data_ptr(), n, mode, st.cuda_stream)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        k = reps if n >= (1 << 28) else reps * 16
+        e0.record(st)
+        for _ in range(k):
+            xpl.atomic_bench(buf.data_ptr(), n, mode, st.cuda_stream)
+        e1.record(st)
+        e1.synchronize()
+        out[name + "_per_s"] = k * n / (e0.elapsed_time(e1) / 1e3)
+    del buf
+    return out
+
+
 def diag_at_scale(xpl, torch, words=1 << 31, reps=3):
     """The diagnose pass over a cfg5-sized shadow (2^31 words = 2 GiB, SURVEY §8(d)
     cfg5 ~2.2e9 words) with a mixed realistic content: CPU-written half (H2D),
@@ -230,6 +254,12 @@ def diag_at_scale(xpl, torch, words=1 << 31, reps=3):
     pf = ctx.profile_read(reset=True)["fold"]
     ctx.sync()
     torch.cuda.synchronize()
+    # shadow u32s the hooks committed to: one RED each (first touch, warp-aggregated)
+    import numpy as np
+    n_red = 0
+    for w0 in range(0, words, 1 << 28):
+        d = ctx.shadow_dump(base, w0, min(1 << 28, words - w0)).view(np.uint32)
+        n_red += int(np.count_nonzero(d & 0xC8C8C8C8))
     for _ in range(reps):
         ctx.diagnose(50, 0, 256, reset=False)
     p0 = ctx.profile_read(reset=True)
@@ -240,6 +270,7 @@ def diag_at_scale(xpl, torch, words=1 << 31, reps=3):
     n_dev = rep[0]["gpu_acc"]  # each word is hooked at most once by the touch kernel
     out = {"record": {"device_accesses": n_dev, "ms": rec_ms, "accesses_per_s": n_dev / (rec_ms / 1e3),
                       "fold_ms": pf["ms"], "fold_gbs": pf["bytes"] / (pf["ms"] / 1e3) / 1e9 if pf["ms"] else None,
+                      "shadow_u32_committed": n_red,
                       "note": "instrumented touch kernel (hooks only, no user data) + epoch close, events on its stream"}}
     for name, p in (("no_reset", p0), ("reset", p1)):  # (the loop below fills these two)
         d = p["diag_tile"]
@@ -493,6 +524,16 @@ def main():
 
     # --- the diagnose pass at cfg5 scale; the other configs -------------------
     at_scale = diag_at_scale(xpl, torch)
+    atom = atomic_peaks(xpl, torch)
+    rec = at_scale["record"]
+    rec["atomic_microbench"] = atom
+    # recording roofline: accesses/s <= min(HBM / shadow bytes per
+    # access, RED rate x accesses per RED); the touch kernel hooks each word once
+    apr = rec["device_accesses"] / max(1, rec["shadow_u32_committed"])
+    pk, _ = peaks()
+    rec["reds_per_s"] = rec["shadow_u32_committed"] / (rec["ms"] / 1e3)
+    rec["roofline_accesses_per_s"] = min(pk * 1e9 / 2.0, atom["red_hbm_per_s"] * apr)
+    rec["frac"] = rec["accesses_per_s"] / rec["roofline_accesses_per_s"]
     sharded = None
     if world > 1:
         try:

@@ -258,6 +258,59 @@ xpl_status xpl_get_device_ctx(xpl_ctx* ctx, struct xpl_dev_ctx* out);
 xpl_status xpl_shadow_dump(xpl_ctx* ctx, const void* base, uint64_t word0, uint64_t n,
                            uint8_t* out);
 
+/* ---- Unified-memory page view ----
+ * The current interval's records aggregated per page of `page_words` words (pages
+ * counted from the allocation base, D31; the last page may be partial): which
+ * processors touched the page, whether some single word was touched by both
+ * (true sharing) or only disjoint words were (the "effect similar to false
+ * sharing" of P:L90), and whether some word alternated (D9).  Page bits: */
+#define XPL_PAGE_CPU 1u    /* some word accessed by the CPU (wC | rCC | rGC)  */
+#define XPL_PAGE_GPU 2u    /* some word accessed by the GPU (wG | rCG | rGG)  */
+#define XPL_PAGE_BOTH 4u   /* some word accessed by both                       */
+#define XPL_PAGE_ALT 8u    /* some alternating word (both, >= 1 a write, D9)   */
+#define XPL_PAGE_CPU_W 16u /* some word written by the CPU                     */
+#define XPL_PAGE_GPU_W 32u /* some word written by the GPU                     */
+
+/* cudaMemAdvise hints recorded per allocation, as bits: */
+#define XPL_ADVICE_READ_MOSTLY 1u
+#define XPL_ADVICE_PREFERRED_GPU 2u
+#define XPL_ADVICE_PREFERRED_CPU 4u
+#define XPL_ADVICE_ACCESSED_BY_GPU 8u
+#define XPL_ADVICE_ACCESSED_BY_CPU 16u
+
+/* Page-report flags (managed allocations only, D8 / P:L84): */
+#define XPL_PAGE_PAT_FALSE_SHARING 1u   /* a page used by both sides on disjoint words */
+#define XPL_PAGE_PAT_ADVICE_MISMATCH 2u /* ReadMostly advised, yet a page alternates (D32) */
+
+typedef struct {
+  uint64_t id, base, words, page_words, pages;
+  uint32_t kind, advice; /* xpl_alloc_kind; XPL_ADVICE_* bits in force           */
+  uint64_t cpu_pages, gpu_pages;
+  uint64_t shared_pages;       /* CPU and GPU pages                                 */
+  uint64_t false_shared_pages; /* shared pages on which no word was used by both    */
+  uint64_t alternating_pages;  /* pages holding an alternating word                 */
+  uint32_t flags, pad;         /* XPL_PAGE_PAT_*                                    */
+} xpl_page_report;
+
+/* The page view of every live row, in id order, into out[0..cap) (*n_out rows;
+ * INVALID_ARG with *n_out = rows needed if cap is too small, or page_words == 0).
+ * Reads the interval bits without changing them: call it before the resetting
+ * diagnose of the interval.  STATE inside an open epoch.  Blocks until done. */
+xpl_status xpl_page_summary(xpl_ctx* ctx, uint64_t page_words, xpl_page_report* out, size_t cap,
+                            size_t* n_out);
+
+/* The page bits (XPL_PAGE_*) of the live row whose base is `base`: out[n_pages],
+ * n_pages must be ceil(words / page_words) (else INVALID_ARG).  The page map
+ * of Fig. 5-style plots.  Blocks until done. */
+xpl_status xpl_page_flags(xpl_ctx* ctx, const void* base, uint64_t page_words, uint8_t* out,
+                          uint64_t n_pages);
+
+/* The cudaMemAdvise wrapper: records advice (cudaMemoryAdvise numbering: 1 Set/2
+ * Unset ReadMostly, 3 Set/4 Unset PreferredLocation, 5 Set/6 Unset AccessedBy;
+ * device < 0 = the CPU) for the allocation holding `ptr`, as a whole (D33).
+ * Untracked pointers are ignored.  INVALID_ARG on another advice value. */
+xpl_status xpl_mem_advise(xpl_ctx* ctx, const void* ptr, size_t bytes, int advice, int device);
+
 /* Apply every staged host record now (normally done lazily at kernel_begin,
  * diagnose and when staging fills up).  Asynchronous. */
 xpl_status xpl_flush(xpl_ctx* ctx);

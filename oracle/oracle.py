@@ -32,6 +32,17 @@ class XoReport(C.Structure):
     _fields_ = REPORT_FIELDS
 
 
+PAGE_FIELDS = [
+    ("id", C.c_uint64), ("base", C.c_uint64), ("words", C.c_uint64), ("page_words", C.c_uint64),
+    ("pages", C.c_uint64), ("kind", C.c_uint32), ("advice", C.c_uint32), ("cpu_pages", C.c_uint64),
+    ("gpu_pages", C.c_uint64), ("shared_pages", C.c_uint64), ("false_shared_pages", C.c_uint64),
+    ("alternating_pages", C.c_uint64), ("flags", C.c_uint32), ("pad", C.c_uint32)]
+
+
+class XoPageReport(C.Structure):
+    _fields_ = PAGE_FIELDS
+
+
 def build():
     """Compile liboracle.so and the CLI with make (plain g++, no CUDA)."""
     subprocess.run(["make", "-s", "-C", HERE], check=True)
@@ -62,6 +73,9 @@ def _load():
         lib.xo_diag.argtypes = [vp, u32, u64, u64, C.c_int, vp, C.c_size_t, vp, C.c_size_t]
         lib.xo_diag.restype = C.c_int64
         lib.xo_peek.argtypes = [vp, u64, u64]
+        lib.xo_pages.argtypes = [vp, u64, vp, C.c_size_t]
+        lib.xo_pages.restype = C.c_int64
+        lib.xo_advise.argtypes = [vp, u64, u32, C.c_int]
         _lib = lib
     return _lib
 
@@ -116,6 +130,10 @@ class Oracle:
             self._ok(lib.xo_copy(s, op[2], op[3], op[4], op[1]), op)
         elif t == "DIAG":
             return self.diag(*op[1:6])
+        elif t == "PAGES":  # ("PAGES", page_words): the UM page view (NEXT-3)
+            return self.pages(op[1])
+        elif t == "ADVISE":  # ("ADVISE", ptr, bytes, advice, device)
+            self._ok(lib.xo_advise(s, op[1], op[3], op[4]), op)
         else:
             raise ValueError(op)
         return None
@@ -131,6 +149,17 @@ class Oracle:
                 raise RuntimeError("oracle rejected DIAG")
             if n <= cap:
                 return [{f: getattr(out[i], f) for f, _ in REPORT_FIELDS} for i in range(n)]
+            cap = n
+
+    def pages(self, page_words):
+        cap = 64
+        while True:
+            out = (XoPageReport * cap)()
+            n = self.lib.xo_pages(self.s, page_words, out, cap)
+            if n < 0:
+                raise RuntimeError("oracle rejected PAGES")
+            if n <= cap:
+                return [{f: getattr(out[i], f) for f, _ in PAGE_FIELDS if f != "pad"} for i in range(n)]
             cap = n
 
     def peek(self, alloc_id, word):

@@ -50,7 +50,12 @@ struct Row {
   uint32_t kind;
   bool live;
   bool ever;
+  uint32_t advice;  // cudaMemAdvise hints in force (bits below), D33
 };
+
+// cudaMemAdvise hints as bits: ReadMostly, PreferredLocation GPU /
+// CPU, AccessedBy GPU / CPU.
+const uint32_t kAdvReadMostly = 1, kAdvPrefGpu = 2, kAdvPrefCpu = 4, kAdvByGpu = 8, kAdvByCpu = 16;
 
 typedef std::pair<uint64_t, uint64_t> Key;  // (allocation id, word)
 
@@ -232,6 +237,7 @@ int64_t xo_reg(xo_state* s, uint64_t ptr, uint64_t bytes, uint32_t kind) {
   r.kind = kind;
   r.live = true;
   r.ever = false;
+  r.advice = 0;
   s->rows.push_back(r);
   s->live[ptr] = r.id;
   return (int64_t)r.id;
@@ -402,6 +408,78 @@ int64_t xo_diag(xo_state* s, uint32_t thr_pct, uint64_t block_words,
     s->dead.clear();
   }
   return (int64_t)ids.size();
+}
+
+// UM page view (NEXT-3).  For page p of a live row (words [p*P, min((p+1)*P,
+// words)), D31) the OR over its words of: accessed by the CPU (wC, rCC or rGC),
+// by the GPU (wG, rCG or rGG), by both, alternating (both and written, D9).
+// A page is shared if both processors touched it -- under unified memory it
+// would move between them; false-shared if no single word was
+// touched by both ("an effect similar to false sharing").  Flags only
+// for managed allocations (D8): FALSE_SHARING = some false-shared page;
+// ADVICE_MISMATCH = ReadMostly advised yet some page alternates, i.e. a write
+// to data the other processor also uses invalidates its read copies (P:L47,
+// P:L86, D32).
+int64_t xo_pages(xo_state* s, uint64_t P, xo_page_report* out, size_t cap) {
+  if (P == 0) return -1;
+  size_t n = 0;
+  for (size_t id = 0; id < s->rows.size(); ++id) {
+    const Row& r = s->rows[id];
+    if (!r.live) continue;
+    if (n < cap) {
+      xo_page_report& o = out[n];
+      std::memset(&o, 0, sizeof o);
+      o.id = r.id;
+      o.base = r.base;
+      o.words = r.words;
+      o.page_words = P;
+      o.pages = (r.words + P - 1) / P;
+      o.kind = r.kind;
+      o.advice = r.advice;
+      for (uint64_t p = 0; p < o.pages; ++p) {
+        bool cpu = false, gpu = false, both = false, alt = false;
+        for (uint64_t w = p * P; w < (p + 1) * P && w < r.words; ++w) {
+          const uint8_t rec = get(s, Key(r.id, w));
+          const bool c = (rec & kWC) || (rec & kRCC) || (rec & kRGC);
+          const bool g = (rec & kWG) || (rec & kRCG) || (rec & kRGG);
+          cpu = cpu || c;
+          gpu = gpu || g;
+          both = both || (c && g);
+          alt = alt || (c && g && ((rec & kWC) || (rec & kWG)));
+        }
+        if (cpu) o.cpu_pages++;
+        if (gpu) o.gpu_pages++;
+        if (cpu && gpu) o.shared_pages++;
+        if (cpu && gpu && !both) o.false_shared_pages++;
+        if (alt) o.alternating_pages++;
+      }
+      if (r.kind == kManaged) {
+        if (o.false_shared_pages > 0) o.flags |= 1;
+        if ((r.advice & kAdvReadMostly) && o.alternating_pages > 0) o.flags |= 2;
+      }
+    }
+    ++n;
+  }
+  return (int64_t)n;
+}
+
+// cudaMemAdvise wrapper: the hint applies to the whole allocation holding ptr
+// (D33); untracked pointers are ignored.  Set/Unset pairs in the
+// order of the cudaMemoryAdvise enum: 1/2 ReadMostly, 3/4 PreferredLocation,
+// 5/6 AccessedBy; a negative device means the CPU (cudaCpuDeviceId).
+int xo_advise(xo_state* s, uint64_t ptr, uint32_t advice, int device) {
+  if (advice < 1 || advice > 6) return -1;
+  uint64_t id, w0, w1;
+  if (!lookup(s, ptr, 1, &id, &w0, &w1)) return 0;
+  uint32_t& a = s->rows[id].advice;
+  const bool cpu = device < 0;
+  if (advice == 1) a |= kAdvReadMostly;
+  if (advice == 2) a &= ~kAdvReadMostly;
+  if (advice == 3) a = (a & ~(kAdvPrefGpu | kAdvPrefCpu)) | (cpu ? kAdvPrefCpu : kAdvPrefGpu);
+  if (advice == 4) a &= ~(kAdvPrefGpu | kAdvPrefCpu);
+  if (advice == 5) a |= cpu ? kAdvByCpu : kAdvByGpu;
+  if (advice == 6) a &= ~(cpu ? kAdvByCpu : kAdvByGpu);
+  return 0;
 }
 
 int xo_peek(xo_state* s, uint64_t id, uint64_t word) {

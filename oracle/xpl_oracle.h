@@ -52,6 +52,18 @@ int xo_copy(xo_state*, uint64_t dst, uint64_t src, uint64_t bytes, uint32_t dir)
 int64_t xo_diag(xo_state*, uint32_t thr_pct, uint64_t block_words,
                 uint64_t min_run, int reset, const uint64_t* name_addrs,
                 size_t n_names, xo_report* out, size_t cap);
+/* UM page view (D31-D33):
+ * per live row, its pages of page_words words counted from the base. */
+typedef struct {
+  uint64_t id, base, words, page_words, pages;
+  uint32_t kind, advice;
+  uint64_t cpu_pages, gpu_pages, shared_pages, false_shared_pages, alternating_pages;
+  uint32_t flags, pad;
+} xo_page_report;
+/* Rows written (or needed, if > cap); negative on error.  Changes nothing. */
+int64_t xo_pages(xo_state*, uint64_t page_words, xo_page_report* out, size_t cap);
+/* cudaMemAdvise: advice 1..6 in cudaMemoryAdvise order, device < 0 = CPU. */
+int xo_advise(xo_state*, uint64_t ptr, uint32_t advice, int device);
 /* The record byte of (allocation id, word); 0 if never touched. */
 int xo_peek(xo_state*, uint64_t id, uint64_t word);
 

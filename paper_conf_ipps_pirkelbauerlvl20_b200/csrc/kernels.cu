@@ -420,38 +420,32 @@ __device__ __noinline__ RunSum run_step_mixed(RunSum a, const uint32_t* bits, ui
 // sharded allocation needs).  Streams the 32 lane masks; rare (once per row).
 __device__ __noinline__ RunSum run_step_exact(RunSum a, const uint32_t* bits, uint32_t shift,
                                               uint32_t n, uint32_t min_run) {
-  const uint32_t m = pack4(bits[0] >> shift) | (pack4(bits[1] >> shift) << 4) |
-                     (pack4(bits[2] >> shift) << 8) | (pack4(bits[3] >> shift) << 12);
-  uint32_t pre = 0, run = 0, cnt = 0, sum = 0;
-  bool seen_zero = false;
-  for (uint32_t l = 0; l < 32; ++l) {
-    const uint32_t ml = __shfl_sync(0xFFFFFFFFu, m, l);
-    for (uint32_t k = 0; k < 16; ++k) {
-      if (l * 16 + k >= n) break;
-      if ((ml >> k) & 1u) {
-        ++run;
-      } else {
-        if (!seen_zero) {
-          pre = run;
-          seen_zero = true;
-        } else if (run >= min_run && run > 0) {
-          ++cnt;
-          sum += run;
-        }
-        run = 0;
-      }
-    }
-  }
+  // warp-parallel: the 512-word summary of the step with the words >= n as
+  // zeros (warp_runs), then the run that reaches word n-1 is reopened -- it is
+  // the exact summary's suffix, not a closed run (len = n).  n in [1, 512).
+  const uint32_t lane = threadIdx.x & 31, base = lane * 16;
+  const uint32_t valid = base >= n ? 0u : (n - base >= 16 ? 0xFFFFu : ((1u << (n - base)) - 1u));
+  const uint32_t m = (pack4(bits[0] >> shift) | (pack4(bits[1] >> shift) << 4) |
+                      (pack4(bits[2] >> shift) << 8) | (pack4(bits[3] >> shift) << 12)) & valid;
+  const RunSum w = warp_runs(m, lane, min_run);
   RunSum b;
   b.len = n;
-  if (!seen_zero) {
+  if (w.pre >= n) {  // all ones in [0, n)
     b.pre = b.suf = n;
+    b.cnt = b.sum = 0;
   } else {
-    b.pre = pre;
-    b.suf = run;
+    const uint32_t z = ~m & valid;  // zeros inside [0, n)
+    const uint32_t lz1 = z ? base + 32 - __clz(z) : 0u;  // (last zero of the lane) + 1
+    const uint32_t t = n - __reduce_max_sync(0xFFFFFFFFu, lz1);  // ones ending at n-1
+    b.pre = w.pre;
+    b.suf = t;
+    b.cnt = w.cnt;
+    b.sum = w.sum;
+    if (t > 0 && t >= min_run) {  // warp_runs closed it at the padding
+      b.cnt -= 1;
+      b.sum -= t;
+    }
   }
-  b.cnt = cnt;
-  b.sum = sum;
   return rs_combine32(a, b, min_run);
 }
 
@@ -622,8 +616,14 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
 // issues a whole ring ahead; each slot's mbarrier counts the bytes in.  No
 // register staging, so the prefetch depth (8 KB per warp) does not cost
 // registers (occupancy), and the wait + refill is paid once per kStageSteps.
-constexpr uint32_t kStageSteps = 4;
-constexpr uint32_t kDiagStages = 4;
+#ifndef XPL_DIAG_STAGE_STEPS
+#define XPL_DIAG_STAGE_STEPS 2
+#endif
+#ifndef XPL_DIAG_STAGES
+#define XPL_DIAG_STAGES 4
+#endif
+constexpr uint32_t kStageSteps = XPL_DIAG_STAGE_STEPS;
+constexpr uint32_t kDiagStages = XPL_DIAG_STAGES;
 struct WarpRing {
   uint4 buf[kDiagStages][kStageSteps * 32];
   uint64_t bar[kDiagStages];
@@ -675,7 +675,7 @@ __device__ __forceinline__ void tile_loop(TileAcc& A, WarpRing& R, uint4* p4, ui
 // 512-word steps, warp_runs() for mixed ones.  Reset fused.  The tile's counts
 // and run summaries go to tiles[t]; the stitch adds and combines them in order.
 #ifndef XPL_DIAG_MINB
-#define XPL_DIAG_MINB 3  // CTAs per SM the register budget is sized for
+#define XPL_DIAG_MINB 4  // CTAs per SM the register budget is sized for (A/B: profiles/r1h_diag_variants.txt)
 #endif
 __global__ void __launch_bounds__(kDiagThreads, XPL_DIAG_MINB) diag_tile_kernel(
     const DiagRow* __restrict__ rows, const uint32_t* __restrict__ tile_row, uint64_t ntiles,
@@ -925,6 +925,79 @@ int grid_for(uint64_t n, int threads, int max_ctas) {
   return (int)g;
 }
 
+
+// ---------------------------------------------------------------------------
+// UM page view (NEXT-3): per page of P words of a row, the
+// OR over its records of: CPU access, GPU access, a word accessed by both, an
+// alternating word (D9), CPU write, GPU write.  One warp per contiguous chunk of
+// pages (so the row changes rarely); lanes stride over the page's shadow u32s,
+// bytes outside the page masked; per-row page counts in registers, flushed with
+// one atomicAdd per counter when the warp leaves a row.
+__device__ __forceinline__ uint32_t page_bits(uint32_t x) {
+  const uint32_t cpu = ((x & 0x34343434u) + 0x7F7F7F7Fu) & 0x80808080u;          // wC|rCC|rGC
+  const uint32_t gpu = (((x & 0x48484848u) + 0x7F7F7F7Fu) | x) & 0x80808080u;    // wG|rCG|rGG
+  const uint32_t wr = ((x & 0x0C0C0C0Cu) + 0x7F7F7F7Fu) & 0x80808080u;           // wC|wG
+  const uint32_t both = cpu & gpu;
+  return (cpu ? 1u : 0u) | (gpu ? 2u : 0u) | (both ? 4u : 0u) | ((both & wr) ? 8u : 0u) |
+         ((x & 0x04040404u) ? 16u : 0u) | ((x & 0x08080808u) ? 32u : 0u);
+}
+
+__global__ void __launch_bounds__(256) page_kernel(const PageRow* __restrict__ rows, uint32_t nrows,
+                                                   uint64_t npages, uint64_t P,
+                                                   const uint32_t* __restrict__ pool,
+                                                   uint8_t* __restrict__ flags,
+                                                   unsigned long long* __restrict__ cnt) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
+  const uint64_t wi = (uint64_t)blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32;
+  const uint64_t chunk = (npages + nw - 1) / nw;
+  const uint64_t p0 = wi * chunk, p1 = min(npages, p0 + chunk);
+  if (p0 >= p1) return;
+  uint32_t lo = 0, hi = nrows;  // the row holding page p0: last row with page0 <= p0
+  while (hi - lo > 1) {
+    const uint32_t mid = (lo + hi) / 2;
+    if (rows[mid].page0 <= p0) lo = mid;
+    else hi = mid;
+  }
+  uint32_t r = lo;
+  unsigned long long c[5] = {0, 0, 0, 0, 0};
+  for (uint64_t p = p0; p < p1; ++p) {
+    while (r + 1 < nrows && rows[r + 1].page0 <= p) {  // next row: flush its counts
+      const unsigned long long v = lane == 0 ? c[0] : lane == 1 ? c[1] : lane == 2 ? c[2] : lane == 3 ? c[3] : c[4];
+      if (lane < 5 && v) atomicAdd(cnt + 5ull * r + lane, v);
+#pragma unroll
+      for (int k = 0; k < 5; ++k) c[k] = 0;
+      ++r;
+    }
+    const PageRow R = rows[r];
+    const uint64_t w0 = R.off + (p - R.page0) * P;                  // pool words [w0, w1)
+    const uint64_t w1 = R.off + min(R.words, (p - R.page0 + 1) * P);
+    uint32_t f = 0;
+    for (uint64_t q = (w0 >> 2) + lane; q <= ((w1 - 1) >> 2); q += 32) {
+      uint32_t x = pool[q];
+      if (q * 4 < w0 || q * 4 + 4 > w1) {
+        uint32_t m = 0;
+#pragma unroll
+        for (uint32_t k = 0; k < 4; ++k)
+          if (q * 4 + k >= w0 && q * 4 + k < w1) m |= 0xFFu << (8 * k);
+        x &= m;
+      }
+      f |= page_bits(x);
+    }
+    f = __reduce_or_sync(0xFFFFFFFFu, f);
+    if (flags && lane == 0) flags[p] = (uint8_t)f;
+    const bool shared = (f & 3u) == 3u;
+    c[0] += f & 1u;
+    c[1] += (f >> 1) & 1u;
+    c[2] += shared;
+    c[3] += shared && !(f & 4u);
+    c[4] += (f >> 3) & 1u;
+  }
+  if (lane < 5) {
+    const unsigned long long v = lane == 0 ? c[0] : lane == 1 ? c[1] : lane == 2 ? c[2] : lane == 3 ? c[3] : c[4];
+    if (v) atomicAdd(cnt + 5ull * r + lane, v);
+  }
+}
 }  // namespace
 
 void launch_fold(cudaStream_t s, bool pdl, uint32_t* pool, uint8_t* cmap, uint8_t* smap,
@@ -979,6 +1052,13 @@ void launch_diag(cudaStream_t s, const DiagRow* rows, uint32_t nrows, const uint
                                                              (RunPair*)segsum, cnt);
   stitch_row_finalize_kernel<<<(nrows * 32 + 255) / 256, 256, 0, s>>>(rows, nrows, (const RunPair*)segsum,
                                                                        p, cnt, out, parts, blk_cnt);
+}
+
+void launch_pages(cudaStream_t s, const PageRow* rows, uint32_t nrows, uint64_t npages, uint64_t page_words,
+                  const uint32_t* pool, uint8_t* flags, unsigned long long* cnt) {
+  if (!npages || !nrows) return;
+  const uint64_t warps = npages < 148ull * 64 ? npages : 148ull * 64;  // <= 8 pages' chunk per warp at small n
+  page_kernel<<<(unsigned)((warps + 7) / 8), 256, 0, s>>>(rows, nrows, npages, page_words, pool, flags, cnt);
 }
 
 void launch_fill_u32(cudaStream_t s, uint32_t* p, uint64_t n, uint32_t v) {

@@ -30,6 +30,7 @@ struct Row {
   uint64_t logical_id, goff, lbytes;           // sharded pieces (else id, 0, bytes)
   uint32_t kind;
   bool live, dropped, ever;
+  uint32_t advice = 0;  // XPL_ADVICE_* bits (xpl_mem_advise)
 };
 
 // First-fit allocator of shadow-pool ranges (16-word granules so every row
@@ -513,6 +514,110 @@ xpl_status join(xpl_ctx* c, cudaStream_t s) {
 
 extern "C" {
 
+// ---- UM page view (NEXT-3; D31-D33) ----------------------
+static xpl_status page_pass(xpl_ctx* c, const std::vector<const Row*>& rows, uint64_t P,
+                            uint8_t* h_flags, unsigned long long* h_cnt) {
+  std::vector<PageRow> pr(rows.size());
+  uint64_t np = 0;
+  for (size_t i = 0; i < rows.size(); ++i) {
+    pr[i].off = rows[i]->off;
+    pr[i].words = rows[i]->words;
+    pr[i].page0 = np;
+    np += (rows[i]->words + P - 1) / P;
+  }
+  PageRow* d_rows = nullptr;
+  unsigned long long* d_cnt = nullptr;
+  uint8_t* d_flags = nullptr;
+  const size_t ncnt = 5 * rows.size();
+  CK(cudaMallocAsync((void**)&d_rows, sizeof(PageRow) * pr.size() + 1, c->cs));
+  CK(cudaMallocAsync((void**)&d_cnt, sizeof(unsigned long long) * ncnt + 8, c->cs));
+  if (h_flags) CK(cudaMallocAsync((void**)&d_flags, np + 1, c->cs));
+  CK(cudaMemcpyAsync(d_rows, pr.data(), sizeof(PageRow) * pr.size(), cudaMemcpyHostToDevice, c->cs));
+  CK(cudaMemsetAsync(d_cnt, 0, sizeof(unsigned long long) * ncnt + 8, c->cs));
+  launch_pages(c->cs, d_rows, (uint32_t)pr.size(), np, P, (const uint32_t*)c->d_pool, d_flags, d_cnt);
+  c->st.kernel_launches += 1;
+  CK(cudaMemcpyAsync(h_cnt, d_cnt, sizeof(unsigned long long) * ncnt, cudaMemcpyDeviceToHost, c->cs));
+  if (h_flags) CK(cudaMemcpyAsync(h_flags, d_flags, np, cudaMemcpyDeviceToHost, c->cs));
+  CK(cudaFreeAsync(d_rows, c->cs));
+  CK(cudaFreeAsync(d_cnt, c->cs));
+  if (d_flags) CK(cudaFreeAsync(d_flags, c->cs));
+  CK(cudaStreamSynchronize(c->cs));
+  return XPL_OK;
+}
+
+xpl_status xpl_page_summary(xpl_ctx* c, uint64_t P, xpl_page_report* out, size_t cap, size_t* n_out) {
+  if (!c || !n_out || P == 0 || (cap && !out)) return XPL_ERR_INVALID_ARG;
+  if (c->depth) return XPL_ERR_STATE;
+  std::vector<const Row*> rows;
+  for (const Row& r : c->rows)
+    if (r.live) rows.push_back(&r);  // (c->rows is in id order)
+  *n_out = rows.size();
+  if (cap < rows.size()) return XPL_ERR_INVALID_ARG;
+  xpl_status st = flush(c);
+  if (st) return st;
+  std::vector<unsigned long long> cnt(5 * rows.size() + 1);
+  if (!rows.empty()) {
+    st = page_pass(c, rows, P, nullptr, cnt.data());
+    if (st) return st;
+  }
+  for (size_t i = 0; i < rows.size(); ++i) {
+    const Row& r = *rows[i];
+    xpl_page_report& o = out[i];
+    memset(&o, 0, sizeof o);
+    o.id = r.id;
+    o.base = r.base;
+    o.words = r.words;
+    o.page_words = P;
+    o.pages = (r.words + P - 1) / P;
+    o.kind = r.kind;
+    o.advice = r.advice;
+    o.cpu_pages = cnt[5 * i + 0];
+    o.gpu_pages = cnt[5 * i + 1];
+    o.shared_pages = cnt[5 * i + 2];
+    o.false_shared_pages = cnt[5 * i + 3];
+    o.alternating_pages = cnt[5 * i + 4];
+    if (r.kind == XPL_ALLOC_MANAGED) {  // D8: page effects exist for unified memory only
+      if (o.false_shared_pages) o.flags |= XPL_PAGE_PAT_FALSE_SHARING;
+      if ((r.advice & XPL_ADVICE_READ_MOSTLY) && o.alternating_pages) o.flags |= XPL_PAGE_PAT_ADVICE_MISMATCH;
+    }
+  }
+  return XPL_OK;
+}
+
+xpl_status xpl_page_flags(xpl_ctx* c, const void* base, uint64_t P, uint8_t* out, uint64_t n_pages) {
+  if (!c || !out || P == 0) return XPL_ERR_INVALID_ARG;
+  if (c->depth) return XPL_ERR_STATE;
+  auto it = c->live.find((uint64_t)base);
+  if (it == c->live.end()) return XPL_ERR_UNKNOWN_PTR;
+  const Row* r = &c->rows[it->second];
+  if (n_pages != (r->words + P - 1) / P) return XPL_ERR_INVALID_ARG;
+  xpl_status st = flush(c);
+  if (st) return st;
+  unsigned long long cnt[5];
+  return page_pass(c, std::vector<const Row*>{r}, P, out, cnt);
+}
+
+xpl_status xpl_mem_advise(xpl_ctx* c, const void* ptr, size_t bytes, int advice, int device) {
+  (void)bytes;  // D33: advice is tracked per allocation
+  if (!c || advice < 1 || advice > 6) return XPL_ERR_INVALID_ARG;
+  const Row* cr = lookup(c, (uint64_t)ptr);
+  if (!cr) return XPL_OK;  // untracked
+  Row& r = c->rows[cr->id];
+  const bool cpu = device < 0;
+  switch (advice) {
+    case 1: r.advice |= XPL_ADVICE_READ_MOSTLY; break;
+    case 2: r.advice &= ~XPL_ADVICE_READ_MOSTLY; break;
+    case 3:
+      r.advice &= ~(XPL_ADVICE_PREFERRED_GPU | XPL_ADVICE_PREFERRED_CPU);
+      r.advice |= cpu ? XPL_ADVICE_PREFERRED_CPU : XPL_ADVICE_PREFERRED_GPU;
+      break;
+    case 4: r.advice &= ~(XPL_ADVICE_PREFERRED_GPU | XPL_ADVICE_PREFERRED_CPU); break;
+    case 5: r.advice |= cpu ? XPL_ADVICE_ACCESSED_BY_CPU : XPL_ADVICE_ACCESSED_BY_GPU; break;
+    default: r.advice &= ~(cpu ? XPL_ADVICE_ACCESSED_BY_CPU : XPL_ADVICE_ACCESSED_BY_GPU); break;
+  }
+  return XPL_OK;
+}
+
 const char* xpl_status_string(xpl_status s) {
   switch (s) {
     case XPL_OK: return "ok";
@@ -660,6 +765,7 @@ static xpl_status register_row(xpl_ctx* c, const void* ptr, size_t bytes, xpl_al
   r.live = true;
   r.dropped = false;
   r.ever = false;
+  r.advice = 0;
   r.logical_id = piece ? logical_id : r.id;
   r.goff = piece ? goff : 0;
   r.lbytes = piece ? lbytes : bytes;

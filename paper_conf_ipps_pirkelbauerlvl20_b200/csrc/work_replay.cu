@@ -68,9 +68,33 @@ __global__ void touch_kernel(unsigned long long base, unsigned long long n, unsi
   }
 }
 
+// Atomic-throughput microbenchmark (the recording roofline):
+// one 32-bit OR per u32 of p[0, n), grid-stride, coalesced.  mode 0: RED
+// (no return value -- what a hook's commit issues); mode 1: ATOM (return value
+// consumed); mode 2: every lane of a warp on the same u32 (the same-word case
+// without warp aggregation).
+__global__ void atomic_bench_kernel(unsigned* p, unsigned long long n, int mode, unsigned* sink) {
+  unsigned acc = 0;
+  for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (unsigned long long)gridDim.x * blockDim.x) {
+    const unsigned v = 1u << (i & 31);
+    if (mode == 0) atomicOr(p + i, v);
+    else if (mode == 1) acc ^= atomicOr(p + i, v);
+    else atomicOr(p + (i >> 5), v);
+  }
+  if (mode == 1 && acc == 0x9E3779B9u) *sink = acc;  // keep the return values live
+}
+
 }  // namespace
 
 extern "C" {
+
+int xplw_atomic_bench(void* buf, unsigned long long n_u32, int mode, void* stream) {
+  atomic_bench_kernel<<<148 * 16, 256, 0, (cudaStream_t)stream>>>((unsigned*)buf, n_u32, mode,
+                                                                  (unsigned*)buf);
+  return cudaGetLastError() == cudaSuccess ? 0 : (int)XPL_ERR_CUDA;
+}
+
 
 // Launch the synthetic touch kernel (between xpl_kernel_begin/_end) over the n
 // words at base, which are logical words i0 .. i0+n-1 of the pattern.

@@ -109,6 +109,11 @@ void launch_diag(cudaStream_t s, const DiagRow* rows, uint32_t nrows, const uint
                  void* segsum, uint32_t* blk_cnt, xpl_alloc_report* out, RowPartial* parts,
                  cudaEvent_t tile_ev0, cudaEvent_t tile_ev1);
 constexpr size_t kRunPairBytes = 80;  // sizeof(RunPair) in kernels.cu
+struct PageRow {  // one live row of a page pass (NEXT-3)
+  uint64_t off, words, page0;  // pool word offset, words, first global page index
+};
+void launch_pages(cudaStream_t s, const PageRow* rows, uint32_t nrows, uint64_t npages, uint64_t page_words,
+                  const uint32_t* pool, uint8_t* flags, unsigned long long* cnt);
 void launch_fill_u32(cudaStream_t s, uint32_t* p, uint64_t n, uint32_t v);
 
 }  // namespace xpl

@@ -160,6 +160,11 @@ def run_trace(ops, ctx: Context | None = None, grid=0, block=256, seed=None, hos
         elif t == "X":
             flush_dev()
             ctx.record_copy(op[2], op[3], op[4], op[1])
+        elif t == "PAGES":
+            flush_dev()
+            results.append(ctx.page_summary(op[1]))
+        elif t == "ADVISE":
+            ctx.mem_advise(op[1], op[2], op[3], op[4])
         elif t == "DIAG":
             results.append(ctx.diagnose(op[1], op[2], op[3], bool(op[4]), op[5]))
         else:

@@ -110,6 +110,19 @@ xpl_format_reports = _sig("xpl_format_reports", [C.POINTER(XplAllocReport), sz, 
                                                  i32, C.c_char_p, sz, C.POINTER(sz)])
 xpl_get_device_ctx = _sig("xpl_get_device_ctx", [vp, C.POINTER(XplDevCtx)])
 xpl_shadow_dump = _sig("xpl_shadow_dump", [vp, vp, u64, u64, vp])
+PAGE_REPORT_FIELDS = [
+    ("id", u64), ("base", u64), ("words", u64), ("page_words", u64), ("pages", u64),
+    ("kind", u32), ("advice", u32), ("cpu_pages", u64), ("gpu_pages", u64), ("shared_pages", u64),
+    ("false_shared_pages", u64), ("alternating_pages", u64), ("flags", u32), ("pad", u32)]
+
+
+class XplPageReport(C.Structure):
+    _fields_ = PAGE_REPORT_FIELDS
+
+
+xpl_page_summary = _sig("xpl_page_summary", [vp, u64, C.POINTER(XplPageReport), sz, C.POINTER(sz)])
+xpl_page_flags = _sig("xpl_page_flags", [vp, vp, u64, vp, u64])
+xpl_mem_advise = _sig("xpl_mem_advise", [vp, vp, sz, i32, i32])
 xpl_flush = _sig("xpl_flush", [vp])
 xpl_sync = _sig("xpl_sync", [vp])
 xpl_join = _sig("xpl_join", [vp, vp])
@@ -131,12 +144,13 @@ EXPORTED = ["xpl_init", "xpl_finalize", "xpl_register_alloc", "xpl_free", "xpl_k
             "xpl_get_device_ctx", "xpl_shadow_dump", "xpl_flush", "xpl_sync", "xpl_join",
             "xpl_runtime_stream", "xpl_get_stats", "xpl_status_string", "xpl_profile",
             "xpl_profile_read", "xpl_register_alloc_piece", "xpl_diagnose_partials", "xpl_combine_partials",
-            "xpl_format_reports"]
+            "xpl_format_reports", "xpl_page_summary", "xpl_page_flags", "xpl_mem_advise"]
 
 if _work is not None:
     xplw_bind = _sig("xplw_bind", [vp], lib=_work)
     xplw_replay = _sig("xplw_replay", [vp, vp, vp, u64, i32, i32, vp], lib=_work)
     xplw_replay_split = _sig("xplw_replay_split", [vp, vp, vp, vp, i32, i32, i32, vp], lib=_work)
+    xplw_atomic_bench = _sig("xplw_atomic_bench", [vp, u64, i32, vp], lib=_work)
     xplw_touch = _sig("xplw_touch", [u64, u64, u32, vp, u64], lib=_work)
 
 
@@ -243,6 +257,27 @@ class Context:
             check("xpl_diagnose_partials", st)
             return bytes(memoryview(out).cast("B")[:n.value * C.sizeof(XplPartial)])
 
+    def page_summary(self, page_words=1024):
+        """The UM page view of every live row (xpl_page_summary), as dicts."""
+        cap = 64
+        while True:
+            out = (XplPageReport * cap)()
+            n = sz(0)
+            st = xpl_page_summary(self.h, page_words, out, cap, C.byref(n))
+            if st == 1 and n.value > cap:
+                cap = n.value
+                continue
+            check("xpl_page_summary", st)
+            return [{f: getattr(out[i], f) for f, _ in PAGE_REPORT_FIELDS if f != "pad"} for i in range(n.value)]
+
+    def page_flags(self, base, page_words, n_pages):
+        out = np.zeros(max(1, n_pages), dtype=np.uint8)
+        check("xpl_page_flags", xpl_page_flags(self.h, base, page_words, out.ctypes.data, n_pages))
+        return out[:n_pages]
+
+    def mem_advise(self, ptr, nbytes, advice, device=0):
+        check("xpl_mem_advise", xpl_mem_advise(self.h, ptr, nbytes, advice, device))
+
     def shadow_dump(self, base, word0, n):
         out = np.zeros(n, dtype=np.uint8)
         check("xpl_shadow_dump", xpl_shadow_dump(self.h, base, word0, n, out.ctypes.data))
@@ -297,6 +332,12 @@ class Context:
         """One cooperative launch of the replay kernel over nseg epochs separated by
         device-side epoch splits (xpl_grid_epoch); d_seg = nseg+1 event offsets."""
         check("xplw_replay_split", xplw_replay_split(d_addr, d_size, d_acc, d_seg, nseg, grid, block, stream))
+
+
+def atomic_bench(buf_ptr, n_u32, mode, stream=0):
+    """Launch the atomic-throughput microbenchmark kernel (libxplwork): one OR
+    per u32 of the device buffer; mode 0 RED, 1 ATOM, 2 same u32 per warp."""
+    check("xplw_atomic_bench", xplw_atomic_bench(buf_ptr, n_u32, mode, stream))
 
 
 def combine_partials(blobs, thr=50, block_words=0, min_run=256):

@@ -357,3 +357,35 @@ def test_device_epoch_split_random_traces(gpu):
     for seed in range(4):
         ops = random_trace(0x58504C30 + seed, n_allocs=5, n_steps=80, max_words=4000, p_device=0.9)
         assert replay.run_trace(ops, split_epochs=True) == oracle_run(ops)
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_page_view(gpu, seed):
+    """NEXT-3: the UM page view (xpl_page_summary, page sizes 1, 5, 16, 1024, huge)
+    and recorded cudaMemAdvise hints, bit-exact vs the oracle on random traces."""
+    replay, _ = gpu
+    from test_oracle_bruteforce import _with_pages
+    ops = _with_pages(random_trace(0x58504C60 + seed, n_allocs=6, n_steps=80, max_words=5000),
+                      (1, 5, 16, 1024, 1 << 40), seed)
+    compare(replay.run_trace(ops), oracle_run(ops), f"pages seed {seed}")
+
+
+def test_page_flags_map(gpu):
+    """xpl_page_flags: the per-page bits of one allocation equal the OR of the
+    per-word classes of its shadow dump (pages of 1000 words, ragged tail)."""
+    _, xpl = gpu
+    ops = random_trace(0x58504C66, n_allocs=3, n_steps=60, max_words=20000, p_device=0.9)
+    ops = [o for o in ops if o[0] != "DIAG"]
+    from paper_conf_ipps_pirkelbauerlvl20_b200 import replay
+    with xpl.Context(pool_words=1 << 22) as ctx:
+        replay.run_trace(ops, ctx=ctx)
+        for r in ctx.page_summary(1000):
+            f = ctx.page_flags(r["base"], 1000, r["pages"])
+            d = ctx.shadow_dump(r["base"], 0, r["words"])
+            for p in range(r["pages"]):
+                w = d[p * 1000:(p + 1) * 1000].astype(np.uint32)
+                cpu, gp = (w & 0x34) != 0, (w & 0xC8) != 0
+                e = (int(cpu.any()) | 2 * int(gp.any()) | 4 * int((cpu & gp).any()) |
+                     8 * int((cpu & gp & ((w & 0x0C) != 0)).any()) | 16 * int(((w & 4) != 0).any()) |
+                     32 * int(((w & 8) != 0).any()))
+                assert f[p] == e, (r["id"], p)

@@ -81,3 +81,53 @@ def test_lulesh_sampled_twin_equals_full_twin():
                 assert o1.peek(2 + k, w) == o2.peek(2 + k, w), (k, w)
     for w in range(L.DOM_BYTES // 4):
         assert o1.peek(0, w) == o2.peek(0, w)
+
+
+def _with_pages(ops, sizes, seed):
+    """Insert the UM page view before every diagnose (several page sizes) and
+    random cudaMemAdvise calls after registrations."""
+    import numpy as np
+    rng = np.random.default_rng(seed)
+    out = []
+    for op in ops:
+        if op[0] == "DIAG":
+            out += [("PAGES", int(P)) for P in sizes]
+        out.append(op)
+        if op[0] == "REG" and rng.random() < 0.6:
+            out.append(("ADVISE", op[1] + int(rng.integers(0, op[2])), 4, int(rng.integers(1, 7)),
+                        int(rng.choice([-1, 0]))))
+    return out
+
+
+def test_page_view_invariants():
+    """NEXT-3 page view tied to the (pinned) diagnose counters: with one word per
+    page the page counts are the per-word classes (gpu_pages = gpu_acc, CPU or
+    GPU pages = any_acc, alternating_pages = alternating); with one page per
+    allocation they are indicators of the same counters; false-shared pages
+    never exceed shared ones; flags only on managed allocations."""
+    from oracle import run_trace
+    from xplgen.trace import random_trace
+    for seed in range(12):
+        ops = _with_pages(random_trace(0x58504C40 + seed, n_allocs=5, n_steps=70, max_words=600),
+                          (1, 7, 1 << 40), seed)
+        res = run_trace(ops)
+        k = 0
+        while k < len(res):
+            p1, p7, pbig, diag = res[k:k + 4]
+            k += 4
+            live = {r["id"]: r for r in diag if r["live"]}
+            assert [r["id"] for r in p1] == sorted(live)
+            for a, b, c in zip(p1, p7, pbig):
+                d = live[a["id"]]
+                assert a["pages"] == d["words"] and c["pages"] == 1 and b["pages"] == -(-d["words"] // 7)
+                assert a["gpu_pages"] == d["gpu_acc"]
+                assert a["cpu_pages"] + a["gpu_pages"] - a["shared_pages"] == d["any_acc"]
+                assert a["alternating_pages"] == d["alternating"] and a["false_shared_pages"] == 0
+                assert c["gpu_pages"] == int(d["gpu_acc"] > 0) and c["alternating_pages"] == int(d["alternating"] > 0)
+                assert c["cpu_pages"] + c["gpu_pages"] - c["shared_pages"] == int(d["any_acc"] > 0)
+                for x in (a, b, c):
+                    assert x["false_shared_pages"] <= x["shared_pages"] <= min(x["cpu_pages"], x["gpu_pages"])
+                    assert x["alternating_pages"] <= x["shared_pages"] - x["false_shared_pages"]
+                    if d["kind"] != 1:
+                        assert x["flags"] == 0
+                    assert bool(x["flags"] & 1) == (d["kind"] == 1 and x["false_shared_pages"] > 0)

@@ -192,3 +192,28 @@ def test_oracle_cli(golden_dir):
                          capture_output=True, text=True, check=True).stdout
     row = json.loads(out.splitlines()[0])
     assert row["w_c"] == 4 and row["alternating"] == 2 and row["flags"] == 3
+
+
+def test_t19_pages(golden_dir):
+    """NEXT-3 page view, by hand from the definitions (T19's header)."""
+    p1024, p1, pbig, adv, adv2, diag, after = run(golden_dir, "T19_pages.trace")
+    FS, MISMATCH = 1, 2
+    check(p1024[0], pages=4, cpu_pages=2, gpu_pages=3, shared_pages=2, false_shared_pages=1,
+          alternating_pages=1, flags=FS, advice=0, words=3500, page_words=1024)
+    check(p1024[1], pages=2, cpu_pages=1, gpu_pages=1, shared_pages=1, false_shared_pages=1,
+          alternating_pages=0, flags=0)  # device: no page effects (P:L84)
+    # one word per page: the per-word classes (CPU words 10 + 1, GPU words 8 + 1 + 3)
+    check(p1[0], pages=3500, cpu_pages=11, gpu_pages=12, shared_pages=1, false_shared_pages=0,
+          alternating_pages=1, flags=0)
+    # one page for the whole allocation
+    check(pbig[0], pages=1, cpu_pages=1, gpu_pages=1, shared_pages=1, false_shared_pages=0,
+          alternating_pages=1, flags=0)
+    # ReadMostly advised while a page alternates (P:L47, P:L86)
+    check(adv[0], advice=1, flags=FS | MISMATCH)
+    # unset ReadMostly; PreferredLocation = CPU (device -1); AccessedBy GPU on B
+    check(adv2[0], advice=4, flags=FS)
+    check(adv2[1], advice=8, flags=0)
+    # the resetting diagnose clears the interval: no page is used any more
+    check(after[0], cpu_pages=0, gpu_pages=0, shared_pages=0, false_shared_pages=0, alternating_pages=0,
+          advice=4, flags=0)
+    assert diag[0]["alternating"] == 1 and diag[0]["any_acc"] == 10 + 1 + 8 + 3

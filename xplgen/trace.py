@@ -50,6 +50,10 @@ def to_text(ops) -> str:
         elif t == "DIAG":
             names = " ".join(f"{a:#x}" for a in op[5])
             out.append(f"DIAG {op[1]} {op[2]} {op[3]} {op[4]} {names}".rstrip())
+        elif t == "PAGES":
+            out.append(f"PAGES {op[1]}")
+        elif t == "ADVISE":
+            out.append(f"ADVISE {op[1]:#x} {op[2]} {op[3]} {op[4]}")
         else:
             raise ValueError(op)
     return "\n".join(out) + "\n"
@@ -78,6 +82,10 @@ def parse_text(text: str):
             ops.append(("X", n(t[1]), n(t[2]), n(t[3]), n(t[4])))
         elif t[0] == "DIAG":
             ops.append(("DIAG", n(t[1]), n(t[2]), n(t[3]), n(t[4]), tuple(n(x) for x in t[5:])))
+        elif t[0] == "PAGES":  # the UM page view of the live rows (NEXT-3)
+            ops.append(("PAGES", n(t[1])))
+        elif t[0] == "ADVISE":  # cudaMemAdvise: ptr bytes advice(1..6) device(-1 = CPU)
+            ops.append(("ADVISE", n(t[1]), n(t[2]), n(t[3]), n(t[4])))
         else:
             raise ValueError(line)
     return ops
