@@ -311,6 +311,52 @@ xpl_status xpl_page_flags(xpl_ctx* ctx, const void* base, uint64_t page_words, u
  * Untracked pointers are ignored.  INVALID_ARG on another advice value. */
 xpl_status xpl_mem_advise(xpl_ctx* ctx, const void* ptr, size_t bytes, int advice, int device);
 
+/* ---- Kernel-launch log (traceKernelLaunch) ----
+ * The paper's launch wrapper "can be used to ... record data before and after
+ * the launch of a CUDA kernel".  With the log on, every launch the
+ * instrumented code reports inside an epoch (xpl_kernel_launch, or the
+ * xpl_trace_kernel_launch template of xpl_launch.cuh) is kept with its launch
+ * parameters, and every epoch gets two measurements taken on the device, in
+ * stream order, without synchronising the host: its GPU time (CUDA events from
+ * the epoch's begin on its first stream to the end of its fold) and the number
+ * of 128-word shadow chunks its fold found GPU-written (the epoch's write
+ * footprint).  Off by default; costs two event records and one 8-byte
+ * device->host copy per epoch when on. */
+typedef struct {
+  const char* name; /* kernel name; copied (interned) by the runtime, may be NULL */
+  uint32_t grid[3], block[3];
+  uint32_t shmem; /* dynamic shared memory bytes */
+} xpl_launch_info;
+
+typedef struct {
+  uint64_t seq;         /* launch number since the log was enabled/reset (0-based)   */
+  uint64_t epoch;       /* epoch number (xpl_stats.epochs counted at its begin)      */
+  uint64_t stream;      /* cudaStream_t of the launch, as an integer                 */
+  uint32_t grid[3], block[3];
+  uint32_t shmem, name_idx; /* name_idx: xpl_launch_name(), UINT32_MAX = none        */
+  uint64_t threads;         /* grid x block                                          */
+  uint64_t launches_in_epoch;
+  uint64_t epoch_written_chunks; /* 128-word chunks the epoch's fold saw written     */
+  double epoch_ms;               /* GPU time of the epoch incl. its fold, -1 if n/a  */
+} xpl_launch_record;
+
+/* Turn the log on (1) or off (0).  Turning it on clears it.  STATE inside an
+ * open epoch. */
+xpl_status xpl_launch_log_enable(xpl_ctx* ctx, int enable);
+/* Log one launch of the open epoch (call between xpl_kernel_begin and _end,
+ * before or after the launch itself).  STATE outside an epoch; INVALID_ARG on
+ * a NULL info; a no-op when the log is off. */
+xpl_status xpl_kernel_launch(xpl_ctx* ctx, void* stream, const xpl_launch_info* info);
+/* The logged launches in order into out[0..cap) (*n_out records; INVALID_ARG
+ * with *n_out = records needed if cap is too small).  Waits for the logged
+ * epochs' events and copies.  reset != 0 clears the log after reading.  STATE
+ * inside an open epoch. */
+xpl_status xpl_launch_log(xpl_ctx* ctx, xpl_launch_record* out, size_t cap, size_t* n_out,
+                          int reset);
+/* The interned kernel name with index idx (owned by the context, valid until
+ * xpl_finalize); NULL if idx is out of range. */
+const char* xpl_launch_name(xpl_ctx* ctx, uint32_t idx);
+
 /* Apply every staged host record now (normally done lazily at kernel_begin,
  * diagnose and when staging fills up).  Asynchronous. */
 xpl_status xpl_flush(xpl_ctx* ctx);

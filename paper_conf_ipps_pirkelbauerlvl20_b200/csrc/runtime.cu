@@ -12,6 +12,8 @@
 #include <algorithm>
 #include <map>
 #include <new>
+#include <string>
+#include <unordered_map>
 #include <vector>
 
 #include "xpl_internal.h"
@@ -172,6 +174,22 @@ struct xpl_ctx {
   xpl_kernel_time prof_acc[XPL_K_NCLASS];
   unsigned long long fold_entries_seen = 0;
   uint64_t folds_host = 0;
+
+  // kernel-launch log (NEXT-4)
+  struct EpochRec {
+    cudaEvent_t a = nullptr, b = nullptr;  // begin on the epoch's first stream / after its fold
+    bool timed = false;
+  };
+  bool llog = false;
+  std::vector<xpl_launch_record> lrecs;
+  std::vector<EpochRec> lepochs;           // logged epochs, in order
+  std::vector<uint64_t> lepoch_no;         // their epoch numbers
+  std::vector<cudaEvent_t> lev_free;
+  unsigned long long* h_lcum = nullptr;    // pinned: d_stats[3] (folded chunks) after each logged fold
+  size_t lcum_cap = 0;
+  bool lepoch_open = false;                // the open epoch has a log entry
+  std::vector<std::string> lnames;
+  std::unordered_map<std::string, uint32_t> lname_idx;
 };
 
 namespace {
@@ -510,9 +528,136 @@ xpl_status join(xpl_ctx* c, cudaStream_t s) {
   return XPL_OK;
 }
 
+// ---- kernel-launch log (NEXT-4) -------------------------------------
+cudaEvent_t log_event(xpl_ctx* c) {
+  if (!c->lev_free.empty()) {
+    cudaEvent_t e = c->lev_free.back();
+    c->lev_free.pop_back();
+    return e;
+  }
+  cudaEvent_t e = nullptr;
+  if (cudaEventCreate(&e) != cudaSuccess) return nullptr;
+  return e;
+}
+
+void log_clear(xpl_ctx* c) {
+  for (auto& r : c->lepochs) {
+    if (r.a) c->lev_free.push_back(r.a);
+    if (r.b) c->lev_free.push_back(r.b);
+  }
+  c->lepochs.clear();
+  c->lepoch_no.clear();
+  c->lrecs.clear();
+}
+
+// Open the log entry of the epoch beginning on stream s (after s joined the
+// runtime's pending work): begin event + the folded-chunk counter before it.
+xpl_status log_epoch_begin(xpl_ctx* c, cudaStream_t s) {
+  const size_t i = c->lepochs.size();
+  if (2 * (i + 1) > c->lcum_cap) {  // grow the pinned snapshot array (rare: doubling)
+    const size_t cap = c->lcum_cap ? 2 * c->lcum_cap : 8192;
+    unsigned long long* h = nullptr;
+    CK(cudaDeviceSynchronize());  // pending snapshot copies target the old array
+    CK(cudaMallocHost((void**)&h, cap * sizeof(unsigned long long)));
+    if (c->h_lcum) {
+      memcpy(h, c->h_lcum, c->lcum_cap * sizeof(unsigned long long));
+      cudaFreeHost(c->h_lcum);
+    }
+    c->h_lcum = h;
+    c->lcum_cap = cap;
+  }
+  xpl_ctx::EpochRec r;
+  r.a = log_event(c);
+  r.b = log_event(c);
+  if (!r.a || !r.b) return XPL_ERR_CUDA;
+  r.timed = true;
+  CK(cudaMemcpyAsync(c->h_lcum + 2 * i, c->d_stats + 3, sizeof(unsigned long long),
+                     cudaMemcpyDeviceToHost, s));
+  CK(cudaEventRecord(r.a, s));
+  c->lepochs.push_back(r);
+  c->lepoch_no.push_back(c->st.epochs);
+  c->lepoch_open = true;
+  return XPL_OK;
+}
+
 }  // namespace
 
 extern "C" {
+
+xpl_status xpl_launch_log_enable(xpl_ctx* c, int enable) {
+  if (!c) return XPL_ERR_INVALID_ARG;
+  if (c->depth) return XPL_ERR_STATE;
+  CK(cudaDeviceSynchronize());  // pending snapshot copies / events of the old log
+  log_clear(c);
+  c->llog = enable != 0;
+  return XPL_OK;
+}
+
+xpl_status xpl_kernel_launch(xpl_ctx* c, void* stream, const xpl_launch_info* li) {
+  if (!c || !li) return XPL_ERR_INVALID_ARG;
+  if (!c->depth) return XPL_ERR_STATE;
+  if (!c->llog) return XPL_OK;
+  xpl_launch_record r;
+  memset(&r, 0, sizeof r);
+  r.seq = c->lrecs.size();
+  r.epoch = c->st.epochs;
+  r.stream = (uint64_t)stream;
+  for (int k = 0; k < 3; ++k) {
+    r.grid[k] = li->grid[k];
+    r.block[k] = li->block[k];
+  }
+  r.shmem = li->shmem;
+  r.threads = (uint64_t)li->grid[0] * li->grid[1] * li->grid[2] * li->block[0] * li->block[1] * li->block[2];
+  r.name_idx = UINT32_MAX;
+  if (li->name) {
+    auto it = c->lname_idx.find(li->name);
+    if (it == c->lname_idx.end()) {
+      it = c->lname_idx.emplace(li->name, (uint32_t)c->lnames.size()).first;
+      c->lnames.push_back(li->name);
+    }
+    r.name_idx = it->second;
+  }
+  r.epoch_ms = -1.0;
+  c->lrecs.push_back(r);
+  return XPL_OK;
+}
+
+xpl_status xpl_launch_log(xpl_ctx* c, xpl_launch_record* out, size_t cap, size_t* n_out, int reset) {
+  if (!c || !n_out || (cap && !out)) return XPL_ERR_INVALID_ARG;
+  if (c->depth) return XPL_ERR_STATE;
+  *n_out = c->lrecs.size();
+  if (cap < c->lrecs.size()) return XPL_ERR_INVALID_ARG;
+  // per logged epoch: GPU time and written chunks (waits for its events / copies)
+  std::unordered_map<uint64_t, size_t> at;
+  std::vector<double> ms(c->lepochs.size(), -1.0);
+  std::vector<uint64_t> chunks(c->lepochs.size(), 0), nl(c->lepochs.size(), 0);
+  for (size_t i = 0; i < c->lepochs.size(); ++i) {
+    at[c->lepoch_no[i]] = i;
+    CK(cudaEventSynchronize(c->lepochs[i].b));
+    float f = 0.f;
+    if (cudaEventElapsedTime(&f, c->lepochs[i].a, c->lepochs[i].b) == cudaSuccess) ms[i] = f;
+    chunks[i] = c->h_lcum[2 * i + 1] - c->h_lcum[2 * i];
+  }
+  for (const auto& r : c->lrecs) {
+    auto it = at.find(r.epoch);
+    if (it != at.end()) nl[it->second]++;
+  }
+  for (size_t k = 0; k < c->lrecs.size(); ++k) {
+    out[k] = c->lrecs[k];
+    auto it = at.find(out[k].epoch);
+    if (it == at.end()) continue;
+    out[k].epoch_ms = ms[it->second];
+    out[k].epoch_written_chunks = chunks[it->second];
+    out[k].launches_in_epoch = nl[it->second];
+  }
+  if (reset) log_clear(c);
+  return XPL_OK;
+}
+
+const char* xpl_launch_name(xpl_ctx* c, uint32_t idx) {
+  if (!c || idx >= c->lnames.size()) return nullptr;
+  return c->lnames[idx].c_str();
+}
 
 // ---- UM page view (NEXT-3; D31-D33) ----------------------
 static xpl_status page_pass(xpl_ctx* c, const std::vector<const Row*>& rows, uint64_t P,
@@ -727,6 +872,12 @@ xpl_status xpl_finalize(xpl_ctx* c) {
   cudaFreeHost(c->h_cnt);
   for (cudaEvent_t e : c->ev_pool) cudaEventDestroy(e);
   for (cudaEvent_t e : c->prof_free) cudaEventDestroy(e);
+  for (cudaEvent_t e : c->lev_free) cudaEventDestroy(e);
+  for (auto& r : c->lepochs) {
+    if (r.a) cudaEventDestroy(r.a);
+    if (r.b) cudaEventDestroy(r.b);
+  }
+  cudaFreeHost(c->h_lcum);
   for (auto& r : c->prof_pending) {
     cudaEventDestroy(r.a);
     cudaEventDestroy(r.b);
@@ -830,6 +981,10 @@ xpl_status xpl_kernel_begin(xpl_ctx* c, void* stream) {
     }
     c->epoch_streams.push_back(s);
   }
+  if (c->llog && !c->lepoch_open) {  // NEXT-4: the epoch starts on its first stream
+    xpl_status st = log_epoch_begin(c, s);
+    if (st) return st;
+  }
   c->depth++;
   return XPL_OK;
 }
@@ -866,6 +1021,13 @@ xpl_status xpl_kernel_end(xpl_ctx* c, void* stream) {
   }
   c->cs = t;
   fold(c, !crossed);
+  if (c->lepoch_open) {  // NEXT-4: after the fold, on its stream
+    const size_t i = c->lepochs.size() - 1;
+    CK(cudaEventRecord(c->lepochs[i].b, c->cs));
+    CK(cudaMemcpyAsync(c->h_lcum + 2 * i + 1, c->d_stats + 3, sizeof(unsigned long long),
+                       cudaMemcpyDeviceToHost, c->cs));
+    c->lepoch_open = false;
+  }
   if (cudaGetLastError() != cudaSuccess) return XPL_ERR_CUDA;
   std::vector<uint64_t> q;
   q.swap(c->deferred);

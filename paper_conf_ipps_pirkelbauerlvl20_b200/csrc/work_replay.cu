@@ -8,6 +8,7 @@
 
 #include "xpl.h"
 #include "xpl_device.cuh"
+#include "xpl_launch.cuh"
 
 namespace {
 
@@ -85,9 +86,34 @@ __global__ void atomic_bench_kernel(unsigned* p, unsigned long long n, int mode,
   if (mode == 1 && acc == 0x9E3779B9u) *sink = acc;  // keep the return values live
 }
 
+// A user kernel that really touches memory (managed memory for the UM-counter
+// check, NEXT-4): word k*stride of base for k < n/stride is read (write = 0) or
+// incremented (write = 1: read then write, hooked as RW), hooks on.
+__global__ void touch_mem_kernel(unsigned* base, unsigned long long n, unsigned long long stride, int write,
+                                 unsigned* sink) {
+  unsigned acc = 0;
+  for (unsigned long long k = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; k * stride < n;
+       k += (unsigned long long)gridDim.x * blockDim.x) {
+    unsigned& w = base[k * stride];
+    if (write) xpl_rw(w) += 1u;
+    else acc ^= xpl_read(w);
+  }
+  if (acc == 0x9E3779B9u) *sink = acc;
+}
+
 }  // namespace
 
 extern "C" {
+
+// Launch touch_mem_kernel on `stream` (between xpl_kernel_begin/_end).
+int xplw_touch_mem(void* base, unsigned long long n_words, unsigned long long stride, int write, void* stream) {
+  if (!stride || !n_words) return 0;
+  const unsigned long long m = (n_words + stride - 1) / stride;
+  const unsigned g = (unsigned)(m < 148ull * 8 * 256 ? (m + 255) / 256 : 148 * 8);
+  touch_mem_kernel<<<g, 256, 0, (cudaStream_t)stream>>>((unsigned*)base, n_words, stride, write,
+                                                        (unsigned*)base);
+  return cudaGetLastError() == cudaSuccess ? 0 : (int)XPL_ERR_CUDA;
+}
 
 int xplw_atomic_bench(void* buf, unsigned long long n_u32, int mode, void* stream) {
   atomic_bench_kernel<<<148 * 16, 256, 0, (cudaStream_t)stream>>>((unsigned*)buf, n_u32, mode,
@@ -126,6 +152,19 @@ int xplw_replay(const unsigned long long* d_addr, const unsigned int* d_size,
   if (n == 0) return 0;
   replay_kernel<<<grid, block, 0, (cudaStream_t)stream>>>(d_addr, d_size, d_acc, n);
   return cudaGetLastError() == cudaSuccess ? 0 : (int)XPL_ERR_CUDA;
+}
+
+// The same launch through the kernel-launch wrapper (traceKernelLaunch, P:L227;
+// NEXT-4): opens (or nests into) an epoch on `stream`, logs the launch, closes it.
+int xplw_replay_traced(xpl_ctx* ctx, const unsigned long long* d_addr, const unsigned int* d_size,
+                       const unsigned char* d_acc, unsigned long long n, int grid, int block,
+                       void* stream) {
+  xpl_status st = XPL_OK;
+  const cudaError_t e = xpl_trace_kernel_launch_st(ctx, &st, "replay_kernel", dim3(grid), dim3(block), 0,
+                                                   (cudaStream_t)stream, replay_kernel, d_addr, d_size,
+                                                   d_acc, n);
+  if (st != XPL_OK) return (int)st;
+  return e == cudaSuccess ? 0 : (int)XPL_ERR_CUDA;
 }
 
 // One cooperative launch replaying nseg epochs (between one xpl_kernel_begin/_end);

@@ -119,9 +119,15 @@ struct App {
       if (dir == XPL_COPY_D2H) ok_cuda(cudaStreamSynchronize(s));  // cudaMemcpy semantics
     }
   }
-  void begin() {
+  // epoch around one launch; the launch parameters go to the runtime's launch
+  // log (xpl_kernel_launch: a no-op unless the log is on; NEXT-4)
+  void begin(const char* name, dim3 grd, dim3 blk) {
     flush();
-    if (on()) ok(xpl_kernel_begin(run->ctx, s));
+    if (on()) {
+      ok(xpl_kernel_begin(run->ctx, s));
+      const xpl_launch_info li = {name, {grd.x, grd.y, grd.z}, {blk.x, blk.y, blk.z}, 0};
+      ok(xpl_kernel_launch(run->ctx, s, &li));
+    }
     mark();
   }
   void end() {
@@ -415,7 +421,7 @@ int xplw_hotspot(xplw_run* run, const xplw_arrays* a, int R, int C, int iters) {
   const dim3 blk(32, 8), grd((C + 31) / 32, (R + 7) / 8);
   int src = 0;
   for (int it = 0; it < iters; ++it) {
-    app.begin();
+    app.begin("hotspot_kernel", grd, blk);
     if (app.on())
       hotspot_kernel<true><<<grd, blk, 0, app.s>>>(d_power, d_temp[src], d_temp[1 - src], R, C, 0.5f, 0.1f, 0.1f, 0.01f, 80.f);
     else
@@ -449,7 +455,7 @@ int xplw_backprop(xplw_run* run, const xplw_arrays* a, int in, int hid) {
   app.copy(input_cuda, input_units, (in + 1) * 4, XPL_COPY_H2D);
   app.copy(input_hidden_cuda, input_weights, nw * 4, XPL_COPY_H2D);
   const dim3 blk(BP, BP), grd(nblk);
-  app.begin();
+  app.begin("bp_layerforward", grd, blk);
   if (app.on()) bp_layerforward<true><<<grd, blk, 0, app.s>>>(input_cuda, input_hidden_cuda, hidden_partial_sum, hid);
   else bp_layerforward<false><<<grd, blk, 0, app.s>>>(input_cuda, input_hidden_cuda, hidden_partial_sum, hid);
   app.end();
@@ -460,7 +466,7 @@ int xplw_backprop(xplw_run* run, const xplw_arrays* a, int in, int hid) {
   app.write_loop(hidden_delta, hid + 1);
   app.copy(hidden_delta_cuda, hidden_delta, (hid + 1) * 4, XPL_COPY_H2D);
   app.copy(input_prev_weights_cuda, prev_weights, nw * 4, XPL_COPY_H2D);
-  app.begin();
+  app.begin("bp_adjust", grd, blk);
   if (app.on()) bp_adjust<true><<<grd, blk, 0, app.s>>>(hidden_delta_cuda, input_cuda, input_hidden_cuda, input_prev_weights_cuda, hid);
   else bp_adjust<false><<<grd, blk, 0, app.s>>>(hidden_delta_cuda, input_cuda, input_hidden_cuda, input_prev_weights_cuda, hid);
   app.end();
@@ -526,11 +532,11 @@ int xplw_bfs(xplw_run* run, const xplw_arrays* a, int n, int deg, unsigned long 
     app.copy(d_over, h_over, 1, XPL_COPY_H2D);
     if (!run->do_copies)  // control data: the loop needs it even when bulk data is resident
       app.ok_cuda(cudaMemcpyAsync(d_over, h_over, 1, cudaMemcpyHostToDevice, app.s));
-    app.begin();
+    app.begin("bfs_kernel1", dim3(blocks), dim3(512));
     if (app.on()) bfs_kernel1<true><<<blocks, 512, 0, app.s>>>(d_nodes, d_edges, d_mask, d_updating, d_visited, d_cost, n, hook_count);
     else bfs_kernel1<false><<<blocks, 512, 0, app.s>>>(d_nodes, d_edges, d_mask, d_updating, d_visited, d_cost, n, hook_count);
     app.end();
-    app.begin();
+    app.begin("bfs_kernel2", dim3(blocks), dim3(512));
     if (app.on()) bfs_kernel2<true><<<blocks, 512, 0, app.s>>>(d_mask, d_updating, d_visited, d_over, n, hook_count);
     else bfs_kernel2<false><<<blocks, 512, 0, app.s>>>(d_mask, d_updating, d_visited, d_over, n, hook_count);
     app.end();
@@ -570,14 +576,14 @@ int xplw_nw(xplw_run* run, const xplw_arrays* a, int n, int penalty, const int* 
   app.copy(mat_d, in, sizeof(int) * rows * cols, XPL_COPY_H2D);
   const int bw = (cols - 1) / NWB;
   for (int i = 1; i <= bw; i++) {
-    app.begin();
+    app.begin("nw_kernel_upper", dim3(i), dim3(NWB));
     if (app.on()) nw_kernel<true, true><<<i, NWB, 0, app.s>>>(ref_d, mat_d, cols, penalty, i, bw);
     else nw_kernel<false, true><<<i, NWB, 0, app.s>>>(ref_d, mat_d, cols, penalty, i, bw);
     app.end();
     run->dev_accesses += (uint64_t)i * (1 + 2 * NWB * NWB + 2 * NWB);
   }
   for (int i = bw - 1; i >= 1; i--) {
-    app.begin();
+    app.begin("nw_kernel_lower", dim3(i), dim3(NWB));
     if (app.on()) nw_kernel<true, false><<<i, NWB, 0, app.s>>>(ref_d, mat_d, cols, penalty, i, bw);
     else nw_kernel<false, false><<<i, NWB, 0, app.s>>>(ref_d, mat_d, cols, penalty, i, bw);
     app.end();

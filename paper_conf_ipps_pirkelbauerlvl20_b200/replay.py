@@ -66,12 +66,14 @@ def _dev_arrays(evs):
 
 
 def run_trace(ops, ctx: Context | None = None, grid=0, block=256, seed=None, host_split=None,
-              pool_words=1 << 24, stream=None, split_epochs=False):
+              pool_words=1 << 24, stream=None, split_epochs=False, traced=False):
     """Replay `ops`.  seed: shuffle device events inside every epoch and split
     host batches at random points (metamorphic variants); grid/block: launch
     shape of the replay kernel (grid 0 = enough CTAs for one event each);
     split_epochs: chains of consecutive epochs run as one cooperative launch
-    with device-side epoch splits (xpl_grid_epoch) -- must give the same reports."""
+    with device-side epoch splits (xpl_grid_epoch) -- must give the same reports;
+    traced: device events are launched through the kernel-launch wrapper
+    (xpl_trace_kernel_launch, nested into the trace's epoch) -- same reports."""
     import torch
 
     if split_epochs:
@@ -113,7 +115,8 @@ def run_trace(ops, ctx: Context | None = None, grid=0, block=256, seed=None, hos
         ta = torch.from_numpy(a.view(np.int64)).cuda()
         ts = torch.from_numpy(s.view(np.int32)).cuda()
         tk = torch.from_numpy(k).cuda()
-        ctx.replay(ta.data_ptr(), ts.data_ptr(), tk.data_ptr(), a.size, grid=grid, block=block, stream=stream)
+        (ctx.replay_traced if traced else ctx.replay)(ta.data_ptr(), ts.data_ptr(), tk.data_ptr(), a.size,
+                                                      grid=grid, block=block, stream=stream)
         torch.cuda.current_stream().synchronize()  # keep the temporaries alive until the launch ran
 
     for op in ops:

@@ -123,6 +123,24 @@ class XplPageReport(C.Structure):
 xpl_page_summary = _sig("xpl_page_summary", [vp, u64, C.POINTER(XplPageReport), sz, C.POINTER(sz)])
 xpl_page_flags = _sig("xpl_page_flags", [vp, vp, u64, vp, u64])
 xpl_mem_advise = _sig("xpl_mem_advise", [vp, vp, sz, i32, i32])
+
+
+class XplLaunchInfo(C.Structure):
+    _fields_ = [("name", C.c_char_p), ("grid", u32 * 3), ("block", u32 * 3), ("shmem", u32)]
+
+
+class XplLaunchRecord(C.Structure):
+    _fields_ = [("seq", u64), ("epoch", u64), ("stream", u64), ("grid", u32 * 3), ("block", u32 * 3),
+                ("shmem", u32), ("name_idx", u32), ("threads", u64), ("launches_in_epoch", u64),
+                ("epoch_written_chunks", u64), ("epoch_ms", C.c_double)]
+
+
+xpl_launch_log_enable = _sig("xpl_launch_log_enable", [vp, i32])
+xpl_kernel_launch = _sig("xpl_kernel_launch", [vp, vp, C.POINTER(XplLaunchInfo)])
+xpl_launch_log = _sig("xpl_launch_log", [vp, C.POINTER(XplLaunchRecord), sz, C.POINTER(sz), i32])
+xpl_launch_name = _lib.xpl_launch_name
+xpl_launch_name.argtypes = [vp, u32]
+xpl_launch_name.restype = C.c_char_p
 xpl_flush = _sig("xpl_flush", [vp])
 xpl_sync = _sig("xpl_sync", [vp])
 xpl_join = _sig("xpl_join", [vp, vp])
@@ -144,11 +162,13 @@ EXPORTED = ["xpl_init", "xpl_finalize", "xpl_register_alloc", "xpl_free", "xpl_k
             "xpl_get_device_ctx", "xpl_shadow_dump", "xpl_flush", "xpl_sync", "xpl_join",
             "xpl_runtime_stream", "xpl_get_stats", "xpl_status_string", "xpl_profile",
             "xpl_profile_read", "xpl_register_alloc_piece", "xpl_diagnose_partials", "xpl_combine_partials",
-            "xpl_format_reports", "xpl_page_summary", "xpl_page_flags", "xpl_mem_advise"]
+            "xpl_format_reports", "xpl_page_summary", "xpl_page_flags", "xpl_mem_advise",
+            "xpl_launch_log_enable", "xpl_kernel_launch", "xpl_launch_log", "xpl_launch_name"]
 
 if _work is not None:
     xplw_bind = _sig("xplw_bind", [vp], lib=_work)
     xplw_replay = _sig("xplw_replay", [vp, vp, vp, u64, i32, i32, vp], lib=_work)
+    xplw_replay_traced = _sig("xplw_replay_traced", [vp, vp, vp, vp, u64, i32, i32, vp], lib=_work)
     xplw_replay_split = _sig("xplw_replay_split", [vp, vp, vp, vp, i32, i32, i32, vp], lib=_work)
     xplw_atomic_bench = _sig("xplw_atomic_bench", [vp, u64, i32, vp], lib=_work)
     xplw_touch = _sig("xplw_touch", [u64, u64, u32, vp, u64], lib=_work)
@@ -277,6 +297,44 @@ class Context:
 
     def mem_advise(self, ptr, nbytes, advice, device=0):
         check("xpl_mem_advise", xpl_mem_advise(self.h, ptr, nbytes, advice, device))
+
+    def launch_log_enable(self, enable=True):
+        check("xpl_launch_log_enable", xpl_launch_log_enable(self.h, int(bool(enable))))
+
+    def kernel_launch(self, stream, name, grid, block, shmem=0):
+        """Log one launch of the open epoch (xpl_kernel_launch)."""
+        g = tuple(grid) + (1,) * (3 - len(grid))
+        b = tuple(block) + (1,) * (3 - len(block))
+        li = XplLaunchInfo(name.encode() if name is not None else None, (u32 * 3)(*g), (u32 * 3)(*b), shmem)
+        check("xpl_kernel_launch", xpl_kernel_launch(self.h, stream, C.byref(li)))
+
+    def launch_log(self, reset=True):
+        """The launch log (xpl_launch_log) as dicts, names resolved."""
+        cap = 256
+        while True:
+            out = (XplLaunchRecord * cap)()
+            n = sz(0)
+            st = xpl_launch_log(self.h, out, cap, C.byref(n), int(bool(reset)))
+            if st == 1 and n.value > cap:
+                cap = n.value
+                continue
+            check("xpl_launch_log", st)
+            res = []
+            for i in range(n.value):
+                r = out[i]
+                d = {f: getattr(r, f) for f, _ in XplLaunchRecord._fields_}
+                d["grid"], d["block"] = tuple(r.grid), tuple(r.block)
+                nm = xpl_launch_name(self.h, r.name_idx)
+                d["name"] = nm.decode() if nm is not None else None
+                res.append(d)
+            return res
+
+    def replay_traced(self, d_addr, d_size, d_acc, n, grid=0, block=256, stream=0):
+        """The replay kernel launched through the kernel-launch wrapper
+        (xpl_trace_kernel_launch: its own or a nested epoch, logged)."""
+        if grid <= 0:
+            grid = max(1, min((n + block - 1) // block, 148 * 8))
+        check("xplw_replay_traced", xplw_replay_traced(self.h, d_addr, d_size, d_acc, n, grid, block, stream))
 
     def shadow_dump(self, base, word0, n):
         out = np.zeros(n, dtype=np.uint8)

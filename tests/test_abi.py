@@ -61,3 +61,22 @@ def test_init_fails_loudly_without_gpu():
     from paper_conf_ipps_pirkelbauerlvl20_b200 import xpl
     with pytest.raises(xpl.XplError):
         xpl.Context()
+
+
+def test_binding_struct_layouts_match_the_header(tmp_path):
+    """sizeof / offsetof of the report structs added for NEXT-3 / NEXT-4, as the C
+    compiler lays them out from include/xpl.h, equal the ctypes mirrors."""
+    import subprocess
+    from paper_conf_ipps_pirkelbauerlvl20_b200 import xpl
+    src = tmp_path / "lay.c"
+    src.write_text('#include <stdio.h>\n#include <stddef.h>\n#include "xpl.h"\nint main(void){\n'
+                   'printf("%zu %zu %zu %zu %zu %zu\\n", sizeof(xpl_page_report), offsetof(xpl_page_report, flags),'
+                   ' sizeof(xpl_launch_record), offsetof(xpl_launch_record, epoch_ms),'
+                   ' sizeof(xpl_launch_info), offsetof(xpl_launch_info, shmem));\nreturn 0;}\n')
+    exe = tmp_path / "lay"
+    subprocess.run(["gcc", "-I", os.path.join(ROOT, "include"), str(src), "-o", str(exe)], check=True)
+    got = [int(x) for x in subprocess.run([str(exe)], capture_output=True, text=True, check=True).stdout.split()]
+    exp = [ctypes.sizeof(xpl.XplPageReport), xpl.XplPageReport.flags.offset,
+           ctypes.sizeof(xpl.XplLaunchRecord), xpl.XplLaunchRecord.epoch_ms.offset,
+           ctypes.sizeof(xpl.XplLaunchInfo), xpl.XplLaunchInfo.shmem.offset]
+    assert got == exp

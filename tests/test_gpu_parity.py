@@ -364,8 +364,8 @@ def test_page_view(gpu, seed):
     """NEXT-3: the UM page view (xpl_page_summary, page sizes 1, 5, 16, 1024, huge)
     and recorded cudaMemAdvise hints, bit-exact vs the oracle on random traces."""
     replay, _ = gpu
-    from test_oracle_bruteforce import _with_pages
-    ops = _with_pages(random_trace(0x58504C60 + seed, n_allocs=6, n_steps=80, max_words=5000),
+    from xplgen.trace import with_pages
+    ops = with_pages(random_trace(0x58504C60 + seed, n_allocs=6, n_steps=80, max_words=5000),
                       (1, 5, 16, 1024, 1 << 40), seed)
     compare(replay.run_trace(ops), oracle_run(ops), f"pages seed {seed}")
 

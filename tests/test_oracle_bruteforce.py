@@ -83,22 +83,6 @@ def test_lulesh_sampled_twin_equals_full_twin():
         assert o1.peek(0, w) == o2.peek(0, w)
 
 
-def _with_pages(ops, sizes, seed):
-    """Insert the UM page view before every diagnose (several page sizes) and
-    random cudaMemAdvise calls after registrations."""
-    import numpy as np
-    rng = np.random.default_rng(seed)
-    out = []
-    for op in ops:
-        if op[0] == "DIAG":
-            out += [("PAGES", int(P)) for P in sizes]
-        out.append(op)
-        if op[0] == "REG" and rng.random() < 0.6:
-            out.append(("ADVISE", op[1] + int(rng.integers(0, op[2])), 4, int(rng.integers(1, 7)),
-                        int(rng.choice([-1, 0]))))
-    return out
-
-
 def test_page_view_invariants():
     """NEXT-3 page view tied to the (pinned) diagnose counters: with one word per
     page the page counts are the per-word classes (gpu_pages = gpu_acc, CPU or
@@ -106,9 +90,9 @@ def test_page_view_invariants():
     allocation they are indicators of the same counters; false-shared pages
     never exceed shared ones; flags only on managed allocations."""
     from oracle import run_trace
-    from xplgen.trace import random_trace
+    from xplgen.trace import random_trace, with_pages
     for seed in range(12):
-        ops = _with_pages(random_trace(0x58504C40 + seed, n_allocs=5, n_steps=70, max_words=600),
+        ops = with_pages(random_trace(0x58504C40 + seed, n_allocs=5, n_steps=70, max_words=600),
                           (1, 7, 1 << 40), seed)
         res = run_trace(ops)
         k = 0

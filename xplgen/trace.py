@@ -262,3 +262,19 @@ def epoch_chain_trace(seed, n_allocs=4, n_chains=3, chain_len=6, max_words=20000
                     int(rng.choice([1, 4, 256])), int(rng.random() < 0.7), ()))
     ops.append(("DIAG", 50, 0, 4, 1, ()))
     return ops
+
+
+def with_pages(ops, sizes, seed):
+    """Insert the UM page view before every diagnose (several page sizes) and
+    random cudaMemAdvise calls after registrations."""
+    import numpy as np
+    rng = np.random.default_rng(seed)
+    out = []
+    for op in ops:
+        if op[0] == "DIAG":
+            out += [("PAGES", int(P)) for P in sizes]
+        out.append(op)
+        if op[0] == "REG" and rng.random() < 0.6:
+            out.append(("ADVISE", op[1] + int(rng.integers(0, op[2])), 4, int(rng.integers(1, 7)),
+                        int(rng.choice([-1, 0]))))
+    return out
