@@ -522,6 +522,21 @@ def main():
     bt = step(None, False, time_kernels=True)
     torch.cuda.synchronize()
 
+    # --- launch log of one untimed step (NEXT-4): per kernel, its epochs' GPU
+    # time (incl. fold) and write footprint, measured in stream order ----------
+    prepare(False)
+    ctx.launch_log_enable(True)
+    step(ctx, False)
+    llog = ctx.launch_log(reset=True)
+    ctx.launch_log_enable(False)
+    launch_log = {}
+    for r in llog:
+        k = launch_log.setdefault(r["name"], {"launches": 0, "epoch_ms_sum": 0.0, "written_chunks": 0,
+                                              "grid_example": r["grid"], "block": r["block"]})
+        k["launches"] += 1
+        k["epoch_ms_sum"] += r["epoch_ms"] / max(1, r["launches_in_epoch"])
+        k["written_chunks"] += r["epoch_written_chunks"] // max(1, r["launches_in_epoch"])
+
     # --- the diagnose pass at cfg5 scale; the other configs -------------------
     at_scale = diag_at_scale(xpl, torch)
     atom = atomic_peaks(xpl, torch)
@@ -584,6 +599,7 @@ def main():
                      "twin_ms_per_step": twin_ms / args.steps,
                      "paper_context": "Table III P:L431-443: 5x-20x, avg ~15x (Intel E5-2695 v4 + Pascal, CUDA 9.2)"},
         "e2e": e2e, "gpu_launches": int(launches), "clocks": clocks,
+        "launch_log": launch_log,
         "other_configs": others,
         "diagnose_sharded": sharded,
     }

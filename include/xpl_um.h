@@ -12,7 +12,8 @@
  *
  * Call xpl_um_enable before the process creates its CUDA context where the
  * platform requires it (CUPTI may refuse unified-memory counters otherwise);
- * every function returns 0 or the CUptiResult / CUDA error code it got.
+ * every function returns 0 or the CUptiResult it got (1000 + CUresult when the
+ * driver could not be initialised).
  * Not thread-safe; one collector per process. */
 #ifndef XPL_UM_H
 #define XPL_UM_H

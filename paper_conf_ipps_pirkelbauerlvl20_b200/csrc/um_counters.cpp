@@ -1,6 +1,7 @@
 // um_counters.cpp -- libxplum.so: CUPTI unified-memory counters kept per record
 // with their addresses (include/xpl_um.h; NEXT-4).
 #include <cupti.h>
+#include <dlfcn.h>
 #include <stdlib.h>
 #include <string.h>
 
@@ -49,6 +50,14 @@ void CUPTIAPI buffer_completed(CUcontext, uint32_t, uint8_t* buf, size_t, size_t
 extern "C" {
 
 int xpl_um_enable(int device) {
+  // "should be called after CUDA driver initialization" (cupti_activity.h): init
+  // the driver, but create no context -- the counters must be set up before it
+  // (libcuda is opened here, not linked: the library must load on driverless hosts)
+  void* drv = dlopen("libcuda.so.1", RTLD_NOW | RTLD_GLOBAL);
+  auto cu_init = drv ? (int (*)(unsigned))dlsym(drv, "cuInit") : nullptr;
+  if (!cu_init) return 1000 + 100;  // CUDA_ERROR_NO_DEVICE-like: no driver
+  const int cr = cu_init(0);
+  if (cr != 0) return 1000 + cr;
   CUptiResult r;
   if (!g_callbacks) {
     r = cuptiActivityRegisterCallbacks(buffer_requested, buffer_completed);

@@ -80,3 +80,13 @@ def test_binding_struct_layouts_match_the_header(tmp_path):
            ctypes.sizeof(xpl.XplLaunchRecord), xpl.XplLaunchRecord.epoch_ms.offset,
            ctypes.sizeof(xpl.XplLaunchInfo), xpl.XplLaunchInfo.shmem.offset]
     assert got == exp
+
+
+def test_um_library_exports_its_header():
+    """libxplum.so (CUPTI unified-memory counters, NEXT-4) loads without a GPU and
+    exports every function include/xpl_um.h declares."""
+    text = re.sub(r"/\*.*?\*/", "", open(os.path.join(ROOT, "include", "xpl_um.h")).read(), flags=re.S)
+    names = set(re.findall(r"^\s*\w+\s+(xpl_um_\w+)\s*\(", text, flags=re.M))
+    assert {"xpl_um_enable", "xpl_um_disable", "xpl_um_read", "xpl_um_dropped"} <= names
+    lib = ctypes.CDLL(os.path.join(ROOT, "paper_conf_ipps_pirkelbauerlvl20_b200", "libxplum.so"))
+    assert all(hasattr(lib, n) for n in names)

@@ -1,0 +1,5 @@
+set -x
+mkdir -p gpurun_out
+timeout 300 python tools/um_faults.py > gpurun_out/r1l_um.json 2> gpurun_out/r1l_um.err
+timeout 600 python -m pytest tests/test_gpu_launch_log.py tests/test_gpu_um_counters.py -x -q -m gpu > gpurun_out/r1l_pytest.log 2>&1; echo "pytest rc=$?" >> gpurun_out/r1l_pytest.log
+timeout 900 python bench.py --no-cpu-baseline --no-other-configs > gpurun_out/r1l_bench.json 2> gpurun_out/r1l_bench.err
