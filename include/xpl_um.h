@@ -40,6 +40,10 @@ int xpl_um_disable(void);
  * address lies in [base, base + bytes) -- bytes == 0: all records, whatever their
  * address.  reset != 0 drops every kept record afterwards.  0 on success. */
 int xpl_um_read(uint64_t base, uint64_t bytes, xpl_um_counts* out, int reset);
+/* The counter kinds the platform accepted at xpl_um_enable, as bits 1 << k in
+ * CUPTI's numbering: 1 HtoD bytes, 2 DtoH bytes, 3 CPU page faults, 4 GPU page
+ * faults, 5 thrashing, 6 throttling, 7 remote map, 8 DtoD bytes. */
+uint32_t xpl_um_kinds(void);
 /* Records dropped because the keep buffer was full (cap 2^22 records). */
 uint64_t xpl_um_dropped(void);
 

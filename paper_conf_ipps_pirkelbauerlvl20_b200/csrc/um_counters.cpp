@@ -21,6 +21,7 @@ std::mutex g_mu;
 std::vector<Rec> g_recs;
 uint64_t g_dropped = 0;
 bool g_callbacks = false;
+uint32_t g_kinds = 0;  // 1 << CUpti_ActivityUnifiedMemoryCounterKind accepted
 constexpr size_t kCap = size_t(1) << 22;
 constexpr size_t kBuf = size_t(8) << 20;
 
@@ -73,21 +74,33 @@ int xpl_um_enable(int device) {
       CUPTI_ACTIVITY_UNIFIED_MEMORY_COUNTER_KIND_THROTTLING,
       CUPTI_ACTIVITY_UNIFIED_MEMORY_COUNTER_KIND_REMOTE_MAP,
       CUPTI_ACTIVITY_UNIFIED_MEMORY_COUNTER_KIND_BYTES_TRANSFER_DTOD};
-  CUpti_ActivityUnifiedMemoryCounterConfig cfg[sizeof kinds / sizeof kinds[0]];
+  // Which kinds / scopes CUPTI accepts differs by platform: probe each kind alone
+  // (single-device scope first, then all devices), then configure the accepted set.
   const uint32_t n = sizeof kinds / sizeof kinds[0];
+  CUpti_ActivityUnifiedMemoryCounterConfig cfg[sizeof kinds / sizeof kinds[0]];
+  uint32_t m = 0;
+  int first_err = 0;
+  g_kinds = 0;
   for (uint32_t i = 0; i < n; ++i) {
-    cfg[i].scope = CUPTI_ACTIVITY_UNIFIED_MEMORY_COUNTER_SCOPE_PROCESS_SINGLE_DEVICE;
-    cfg[i].kind = kinds[i];
-    cfg[i].deviceId = (uint32_t)device;
-    cfg[i].enable = 1;
+    for (CUpti_ActivityUnifiedMemoryCounterScope sc : {CUPTI_ACTIVITY_UNIFIED_MEMORY_COUNTER_SCOPE_PROCESS_SINGLE_DEVICE,
+                                                       CUPTI_ACTIVITY_UNIFIED_MEMORY_COUNTER_SCOPE_PROCESS_ALL_DEVICES}) {
+      CUpti_ActivityUnifiedMemoryCounterConfig c;
+      c.scope = sc;
+      c.kind = kinds[i];
+      c.deviceId = (uint32_t)device;
+      c.enable = 1;
+      r = cuptiActivityConfigureUnifiedMemoryCounter(&c, 1);
+      if (r == CUPTI_SUCCESS) {
+        cfg[m++] = c;
+        g_kinds |= 1u << (uint32_t)kinds[i];
+        break;
+      }
+      if (!first_err) first_err = (int)r;
+    }
   }
-  r = cuptiActivityConfigureUnifiedMemoryCounter(cfg, n);
-  if (r != CUPTI_SUCCESS) {
-    // some kinds (thrashing / throttling / remote map) are not supported on
-    // every platform: retry with the four basic ones
-    r = cuptiActivityConfigureUnifiedMemoryCounter(cfg, 4);
-    if (r != CUPTI_SUCCESS) return (int)r;
-  }
+  if (!m) return first_err ? first_err : -1;
+  r = cuptiActivityConfigureUnifiedMemoryCounter(cfg, m);
+  if (r != CUPTI_SUCCESS) return (int)r;
   r = cuptiActivityEnable(CUPTI_ACTIVITY_KIND_UNIFIED_MEMORY_COUNTER);
   return (int)r;
 }
@@ -121,6 +134,8 @@ int xpl_um_read(uint64_t base, uint64_t bytes, xpl_um_counts* out, int reset) {
   if (reset) g_recs.clear();
   return 0;
 }
+
+uint32_t xpl_um_kinds(void) { return g_kinds; }
 
 uint64_t xpl_um_dropped(void) {
   std::lock_guard<std::mutex> g(g_mu);

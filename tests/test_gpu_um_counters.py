@@ -26,8 +26,11 @@ def test_um_counters_match_page_view():
     assert a["diagnose"]["alternating"] == pages and a["diagnose"]["flags"] & 1
     assert b["pages"]["gpu_pages"] == 0 and b["pages"]["cpu_pages"] == pages and b["diagnose"]["gpu_acc"] == 0
     assert c["pages"]["cpu_pages"] == 0 and c["pages"]["gpu_pages"] == pages
-    assert a["um"]["gpu_page_fault_groups"] > 0 and a["um"]["htod_bytes"] > 0
-    assert a["um"]["dtoh_bytes"] > 0 or a["um"]["cpu_page_faults"] > 0
-    assert b["um"]["gpu_page_fault_groups"] == 0 and b["um"]["htod_bytes"] == 0
+    k = set(out["kinds"])  # the counter kinds this platform's CUPTI accepted
+    assert {"htod_bytes", "dtoh_bytes"} <= k, out["kinds"]
+    assert a["um"]["htod_bytes"] > 0 and a["um"]["dtoh_bytes"] > 0
+    if "gpu_page_fault_groups" in k:
+        assert a["um"]["gpu_page_fault_groups"] > 0 and b["um"]["gpu_page_fault_groups"] == 0
+    assert b["um"]["htod_bytes"] == 0
     assert c["um"]["records"] == 0
     assert out["dropped"] == 0

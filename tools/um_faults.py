@@ -30,10 +30,12 @@ def main():
     um = C.CDLL(os.path.join(PKG, "libxplum.so"))
     um.xpl_um_read.argtypes = [C.c_uint64, C.c_uint64, C.POINTER(UmCounts), C.c_int]
     um.xpl_um_dropped.restype = C.c_uint64
+    um.xpl_um_kinds.restype = C.c_uint32
     st = um.xpl_um_enable(0)  # before any CUDA context
     if st != 0:
         print(json.dumps({"um_enable_status": st}))
         return 1
+    kinds = um.xpl_um_kinds()
 
     import numpy as np
     import torch
@@ -56,7 +58,10 @@ def main():
         rng_w[0] = (addr, nbytes, kind)
         ctx.record_host_ranges(rng_w)
 
-    out = {"config": {"bytes_per_alloc": nbytes, "gpu_stride_words": stride, "rounds": 3}}
+    names = {1: "htod_bytes", 2: "dtoh_bytes", 3: "cpu_page_faults", 4: "gpu_page_fault_groups", 5: "thrashing",
+             6: "throttling", 7: "remote_map", 8: "dtod_bytes"}
+    out = {"config": {"bytes_per_alloc": nbytes, "gpu_stride_words": stride, "rounds": 3},
+           "kinds": [v for k, v in names.items() if kinds >> k & 1]}
     with xpl.Context(pool_words=1 << 25) as ctx:
         ctx.bind()
         ctx.register(A, nbytes, 1)
