@@ -135,6 +135,19 @@ static __device__ __forceinline__ void xpld_commit(unsigned needers, unsigned q,
                        ((n0 & b1) ? 0x00FF0000u : 0u) | ((b0 & b1) ? 0xFF000000u : 0u);
     rb = (K & XPL_ACC_R) ? u : 0u;
     wb = (K & XPL_ACC_W) ? u : 0u;
+  } else if (SINGLE) {
+    /* per-lane kinds, one byte lane each: four ballots (byte-lane bits, R, W)
+     * name, per byte lane, whether some lane of the group reads / writes it */
+    const unsigned b = (unsigned)(__ffs(bytes) - 1) >> 3;
+    const unsigned b0 = __ballot_sync(needers, b & 1) & grp, b1 = __ballot_sync(needers, b & 2) & grp;
+    const unsigned r = __ballot_sync(needers, acc & XPL_ACC_R) & grp;
+    const unsigned w = __ballot_sync(needers, acc & XPL_ACC_W) & grp;
+    const unsigned n0 = grp & ~b0, n1 = grp & ~b1;
+    const unsigned l0 = n0 & n1, l1 = b0 & n1, l2 = n0 & b1, l3 = b0 & b1;
+    rb = ((l0 & r) ? 0x000000FFu : 0u) | ((l1 & r) ? 0x0000FF00u : 0u) | ((l2 & r) ? 0x00FF0000u : 0u) |
+         ((l3 & r) ? 0xFF000000u : 0u);
+    wb = ((l0 & w) ? 0x000000FFu : 0u) | ((l1 & w) ? 0x0000FF00u : 0u) | ((l2 & w) ? 0x00FF0000u : 0u) |
+         ((l3 & w) ? 0xFF000000u : 0u);
   } else {
 #pragma unroll
     for (unsigned k = 0; k < 4; ++k) {

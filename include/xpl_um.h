@@ -12,8 +12,10 @@
  *
  * Call xpl_um_enable before the process creates its CUDA context where the
  * platform requires it (CUPTI may refuse unified-memory counters otherwise);
- * every function returns 0 or the CUptiResult it got (1000 + CUresult when the
- * driver could not be initialised).
+ * every function returns 0 or an error: xpl_um_enable returns 1000 + CUresult
+ * (driver init), 4000 + / 3000 + / 2000 + CUptiResult (callback registration /
+ * counter configuration / activity enable), or the CUptiResult of the probe of
+ * the first kind when no kind is accepted; the others return the CUptiResult.
  * Not thread-safe; one collector per process. */
 #ifndef XPL_UM_H
 #define XPL_UM_H

@@ -62,7 +62,7 @@ int xpl_um_enable(int device) {
   CUptiResult r;
   if (!g_callbacks) {
     r = cuptiActivityRegisterCallbacks(buffer_requested, buffer_completed);
-    if (r != CUPTI_SUCCESS) return (int)r;
+    if (r != CUPTI_SUCCESS) return 4000 + (int)r;
     g_callbacks = true;
   }
   const CUpti_ActivityUnifiedMemoryCounterKind kinds[] = {
@@ -100,9 +100,9 @@ int xpl_um_enable(int device) {
   }
   if (!m) return first_err ? first_err : -1;
   r = cuptiActivityConfigureUnifiedMemoryCounter(cfg, m);
-  if (r != CUPTI_SUCCESS) return (int)r;
+  if (r != CUPTI_SUCCESS) return 3000 + (int)r;
   r = cuptiActivityEnable(CUPTI_ACTIVITY_KIND_UNIFIED_MEMORY_COUNTER);
-  return (int)r;
+  return r == CUPTI_SUCCESS ? 0 : 2000 + (int)r;
 }
 
 int xpl_um_disable(void) {
