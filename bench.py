@@ -263,6 +263,16 @@ def diag_at_scale(xpl, torch, words=1 << 31, reps=3):
     for _ in range(reps):
         ctx.diagnose(50, 0, 256, reset=False)
     p0 = ctx.profile_read(reset=True)
+    # the UM page view (NEXT-3) over the same shadow: one read pass; blocking
+    # call, timed whole (host wall clock around it, device work dominates)
+    import time
+    ctx.page_summary(1024)
+    pv = []
+    for _ in range(reps):
+        t0 = time.perf_counter()
+        ctx.page_summary(1024)
+        pv.append((time.perf_counter() - t0) * 1e3)
+    pv_ms = min(pv)
     rep = ctx.diagnose(50, 0, 256, reset=True)
     p1 = ctx.profile_read(reset=True)
     ctx.profile(False)
@@ -271,7 +281,10 @@ def diag_at_scale(xpl, torch, words=1 << 31, reps=3):
     out = {"record": {"device_accesses": n_dev, "ms": rec_ms, "accesses_per_s": n_dev / (rec_ms / 1e3),
                       "fold_ms": pf["ms"], "fold_gbs": pf["bytes"] / (pf["ms"] / 1e3) / 1e9 if pf["ms"] else None,
                       "shadow_u32_committed": n_red,
-                      "note": "instrumented touch kernel (hooks only, no user data) + epoch close, events on its stream"}}
+                      "note": "instrumented touch kernel (hooks only, no user data) + epoch close, events on its stream"},
+           "page_view": {"words": words, "page_words": 1024, "whole_call_ms": pv_ms,
+                         "gbs": words / (pv_ms / 1e3) / 1e9,
+                         "note": "xpl_page_summary (page_kernel: 1 B per word read), best of 3 blocking calls, wall clock"}}
     for name, p in (("no_reset", p0), ("reset", p1)):  # (the loop below fills these two)
         d = p["diag_tile"]
         ms = d["ms"] / d["launches"]

@@ -37,6 +37,9 @@ constexpr uint32_t kP4 = 0x02020202u;
 // kernels on their stream: griddepcontrol.wait holds it until they are
 // complete, while its own launch overlaps their tail.
 constexpr int kFoldThreads = 256;
+#ifndef XPL_FOLD_CTAS
+#define XPL_FOLD_CTAS (148 * 4)  // grid cap (A/B: profiles/r1_fold_grid_ab.txt)
+#endif
 
 __global__ void __launch_bounds__(kFoldThreads) fold_kernel(uint32_t* __restrict__ pool,
                                                             uint8_t* __restrict__ cmap,
@@ -1004,7 +1007,7 @@ void launch_fold(cudaStream_t s, bool pdl, uint32_t* pool, uint8_t* cmap, uint8_
                  uint64_t n_super, unsigned long long* stats) {
   if (!n_super) return;
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3((unsigned)(n_super < 148 * 4 ? n_super : 148 * 4));  // one wave
+  cfg.gridDim = dim3((unsigned)(n_super < XPL_FOLD_CTAS ? n_super : XPL_FOLD_CTAS));  // one wave
   cfg.blockDim = dim3(kFoldThreads);
   cfg.stream = s;
   cudaLaunchAttribute at[1];
