@@ -283,8 +283,9 @@ def diag_at_scale(xpl, torch, words=1 << 31, reps=3):
                       "shadow_u32_committed": n_red,
                       "note": "instrumented touch kernel (hooks only, no user data) + epoch close, events on its stream"},
            "page_view": {"words": words, "page_words": 1024, "whole_call_ms": pv_ms,
-                         "gbs": words / (pv_ms / 1e3) / 1e9,
-                         "note": "xpl_page_summary (page_kernel: 1 B per word read), best of 3 blocking calls, wall clock"}}
+                         "kernel_ms": p1["pages"]["ms"] / max(1, p1["pages"]["launches"]),
+                         "gbs": (p1["pages"]["bytes"] / (p1["pages"]["ms"] / 1e3) / 1e9) if p1["pages"]["ms"] else None,
+                         "note": "xpl_page_summary's page_kernel (1 B per word read), CUDA events, mean of 4 calls"}}
     for name, p in (("no_reset", p0), ("reset", p1)):  # (the loop below fills these two)
         d = p["diag_tile"]
         ms = d["ms"] / d["launches"]

@@ -378,14 +378,16 @@ xpl_status xpl_get_stats(xpl_ctx* ctx, xpl_stats* out);
  * xpl_profile_read waits for the runtime stream and returns, per kernel class,
  * the launches, the summed event time and the ALGORITHMIC bytes moved
  * (fold 256 B per written 128-word chunk; merge 8 B per record + 2 B per word;
- * range 2 B per word; diagnose 1 B per word + 1 B per word when resetting). */
+ * range 2 B per word; diagnose 1 B per word + 1 B per word when resetting;
+ * page view 1 B per word). */
 typedef enum {
   XPL_K_FOLD = 0,
   XPL_K_MERGE = 1,
   XPL_K_RANGE = 2,
   XPL_K_DIAG_TILE = 3, /* the one-pass shadow kernel of diagnose               */
   XPL_K_DIAGNOSE = 4,  /* the whole diagnose call (all its kernels + copies)   */
-  XPL_K_NCLASS = 5
+  XPL_K_PAGES = 5,     /* the page-view kernel (NEXT-3; 1 B per word read)    */
+  XPL_K_NCLASS = 6
 } xpl_kernel_class;
 typedef struct {
   uint64_t launches;

@@ -38,7 +38,7 @@ constexpr uint32_t kP4 = 0x02020202u;
 // complete, while its own launch overlaps their tail.
 constexpr int kFoldThreads = 256;
 #ifndef XPL_FOLD_CTAS
-#define XPL_FOLD_CTAS (148 * 4)  // grid cap (A/B: profiles/r1_fold_grid_ab.txt)
+#define XPL_FOLD_CTAS (148 * 8)  // grid cap (A/B: profiles/r1_fold_grid_ab.txt)
 #endif
 
 __global__ void __launch_bounds__(kFoldThreads) fold_kernel(uint32_t* __restrict__ pool,
@@ -976,13 +976,26 @@ __global__ void __launch_bounds__(256) page_kernel(const PageRow* __restrict__ r
     const uint64_t w0 = R.off + (p - R.page0) * P;                  // pool words [w0, w1)
     const uint64_t w1 = R.off + min(R.words, (p - R.page0 + 1) * P);
     uint32_t f = 0;
-    for (uint64_t q = (w0 >> 2) + lane; q <= ((w1 - 1) >> 2); q += 32) {
+    uint64_t wa = w0;  // words [w0, wa) done by the 16-byte path
+    if ((w0 & 15) == 0) {  // page starts on a uint4 (pool rows are 16-word aligned): 16 records
+      const uint4* p4 = reinterpret_cast<const uint4*>(pool);  // per lane, 4 loads in flight
+      const uint64_t v0 = w0 >> 4, v1 = w1 >> 4;
+      for (uint64_t v = v0 + lane; v < v1; v += 128) {
+        uint4 x[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) x[k] = v + 32 * k < v1 ? __ldg(p4 + v + 32 * k) : make_uint4(0, 0, 0, 0);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) f |= page_bits(x[k].x) | page_bits(x[k].y) | page_bits(x[k].z) | page_bits(x[k].w);
+      }
+      wa = v1 << 4;
+    }
+    for (uint64_t q = (wa >> 2) + lane; wa < w1 && q <= ((w1 - 1) >> 2); q += 32) {
       uint32_t x = pool[q];
-      if (q * 4 < w0 || q * 4 + 4 > w1) {
+      if (q * 4 < wa || q * 4 + 4 > w1) {
         uint32_t m = 0;
 #pragma unroll
         for (uint32_t k = 0; k < 4; ++k)
-          if (q * 4 + k >= w0 && q * 4 + k < w1) m |= 0xFFu << (8 * k);
+          if (q * 4 + k >= wa && q * 4 + k < w1) m |= 0xFFu << (8 * k);
         x &= m;
       }
       f |= page_bits(x);

@@ -679,7 +679,11 @@ static xpl_status page_pass(xpl_ctx* c, const std::vector<const Row*>& rows, uin
   if (h_flags) CK(cudaMallocAsync((void**)&d_flags, np + 1, c->cs));
   CK(cudaMemcpyAsync(d_rows, pr.data(), sizeof(PageRow) * pr.size(), cudaMemcpyHostToDevice, c->cs));
   CK(cudaMemsetAsync(d_cnt, 0, sizeof(unsigned long long) * ncnt + 8, c->cs));
+  uint64_t words = 0;
+  for (const Row* r : rows) words += r->words;
+  const int pi = prof_begin(c, XPL_K_PAGES, words);
   launch_pages(c->cs, d_rows, (uint32_t)pr.size(), np, P, (const uint32_t*)c->d_pool, d_flags, d_cnt);
+  prof_end(c, pi);
   c->st.kernel_launches += 1;
   CK(cudaMemcpyAsync(h_cnt, d_cnt, sizeof(unsigned long long) * ncnt, cudaMemcpyDeviceToHost, c->cs));
   if (h_flags) CK(cudaMemcpyAsync(h_flags, d_flags, np, cudaMemcpyDeviceToHost, c->cs));

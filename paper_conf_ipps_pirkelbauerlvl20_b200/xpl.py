@@ -154,7 +154,7 @@ class XplKernelTime(C.Structure):
     _fields_ = [("launches", u64), ("ms", C.c_double), ("bytes", u64)]
 
 
-KERNEL_CLASSES = ["fold", "merge", "range", "diag_tile", "diagnose"]
+KERNEL_CLASSES = ["fold", "merge", "range", "diag_tile", "diagnose", "pages"]
 xpl_profile_read = _sig("xpl_profile_read", [vp, C.POINTER(XplKernelTime), i32])
 
 EXPORTED = ["xpl_init", "xpl_finalize", "xpl_register_alloc", "xpl_free", "xpl_kernel_begin",
