@@ -978,15 +978,31 @@ __global__ void __launch_bounds__(256) page_kernel(const PageRow* __restrict__ r
     uint32_t f = 0;
     uint64_t wa = w0;  // words [w0, wa) done by the 16-byte path
     if ((w0 & 15) == 0) {  // page starts on a uint4 (pool rows are 16-word aligned): 16 records
-      const uint4* p4 = reinterpret_cast<const uint4*>(pool);  // per lane, 4 loads in flight
+      // per lane, up to 4 loads in flight; the class bits are accumulated per
+      // record byte in 64-bit SWAR registers and turned into page bits once
+      const ulonglong2* p4 = reinterpret_cast<const ulonglong2*>(pool);
       const uint64_t v0 = w0 >> 4, v1 = w1 >> 4;
+      unsigned long long a_cpu = 0, a_gpu = 0, a_both = 0, a_alt = 0, a_w = 0;
       for (uint64_t v = v0 + lane; v < v1; v += 128) {
-        uint4 x[4];
+        ulonglong2 x[4];
 #pragma unroll
-        for (int k = 0; k < 4; ++k) x[k] = v + 32 * k < v1 ? __ldg(p4 + v + 32 * k) : make_uint4(0, 0, 0, 0);
+        for (int k = 0; k < 4; ++k) x[k] = v + 32 * k < v1 ? __ldg(p4 + v + 32 * k) : make_ulonglong2(0, 0);
 #pragma unroll
-        for (int k = 0; k < 4; ++k) f |= page_bits(x[k].x) | page_bits(x[k].y) | page_bits(x[k].z) | page_bits(x[k].w);
+        for (int k = 0; k < 8; ++k) {
+          const unsigned long long y = (k & 1) ? x[k >> 1].y : x[k >> 1].x;
+          const unsigned long long c = ((y & 0x3434343434343434ull) + 0x7F7F7F7F7F7F7F7Full) & 0x8080808080808080ull;
+          const unsigned long long g =
+              (((y & 0x4848484848484848ull) + 0x7F7F7F7F7F7F7F7Full) | y) & 0x8080808080808080ull;
+          const unsigned long long w = ((y & 0x0C0C0C0C0C0C0C0Cull) + 0x7F7F7F7F7F7F7F7Full) & 0x8080808080808080ull;
+          a_cpu |= c;
+          a_gpu |= g;
+          a_both |= c & g;
+          a_alt |= c & g & w;
+          a_w |= y & 0x0C0C0C0C0C0C0C0Cull;
+        }
       }
+      f = (a_cpu ? 1u : 0u) | (a_gpu ? 2u : 0u) | (a_both ? 4u : 0u) | (a_alt ? 8u : 0u) |
+          ((a_w & 0x0404040404040404ull) ? 16u : 0u) | ((a_w & 0x0808080808080808ull) ? 32u : 0u);
       wa = v1 << 4;
     }
     for (uint64_t q = (wa >> 2) + lane; wa < w1 && q <= ((w1 - 1) >> 2); q += 32) {
