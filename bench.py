@@ -81,6 +81,16 @@ class Clocks:
                                        "-lms", "100"], stdout=self.f, stderr=subprocess.DEVNULL)
         except Exception:
             self.p = None
+        self.off = 0
+
+    def mark(self):
+        """Start of the timed region: only samples written from here on count.  (The
+        sampler is started before the warm-up, so nvidia-smi's own start-up -- NVML
+        init, a cold exec -- does not land in the timed host-bound step.)"""
+        try:
+            self.off = os.path.getsize(self.f.name)
+        except OSError:
+            self.off = 0
 
     def stop(self):
         if self.p is None:
@@ -88,7 +98,7 @@ class Clocks:
         self.p.terminate()
         self.p.wait()
         self.f.flush()
-        self.f.seek(0)
+        self.f.seek(self.off)
         sm, mx, reasons = [], None, set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         for line in self.f.read().splitlines():
@@ -479,6 +489,7 @@ def main():
                 hook_ctr.zero_()
         return total, counts
 
+    clk = Clocks(local)  # sampler up before the warm-up; clk.mark() opens the timed window
     for _ in range(args.warmup):
         prepare(False)
         step(ctx, False)
@@ -490,7 +501,7 @@ def main():
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    clk = Clocks(local)
+    clk.mark()
     ms_total, counts = timed(ctx, False, args.steps, rs)
     clocks = clk.stop()
     prof = ctx.profile_read(reset=True)

@@ -340,8 +340,8 @@ typedef struct {
   double epoch_ms;               /* GPU time of the epoch incl. its fold, -1 if n/a  */
 } xpl_launch_record;
 
-/* Turn the log on (1) or off (0).  Turning it on clears it.  STATE inside an
- * open epoch. */
+/* Turn the log on (1) or off (0); either clears it.  Synchronises the device
+ * (pending per-epoch copies of the old log).  STATE inside an open epoch. */
 xpl_status xpl_launch_log_enable(xpl_ctx* ctx, int enable);
 /* Log one launch of the open epoch (call between xpl_kernel_begin and _end,
  * before or after the launch itself).  STATE outside an epoch; INVALID_ARG on

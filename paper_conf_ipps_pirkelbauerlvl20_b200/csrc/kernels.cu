@@ -983,12 +983,14 @@ __global__ void __launch_bounds__(256) page_kernel(const PageRow* __restrict__ r
       const ulonglong2* p4 = reinterpret_cast<const ulonglong2*>(pool);
       const uint64_t v0 = w0 >> 4, v1 = w1 >> 4;
       unsigned long long a_cpu = 0, a_gpu = 0, a_both = 0, a_alt = 0, a_w = 0;
-      for (uint64_t v = v0 + lane; v < v1; v += 128) {
+      for (uint64_t b = v0; b < v1; b += 128) {  // (b is warp-uniform)
         ulonglong2 x[4];
 #pragma unroll
-        for (int k = 0; k < 4; ++k) x[k] = v + 32 * k < v1 ? __ldg(p4 + v + 32 * k) : make_ulonglong2(0, 0);
+        for (int k = 0; k < 4; ++k)
+          x[k] = b + 32 * k + lane < v1 ? __ldg(p4 + b + 32 * k + lane) : make_ulonglong2(0, 0);
 #pragma unroll
         for (int k = 0; k < 8; ++k) {
+          if (b + 32 * (k >> 1) >= v1) break;  // uniform: no ALU on groups past the page
           const unsigned long long y = (k & 1) ? x[k >> 1].y : x[k >> 1].x;
           const unsigned long long c = ((y & 0x3434343434343434ull) + 0x7F7F7F7F7F7F7F7Full) & 0x8080808080808080ull;
           const unsigned long long g =
