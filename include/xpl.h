@@ -320,8 +320,8 @@ xpl_status xpl_mem_advise(xpl_ctx* ctx, const void* ptr, size_t bytes, int advic
  * stream order, without synchronising the host: its GPU time (CUDA events from
  * the epoch's begin on its first stream to the end of its fold) and the number
  * of 128-word shadow chunks its fold found GPU-written (the epoch's write
- * footprint).  Off by default; costs two event records and one 8-byte
- * device->host copy per epoch when on. */
+ * footprint).  Off by default; costs three event records and two 8-byte
+ * device->host copies per epoch when on. */
 typedef struct {
   const char* name; /* kernel name; copied (interned) by the runtime, may be NULL */
   uint32_t grid[3], block[3];

@@ -178,7 +178,7 @@ struct xpl_ctx {
   // kernel-launch log (NEXT-4)
   struct EpochRec {
     cudaEvent_t a = nullptr, b = nullptr;  // begin on the epoch's first stream / after its fold
-    bool timed = false;
+    cudaEvent_t c = nullptr;               // after the end snapshot copy (what a read waits for)
   };
   bool llog = false;
   std::vector<xpl_launch_record> lrecs;
@@ -541,10 +541,9 @@ cudaEvent_t log_event(xpl_ctx* c) {
 }
 
 void log_clear(xpl_ctx* c) {
-  for (auto& r : c->lepochs) {
-    if (r.a) c->lev_free.push_back(r.a);
-    if (r.b) c->lev_free.push_back(r.b);
-  }
+  for (auto& r : c->lepochs)
+    for (cudaEvent_t e : {r.a, r.b, r.c})
+      if (e) c->lev_free.push_back(e);
   c->lepochs.clear();
   c->lepoch_no.clear();
   c->lrecs.clear();
@@ -569,8 +568,8 @@ xpl_status log_epoch_begin(xpl_ctx* c, cudaStream_t s) {
   xpl_ctx::EpochRec r;
   r.a = log_event(c);
   r.b = log_event(c);
-  if (!r.a || !r.b) return XPL_ERR_CUDA;
-  r.timed = true;
+  r.c = log_event(c);
+  if (!r.a || !r.b || !r.c) return XPL_ERR_CUDA;
   CK(cudaMemcpyAsync(c->h_lcum + 2 * i, c->d_stats + 3, sizeof(unsigned long long),
                      cudaMemcpyDeviceToHost, s));
   CK(cudaEventRecord(r.a, s));
@@ -633,7 +632,7 @@ xpl_status xpl_launch_log(xpl_ctx* c, xpl_launch_record* out, size_t cap, size_t
   std::vector<uint64_t> chunks(c->lepochs.size(), 0), nl(c->lepochs.size(), 0);
   for (size_t i = 0; i < c->lepochs.size(); ++i) {
     at[c->lepoch_no[i]] = i;
-    CK(cudaEventSynchronize(c->lepochs[i].b));
+    CK(cudaEventSynchronize(c->lepochs[i].c));  // (after b and the end snapshot copy)
     float f = 0.f;
     if (cudaEventElapsedTime(&f, c->lepochs[i].a, c->lepochs[i].b) == cudaSuccess) ms[i] = f;
     chunks[i] = c->h_lcum[2 * i + 1] - c->h_lcum[2 * i];
@@ -877,10 +876,9 @@ xpl_status xpl_finalize(xpl_ctx* c) {
   for (cudaEvent_t e : c->ev_pool) cudaEventDestroy(e);
   for (cudaEvent_t e : c->prof_free) cudaEventDestroy(e);
   for (cudaEvent_t e : c->lev_free) cudaEventDestroy(e);
-  for (auto& r : c->lepochs) {
-    if (r.a) cudaEventDestroy(r.a);
-    if (r.b) cudaEventDestroy(r.b);
-  }
+  for (auto& r : c->lepochs)
+    for (cudaEvent_t e : {r.a, r.b, r.c})
+      if (e) cudaEventDestroy(e);
   cudaFreeHost(c->h_lcum);
   for (auto& r : c->prof_pending) {
     cudaEventDestroy(r.a);
@@ -1030,6 +1028,7 @@ xpl_status xpl_kernel_end(xpl_ctx* c, void* stream) {
     CK(cudaEventRecord(c->lepochs[i].b, c->cs));
     CK(cudaMemcpyAsync(c->h_lcum + 2 * i + 1, c->d_stats + 3, sizeof(unsigned long long),
                        cudaMemcpyDeviceToHost, c->cs));
+    CK(cudaEventRecord(c->lepochs[i].c, c->cs));
     c->lepoch_open = false;
   }
   if (cudaGetLastError() != cudaSuccess) return XPL_ERR_CUDA;
