@@ -962,25 +962,35 @@ __global__ void __launch_bounds__(256) page_kernel(const PageRow* __restrict__ r
     if (rows[mid].page0 <= p0) lo = mid;
     else hi = mid;
   }
+  // the warp's row state lives in registers: the row, the first page of the next
+  // row, the pool word where page p starts; counters are 32-bit (a warp's chunk
+  // of pages fits) and go out with one atomicAdd each when the row changes
   uint32_t r = lo;
-  unsigned long long c[5] = {0, 0, 0, 0, 0};
-  for (uint64_t p = p0; p < p1; ++p) {
-    while (r + 1 < nrows && rows[r + 1].page0 <= p) {  // next row: flush its counts
-      const unsigned long long v = lane == 0 ? c[0] : lane == 1 ? c[1] : lane == 2 ? c[2] : lane == 3 ? c[3] : c[4];
-      if (lane < 5 && v) atomicAdd(cnt + 5ull * r + lane, v);
-#pragma unroll
-      for (int k = 0; k < 5; ++k) c[k] = 0;
+  PageRow R = rows[r];
+  uint64_t next0 = r + 1 < nrows ? rows[r + 1].page0 : npages;
+  uint64_t pw = R.off + (p0 - R.page0) * P;  // pool word of page p's first record
+  uint32_t c0 = 0, c1 = 0, c2 = 0, c3 = 0, c4 = 0;
+  auto flush_counts = [&]() {
+    const uint32_t v = lane == 0 ? c0 : lane == 1 ? c1 : lane == 2 ? c2 : lane == 3 ? c3 : c4;
+    if (lane < 5 && v) atomicAdd(cnt + 5ull * r + lane, (unsigned long long)v);
+    c0 = c1 = c2 = c3 = c4 = 0;
+  };
+  const ulonglong2* p4 = reinterpret_cast<const ulonglong2*>(pool);
+  for (uint64_t p = p0; p < p1; ++p, pw += P) {
+    while (p >= next0) {  // the next row (empty rows have no pages: skipped)
+      flush_counts();
       ++r;
+      R = rows[r];
+      next0 = r + 1 < nrows ? rows[r + 1].page0 : npages;
+      pw = R.off;
     }
-    const PageRow R = rows[r];
-    const uint64_t w0 = R.off + (p - R.page0) * P;                  // pool words [w0, w1)
-    const uint64_t w1 = R.off + min(R.words, (p - R.page0 + 1) * P);
+    const uint64_t w0 = pw;                                 // pool words [w0, w1)
+    const uint64_t w1 = min(pw + P, R.off + R.words);
     uint32_t f = 0;
     uint64_t wa = w0;  // words [w0, wa) done by the 16-byte path
     if ((w0 & 15) == 0) {  // page starts on a uint4 (pool rows are 16-word aligned): 16 records
       // per lane, up to 4 loads in flight; the class bits are accumulated per
       // record byte in 64-bit SWAR registers and turned into page bits once
-      const ulonglong2* p4 = reinterpret_cast<const ulonglong2*>(pool);
       const uint64_t v0 = w0 >> 4, v1 = w1 >> 4;
       unsigned long long a_cpu = 0, a_gpu = 0, a_both = 0, a_alt = 0, a_w = 0;
       for (uint64_t b = v0; b < v1; b += 128) {  // (b is warp-uniform)
@@ -1007,30 +1017,29 @@ __global__ void __launch_bounds__(256) page_kernel(const PageRow* __restrict__ r
           ((a_w & 0x0404040404040404ull) ? 16u : 0u) | ((a_w & 0x0808080808080808ull) ? 32u : 0u);
       wa = v1 << 4;
     }
-    for (uint64_t q = (wa >> 2) + lane; wa < w1 && q <= ((w1 - 1) >> 2); q += 32) {
-      uint32_t x = pool[q];
-      if (q * 4 < wa || q * 4 + 4 > w1) {
-        uint32_t m = 0;
+    if (wa < w1) {  // unaligned page start or a tail of < 16 words: u32 loads, bytes outside masked
+      for (uint64_t q = (wa >> 2) + lane; q <= ((w1 - 1) >> 2); q += 32) {
+        uint32_t x = pool[q];
+        if (q * 4 < wa || q * 4 + 4 > w1) {
+          uint32_t m = 0;
 #pragma unroll
-        for (uint32_t k = 0; k < 4; ++k)
-          if (q * 4 + k >= wa && q * 4 + k < w1) m |= 0xFFu << (8 * k);
-        x &= m;
+          for (uint32_t k = 0; k < 4; ++k)
+            if (q * 4 + k >= wa && q * 4 + k < w1) m |= 0xFFu << (8 * k);
+          x &= m;
+        }
+        f |= page_bits(x);
       }
-      f |= page_bits(x);
     }
     f = __reduce_or_sync(0xFFFFFFFFu, f);
     if (flags && lane == 0) flags[p] = (uint8_t)f;
-    const bool shared = (f & 3u) == 3u;
-    c[0] += f & 1u;
-    c[1] += (f >> 1) & 1u;
-    c[2] += shared;
-    c[3] += shared && !(f & 4u);
-    c[4] += (f >> 3) & 1u;
+    const uint32_t shared = (f & 3u) == 3u;
+    c0 += f & 1u;
+    c1 += (f >> 1) & 1u;
+    c2 += shared;
+    c3 += shared & ((f >> 2) ^ 1u);
+    c4 += (f >> 3) & 1u;
   }
-  if (lane < 5) {
-    const unsigned long long v = lane == 0 ? c[0] : lane == 1 ? c[1] : lane == 2 ? c[2] : lane == 3 ? c[3] : c[4];
-    if (v) atomicAdd(cnt + 5ull * r + lane, v);
-  }
+  flush_counts();
 }
 }  // namespace
 
