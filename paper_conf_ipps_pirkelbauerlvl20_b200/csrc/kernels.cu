@@ -992,29 +992,35 @@ __global__ void __launch_bounds__(256) page_kernel(const PageRow* __restrict__ r
       // per lane, up to 4 loads in flight; the class bits are accumulated per
       // record byte in 64-bit SWAR registers and turned into page bits once
       const uint64_t v0 = w0 >> 4, v1 = w1 >> 4;
-      unsigned long long a_cpu = 0, a_gpu = 0, a_both = 0, a_alt = 0, a_w = 0;
+      // CPU / GPU / CPU-write / GPU-write presence is a property of the OR of
+      // the records; only "both on one word" and "alternating" need per-record
+      // work, and only where the lane's 64 records hold both classes at all
+      uint32_t a_raw = 0;
+      unsigned long long a_both = 0, a_alt = 0;
       for (uint64_t b = v0; b < v1; b += 128) {  // (b is warp-uniform)
         ulonglong2 x[4];
 #pragma unroll
         for (int k = 0; k < 4; ++k)
           x[k] = b + 32 * k + lane < v1 ? __ldg(p4 + b + 32 * k + lane) : make_ulonglong2(0, 0);
+        unsigned long long o = 0;
 #pragma unroll
-        for (int k = 0; k < 8; ++k) {
-          if (b + 32 * (k >> 1) >= v1) break;  // uniform: no ALU on groups past the page
-          const unsigned long long y = (k & 1) ? x[k >> 1].y : x[k >> 1].x;
-          const unsigned long long c = ((y & 0x3434343434343434ull) + 0x7F7F7F7F7F7F7F7Full) & 0x8080808080808080ull;
-          const unsigned long long g =
-              (((y & 0x4848484848484848ull) + 0x7F7F7F7F7F7F7F7Full) | y) & 0x8080808080808080ull;
-          const unsigned long long w = ((y & 0x0C0C0C0C0C0C0C0Cull) + 0x7F7F7F7F7F7F7F7Full) & 0x8080808080808080ull;
-          a_cpu |= c;
-          a_gpu |= g;
-          a_both |= c & g;
-          a_alt |= c & g & w;
-          a_w |= y & 0x0C0C0C0C0C0C0C0Cull;
+        for (int k = 0; k < 4; ++k) o |= x[k].x | x[k].y;  // (zeros past the page add nothing)
+        const uint32_t o32 = (uint32_t)o | (uint32_t)(o >> 32);
+        a_raw |= o32;
+        if ((o32 & 0x34343434u) && (o32 & 0xC8C8C8C8u)) {
+#pragma unroll
+          for (int k = 0; k < 8; ++k) {
+            const unsigned long long y = (k & 1) ? x[k >> 1].y : x[k >> 1].x;
+            const unsigned long long c = (y & 0x3434343434343434ull) + 0x7F7F7F7F7F7F7F7Full;
+            const unsigned long long g = ((y & 0x4848484848484848ull) + 0x7F7F7F7F7F7F7F7Full) | y;
+            const unsigned long long cg = c & g & 0x8080808080808080ull;
+            a_both |= cg;
+            a_alt |= cg & ((y & 0x0C0C0C0C0C0C0C0Cull) + 0x7F7F7F7F7F7F7F7Full);
+          }
         }
       }
-      f = (a_cpu ? 1u : 0u) | (a_gpu ? 2u : 0u) | (a_both ? 4u : 0u) | (a_alt ? 8u : 0u) |
-          ((a_w & 0x0404040404040404ull) ? 16u : 0u) | ((a_w & 0x0808080808080808ull) ? 32u : 0u);
+      f = ((a_raw & 0x34343434u) ? 1u : 0u) | ((a_raw & 0xC8C8C8C8u) ? 2u : 0u) | (a_both ? 4u : 0u) |
+          (a_alt ? 8u : 0u) | ((a_raw & 0x04040404u) ? 16u : 0u) | ((a_raw & 0x08080808u) ? 32u : 0u);
       wa = v1 << 4;
     }
     if (wa < w1) {  // unaligned page start or a tail of < 16 words: u32 loads, bytes outside masked
