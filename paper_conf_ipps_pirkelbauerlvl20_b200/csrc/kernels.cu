@@ -969,20 +969,76 @@ __global__ void __launch_bounds__(256) page_kernel(const PageRow* __restrict__ r
   PageRow R = rows[r];
   uint64_t next0 = r + 1 < nrows ? rows[r + 1].page0 : npages;
   uint64_t pw = R.off + (p0 - R.page0) * P;  // pool word of page p's first record
+  // per-lane counts (the lane that judged a page counts it), summed over the
+  // warp when the row changes
   uint32_t c0 = 0, c1 = 0, c2 = 0, c3 = 0, c4 = 0;
   auto flush_counts = [&]() {
-    const uint32_t v = lane == 0 ? c0 : lane == 1 ? c1 : lane == 2 ? c2 : lane == 3 ? c3 : c4;
+    const uint32_t s0 = __reduce_add_sync(0xFFFFFFFFu, c0), s1 = __reduce_add_sync(0xFFFFFFFFu, c1),
+                   s2 = __reduce_add_sync(0xFFFFFFFFu, c2), s3 = __reduce_add_sync(0xFFFFFFFFu, c3),
+                   s4 = __reduce_add_sync(0xFFFFFFFFu, c4);
+    const uint32_t v = lane == 0 ? s0 : lane == 1 ? s1 : lane == 2 ? s2 : lane == 3 ? s3 : s4;
     if (lane < 5 && v) atomicAdd(cnt + 5ull * r + lane, (unsigned long long)v);
     c0 = c1 = c2 = c3 = c4 = 0;
   };
+  auto count = [&](uint32_t f) {
+    const uint32_t shared = (f & 3u) == 3u;
+    c0 += f & 1u;
+    c1 += (f >> 1) & 1u;
+    c2 += shared;
+    c3 += shared & ((f >> 2) ^ 1u);
+    c4 += (f >> 3) & 1u;
+  };
   const ulonglong2* p4 = reinterpret_cast<const ulonglong2*>(pool);
-  for (uint64_t p = p0; p < p1; ++p, pw += P) {
+  // small pages (P % 16 == 0, at most 128 uint4 of records): L lanes per page,
+  // 32 / L pages per warp step, so the per-page bookkeeping is shared by the warp
+  const uint64_t u4 = P >> 4;  // uint4 per page
+  uint32_t L = 32;
+  if ((P & 15) == 0 && u4 <= 128)
+    while (L > 1 && (uint64_t)(L >> 1) * 4 >= u4) L >>= 1;  // smallest power of 2 with 4 L >= u4
+  const uint32_t G = 32 / L, gi = lane / L, li = lane % L;
+  const uint32_t gmask = L == 32 ? 0xFFFFFFFFu : ((1u << L) - 1u) << (gi * L);
+  for (uint64_t p = p0; p < p1;) {
     while (p >= next0) {  // the next row (empty rows have no pages: skipped)
       flush_counts();
       ++r;
       R = rows[r];
       next0 = r + 1 < nrows ? rows[r + 1].page0 : npages;
       pw = R.off;
+    }
+    if (G > 1 && p + G <= p1 && p + G <= next0 && (p + G - R.page0) * P <= R.words) {
+      // G whole pages of this row, page p + gi for lane group gi (16-byte aligned:
+      // rows start on 16 words, P % 16 == 0)
+      const uint64_t v0 = (pw + (uint64_t)gi * P) >> 4;
+      ulonglong2 x[4];
+#pragma unroll
+      for (int k = 0; k < 4; ++k)
+        x[k] = li + L * k < u4 ? __ldg(p4 + v0 + li + L * k) : make_ulonglong2(0, 0);
+      unsigned long long o = 0;
+#pragma unroll
+      for (int k = 0; k < 4; ++k) o |= x[k].x | x[k].y;
+      const uint32_t o32 = (uint32_t)o | (uint32_t)(o >> 32);
+      unsigned long long a_both = 0, a_alt = 0;
+      if ((o32 & 0x34343434u) && (o32 & 0xC8C8C8C8u)) {
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+          const unsigned long long y = (k & 1) ? x[k >> 1].y : x[k >> 1].x;
+          const unsigned long long c = (y & 0x3434343434343434ull) + 0x7F7F7F7F7F7F7F7Full;
+          const unsigned long long g = ((y & 0x4848484848484848ull) + 0x7F7F7F7F7F7F7F7Full) | y;
+          const unsigned long long cg = c & g & 0x8080808080808080ull;
+          a_both |= cg;
+          a_alt |= cg & ((y & 0x0C0C0C0C0C0C0C0Cull) + 0x7F7F7F7F7F7F7F7Full);
+        }
+      }
+      uint32_t f = ((o32 & 0x34343434u) ? 1u : 0u) | ((o32 & 0xC8C8C8C8u) ? 2u : 0u) | (a_both ? 4u : 0u) |
+                   (a_alt ? 8u : 0u) | ((o32 & 0x04040404u) ? 16u : 0u) | ((o32 & 0x08080808u) ? 32u : 0u);
+      f = __reduce_or_sync(gmask, f);
+      if (li == 0) {
+        if (flags) flags[p + gi] = (uint8_t)f;
+        count(f);
+      }
+      p += G;
+      pw += (uint64_t)G * P;
+      continue;
     }
     const uint64_t w0 = pw;                                 // pool words [w0, w1)
     const uint64_t w1 = min(pw + P, R.off + R.words);
@@ -1037,13 +1093,12 @@ __global__ void __launch_bounds__(256) page_kernel(const PageRow* __restrict__ r
       }
     }
     f = __reduce_or_sync(0xFFFFFFFFu, f);
-    if (flags && lane == 0) flags[p] = (uint8_t)f;
-    const uint32_t shared = (f & 3u) == 3u;
-    c0 += f & 1u;
-    c1 += (f >> 1) & 1u;
-    c2 += shared;
-    c3 += shared & ((f >> 2) ^ 1u);
-    c4 += (f >> 3) & 1u;
+    if (lane == 0) {
+      if (flags) flags[p] = (uint8_t)f;
+      count(f);
+    }
+    ++p;
+    pw += P;
   }
   flush_counts();
 }

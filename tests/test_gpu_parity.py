@@ -366,7 +366,7 @@ def test_page_view(gpu, seed):
     replay, _ = gpu
     from xplgen.trace import with_pages
     ops = with_pages(random_trace(0x58504C60 + seed, n_allocs=6, n_steps=80, max_words=5000),
-                      (1, 5, 16, 1024, 1 << 40), seed)
+                      (1, 5, 16, 256, 512, 1024, 1 << 40), seed)
     compare(replay.run_trace(ops), oracle_run(ops), f"pages seed {seed}")
 
 
