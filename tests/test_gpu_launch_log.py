@@ -139,3 +139,35 @@ def test_rodinia_launch_log(gpu):
         assert r["grid"] == ((Cc + 31) // 32, (R + 7) // 8, 1) and r["block"] == (32, 8, 1)
         assert r["launches_in_epoch"] == 1 and r["stream"] == s.cuda_stream
         assert 600 <= r["epoch_written_chunks"] <= 601 and r["epoch_ms"] > 0
+
+
+def test_launch_log_multi_stream_epoch(gpu):
+    """One epoch spanning two streams (D19: begin on s1, a nested begin on s2, the
+    outermost end on s1): one epoch entry, both launches in it, its footprint the
+    chunks both launches write, reports still bit-exact vs the oracle."""
+    replay, xpl = gpu
+    import torch
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    base = 1 << 44
+    words = 1 << 16
+    with xpl.Context(pool_words=1 << 20) as ctx:
+        ctx.register(base, 4 * words, 0)
+        ctx.launch_log_enable(True)
+        ctx.kernel_begin(s1.cuda_stream)
+        ctx.kernel_begin(s2.cuda_stream)
+        for st, w0 in ((s1, 0), (s2, 128 * 20)):  # 10 + 10 chunks, disjoint
+            addr = torch.arange(base + 4 * w0, base + 4 * (w0 + 128 * 10), 4, dtype=torch.int64, device="cuda")
+            sz = torch.full_like(addr, 4, dtype=torch.int32)
+            acc = torch.full_like(addr, 2, dtype=torch.uint8)
+            torch.cuda.synchronize()
+            ctx.kernel_launch(st.cuda_stream, "writer", (addr.numel() // 256,), (256,))
+            ctx.replay(addr.data_ptr(), sz.data_ptr(), acc.data_ptr(), addr.numel(), stream=st.cuda_stream)
+            torch.cuda.synchronize()
+        ctx.kernel_end(s2.cuda_stream)
+        ctx.kernel_end(s1.cuda_stream)
+        log = ctx.launch_log()
+        rep = ctx.diagnose(50, 0, 256, True, ())
+    assert [r["stream"] for r in log] == [s1.cuda_stream, s2.cuda_stream]
+    assert log[0]["epoch"] == log[1]["epoch"] and log[0]["launches_in_epoch"] == 2
+    assert 20 <= log[0]["epoch_written_chunks"] <= 22 and log[0]["epoch_ms"] > 0  # (row start vs chunk grid)
+    assert rep[0]["w_g"] == 128 * 20
