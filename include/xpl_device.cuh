@@ -89,12 +89,18 @@ static __device__ __forceinline__ unsigned xpld_lane() {
  * write: plain idempotent byte stores, tested first (a stale cached 0 only
  * costs a redundant store).  Both bytes are loaded before either store, so
  * the two loads overlap.  Only first writes of a shadow u32 get here. */
+template <bool TESTED = true>
 static __device__ __forceinline__ void xpld_mark(unsigned q) {
   unsigned char* c = xpl_dctx.cmap + (q >> 5);
   unsigned char* s = xpl_dctx.smap + (q >> 12);
-  const unsigned cv = *c, sv = *s;
-  if (!cv) *c = 1;
-  if (!sv) *s = 1;
+  if (TESTED) {
+    const unsigned cv = *c, sv = *s;
+    if (!cv) *c = 1;
+    if (!sv) *s = 1;
+  } else {  /* latency variant: plain stores, nothing to wait for */
+    *c = 1;
+    *s = 1;
+  }
 }
 
 /* The record bits a read of the byte lanes rb and a write of the byte lanes wb
@@ -122,7 +128,7 @@ static __device__ __forceinline__ unsigned xpld_bits(unsigned cur, unsigned byte
  * fixes it), 0 when each lane brings its own (acc).  SINGLE: every lane touches
  * one byte lane, bytes == 0xFF << 8*b, so two ballots of b's bits name the
  * group's byte lanes.  Only the lanes of `needers` may call it. */
-template <unsigned K, bool SINGLE>
+template <unsigned K, bool SINGLE, bool TM = true>
 static __device__ __forceinline__ void xpld_commit(unsigned needers, unsigned q, unsigned cur,
                                                    unsigned bytes, unsigned acc) {
   const unsigned grp = __match_any_sync(needers, q);
@@ -166,14 +172,14 @@ static __device__ __forceinline__ void xpld_commit(unsigned needers, unsigned q,
   }
   if (xpld_lane() == (unsigned)(__ffs(grp) - 1)) {
     atomicOr(xpl_dctx.pool + q, xpld_bits2(cur, rb, wb)); /* no return value needed: RED */
-    if (wb) xpld_mark(q);
+    if (wb) xpld_mark<TM>(q);
   }
 }
 
 /* Apply a GPU access to the shadow words [g0, g1] (global pool word indices;
  * empty when g0 > g1).  All active lanes of the calling warp must call it.
  * K: the access kind if uniform over the warp (a compile-time call site), else 0. */
-template <unsigned K>
+template <unsigned K, bool TM = true>
 static __device__ __forceinline__ void xpl_dev_apply(unsigned long long g0,
                                                      unsigned long long g1,
                                                      unsigned acc) {
@@ -193,7 +199,7 @@ static __device__ __forceinline__ void xpl_dev_apply(unsigned long long g0,
     }
     const bool need = hit && (K == XPL_ACC_W || (cur & m) != m);
     const unsigned needers = __ballot_sync(singles, need);
-    if (need) xpld_commit<K, true>(needers, q, cur, bytes, acc);
+    if (need) xpld_commit<K, true, TM>(needers, q, cur, bytes, acc);
   }
   if (singles == active) return;
   /* multi-word accesses: one shadow u32 per iteration */
@@ -214,7 +220,7 @@ static __device__ __forceinline__ void xpl_dev_apply(unsigned long long g0,
     }
     const bool need = more && (K == XPL_ACC_W || (cur & m) != m);
     const unsigned needers = __ballot_sync(active, need);
-    if (need) xpld_commit<K, false>(needers, (unsigned)q, cur, bytes, acc);
+    if (need) xpld_commit<K, false, TM>(needers, (unsigned)q, cur, bytes, acc);
     more = more && q < ql;
     ++q;
   }
@@ -231,7 +237,7 @@ static __device__ __forceinline__ unsigned* xpld_row_cache() {
   return c;
 }
 
-template <unsigned K>
+template <unsigned K, bool TM = true>
 static __device__ __forceinline__ void xpl_dev_record_k(const void* p, unsigned size,
                                                         unsigned acc) {
 #ifndef XPL_OFF
@@ -270,7 +276,7 @@ static __device__ __forceinline__ void xpl_dev_record_k(const void* p, unsigned 
     g0 = ow.x + w0;
     g1 = ow.x + wl;
   }
-  xpl_dev_apply<K>(g0, g1, K ? K : acc);
+  xpl_dev_apply<K, TM>(g0, g1, K ? K : acc);
 #else
   (void)p; (void)size; (void)acc;
 #endif
@@ -295,6 +301,16 @@ static __device__ __forceinline__ T& xpl_write(T& x) {
 template <class T>
 static __device__ __forceinline__ T& xpl_rw(T& x) {
   xpl_dev_record_k<XPL_ACC_RW>(&x, sizeof(T), XPL_ACC_RW);
+  return x;
+}
+/* traceW for latency-bound kernels (few threads, a few writes each, e.g. one
+ * small block per tile of a wavefront): the same record, but the write's chunk
+ * mark is stored without first testing it, so the hook issues only stores and
+ * atomics and never waits on memory.  Do not use it where many warps write one
+ * 2M-word region per epoch (every commit would store the same super-chunk byte). */
+template <class T>
+static __device__ __forceinline__ T& xpl_write_lat(T& x) {
+  xpl_dev_record_k<XPL_ACC_W, false>(&x, sizeof(T), XPL_ACC_W);
   return x;
 }
 

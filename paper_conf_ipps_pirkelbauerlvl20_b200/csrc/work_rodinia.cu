@@ -31,6 +31,11 @@ __device__ __forceinline__ T& WR(T& x) {
   else return x;
 }
 template <bool I, class T>
+__device__ __forceinline__ T& WRL(T& x) {  // the latency-variant write hook (xpl_write_lat)
+  if constexpr (I) return xpl_write_lat(x);
+  else return x;
+}
+template <bool I, class T>
 __device__ __forceinline__ T& RW(T& x) {
   if constexpr (I) return xpl_rw(x);
   else return x;
@@ -340,7 +345,7 @@ __global__ void __launch_bounds__(NWB) nw_kernel(int* ref, int* mat, int cols, i
     }
     __syncthreads();
   }
-  for (int ty = 0; ty < NWB; ty++) WR<I>(mat[index + ty * cols]) = temp[ty + 1][tx + 1];
+  for (int ty = 0; ty < NWB; ty++) WRL<I>(mat[index + ty * cols]) = temp[ty + 1][tx + 1];  // 16-thread blocks
 }
 
 // ---------------------------------------------------------------------------
