@@ -303,6 +303,84 @@ static __device__ __forceinline__ T& xpl_rw(T& x) {
   xpl_dev_record_k<XPL_ACC_RW>(&x, sizeof(T), XPL_ACC_RW);
   return x;
 }
+/* traceR for latency-bound kernels: xpl_read_lat(x) returns a proxy.  The hook's
+ * lookup and shadow load are issued when the proxy is made; the proxy converts
+ * to `const T&` (the user's own load of x follows, with the shadow load still in
+ * flight); its destructor -- at the end of the full expression, e.g. after
+ * `v = xpl_read_lat(a[i]);` -- tests and commits the record exactly as xpl_read
+ * does.  So the shadow load's latency overlaps the user's load instead of
+ * adding to it.  All lanes that made the proxy must reach its destructor (it
+ * is warp-synchronous, like every hook); accesses of more than one word commit
+ * at once. */
+template <class T>
+struct xpl_read_proxy {
+  const T& x;
+  unsigned q, cur, bytes, active, singles;
+  bool hit;
+  __device__ __forceinline__ explicit xpl_read_proxy(const T& v) : x(v) {
+#ifndef XPL_OFF
+    unsigned* const xpl_row_cache = xpld_row_cache();
+    const unsigned long long a = (unsigned long long)&v;
+    const xpl_dev_row* rows = xpl_dctx.rows;
+    const unsigned n = __ldg(xpl_dctx.n_rows);
+    const unsigned slot = ((threadIdx.z * blockDim.y + threadIdx.y) * blockDim.x + threadIdx.x) >> 5 & 31;
+    unsigned ri = xpl_row_cache[slot];
+    const unsigned rc = ri < n ? ri : 0;
+    ulonglong2 be = __ldg(reinterpret_cast<const ulonglong2*>(rows + rc));
+    ulonglong2 ow = __ldg(reinterpret_cast<const ulonglong2*>(rows + rc) + 1);
+    bool h = ri < n && be.x <= a && a < be.y;
+    if (!h) {
+      unsigned lo = 0, hi = n;
+      while (lo < hi) {
+        const unsigned mid = (lo + hi) >> 1;
+        if (__ldg(&rows[mid].base) <= a) lo = mid + 1;
+        else hi = mid;
+      }
+      if (lo > 0 && a < __ldg(&rows[lo - 1].end)) {
+        ri = lo - 1;
+        h = true;
+        xpl_row_cache[slot] = ri;
+        be = __ldg(reinterpret_cast<const ulonglong2*>(rows + ri));
+        ow = __ldg(reinterpret_cast<const ulonglong2*>(rows + ri) + 1);
+      }
+    }
+    unsigned long long g0 = 1, g1 = 0;
+    if (h) {
+      const unsigned long long w0 = (a - be.x) >> 2;
+      unsigned long long wl = (a + sizeof(T) - 1 - be.x) >> 2;
+      if (wl > ow.y - 1) wl = ow.y - 1;
+      g0 = ow.x + w0;
+      g1 = ow.x + wl;
+    }
+    active = __activemask();
+    const bool single = g0 >= g1;
+    singles = __ballot_sync(active, single);
+    hit = single && g0 == g1;
+    q = (unsigned)(g0 >> 2);
+    bytes = 0xFFu << (8 * (unsigned)(g0 & 3));
+    cur = hit ? xpl_dctx.pool[q] : 0u;  /* issued now, consumed in the destructor */
+    if (singles != active) xpl_dev_apply<XPL_ACC_R>(single ? 1ull : g0, single ? 0ull : g1, XPL_ACC_R);
+#endif
+  }
+  __device__ __forceinline__ operator const T&() const { return x; }
+  __device__ __forceinline__ ~xpl_read_proxy() {
+#ifndef XPL_OFF
+    if (singles & (1u << xpld_lane())) {
+      const unsigned m = xpld_bits(cur, bytes, XPL_ACC_R);
+      const bool need = hit && (cur & m) != m;
+      const unsigned needers = __ballot_sync(singles, need);
+      if (need) xpld_commit<XPL_ACC_R, true>(needers, q, cur, bytes, XPL_ACC_R);
+    }
+#endif
+  }
+  xpl_read_proxy(const xpl_read_proxy&) = delete;
+  xpl_read_proxy& operator=(const xpl_read_proxy&) = delete;
+};
+template <class T>
+static __device__ __forceinline__ xpl_read_proxy<T> xpl_read_lat(const T& x) {
+  return xpl_read_proxy<T>(x);
+}
+
 /* traceW for latency-bound kernels (few threads, a few writes each, e.g. one
  * small block per tile of a wavefront): the same record, but the write's chunk
  * mark is stored without first testing it, so the hook issues only stores and

@@ -31,6 +31,11 @@ __device__ __forceinline__ T& WR(T& x) {
   else return x;
 }
 template <bool I, class T>
+__device__ __forceinline__ decltype(auto) RDL(const T& x) {  // the latency-variant read hook (xpl_read_lat)
+  if constexpr (I) return xpl_read_lat(x);
+  else return (x);
+}
+template <bool I, class T>
 __device__ __forceinline__ T& WRL(T& x) {  // the latency-variant write hook (xpl_write_lat)
   if constexpr (I) return xpl_write_lat(x);
   else return x;
@@ -322,12 +327,12 @@ __global__ void __launch_bounds__(NWB) nw_kernel(int* ref, int* mat, int cols, i
   const int index_nw = cols * NWB * b_index_y + NWB * b_index_x;
   __shared__ int temp[NWB + 1][NWB + 1];
   __shared__ int rf[NWB][NWB];
-  if (tx == 0) temp[tx][0] = RD<I>(mat[index_nw]);
-  for (int ty = 0; ty < NWB; ty++) rf[ty][tx] = RD<I>(ref[index + cols * ty]);
+  if (tx == 0) temp[tx][0] = RDL<I>(mat[index_nw]);
+  for (int ty = 0; ty < NWB; ty++) rf[ty][tx] = RDL<I>(ref[index + cols * ty]);
   __syncthreads();
-  temp[tx + 1][0] = RD<I>(mat[index_w + cols * tx]);
+  temp[tx + 1][0] = RDL<I>(mat[index_w + cols * tx]);
   __syncthreads();
-  temp[0][tx + 1] = RD<I>(mat[index_n]);
+  temp[0][tx + 1] = RDL<I>(mat[index_n]);
   __syncthreads();
   for (int m = 0; m < NWB; m++) {
     if (tx <= m) {
