@@ -101,9 +101,37 @@ __global__ void touch_mem_kernel(unsigned* base, unsigned long long n, unsigned 
   if (acc == 0x9E3779B9u) *sink = acc;
 }
 
+// Reads through the deferred-commit hook (xpl_read_lat): element i reads a T at
+// addr[i] (addresses only: the proxy is never converted, so no user load).
+template <class T>
+__global__ void read_lat_kernel(const unsigned long long* __restrict__ addr, unsigned long long n) {
+  for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (unsigned long long)gridDim.x * blockDim.x) {
+    auto pr = xpl_read_lat(*reinterpret_cast<const T*>(addr[i]));
+    (void)pr;
+  }
+}
+
 }  // namespace
 
 extern "C" {
+
+// Launch read_lat_kernel<T> with sizeof(T) = size (1, 2, 4, 8 or 16) on `stream`
+// (between xpl_kernel_begin/_end); grid-stride, so odd grids are allowed.
+int xplw_read_lat(const unsigned long long* d_addr, unsigned long long n, int size, int grid, int block,
+                  void* stream) {
+  if (n == 0) return 0;
+  cudaStream_t s = (cudaStream_t)stream;
+  switch (size) {
+    case 1: read_lat_kernel<unsigned char><<<grid, block, 0, s>>>(d_addr, n); break;
+    case 2: read_lat_kernel<unsigned short><<<grid, block, 0, s>>>(d_addr, n); break;
+    case 4: read_lat_kernel<unsigned int><<<grid, block, 0, s>>>(d_addr, n); break;
+    case 8: read_lat_kernel<unsigned long long><<<grid, block, 0, s>>>(d_addr, n); break;
+    case 16: read_lat_kernel<uint4><<<grid, block, 0, s>>>(d_addr, n); break;
+    default: return (int)XPL_ERR_INVALID_ARG;
+  }
+  return cudaGetLastError() == cudaSuccess ? 0 : (int)XPL_ERR_CUDA;
+}
 
 // Launch touch_mem_kernel on `stream` (between xpl_kernel_begin/_end).
 int xplw_touch_mem(void* base, unsigned long long n_words, unsigned long long stride, int write, void* stream) {

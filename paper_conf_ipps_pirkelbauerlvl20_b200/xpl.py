@@ -172,6 +172,9 @@ if _work is not None:
     xplw_replay_split = _sig("xplw_replay_split", [vp, vp, vp, vp, i32, i32, i32, vp], lib=_work)
     xplw_atomic_bench = _sig("xplw_atomic_bench", [vp, u64, i32, vp], lib=_work)
     xplw_touch = _sig("xplw_touch", [u64, u64, u32, vp, u64], lib=_work)
+    # (optional so that A/B builds of the workload library without it still load)
+    xplw_read_lat = (_sig("xplw_read_lat", [vp, u64, i32, i32, i32, vp], lib=_work)
+                     if hasattr(_work, "xplw_read_lat") else None)
 
 
 class XplError(RuntimeError):

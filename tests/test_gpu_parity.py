@@ -389,3 +389,49 @@ def test_page_flags_map(gpu):
                      8 * int((cpu & gp & ((w & 0x0C) != 0)).any()) | 16 * int(((w & 4) != 0).any()) |
                      32 * int(((w & 8) != 0).any()))
                 assert f[p] == e, (r["id"], p)
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_read_lat_deferred_commit(gpu, seed):
+    """xpl_read_lat (the read hook whose commit runs at the end of the full
+    expression) gives the records xpl_read gives: device reads of 1, 2, 4, 8 and
+    16 bytes (sub-word, one word, multi-word), hits and misses, after random host
+    writes, bit-exact vs the oracle through several epochs and diagnoses."""
+    _, xpl = gpu
+    import torch
+    rng = np.random.default_rng(0x58504C80 + seed)
+    allocs = [(0x10000000 + k * 0x100000, int(rng.integers(100, 5000)) * 4 + int(rng.integers(0, 4)))
+              for k in range(4)]
+    ops = [("REG", a, b, int(rng.integers(0, 3))) for a, b in allocs]
+    for e in range(10):
+        for _ in range(6):
+            a, b = allocs[int(rng.integers(4))]
+            ops.append(("H", a + int(rng.integers(0, b)), int(rng.integers(1, 64)), int(rng.integers(1, 4))))
+        sz = (1, 2, 4, 8, 16)[e % 5]
+        n = int(rng.integers(1, 3000))
+        picks = rng.integers(0, 4, n)
+        addrs = np.array([allocs[p][0] + int(rng.integers(0, allocs[p][1] + 64)) // sz * sz for p in picks],
+                         dtype=np.uint64)  # (+64: some reads miss past the end)
+        ops += [("KB",), ("DB", addrs, np.full(n, sz, np.uint32), np.full(n, R, np.uint8)), ("KE",),
+                ("DIAG", 50, 0, 256, int(e % 3 != 0), ())]
+    s = torch.cuda.current_stream().cuda_stream
+    got = []
+    with xpl.Context(pool_words=1 << 22) as ctx:
+        for op in ops:
+            t = op[0]
+            if t == "REG":
+                ctx.register(op[1], op[2], op[3])
+            elif t == "H":
+                ctx.record_host(np.array([(op[1], op[2], op[3])], dtype=xpl.HOST_ACCESS_DTYPE))
+            elif t == "KB":
+                ctx.kernel_begin(s)
+            elif t == "KE":
+                ctx.kernel_end(s)
+            elif t == "DB":
+                d = torch.from_numpy(op[1].view(np.int64)).cuda()
+                grid = int(rng.integers(1, 64))
+                xpl.check("xplw_read_lat", xpl.xplw_read_lat(d.data_ptr(), d.numel(), int(op[2][0]), grid, 96, s))
+                torch.cuda.synchronize()
+            elif t == "DIAG":
+                got.append(ctx.diagnose(*op[1:5], names=op[5]))
+    compare(got, oracle_run(ops), f"read_lat seed {seed}")
