@@ -189,12 +189,12 @@ __global__ void __launch_bounds__(256) hotspot_kernel(const float* power, const 
   const int i = blockIdx.y * blockDim.y + threadIdx.y;
   if (i >= R || j >= C) return;
   const int idx = i * C + j;
-  const float c = RDL<I>(src[idx]);
-  const float n = RDL<I>(src[(i > 0 ? i - 1 : 0) * C + j]);
-  const float s = RDL<I>(src[(i < R - 1 ? i + 1 : R - 1) * C + j]);
-  const float w = RDL<I>(src[i * C + (j > 0 ? j - 1 : 0)]);
-  const float e = RDL<I>(src[i * C + (j < C - 1 ? j + 1 : C - 1)]);
-  const float p = RDL<I>(power[idx]);
+  const float c = RD<I>(src[idx]);
+  const float n = RD<I>(src[(i > 0 ? i - 1 : 0) * C + j]);
+  const float s = RD<I>(src[(i < R - 1 ? i + 1 : R - 1) * C + j]);
+  const float w = RD<I>(src[i * C + (j > 0 ? j - 1 : 0)]);
+  const float e = RD<I>(src[i * C + (j < C - 1 ? j + 1 : C - 1)]);
+  const float p = RD<I>(power[idx]);
   WR<I>(dst[idx]) = c + k_step * (p + (s + n - 2.f * c) * ry1 + (e + w - 2.f * c) * rx1 + (amb - c) * rz1);
 }
 
@@ -211,9 +211,9 @@ __global__ void __launch_bounds__(256) bp_layerforward(const float* input, float
   const int by = blockIdx.x, tx = threadIdx.x, ty = threadIdx.y;
   const int index = (hid + 1) * BP * by + (hid + 1) * ty + tx + 1 + (hid + 1);
   const int index_in = BP * by + ty + 1;
-  if (tx == 0) in_node[ty] = RDL<I>(input[index_in]);
+  if (tx == 0) in_node[ty] = RD<I>(input[index_in]);
   __syncthreads();
-  wm[ty][tx] = RDL<I>(weights[index]) * in_node[ty];
+  wm[ty][tx] = RD<I>(weights[index]) * in_node[ty];
   WR<I>(weights[index]) = wm[ty][tx];
   __syncthreads();
   for (int stride = 1; stride < BP; stride <<= 1) {
@@ -231,12 +231,12 @@ __global__ void __launch_bounds__(256) bp_adjust(const float* delta, const float
   const int index_y = BP * by + ty + 1;
   const int index_x = tx + 1;
   const float eta = 0.3f, momentum = 0.3f;
-  const float d = RDL<I>(delta[index_x]) * RDL<I>(ly[index_y]);
+  const float d = RD<I>(delta[index_x]) * RD<I>(ly[index_y]);
   const float nw = eta * d + momentum * RW<I>(oldw[index]);
   RW<I>(w[index]) += nw;
   RW<I>(oldw[index]) = nw;
   if (ty == 0 && by == 0) {  // the bias row
-    const float nb = eta * RDL<I>(delta[index_x]) + momentum * RW<I>(oldw[index_x]);
+    const float nb = eta * RD<I>(delta[index_x]) + momentum * RW<I>(oldw[index_x]);
     RW<I>(w[index_x]) += nb;
     RW<I>(oldw[index_x]) = nb;
   }
@@ -270,15 +270,15 @@ __global__ void __launch_bounds__(512) bfs_kernel1(BfsNode* nodes, int* edges, b
   unsigned c = 0;
   if (tid < n) {
     ++c;
-    if (RDL<I>(mask[tid])) {
+    if (RD<I>(mask[tid])) {
       WR<I>(mask[tid]) = false;
       c += 4;  // the write, the loop init and the first loop test (2 reads)
-      for (int i = RDL<I>(nodes[tid].starting);
-           i < (RDL<I>(nodes[tid].no_of_edges) + RDL<I>(nodes[tid].starting)); i++) {
-        const int id = RDL<I>(edges[i]);
+      for (int i = RD<I>(nodes[tid].starting);
+           i < (RD<I>(nodes[tid].no_of_edges) + RD<I>(nodes[tid].starting)); i++) {
+        const int id = RD<I>(edges[i]);
         c += 4;  // edges, visited, and the next loop test (2 reads)
-        if (!RDL<I>(visited[id])) {
-          WR<I>(cost[id]) = RDL<I>(cost[tid]) + 1;
+        if (!RD<I>(visited[id])) {
+          WR<I>(cost[id]) = RD<I>(cost[tid]) + 1;
           WR<I>(updating[id]) = true;
           c += 3;
         }
@@ -295,7 +295,7 @@ __global__ void __launch_bounds__(512) bfs_kernel2(bool* mask, bool* updating, b
   unsigned c = 0;
   if (tid < n) {
     ++c;
-    if (RDL<I>(updating[tid])) {
+    if (RD<I>(updating[tid])) {
       WR<I>(mask[tid]) = true;
       WR<I>(visited[tid]) = true;
       WR<I>(*over) = true;
