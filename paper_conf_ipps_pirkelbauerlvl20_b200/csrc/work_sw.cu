@@ -27,28 +27,15 @@ __device__ __forceinline__ T& WR(T& x) {
   else return x;
 }
 
-// the latency variants (xpl_read_lat / xpl_write_lat): a cell is five reads and
-// one write, one cell per thread per diagonal -- latency-bound
-template <bool I, class T>
-__device__ __forceinline__ decltype(auto) RDL(const T& x) {
-  if constexpr (I) return xpl_read_lat(x);
-  else return (x);
-}
-template <bool I, class T>
-__device__ __forceinline__ T& WRL(T& x) {
-  if constexpr (I) return xpl_write_lat(x);
-  else return x;
-}
-
 template <bool I>
 __device__ __forceinline__ void sw_cell(const int* a, const int* b, int* H, int ld, int i, int j) {
-  const int s = RDL<I>(a[i - 1]) == RDL<I>(b[j - 1]) ? kMatch : kMismatch;
-  const int d = RDL<I>(H[(i - 1) * ld + j - 1]) + s;
-  const int u = RDL<I>(H[(i - 1) * ld + j]) - kGap;
-  const int l = RDL<I>(H[i * ld + j - 1]) - kGap;
+  const int s = RD<I>(a[i - 1]) == RD<I>(b[j - 1]) ? kMatch : kMismatch;
+  const int d = RD<I>(H[(i - 1) * ld + j - 1]) + s;
+  const int u = RD<I>(H[(i - 1) * ld + j]) - kGap;
+  const int l = RD<I>(H[i * ld + j - 1]) - kGap;
   int h = d > u ? d : u;
   h = h > l ? h : l;
-  WRL<I>(H[i * ld + j]) = h > 0 ? h : 0;
+  WR<I>(H[i * ld + j]) = h > 0 ? h : 0;
 }
 
 // cfg1: one CTA, thread t owns row i = t + 1, sweeping the anti-diagonals.
