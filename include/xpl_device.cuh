@@ -11,8 +11,9 @@
  * Compile the same kernel with -DXPL_OFF to get the uninstrumented twin.
  * Latency variants (same records, for latency-bound kernels -- few threads, one
  * access after another): xpl_read_lat(x) defers the commit to the end of the
- * full expression so its shadow load overlaps the user's load; xpl_write_lat(x)
- * stores the chunk mark without testing it first, so it never waits.
+ * full expression so its shadow load overlaps the user's load (C++17: the proxy
+ * is returned by guaranteed copy elision); xpl_write_lat(x) stores the chunk
+ * mark without testing it first, so it never waits.
  *
  * What a hook does (design: DESIGN.md §5):
  *  1. lookup: binary search of the address in the live-allocation table
