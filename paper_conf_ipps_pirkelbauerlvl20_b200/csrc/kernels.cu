@@ -30,7 +30,7 @@ constexpr uint32_t kP4 = 0x02020202u;
 // byte per thread per round) and lists the marked ones in shared memory, so
 // an epoch that wrote little costs one launch and one read of the super map;
 // then, per listed super-chunk, warp w checks chunks [16w, 16w+16) and folds
-// the marked ones four at a time (128 B coalesced each).  Consecutive
+// all its marked ones with one round trip (128 B coalesced each).  Consecutive
 // super-chunks go to different CTAs, so a dense epoch spreads over the grid.
 // No global list, no atomics; cost O(super map + chunks written).  Launched
 // with programmatic stream serialization when it directly follows the epoch's
@@ -69,25 +69,15 @@ __global__ void __launch_bounds__(kFoldThreads) fold_kernel(uint32_t* __restrict
       const bool m = lane < 16 && cmap[c0 + lane] != 0;
       uint32_t marked = __ballot_sync(0xFFFFFFFFu, m);
       folded += __popc(marked);
-      while (marked) {
-        uint64_t at[4];
-        uint32_t v[4];
+      // All of the warp's marked chunks in one round trip: 16 predicated
+      // loads (warp-uniform predicates) issued back to back, then the stores.
+      uint32_t v[16];
+      uint32_t* const base = pool + c0 * 32 + lane;
 #pragma unroll
-        for (uint32_t j4 = 0; j4 < 4; ++j4) {
-          if (marked) {
-            const uint32_t j = __ffs(marked) - 1;
-            marked &= marked - 1;
-            at[j4] = (c0 + j) * 32 + lane;
-            v[j4] = pool[at[j4]];
-          } else {
-            at[j4] = ~0ull;
-            v[j4] = 0;
-          }
-        }
+      for (uint32_t j = 0; j < 16; ++j) v[j] = (marked >> j) & 1u ? base[j * 32] : 0u;
 #pragma unroll
-        for (uint32_t j4 = 0; j4 < 4; ++j4)
-          if (v[j4] & kP4) pool[at[j4]] = (v[j4] & ~kP4) | ((v[j4] & kP4) >> 1);
-      }
+      for (uint32_t j = 0; j < 16; ++j)
+        if (v[j] & kP4) base[j * 32] = (v[j] & ~kP4) | ((v[j] & kP4) >> 1);
       if (m) cmap[c0 + lane] = 0;
       if (threadIdx.x == 0) smap[sc] = 0;
     }
