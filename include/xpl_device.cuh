@@ -423,16 +423,28 @@ static __device__ __forceinline__ void xpl_grid_epoch() {
     if (!__ldcg(xpl_dctx.smap + sc)) continue; /* (uniform over the warp) */
     for (unsigned c0 = 0; c0 < 128; c0 += 32) {
       const unsigned long long ch = sc * 128 + c0 + lane;
-      const bool m = __ldcg(xpl_dctx.cmap + ch) != 0;
-      unsigned marked = __ballot_sync(0xFFFFFFFFu, m);
-      while (marked) {
-        const unsigned j = __ffs(marked) - 1;
-        marked &= marked - 1;
-        unsigned* w = xpl_dctx.pool + (sc * 128 + c0 + j) * 32 + lane;
-        const unsigned v = __ldcg(w);
-        if (v & XPLD_P4) *w = (v & ~XPLD_P4) | ((v & XPLD_P4) >> 1); /* P -> L */
+      if (__ldcg(xpl_dctx.cmap + ch)) {
+        /* lane-per-chunk: the lane folds its own 128-word chunk (32 u32, one
+         * 128 B line, 8 x 16 B loads in flight together), so a round of 32
+         * chunks costs one round trip.  No hook runs between the two grid
+         * barriers, so whole-vector stores race with nothing. */
+        uint4* w = reinterpret_cast<uint4*>(xpl_dctx.pool + ch * 32);
+        uint4 v[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) v[k] = __ldcg(w + k);
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+          const unsigned any = (v[k].x | v[k].y | v[k].z | v[k].w) & XPLD_P4;
+          if (any) {
+            v[k].x = (v[k].x & ~XPLD_P4) | ((v[k].x & XPLD_P4) >> 1); /* P -> L */
+            v[k].y = (v[k].y & ~XPLD_P4) | ((v[k].y & XPLD_P4) >> 1);
+            v[k].z = (v[k].z & ~XPLD_P4) | ((v[k].z & XPLD_P4) >> 1);
+            v[k].w = (v[k].w & ~XPLD_P4) | ((v[k].w & XPLD_P4) >> 1);
+            w[k] = v[k];
+          }
+        }
+        xpl_dctx.cmap[ch] = 0;
       }
-      if (m) xpl_dctx.cmap[ch] = 0;
     }
     if (lane == 0) xpl_dctx.smap[sc] = 0;
   }
