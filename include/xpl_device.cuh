@@ -404,7 +404,7 @@ static __device__ __forceinline__ T& xpl_write_lat(T& x) {
  * new one, exactly like xpl_kernel_end + xpl_kernel_begin between two launches
  * (trace: KE KB).  Steps: grid barrier (all hooks of the segment have landed),
  * the fold of that segment's pending writes (P -> L, D5) spread over the warps
- * of the grid, grid barrier (reads of the next segment see the new L).  The
+ * of the grid (a warp per marked super-chunk, a lane per marked chunk), grid barrier (reads of the next segment see the new L).  The
  * barrier's release/acquire at gpu scope orders the plain shadow loads of the
  * hooks after the fold.  Must not be called from a non-cooperative launch (the
  * grid barrier would deadlock or fault); a no-op under -DXPL_OFF except for the
