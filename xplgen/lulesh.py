@@ -106,12 +106,20 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs, windows=None, r
     (their REG/FREE stay, so ids match); hooks is then None.  reset: the
     diagnoses' reset flag; final=False: no final frees + diagnose (the
     program's keep_allocs)."""
+    ops = list(lulesh_trace_iter(addrs, spec, s, steps, topo, params, tmp_addrs, windows, reset, final))
+    hooks = None if windows is not None else sum(op[1].size for op in ops if op[0] == "DB")
+    return ops, hooks
+
+
+def lulesh_trace_iter(addrs, spec, s, steps, topo, params, tmp_addrs, windows=None, reset=1, final=True):
+    """lulesh_trace op by op (a generator: the full cfg4 trace, ~4e8 events per
+    timestep, never has to exist at once)."""
     ne, nn, nsym, nblk = sizes(s)
     dom, dtb = addrs[0], addrs[1]
     A = [addrs[2 + k] for k in range(48)]
     u = lambda x: np.asarray(x, dtype=np.uint64)
-    ops = [("REG", a, sp[1], sp[2]) for a, sp in zip(addrs, spec)]
-    hooks = 0 if windows is None else None
+    for a, sp in zip(addrs, spec):
+        yield ("REG", a, sp[1], sp[2])
     sampled = windows is not None
     if sampled:
         tab = {}
@@ -151,7 +159,7 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs, windows=None, r
         else:  # int arrays, and the never-used ones zero-filled as 4-byte words
             h.add(I4(k, np.arange(nb // 4)), 4, W)
     h.add(dtb + 8 * u(np.arange(2 * nblk)), 8, W)
-    ops.append(h.op("HB"))
+    yield h.op("HB")
 
     ptr = lambda k, n: rep(dom + 8 * k, n)
     e = np.arange(ne)
@@ -168,8 +176,8 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs, windows=None, r
 
     for step in range(steps):
         tf, tg = tmp_addrs[step]
-        ops.append(("REG", tf, 8 * 24 * ne, MANAGED))
-        ops.append(("H", dom + 8 * TMP_FORCE, 8, W))
+        yield ("REG", tf, 8 * 24 * ne, MANAGED)
+        yield ("H", dom + 8 * TMP_FORCE, 8, W)
         kernels = []
         # 1 zero forces
         ev = _Ev()
@@ -217,11 +225,11 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs, windows=None, r
             ev.add(D(k, nidx), 8, W)
         kernels.append(ev)
         for ev in kernels:
-            ops += [("KB",), ev.op("DB"), ("KE",)]
-            if hooks is not None:
-                hooks += ev.op("DB")[1].size
-        ops.append(("H", dom + 8 * TMP_FORCE, 8, W))
-        ops.append(("FREE", tf))
+            yield ("KB",)
+            yield ev.op("DB")
+            yield ("KE",)
+        yield ("H", dom + 8 * TMP_FORCE, 8, W)
+        yield ("FREE", tf)
         kernels = []
         # 5 accel
         ev = _Ev()
@@ -252,11 +260,11 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs, windows=None, r
                 ev.add(D(k, nidx), 8, RW)
             kernels.append(ev)
         for ev in kernels:
-            ops += [("KB",), ev.op("DB"), ("KE",)]
-            if hooks is not None:
-                hooks += ev.op("DB")[1].size
-        ops.append(("REG", tg, 8 * 3 * ne, MANAGED))
-        ops.append(("H", dom + 8 * TMP_DVDX, 8, W))
+            yield ("KB",)
+            yield ev.op("DB")
+            yield ("KE",)
+        yield ("REG", tg, 8 * 3 * ne, MANAGED)
+        yield ("H", dom + 8 * TMP_DVDX, 8, W)
         kernels = []
         # 9 kinematics
         ev = _Ev()
@@ -286,11 +294,11 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs, windows=None, r
         ev.add(D(VDOV, e), 8, W)
         kernels.append(ev)
         for ev in kernels:
-            ops += [("KB",), ev.op("DB"), ("KE",)]
-            if hooks is not None:
-                hooks += ev.op("DB")[1].size
-        ops.append(("H", dom + 8 * TMP_DVDX, 8, W))
-        ops.append(("FREE", tg))
+            yield ("KB",)
+            yield ev.op("DB")
+            yield ("KE",)
+        yield ("H", dom + 8 * TMP_DVDX, 8, W)
+        yield ("FREE", tg)
         kernels = []
         lxim, lxip = topo[LXIM].astype(np.int64), topo[LXIP].astype(np.int64)
         # 11 monoq gradient
@@ -350,9 +358,9 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs, windows=None, r
             ev.add(dtb + 8 * u((0 if courant else nblk) + np.arange(nblk)), 8, W)
             kernels.append(ev)
         for ev in kernels:
-            ops += [("KB",), ev.op("DB"), ("KE",)]
-            if hooks is not None:
-                hooks += ev.op("DB")[1].size
+            yield ("KB",)
+            yield ev.op("DB")
+            yield ("KE",)
         # TimeIncrement (host)
         h = _Ev()
         h.add(dtb + 8 * u(np.arange(2 * nblk)), 8, R)
@@ -363,9 +371,9 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs, windows=None, r
         h.add([dom + OFF_TIME], 8, W)
         h.add([dom + OFF_CYCLE], 4, W)
         h.add(dom + OFF_MISC + 4 * u(np.arange(14)), 4, W)
-        ops.append(h.op("HB"))
-        ops.append(("DIAG",) + params + (reset, ()))
+        yield h.op("HB")
+        yield ("DIAG",) + params + (reset, ())
     if final:
-        ops += [("FREE", a) for a in addrs]
-        ops.append(("DIAG",) + params + (reset, ()))
-    return ops, hooks
+        for a in addrs:
+            yield ("FREE", a)
+        yield ("DIAG",) + params + (reset, ())

@@ -69,13 +69,20 @@ def _diag_cells(n, m, d):
 
 
 def sw_trace(addrs, spec, n, m, per_diagonal, tb_every, diag_every, inp, params):
+    return list(sw_trace_iter(addrs, spec, n, m, per_diagonal, tb_every, diag_every, inp, params))
+
+
+def sw_trace_iter(addrs, spec, n, m, per_diagonal, tb_every, diag_every, inp, params):
+    """The CPU twin of xplw_sw, op by op (a generator: cfg3's full trace, ~2e9
+    events, never has to exist at once)."""
     A, B, Hh = addrs
     ld = m + 1
     u64 = lambda x: np.asarray(x, dtype=np.uint64)
-    ops = [("REG", x, s[1], s[2]) for x, s in zip(addrs, spec)]
-    ops.append(batch("HB", A + 4 * u64(np.arange(n)), 4, W))
-    ops.append(batch("HB", B + 4 * u64(np.arange(m)), 4, W))
-    ops.append(batch("HB", Hh + 4 * u64(np.arange((n + 1) * (m + 1))), 4, W))
+    for x, s in zip(addrs, spec):
+        yield ("REG", x, s[1], s[2])
+    yield batch("HB", A + 4 * u64(np.arange(n)), 4, W)
+    yield batch("HB", B + 4 * u64(np.arange(m)), 4, W)
+    yield batch("HB", Hh + 4 * u64(np.arange((n + 1) * (m + 1))), 4, W)
 
     def cell_events(i, j):
         rd = np.concatenate([A + 4 * u64(i - 1), B + 4 * u64(j - 1), Hh + 4 * u64((i - 1) * ld + j - 1),
@@ -87,32 +94,40 @@ def sw_trace(addrs, spec, n, m, per_diagonal, tb_every, diag_every, inp, params)
     if not per_diagonal:
         ii = np.repeat(np.arange(1, n + 1, dtype=np.int64), m)
         jj = np.tile(np.arange(1, m + 1, dtype=np.int64), n)
-        ops += [("KB",), cell_events(ii, jj), ("KE",)]
+        yield ("KB",)
+        yield cell_events(ii, jj)
+        yield ("KE",)
     elif per_diagonal == 2:
         # one launch with a device-side epoch split after every anti-diagonal:
         # the same event sequence as one launch per diagonal (KE KB at a split)
         for d in range(2, n + m + 1):
             i, j = _diag_cells(n, m, d)
-            ops += [("KB",), cell_events(i, j), ("KE",)]
+            yield ("KB",)
+            yield cell_events(i, j)
+            yield ("KE",)
     else:
         for d in range(2, n + m + 1):
             i, j = _diag_cells(n, m, d)
-            ops += [("KB",), cell_events(i, j), ("KE",)]
+            yield ("KB",)
+            yield cell_events(i, j)
+            yield ("KE",)
             if tb_every > 0 and (d - 1) % tb_every == 0:
-                ops.append(batch("HB", Hh + 4 * u64(i * ld + j), 4, R))
+                yield batch("HB", Hh + 4 * u64(i * ld + j), 4, R)
             if diag_every > 0 and (d - 1) % diag_every == 0:
-                ops.append(("DIAG",) + params + (1, ()))
+                yield ("DIAG",) + params + (1, ())
     H = sw_dp(inp["a"], inp["b"])
-    ops.append(batch("HB", Hh + 4 * u64(np.arange((n + 1) * (m + 1))), 4, R))
+    yield batch("HB", Hh + 4 * u64(np.arange((n + 1) * (m + 1))), 4, R)
     rh, ra, rb, _ = sw_traceback(H, inp["a"], inp["b"])
-    ops.append(batch("HB", np.concatenate([Hh + 4 * u64(rh), A + 4 * u64(ra), B + 4 * u64(rb)]), 4, R))
+    yield batch("HB", np.concatenate([Hh + 4 * u64(rh), A + 4 * u64(ra), B + 4 * u64(rb)]), 4, R)
     if per_diagonal != 1:
         ii = np.repeat(np.arange(1, n + 1, dtype=np.int64), m)
         jj = np.tile(np.arange(1, m + 1, dtype=np.int64), n)
-        ops += [("KB",), batch("DB", Hh + 4 * u64(ii * ld + jj), 4, W), ("KE",)]
-    ops += [("FREE", x) for x in addrs]
-    ops.append(("DIAG",) + params + (1, ()))
-    return ops
+        yield ("KB",)
+        yield batch("DB", Hh + 4 * u64(ii * ld + jj), 4, W)
+        yield ("KE",)
+    for x in addrs:
+        yield ("FREE", x)
+    yield ("DIAG",) + params + (1, ())
 
 
 def sw_accesses(n, m, per_diagonal):
