@@ -181,6 +181,123 @@ static __device__ __forceinline__ void xpld_commit(unsigned needers, unsigned q,
   }
 }
 
+/* Test-before-set commit of one shadow u32 q by one lane: bits = the record
+ * bits of the byte lanes rb (read) / wb (written) given the u32's current
+ * value cur (cur unused and 0 for write-only call sites K == W: wG | P does not
+ * depend on the record, so no load is needed and the RED is always issued). */
+template <unsigned K, bool TM>
+static __device__ __forceinline__ void xpld_put(unsigned q, unsigned cur, unsigned rb, unsigned wb) {
+  const unsigned bits = xpld_bits2(cur, rb, wb);
+  if (K == XPL_ACC_W || (cur & bits) != bits) {
+    atomicOr(xpl_dctx.pool + q, bits); /* no return value needed: RED */
+    if (wb) xpld_mark<TM>(q);
+  }
+}
+
+/* OR, over the lanes of group mask gm, of the byte lanes each lane of `mask`
+ * sets in v (a 0xFF-per-record byte mask): four ballots, one per byte lane. */
+static __device__ __forceinline__ unsigned xpld_group_bytes(unsigned mask, unsigned v, unsigned gm) {
+  unsigned u = 0;
+#pragma unroll
+  for (unsigned k = 0; k < 4; ++k)
+    if (__ballot_sync(mask, (v >> (8 * k)) & 1u) & gm) u |= 0xFFu << (8 * k);
+  return u;
+}
+
+/* The lanes of `ones` each access words [g0, g0+nb1] inside ONE shadow u32
+ * (every aligned access of <= 4 words: ints, floats, doubles, ...).  Three
+ * cases, decided warp-uniformly:
+ *  (1) contiguous warp: all 32 lanes, lane l at words G + l*w (w = nb1+1, the
+ *      a[i] of a coalesced kernel) -- the warp covers <= 32 consecutive shadow
+ *      u32s; lane j commits u32 j with the byte lanes the warp covers in it
+ *      (one coalesced shadow load, no grouping work at all);
+ *  (2) one address: every lane on the same u32 (the domain words every thread
+ *      of a kernel reads) -- one REDUX for the byte lanes, one lane commits;
+ *  (3) anything else (gathers, partial warps): groups = maximal runs of
+ *      consecutive lanes on the same u32, their byte lanes from four ballots,
+ *      the group's first lane commits.  Lanes of one u32 in different runs
+ *      commit separately, which is equally exact (atomicOr commutes, every
+ *      commit is tested against the same epoch-start record).
+ * K: the access kind if uniform (compile-time call site), else 0 (per lane). */
+template <unsigned K, bool TM>
+static __device__ __forceinline__ void xpld_one(unsigned ones, unsigned long long g0, unsigned nb1,
+                                                unsigned acc) {
+  constexpr unsigned FULL = 0xFFFFFFFFu;
+  const unsigned lane = xpld_lane();
+  const unsigned q = (unsigned)(g0 >> 2);
+  const unsigned bm = (FULL >> (24 - 8 * nb1)) << (8 * ((unsigned)g0 & 3u));
+  if (ones == FULL) { /* (1) */
+    const unsigned w = nb1 + 1;
+    const unsigned long long G = g0 - (unsigned long long)lane * w;
+    const unsigned glo = (unsigned)G, ghi = (unsigned)(G >> 32);
+    const bool same = __shfl_sync(FULL, glo, 0) == glo && __shfl_sync(FULL, ghi, 0) == ghi &&
+                      __shfl_sync(FULL, nb1, 0) == nb1;
+    const unsigned long long E = G + 32ull * w - 1; /* last word the warp covers */
+    const unsigned Q0 = (unsigned)(G >> 2), nq = (unsigned)(E >> 2) - Q0 + 1;
+    if (__all_sync(FULL, same && nq <= 32 && (K != 0 || w == 1))) {
+      unsigned rb = 0, wb = 0;
+      const unsigned lo = lane == 0 ? glo & 3u : 0u, hi = lane == nq - 1 ? (unsigned)E & 3u : 3u;
+      const unsigned m = lane < nq ? (FULL >> (24 - 8 * (hi - lo))) << (8 * lo) : 0u;
+      if (K != 0) {
+        rb = (K & XPL_ACC_R) ? m : 0u;
+        wb = (K & XPL_ACC_W) ? m : 0u;
+      } else { /* per-lane kinds, one word per lane: byte k of u32 j is lane 4j + k - (G & 3) */
+        const unsigned br = __ballot_sync(FULL, acc & XPL_ACC_R), bw = __ballot_sync(FULL, acc & XPL_ACC_W);
+        const int l0 = 4 * (int)lane - (int)(glo & 3u);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const unsigned sel = 0xFFu << (8 * k);
+          const int l = l0 + k;
+          if ((m & sel) && l >= 0 && l < 32) {
+            if ((br >> l) & 1u) rb |= sel;
+            if ((bw >> l) & 1u) wb |= sel;
+          }
+        }
+      }
+      if (lane < nq) {
+        const unsigned qq = Q0 + lane;
+        xpld_put<K, TM>(qq, K == XPL_ACC_W ? 0u : xpl_dctx.pool[qq], rb, wb);
+      }
+      return;
+    }
+  }
+  const unsigned lead = (unsigned)__ffs(ones) - 1;
+  if (__all_sync(ones, q == __shfl_sync(ones, q, lead))) { /* (2) */
+    unsigned rb, wb;
+    if (K != 0) {
+      const unsigned u = __reduce_or_sync(ones, bm);
+      rb = (K & XPL_ACC_R) ? u : 0u;
+      wb = (K & XPL_ACC_W) ? u : 0u;
+    } else {
+      rb = __reduce_or_sync(ones, (acc & XPL_ACC_R) ? bm : 0u);
+      wb = __reduce_or_sync(ones, (acc & XPL_ACC_W) ? bm : 0u);
+    }
+    if (lane == lead) xpld_put<K, TM>(q, K == XPL_ACC_W ? 0u : xpl_dctx.pool[q], rb, wb);
+    return;
+  }
+  /* (3) */
+  const unsigned cur = K == XPL_ACC_W ? 0u : xpl_dctx.pool[q];
+  if (K != XPL_ACC_W) { /* nothing missing anywhere (a re-touch): done */
+    const unsigned mine = xpld_bits(cur, bm, K ? K : acc);
+    if (!__ballot_sync(ones, (cur & mine) != mine)) return;
+  }
+  const unsigned qp = __shfl_up_sync(ones, q, 1);
+  const bool start = lane == 0 || !((ones >> (lane - 1)) & 1u) || qp != q;
+  const unsigned S = __ballot_sync(ones, start);
+  const unsigned above = S & (0xFFFFFFFEu << lane); /* group starts after this lane */
+  const unsigned gm = (above ? ((1u << (__ffs(above) - 1)) - 1u) : FULL) & (FULL << lane);
+  unsigned rb, wb;
+  if (K != 0) {
+    const unsigned u = xpld_group_bytes(ones, bm, gm);
+    rb = (K & XPL_ACC_R) ? u : 0u;
+    wb = (K & XPL_ACC_W) ? u : 0u;
+  } else {
+    rb = xpld_group_bytes(ones, (acc & XPL_ACC_R) ? bm : 0u, gm);
+    wb = xpld_group_bytes(ones, (acc & XPL_ACC_W) ? bm : 0u, gm);
+  }
+  if (start) xpld_put<K, TM>(q, cur, rb, wb);
+}
+
 /* Apply a GPU access to the shadow words [g0, g1] (global pool word indices;
  * empty when g0 > g1).  All active lanes of the calling warp must call it.
  * K: the access kind if uniform over the warp (a compile-time call site), else 0. */
@@ -189,30 +306,18 @@ static __device__ __forceinline__ void xpl_dev_apply(unsigned long long g0,
                                                      unsigned long long g1,
                                                      unsigned acc) {
   const unsigned active = __activemask();
-  const bool single = g0 >= g1; /* one word (g0 == g1) or none (g0 > g1) */
-  const unsigned singles = __ballot_sync(active, single);
-  if (single) { /* the short path */
-    const bool hit = g0 == g1;
-    const unsigned q = (unsigned)(g0 >> 2);
-    const unsigned bytes = 0xFFu << (8 * (unsigned)(g0 & 3));
-    unsigned cur = 0, m = 0;
-    if (hit) {
-      /* a write's bits (wG | P) do not depend on L: write-only call sites skip
-       * the shadow load (and its latency) and always commit */
-      cur = K == XPL_ACC_W ? 0u : xpl_dctx.pool[q];
-      m = xpld_bits(cur, bytes, acc);
-    }
-    const bool need = hit && (K == XPL_ACC_W || (cur & m) != m);
-    const unsigned needers = __ballot_sync(singles, need);
-    if (need) xpld_commit<K, true, TM>(needers, q, cur, bytes, acc);
-  }
-  if (singles == active) return;
-  /* multi-word accesses: one shadow u32 per iteration */
-  const bool multi = g0 < g1;
+  const bool hit = g0 <= g1;
+  const bool one = hit && (g0 >> 2) == (g1 >> 2); /* inside one shadow u32 */
+  const unsigned ones = __ballot_sync(active, one);
+  if (one) xpld_one<K, TM>(ones, g0, (unsigned)(g1 - g0), acc);
+  const bool multi = hit && !one;
+  const unsigned multis = __ballot_sync(active, multi);
+  if (!multi) return;
+  /* accesses over several shadow u32s: one u32 per iteration */
   unsigned long long q = g0 >> 2;
   const unsigned long long ql = g1 >> 2;
-  bool more = multi;
-  while (__any_sync(active, more)) {
+  bool more = true;
+  while (__any_sync(multis, more)) {
     unsigned cur = 0, m = 0, bytes = 0;
     if (more) {
       cur = K == XPL_ACC_W ? 0u : xpl_dctx.pool[q];
@@ -224,7 +329,7 @@ static __device__ __forceinline__ void xpl_dev_apply(unsigned long long g0,
       m = xpld_bits(cur, bytes, acc);
     }
     const bool need = more && (K == XPL_ACC_W || (cur & m) != m);
-    const unsigned needers = __ballot_sync(active, need);
+    const unsigned needers = __ballot_sync(multis, need);
     if (need) xpld_commit<K, false, TM>(needers, (unsigned)q, cur, bytes, acc);
     more = more && q < ql;
     ++q;

@@ -20,6 +20,7 @@
 #include <stdint.h>
 
 #include <chrono>
+#include <vector>
 
 #include "xpl.h"
 #include "xpl_device.cuh"
@@ -426,15 +427,37 @@ int xplw_lulesh(xplw_run* run, const xplw_arrays* arr, int s, int steps, unsigne
       ok(x);
     }
   };
-  // one instrumented launch = one GPU epoch (the kernel-launch wrapper)
+  // one instrumented launch = one GPU epoch (the kernel-launch wrapper);
+  // time_kernels: CUDA events around the kernel alone (its epoch close excluded)
+  std::vector<cudaEvent_t> evs;
+  auto mark = [&]() {
+    if (!run->time_kernels) return;
+    cudaEvent_t e;
+    okc(cudaEventCreate(&e));
+    okc(cudaEventRecord(e, st));
+    evs.push_back(e);
+  };
   auto launch = [&](auto fi, auto ft, int grid) {
     flush();
     if (on) ok(xpl_kernel_begin(run->ctx, st));
+    mark();
     if (on) fi(grid);
     else ft(grid);
+    mark();
     okc(cudaGetLastError());
     if (on) ok(xpl_kernel_end(run->ctx, st));
     run->epochs++;
+  };
+  auto sum_events = [&]() {
+    if (evs.empty()) return;
+    okc(cudaStreamSynchronize(st));
+    for (size_t i = 0; i + 1 < evs.size(); i += 2) {
+      float ms = 0.f;
+      cudaEventElapsedTime(&ms, evs[i], evs[i + 1]);
+      run->kernel_ms += ms;
+    }
+    for (cudaEvent_t e : evs) cudaEventDestroy(e);
+    evs.clear();
   };
 #define LAUNCH(KER, GRID, ...)                                                          \
   launch([&](int g) { KER<true><<<g, 256, 0, st>>>(__VA_ARGS__); },                    \
@@ -554,12 +577,14 @@ int xplw_lulesh(xplw_run* run, const xplw_arrays* arr, int s, int steps, unsigne
   if (run->keep_allocs) {
     if (on) ok(xpl_sync(run->ctx));
     okc(cudaStreamSynchronize(st));
+    sum_events();
     return run->status;
   }
   if (on)
     for (int k = 0; k < arr->n; ++k) ok(xpl_free(run->ctx, (const void*)arr->addr[k]));
   diag();
   okc(cudaStreamSynchronize(st));
+  sum_events();
   return run->status;
 }
 

@@ -20,6 +20,17 @@ __global__ void replay_kernel(const unsigned long long* __restrict__ addr,
     xpl_dev_record((const void*)addr[i], size[i], acc[i]);
 }
 
+// The replay with a compile-time access kind (every event of the launch has
+// kind K): the K-uniform form of the hooks that xpl_read / xpl_write / xpl_rw
+// call sites use (fast paths of xpl_device.cuh).
+template <unsigned K>
+__global__ void replay_k_kernel(const unsigned long long* __restrict__ addr,
+                                const unsigned int* __restrict__ size, unsigned long long n) {
+  for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (unsigned long long)gridDim.x * blockDim.x)
+    xpl_dev_record_k<K>((const void*)addr[i], size[i], K);
+}
+
 // The same replay as ONE cooperative launch over several epochs: segment k is
 // events [seg[k], seg[k+1]); a device-side epoch split (xpl_grid_epoch,
 // NEXT-2) separates consecutive segments.  Equal to one launch per segment.
@@ -86,6 +97,25 @@ __global__ void atomic_bench_kernel(unsigned* p, unsigned long long n, int mode,
   if (mode == 1 && acc == 0x9E3779B9u) *sink = acc;  // keep the return values live
 }
 
+// Streaming user kernel with real data (the recording roofline and the
+// slowdown floor of a bandwidth-bound kernel): y[i] = x[i] + x[i]
+// over n elements of T, every read through traceR and every write through
+// traceW (I = instrumented), or the uninstrumented twin (I = false).
+template <class T, bool I>
+__global__ void __launch_bounds__(256) stream_kernel(const T* __restrict__ x, T* __restrict__ y,
+                                                     unsigned long long n) {
+  for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (unsigned long long)gridDim.x * blockDim.x) {
+    if constexpr (I) {
+      const T v = xpl_read(x[i]);
+      xpl_write(y[i]) = v + v;
+    } else {
+      const T v = x[i];
+      y[i] = v + v;
+    }
+  }
+}
+
 // A user kernel that really touches memory (managed memory for the UM-counter
 // check, NEXT-4): word k*stride of base for k < n/stride is read (write = 0) or
 // incremented (write = 1: read then write, hooked as RW), hooks on.
@@ -143,6 +173,25 @@ int xplw_touch_mem(void* base, unsigned long long n_words, unsigned long long st
   return cudaGetLastError() == cudaSuccess ? 0 : (int)XPL_ERR_CUDA;
 }
 
+// Launch the streaming kernel: elem = 4 or 8 bytes, instrumented (between
+// xpl_kernel_begin/_end) or the twin; one wave of 148 x 8 CTAs, grid-stride.
+int xplw_stream(const void* x, void* y, unsigned long long n, int elem, int instrumented, void* stream) {
+  cudaStream_t s = (cudaStream_t)stream;
+  const unsigned g = 148 * 8;
+  if (elem == 4) {
+    if (instrumented) stream_kernel<unsigned, true><<<g, 256, 0, s>>>((const unsigned*)x, (unsigned*)y, n);
+    else stream_kernel<unsigned, false><<<g, 256, 0, s>>>((const unsigned*)x, (unsigned*)y, n);
+  } else if (elem == 8) {
+    if (instrumented) stream_kernel<unsigned long long, true><<<g, 256, 0, s>>>(
+        (const unsigned long long*)x, (unsigned long long*)y, n);
+    else stream_kernel<unsigned long long, false><<<g, 256, 0, s>>>(
+        (const unsigned long long*)x, (unsigned long long*)y, n);
+  } else {
+    return (int)XPL_ERR_INVALID_ARG;
+  }
+  return cudaGetLastError() == cudaSuccess ? 0 : (int)XPL_ERR_CUDA;
+}
+
 int xplw_atomic_bench(void* buf, unsigned long long n_u32, int mode, void* stream) {
   atomic_bench_kernel<<<148 * 16, 256, 0, (cudaStream_t)stream>>>((unsigned*)buf, n_u32, mode,
                                                                   (unsigned*)buf);
@@ -179,6 +228,20 @@ int xplw_replay(const unsigned long long* d_addr, const unsigned int* d_size,
                 void* stream) {
   if (n == 0) return 0;
   replay_kernel<<<grid, block, 0, (cudaStream_t)stream>>>(d_addr, d_size, d_acc, n);
+  return cudaGetLastError() == cudaSuccess ? 0 : (int)XPL_ERR_CUDA;
+}
+
+// Launch the K-uniform replay kernel (kind = 1 R, 2 W, 3 RW) on `stream`.
+int xplw_replay_k(const unsigned long long* d_addr, const unsigned int* d_size, unsigned long long n,
+                  int kind, int grid, int block, void* stream) {
+  if (n == 0) return 0;
+  cudaStream_t s = (cudaStream_t)stream;
+  switch (kind) {
+    case XPL_ACC_R: replay_k_kernel<XPL_ACC_R><<<grid, block, 0, s>>>(d_addr, d_size, n); break;
+    case XPL_ACC_W: replay_k_kernel<XPL_ACC_W><<<grid, block, 0, s>>>(d_addr, d_size, n); break;
+    case XPL_ACC_RW: replay_k_kernel<XPL_ACC_RW><<<grid, block, 0, s>>>(d_addr, d_size, n); break;
+    default: return (int)XPL_ERR_INVALID_ARG;
+  }
   return cudaGetLastError() == cudaSuccess ? 0 : (int)XPL_ERR_CUDA;
 }
 

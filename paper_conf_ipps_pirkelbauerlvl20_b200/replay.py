@@ -66,14 +66,17 @@ def _dev_arrays(evs):
 
 
 def run_trace(ops, ctx: Context | None = None, grid=0, block=256, seed=None, host_split=None,
-              pool_words=1 << 24, stream=None, split_epochs=False, traced=False):
+              pool_words=1 << 24, stream=None, split_epochs=False, traced=False, uniform=False):
     """Replay `ops`.  seed: shuffle device events inside every epoch and split
     host batches at random points (metamorphic variants); grid/block: launch
     shape of the replay kernel (grid 0 = enough CTAs for one event each);
     split_epochs: chains of consecutive epochs run as one cooperative launch
     with device-side epoch splits (xpl_grid_epoch) -- must give the same reports;
     traced: device events are launched through the kernel-launch wrapper
-    (xpl_trace_kernel_launch, nested into the trace's epoch) -- same reports."""
+    (xpl_trace_kernel_launch, nested into the trace's epoch) -- same reports;
+    uniform: an epoch's device events are launched as one K-uniform replay per
+    access kind (the compile-time-kind hooks of xpl_read/_write/_rw call sites;
+    order inside an epoch does not matter, D5) -- same reports."""
     import torch
 
     if split_epochs:
@@ -112,6 +115,19 @@ def run_trace(ops, ctx: Context | None = None, grid=0, block=256, seed=None, hos
         if rng is not None:
             p = rng.permutation(a.size)
             a, s, k = a[p], s[p], k[p]
+        if uniform:
+            keep = []
+            for kind in (1, 2, 3):
+                m = k == kind
+                if not m.any():
+                    continue
+                ta = torch.from_numpy(np.ascontiguousarray(a[m]).view(np.int64)).cuda()
+                ts = torch.from_numpy(np.ascontiguousarray(s[m]).view(np.int32)).cuda()
+                keep += [ta, ts]
+                ctx.replay_k(ta.data_ptr(), ts.data_ptr(), int(m.sum()), kind, grid=grid, block=block,
+                             stream=stream)
+            torch.cuda.current_stream().synchronize()
+            return
         ta = torch.from_numpy(a.view(np.int64)).cuda()
         ts = torch.from_numpy(s.view(np.int32)).cuda()
         tk = torch.from_numpy(k).cuda()

@@ -172,6 +172,8 @@ if _work is not None:
     xplw_replay_split = _sig("xplw_replay_split", [vp, vp, vp, vp, i32, i32, i32, vp], lib=_work)
     xplw_atomic_bench = _sig("xplw_atomic_bench", [vp, u64, i32, vp], lib=_work)
     xplw_touch = _sig("xplw_touch", [u64, u64, u32, vp, u64], lib=_work)
+    xplw_stream = _sig("xplw_stream", [vp, vp, u64, i32, i32, vp], lib=_work)
+    xplw_replay_k = _sig("xplw_replay_k", [vp, vp, u64, i32, i32, i32, vp], lib=_work)
     # (optional so that A/B builds of the workload library without it still load)
     xplw_read_lat = (_sig("xplw_read_lat", [vp, u64, i32, i32, i32, vp], lib=_work)
                      if hasattr(_work, "xplw_read_lat") else None)
@@ -389,10 +391,22 @@ class Context:
             grid = max(1, min((n + block - 1) // block, 148 * 8))
         check("xplw_replay", xplw_replay(d_addr, d_size, d_acc, n, grid, block, stream))
 
+    def replay_k(self, d_addr, d_size, n, kind, grid=0, block=256, stream=0):
+        """The replay kernel with one compile-time access kind for all n events."""
+        if grid <= 0:
+            grid = max(1, min((n + block - 1) // block, 148 * 8))
+        check("xplw_replay_k", xplw_replay_k(d_addr, d_size, n, kind, grid, block, stream))
+
     def replay_split(self, d_addr, d_size, d_acc, d_seg, nseg, grid=0, block=256, stream=0):
         """One cooperative launch of the replay kernel over nseg epochs separated by
         device-side epoch splits (xpl_grid_epoch); d_seg = nseg+1 event offsets."""
         check("xplw_replay_split", xplw_replay_split(d_addr, d_size, d_acc, d_seg, nseg, grid, block, stream))
+
+
+def stream_kernel(x_ptr, y_ptr, n, elem, instrumented, stream=0):
+    """y[i] = 2 x[i] over n elements of `elem` bytes (4 or 8): the instrumented
+    streaming kernel (inside an epoch) or its twin (libxplwork.so)."""
+    check("xplw_stream", xplw_stream(x_ptr, y_ptr, n, elem, int(bool(instrumented)), stream))
 
 
 def atomic_bench(buf_ptr, n_u32, mode, stream=0):

@@ -1,0 +1,40 @@
+#!/bin/bash
+# One gpurun job (replaces the per-run scripts of round 1):
+#   gpurun --timeout S -- bash tools/gpu_job.sh TAG STEP [STEP ...]
+# Runs the steps in order on the GPU box; every step logs to gpurun_out/TAG_<step>.*
+# Steps:
+#   build                  make the libraries (they normally travel in-tree)
+#   smoke                  __graft_entry__.smoke()
+#   pytest[:ARGS]          python -m pytest tests -q -m gpu ARGS  (ARGS: '+'-separated, e.g. -k+lulesh)
+#   bench[:ARGS]           python bench.py ARGS > TAG_bench.json
+#   launches               ncu launch list (gpu__time_duration.sum) of a short bench run
+#   ncu:REGEX[:SKIP[:CMD]] ncu --set full of one launch of kernel REGEX (default command: bench.py --step-only)
+#   py:SCRIPT[:ARGS]       python SCRIPT ARGS > TAG_<name>.json
+TAG=$1; shift
+mkdir -p gpurun_out
+echo "nproc=$(nproc) $(nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv,noheader)" > gpurun_out/${TAG}_box.txt
+for step in "$@"; do
+  kind=${step%%:*}; rest=${step#*:}; [ "$rest" = "$step" ] && rest=""
+  args=${rest//+/ }
+  case $kind in
+    build) make -s -C paper_conf_ipps_pirkelbauerlvl20_b200/csrc -j8 > gpurun_out/${TAG}_build.log 2>&1 ;;
+    smoke) python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/${TAG}_smoke.log 2>&1
+           echo "rc=$?" >> gpurun_out/${TAG}_smoke.log ;;
+    pytest) timeout 2400 python -m pytest tests -q -m gpu --durations=15 $args > gpurun_out/${TAG}_pytest.log 2>&1
+            echo "pytest rc=$?" >> gpurun_out/${TAG}_pytest.log ;;
+    bench) timeout 1800 python bench.py $args > gpurun_out/${TAG}_bench.json 2> gpurun_out/${TAG}_bench.err ;;
+    launches) timeout 1200 ncu --metrics gpu__time_duration.sum --clock-control none -c 2000 --csv \
+                --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 1 --warmup 1 --step-only \
+                > gpurun_out/${TAG}_launches.log 2>&1 ;;
+    ncu) re=${rest%%:*}; r2=${rest#*:}; [ "$r2" = "$rest" ] && r2=""
+         skip=${r2%%:*}; cmd=${r2#*:}; [ "$cmd" = "$r2" ] && cmd=""
+         [ -z "$skip" ] && skip=0; [ -z "$cmd" ] && cmd="bench.py --step-only --steps 1 --warmup 0"
+         name=$(echo "$re" | tr -cd 'A-Za-z0-9_')
+         timeout 1200 ncu --set full --import-source on --clock-control none -k "regex:$re" --launch-skip $skip \
+           --launch-count 1 -o gpurun_out/${TAG}_ncu_$name python ${cmd//+/ } > gpurun_out/${TAG}_ncu_$name.log 2>&1 ;;
+    py) script=${rest%%:*}; a2=${rest#*:}; [ "$a2" = "$rest" ] && a2=""
+        name=$(basename "$script" .py)
+        timeout 1800 python $script ${a2//+/ } > gpurun_out/${TAG}_$name.json 2> gpurun_out/${TAG}_$name.err ;;
+    *) echo "unknown step $step" >> gpurun_out/${TAG}_box.txt ;;
+  esac
+done
