@@ -158,7 +158,13 @@ xpl_status xpl_free(xpl_ctx* ctx, const void* ptr);
  * `stream` after all pending runtime work; end orders the runtime after
  * `stream` (and every stream that began inside the epoch) and enqueues the
  * epoch close (fold).  Nothing synchronises the host.  end without an open
- * epoch -> STATE. */
+ * epoch -> STATE.
+ * Stream lifetime: after an epoch whose kernels all ran on one (non-default)
+ * stream, the epoch close is enqueued right behind them on that stream and the
+ * runtime keeps using it for its next work (no cross-stream event for the next
+ * epoch there).  Such a stream must stay valid until xpl_release_stream() names
+ * it or xpl_finalize(); the legacy / per-thread default streams are never
+ * adopted. */
 xpl_status xpl_kernel_begin(xpl_ctx* ctx, void* stream);
 xpl_status xpl_kernel_end(xpl_ctx* ctx, void* stream);
 
@@ -191,7 +197,8 @@ xpl_status xpl_record_copy(xpl_ctx* ctx, const void* dst, const void* src, size_
  * last reset, write one report per row in id order into out[0..cap), set
  * *n_out.  INVALID_ARG with *n_out = rows needed if cap is too small.  With
  * reset != 0 the interval bits are cleared (the last writer is kept, D4) and
- * freed rows are dropped.  STATE inside an open epoch.  Blocks until done.
+ * freed rows are dropped.  STATE inside an open epoch, or (like xpl_sync) after
+ * a forbidden device-side split.  Blocks until done.
  * params NULL = defaults; names may be NULL when n_names == 0. */
 xpl_status xpl_diagnose(xpl_ctx* ctx, const xpl_diag_params* params, const xpl_name* names,
                         size_t n_names, xpl_alloc_report* out, size_t cap, size_t* n_out,
@@ -360,8 +367,14 @@ const char* xpl_launch_name(xpl_ctx* ctx, uint32_t idx);
 /* Apply every staged host record now (normally done lazily at kernel_begin,
  * diagnose and when staging fills up).  Asynchronous. */
 xpl_status xpl_flush(xpl_ctx* ctx);
-/* Wait for all runtime work enqueued so far. */
+/* Wait for all runtime work enqueued so far.  STATE if a device-side epoch split
+ * (xpl_grid_epoch) ran in an epoch with several streams or with D2D / memset
+ * shadow work (reported once; the records of that epoch are unreliable). */
 xpl_status xpl_sync(xpl_ctx* ctx);
+/* The runtime stops using `stream` for its own work (moves it back onto its own
+ * stream, ordered after everything enqueued on `stream` so far).  Call before
+ * destroying a stream that ended an epoch.  STATE inside an epoch. */
+xpl_status xpl_release_stream(xpl_ctx* ctx, void* stream);
 /* Make `stream` (cudaStream_t as void*) wait on the device for every runtime
  * operation enqueued so far (host merges, transfers' shadow updates, the last
  * epoch's fold).  Runtime work runs on the runtime's own stream, or on the

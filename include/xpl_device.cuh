@@ -58,6 +58,7 @@ struct xpl_dev_ctx {
   unsigned char* cmap;            /* 1 byte per 128-word chunk: GPU write pending */
   unsigned char* smap;            /* 1 byte per 128 chunks (16K words)            */
   const unsigned long long* n_super; /* super-chunks below the pool's high-water mark */
+  unsigned int* flags;            /* [0]: a device-side epoch split ran in the open epoch */
 };
 
 #ifdef __CUDACC__
@@ -513,11 +514,19 @@ static __device__ __forceinline__ T& xpl_write_lat(T& x) {
  * barrier's release/acquire at gpu scope orders the plain shadow loads of the
  * hooks after the fold.  Must not be called from a non-cooperative launch (the
  * grid barrier would deadlock or fault); a no-op under -DXPL_OFF except for the
- * barrier itself, which keeps the twin's control flow. */
+ * barrier itself, which keeps the twin's control flow.  The fold stores whole
+ * shadow vectors, so nothing else may record into the pool while it runs: the
+ * epoch holding the launch must have a single stream and no D2D / memset
+ * shadow work of the runtime (xpl_record_copy inside the epoch); the epoch
+ * close checks this and the next xpl_sync / xpl_diagnose returns XPL_ERR_STATE
+ * if it was violated. */
 static __device__ __forceinline__ void xpl_grid_epoch() {
   cooperative_groups::grid_group g = cooperative_groups::this_grid();
   g.sync();
 #ifndef XPL_OFF
+  /* tell the epoch close a split ran: an epoch with a split must be one stream
+   * without runtime range work of its own (else its close reports XPL_ERR_STATE) */
+  if (g.thread_rank() == 0) xpl_dctx.flags[0] = 1u;
   const unsigned lane = xpld_lane();
   const unsigned long long nthreads = (unsigned long long)gridDim.x * gridDim.y * gridDim.z *
                                       blockDim.x * blockDim.y * blockDim.z;

@@ -42,6 +42,8 @@ _w.xplw_lulesh_layout.restype = i32
 _w.xplw_alloc_managed.argtypes = [u64]
 _w.xplw_alloc_managed.restype = vp
 _w.xplw_free_managed.argtypes = [vp]
+_w.xplw_memcpy_async.argtypes = [vp, vp, u64, vp]
+_w.xplw_memcpy_async.restype = i32
 for f in ("xplw_hotspot", "xplw_backprop", "xplw_bfs", "xplw_nw", "xplw_sw", "xplw_free_managed", "xplw_lulesh"):
     getattr(_w, f).restype = i32
 
@@ -198,6 +200,26 @@ def lulesh_prepare(arena: Arena, s, topo):
     for k, arr in topo.items():
         arena.view(L.NAMES[k]).view(np.int32)[:] = arr
     torch.cuda.synchronize()
+
+
+def lulesh_topology_host(topo):
+    """Pinned host copies of the mesh topology (the e2e input upload's source)."""
+    import torch
+    return {k: torch.from_numpy(np.ascontiguousarray(v)).pin_memory() for k, v in topo.items()}
+
+
+def lulesh_upload(arena: Arena, host_topo, stream):
+    """Upload the topology from pinned host memory into the managed arrays on
+    `stream` (cudaMemcpyAsync); returns the bytes copied."""
+    from xplgen import lulesh as L
+    nb = 0
+    for k, t in host_topo.items():
+        a = arena.addrs[[sp[0] for sp in arena.spec].index(L.NAMES[k])]
+        n = t.numel() * t.element_size()
+        if _w.xplw_memcpy_async(a, t.data_ptr(), n, stream):
+            raise xpl.XplError("cudaMemcpyAsync", 6)
+        nb += n
+    return nb
 
 
 def lulesh(run: Run, arena: Arena, s, steps, hook_counter):

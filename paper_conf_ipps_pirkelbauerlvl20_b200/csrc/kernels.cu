@@ -45,8 +45,13 @@ __global__ void __launch_bounds__(kFoldThreads) fold_kernel(uint32_t* __restrict
                                                             uint8_t* __restrict__ cmap,
                                                             uint8_t* __restrict__ smap,
                                                             uint64_t n_super,
-                                                            unsigned long long* stats) {
+                                                            unsigned long long* stats,
+                                                            uint32_t* flags, int strict) {
   asm volatile("griddepcontrol.wait;" ::: "memory");
+  if (blockIdx.x == 0 && threadIdx.x == 0) {  // a device-side split in an epoch that forbids it
+    if (strict && flags[0]) flags[1] = 1u;
+    flags[0] = 0u;
+  }
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   __shared__ uint64_t s_list[kFoldThreads];
   __shared__ uint32_t s_n;
@@ -1095,10 +1100,9 @@ __global__ void __launch_bounds__(256) page_kernel(const PageRow* __restrict__ r
 }  // namespace
 
 void launch_fold(cudaStream_t s, bool pdl, uint32_t* pool, uint8_t* cmap, uint8_t* smap,
-                 uint64_t n_super, unsigned long long* stats) {
-  if (!n_super) return;
+                 uint64_t n_super, unsigned long long* stats, uint32_t* flags, int strict) {
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3((unsigned)(n_super < XPL_FOLD_CTAS ? n_super : XPL_FOLD_CTAS));  // one wave
+  cfg.gridDim = dim3((unsigned)(n_super == 0 ? 1 : n_super < XPL_FOLD_CTAS ? n_super : XPL_FOLD_CTAS));  // one wave
   cfg.blockDim = dim3(kFoldThreads);
   cfg.stream = s;
   cudaLaunchAttribute at[1];
@@ -1106,7 +1110,7 @@ void launch_fold(cudaStream_t s, bool pdl, uint32_t* pool, uint8_t* cmap, uint8_
   at[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = at;
   cfg.numAttrs = pdl ? 1 : 0;
-  cudaLaunchKernelEx(&cfg, fold_kernel, pool, cmap, smap, n_super, stats);
+  cudaLaunchKernelEx(&cfg, fold_kernel, pool, cmap, smap, n_super, stats, flags, strict);
 }
 
 void launch_merge(cudaStream_t s, const uint64_t* recs, uint32_t n, bool has_r, bool has_w,

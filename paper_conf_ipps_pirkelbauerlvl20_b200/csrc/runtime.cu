@@ -106,7 +106,8 @@ struct xpl_ctx {
   // epoch close: chunk maps (1 B per 128 words, 1 B per 16K words) + chunk list
   uint8_t* d_cmap = nullptr;           // 1 byte per 128-word chunk: GPU write pending
   uint8_t* d_smap = nullptr;           // 1 byte per 16K-word super-chunk
-  uint32_t* d_misc = nullptr;          // scratch counters
+  uint32_t* d_misc = nullptr;          // [0] split seen in the open epoch, [1] split in a forbidden epoch
+  uint32_t* h_misc = nullptr;          // pinned mirror of d_misc (read back with the diagnose copies)
   unsigned long long* d_stats = nullptr;
 
   // epochs (D19)
@@ -510,11 +511,13 @@ xpl_status gpu_ranges(xpl_ctx* c, const RangeDesc* rd, size_t nr) {
 
 // Epoch close (D5): the fold on cs.  pdl = it directly follows the
 // epoch's kernels on the same stream (programmatic stream serialization).
-void fold(xpl_ctx* c, bool pdl) {
+// strict = the epoch had several streams or runtime range work of its own, so a
+// device-side split (xpl_grid_epoch) inside it is an error (its fold would race).
+void fold(xpl_ctx* c, bool pdl, bool strict = false) {
   const int pi = prof_begin(c, XPL_K_FOLD, 0);
   // only super-chunks below the pool's high-water mark can be flagged
   launch_fold(c->cs, pdl && pi < 0, (uint32_t*)c->d_pool, c->d_cmap, c->d_smap,
-              (c->pa.hwm + 16383) / 16384, c->d_stats);
+              (c->pa.hwm + 16383) / 16384, c->d_stats, c->d_misc, strict ? 1 : 0);
   c->folds_host++;
   c->st.kernel_launches += 1;
   prof_end(c, pi);
@@ -577,6 +580,17 @@ xpl_status log_epoch_begin(xpl_ctx* c, cudaStream_t s) {
   c->lepoch_no.push_back(c->st.epochs);
   c->lepoch_open = true;
   return XPL_OK;
+}
+
+// A device-side epoch split ran in an epoch that forbids it (see fold()): reported
+// once, by the first blocking call that reads the flags back (h_misc).
+xpl_status split_error(xpl_ctx* c) {
+  if (!c->h_misc[1]) return XPL_OK;
+  c->h_misc[1] = 0;
+  const uint32_t zero = 0;
+  CK(cudaMemcpyAsync(c->d_misc + 1, &zero, 4, cudaMemcpyHostToDevice, c->cs));
+  CK(cudaStreamSynchronize(c->cs));
+  return XPL_ERR_STATE;
 }
 
 }  // namespace
@@ -814,6 +828,8 @@ xpl_status xpl_init(const xpl_config* cfg, xpl_ctx** out) {
   CKI(cudaMemsetAsync(c->d_smap, 0, c->pool_words / 16384, c->cs));
   CKI(cudaMalloc(&c->d_misc, 64));
   CKI(cudaMemsetAsync(c->d_misc, 0, 64, c->cs));
+  CKI(host_alloc(&c->h_misc, 16));
+  memset(c->h_misc, 0, 64);
   CKI(cudaMalloc(&c->d_stats, 64));
   CKI(cudaMemsetAsync(c->d_stats, 0, 64, c->cs));
   c->stage_cap = c->cfg.staging_recs;
@@ -852,6 +868,7 @@ xpl_status xpl_finalize(xpl_ctx* c) {
   cudaFree(c->d_cmap);
   cudaFree(c->d_smap);
   cudaFree(c->d_misc);
+  cudaFreeHost(c->h_misc);
   cudaFree(c->d_stats);
   cudaFreeHost(c->h_stage[0]);
   cudaFreeHost(c->h_stage[1]);
@@ -1021,8 +1038,9 @@ xpl_status xpl_kernel_end(xpl_ctx* c, void* stream) {
     CK(cudaStreamWaitEvent(t, e, 0));
     crossed = true;
   }
+  const bool strict = !single || c->cs_in_epoch;
   c->cs = t;
-  fold(c, !crossed);
+  fold(c, !crossed, strict);
   if (c->lepoch_open) {  // NEXT-4: after the fold, on its stream
     const size_t i = c->lepochs.size() - 1;
     CK(cudaEventRecord(c->lepochs[i].b, c->cs));
@@ -1030,6 +1048,13 @@ xpl_status xpl_kernel_end(xpl_ctx* c, void* stream) {
                        cudaMemcpyDeviceToHost, c->cs));
     CK(cudaEventRecord(c->lepochs[i].c, c->cs));
     c->lepoch_open = false;
+  }
+  if (t == nullptr || t == cudaStreamLegacy || t == cudaStreamPerThread) {
+    // never adopt a default stream as the runtime's stream: it would serialise the
+    // runtime's later work with every blocking stream of the process
+    CK(cudaEventRecord(c->ev_join, t));
+    CK(cudaStreamWaitEvent(c->rs, c->ev_join, 0));
+    c->cs = c->rs;
   }
   if (cudaGetLastError() != cudaSuccess) return XPL_ERR_CUDA;
   std::vector<uint64_t> q;
@@ -1167,17 +1192,14 @@ xpl_status xpl_record_copy(xpl_ctx* c, const void* dst, const void* src, size_t 
     return XPL_OK;
   }
   // GPU-side: D2D = GPU read src + GPU write dst; memset = GPU write dst (D7).
-  RangeDesc rd[2 * 64];
+  // One range per side, of any length (RangeDesc.nw and the range kernel's
+  // vector indices are 64-bit).
+  RangeDesc rd[2];
   size_t nr = 0;
   auto add = [&](uint64_t addr, uint32_t acc) {
     uint64_t g0, nw;
     if (!to_words(c, addr, bytes, &g0, &nw)) return;
-    while (nw && nr < 128) {
-      const uint64_t k = std::min<uint64_t>(nw, kMaxRecWords);
-      rd[nr++] = {g0, k, 0, acc, 1};
-      g0 += k;
-      nw -= k;
-    }
+    rd[nr++] = {g0, nw, 0, acc, 1};
   };
   if (dir == XPL_COPY_D2D) add((uint64_t)src, XPL_ACC_R);
   add((uint64_t)dst, XPL_ACC_W);
@@ -1200,8 +1222,21 @@ xpl_status xpl_flush(xpl_ctx* c) {
 
 xpl_status xpl_sync(xpl_ctx* c) {
   if (!c) return XPL_ERR_INVALID_ARG;
+  CK(cudaMemcpyAsync(c->h_misc, c->d_misc, 8, cudaMemcpyDeviceToHost, c->cs));
   CK(cudaStreamSynchronize(c->cs));
   if (c->cs != c->rs) CK(cudaStreamSynchronize(c->rs));
+  return split_error(c);
+}
+
+xpl_status xpl_release_stream(xpl_ctx* c, void* stream) {
+  if (!c) return XPL_ERR_INVALID_ARG;
+  if (c->depth) return XPL_ERR_STATE;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (c->cs == s && s != c->rs) {  // move the runtime's pending work back onto its own stream
+    CK(cudaEventRecord(c->ev_join, s));
+    CK(cudaStreamWaitEvent(c->rs, c->ev_join, 0));
+    c->cs = c->rs;
+  }
   return XPL_OK;
 }
 
@@ -1225,6 +1260,7 @@ xpl_status xpl_get_device_ctx(xpl_ctx* c, struct xpl_dev_ctx* d) {
   d->cmap = c->d_cmap;
   d->smap = c->d_smap;
   d->n_super = (const unsigned long long*)(c->d_tab + 8);
+  d->flags = c->d_misc;
   return XPL_OK;
 }
 
@@ -1429,7 +1465,10 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
                        cudaMemcpyDeviceToHost, c->cs));
   }
   prof_end(c, pall);
+  CK(cudaMemcpyAsync(c->h_misc, c->d_misc, 8, cudaMemcpyDeviceToHost, c->cs));
   CK(cudaStreamSynchronize(c->cs));
+  s = split_error(c);
+  if (s) return s;
 
   std::vector<uint32_t> name_of(nr, 0xFFFFFFFFu);
   c->cache = nullptr;  // names (XplAllocData): the first name inside a live row

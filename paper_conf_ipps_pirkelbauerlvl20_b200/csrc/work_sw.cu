@@ -254,4 +254,9 @@ void* xplw_alloc_managed(unsigned long long bytes) {
   return cudaMallocManaged(&p, bytes) == cudaSuccess ? p : nullptr;
 }
 int xplw_free_managed(void* p) { return cudaFree(p) == cudaSuccess ? 0 : (int)XPL_ERR_CUDA; }
+// The programs' input upload (bench e2e: pinned host -> managed/device, on a stream).
+int xplw_memcpy_async(void* dst, const void* src, unsigned long long bytes, void* stream) {
+  return cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDefault, (cudaStream_t)stream) == cudaSuccess
+             ? 0 : (int)XPL_ERR_CUDA;
+}
 }

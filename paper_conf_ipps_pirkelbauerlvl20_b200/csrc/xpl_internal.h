@@ -98,7 +98,7 @@ struct DiagParams {
 
 // ---- launchers (kernels.cu) ----
 void launch_fold(cudaStream_t s, bool pdl, uint32_t* pool, uint8_t* cmap, uint8_t* smap,
-                 uint64_t n_super, unsigned long long* stats);
+                 uint64_t n_super, unsigned long long* stats, uint32_t* flags, int strict);
 void launch_merge(cudaStream_t s, const uint64_t* recs, uint32_t n, bool has_r, bool has_w,
                   uint32_t* first_w, uint32_t* pool);
 void launch_range(cudaStream_t s, const RangeDesc* d_ranges, uint32_t nr, uint64_t nvec,

@@ -63,6 +63,9 @@ class XplAllocReport(C.Structure):
     _fields_ = REPORT_FIELDS
 
 
+REPORT_BYTES = C.sizeof(XplAllocReport)
+
+
 class XplPartial(C.Structure):
     _fields_ = [("logical_id", u64), ("word_offset", u64), ("words", u64), ("logical_words", u64),
                 ("logical_bytes", u64), ("base", u64), ("kind", u32), ("live", u32), ("name_idx", u32),
@@ -79,7 +82,8 @@ class XplStats(C.Structure):
 
 
 class XplDevCtx(C.Structure):
-    _fields_ = [("rows", vp), ("n_rows", vp), ("pool", vp), ("cmap", vp), ("smap", vp)]
+    _fields_ = [("rows", vp), ("n_rows", vp), ("pool", vp), ("cmap", vp), ("smap", vp), ("n_super", vp),
+                ("flags", vp)]
 
 
 def _sig(name, args, res=i32, lib=_lib):
@@ -109,6 +113,7 @@ xpl_combine_partials = _sig("xpl_combine_partials", [C.POINTER(XplPartial), sz, 
 xpl_format_reports = _sig("xpl_format_reports", [C.POINTER(XplAllocReport), sz, C.POINTER(XplName), sz, i32,
                                                  i32, C.c_char_p, sz, C.POINTER(sz)])
 xpl_get_device_ctx = _sig("xpl_get_device_ctx", [vp, C.POINTER(XplDevCtx)])
+xpl_release_stream = _sig("xpl_release_stream", [vp, vp])
 xpl_shadow_dump = _sig("xpl_shadow_dump", [vp, vp, u64, u64, vp])
 PAGE_REPORT_FIELDS = [
     ("id", u64), ("base", u64), ("words", u64), ("page_words", u64), ("pages", u64),
@@ -163,7 +168,8 @@ EXPORTED = ["xpl_init", "xpl_finalize", "xpl_register_alloc", "xpl_free", "xpl_k
             "xpl_runtime_stream", "xpl_get_stats", "xpl_status_string", "xpl_profile",
             "xpl_profile_read", "xpl_register_alloc_piece", "xpl_diagnose_partials", "xpl_combine_partials",
             "xpl_format_reports", "xpl_page_summary", "xpl_page_flags", "xpl_mem_advise",
-            "xpl_launch_log_enable", "xpl_kernel_launch", "xpl_launch_log", "xpl_launch_name"]
+            "xpl_launch_log_enable", "xpl_kernel_launch", "xpl_launch_log", "xpl_launch_name",
+            "xpl_release_stream"]
 
 if _work is not None:
     xplw_bind = _sig("xplw_bind", [vp], lib=_work)
@@ -355,6 +361,10 @@ class Context:
     def join(self, stream):
         """Make `stream` wait (on the device) for all runtime work enqueued so far."""
         check("xpl_join", xpl_join(self.h, stream))
+
+    def release_stream(self, stream):
+        """The runtime stops using `stream` (before the caller destroys it)."""
+        check("xpl_release_stream", xpl_release_stream(self.h, stream))
 
     def runtime_stream(self):
         s = vp()
