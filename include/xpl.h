@@ -13,7 +13,8 @@
  *  - "host" arguments are host pointers; the library copies what it needs
  *    before returning, so the caller may reuse its buffers at once;
  *  - one host thread per context; one context per process and GPU.  With
- *    world > 1 every rank makes every call, in the same order;
+ *    world > 1 (sharded mode, below) every rank makes every call marked
+ *    COLLECTIVE, in the same order;
  *  - `stream` arguments are cudaStream_t values passed as void*.
  */
 #ifndef XPL_H
@@ -89,14 +90,67 @@ typedef struct {
   uint32_t elem_size;
 } xpl_name;
 
+/* ---- Sharded mode (world > 1) --------------------------------
+ * One logical program runs SPMD over `world` processes, one GPU each; its shadow
+ * memory is partitioned over the ranks' pools by logical word:
+ *  - every allocation is registered by every rank (COLLECTIVE, same bytes and
+ *    kind in the same order; the address may differ per rank -- each rank's
+ *    table maps ITS address range).  An allocation of < 65536 words is owned
+ *    whole by rank (logical id mod world); a larger one is cut into world
+ *    pieces of ceil(words / world) words rounded up to 1024 (4 KiB), piece r
+ *    owned by rank r.  Logical ids count registrations, as with one rank;
+ *  - device hooks record into the owner's pool: local atomics for owned words,
+ *    atomics over NVLink/NVSwitch into the peer-mapped pool for the others;
+ *  - host records: between two collective calls each rank records its own
+ *    slice of the logical host stream; the slices are ordered by rank (the
+ *    logical host stream = rank 0's slice, then rank 1's, ...).  At the next
+ *    collective call the records are routed to their owners (all-to-all) and
+ *    merged there in that order;
+ *  - epochs are collective (all ranks' kernels between kernel_begin/_end form
+ *    one GPU epoch); the close waits for every rank's kernels (barrier) before
+ *    each owner folds its pool;
+ *  - xpl_diagnose is collective: each owner analyses its pieces, the partials
+ *    are exchanged (all-gather) and combined on every rank: every rank gets the
+ *    same reports, equal to the unsharded run's (field `base`: the piece-0
+ *    owner's address);
+ *  - xpl_record_copy is collective; rank 0's call is the one recorded.
+ * Reading D36: pieces are cut on 4 KiB boundaries of the
+ * allocation, so only an access that is not aligned to its size can straddle
+ * two pieces; such an access records only its words in the first piece.
+ *
+ * The collectives, on HOST buffers, blocking; every rank calls them in the same
+ * order.  Return 0 on success.  Provided by xpl_comm_nccl_create (NCCL over
+ * NVLink / NVSwitch) or by the caller (e.g. a gloo process group). */
+typedef struct {
+  void* user;
+  /* recv[world * bytes] = every rank's send[bytes], in rank order */
+  int (*allgather)(void* user, const void* send, size_t bytes, void* recv);
+  /* rank r sends send_bytes[q] bytes (packed in q order in send) to every rank q
+   * and receives recv_bytes[q] bytes from every q (packed in q order in recv) */
+  int (*alltoallv)(void* user, const void* send, const uint64_t* send_bytes, void* recv,
+                   const uint64_t* recv_bytes);
+  int (*barrier)(void* user);
+} xpl_comm;
+
+#define XPL_MAX_RANKS 8
+
 typedef struct {
   int device;            /* CUDA device ordinal                                   */
-  int rank, world;       /* world > 1 => address-range sharding over the ranks    */
-  void* nccl_comm;       /* ncclComm_t when world > 1, else NULL                  */
+  int rank, world;       /* world > 1 => sharded mode (above), world <= XPL_MAX_RANKS */
+  const xpl_comm* comm;  /* the collectives when world > 1 (kept by pointer), else NULL */
   uint64_t pool_words;   /* shadow pool capacity in words (1 byte each)   */
   uint64_t staging_recs; /* host-record staging capacity (records)                */
   uint32_t max_rows;     /* capacity of the allocation table                      */
 } xpl_config;
+
+/* NCCL collectives for a sharded context: rank 0 creates the id, the caller
+ * broadcasts its 128 bytes (any transport), every rank creates its comm (one
+ * NCCL communicator on `device`; buffers bounce through device memory, the
+ * exchange runs over NVLink / NVSwitch).  *out is owned by the caller until
+ * xpl_comm_nccl_destroy (after xpl_finalize of the contexts using it). */
+xpl_status xpl_comm_nccl_unique_id(uint8_t id[128]);
+xpl_status xpl_comm_nccl_create(const uint8_t id[128], int rank, int world, int device, xpl_comm** out);
+xpl_status xpl_comm_nccl_destroy(xpl_comm* comm);
 
 /* Diagnosis parameters. */
 typedef struct {
@@ -141,7 +195,10 @@ typedef struct {
 /* Create a context on cfg->device.  *out is owned by the caller until
  * xpl_finalize.  Zero fields of cfg take defaults (pool_words 2^28,
  * staging_recs 2^22, max_rows 4096).  Allocates the shadow pool in HBM (plus
- * 1/128 of it for the chunk maps of the epoch close). */
+ * 1/128 of it for the chunk maps of the epoch close).  world > 1: COLLECTIVE;
+ * INVALID_ARG without cfg->comm, with rank outside [0, world) or world >
+ * XPL_MAX_RANKS; the ranks' pools are mapped into each other (CUDA IPC) for the
+ * hooks' remote atomics (every rank's pool_words must be equal). */
 xpl_status xpl_init(const xpl_config* cfg, xpl_ctx** out);
 xpl_status xpl_finalize(xpl_ctx* ctx);
 

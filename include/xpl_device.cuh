@@ -59,6 +59,12 @@ struct xpl_dev_ctx {
   unsigned char* smap;            /* 1 byte per 128 chunks (16K words)            */
   const unsigned long long* n_super; /* super-chunks below the pool's high-water mark */
   unsigned int* flags;            /* [0]: a device-side epoch split ran in the open epoch */
+  /* sharded mode (xpl.h): a row's `off` carries its owner rank in the top byte;
+   * the other ranks' pools and chunk maps are mapped here (CUDA IPC, NVLink) */
+  unsigned int rank, world;
+  unsigned int* pools[XPL_MAX_RANKS];
+  unsigned char* cmaps[XPL_MAX_RANKS];
+  unsigned char* smaps[XPL_MAX_RANKS];
 };
 
 #ifdef __CUDACC__
@@ -179,6 +185,52 @@ static __device__ __forceinline__ void xpld_commit(unsigned needers, unsigned q,
   if (xpld_lane() == (unsigned)(__ffs(grp) - 1)) {
     atomicOr(xpl_dctx.pool + q, xpld_bits2(cur, rb, wb)); /* no return value needed: RED */
     if (wb) xpld_mark<TM>(q);
+  }
+}
+
+/* A row's `off` holds its owner rank in the top byte (sharded mode). */
+#define XPLD_OFF_MASK 0x00FFFFFFFFFFFFFFull
+
+/* Sharded mode: the lanes whose access falls in a piece another rank owns
+ * record it in that rank's pool (peer-mapped, CUDA IPC), with the same bits
+ * and test-before-set as a local hook; lanes on one (owner, shadow u32) are
+ * grouped (match + OR) so one atomic crosses NVLink per group.  Out of line:
+ * remote words are the exception (halo and small shared objects). */
+template <unsigned K>
+static __device__ __noinline__ void xpld_remote(unsigned owner, unsigned long long g0,
+                                                unsigned long long g1, unsigned acc) {
+  unsigned* const P = xpl_dctx.pools[owner];
+  unsigned long long q = g0 >> 2;
+  const unsigned long long ql = g1 >> 2;
+  bool more = true;
+  while (__any_sync(__activemask(), more)) {
+    if (more) {
+      unsigned bytes = 0;
+#pragma unroll
+      for (unsigned k = 0; k < 4; ++k) {
+        const unsigned long long gw = q * 4 + k;
+        if (gw >= g0 && gw <= g1) bytes |= 0xFFu << (8 * k);
+      }
+      const unsigned cur = K == XPL_ACC_W ? 0u : __ldcg(P + q);
+      const unsigned m = xpld_bits(cur, bytes, acc);
+      const bool need = K == XPL_ACC_W || (cur & m) != m;
+      const unsigned needers = __ballot_sync(__activemask(), need);
+      if (need) {
+        const unsigned grp = __match_any_sync(needers, ((unsigned long long)owner << 40) | q);
+        const unsigned bits = __reduce_or_sync(grp, m);
+        if (xpld_lane() == (unsigned)(__ffs(grp) - 1)) {
+          atomicOr(P + q, bits);
+          if (bits & XPLD_P4) {
+            unsigned char* c = xpl_dctx.cmaps[owner] + (q >> 5);
+            unsigned char* sm = xpl_dctx.smaps[owner] + (q >> 12);
+            if (!*c) *c = 1;
+            if (!*sm) *sm = 1;
+          }
+        }
+      }
+    }
+    more = more && q < ql;
+    ++q;
   }
 }
 
@@ -378,16 +430,22 @@ static __device__ __forceinline__ void xpl_dev_record_k(const void* p, unsigned 
     }
   }
   unsigned long long g0 = 1, g1 = 0;
+  unsigned owner = 0;
   if (hit && size > 0) {
     const unsigned long long base = be.x;
     const unsigned long long w0 = (a - base) >> 2;
     unsigned long long wl = (a + size - 1 - base) >> 2;
     const unsigned long long wmax = ow.y - 1;
     if (wl > wmax) wl = wmax;
-    g0 = ow.x + w0;
-    g1 = ow.x + wl;
+    owner = (unsigned)(ow.x >> 56);
+    g0 = (ow.x & XPLD_OFF_MASK) + w0;
+    g1 = (ow.x & XPLD_OFF_MASK) + wl;
   }
-  xpl_dev_apply<K, TM>(g0, g1, K ? K : acc);
+  /* sharded mode: words another rank owns go to its pool over NVLink (rare) */
+  const bool remote = owner != xpl_dctx.rank && g0 <= g1;
+  const unsigned long long l0 = remote ? 1ull : g0, l1 = remote ? 0ull : g1;
+  xpl_dev_apply<K, TM>(l0, l1, K ? K : acc);
+  if (__any_sync(__activemask(), remote) && remote) xpld_remote<K>(owner, g0, g1, K ? K : acc);
 #else
   (void)p; (void)size; (void)acc;
 #endif
@@ -456,12 +514,21 @@ struct xpl_read_proxy {
       }
     }
     unsigned long long g0 = 1, g1 = 0;
+    unsigned owner = 0;
     if (h) {
       const unsigned long long w0 = (a - be.x) >> 2;
       unsigned long long wl = (a + sizeof(T) - 1 - be.x) >> 2;
       if (wl > ow.y - 1) wl = ow.y - 1;
-      g0 = ow.x + w0;
-      g1 = ow.x + wl;
+      owner = (unsigned)(ow.x >> 56);
+      g0 = (ow.x & XPLD_OFF_MASK) + w0;
+      g1 = (ow.x & XPLD_OFF_MASK) + wl;
+    }
+    if (__any_sync(__activemask(), owner != xpl_dctx.rank && h)) {  /* sharded: remote words now */
+      if (owner != xpl_dctx.rank && h) {
+        xpld_remote<XPL_ACC_R>(owner, g0, g1, XPL_ACC_R);
+        g0 = 1;
+        g1 = 0;
+      }
     }
     active = __activemask();
     const bool single = g0 >= g1;

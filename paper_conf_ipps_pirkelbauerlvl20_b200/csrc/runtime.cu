@@ -10,6 +10,7 @@
 #include <string.h>
 
 #include <algorithm>
+#include <array>
 #include <map>
 #include <new>
 #include <string>
@@ -33,6 +34,7 @@ struct Row {
   uint32_t kind;
   bool live, dropped, ever;
   uint32_t advice = 0;  // XPL_ADVICE_* bits (xpl_mem_advise)
+  uint32_t owner = 0;   // rank whose pool holds the shadow (sharded mode; else 0)
 };
 
 // First-fit allocator of shadow-pool ranges (16-word granules so every row
@@ -90,7 +92,19 @@ struct xpl_ctx {
   // shadow pool: 1 byte per word
   uint8_t* d_pool = nullptr;
   uint64_t pool_words = 0;
-  PoolAlloc pa;
+  // every rank's pool allocator: in sharded mode all ranks replay the same
+  // registrations and frees, so each computes every piece's offset identically
+  std::vector<PoolAlloc> pas;
+
+  // sharded mode (world > 1, xpl.h): collectives, routing lists, peer pools
+  int rank = 0, world = 1;
+  const xpl_comm* comm = nullptr;
+  std::vector<std::vector<uint64_t>> route;  // staged host records per owner rank
+  uint64_t n_logical = 0;                    // logical ids handed out by xpl_register_alloc
+  std::unordered_map<uint64_t, std::vector<uint64_t>> lrows;  // logical id -> its rows (pieces)
+  void* peer_pool[XPL_MAX_RANKS] = {};       // IPC-mapped pools / chunk maps of the other ranks
+  void* peer_cmap[XPL_MAX_RANKS] = {};
+  void* peer_smap[XPL_MAX_RANKS] = {};
   uint32_t* d_first_w = nullptr;  // merge scratch, lazily allocated
 
   // shadow memory table
@@ -126,7 +140,7 @@ struct xpl_ctx {
   size_t stage_n = 0, stage_cap = 0, stage_ranges = 0;
   bool stage_has_r = false, stage_has_w = false;
   uint64_t* d_stage = nullptr;
-  std::vector<uint64_t> deferred;      // host records inside an open epoch (D20)
+  std::vector<std::pair<uint32_t, uint64_t>> deferred;  // (owner, record) inside an open epoch (D20)
 
   // merge pieces (records split to <= kPieceWords words)
   uint64_t* h_pieces = nullptr;
@@ -208,11 +222,14 @@ const Row* lookup(xpl_ctx* c, uint64_t addr) {
   return r;
 }
 
-// words [g0, g0+nw) of the access (addr, size), clipped (D1, D18)
-bool to_words(xpl_ctx* c, uint64_t addr, uint64_t size, uint64_t* g0, uint64_t* nw) {
+// words [g0, g0+nw) of the access (addr, size), clipped (D1, D18); *owner =
+// the rank whose pool holds them (sharded mode; D36: clipped to the piece)
+bool to_words(xpl_ctx* c, uint64_t addr, uint64_t size, uint64_t* g0, uint64_t* nw,
+              uint32_t* owner = nullptr) {
   if (size == 0) return false;
   const Row* r = lookup(c, addr);
   if (!r) return false;
+  if (owner) *owner = r->owner;
   const uint64_t w0 = (addr - r->base) >> 2;
   uint64_t wl = (addr + size - 1 - r->base) >> 2;
   if (wl > r->words - 1) wl = r->words - 1;
@@ -222,6 +239,7 @@ bool to_words(xpl_ctx* c, uint64_t addr, uint64_t size, uint64_t* g0, uint64_t* 
 }
 
 xpl_status flush(xpl_ctx* c);
+xpl_status flush_local(xpl_ctx* c);
 
 cudaEvent_t prof_event(xpl_ctx* c) {
   if (!c->prof_free.empty()) {
@@ -253,10 +271,53 @@ uint64_t words_of(const uint64_t* h, size_t n) {
 }
 
 
+// Coalesce record (g0, nw, acc) into `last` when that is exact: same access
+// kind and touching/overlapping words for R or W (idempotent per word),
+// adjacent disjoint words for RW.  Returns whether it did.
+bool coalesce(uint64_t& last, uint64_t g0, uint64_t nw, uint32_t acc, bool* became_range) {
+  const uint32_t la = rec_acc(last);
+  const uint64_t l0 = rec_g0(last), ln = rec_nw(last);
+  if (la != acc) return false;
+  uint64_t u0 = 0, u1 = 0;
+  bool ok = false;
+  if (acc != XPL_ACC_RW) {
+    if (g0 <= l0 + ln && g0 + nw >= l0) {
+      u0 = std::min(g0, l0);
+      u1 = std::max(g0 + nw, l0 + ln);
+      ok = true;
+    }
+  } else if (g0 == l0 + ln) {
+    u0 = l0;
+    u1 = g0 + nw;
+    ok = true;
+  }
+  if (!ok || u1 - u0 > kMaxRecWords) return false;
+  *became_range = ln <= kRangeWords && u1 - u0 > kRangeWords;
+  last = pack_rec(u0, u1 - u0, acc);
+  return true;
+}
+
+// Sharded mode: stage a record on its owner's routing list (sent at the next
+// collective call).  Lists are per owner, so coalescing with the list's last
+// record never reorders accesses of one word.
+xpl_status route_push(xpl_ctx* c, uint32_t owner, uint64_t g0, uint64_t nw, uint32_t acc) {
+  for (; nw > kMaxRecWords; g0 += kMaxRecWords, nw -= kMaxRecWords) {
+    xpl_status s = route_push(c, owner, g0, kMaxRecWords, acc);
+    if (s) return s;
+  }
+  c->st.host_records++;
+  std::vector<uint64_t>& L = c->route[owner];
+  bool rng = false;
+  if (!L.empty() && coalesce(L.back(), g0, nw, acc, &rng)) return XPL_OK;
+  L.push_back(pack_rec(g0, nw, acc));
+  c->st.host_records_packed++;
+  return XPL_OK;
+}
+
 // Append one packed record to staging, coalescing with the previous one when
-// that is exact: same access kind and touching/overlapping words for R or W
-// (idempotent per word), adjacent disjoint words for RW.
-xpl_status stage_push(xpl_ctx* c, uint64_t g0, uint64_t nw, uint32_t acc) {
+// that is exact (coalesce()).  owner: the rank holding the words (sharded mode).
+xpl_status stage_push(xpl_ctx* c, uint64_t g0, uint64_t nw, uint32_t acc, uint32_t owner = 0) {
+  if (c->world > 1) return route_push(c, owner, g0, nw, acc);
   while (nw > kMaxRecWords) {  // split very long ranges (disjoint pieces)
     xpl_status s = stage_push(c, g0, kMaxRecWords, acc);
     if (s) return s;
@@ -265,28 +326,10 @@ xpl_status stage_push(xpl_ctx* c, uint64_t g0, uint64_t nw, uint32_t acc) {
   }
   c->st.host_records++;
   if (c->stage_n) {
-    uint64_t& last = c->h_stage[c->cur][c->stage_n - 1];
-    const uint32_t la = rec_acc(last);
-    const uint64_t l0 = rec_g0(last), ln = rec_nw(last);
-    if (la == acc) {
-      uint64_t u0 = 0, u1 = 0;
-      bool ok = false;
-      if (acc != XPL_ACC_RW) {
-        if (g0 <= l0 + ln && g0 + nw >= l0) {
-          u0 = std::min(g0, l0);
-          u1 = std::max(g0 + nw, l0 + ln);
-          ok = true;
-        }
-      } else if (g0 == l0 + ln) {
-        u0 = l0;
-        u1 = g0 + nw;
-        ok = true;
-      }
-      if (ok && u1 - u0 <= kMaxRecWords) {
-        if (ln <= kRangeWords && u1 - u0 > kRangeWords) c->stage_ranges++;
-        last = pack_rec(u0, u1 - u0, acc);
-        return XPL_OK;
-      }
+    bool rng = false;
+    if (coalesce(c->h_stage[c->cur][c->stage_n - 1], g0, nw, acc, &rng)) {
+      if (rng) c->stage_ranges++;
+      return XPL_OK;
     }
   }
   if (c->stage_n == c->stage_cap) {
@@ -324,12 +367,57 @@ xpl_status ensure_first_w(xpl_ctx* c) {
   return XPL_OK;
 }
 
+// Sharded mode: route every rank's staged records to their owners (all-gather
+// of the per-owner byte counts, then one all-to-all of the records) and apply
+// what this rank received, in source-rank order = the logical host stream's
+// order (xpl.h).  COLLECTIVE.
+xpl_status route_flush(xpl_ctx* c) {
+  const int R = c->world;
+  std::vector<uint64_t> sb(R), all((size_t)R * R), rb(R);
+  for (int q = 0; q < R; ++q) sb[q] = 8 * c->route[q].size();
+  if (c->comm->allgather(c->comm->user, sb.data(), 8 * (size_t)R, all.data())) return XPL_ERR_NCCL;
+  uint64_t tot = 0, any = 0;
+  for (int q = 0; q < R; ++q) {
+    rb[q] = all[(size_t)q * R + c->rank];
+    tot += rb[q];
+  }
+  for (uint64_t v : all) any |= v;
+  if (!any) return XPL_OK;  // (every rank sees the same matrix: all skip together)
+  std::vector<uint64_t> send;
+  for (int q = 0; q < R; ++q) {
+    send.insert(send.end(), c->route[q].begin(), c->route[q].end());
+    c->route[q].clear();
+  }
+  std::vector<uint64_t> recv(tot / 8 + 1);
+  if (c->comm->alltoallv(c->comm->user, send.data(), sb.data(), recv.data(), rb.data())) return XPL_ERR_NCCL;
+  const size_t n = tot / 8;
+  for (size_t i = 0; i < n;) {
+    const size_t k = std::min(n - i, c->stage_cap);
+    memcpy(c->h_stage[c->cur], recv.data() + i, 8 * k);
+    c->stage_n = k;
+    c->stage_ranges = 0;
+    c->stage_has_r = c->stage_has_w = false;
+    for (size_t j = 0; j < k; ++j) {
+      const uint64_t r = recv[i + j];
+      if (rec_acc(r) & XPL_ACC_R) c->stage_has_r = true;
+      if (rec_acc(r) & XPL_ACC_W) c->stage_has_w = true;
+      if (rec_nw(r) > kRangeWords) c->stage_ranges++;
+    }
+    xpl_status s = flush_local(c);
+    if (s) return s;
+    i += k;
+  }
+  return XPL_OK;
+}
+
+xpl_status flush(xpl_ctx* c) { return c->world > 1 ? route_flush(c) : flush_local(c); }
+
 // Apply all staged host records on the runtime stream, in order.  Records of
 // more than kRangeWords words cut the batch and go through range_apply (runs of
 // pairwise-disjoint ones share a launch); everything between them is one merge
 // segment, with records longer than kPieceWords split into consecutive pieces
 // (pieces of one record are disjoint, so program order is kept).
-xpl_status flush(xpl_ctx* c) {
+xpl_status flush_local(xpl_ctx* c) {
   if (c->stage_n == 0) return XPL_OK;
   const size_t n = c->stage_n;
   uint64_t* h = c->h_stage[c->cur];
@@ -464,12 +552,12 @@ xpl_status upload_table(xpl_ctx* c) {
     const Row& r = c->rows[kv.second];
     hr[n].base = r.base;
     hr[n].end = r.base + r.bytes;
-    hr[n].off = r.off;
+    hr[n].off = r.off | (uint64_t)r.owner << 56;  // the owner rank rides in the top byte
     hr[n].words = r.words;
     ++n;
   }
   memcpy(c->h_tab, &n, sizeof n);
-  const unsigned long long n_super = (c->pa.hwm + 16383) / 16384;  // for xpl_grid_epoch
+  const unsigned long long n_super = (c->pas[c->rank].hwm + 16383) / 16384;  // for xpl_grid_epoch
   memcpy(c->h_tab + 8, &n_super, sizeof n_super);
   CK(cudaMemcpyAsync(c->d_tab, c->h_tab, 32 + sizeof(xpl_dev_row) * n, cudaMemcpyHostToDevice, c->cs));
   CK(cudaEventRecord(c->table_ev, c->cs));
@@ -517,7 +605,7 @@ void fold(xpl_ctx* c, bool pdl, bool strict = false) {
   const int pi = prof_begin(c, XPL_K_FOLD, 0);
   // only super-chunks below the pool's high-water mark can be flagged
   launch_fold(c->cs, pdl && pi < 0, (uint32_t*)c->d_pool, c->d_cmap, c->d_smap,
-              (c->pa.hwm + 16383) / 16384, c->d_stats, c->d_misc, strict ? 1 : 0);
+              (c->pas[c->rank].hwm + 16383) / 16384, c->d_stats, c->d_misc, strict ? 1 : 0);
   c->folds_host++;
   c->st.kernel_launches += 1;
   prof_end(c, pi);
@@ -709,7 +797,7 @@ static xpl_status page_pass(xpl_ctx* c, const std::vector<const Row*>& rows, uin
 
 xpl_status xpl_page_summary(xpl_ctx* c, uint64_t P, xpl_page_report* out, size_t cap, size_t* n_out) {
   if (!c || !n_out || P == 0 || (cap && !out)) return XPL_ERR_INVALID_ARG;
-  if (c->depth) return XPL_ERR_STATE;
+  if (c->depth || c->world > 1) return XPL_ERR_STATE;  // (the page view is single-GPU)
   std::vector<const Row*> rows;
   for (const Row& r : c->rows)
     if (r.live) rows.push_back(&r);  // (c->rows is in id order)
@@ -748,7 +836,7 @@ xpl_status xpl_page_summary(xpl_ctx* c, uint64_t P, xpl_page_report* out, size_t
 
 xpl_status xpl_page_flags(xpl_ctx* c, const void* base, uint64_t P, uint8_t* out, uint64_t n_pages) {
   if (!c || !out || P == 0) return XPL_ERR_INVALID_ARG;
-  if (c->depth) return XPL_ERR_STATE;
+  if (c->depth || c->world > 1) return XPL_ERR_STATE;
   auto it = c->live.find((uint64_t)base);
   if (it == c->live.end()) return XPL_ERR_UNKNOWN_PTR;
   const Row* r = &c->rows[it->second];
@@ -797,10 +885,16 @@ const char* xpl_status_string(xpl_status s) {
 
 xpl_status xpl_init(const xpl_config* cfg, xpl_ctx** out) {
   if (!cfg || !out) return XPL_ERR_INVALID_ARG;
-  if (cfg->world > 1) return XPL_ERR_INVALID_ARG;  // sharding: see DESIGN.md §8
+  const int world = cfg->world > 1 ? cfg->world : 1;
+  if (world > XPL_MAX_RANKS || (world > 1 && (!cfg->comm || cfg->rank < 0 || cfg->rank >= world)))
+    return XPL_ERR_INVALID_ARG;
   xpl_ctx* c = new (std::nothrow) xpl_ctx();
   if (!c) return XPL_ERR_OOM;
   c->cfg = *cfg;
+  c->world = world;
+  c->rank = world > 1 ? cfg->rank : 0;
+  c->comm = world > 1 ? cfg->comm : nullptr;
+  c->route.assign(world, {});
   if (!c->cfg.pool_words) c->cfg.pool_words = 1ull << 28;
   if (!c->cfg.staging_recs) c->cfg.staging_recs = 1ull << 22;
   if (!c->cfg.max_rows) c->cfg.max_rows = 4096;
@@ -818,7 +912,8 @@ xpl_status xpl_init(const xpl_config* cfg, xpl_ctx** out) {
   c->cs = c->rs;
   CKI(cudaMalloc(&c->d_pool, c->pool_words));
   CKI(cudaMemsetAsync(c->d_pool, 0, c->pool_words, c->cs));
-  c->pa.init(c->pool_words);
+  c->pas.assign(world, PoolAlloc());
+  for (PoolAlloc& a : c->pas) a.init(c->pool_words);
   CKI(cudaMalloc(&c->d_tab, 32 + sizeof(xpl_dev_row) * c->cfg.max_rows));
   CKI(cudaMemsetAsync(c->d_tab, 0, 32, c->cs));
   CKI(host_alloc(&c->h_tab, 32 + sizeof(xpl_dev_row) * c->cfg.max_rows));
@@ -851,6 +946,25 @@ xpl_status xpl_init(const xpl_config* cfg, xpl_ctx** out) {
   xpl_status s = ensure_ranges(c, 1024);
   if (s) { xpl_finalize(c); return s; }
   CKI(cudaStreamSynchronize(c->cs));
+  if (world > 1) {  // map the other ranks' pools and chunk maps (CUDA IPC; NVLink / NVSwitch peers)
+    struct Ex { cudaIpcMemHandle_t h[3]; uint64_t pool_words; };
+    Ex mine;
+    memset(&mine, 0, sizeof mine);
+    CKI(cudaIpcGetMemHandle(&mine.h[0], c->d_pool));
+    CKI(cudaIpcGetMemHandle(&mine.h[1], c->d_cmap));
+    CKI(cudaIpcGetMemHandle(&mine.h[2], c->d_smap));
+    mine.pool_words = c->pool_words;
+    std::vector<Ex> all(world);
+    if (c->comm->allgather(c->comm->user, &mine, sizeof(Ex), all.data())) { xpl_finalize(c); return XPL_ERR_NCCL; }
+    for (int q = 0; q < world; ++q) {
+      if (all[q].pool_words != c->pool_words) { xpl_finalize(c); return XPL_ERR_INVALID_ARG; }
+      if (q == c->rank) continue;
+      CKI(cudaIpcOpenMemHandle(&c->peer_pool[q], all[q].h[0], cudaIpcMemLazyEnablePeerAccess));
+      CKI(cudaIpcOpenMemHandle(&c->peer_cmap[q], all[q].h[1], cudaIpcMemLazyEnablePeerAccess));
+      CKI(cudaIpcOpenMemHandle(&c->peer_smap[q], all[q].h[2], cudaIpcMemLazyEnablePeerAccess));
+    }
+    if (c->comm->barrier(c->comm->user)) { xpl_finalize(c); return XPL_ERR_NCCL; }
+  }
   memset(&c->st, 0, sizeof c->st);
   *out = c;
   return XPL_OK;
@@ -861,6 +975,11 @@ xpl_status xpl_finalize(xpl_ctx* c) {
   if (!c) return XPL_ERR_INVALID_ARG;
   if (c->cs) cudaStreamSynchronize(c->cs);
   if (c->rs) cudaStreamSynchronize(c->rs);
+  // (sharded: every rank finalises; no rank may unmap a pool a peer still writes)
+  if (c->world > 1 && c->comm && c->d_pool) c->comm->barrier(c->comm->user);
+  for (int q = 0; q < XPL_MAX_RANKS; ++q)
+    for (void* p : {c->peer_pool[q], c->peer_cmap[q], c->peer_smap[q]})
+      if (p) cudaIpcCloseMemHandle(p);
   cudaFree(c->d_pool);
   cudaFree(c->d_first_w);
   cudaFree(c->d_tab);
@@ -912,7 +1031,8 @@ xpl_status xpl_finalize(xpl_ctx* c) {
 }
 
 static xpl_status register_row(xpl_ctx* c, const void* ptr, size_t bytes, xpl_alloc_kind kind,
-                               bool piece, uint64_t logical_id, uint64_t goff, uint64_t lbytes) {
+                               bool piece, uint64_t logical_id, uint64_t goff, uint64_t lbytes,
+                               uint32_t owner = 0) {
   if (!c || !ptr || bytes == 0 || (unsigned)kind > 2) return XPL_ERR_INVALID_ARG;
   if (piece && (lbytes == 0 || goff + (bytes + 3) / 4 > (lbytes + 3) / 4)) return XPL_ERR_INVALID_ARG;
   if (c->depth) return XPL_ERR_STATE;
@@ -939,24 +1059,71 @@ static xpl_status register_row(xpl_ctx* c, const void* ptr, size_t bytes, xpl_al
   r.logical_id = piece ? logical_id : r.id;
   r.goff = piece ? goff : 0;
   r.lbytes = piece ? lbytes : bytes;
-  if (!c->pa.alloc(r.span, &r.off)) return XPL_ERR_OOM;
-  CK(cudaMemsetAsync(c->d_pool + r.off, 0, r.span, c->cs));  // D3: last writer = CPU
+  r.owner = owner;
+  if (!c->pas[owner].alloc(r.span, &r.off)) return XPL_ERR_OOM;
+  if (owner == (uint32_t)c->rank)
+    CK(cudaMemsetAsync(c->d_pool + r.off, 0, r.span, c->cs));  // D3: last writer = CPU
   const size_t cap_before = c->rows.capacity();
   c->rows.push_back(r);
   if (c->rows.capacity() != cap_before) c->cache = nullptr;
   c->live[p] = r.id;
+  c->lrows[r.logical_id].push_back(r.id);
   c->table_dirty = true;
   c->cache = nullptr;
   return XPL_OK;
 }
 
+// The pieces of a logical allocation of lw words over R ranks (xpl.h sharded
+// mode): < 65536 words -> one piece owned by rank (lid mod R); else R pieces of
+// ceil(lw/R) words rounded up to 1024, piece r owned by rank r (empty tail
+// pieces dropped).  (goff, words, owner) each.
+static std::vector<std::array<uint64_t, 3>> shard_pieces(uint64_t lid, uint64_t lw, int R) {
+  std::vector<std::array<uint64_t, 3>> v;
+  if (lw < 65536) {
+    v.push_back({0, lw, lid % (uint64_t)R});
+    return v;
+  }
+  const uint64_t chunk = ((lw + R - 1) / R + 1023) & ~1023ull;
+  for (int r = 0; r < R; ++r) {
+    const uint64_t g = (uint64_t)r * chunk;
+    if (g >= lw) break;
+    v.push_back({g, std::min(lw, g + chunk) - g, (uint64_t)r});
+  }
+  return v;
+}
+
 xpl_status xpl_register_alloc(xpl_ctx* c, const void* ptr, size_t bytes, xpl_alloc_kind kind) {
-  return register_row(c, ptr, bytes, kind, false, 0, 0, 0);
+  if (!c) return XPL_ERR_INVALID_ARG;
+  if (c->world <= 1) return register_row(c, ptr, bytes, kind, false, 0, 0, 0);
+  // sharded mode (COLLECTIVE): one row per piece, each in its owner's pool
+  if (!ptr || bytes == 0 || (unsigned)kind > 2) return XPL_ERR_INVALID_ARG;
+  if (c->depth) return XPL_ERR_STATE;
+  const uint64_t lid = c->n_logical;
+  const uint64_t lw = (bytes + 3) / 4;
+  const auto pcs = shard_pieces(lid, lw, c->world);
+  if (c->live.size() + pcs.size() > c->cfg.max_rows) return XPL_ERR_OOM;
+  for (const auto& pc : pcs) {  // (overlap of any piece = overlap of the whole range)
+    const uint64_t b0 = 4 * pc[0], b1 = std::min<uint64_t>(bytes, 4 * (pc[0] + pc[1]));
+    xpl_status st = register_row(c, (const uint8_t*)ptr + b0, b1 - b0, kind, true, lid, pc[0], bytes,
+                                 (uint32_t)pc[2]);
+    if (st) return st;  // (only the first piece can fail on overlap; OOM is fatal anyway)
+  }
+  c->n_logical++;
+  return XPL_OK;
 }
 
 xpl_status xpl_register_alloc_piece(xpl_ctx* c, const void* ptr, size_t bytes, xpl_alloc_kind kind,
                                     uint64_t logical_id, uint64_t word_offset, uint64_t logical_bytes) {
+  if (!c) return XPL_ERR_INVALID_ARG;
+  if (c->world > 1) return XPL_ERR_STATE;  // sharded mode cuts the pieces itself
   return register_row(c, ptr, bytes, kind, true, logical_id, word_offset, logical_bytes);
+}
+
+static void kill_row(xpl_ctx* c, uint64_t id) {
+  Row& r = c->rows[id];
+  r.live = false;  // shadow kept until the next diagnose
+  c->live.erase(r.base);
+  c->n_dead++;
 }
 
 xpl_status xpl_free(xpl_ctx* c, const void* ptr) {
@@ -964,9 +1131,14 @@ xpl_status xpl_free(xpl_ctx* c, const void* ptr) {
   if (c->depth) return XPL_ERR_STATE;
   auto it = c->live.find((uint64_t)ptr);
   if (it == c->live.end()) return XPL_ERR_UNKNOWN_PTR;
-  c->rows[it->second].live = false;  // shadow kept until the next diagnose
-  c->live.erase(it);
-  c->n_dead++;
+  if (c->world > 1) {  // every piece of the logical allocation (COLLECTIVE)
+    const Row& r = c->rows[it->second];
+    if (r.goff != 0) return XPL_ERR_UNKNOWN_PTR;  // not the allocation's base
+    const std::vector<uint64_t> ids = c->lrows[r.logical_id];
+    for (uint64_t id : ids) kill_row(c, id);
+  } else {
+    kill_row(c, it->second);
+  }
   c->table_dirty = true;
   c->cache = nullptr;
   return XPL_OK;
@@ -1021,6 +1193,13 @@ xpl_status xpl_kernel_end(xpl_ctx* c, void* stream) {
     c->epoch_streams.push_back(s);
   }
   if (--c->depth) return XPL_OK;
+  if (c->world > 1) {
+    // sharded: every rank's kernels of the epoch -- including their atomics into
+    // this rank's pool over NVLink -- have completed before any owner folds
+    for (cudaStream_t x : c->epoch_streams) CK(cudaStreamSynchronize(x));
+    CK(cudaStreamSynchronize(c->cs));
+    if (c->comm->barrier(c->comm->user)) return XPL_ERR_NCCL;
+  }
   // the stream the fold goes on, and everything of the epoch that must precede it
   const bool single = c->epoch_streams.size() == 1;
   cudaStream_t t = single ? c->epoch_streams[0] : c->rs;
@@ -1038,7 +1217,7 @@ xpl_status xpl_kernel_end(xpl_ctx* c, void* stream) {
     CK(cudaStreamWaitEvent(t, e, 0));
     crossed = true;
   }
-  const bool strict = !single || c->cs_in_epoch;
+  const bool strict = !single || c->cs_in_epoch || c->world > 1;  // (a split cannot span ranks)
   c->cs = t;
   fold(c, !crossed, strict);
   if (c->lepoch_open) {  // NEXT-4: after the fold, on its stream
@@ -1057,10 +1236,11 @@ xpl_status xpl_kernel_end(xpl_ctx* c, void* stream) {
     c->cs = c->rs;
   }
   if (cudaGetLastError() != cudaSuccess) return XPL_ERR_CUDA;
-  std::vector<uint64_t> q;
+  std::vector<std::pair<uint32_t, uint64_t>> q;
   q.swap(c->deferred);
-  for (uint64_t r : q) {
-    xpl_status st = stage_push(c, rec_g0(r), rec_nw(r), rec_acc(r));
+  for (const auto& d : q) {
+    const uint64_t r = d.second;
+    xpl_status st = stage_push(c, rec_g0(r), rec_nw(r), rec_acc(r), d.first);
     if (st) return st;
   }
   return XPL_OK;
@@ -1072,17 +1252,18 @@ xpl_status xpl_record_host(xpl_ctx* c, const xpl_host_access* recs, size_t n) {
     const uint32_t acc = recs[i].kind;
     if (acc < 1 || acc > 3) return XPL_ERR_INVALID_ARG;
     uint64_t g0, nw;
-    if (!to_words(c, recs[i].addr, recs[i].size, &g0, &nw)) continue;  // untracked
+    uint32_t own = 0;
+    if (!to_words(c, recs[i].addr, recs[i].size, &g0, &nw, &own)) continue;  // untracked
     if (c->depth) {
       while (nw > kMaxRecWords) {
-        c->deferred.push_back(pack_rec(g0, kMaxRecWords, acc));
+        c->deferred.push_back({own, pack_rec(g0, kMaxRecWords, acc)});
         g0 += kMaxRecWords;
         nw -= kMaxRecWords;
       }
-      c->deferred.push_back(pack_rec(g0, nw, acc));
+      c->deferred.push_back({own, pack_rec(g0, nw, acc)});
       continue;
     }
-    xpl_status s = stage_push(c, g0, nw, acc);
+    xpl_status s = stage_push(c, g0, nw, acc, own);
     if (s) return s;
   }
   return XPL_OK;
@@ -1106,16 +1287,17 @@ xpl_status xpl_record_host_ranges(xpl_ctx* c, const xpl_host_access* recs, size_
       const uint64_t re = r->base + r->bytes;
       const uint64_t pe = e < re ? e : re;
       uint64_t g0, nw;
-      if (to_words(c, a, pe - a, &g0, &nw)) {
+      uint32_t own = 0;
+      if (to_words(c, a, pe - a, &g0, &nw, &own)) {
         if (c->depth) {
           while (nw > kMaxRecWords) {
-            c->deferred.push_back(pack_rec(g0, kMaxRecWords, acc));
+            c->deferred.push_back({own, pack_rec(g0, kMaxRecWords, acc)});
             g0 += kMaxRecWords;
             nw -= kMaxRecWords;
           }
-          c->deferred.push_back(pack_rec(g0, nw, acc));
+          c->deferred.push_back({own, pack_rec(g0, nw, acc)});
         } else {
-          xpl_status s = stage_push(c, g0, nw, acc);
+          xpl_status s = stage_push(c, g0, nw, acc, own);
           if (s) return s;
         }
       }
@@ -1147,10 +1329,10 @@ xpl_status xpl_record_host_strided(xpl_ctx* c, const xpl_host_strided* recs, siz
         uint64_t g0 = r->off + w0, nw = wl - w0 + 1;
         if (c->depth) {
           for (; nw > kMaxRecWords; g0 += kMaxRecWords, nw -= kMaxRecWords)
-            c->deferred.push_back(pack_rec(g0, kMaxRecWords, q.kind));
-          c->deferred.push_back(pack_rec(g0, nw, q.kind));
+            c->deferred.push_back({r->owner, pack_rec(g0, kMaxRecWords, q.kind)});
+          c->deferred.push_back({r->owner, pack_rec(g0, nw, q.kind)});
         } else {
-          xpl_status s = stage_push(c, g0, nw, q.kind);
+          xpl_status s = stage_push(c, g0, nw, q.kind, r->owner);
           if (s) return s;
         }
       }
@@ -1166,40 +1348,77 @@ xpl_status xpl_record_host_strided(xpl_ctx* c, const xpl_host_strided* recs, siz
   return XPL_OK;
 }
 
+}  // extern "C"
+
+// The pieces (row, first pool word, words) of [addr, addr+bytes) clipped to the
+// logical allocation holding addr (D18): its one row, or, in sharded mode, the
+// pieces it spans.  False if addr is untracked.
+template <class F>
+static bool for_logical_range(xpl_ctx* c, uint64_t addr, uint64_t bytes, F fn) {
+  const Row* r = lookup(c, addr);
+  if (!r) return false;
+  const uint64_t lend = r->base - 4 * r->goff + r->lbytes;  // pieces are contiguous in address
+  const uint64_t e = bytes < lend - addr ? addr + bytes : lend;
+  const std::vector<uint64_t> ids = c->lrows[r->logical_id];
+  for (uint64_t id : ids) {
+    const Row& p = c->rows[id];
+    if (!p.live) continue;
+    const uint64_t a0 = std::max(addr, p.base), a1 = std::min(e, p.base + p.bytes);
+    if (a0 >= a1) continue;
+    const uint64_t w0 = (a0 - p.base) >> 2, wl = std::min((a1 - 1 - p.base) >> 2, p.words - 1);
+    fn(p, p.off + w0, wl - w0 + 1);
+  }
+  return true;
+}
+
+static xpl_status push_or_defer(xpl_ctx* c, uint32_t owner, uint64_t g0, uint64_t nw, uint32_t acc) {
+  if (!c->depth) return stage_push(c, g0, nw, acc, owner);
+  for (; nw > kMaxRecWords; g0 += kMaxRecWords, nw -= kMaxRecWords)
+    c->deferred.push_back({owner, pack_rec(g0, kMaxRecWords, acc)});
+  c->deferred.push_back({owner, pack_rec(g0, nw, acc)});
+  return XPL_OK;
+}
+
+extern "C" {
+
 xpl_status xpl_record_copy(xpl_ctx* c, const void* dst, const void* src, size_t bytes,
                            xpl_copy_dir dir) {
   if (!c || (unsigned)dir > 4) return XPL_ERR_INVALID_ARG;
   if (bytes == 0) return XPL_OK;
-  if (dir <= XPL_COPY_H2H) {  // CPU-side
-    xpl_host_access a[2];
-    size_t n = 0;
-    if (dir == XPL_COPY_H2D) a[n++] = {(uint64_t)dst, 0, XPL_ACC_W};
-    if (dir == XPL_COPY_D2H) a[n++] = {(uint64_t)src, 0, XPL_ACC_R};
-    if (dir == XPL_COPY_H2H) {
-      a[n++] = {(uint64_t)src, 0, XPL_ACC_R};
-      a[n++] = {(uint64_t)dst, 0, XPL_ACC_W};
-    }
-    for (size_t i = 0; i < n; ++i) {  // sizes may exceed 32 bits: split
-      uint64_t off = 0;
-      while (off < bytes) {
-        const uint64_t chunk = std::min<uint64_t>(bytes - off, 1ull << 30);
-        xpl_host_access r = {a[i].addr + off, (uint32_t)chunk, a[i].kind};
-        xpl_status s = xpl_record_host(c, &r, 1);
+  if (dir <= XPL_COPY_H2H) {  // CPU-side: one ordered range per side
+    if (c->world > 1) {
+      // COLLECTIVE: route what came before; rank 0's call is the one recorded
+      // (first in the next slice order, xpl.h)
+      if (!c->depth) {
+        xpl_status s = flush(c);
         if (s) return s;
-        off += chunk;
       }
+      if (c->rank != 0) return XPL_OK;
     }
-    return XPL_OK;
+    struct Side { uint64_t addr; uint32_t acc; } a[2];
+    size_t n = 0;
+    if (dir == XPL_COPY_H2D) a[n++] = {(uint64_t)dst, XPL_ACC_W};
+    if (dir == XPL_COPY_D2H) a[n++] = {(uint64_t)src, XPL_ACC_R};
+    if (dir == XPL_COPY_H2H) {
+      a[n++] = {(uint64_t)src, XPL_ACC_R};
+      a[n++] = {(uint64_t)dst, XPL_ACC_W};
+    }
+    xpl_status st = XPL_OK;
+    for (size_t i = 0; i < n; ++i)
+      for_logical_range(c, a[i].addr, bytes, [&](const Row& p, uint64_t g0, uint64_t nw) {
+        if (!st) st = push_or_defer(c, p.owner, g0, nw, a[i].acc);
+      });
+    return st;
   }
   // GPU-side: D2D = GPU read src + GPU write dst; memset = GPU write dst (D7).
-  // One range per side, of any length (RangeDesc.nw and the range kernel's
-  // vector indices are 64-bit).
-  RangeDesc rd[2];
-  size_t nr = 0;
+  // One range per side and piece, of any length (RangeDesc.nw and the range
+  // kernel's vector indices are 64-bit); in sharded mode each owner applies
+  // its own pieces.
+  std::vector<RangeDesc> rd;
   auto add = [&](uint64_t addr, uint32_t acc) {
-    uint64_t g0, nw;
-    if (!to_words(c, addr, bytes, &g0, &nw)) return;
-    rd[nr++] = {g0, nw, 0, acc, 1};
+    for_logical_range(c, addr, bytes, [&](const Row& p, uint64_t g0, uint64_t nw) {
+      if (p.owner == (uint32_t)c->rank) rd.push_back({g0, nw, 0, acc, 1});
+    });
   };
   if (dir == XPL_COPY_D2D) add((uint64_t)src, XPL_ACC_R);
   add((uint64_t)dst, XPL_ACC_W);
@@ -1209,7 +1428,7 @@ xpl_status xpl_record_copy(xpl_ctx* c, const void* dst, const void* src, size_t 
     if (s) return s;
     c->st.epochs++;
   }
-  xpl_status s = gpu_ranges(c, rd, nr);
+  xpl_status s = gpu_ranges(c, rd.data(), rd.size());
   if (s) return s;
   if (own) fold(c, false);
   return cudaGetLastError() == cudaSuccess ? XPL_OK : XPL_ERR_CUDA;
@@ -1261,6 +1480,14 @@ xpl_status xpl_get_device_ctx(xpl_ctx* c, struct xpl_dev_ctx* d) {
   d->smap = c->d_smap;
   d->n_super = (const unsigned long long*)(c->d_tab + 8);
   d->flags = c->d_misc;
+  d->rank = (unsigned)c->rank;
+  d->world = (unsigned)c->world;
+  for (int q = 0; q < XPL_MAX_RANKS; ++q) {
+    const bool me = q == c->rank;
+    d->pools[q] = (unsigned int*)(me ? (void*)c->d_pool : c->peer_pool[q]);
+    d->cmaps[q] = (unsigned char*)(me ? (void*)c->d_cmap : c->peer_cmap[q]);
+    d->smaps[q] = (unsigned char*)(me ? (void*)c->d_smap : c->peer_smap[q]);
+  }
   return XPL_OK;
 }
 
@@ -1318,6 +1545,7 @@ xpl_status xpl_shadow_dump(xpl_ctx* c, const void* base, uint64_t word0, uint64_
   if (it == c->live.end()) return XPL_ERR_UNKNOWN_PTR;
   const Row& r = c->rows[it->second];
   if (word0 > r.words || n > r.words - word0) return XPL_ERR_INVALID_ARG;
+  if (r.owner != (uint32_t)c->rank) return XPL_ERR_INVALID_ARG;  // (sharded: another rank's piece)
   xpl_status s = flush(c);
   if (s) return s;
   CK(cudaMemcpyAsync(out, c->d_pool + r.off + word0, n, cudaMemcpyDeviceToHost, c->cs));
@@ -1325,11 +1553,31 @@ xpl_status xpl_shadow_dump(xpl_ctx* c, const void* base, uint64_t word0, uint64_
   return XPL_OK;
 }
 
+// A resetting diagnose drops the rows freed since the last one and recycles
+// their shadow (D17); in sharded mode every rank drops every piece
+// (each rank keeps every owner's pool allocator in step).
+static void drop_dead(xpl_ctx* c) {
+  for (Row& r : c->rows) {
+    if (!r.live && !r.dropped) {
+      r.dropped = true;
+      c->pas[r.owner].release(r.off, r.span);
+      auto it = c->lrows.find(r.logical_id);
+      if (it != c->lrows.end()) {
+        auto& v = it->second;
+        v.erase(std::remove(v.begin(), v.end(), r.id), v.end());
+        if (v.empty()) c->lrows.erase(it);
+      }
+    }
+  }
+  c->n_dead = 0;
+}
+
 // The diagnosis of every live row and every row freed since the last reset
 // (tracePrint).  Fills `out` (reports) or `pout` (sharding partials).
 static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const xpl_name* names,
                                 size_t n_names, xpl_alloc_report* out, xpl_partial* pout, size_t cap,
                                 size_t* n_out, int reset) {
+  // (sharded mode: this rank analyses the pieces it owns)
   if (!c || !n_out || (n_names && !names)) return XPL_ERR_INVALID_ARG;
   if (c->depth) return XPL_ERR_STATE;
   DiagParams p;
@@ -1342,7 +1590,7 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
 
   std::vector<uint64_t> ids;  // live rows + rows freed since the last reset, id order (D23)
   for (const Row& r : c->rows)
-    if (r.live || !r.dropped) ids.push_back(r.id);
+    if ((r.live || !r.dropped) && r.owner == (uint32_t)c->rank) ids.push_back(r.id);
   *n_out = ids.size();
   if (cap < ids.size() || (!out && !pout && ids.size())) return XPL_ERR_INVALID_ARG;
 
@@ -1350,7 +1598,10 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
   if (s) return s;
   const size_t nr = ids.size();
   c->st.diagnoses++;
-  if (nr == 0) return XPL_OK;
+  if (nr == 0) {
+    if (reset) drop_dead(c);
+    return XPL_OK;
+  }
 
   auto row_blocks = [&](const Row& r) -> uint64_t {  // logical blocks the row touches
     return B ? (r.goff + r.words - 1) / B - r.goff / B + 1 : 0;
@@ -1540,22 +1791,51 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
       pout[i] = o;
     }
   }
-  if (reset) {  // drop freed rows and recycle their shadow (D17)
-    for (Row& r : c->rows) {
-      if (!r.live && !r.dropped) {
-        r.dropped = true;
-        c->pa.release(r.off, r.span);
-      }
-    }
-    c->n_dead = 0;
-  }
+  if (reset) drop_dead(c);
   return XPL_OK;
 }
 
 xpl_status xpl_diagnose(xpl_ctx* c, const xpl_diag_params* params, const xpl_name* names,
                         size_t n_names, xpl_alloc_report* out, size_t cap, size_t* n_out,
                         int reset) {
-  return diagnose_impl(c, params, names, n_names, out, nullptr, cap, n_out, reset);
+  if (!c || c->world <= 1) return diagnose_impl(c, params, names, n_names, out, nullptr, cap, n_out, reset);
+  // sharded (COLLECTIVE): partials of the owned pieces -> all-gather -> combine
+  if (!n_out || (n_names && !names)) return XPL_ERR_INVALID_ARG;
+  if (c->depth) return XPL_ERR_STATE;
+  std::vector<uint64_t> lids;
+  size_t n_own = 0;
+  for (const Row& r : c->rows)
+    if (r.live || !r.dropped) {
+      lids.push_back(r.logical_id);
+      if (r.owner == (uint32_t)c->rank) ++n_own;
+    }
+  std::sort(lids.begin(), lids.end());
+  lids.erase(std::unique(lids.begin(), lids.end()), lids.end());
+  *n_out = lids.size();
+  if (cap < lids.size() || (!out && !lids.empty())) return XPL_ERR_INVALID_ARG;  // (before any collective)
+  std::vector<xpl_partial> mine(n_own + 1);
+  size_t k = 0;
+  xpl_status s = diagnose_impl(c, params, names, n_names, nullptr, mine.data(), n_own, &k, reset);
+  if (s) return s;
+  const int R = c->world;
+  std::vector<uint64_t> cnt(R), sb(R), rb(R);
+  const uint64_t my = k * sizeof(xpl_partial);
+  if (c->comm->allgather(c->comm->user, &my, 8, cnt.data())) return XPL_ERR_NCCL;
+  std::vector<uint8_t> send((size_t)my * R + 1);
+  uint64_t tot = 0;
+  for (int q = 0; q < R; ++q) {
+    sb[q] = my;
+    rb[q] = cnt[q];
+    tot += cnt[q];
+    memcpy(send.data() + (size_t)q * my, mine.data(), my);
+  }
+  std::vector<uint8_t> recv(tot + 1);
+  if (c->comm->alltoallv(c->comm->user, send.data(), sb.data(), recv.data(), rb.data())) return XPL_ERR_NCCL;
+  size_t no = 0;
+  s = xpl_combine_partials((const xpl_partial*)recv.data(), tot / sizeof(xpl_partial), params, out, cap, &no);
+  if (s) return s;
+  *n_out = no;
+  return XPL_OK;
 }
 
 xpl_status xpl_diagnose_partials(xpl_ctx* c, const xpl_diag_params* params, const xpl_name* names,

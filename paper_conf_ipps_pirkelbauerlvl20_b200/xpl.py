@@ -34,8 +34,18 @@ HOST_STRIDED_DTYPE = np.dtype([("addr", "<u8"), ("size", "<u4"), ("kind", "<u4")
                                ("count", "<u8")])
 
 
+_ALLGATHER = C.CFUNCTYPE(i32, vp, vp, C.c_size_t, vp)
+_ALLTOALLV = C.CFUNCTYPE(i32, vp, vp, C.POINTER(u64), vp, C.POINTER(u64))
+_BARRIER = C.CFUNCTYPE(i32, vp)
+
+
+class XplComm(C.Structure):
+    """xpl_comm: the collectives of a sharded context (host buffers, blocking)."""
+    _fields_ = [("user", vp), ("allgather", _ALLGATHER), ("alltoallv", _ALLTOALLV), ("barrier", _BARRIER)]
+
+
 class XplConfig(C.Structure):
-    _fields_ = [("device", i32), ("rank", i32), ("world", i32), ("nccl_comm", vp),
+    _fields_ = [("device", i32), ("rank", i32), ("world", i32), ("comm", C.POINTER(XplComm)),
                 ("pool_words", u64), ("staging_recs", u64), ("max_rows", u32)]
 
 
@@ -114,6 +124,9 @@ xpl_format_reports = _sig("xpl_format_reports", [C.POINTER(XplAllocReport), sz, 
                                                  i32, C.c_char_p, sz, C.POINTER(sz)])
 xpl_get_device_ctx = _sig("xpl_get_device_ctx", [vp, C.POINTER(XplDevCtx)])
 xpl_release_stream = _sig("xpl_release_stream", [vp, vp])
+xpl_comm_nccl_unique_id = _sig("xpl_comm_nccl_unique_id", [vp])
+xpl_comm_nccl_create = _sig("xpl_comm_nccl_create", [vp, i32, i32, i32, C.POINTER(C.POINTER(XplComm))])
+xpl_comm_nccl_destroy = _sig("xpl_comm_nccl_destroy", [C.POINTER(XplComm)])
 xpl_shadow_dump = _sig("xpl_shadow_dump", [vp, vp, u64, u64, vp])
 PAGE_REPORT_FIELDS = [
     ("id", u64), ("base", u64), ("words", u64), ("page_words", u64), ("pages", u64),
@@ -169,7 +182,8 @@ EXPORTED = ["xpl_init", "xpl_finalize", "xpl_register_alloc", "xpl_free", "xpl_k
             "xpl_profile_read", "xpl_register_alloc_piece", "xpl_diagnose_partials", "xpl_combine_partials",
             "xpl_format_reports", "xpl_page_summary", "xpl_page_flags", "xpl_mem_advise",
             "xpl_launch_log_enable", "xpl_kernel_launch", "xpl_launch_log", "xpl_launch_name",
-            "xpl_release_stream"]
+            "xpl_release_stream", "xpl_comm_nccl_unique_id", "xpl_comm_nccl_create",
+            "xpl_comm_nccl_destroy"]
 
 if _work is not None:
     xplw_bind = _sig("xplw_bind", [vp], lib=_work)
@@ -196,11 +210,98 @@ def check(fn, status):
         raise XplError(fn, status)
 
 
-class Context:
-    """One xpl_ctx (one process, one GPU)."""
+class TorchComm:
+    """xpl_comm over a torch.distributed process group (argument marshalling
+    only: the runtime calls these from xpl_init / collective calls).  Host
+    tensors, so any backend works (gloo in the tests; use NcclComm on GPUs)."""
 
-    def __init__(self, device=0, pool_words=0, staging_recs=0, max_rows=0):
-        cfg = XplConfig(device, 0, 1, None, pool_words, staging_recs, max_rows)
+    def __init__(self, group=None):
+        import torch.distributed as dist
+        self.dist, self.group = dist, group
+        self.world = dist.get_world_size(group)
+        self.rank = dist.get_rank(group)
+        self._cb = (_ALLGATHER(self._allgather), _ALLTOALLV(self._alltoallv), _BARRIER(self._barrier))
+        self.c = XplComm(None, *self._cb)
+
+    def _gather_bytes(self, data):
+        import torch
+        n = torch.tensor([len(data)], dtype=torch.int64)
+        ns = [torch.zeros(1, dtype=torch.int64) for _ in range(self.world)]
+        self.dist.all_gather(ns, n, group=self.group)
+        m = max(int(x.item()) for x in ns)
+        t = torch.zeros(max(m, 1), dtype=torch.uint8)
+        if data:
+            t[:len(data)] = torch.frombuffer(bytearray(data), dtype=torch.uint8)
+        outs = [torch.zeros(max(m, 1), dtype=torch.uint8) for _ in range(self.world)]
+        self.dist.all_gather(outs, t, group=self.group)
+        return [bytes(o[:int(k.item())].numpy()) for o, k in zip(outs, ns)]
+
+    def _allgather(self, user, send, nbytes, recv):
+        try:
+            parts = self._gather_bytes(C.string_at(send, nbytes) if nbytes else b"")
+            C.memmove(recv, b"".join(parts), nbytes * self.world)
+            return 0
+        except Exception:  # noqa: BLE001 (reported to the runtime as a failed collective)
+            return 1
+
+    def _alltoallv(self, user, send, sb, recv, rb):
+        """All-to-all as two all-gathers (the send sizes, then the send
+        buffers): each rank cuts its part out of every rank's buffer."""
+        try:
+            import numpy as np
+            R = self.world
+            tot = sum(sb[q] for q in range(R))
+            blobs = self._gather_bytes(C.string_at(send, tot) if tot else b"")
+            sz = np.frombuffer(b"".join(self._gather_bytes(np.array([sb[q] for q in range(R)], np.uint64).tobytes())),
+                               np.uint64).reshape(R, R)
+            mine = b"".join(blobs[q][int(sz[q, :self.rank].sum()):int(sz[q, :self.rank + 1].sum())] for q in range(R))
+            if len(mine) != sum(rb[q] for q in range(R)):
+                return 2
+            if mine:
+                C.memmove(recv, mine, len(mine))
+            return 0
+        except Exception:  # noqa: BLE001
+            return 1
+
+    def _barrier(self, user):
+        try:
+            self.dist.barrier(group=self.group)
+            return 0
+        except Exception:  # noqa: BLE001
+            return 1
+
+
+class NcclComm:
+    """xpl_comm over NCCL (libxpl.so's own, xpl_comm_nccl_create): rank 0's
+    unique id reaches the others through `broadcast_id(bytes) -> bytes`."""
+
+    def __init__(self, rank, world, device, broadcast_id):
+        uid = (C.c_uint8 * 128)()
+        if rank == 0:
+            check("xpl_comm_nccl_unique_id", xpl_comm_nccl_unique_id(uid))
+        got = broadcast_id(bytes(uid))
+        C.memmove(uid, got, 128)
+        p = C.POINTER(XplComm)()
+        check("xpl_comm_nccl_create", xpl_comm_nccl_create(uid, rank, world, device, C.byref(p)))
+        self.p, self.rank, self.world = p, rank, world
+
+    def close(self):
+        if self.p:
+            check("xpl_comm_nccl_destroy", xpl_comm_nccl_destroy(self.p))
+            self.p = None
+
+
+class Context:
+    """One xpl_ctx (one process, one GPU).  comm (TorchComm / NcclComm) with
+    world > 1: a sharded context (COLLECTIVE calls, include/xpl.h)."""
+
+    def __init__(self, device=0, pool_words=0, staging_recs=0, max_rows=0, comm=None):
+        self.comm = comm  # (kept alive: the runtime holds its pointer)
+        if comm is None:
+            cfg = XplConfig(device, 0, 1, None, pool_words, staging_recs, max_rows)
+        else:
+            cp = C.pointer(comm.c) if isinstance(comm, TorchComm) else comm.p
+            cfg = XplConfig(device, comm.rank, comm.world, cp, pool_words, staging_recs, max_rows)
         h = vp()
         check("xpl_init", xpl_init(C.byref(cfg), C.byref(h)))
         self.h = h
