@@ -283,8 +283,11 @@ static __device__ __forceinline__ void xpld_one(unsigned ones, unsigned long lon
     const unsigned w = nb1 + 1;
     const unsigned long long G = g0 - (unsigned long long)lane * w;
     const unsigned glo = (unsigned)G, ghi = (unsigned)(G >> 32);
-    const bool same = __shfl_sync(FULL, glo, 0) == glo && __shfl_sync(FULL, ghi, 0) == ghi &&
-                      __shfl_sync(FULL, nb1, 0) == nb1;
+    /* (all three shuffles unconditionally: a short-circuit && would leave lanes
+     * out of a full-warp shuffle) */
+    const unsigned s_lo = __shfl_sync(FULL, glo, 0), s_hi = __shfl_sync(FULL, ghi, 0),
+                   s_nb = __shfl_sync(FULL, nb1, 0);
+    const bool same = (s_lo == glo) & (s_hi == ghi) & (s_nb == nb1);
     const unsigned long long E = G + 32ull * w - 1; /* last word the warp covers */
     const unsigned Q0 = (unsigned)(G >> 2), nq = (unsigned)(E >> 2) - Q0 + 1;
     if (__all_sync(FULL, same && nq <= 32 && (K != 0 || w == 1))) {

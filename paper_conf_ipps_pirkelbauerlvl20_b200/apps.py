@@ -27,7 +27,7 @@ class XplwRun(C.Structure):
                 ("diag_rows", vp), ("diag_cap", sz), ("n_diag", sz), ("dev_accesses", u64),
                 ("host_accesses", u64), ("copy_words", u64), ("epochs", u64), ("status", i32),
                 ("time_kernels", i32), ("kernel_ms", C.c_double), ("host_ms", C.c_double),
-                ("diag_no_reset", i32), ("keep_allocs", i32)]
+                ("diag_no_reset", i32), ("keep_allocs", i32), ("rank", i32), ("world", i32)]
 
 
 _w = xpl._work
@@ -110,8 +110,9 @@ class Run:
     """One xplw_run: the context (or None = uninstrumented twin) and outputs."""
 
     def __init__(self, ctx, stream, do_copies=False, diag_each=True, params=(50, 0, 256), out_cap=4096,
-                 time_kernels=False, diag_reset=True, keep_allocs=False):
+                 time_kernels=False, diag_reset=True, keep_allocs=False, rank=0, world=1):
         self.r = XplwRun()
+        self.r.rank, self.r.world = rank, world
         self.r.diag_no_reset = int(not diag_reset)
         self.r.keep_allocs = int(keep_allocs)
         self.r.time_kernels = int(time_kernels)

@@ -19,6 +19,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <algorithm>
 #include <chrono>
 #include <vector>
 
@@ -53,6 +54,13 @@ struct Dom {
 };
 static_assert(NSLOT == 50, "50 pointer slots");
 static_assert(sizeof(Dom) == 3736, "the domain object of Fig. 5 has 3736 bytes (P:L315)");
+
+// The index ranges one rank's kernels cover (sharded program, xplw_run.world >
+// 1): elements [e0, e1) (e0 a multiple of 256, so dt blocks stay whole), nodes
+// [n0, n1), symmetry-plane nodes [s0, s1).  One rank: everything.
+struct Part {
+  int e0, e1, n0, n1, s0, s1;
+};
 
 template <bool I, class T>
 __device__ __forceinline__ const T& RD(const T& x) {
@@ -92,10 +100,10 @@ __device__ __forceinline__ void count_hooks(unsigned long long* hc, unsigned c) 
 
 // 1. zero the nodal forces
 template <bool I>
-__global__ void k_zero_forces(Dom* d, int nn, unsigned long long* hc) {
-  const int n = blockIdx.x * blockDim.x + threadIdx.x;
+__global__ void k_zero_forces(Part P_, Dom* d, int nn, unsigned long long* hc) {
+  const int n = P_.n0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (n < nn) {
+  if (n < P_.n1 && n < nn) {
     double *fx = PTR(double, FX), *fy = PTR(double, FY), *fz = PTR(double, FZ);
     W_(fx[n]) = 0.0;
     W_(fy[n]) = 0.0;
@@ -106,10 +114,10 @@ __global__ void k_zero_forces(Dom* d, int nn, unsigned long long* hc) {
 
 // 2. stress integration: gather the 8 nodes, write 8 corner forces x 3
 template <bool I>
-__global__ void k_integrate_stress(Dom* d, unsigned long long* hc) {
-  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+__global__ void k_integrate_stress(Part P_, Dom* d, unsigned long long* hc) {
+  const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (e < NE()) {
+  if (e < P_.e1 && e < NE()) {
     const int* nl = PTR(const int, NODELIST);
     const double *x = PTR(const double, X), *y = PTR(const double, Y), *z = PTR(const double, Z);
     const double sig = -(R_(PTR(const double, P)[e]) + R_(PTR(const double, Q)[e]));
@@ -127,10 +135,10 @@ __global__ void k_integrate_stress(Dom* d, unsigned long long* hc) {
 
 // 3. hourglass control: gather nodal velocities, add to the corner forces
 template <bool I>
-__global__ void k_hourglass(Dom* d, unsigned long long* hc) {
-  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+__global__ void k_hourglass(Part P_, Dom* d, unsigned long long* hc) {
+  const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (e < NE()) {
+  if (e < P_.e1 && e < NE()) {
     const int* nl = PTR(const int, NODELIST);
     const double *xd = PTR(const double, XD), *yd = PTR(const double, YD), *zd = PTR(const double, ZD);
     const double coef = R_(PTR(const double, SS)[e]) * R_(PTR(const double, ELEMMASS)[e]) /
@@ -149,10 +157,10 @@ __global__ void k_hourglass(Dom* d, unsigned long long* hc) {
 
 // 4. sum the corner forces into the nodes through the node->corner lists
 template <bool I>
-__global__ void k_corner_sum(Dom* d, int nn, unsigned long long* hc) {
-  const int n = blockIdx.x * blockDim.x + threadIdx.x;
+__global__ void k_corner_sum(Part P_, Dom* d, int nn, unsigned long long* hc) {
+  const int n = P_.n0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (n < nn) {
+  if (n < P_.n1 && n < nn) {
     const int *st = PTR(const int, NODEELEMSTART), *cl = PTR(const int, CORNERLIST);
     const double* f = PTR(const double, TMP_FORCE);
     double *fx = PTR(double, FX), *fy = PTR(double, FY), *fz = PTR(double, FZ);
@@ -173,10 +181,10 @@ __global__ void k_corner_sum(Dom* d, int nn, unsigned long long* hc) {
 
 // 5. nodal accelerations
 template <bool I>
-__global__ void k_accel(Dom* d, int nn, unsigned long long* hc) {
-  const int n = blockIdx.x * blockDim.x + threadIdx.x;
+__global__ void k_accel(Part P_, Dom* d, int nn, unsigned long long* hc) {
+  const int n = P_.n0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (n < nn) {
+  if (n < P_.n1 && n < nn) {
     const double m = R_(PTR(const double, NODALMASS)[n]);
     const double ax = R_(PTR(const double, FX)[n]) / m, ay = R_(PTR(const double, FY)[n]) / m,
                  az = R_(PTR(const double, FZ)[n]) / m;
@@ -189,10 +197,10 @@ __global__ void k_accel(Dom* d, int nn, unsigned long long* hc) {
 
 // 6. symmetry plane: zero the accelerations of the plane's nodes
 template <bool I>
-__global__ void k_symm(Dom* d, int ns, unsigned long long* hc) {
-  const int k = blockIdx.x * blockDim.x + threadIdx.x;
+__global__ void k_symm(Part P_, Dom* d, int ns, unsigned long long* hc) {
+  const int k = P_.s0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (k < ns) {
+  if (k < P_.s1 && k < ns) {
     const int n = R_(PTR(const int, SYMMX)[k]);
     W_(PTR(double, XDD)[n]) = 0.0;
     W_(PTR(double, YDD)[n]) = 0.0;
@@ -203,10 +211,10 @@ __global__ void k_symm(Dom* d, int ns, unsigned long long* hc) {
 
 // 7./8. velocity and position updates
 template <bool I>
-__global__ void k_velocity(Dom* d, int nn, unsigned long long* hc) {
-  const int n = blockIdx.x * blockDim.x + threadIdx.x;
+__global__ void k_velocity(Part P_, Dom* d, int nn, unsigned long long* hc) {
+  const int n = P_.n0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (n < nn) {
+  if (n < P_.n1 && n < nn) {
     const double dt = R_(d->dt);
     const double ax = R_(PTR(const double, XDD)[n]), ay = R_(PTR(const double, YDD)[n]),
                  az = R_(PTR(const double, ZDD)[n]);
@@ -217,10 +225,10 @@ __global__ void k_velocity(Dom* d, int nn, unsigned long long* hc) {
   count_hooks<I>(hc, c);
 }
 template <bool I>
-__global__ void k_position(Dom* d, int nn, unsigned long long* hc) {
-  const int n = blockIdx.x * blockDim.x + threadIdx.x;
+__global__ void k_position(Part P_, Dom* d, int nn, unsigned long long* hc) {
+  const int n = P_.n0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (n < nn) {
+  if (n < P_.n1 && n < nn) {
     const double dt = R_(d->dt);
     const double vx = R_(PTR(const double, XD)[n]), vy = R_(PTR(const double, YD)[n]),
                  vz = R_(PTR(const double, ZD)[n]);
@@ -233,10 +241,10 @@ __global__ void k_position(Dom* d, int nn, unsigned long long* hc) {
 
 // 9. element kinematics: gather positions and velocities, new volume, gradients
 template <bool I>
-__global__ void k_kinematics(Dom* d, unsigned long long* hc) {
-  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+__global__ void k_kinematics(Part P_, Dom* d, unsigned long long* hc) {
+  const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (e < NE()) {
+  if (e < P_.e1 && e < NE()) {
     const int* nl = PTR(const int, NODELIST);
     const double *x = PTR(const double, X), *y = PTR(const double, Y), *z = PTR(const double, Z);
     const double *xd = PTR(const double, XD), *yd = PTR(const double, YD), *zd = PTR(const double, ZD);
@@ -261,10 +269,10 @@ __global__ void k_kinematics(Dom* d, unsigned long long* hc) {
 
 // 10. strain rate from the gradients
 template <bool I>
-__global__ void k_lagrange(Dom* d, unsigned long long* hc) {
-  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+__global__ void k_lagrange(Part P_, Dom* d, unsigned long long* hc) {
+  const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (e < NE()) {
+  if (e < P_.e1 && e < NE()) {
     const double* g = PTR(const double, TMP_DVDX);
     const double r = (R_(g[3 * e]) + R_(g[3 * e + 1]) + R_(g[3 * e + 2])) / (R_(PTR(const double, VNEW)[e]) + 1.0);
     W_(PTR(double, VDOV)[e]) = r;
@@ -274,10 +282,10 @@ __global__ void k_lagrange(Dom* d, unsigned long long* hc) {
 
 // 11./12. monotonic Q: gradients over the xi face neighbours, region limiter
 template <bool I>
-__global__ void k_monoq_grad(Dom* d, unsigned long long* hc) {
-  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+__global__ void k_monoq_grad(Part P_, Dom* d, unsigned long long* hc) {
+  const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (e < NE()) {
+  if (e < P_.e1 && e < NE()) {
     const double* vdov = PTR(const double, VDOV);
     const int m = R_(PTR(const int, LXIM)[e]), p = R_(PTR(const int, LXIP)[e]);
     const double r = R_(vdov[p]) - R_(vdov[m]) + R_(PTR(const double, VNEW)[e]);
@@ -286,10 +294,10 @@ __global__ void k_monoq_grad(Dom* d, unsigned long long* hc) {
   count_hooks<I>(hc, c);
 }
 template <bool I>
-__global__ void k_monoq_region(Dom* d, unsigned long long* hc) {
-  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+__global__ void k_monoq_region(Part P_, Dom* d, unsigned long long* hc) {
+  const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (e < NE()) {
+  if (e < P_.e1 && e < NE()) {
     const int bc = R_(PTR(const int, ELEMBC)[e]);
     const double r = (bc & 1 ? 0.5 : 1.0) * R_(PTR(const double, QL)[e]) * R_(PTR(const double, VDOV)[e]);
     W_(PTR(double, QQ)[e]) = r;
@@ -299,10 +307,10 @@ __global__ void k_monoq_region(Dom* d, unsigned long long* hc) {
 
 // 13. the four EOS stages (they read material parameters from the domain)
 template <bool I>
-__global__ void k_eos(Dom* d, int stage, unsigned long long* hc) {
-  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+__global__ void k_eos(Part P_, Dom* d, int stage, unsigned long long* hc) {
+  const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (e < NE()) {
+  if (e < P_.e1 && e < NE()) {
     const double t = R_(d->time);
     if (stage == 0) {  // energy
       const double w = R_(d->misc[0]) * 1e-6 + R_(d->misc[1]) * 1e-6 + R_(d->misc[2]);
@@ -331,10 +339,10 @@ __global__ void k_eos(Dom* d, int stage, unsigned long long* hc) {
 
 // 14. volumes
 template <bool I>
-__global__ void k_update_volumes(Dom* d, unsigned long long* hc) {
-  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+__global__ void k_update_volumes(Part P_, Dom* d, unsigned long long* hc) {
+  const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (e < NE()) {
+  if (e < P_.e1 && e < NE()) {
     const double v = R_(PTR(const double, VNEW)[e]);
     W_(PTR(double, V)[e]) = v;
   }
@@ -343,12 +351,12 @@ __global__ void k_update_volumes(Dom* d, unsigned long long* hc) {
 
 // 15./16. dt reductions: one minimum per 256-element block into dtb (GPU W, host R)
 template <bool I, bool COURANT>
-__global__ void __launch_bounds__(256) k_dt(Dom* d, double* dtb, int nblk, unsigned long long* hc) {
+__global__ void __launch_bounds__(256) k_dt(Part P_, Dom* d, double* dtb, int nblk, unsigned long long* hc) {
   __shared__ double s_min[256];
-  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+  const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   double v = 1e30;
-  if (e < NE()) {
+  if (e < P_.e1 && e < NE()) {
     if (COURANT) {
       const double ss = R_(PTR(const double, SS)[e]), vd = R_(PTR(const double, VDOV)[e]),
                    ar = R_(PTR(const double, AREALG)[e]);
@@ -364,7 +372,7 @@ __global__ void __launch_bounds__(256) k_dt(Dom* d, double* dtb, int nblk, unsig
     if (threadIdx.x < o && s_min[threadIdx.x + o] < s_min[threadIdx.x]) s_min[threadIdx.x] = s_min[threadIdx.x + o];
     __syncthreads();
   }
-  if (threadIdx.x == 0) W_(dtb[(COURANT ? 0 : nblk) + blockIdx.x]) = s_min[0];
+  if (threadIdx.x == 0) W_(dtb[(COURANT ? 0 : nblk) + P_.e0 / 256 + blockIdx.x]) = s_min[0];
   count_hooks<I>(hc, c);
 }
 
@@ -396,6 +404,20 @@ int xplw_lulesh(xplw_run* run, const xplw_arrays* arr, int s, int steps, unsigne
   cudaStream_t st = (cudaStream_t)run->stream;
   const int ne = s * s * s, nn = (s + 1) * (s + 1) * (s + 1), nsym = (s + 1) * (s + 1);
   const int nblk = (ne + 255) / 256;
+  // sharded program (run->world > 1, one rank per GPU, a sharded context): this
+  // rank's kernels cover an element range (whole dt blocks), a node range and a
+  // symmetry-node range; its host traces its slice of every array's init; rank 0
+  // traces the single-copy host segments (domain init, TimeIncrement).
+  const int R = run->world > 1 ? run->world : 1, rk = R > 1 ? run->rank : 0;
+  Part P;
+  {
+    const int pe = ((ne + R - 1) / R + 255) / 256 * 256, pn = (nn + R - 1) / R, ps = (nsym + R - 1) / R;
+    P.e0 = std::min(ne, rk * pe), P.e1 = std::min(ne, P.e0 + pe);
+    P.n0 = std::min(nn, rk * pn), P.n1 = std::min(nn, P.n0 + pn);
+    P.s0 = std::min(nsym, rk * ps), P.s1 = std::min(nsym, P.s0 + ps);
+  }
+  const int GE = std::max(1, (P.e1 - P.e0 + 255) / 256), GN = std::max(1, (P.n1 - P.n0 + 255) / 256),
+            GS = std::max(1, (P.s1 - P.s0 + 255) / 256);
   Dom* dom = (Dom*)arr->addr[0];
   double* dtb = (double*)arr->addr[1];
   // arr->addr[2 + k] = the array of pointer slot k (k < TMP_FORCE)
@@ -460,8 +482,8 @@ int xplw_lulesh(xplw_run* run, const xplw_arrays* arr, int s, int steps, unsigne
     evs.clear();
   };
 #define LAUNCH(KER, GRID, ...)                                                          \
-  launch([&](int g) { KER<true><<<g, 256, 0, st>>>(__VA_ARGS__); },                    \
-         [&](int g) { KER<false><<<g, 256, 0, st>>>(__VA_ARGS__); }, GRID)
+  launch([&](int g) { KER<true><<<g, 256, 0, st>>>(P, __VA_ARGS__); },                 \
+         [&](int g) { KER<false><<<g, 256, 0, st>>>(P, __VA_ARGS__); }, GRID)
   auto managed = [&](size_t bytes) -> void* {
     void* p = nullptr;
     okc(cudaMallocManaged(&p, bytes));
@@ -477,97 +499,131 @@ int xplw_lulesh(xplw_run* run, const xplw_arrays* arr, int s, int steps, unsigne
     else x = v;
     run->host_accesses++;
   };
+  xpl_host_tracer* const tr0 = rk == 0 ? tr : nullptr;  // the single-copy host segments
+  auto hw0 = [&](auto& x, auto v) {
+    if (tr0) {
+      tr0->write(x) = v;
+      run->host_accesses++;
+    } else {
+      x = v;
+      if (!tr) run->host_accesses++;
+    }
+  };
 
   if (on)
     for (int k = 0; k < arr->n; ++k)
       ok(xpl_register_alloc(run->ctx, (const void*)arr->addr[k], arr->bytes[k], (xpl_alloc_kind)arr->kind[k]));
   // ---- initialisation (host): the domain, the arrays, the mesh topology ----
   auto t0 = std::chrono::steady_clock::now();
-  for (int k = 0; k < NSLOT; ++k) hw(dom->ptr[k], k < TMP_FORCE ? (void*)arr->addr[2 + k] : (void*)nullptr);
-  hw(dom->numElem, (uint32_t)ne);
-  hw(dom->numNode, (uint32_t)nn);
-  hw(dom->dt, 1e-3);
-  hw(dom->time, 0.0);
-  hw(dom->cycle, 0u);
-  hw(dom->pad107, 0u);
-  hw(dom->dtcourant, 1e20);
-  hw(dom->dthydro, 1e20);
-  for (int k = 0; k < 14; ++k) hw(dom->misc[k], (uint32_t)(k + 1));
-  for (int k = 0; k < 808; ++k) hw(dom->params[k], (uint32_t)k);
-  for (int k = 0; k < TMP_FORCE; ++k) {  // every array: its initial values (topology arrays: the input)
+  for (int k = 0; k < NSLOT; ++k) hw0(dom->ptr[k], k < TMP_FORCE ? (void*)arr->addr[2 + k] : (void*)nullptr);
+  hw0(dom->numElem, (uint32_t)ne);
+  hw0(dom->numNode, (uint32_t)nn);
+  hw0(dom->dt, 1e-3);
+  hw0(dom->time, 0.0);
+  hw0(dom->cycle, 0u);
+  hw0(dom->pad107, 0u);
+  hw0(dom->dtcourant, 1e20);
+  hw0(dom->dthydro, 1e20);
+  for (int k = 0; k < 14; ++k) hw0(dom->misc[k], (uint32_t)(k + 1));
+  for (int k = 0; k < 808; ++k) hw0(dom->params[k], (uint32_t)k);
+  // every array: its initial values (topology arrays: the input); a rank traces
+  // its slice [i0, i1) of the element indices and writes the rest untraced
+  auto slice = [&](uint64_t n, uint64_t* i0, uint64_t* i1) {
+    const uint64_t per = (n + R - 1) / R;
+    *i0 = std::min<uint64_t>(n, per * rk);
+    *i1 = std::min<uint64_t>(n, *i0 + per);
+  };
+  for (int k = 0; k < TMP_FORCE; ++k) {
     const uint64_t bytes = arr->bytes[2 + k];
-    if (k >= NODELIST && k <= ELEMBC) {
+    uint64_t i0, i1;
+    if (k >= NODELIST) {
       int* a = (int*)arr->addr[2 + k];
-      for (uint64_t i = 0; i < bytes / 4; ++i) hw(a[i], a[i]);
-    } else if (k >= NODELIST) {
-      int* a = (int*)arr->addr[2 + k];
-      for (uint64_t i = 0; i < bytes / 4; ++i) hw(a[i], 0);
+      slice(bytes / 4, &i0, &i1);
+      const bool topo = k <= ELEMBC;
+      for (uint64_t i = 0; i < bytes / 4; ++i) {
+        const int v = topo ? a[i] : 0;
+        if (i >= i0 && i < i1) hw(a[i], v);
+        else a[i] = v;
+      }
     } else {
       double* a = (double*)arr->addr[2 + k];
-      for (uint64_t i = 0; i < bytes / 8; ++i) hw(a[i], 1.0 + (double)(i & 7) * 0.125);
+      slice(bytes / 8, &i0, &i1);
+      for (uint64_t i = 0; i < bytes / 8; ++i) {
+        const double v = 1.0 + (double)(i & 7) * 0.125;
+        if (i >= i0 && i < i1) hw(a[i], v);
+        else a[i] = v;
+      }
     }
   }
-  for (int b = 0; b < 2 * nblk; ++b) hw(dtb[b], 0.0);
+  {
+    uint64_t i0, i1;
+    slice(2 * nblk, &i0, &i1);
+    for (int b = 0; b < 2 * nblk; ++b) {
+      if ((uint64_t)b >= i0 && (uint64_t)b < i1) hw(dtb[b], 0.0);
+      else dtb[b] = 0.0;
+    }
+  }
   host_t(t0);
 
   for (int step = 0; step < steps; ++step) {
     // forces: a temporary for the 8 corner forces of every element
     void* tf = managed(sizeof(double) * 24 * (size_t)ne);
     if (tmp_addrs) tmp_addrs[2 * step] = (unsigned long long)tf;
-    hw(dom->ptr[TMP_FORCE], tf);
-    LAUNCH(k_zero_forces, (nn + 255) / 256, dom, nn, hook_count);
-    LAUNCH(k_integrate_stress, nblk, dom, hook_count);
-    LAUNCH(k_hourglass, nblk, dom, hook_count);
-    LAUNCH(k_corner_sum, (nn + 255) / 256, dom, nn, hook_count);
+    hw0(dom->ptr[TMP_FORCE], tf);
+    LAUNCH(k_zero_forces, GN, dom, nn, hook_count);
+    LAUNCH(k_integrate_stress, GE, dom, hook_count);
+    LAUNCH(k_hourglass, GE, dom, hook_count);
+    LAUNCH(k_corner_sum, GN, dom, nn, hook_count);
     okc(cudaStreamSynchronize(st));
-    hw(dom->ptr[TMP_FORCE], (void*)nullptr);
+    hw0(dom->ptr[TMP_FORCE], (void*)nullptr);
     flush();
     release(tf);
-    LAUNCH(k_accel, (nn + 255) / 256, dom, nn, hook_count);
-    LAUNCH(k_symm, (nsym + 255) / 256, dom, nsym, hook_count);
-    LAUNCH(k_velocity, (nn + 255) / 256, dom, nn, hook_count);
-    LAUNCH(k_position, (nn + 255) / 256, dom, nn, hook_count);
+    LAUNCH(k_accel, GN, dom, nn, hook_count);
+    LAUNCH(k_symm, GS, dom, nsym, hook_count);
+    LAUNCH(k_velocity, GN, dom, nn, hook_count);
+    LAUNCH(k_position, GN, dom, nn, hook_count);
     // kinematics: a temporary for the velocity gradients
     void* tg = managed(sizeof(double) * 3 * (size_t)ne);
     if (tmp_addrs) tmp_addrs[2 * step + 1] = (unsigned long long)tg;
-    hw(dom->ptr[TMP_DVDX], tg);
-    LAUNCH(k_kinematics, nblk, dom, hook_count);
-    LAUNCH(k_lagrange, nblk, dom, hook_count);
+    hw0(dom->ptr[TMP_DVDX], tg);
+    LAUNCH(k_kinematics, GE, dom, hook_count);
+    LAUNCH(k_lagrange, GE, dom, hook_count);
     okc(cudaStreamSynchronize(st));
-    hw(dom->ptr[TMP_DVDX], (void*)nullptr);
+    hw0(dom->ptr[TMP_DVDX], (void*)nullptr);
     flush();
     release(tg);
-    LAUNCH(k_monoq_grad, nblk, dom, hook_count);
-    LAUNCH(k_monoq_region, nblk, dom, hook_count);
-    for (int stage = 0; stage < 4; ++stage) LAUNCH(k_eos, nblk, dom, stage, hook_count);
-    LAUNCH(k_update_volumes, nblk, dom, hook_count);
-    launch([&](int g) { k_dt<true, true><<<g, 256, 0, st>>>(dom, dtb, nblk, hook_count); },
-           [&](int g) { k_dt<false, true><<<g, 256, 0, st>>>(dom, dtb, nblk, hook_count); }, nblk);
-    launch([&](int g) { k_dt<true, false><<<g, 256, 0, st>>>(dom, dtb, nblk, hook_count); },
-           [&](int g) { k_dt<false, false><<<g, 256, 0, st>>>(dom, dtb, nblk, hook_count); }, nblk);
+    LAUNCH(k_monoq_grad, GE, dom, hook_count);
+    LAUNCH(k_monoq_region, GE, dom, hook_count);
+    for (int stage = 0; stage < 4; ++stage) LAUNCH(k_eos, GE, dom, stage, hook_count);
+    LAUNCH(k_update_volumes, GE, dom, hook_count);
+    launch([&](int g) { k_dt<true, true><<<g, 256, 0, st>>>(P, dom, dtb, nblk, hook_count); },
+           [&](int g) { k_dt<false, true><<<g, 256, 0, st>>>(P, dom, dtb, nblk, hook_count); }, GE);
+    launch([&](int g) { k_dt<true, false><<<g, 256, 0, st>>>(P, dom, dtb, nblk, hook_count); },
+           [&](int g) { k_dt<false, false><<<g, 256, 0, st>>>(P, dom, dtb, nblk, hook_count); }, GE);
     okc(cudaStreamSynchronize(st));
     // TimeIncrement (host): the dt minima, the domain's parameters, the new dt
+    // (traced by rank 0: one copy in the logical program)
     t0 = std::chrono::steady_clock::now();
     double dc = 1e30, dh = 1e30;
     for (int b = 0; b < nblk; ++b) {
-      const double v = tr ? tr->read(dtb[b]) : dtb[b];
+      const double v = tr0 ? tr0->read(dtb[b]) : dtb[b];
       dc = v < dc ? v : dc;
     }
     for (int b = 0; b < nblk; ++b) {
-      const double v = tr ? tr->read(dtb[nblk + b]) : dtb[nblk + b];
+      const double v = tr0 ? tr0->read(dtb[nblk + b]) : dtb[nblk + b];
       dh = v < dh ? v : dh;
     }
-    run->host_accesses += 2 * nblk;
-    hw(dom->dtcourant, dc);
-    hw(dom->dthydro, dh);
+    if (rk == 0) run->host_accesses += 2 * nblk;
+    hw0(dom->dtcourant, dc);
+    hw0(dom->dthydro, dh);
     const uint32_t* w = (const uint32_t*)dom;
     uint64_t chk = 0;
-    for (int k = 100; k < 780; ++k) chk += tr ? tr->read(w[k]) : w[k];  // 680 words of parameters
-    run->host_accesses += 680;
-    hw(dom->dt, 1e-3 + (double)(chk & 1) * 1e-9);
-    hw(dom->time, dom->time + 1e-3);
-    hw(dom->cycle, (uint32_t)(step + 1));
-    for (int k = 0; k < 14; ++k) hw(dom->misc[k], (uint32_t)(k + 1));
+    for (int k = 100; k < 780; ++k) chk += tr0 ? tr0->read(w[k]) : w[k];  // 680 words of parameters
+    if (rk == 0) run->host_accesses += 680;
+    hw0(dom->dt, 1e-3 + (double)(chk & 1) * 1e-9);
+    hw0(dom->time, dom->time + 1e-3);
+    hw0(dom->cycle, (uint32_t)(step + 1));
+    for (int k = 0; k < 14; ++k) hw0(dom->misc[k], (uint32_t)(k + 1));
     host_t(t0);
     if (run->diag_each) diag();  // "diagnostics are called at the end of every timestep"
   }

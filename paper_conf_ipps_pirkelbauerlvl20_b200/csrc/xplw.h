@@ -50,6 +50,8 @@ typedef struct {
   int diag_no_reset;      /* 1 = diagnoses keep the interval bits (D25)            */
   int keep_allocs;        /* 1 = leave the arrays registered at the end (no final  *
                            *     frees + diagnose), for shadow dumps (LULESH)      */
+  int rank, world;        /* world > 1: this process is rank `rank` of a sharded  *
+                           * run (ctx sharded too); LULESH runs its slab only     */
 } xplw_run;
 
 /* Rodinia hotspot: rows x cols temperatures, `iters` 5-point stencil steps.

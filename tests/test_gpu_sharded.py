@@ -170,3 +170,71 @@ def test_nccl_comm_single_rank():
         assert c.barrier(c.user) == 0
     finally:
         comm.close()
+
+
+def _lulesh_rank(rank, world, port, s, steps, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    import torch
+    import torch.distributed as dist
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        torch.cuda.set_device(0)
+        from paper_conf_ipps_pirkelbauerlvl20_b200 import apps, xpl
+        from xplgen import lulesh as L
+        spec = L.lulesh_spec(s)
+        ar = apps.Arena(spec)
+        apps.lulesh_prepare(ar, s, L.topology(s, 0x58504C05))
+        hc = torch.zeros(1, dtype=torch.int64, device="cuda")
+        st = torch.cuda.Stream()
+        with xpl.Context(pool_words=1 << 24, max_rows=256, comm=xpl.TorchComm()) as ctx:
+            run = apps.Run(ctx, st.cuda_stream, params=(50, 0, 256), rank=rank, world=world)
+            apps.lulesh(run, ar, s, steps, hc)
+            q.put((rank, run.reports(), int(hc.item())))
+    except Exception as ex:  # noqa: BLE001
+        import traceback
+        q.put((rank, "ERR " + repr(ex) + traceback.format_exc(), 0))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,s", [(2, 8), (3, 24)])
+def test_sharded_lulesh_equals_one_gpu_and_oracle(world, s):
+    """The sharded LULESH-shaped program (each rank its slab of elements and
+    nodes, its slice of the host init; rank 0 the domain's host segments) on a
+    sharded context: every rank's reports equal the oracle's replay of the
+    single-GPU program (all fields but `base`, the piece owners' addresses) --
+    the 1-GPU vs N-GPU report identity of SURVEY §8(d) cfg5."""
+    import torch
+    import torch.multiprocessing as mp
+    from oracle import run_trace
+    from paper_conf_ipps_pirkelbauerlvl20_b200 import apps, xpl
+    from xplgen import lulesh as L
+    steps = 3
+    # the single-GPU program and its oracle
+    spec = L.lulesh_spec(s)
+    ar = apps.Arena(spec)
+    topo = L.topology(s, 0x58504C05)
+    apps.lulesh_prepare(ar, s, topo)
+    hc = torch.zeros(1, dtype=torch.int64, device="cuda")
+    st = torch.cuda.Stream()
+    with xpl.Context(pool_words=1 << 24) as ctx1:
+        run = apps.Run(ctx1, st.cuda_stream, params=(50, 0, 256))
+        tmps = apps.lulesh(run, ar, s, steps, hc)
+        one = run.reports()
+    ops, hooks = L.lulesh_trace(ar.addrs, spec, s, steps, topo, (50, 0, 256), tmps)
+    exp = run_trace(ops)
+    strip = lambda ds: [[{f: v for f, v in r.items() if f != "base"} for r in d] for d in ds]
+    assert strip(one) == strip(exp)
+    ctxm = mp.get_context("spawn")
+    q = ctxm.Queue()
+    port = 29800 + s + world + os.getpid() % 500
+    procs = [ctxm.Process(target=_lulesh_rank, args=(r, world, port, s, steps, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = {r: (g, h) for r, g, h in (q.get(timeout=600) for _ in procs)}
+    for p in procs:
+        p.join(timeout=60)
+    for r in range(world):
+        assert not isinstance(res[r][0], str), res[r][0]
+        assert strip(res[r][0]) == strip(exp), f"rank {r}"
