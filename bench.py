@@ -161,6 +161,28 @@ def cpu_baseline(seconds_budget=None):
                       f"{dt:.1f} s, 1 thread)"}
 
 
+def _allsum(torch, dist, x):
+    if not dist.is_available() or not dist.is_initialized():
+        return x
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([x], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.SUM)
+    return float(t.item())
+
+
+def make_comm(xpl, torch, dist, rank, world, local, backend):
+    """The sharded context's collectives: libxpl.so's own NCCL communicator (its
+    unique id broadcast over the process group), or gloo through torch."""
+    if backend != "nccl":
+        return xpl.TorchComm()
+
+    def bcast(b):
+        t = torch.tensor(list(b), dtype=torch.uint8, device="cuda")
+        dist.broadcast(t, 0)
+        return bytes(t.cpu().tolist())
+    return xpl.NcclComm(rank, world, local, bcast)
+
+
 def _allmax(torch, dist, x):
     if not dist.is_available() or not dist.is_initialized():
         return x
@@ -300,9 +322,10 @@ def diag_at_scale(xpl, torch, words=1 << 31, reps=3):
 class Cfg4:
     """The cfg4 program's arrays, input and runs."""
 
-    def __init__(self, torch, apps, timesteps):
+    def __init__(self, torch, apps, timesteps, rank=0, world=1):
         from xplgen import lulesh as L
         self.torch, self.apps, self.T = torch, apps, timesteps
+        self.rank, self.world = rank, world  # world > 1: the sharded program (this rank's slab)
         self.spec = L.lulesh_spec(S4)
         self.ar = apps.Arena(self.spec)
         self.topo = L.topology(S4, SEED4)
@@ -321,7 +344,7 @@ class Cfg4:
         if upload:
             self.apps.lulesh_upload(self.ar, self.host_topo, self.us.cuda_stream)
         run = self.apps.Run(ctx, self.us.cuda_stream, params=params, out_cap=64 * (self.T + 2),
-                            time_kernels=time_kernels)
+                            time_kernels=time_kernels, rank=self.rank, world=self.world)
         self.apps.lulesh(run, self.ar, S4, self.T, self.hc)
         return run
 
@@ -350,6 +373,7 @@ def timed_steps(torch, c4, ctx, steps, upload=False, flush=None):
         torch.cuda.synchronize()
         total += e0.elapsed_time(e1)
         acc.append((int(c4.hc.item()), run.r.host_accesses, run.r.epochs, run.r.n_diag, run.r.n_out))
+    c4.last_reports = run.reports() if ctx is not None else None
     return total, acc
 
 
@@ -477,6 +501,56 @@ def other_configs(xpl, apps, torch, lulesh250_steps=100):
     return out
 
 
+def hook_roofline(args, k_instr, k_twin, ms_step, prof, peak, peak_src):
+    hook_ms = (k_instr - k_twin) / args.timesteps  # per timestep
+    hook_bytes = HOOK_BYTES_PER_WORD * CFG4_WORDS_PER_TIMESTEP
+    ach = hook_bytes / (hook_ms / 1e3) / 1e9 if hook_ms > 0 else None
+    return {"kernel": "device hooks (a3), inlined in the 19 instrumented launches of each timestep",
+            "bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s",
+            "frac": (ach / peak) if ach else None, "traffic": None, "peak_source": peak_src,
+            "algorithmic_bytes_per_timestep": hook_bytes,
+            "algorithmic_model": "2 B (shadow byte read + written) per distinct word per epoch; "
+                                 f"{CFG4_WORDS_PER_TIMESTEP} distinct words per timestep (tools/lulesh_words.py)",
+            "hook_ms_per_timestep": hook_ms,
+            "timing": "sum of CUDA-event kernel times on the program's stream, instrumented minus twin, one step each",
+            "share_of_step": (k_instr - k_twin) / ms_step,
+            "runtime_kernels_ms_per_step": {k: v["ms"] for k, v in prof.items() if k != "diagnose"}}
+
+
+def sharded_tail(args, torch, dist, apps, xpl, rank, world, value, ms_max, per_step, epochs, n_diag, e2e,
+                 launches, clocks, twin_ms, k_instr, k_twin, prof, sharded_reports, peak, peak_src, backend):
+    """N > 1: the line of the sharded cfg4 program; rank 0 also runs the 1-GPU
+    program and checks every report (but `base`) is identical."""
+    identical = None
+    if rank == 0:
+        c1 = Cfg4(torch, apps, args.timesteps)
+        with xpl.Context(device=torch.cuda.current_device(), pool_words=1 << 28, max_rows=64) as ctx1:
+            c1.prepare()
+            one = c1.run(ctx1).reports()
+        strip = lambda ds: [[{f: v for f, v in r.items() if f != "base"} for r in d] for d in ds]
+        identical = strip(one) == strip(sharded_reports)
+    roof = hook_roofline(args, k_instr, k_twin, ms_max / args.steps, prof, peak, peak_src)
+    line = {"metric": METRIC, "value": value, "unit": "accesses/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+            "config": {"workload": WORKLOAD + f", sharded over {world} GPUs (one logical program: each rank "
+                                              "its slab of elements/nodes; shadow partitioned by word, host "
+                                              "records routed all-to-all, remote hook atomics, partials combined)",
+                       "timesteps": args.timesteps, "accesses_per_step": per_step, "epochs_per_step": epochs,
+                       "diagnoses_per_step": n_diag, "parallelism": f"sharded x{world}",
+                       "collectives": "NCCL (libxpl.so xpl_comm_nccl)" if backend == "nccl" else backend,
+                       "l2": "flushed between steps (256 MB write, untimed)"},
+            "roofline": roof, "e2e": e2e, "gpu_launches": int(launches), "clocks": clocks,
+            "summary": {"accesses_per_s": value, "e2e_accesses_per_s": e2e["value"],
+                        "reports_identical_to_1gpu": identical,
+                        "slowdown_whole_program": (ms_max / args.steps) / (twin_ms / args.steps),
+                        "slowdown_kernels": k_instr / k_twin if k_twin else None}}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    dist.barrier()
+    dist.destroy_process_group()
+
+
 def reference_main(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
@@ -515,8 +589,11 @@ def main():
 
     from paper_conf_ipps_pirkelbauerlvl20_b200 import apps, xpl
 
-    c4 = Cfg4(torch, apps, args.timesteps)
-    ctx = xpl.Context(device=local, pool_words=1 << 28, max_rows=64)
+    # N > 1: the cfg4 program sharded over the ranks (each its slab; one logical
+    # program, shadow partitioned by word over the GPUs, xpl.h sharded mode)
+    c4 = Cfg4(torch, apps, args.timesteps, rank, world)
+    comm = make_comm(xpl, torch, dist, rank, world, local, backend) if world > 1 else None
+    ctx = xpl.Context(device=local, pool_words=1 << 28, max_rows=256, comm=comm)
     flush_buf = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")  # > 126 MB L2
 
     clk = Clocks(local)
@@ -535,9 +612,9 @@ def main():
     clocks = clk.stop()
     st1 = ctx.stats()
     hooks, host_acc, epochs, n_diag, n_rows = acc[-1]
-    per_step = hooks + host_acc
+    per_step = int(_allsum(torch, dist, hooks + host_acc))  # the logical program's accesses
     ms_max = _allmax(torch, dist, ms_total)
-    value = per_step * args.steps * world / (ms_max / 1e3)
+    value = per_step * args.steps / (ms_max / 1e3)
     launches = (st1["kernel_launches"] - st0["kernel_launches"]) + epochs * args.steps
     if args.step_only:
         ctx.close()
@@ -551,12 +628,14 @@ def main():
     st1 = ctx.stats()
     e2e_ms = _allmax(torch, dist, e2e_ms)
     rec_bytes = 8 * (st1["host_records_packed"] - st0["host_records_packed"]) // args.steps
-    e2e = {"value": per_step * args.steps * world / (e2e_ms / 1e3), "unit": "accesses/s",
+    e2e = {"value": per_step * args.steps / (e2e_ms / 1e3), "unit": "accesses/s",
            "h2d_bytes_per_step": c4.input_bytes + rec_bytes,
            "d2h_bytes_per_step": xpl.REPORT_BYTES * n_rows}
 
     # --- uninstrumented twin (whole-program slowdown) ---------------------------
     twin_ms, _ = timed_steps(torch, c4, None, args.steps, flush=flush_buf)
+    twin_ms = _allmax(torch, dist, twin_ms)
+    sharded_reports = c4.last_reports if world > 1 else None
 
     # --- hook path: kernels alone, instrumented vs twin, events on their stream --
     c4.prepare()
@@ -564,7 +643,7 @@ def main():
     c4.prepare()
     rt = c4.run(None, time_kernels=True)
     torch.cuda.synchronize()
-    k_instr, k_twin = ri.r.kernel_ms, rt.r.kernel_ms
+    k_instr, k_twin = _allmax(torch, dist, ri.r.kernel_ms), _allmax(torch, dist, rt.r.kernel_ms)
 
     # --- runtime kernels: a profiled re-run (events around every runtime kernel) --
     ctx.profile(True)
@@ -572,31 +651,26 @@ def main():
     prof = ctx.profile_read(reset=True)
     ctx.profile(False)
     ctx.close()
+    if comm is not None and hasattr(comm, "close"):
+        comm.close()
     del flush_buf
     torch.cuda.empty_cache()
 
-    # --- microbenchmarks and the other configs --------------------------------
     peak, peak_src = peaks()
+    if world > 1:
+        return sharded_tail(args, torch, dist, apps, xpl, rank, world, value, ms_max, per_step, epochs, n_diag,
+                            e2e, launches, clocks, twin_ms, k_instr, k_twin, prof, sharded_reports, peak, peak_src,
+                            backend)
+
+    # --- microbenchmarks and the other configs --------------------------------
     smb = stream_microbench(xpl, torch)
     at_scale = diag_at_scale(xpl, torch)
     atom = atomic_peaks(xpl, torch)
     others = other_configs(xpl, apps, torch) if not args.no_other_configs else None
 
     # --- roofline: the dominant cost of our path in the step = the device hooks --
-    hook_ms = (k_instr - k_twin) / args.timesteps          # per timestep
-    hook_bytes = HOOK_BYTES_PER_WORD * CFG4_WORDS_PER_TIMESTEP
-    ach = hook_bytes / (hook_ms / 1e3) / 1e9 if hook_ms > 0 else None
-    rt_ms = {k: v["ms"] for k, v in prof.items() if k != "diagnose"}
-    roof = {"kernel": "device hooks (a3), inlined in the 19 instrumented launches of each timestep",
-            "bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s",
-            "frac": (ach / peak) if ach else None, "traffic": None, "peak_source": peak_src,
-            "algorithmic_bytes_per_timestep": hook_bytes,
-            "algorithmic_model": "2 B (shadow byte read + written) per distinct word per epoch; "
-                                 f"{CFG4_WORDS_PER_TIMESTEP} distinct words per timestep (tools/lulesh_words.py)",
-            "hook_ms_per_timestep": hook_ms,
-            "timing": "sum of CUDA-event kernel times on the program's stream, instrumented minus twin, one step each",
-            "share_of_step": (k_instr - k_twin) / (ms_total / args.steps),
-            "runtime_kernels_ms_per_step": rt_ms}
+    roof = hook_roofline(args, k_instr, k_twin, ms_total / args.steps, prof, peak, peak_src)
+    rt_ms = roof["runtime_kernels_ms_per_step"]
     dg = prof["diag_tile"]
     line = {
         "metric": METRIC,

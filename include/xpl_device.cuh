@@ -340,6 +340,10 @@ static __device__ __forceinline__ void xpld_one(unsigned ones, unsigned long lon
   const unsigned qp = __shfl_up_sync(ones, q, 1);
   const bool start = lane == 0 || !((ones >> (lane - 1)) & 1u) || qp != q;
   const unsigned S = __ballot_sync(ones, start);
+  if (S == ones) { /* every lane its own group (strided or scattered): no grouping work */
+    xpld_put<K, TM>(q, cur, ((K ? K : acc) & XPL_ACC_R) ? bm : 0u, ((K ? K : acc) & XPL_ACC_W) ? bm : 0u);
+    return;
+  }
   const unsigned above = S & (0xFFFFFFFEu << lane); /* group starts after this lane */
   const unsigned gm = (above ? ((1u << (__ffs(above) - 1)) - 1u) : FULL) & (FULL << lane);
   unsigned rb, wb;
@@ -403,19 +407,17 @@ static __device__ __forceinline__ unsigned* xpld_row_cache() {
   return c;
 }
 
-template <unsigned K, bool TM = true>
-static __device__ __forceinline__ void xpl_dev_record_k(const void* p, unsigned size,
-                                                        unsigned acc) {
-#ifndef XPL_OFF
+/* The row (live allocation) holding address a: (base, end) and (off | owner
+ * << 56, words); false = untracked. */
+static __device__ __forceinline__ bool xpld_find(unsigned long long a, ulonglong2& be, ulonglong2& ow) {
   unsigned* const xpl_row_cache = xpld_row_cache();
-  const unsigned long long a = (unsigned long long)p;
   const xpl_dev_row* rows = xpl_dctx.rows;
   const unsigned n = __ldg(xpl_dctx.n_rows);
   const unsigned slot = ((threadIdx.z * blockDim.y + threadIdx.y) * blockDim.x + threadIdx.x) >> 5 & 31;
   unsigned ri = xpl_row_cache[slot];
   const unsigned rc = ri < n ? ri : 0; /* (n == 0: nothing matches below) */
-  ulonglong2 be = __ldg(reinterpret_cast<const ulonglong2*>(rows + rc));     /* base, end  */
-  ulonglong2 ow = __ldg(reinterpret_cast<const ulonglong2*>(rows + rc) + 1); /* off, words */
+  be = __ldg(reinterpret_cast<const ulonglong2*>(rows + rc));     /* base, end  */
+  ow = __ldg(reinterpret_cast<const ulonglong2*>(rows + rc) + 1); /* off, words */
   bool hit = ri < n && be.x <= a && a < be.y;
   if (!hit) {
     unsigned lo = 0, hi = n;
@@ -432,27 +434,85 @@ static __device__ __forceinline__ void xpl_dev_record_k(const void* p, unsigned 
       ow = __ldg(reinterpret_cast<const ulonglong2*>(rows + ri) + 1);
     }
   }
-  unsigned long long g0 = 1, g1 = 0;
-  unsigned owner = 0;
-  if (hit && size > 0) {
-    const unsigned long long base = be.x;
-    const unsigned long long w0 = (a - base) >> 2;
-    unsigned long long wl = (a + size - 1 - base) >> 2;
-    const unsigned long long wmax = ow.y - 1;
-    if (wl > wmax) wl = wmax;
-    owner = (unsigned)(ow.x >> 56);
-    g0 = (ow.x & XPLD_OFF_MASK) + w0;
-    g1 = (ow.x & XPLD_OFF_MASK) + wl;
-  }
+  return hit;
+}
+
+/* Words [g0, g1] (in the owner's pool) of an access of `size` bytes at a in the
+ * row (be, ow): clipped to the row (D1, D18). */
+static __device__ __forceinline__ void xpld_words(unsigned long long a, unsigned size, const ulonglong2& be,
+                                                  const ulonglong2& ow, unsigned long long& g0,
+                                                  unsigned long long& g1, unsigned& owner) {
+  const unsigned long long w0 = (a - be.x) >> 2;
+  unsigned long long wl = (a + size - 1 - be.x) >> 2;
+  if (wl > ow.y - 1) wl = ow.y - 1;
+  owner = (unsigned)(ow.x >> 56);
+  g0 = (ow.x & XPLD_OFF_MASK) + w0;
+  g1 = (ow.x & XPLD_OFF_MASK) + wl;
+}
+
+/* Record words [g0, g1] of rank `owner`'s pool (g0 > g1: nothing).  All active
+ * lanes of the warp call it. */
+template <unsigned K, bool TM = true>
+static __device__ __forceinline__ void xpld_record_words(unsigned long long g0, unsigned long long g1,
+                                                         unsigned owner, unsigned acc) {
   /* sharded mode: words another rank owns go to its pool over NVLink (rare) */
   const bool remote = owner != xpl_dctx.rank && g0 <= g1;
   const unsigned long long l0 = remote ? 1ull : g0, l1 = remote ? 0ull : g1;
-  xpl_dev_apply<K, TM>(l0, l1, K ? K : acc);
-  if (__any_sync(__activemask(), remote) && remote) xpld_remote<K>(owner, g0, g1, K ? K : acc);
+  xpl_dev_apply<K, TM>(l0, l1, acc);
+  if (__any_sync(__activemask(), remote) && remote) xpld_remote<K>(owner, g0, g1, acc);
+}
+
+template <unsigned K, bool TM = true>
+static __device__ __forceinline__ void xpl_dev_record_k(const void* p, unsigned size,
+                                                        unsigned acc) {
+#ifndef XPL_OFF
+  const unsigned long long a = (unsigned long long)p;
+  ulonglong2 be, ow;
+  unsigned long long g0 = 1, g1 = 0;
+  unsigned owner = xpl_dctx.rank;
+  if (xpld_find(a, be, ow) && size > 0) xpld_words(a, size, be, ow, g0, g1, owner);
+  xpld_record_words<K, TM>(g0, g1, owner, K ? K : acc);
 #else
   (void)p; (void)size; (void)acc;
 #endif
 }
+
+/* traceR / traceW / traceRW through an array handle: the row lookup of the
+ * array's base pointer is done once (when the handle is made) instead of once
+ * per access -- the hoisting an instrumenting compiler does for a loop-invariant
+ * base.  Same records as xpl_read(p[i]) etc.: an element outside the handle's
+ * row falls back to the full lookup (D18: an access belongs to the row holding
+ * its first byte). */
+template <class T>
+struct xpl_array {
+  T* p;
+  ulonglong2 be, ow; /* the row of p; be = {0, 0}: none */
+  __device__ __forceinline__ explicit xpl_array(T* ptr) : p(ptr) {
+#ifndef XPL_OFF
+    if (!xpld_find((unsigned long long)ptr, be, ow)) be = make_ulonglong2(0, 0);
+#endif
+  }
+  template <unsigned K>
+  __device__ __forceinline__ void rec(unsigned long long i) const {
+#ifndef XPL_OFF
+    const unsigned long long a = (unsigned long long)(p + i);
+    unsigned long long g0 = 1, g1 = 0;
+    unsigned owner = xpl_dctx.rank;
+    if (a - be.x < be.y - be.x) {
+      xpld_words(a, sizeof(T), be, ow, g0, g1, owner);
+    } else {
+      ulonglong2 b2, o2;
+      if (xpld_find(a, b2, o2)) xpld_words(a, sizeof(T), b2, o2, g0, g1, owner);
+    }
+    xpld_record_words<K>(g0, g1, owner, K);
+#else
+    (void)i;
+#endif
+  }
+  __device__ __forceinline__ const T& read(unsigned long long i) const { rec<XPL_ACC_R>(i); return p[i]; }
+  __device__ __forceinline__ T& write(unsigned long long i) const { rec<XPL_ACC_W>(i); return p[i]; }
+  __device__ __forceinline__ T& rw(unsigned long long i) const { rec<XPL_ACC_RW>(i); return p[i]; }
+};
 
 /* Generic form: acc may differ from lane to lane. */
 static __device__ __forceinline__ void xpl_dev_record(const void* p, unsigned size, unsigned acc) {

@@ -78,6 +78,22 @@ __device__ __forceinline__ T& RW(T& x) {
   else return x;
 }
 
+// Arrays a thread accesses several times go through array handles (the row
+// lookup of the base pointer hoisted out of the accesses, xpl_array); the twin
+// gets a plain pointer with the same interface.
+template <bool I, class T>
+struct Arr : xpl_array<T> {
+  __device__ __forceinline__ explicit Arr(T* q) : xpl_array<T>(q) {}
+};
+template <class T>
+struct Arr<false, T> {
+  T* p;
+  __device__ __forceinline__ explicit Arr(T* q) : p(q) {}
+  __device__ __forceinline__ const T& read(unsigned long long i) const { return p[i]; }
+  __device__ __forceinline__ T& write(unsigned long long i) const { return p[i]; }
+  __device__ __forceinline__ T& rw(unsigned long long i) const { return p[i]; }
+};
+
 // Hook calls are counted per thread (c) and added once per block (exact counts).
 template <bool I>
 __device__ __forceinline__ void count_hooks(unsigned long long* hc, unsigned c) {
@@ -96,6 +112,10 @@ __device__ __forceinline__ void count_hooks(unsigned long long* hc, unsigned c) 
 #define W_(x) (++c, WR<I>(x))
 #define RW_(x) (++c, RW<I>(x))
 #define PTR(T, slot) static_cast<T*>(R_(d->ptr[slot]))
+#define ARR(T, slot) Arr<I, T>(PTR(T, slot))
+#define RA_(h, i) (++c, (h).read(i))
+#define WA_(h, i) (++c, (h).write(i))
+#define RWA_(h, i) (++c, (h).rw(i))
 #define NE() (int)R_(d->numElem)
 
 // 1. zero the nodal forces
@@ -118,16 +138,16 @@ __global__ void k_integrate_stress(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   if (e < P_.e1 && e < NE()) {
-    const int* nl = PTR(const int, NODELIST);
-    const double *x = PTR(const double, X), *y = PTR(const double, Y), *z = PTR(const double, Z);
+    const auto nl = ARR(const int, NODELIST);
+    const auto x = ARR(const double, X), y = ARR(const double, Y), z = ARR(const double, Z);
     const double sig = -(R_(PTR(const double, P)[e]) + R_(PTR(const double, Q)[e]));
-    double* f = PTR(double, TMP_FORCE);
+    const auto f = ARR(double, TMP_FORCE);
     for (int k = 0; k < 8; ++k) {
-      const int n = R_(nl[8 * e + k]);
-      const double g = R_(x[n]) + R_(y[n]) + R_(z[n]);
-      W_(f[24 * e + 3 * k + 0]) = sig * g;
-      W_(f[24 * e + 3 * k + 1]) = sig * g * 0.5;
-      W_(f[24 * e + 3 * k + 2]) = sig * g * 0.25;
+      const int n = RA_(nl, 8 * e + k);
+      const double g = RA_(x, n) + RA_(y, n) + RA_(z, n);
+      WA_(f, 24 * e + 3 * k + 0) = sig * g;
+      WA_(f, 24 * e + 3 * k + 1) = sig * g * 0.5;
+      WA_(f, 24 * e + 3 * k + 2) = sig * g * 0.25;
     }
   }
   count_hooks<I>(hc, c);
@@ -139,17 +159,17 @@ __global__ void k_hourglass(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   if (e < P_.e1 && e < NE()) {
-    const int* nl = PTR(const int, NODELIST);
-    const double *xd = PTR(const double, XD), *yd = PTR(const double, YD), *zd = PTR(const double, ZD);
+    const auto nl = ARR(const int, NODELIST);
+    const auto xd = ARR(const double, XD), yd = ARR(const double, YD), zd = ARR(const double, ZD);
     const double coef = R_(PTR(const double, SS)[e]) * R_(PTR(const double, ELEMMASS)[e]) /
                         (R_(PTR(const double, VOLO)[e]) * R_(PTR(const double, V)[e]) + 1.0);
-    double* f = PTR(double, TMP_FORCE);
+    const auto f = ARR(double, TMP_FORCE);
     for (int k = 0; k < 8; ++k) {
-      const int n = R_(nl[8 * e + k]);
-      const double a = R_(xd[n]), b = R_(yd[n]), g = R_(zd[n]);
-      RW_(f[24 * e + 3 * k + 0]) += coef * a;
-      RW_(f[24 * e + 3 * k + 1]) += coef * b;
-      RW_(f[24 * e + 3 * k + 2]) += coef * g;
+      const int n = RA_(nl, 8 * e + k);
+      const double a = RA_(xd, n), b = RA_(yd, n), g = RA_(zd, n);
+      RWA_(f, 24 * e + 3 * k + 0) += coef * a;
+      RWA_(f, 24 * e + 3 * k + 1) += coef * b;
+      RWA_(f, 24 * e + 3 * k + 2) += coef * g;
     }
   }
   count_hooks<I>(hc, c);
@@ -161,16 +181,16 @@ __global__ void k_corner_sum(Part P_, Dom* d, int nn, unsigned long long* hc) {
   const int n = P_.n0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   if (n < P_.n1 && n < nn) {
-    const int *st = PTR(const int, NODEELEMSTART), *cl = PTR(const int, CORNERLIST);
-    const double* f = PTR(const double, TMP_FORCE);
+    const auto st = ARR(const int, NODEELEMSTART), cl = ARR(const int, CORNERLIST);
+    const auto f = ARR(const double, TMP_FORCE);
     double *fx = PTR(double, FX), *fy = PTR(double, FY), *fz = PTR(double, FZ);
-    const int b = R_(st[n]), en = R_(st[n + 1]);
+    const int b = RA_(st, n), en = RA_(st, n + 1);
     double sx = 0, sy = 0, sz = 0;
     for (int k = b; k < en; ++k) {
-      const int corner = R_(cl[k]);
-      sx += R_(f[3 * corner + 0]);
-      sy += R_(f[3 * corner + 1]);
-      sz += R_(f[3 * corner + 2]);
+      const int corner = RA_(cl, k);
+      sx += RA_(f, 3 * corner + 0);
+      sy += RA_(f, 3 * corner + 1);
+      sz += RA_(f, 3 * corner + 2);
     }
     W_(fx[n]) = sx;
     W_(fy[n]) = sy;
@@ -245,24 +265,24 @@ __global__ void k_kinematics(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   if (e < P_.e1 && e < NE()) {
-    const int* nl = PTR(const int, NODELIST);
-    const double *x = PTR(const double, X), *y = PTR(const double, Y), *z = PTR(const double, Z);
-    const double *xd = PTR(const double, XD), *yd = PTR(const double, YD), *zd = PTR(const double, ZD);
+    const auto nl = ARR(const int, NODELIST);
+    const auto x = ARR(const double, X), y = ARR(const double, Y), z = ARR(const double, Z);
+    const auto xd = ARR(const double, XD), yd = ARR(const double, YD), zd = ARR(const double, ZD);
     double vol = 0, dv = 0;
     for (int k = 0; k < 8; ++k) {
-      const int n = R_(nl[8 * e + k]);
-      vol += R_(x[n]) * R_(y[n]) + R_(z[n]);
-      dv += R_(xd[n]) + R_(yd[n]) + R_(zd[n]);
+      const int n = RA_(nl, 8 * e + k);
+      vol += RA_(x, n) * RA_(y, n) + RA_(z, n);
+      dv += RA_(xd, n) + RA_(yd, n) + RA_(zd, n);
     }
     const double vnew = vol / (R_(PTR(const double, VOLO)[e]) + 1.0);
     const double vold = R_(PTR(const double, V)[e]);
     W_(PTR(double, VNEW)[e]) = vnew;
     W_(PTR(double, DELV)[e]) = vnew - vold;
     W_(PTR(double, AREALG)[e]) = vol;
-    double* g = PTR(double, TMP_DVDX);
-    W_(g[3 * e + 0]) = dv;
-    W_(g[3 * e + 1]) = dv * 0.5;
-    W_(g[3 * e + 2]) = dv * 0.25;
+    const auto g = ARR(double, TMP_DVDX);
+    WA_(g, 3 * e + 0) = dv;
+    WA_(g, 3 * e + 1) = dv * 0.5;
+    WA_(g, 3 * e + 2) = dv * 0.25;
   }
   count_hooks<I>(hc, c);
 }
@@ -273,8 +293,8 @@ __global__ void k_lagrange(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   if (e < P_.e1 && e < NE()) {
-    const double* g = PTR(const double, TMP_DVDX);
-    const double r = (R_(g[3 * e]) + R_(g[3 * e + 1]) + R_(g[3 * e + 2])) / (R_(PTR(const double, VNEW)[e]) + 1.0);
+    const auto g = ARR(const double, TMP_DVDX);
+    const double r = (RA_(g, 3 * e) + RA_(g, 3 * e + 1) + RA_(g, 3 * e + 2)) / (R_(PTR(const double, VNEW)[e]) + 1.0);
     W_(PTR(double, VDOV)[e]) = r;
   }
   count_hooks<I>(hc, c);

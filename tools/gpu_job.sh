@@ -10,6 +10,7 @@
 #   launches               ncu launch list (gpu__time_duration.sum) of a short bench run
 #   ncu:REGEX[:SKIP[:CMD]] ncu --set full of one launch of kernel REGEX (default command: bench.py --step-only)
 #   py:SCRIPT[:ARGS]       python SCRIPT ARGS > TAG_<name>.json
+#   sanitize:TOOL          compute-sanitizer --tool TOOL (memcheck|synccheck|racecheck) over tools/sanitize_driver.py
 TAG=$1; shift
 mkdir -p gpurun_out
 echo "nproc=$(nproc) $(nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv,noheader)" > gpurun_out/${TAG}_box.txt
@@ -35,6 +36,8 @@ for step in "$@"; do
     py) script=${rest%%:*}; a2=${rest#*:}; [ "$a2" = "$rest" ] && a2=""
         name=$(basename "$script" .py)
         timeout 1800 python $script ${a2//+/ } > gpurun_out/${TAG}_$name.json 2> gpurun_out/${TAG}_$name.err ;;
+    sanitize) timeout 1500 compute-sanitizer --tool $rest --print-limit 50 python tools/sanitize_driver.py \
+                > gpurun_out/${TAG}_sanitize_$rest.log 2>&1; echo "rc=$?" >> gpurun_out/${TAG}_sanitize_$rest.log ;;
     *) echo "unknown step $step" >> gpurun_out/${TAG}_box.txt ;;
   esac
 done
