@@ -258,104 +258,53 @@ static __device__ __forceinline__ unsigned xpld_group_bytes(unsigned mask, unsig
 }
 
 /* The lanes of `ones` each access words [g0, g0+nb1] inside ONE shadow u32
- * (every aligned access of <= 4 words: ints, floats, doubles, ...).  Three
- * cases, decided warp-uniformly:
- *  (1) contiguous warp: all 32 lanes, lane l at words G + l*w (w = nb1+1, the
- *      a[i] of a coalesced kernel) -- the warp covers <= 32 consecutive shadow
- *      u32s; lane j commits u32 j with the byte lanes the warp covers in it
- *      (one coalesced shadow load, no grouping work at all);
- *  (2) one address: every lane on the same u32 (the domain words every thread
- *      of a kernel reads) -- one REDUX for the byte lanes, one lane commits;
- *  (3) anything else (gathers, partial warps): groups = maximal runs of
- *      consecutive lanes on the same u32, their byte lanes from four ballots,
- *      the group's first lane commits.  Lanes of one u32 in different runs
- *      commit separately, which is equally exact (atomicOr commutes, every
- *      commit is tested against the same epoch-start record).
+ * (every aligned access of <= 4 words: ints, floats, doubles, ...):
+ *  1. each lane loads its shadow u32 and tests whether a bit of its access is
+ *     still missing (test before set; a write-only call site K == W always
+ *     commits: wG | P do not depend on the record, so it loads nothing); a warp
+ *     with nothing missing (a re-touch) is done after one load and one ballot;
+ *  2. lanes on the same u32 are grouped (__match_any_sync); a lane alone in its
+ *     group (strided or scattered accesses) commits its own bits at once;
+ *  3. a larger group's byte lanes come from four ballots (one per byte lane of
+ *     the u32, uniform over the remaining lanes, so no serialisation over the
+ *     groups) and its first lane commits.
  * K: the access kind if uniform (compile-time call site), else 0 (per lane). */
 template <unsigned K, bool TM>
 static __device__ __forceinline__ void xpld_one(unsigned ones, unsigned long long g0, unsigned nb1,
                                                 unsigned acc) {
-  constexpr unsigned FULL = 0xFFFFFFFFu;
   const unsigned lane = xpld_lane();
   const unsigned q = (unsigned)(g0 >> 2);
-  const unsigned bm = (FULL >> (24 - 8 * nb1)) << (8 * ((unsigned)g0 & 3u));
-  if (ones == FULL) { /* (1) */
-    const unsigned w = nb1 + 1;
-    const unsigned long long G = g0 - (unsigned long long)lane * w;
-    const unsigned glo = (unsigned)G, ghi = (unsigned)(G >> 32);
-    /* (all three shuffles unconditionally: a short-circuit && would leave lanes
-     * out of a full-warp shuffle) */
-    const unsigned s_lo = __shfl_sync(FULL, glo, 0), s_hi = __shfl_sync(FULL, ghi, 0),
-                   s_nb = __shfl_sync(FULL, nb1, 0);
-    const bool same = (s_lo == glo) & (s_hi == ghi) & (s_nb == nb1);
-    const unsigned long long E = G + 32ull * w - 1; /* last word the warp covers */
-    const unsigned Q0 = (unsigned)(G >> 2), nq = (unsigned)(E >> 2) - Q0 + 1;
-    if (__all_sync(FULL, same && nq <= 32 && (K != 0 || w == 1))) {
-      unsigned rb = 0, wb = 0;
-      const unsigned lo = lane == 0 ? glo & 3u : 0u, hi = lane == nq - 1 ? (unsigned)E & 3u : 3u;
-      const unsigned m = lane < nq ? (FULL >> (24 - 8 * (hi - lo))) << (8 * lo) : 0u;
-      if (K != 0) {
-        rb = (K & XPL_ACC_R) ? m : 0u;
-        wb = (K & XPL_ACC_W) ? m : 0u;
-      } else { /* per-lane kinds, one word per lane: byte k of u32 j is lane 4j + k - (G & 3) */
-        const unsigned br = __ballot_sync(FULL, acc & XPL_ACC_R), bw = __ballot_sync(FULL, acc & XPL_ACC_W);
-        const int l0 = 4 * (int)lane - (int)(glo & 3u);
-#pragma unroll
-        for (int k = 0; k < 4; ++k) {
-          const unsigned sel = 0xFFu << (8 * k);
-          const int l = l0 + k;
-          if ((m & sel) && l >= 0 && l < 32) {
-            if ((br >> l) & 1u) rb |= sel;
-            if ((bw >> l) & 1u) wb |= sel;
-          }
-        }
-      }
-      if (lane < nq) {
-        const unsigned qq = Q0 + lane;
-        xpld_put<K, TM>(qq, K == XPL_ACC_W ? 0u : xpl_dctx.pool[qq], rb, wb);
-      }
-      return;
-    }
-  }
-  const unsigned lead = (unsigned)__ffs(ones) - 1;
-  if (__all_sync(ones, q == __shfl_sync(ones, q, lead))) { /* (2) */
-    unsigned rb, wb;
-    if (K != 0) {
-      const unsigned u = __reduce_or_sync(ones, bm);
-      rb = (K & XPL_ACC_R) ? u : 0u;
-      wb = (K & XPL_ACC_W) ? u : 0u;
-    } else {
-      rb = __reduce_or_sync(ones, (acc & XPL_ACC_R) ? bm : 0u);
-      wb = __reduce_or_sync(ones, (acc & XPL_ACC_W) ? bm : 0u);
-    }
-    if (lane == lead) xpld_put<K, TM>(q, K == XPL_ACC_W ? 0u : xpl_dctx.pool[q], rb, wb);
-    return;
-  }
-  /* (3) */
+  const unsigned bm = (0xFFFFFFFFu >> (24 - 8 * nb1)) << (8 * ((unsigned)g0 & 3u));
+  const unsigned kind = K ? K : acc;
   const unsigned cur = K == XPL_ACC_W ? 0u : xpl_dctx.pool[q];
-  if (K != XPL_ACC_W) { /* nothing missing anywhere (a re-touch): done */
-    const unsigned mine = xpld_bits(cur, bm, K ? K : acc);
-    if (!__ballot_sync(ones, (cur & mine) != mine)) return;
-  }
-  const unsigned qp = __shfl_up_sync(ones, q, 1);
-  const bool start = lane == 0 || !((ones >> (lane - 1)) & 1u) || qp != q;
-  const unsigned S = __ballot_sync(ones, start);
-  if (S == ones) { /* every lane its own group (strided or scattered): no grouping work */
-    xpld_put<K, TM>(q, cur, ((K ? K : acc) & XPL_ACC_R) ? bm : 0u, ((K ? K : acc) & XPL_ACC_W) ? bm : 0u);
+  const unsigned rb = (kind & XPL_ACC_R) ? bm : 0u, wb = (kind & XPL_ACC_W) ? bm : 0u;
+  const unsigned mine = xpld_bits2(cur, rb, wb);
+  const bool need = K == XPL_ACC_W || (cur & mine) != mine;
+  const unsigned needers = __ballot_sync(ones, need);
+  if (!need) return;
+  const unsigned grp = __match_any_sync(needers, q);
+  const unsigned me = 1u << lane;
+  const unsigned alone = __ballot_sync(needers, grp == me);
+  if (grp == me) {
+    xpld_put<K, TM>(q, cur, rb, wb);
     return;
   }
-  const unsigned above = S & (0xFFFFFFFEu << lane); /* group starts after this lane */
-  const unsigned gm = (above ? ((1u << (__ffs(above) - 1)) - 1u) : FULL) & (FULL << lane);
-  unsigned rb, wb;
-  if (K != 0) {
-    const unsigned u = xpld_group_bytes(ones, bm, gm);
-    rb = (K & XPL_ACC_R) ? u : 0u;
-    wb = (K & XPL_ACC_W) ? u : 0u;
-  } else {
-    rb = xpld_group_bytes(ones, (acc & XPL_ACC_R) ? bm : 0u, gm);
-    wb = xpld_group_bytes(ones, (acc & XPL_ACC_W) ? bm : 0u, gm);
+  const unsigned rest = needers & ~alone;
+  unsigned gr = 0, gw = 0;
+#pragma unroll
+  for (unsigned k = 0; k < 4; ++k) {
+    const unsigned sel = 0xFFu << (8 * k);
+    if (K != 0) {
+      if (__ballot_sync(rest, (bm & sel) != 0) & grp) {
+        if (K & XPL_ACC_R) gr |= sel;
+        if (K & XPL_ACC_W) gw |= sel;
+      }
+    } else {
+      if (__ballot_sync(rest, (rb & sel) != 0) & grp) gr |= sel;
+      if (__ballot_sync(rest, (wb & sel) != 0) & grp) gw |= sel;
+    }
   }
-  if (start) xpld_put<K, TM>(q, cur, rb, wb);
+  if (lane == (unsigned)(__ffs(grp) - 1)) xpld_put<K, TM>(q, cur, gr, gw);
 }
 
 /* Apply a GPU access to the shadow words [g0, g1] (global pool word indices;

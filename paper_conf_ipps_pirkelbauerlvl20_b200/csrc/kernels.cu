@@ -24,22 +24,41 @@ constexpr uint32_t kP4 = 0x02020202u;
 
 // ---------------------------------------------------------------------------
 // fold (epoch close): every 128-word chunk a GPU write marked (cmap) gets
-// P -> L=1 and P cleared (snapshot semantics D5).  A one-wave grid:
-// CTA b owns the super-chunks b, b+G, b+2G, ... (16K words each, below the
-// pool's high-water mark).  It first reads all its super bytes at once (one
-// byte per thread per round) and lists the marked ones in shared memory, so
-// an epoch that wrote little costs one launch and one read of the super map;
-// then, per listed super-chunk, warp w checks chunks [16w, 16w+16) and folds
-// all its marked ones with one round trip (128 B coalesced each).  Consecutive
-// super-chunks go to different CTAs, so a dense epoch spreads over the grid.
-// No global list, no atomics; cost O(super map + chunks written).  Launched
-// with programmatic stream serialization when it directly follows the epoch's
-// kernels on their stream: griddepcontrol.wait holds it until they are
-// complete, while its own launch overlaps their tail.
+// P -> L=1 and P cleared (snapshot semantics D5).  A one-wave grid of
+// W warps; warp w owns the super-chunks (16K words) w, w + W, w + 2W, ... below
+// the pool's high-water mark: it reads 32 of its super bytes at once (one per
+// lane), and for each marked one folds its marked chunks lane-per-chunk (lane
+// l checks chunks l, l+32, l+64, l+96; a marked chunk = one 128 B line, eight
+// 16 B loads in flight together).  Spreading the super-chunks over all warps
+// keeps the chain per warp short whatever the epoch's write pattern: an epoch
+// that touched one word in every super-chunk (a Smith-Waterman anti-diagonal)
+// costs every warp ~2 supers, not one CTA a long list.  No global list, no
+// atomics; cost O(super map + chunks written).  Launched with programmatic
+// stream serialization when it directly follows the epoch's kernels on their
+// stream: griddepcontrol.wait holds it until they are complete, while its own
+// launch overlaps their tail.
 constexpr int kFoldThreads = 256;
 #ifndef XPL_FOLD_CTAS
 #define XPL_FOLD_CTAS (148 * 8)  // grid cap (A/B: profiles/r1_fold_grid_ab.txt)
 #endif
+
+__device__ __forceinline__ uint32_t fold_chunk(uint32_t* pool, uint64_t ch) {
+  uint4* w = reinterpret_cast<uint4*>(pool + ch * 32);
+  uint4 v[8];
+#pragma unroll
+  for (int k = 0; k < 8; ++k) v[k] = w[k];
+#pragma unroll
+  for (int k = 0; k < 8; ++k) {
+    if ((v[k].x | v[k].y | v[k].z | v[k].w) & kP4) {
+      v[k].x = (v[k].x & ~kP4) | ((v[k].x & kP4) >> 1);
+      v[k].y = (v[k].y & ~kP4) | ((v[k].y & kP4) >> 1);
+      v[k].z = (v[k].z & ~kP4) | ((v[k].z & kP4) >> 1);
+      v[k].w = (v[k].w & ~kP4) | ((v[k].w & kP4) >> 1);
+      w[k] = v[k];
+    }
+  }
+  return 1;
+}
 
 __global__ void __launch_bounds__(kFoldThreads) fold_kernel(uint32_t* __restrict__ pool,
                                                             uint8_t* __restrict__ cmap,
@@ -52,42 +71,27 @@ __global__ void __launch_bounds__(kFoldThreads) fold_kernel(uint32_t* __restrict
     if (strict && flags[0]) flags[1] = 1u;
     flags[0] = 0u;
   }
-  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  __shared__ uint64_t s_list[kFoldThreads];
-  __shared__ uint32_t s_n;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t W = (uint64_t)gridDim.x * (kFoldThreads / 32);
+  const uint64_t w = (uint64_t)blockIdx.x * (kFoldThreads / 32) + (threadIdx.x >> 5);
   uint32_t folded = 0;
-  const uint64_t G = gridDim.x;
-  const uint64_t mine = n_super > blockIdx.x ? (n_super - blockIdx.x + G - 1) / G : 0;
-  for (uint64_t r0 = 0; r0 < mine; r0 += kFoldThreads) {
-    if (threadIdx.x == 0) s_n = 0;
-    __syncthreads();
-    const uint64_t it = r0 + threadIdx.x;
-    if (it < mine) {
-      const uint64_t sc = blockIdx.x + it * G;
-      if (smap[sc]) s_list[atomicAdd(&s_n, 1u)] = sc;
+  for (uint64_t k0 = 0; w + k0 * W < n_super; k0 += 32) {
+    const uint64_t sc = w + (k0 + lane) * W;
+    uint32_t ms = __ballot_sync(0xFFFFFFFFu, sc < n_super && smap[sc] != 0);
+    while (ms) {
+      const uint32_t j = __ffs(ms) - 1;
+      ms &= ms - 1;
+      const uint64_t s = w + (k0 + j) * W;
+      const uint64_t c0 = s * 128 + lane;
+      const uint8_t m0 = cmap[c0], m1 = cmap[c0 + 32], m2 = cmap[c0 + 64], m3 = cmap[c0 + 96];
+      if (m0) { folded += fold_chunk(pool, c0); cmap[c0] = 0; }
+      if (m1) { folded += fold_chunk(pool, c0 + 32); cmap[c0 + 32] = 0; }
+      if (m2) { folded += fold_chunk(pool, c0 + 64); cmap[c0 + 64] = 0; }
+      if (m3) { folded += fold_chunk(pool, c0 + 96); cmap[c0 + 96] = 0; }
+      if (lane == 0) smap[s] = 0;
     }
-    __syncthreads();
-    const uint32_t n = s_n;
-    for (uint32_t k = 0; k < n; ++k) {
-      const uint64_t sc = s_list[k];
-      const uint64_t c0 = sc * 128 + warp * 16;
-      const bool m = lane < 16 && cmap[c0 + lane] != 0;
-      uint32_t marked = __ballot_sync(0xFFFFFFFFu, m);
-      folded += __popc(marked);
-      // All of the warp's marked chunks in one round trip: 16 predicated
-      // loads (warp-uniform predicates) issued back to back, then the stores.
-      uint32_t v[16];
-      uint32_t* const base = pool + c0 * 32 + lane;
-#pragma unroll
-      for (uint32_t j = 0; j < 16; ++j) v[j] = (marked >> j) & 1u ? base[j * 32] : 0u;
-#pragma unroll
-      for (uint32_t j = 0; j < 16; ++j)
-        if (v[j] & kP4) base[j * 32] = (v[j] & ~kP4) | ((v[j] & kP4) >> 1);
-      if (m) cmap[c0 + lane] = 0;
-      if (threadIdx.x == 0) smap[sc] = 0;
-    }
-    __syncthreads();  // s_list / s_n are rewritten by the next round
   }
+  folded = __reduce_add_sync(0xFFFFFFFFu, folded);
   if (lane == 0 && folded) atomicAdd(stats + 3, (unsigned long long)folded);
 }
 
@@ -1102,7 +1106,8 @@ __global__ void __launch_bounds__(256) page_kernel(const PageRow* __restrict__ r
 void launch_fold(cudaStream_t s, bool pdl, uint32_t* pool, uint8_t* cmap, uint8_t* smap,
                  uint64_t n_super, unsigned long long* stats, uint32_t* flags, int strict) {
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3((unsigned)(n_super == 0 ? 1 : n_super < XPL_FOLD_CTAS ? n_super : XPL_FOLD_CTAS));  // one wave
+  const uint64_t ctas = (n_super + 7) / 8;  // (one warp per super-chunk at most)
+  cfg.gridDim = dim3((unsigned)(ctas == 0 ? 1 : ctas < XPL_FOLD_CTAS ? ctas : XPL_FOLD_CTAS));  // one wave
   cfg.blockDim = dim3(kFoldThreads);
   cfg.stream = s;
   cudaLaunchAttribute at[1];

@@ -137,7 +137,7 @@ template <bool I>
 __global__ void k_integrate_stress(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (e < P_.e1 && e < NE()) {
+  if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const auto nl = ARR(const int, NODELIST);
     const auto x = ARR(const double, X), y = ARR(const double, Y), z = ARR(const double, Z);
     const double sig = -(R_(PTR(const double, P)[e]) + R_(PTR(const double, Q)[e]));
@@ -158,7 +158,7 @@ template <bool I>
 __global__ void k_hourglass(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (e < P_.e1 && e < NE()) {
+  if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const auto nl = ARR(const int, NODELIST);
     const auto xd = ARR(const double, XD), yd = ARR(const double, YD), zd = ARR(const double, ZD);
     const double coef = R_(PTR(const double, SS)[e]) * R_(PTR(const double, ELEMMASS)[e]) /
@@ -264,7 +264,7 @@ template <bool I>
 __global__ void k_kinematics(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (e < P_.e1 && e < NE()) {
+  if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const auto nl = ARR(const int, NODELIST);
     const auto x = ARR(const double, X), y = ARR(const double, Y), z = ARR(const double, Z);
     const auto xd = ARR(const double, XD), yd = ARR(const double, YD), zd = ARR(const double, ZD);
@@ -292,7 +292,7 @@ template <bool I>
 __global__ void k_lagrange(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (e < P_.e1 && e < NE()) {
+  if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const auto g = ARR(const double, TMP_DVDX);
     const double r = (RA_(g, 3 * e) + RA_(g, 3 * e + 1) + RA_(g, 3 * e + 2)) / (R_(PTR(const double, VNEW)[e]) + 1.0);
     W_(PTR(double, VDOV)[e]) = r;
@@ -305,7 +305,7 @@ template <bool I>
 __global__ void k_monoq_grad(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (e < P_.e1 && e < NE()) {
+  if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const double* vdov = PTR(const double, VDOV);
     const int m = R_(PTR(const int, LXIM)[e]), p = R_(PTR(const int, LXIP)[e]);
     const double r = R_(vdov[p]) - R_(vdov[m]) + R_(PTR(const double, VNEW)[e]);
@@ -317,7 +317,7 @@ template <bool I>
 __global__ void k_monoq_region(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (e < P_.e1 && e < NE()) {
+  if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const int bc = R_(PTR(const int, ELEMBC)[e]);
     const double r = (bc & 1 ? 0.5 : 1.0) * R_(PTR(const double, QL)[e]) * R_(PTR(const double, VDOV)[e]);
     W_(PTR(double, QQ)[e]) = r;
@@ -330,7 +330,7 @@ template <bool I>
 __global__ void k_eos(Part P_, Dom* d, int stage, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (e < P_.e1 && e < NE()) {
+  if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const double t = R_(d->time);
     if (stage == 0) {  // energy
       const double w = R_(d->misc[0]) * 1e-6 + R_(d->misc[1]) * 1e-6 + R_(d->misc[2]);
@@ -362,7 +362,7 @@ template <bool I>
 __global__ void k_update_volumes(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
-  if (e < P_.e1 && e < NE()) {
+  if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const double v = R_(PTR(const double, VNEW)[e]);
     W_(PTR(double, V)[e]) = v;
   }
@@ -376,7 +376,7 @@ __global__ void __launch_bounds__(256) k_dt(Part P_, Dom* d, double* dtb, int nb
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   double v = 1e30;
-  if (e < P_.e1 && e < NE()) {
+  if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     if (COURANT) {
       const double ss = R_(PTR(const double, SS)[e]), vd = R_(PTR(const double, VDOV)[e]),
                    ar = R_(PTR(const double, AREALG)[e]);
