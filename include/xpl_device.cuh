@@ -411,6 +411,44 @@ static __device__ __forceinline__ void xpld_record_words(unsigned long long g0, 
   if (__any_sync(__activemask(), remote) && remote) xpld_remote<K>(owner, g0, g1, acc);
 }
 
+/* The compile-time-kind hook (every xpl_read / xpl_write / xpl_rw call site):
+ * when every active lane's access is local and inside one shadow u32 (or
+ * misses) -- the common case -- one straight-line, warp-convergent sequence:
+ * a predicated shadow load, the test before set, one ballot (a re-touching
+ * warp is done here), then match_any groups, four byte-lane ballots and one
+ * atomicOr per group.  Every warp-synchronous op runs at the same level for
+ * all active lanes (no divergent collectives).  Anything else (multi-u32
+ * accesses, remote pieces) takes the general path, decided warp-uniformly. */
+template <unsigned K, bool TM = true>
+static __device__ __forceinline__ void xpld_record_fast(unsigned long long g0, unsigned long long g1,
+                                                        unsigned owner) {
+  const unsigned act = __activemask();
+  const bool hit = g0 <= g1;
+  const bool fast = !hit || (owner == xpl_dctx.rank && (g0 ^ g1) < 4ull);
+  if (__ballot_sync(act, !fast)) { /* uniform: some lane needs the general path */
+    xpld_record_words<K, TM>(g0, g1, owner, K);
+    return;
+  }
+  const unsigned lane = xpld_lane();
+  const unsigned q = (unsigned)(g0 >> 2);
+  const unsigned bm = hit ? (0xFFFFFFFFu >> (24 - 8 * (unsigned)(g1 - g0))) << (8 * ((unsigned)g0 & 3u)) : 0u;
+  const unsigned cur = (K == XPL_ACC_W || !hit) ? 0u : xpl_dctx.pool[q];
+  const unsigned rb = (K & XPL_ACC_R) ? bm : 0u, wb = (K & XPL_ACC_W) ? bm : 0u;
+  const unsigned mine = xpld_bits2(cur, rb, wb);
+  const bool need = hit && (K == XPL_ACC_W || (cur & mine) != mine);
+  const unsigned needers = __ballot_sync(act, need);
+  if (!needers) return; /* uniform: nothing missing (a re-touch) */
+  const unsigned grp = __match_any_sync(act, need ? q : 0xFFFFFFFFu) & needers;
+  unsigned gb = 0;
+#pragma unroll
+  for (unsigned k = 0; k < 4; ++k) {
+    const unsigned sel = 0xFFu << (8 * k);
+    if (__ballot_sync(act, need && (bm & sel)) & grp) gb |= sel;
+  }
+  if (need && lane == (unsigned)(__ffs(grp) - 1))
+    xpld_put<K, TM>(q, cur, (K & XPL_ACC_R) ? gb : 0u, (K & XPL_ACC_W) ? gb : 0u);
+}
+
 template <unsigned K, bool TM = true>
 static __device__ __forceinline__ void xpl_dev_record_k(const void* p, unsigned size,
                                                         unsigned acc) {
@@ -420,7 +458,8 @@ static __device__ __forceinline__ void xpl_dev_record_k(const void* p, unsigned 
   unsigned long long g0 = 1, g1 = 0;
   unsigned owner = xpl_dctx.rank;
   if (xpld_find(a, be, ow) && size > 0) xpld_words(a, size, be, ow, g0, g1, owner);
-  xpld_record_words<K, TM>(g0, g1, owner, K ? K : acc);
+  if (K != 0) xpld_record_fast<K, TM>(g0, g1, owner);
+  else xpld_record_words<K, TM>(g0, g1, owner, acc);
 #else
   (void)p; (void)size; (void)acc;
 #endif
@@ -453,7 +492,7 @@ struct xpl_array {
       ulonglong2 b2, o2;
       if (xpld_find(a, b2, o2)) xpld_words(a, sizeof(T), b2, o2, g0, g1, owner);
     }
-    xpld_record_words<K>(g0, g1, owner, K);
+    xpld_record_fast<K>(g0, g1, owner);
 #else
     (void)i;
 #endif
