@@ -101,20 +101,21 @@ __global__ void __launch_bounds__(kFoldThreads) fold_kernel(uint32_t* __restrict
 // a read after it sees the CPU; any write sets wC and makes the CPU the last
 // writer.  Pass 1 finds each word's first writing record
 // (atomicMin of the record index), pass 2 sets read/write bits, pass 3 clears L
-// of written words and resets the scratch.
+// of written words and resets the scratch.  The scratch covers only the pool
+// words [fw0, fw0 + span) the batch touches (fw[w - fw0]).
 
 __global__ void merge_firstw_kernel(const uint64_t* __restrict__ recs, uint32_t n,
-                                    uint32_t* __restrict__ fw) {
+                                    uint32_t* __restrict__ fw, uint64_t fw0) {
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     const uint64_t r = recs[i];
     if (!(rec_acc(r) & XPL_ACC_W)) continue;
     const uint64_t g0 = rec_g0(r), nw = rec_nw(r);
-    for (uint64_t w = g0; w < g0 + nw; ++w) atomicMin(fw + w, i);
+    for (uint64_t w = g0; w < g0 + nw; ++w) atomicMin(fw + (w - fw0), i);
   }
 }
 
 __global__ void merge_apply_kernel(const uint64_t* __restrict__ recs, uint32_t n,
-                                   const uint32_t* __restrict__ fw, uint32_t* pool) {
+                                   const uint32_t* __restrict__ fw, uint64_t fw0, uint32_t* pool) {
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     const uint64_t r = recs[i];
     const uint32_t acc = rec_acc(r);
@@ -128,7 +129,7 @@ __global__ void merge_apply_kernel(const uint64_t* __restrict__ recs, uint32_t n
         if (w < g0 || w > g1) continue;
         uint32_t b = 0;
         if (acc & XPL_ACC_R) {
-          const bool before = (fw == nullptr) || i <= fw[w];
+          const bool before = (fw == nullptr) || i <= fw[w - fw0];
           b = before ? (((cur >> (8 * k)) & 1u) ? kRGC : kRCC) : kRCC;
         }
         if (acc & XPL_ACC_W) b |= kWC;
@@ -140,7 +141,7 @@ __global__ void merge_apply_kernel(const uint64_t* __restrict__ recs, uint32_t n
 }
 
 __global__ void merge_clear_kernel(const uint64_t* __restrict__ recs, uint32_t n,
-                                   uint32_t* __restrict__ fw, uint32_t* pool) {
+                                   uint32_t* __restrict__ fw, uint64_t fw0, uint32_t* pool) {
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     const uint64_t r = recs[i];
     if (!(rec_acc(r) & XPL_ACC_W)) continue;
@@ -155,7 +156,7 @@ __global__ void merge_clear_kernel(const uint64_t* __restrict__ recs, uint32_t n
       if (pool[q] & lm) atomicAnd(pool + q, ~lm);
     }
     if (fw)
-      for (uint64_t w = g0; w <= g1; ++w) fw[w] = 0xFFFFFFFFu;
+      for (uint64_t w = g0; w <= g1; ++w) fw[w - fw0] = 0xFFFFFFFFu;
   }
 }
 
@@ -1119,12 +1120,12 @@ void launch_fold(cudaStream_t s, bool pdl, uint32_t* pool, uint8_t* cmap, uint8_
 }
 
 void launch_merge(cudaStream_t s, const uint64_t* recs, uint32_t n, bool has_r, bool has_w,
-                  uint32_t* first_w, uint32_t* pool) {
+                  uint32_t* first_w, uint64_t fw0, uint32_t* pool) {
   const int g = grid_for(n, 256, 148 * 16);
   const bool both = has_r && has_w;
-  if (both) merge_firstw_kernel<<<g, 256, 0, s>>>(recs, n, first_w);
-  merge_apply_kernel<<<g, 256, 0, s>>>(recs, n, both ? first_w : nullptr, pool);
-  if (has_w) merge_clear_kernel<<<g, 256, 0, s>>>(recs, n, both ? first_w : nullptr, pool);
+  if (both) merge_firstw_kernel<<<g, 256, 0, s>>>(recs, n, first_w, fw0);
+  merge_apply_kernel<<<g, 256, 0, s>>>(recs, n, both ? first_w : nullptr, fw0, pool);
+  if (has_w) merge_clear_kernel<<<g, 256, 0, s>>>(recs, n, both ? first_w : nullptr, fw0, pool);
 }
 
 void launch_range(cudaStream_t s, const RangeDesc* d_ranges, uint32_t nr, uint64_t nvec,

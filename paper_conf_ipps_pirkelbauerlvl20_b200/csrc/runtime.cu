@@ -105,7 +105,8 @@ struct xpl_ctx {
   void* peer_pool[XPL_MAX_RANKS] = {};       // IPC-mapped pools / chunk maps of the other ranks
   void* peer_cmap[XPL_MAX_RANKS] = {};
   void* peer_smap[XPL_MAX_RANKS] = {};
-  uint32_t* d_first_w = nullptr;  // merge scratch, lazily allocated
+  uint32_t* d_first_w = nullptr;  // merge scratch (first writer per word of a batch's span), grown lazily
+  uint64_t first_w_cap = 0;
 
   // shadow memory table
   std::vector<Row> rows;               // by id
@@ -359,10 +360,26 @@ xpl_status ensure_ranges(xpl_ctx* c, size_t n) {
   return XPL_OK;
 }
 
-xpl_status ensure_first_w(xpl_ctx* c) {
-  if (c->d_first_w) return XPL_OK;
-  CK(cudaMalloc(&c->d_first_w, sizeof(uint32_t) * c->pool_words));
-  launch_fill_u32(c->cs, c->d_first_w, c->pool_words, 0xFFFFFFFFu);
+// The merge scratch for a batch of records h[0, n) mixing reads and writes: one
+// u32 per pool word of the batch's span [*lo, hi) (not per pool word: 4 B x the
+// span, e.g. a host segment over two small allocations); all-ones between uses.
+xpl_status ensure_first_w(xpl_ctx* c, const uint64_t* h, size_t n, uint64_t* lo) {
+  uint64_t a = ~0ull, b = 0;
+  for (size_t i = 0; i < n; ++i) {
+    a = std::min(a, rec_g0(h[i]));
+    b = std::max(b, rec_g0(h[i]) + rec_nw(h[i]));
+  }
+  *lo = a;
+  const uint64_t span = b > a ? b - a : 1;
+  if (span <= c->first_w_cap) return XPL_OK;
+  if (c->d_first_w) {
+    CK(cudaStreamSynchronize(c->cs));
+    cudaFree(c->d_first_w);
+  }
+  const uint64_t cap = std::max<uint64_t>(span + span / 2, 1 << 16);
+  CK(cudaMalloc(&c->d_first_w, sizeof(uint32_t) * cap));
+  launch_fill_u32(c->cs, c->d_first_w, cap, 0xFFFFFFFFu);
+  c->first_w_cap = cap;
   c->st.kernel_launches += 1;
   return XPL_OK;
 }
@@ -431,10 +448,11 @@ xpl_status flush_local(xpl_ctx* c) {
     CK(cudaMemcpyAsync(c->d_stage, h, n * sizeof(uint64_t), cudaMemcpyHostToDevice, c->cs));
     CK(cudaEventRecord(c->stage_ev[c->cur], c->cs));
     xpl_status s = XPL_OK;
-    if (c->stage_has_r && c->stage_has_w) s = ensure_first_w(c);
+    uint64_t fw0 = 0;
+    if (c->stage_has_r && c->stage_has_w) s = ensure_first_w(c, h, n, &fw0);
     if (s) return s;
     const int pi = prof_begin(c, XPL_K_MERGE, c->prof ? 8 * n + 2 * words_of(h, n) : 0);
-    launch_merge(c->cs, c->d_stage, (uint32_t)n, c->stage_has_r, c->stage_has_w, c->d_first_w,
+    launch_merge(c->cs, c->d_stage, (uint32_t)n, c->stage_has_r, c->stage_has_w, c->d_first_w, fw0,
                  (uint32_t*)c->d_pool);
     prof_end(c, pi);
     c->st.kernel_launches += 1 + c->stage_has_w + (c->stage_has_r && c->stage_has_w);
@@ -521,13 +539,14 @@ xpl_status flush_local(xpl_ctx* c) {
         c->st.kernel_launches += 1;
         c->st.range_segments++;
       } else {
+        uint64_t fw0 = 0;
         if (sg.has_r && sg.has_w) {
-          s = ensure_first_w(c);
+          s = ensure_first_w(c, c->h_pieces + sg.start, sg.n, &fw0);
           if (s) return s;
         }
         const int pi = prof_begin(c, XPL_K_MERGE, c->prof ? 8 * sg.n + 2 * words_of(c->h_pieces + sg.start, sg.n) : 0);
         launch_merge(c->cs, c->d_pieces + sg.start, (uint32_t)sg.n, sg.has_r, sg.has_w,
-                     c->d_first_w, (uint32_t*)c->d_pool);
+                     c->d_first_w, fw0, (uint32_t*)c->d_pool);
         prof_end(c, pi);
         c->st.kernel_launches += 1 + sg.has_w + (sg.has_r && sg.has_w);
         c->st.merge_segments++;
