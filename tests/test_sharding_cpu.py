@@ -140,3 +140,48 @@ def test_two_rank_combine_matches_unsharded_oracle(seed, params):
     for p in procs:
         p.join(timeout=60)
     assert res == {0: "ok", 1: "ok"}, res
+
+
+def _comm_rank(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from paper_conf_ipps_pirkelbauerlvl20_b200 import xpl
+        comm = xpl.TorchComm()
+        c = comm.c
+        # all-gather: every rank's 13 bytes, in rank order
+        src = (C.c_uint8 * 13)(*[(rank * 31 + i) % 256 for i in range(13)])
+        dst = (C.c_uint8 * (13 * world))()
+        assert c.allgather(c.user, src, 13, dst) == 0
+        assert bytes(dst) == b"".join(bytes((r * 31 + i) % 256 for i in range(13)) for r in range(world))
+        # all-to-all with uneven sizes: rank r sends (r + q + 1) bytes of value 16 r + q to rank q
+        sb = (C.c_uint64 * world)(*[rank + q + 1 for q in range(world)])
+        rb = (C.c_uint64 * world)(*[q + rank + 1 for q in range(world)])
+        send = b"".join(bytes([16 * rank + q]) * (rank + q + 1) for q in range(world))
+        recv = (C.c_uint8 * sum(rb))()
+        assert c.alltoallv(c.user, send, sb, recv, rb) == 0
+        assert bytes(recv) == b"".join(bytes([16 * q + rank]) * (q + rank + 1) for q in range(world))
+        assert c.barrier(c.user) == 0
+        q.put((rank, "ok"))
+    except Exception as ex:  # noqa: BLE001
+        q.put((rank, repr(ex)))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_torch_comm_collectives_gloo(world):
+    """The collectives a sharded context calls (xpl.TorchComm, the xpl_comm the
+    runtime gets): all-gather and the uneven all-to-all that routes host records
+    to their owners, through the same ctypes function pointers libxpl.so calls."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = 29700 + world * 11 + os.getpid() % 1000
+    procs = [ctx.Process(target=_comm_rank, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=240) for _ in procs)
+    for p in procs:
+        p.join(timeout=60)
+    assert res == {r: "ok" for r in range(world)}, res
