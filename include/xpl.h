@@ -400,7 +400,9 @@ typedef struct {
   uint32_t shmem, name_idx; /* name_idx: xpl_launch_name(), UINT32_MAX = none        */
   uint64_t threads;         /* grid x block                                          */
   uint64_t launches_in_epoch;
-  uint64_t epoch_written_chunks; /* 128-word chunks the epoch's fold saw written     */
+  uint64_t epoch_written_chunks; /* 128-word chunks the epoch's fold folded: chunks
+                                  * holding a word the epoch wrote while its last
+                                  * writer was the CPU (D34)                         */
   double epoch_ms;               /* GPU time of the epoch incl. its fold, -1 if n/a  */
 } xpl_launch_record;
 

@@ -13,7 +13,8 @@
  * access after another): xpl_read_lat(x) defers the commit to the end of the
  * full expression so its shadow load overlaps the user's load (C++17: the proxy
  * is returned by guaranteed copy elision); xpl_write_lat(x) stores the chunk
- * mark without testing it first, so it never waits.
+ * mark without testing it first.  Array handles (xpl_array<T>) hoist the
+ * lookup of a base pointer out of repeated accesses.
  *
  * What a hook does (design: DESIGN.md §5):
  *  1. lookup: binary search of the address in the live-allocation table
@@ -22,15 +23,17 @@
  *       read  -> rCG (value written by the CPU) or rGG (by the GPU), chosen by the
  *                record's last-writer bit L, which is frozen for the whole epoch
  *                (snapshot semantics, D5);
- *       write -> wG and P ("GPU write pending"; the epoch close turns P into L=1);
+ *       write -> wG, and P ("GPU write pending"; the epoch close turns P into
+ *                L=1) where L is still the CPU (where it is the GPU already,
+ *                the epoch ends with L=1 anyway: no P, no fold work);
  *  3. warp aggregation: lanes that hit the same shadow u32 (4 records) are grouped
  *     with __match_any_sync, their bits combined (per-byte-lane ballots), and one
  *     leader issues a single atomicOr -- and only if some bit is still missing
- *     (test before set; write-only call sites skip the test: their bits do not
- *     depend on the record, so they need no shadow load at all);
- *  4. a write also marks its 128-word chunk (and 16K-word super-chunk) in two
- *     byte maps with plain idempotent stores (test before store, no atomics),
- *     so closing the epoch costs O(chunks written), not O(shadow).
+ *     (test before set);
+ *  4. a write that sets P also marks its 128-word chunk (and 16K-word
+ *     super-chunk) in two byte maps with plain idempotent stores (test before
+ *     store, no atomics), so closing the epoch costs O(chunks with P), not
+ *     O(shadow).
  * A single-word access (the common case: an aligned scalar) takes a short path
  * with one ballot; multi-word accesses loop over the shadow u32s they cover.
  * Device hooks never fail and never block.
@@ -116,11 +119,15 @@ static __device__ __forceinline__ void xpld_mark(unsigned q) {
 }
 
 /* The record bits a read of the byte lanes rb and a write of the byte lanes wb
- * (0xFF per record) set on the 4 records of shadow u32 cur. */
+ * (0xFF per record) set on the 4 records of shadow u32 cur.  A write sets wG,
+ * and P ("make L = GPU at the epoch close") only where L is still the CPU: L is
+ * constant within an epoch (D5), so a word the GPU wrote last already ends the
+ * epoch with L = GPU -- no P, no chunk mark, no fold work for it. */
 static __device__ __forceinline__ unsigned xpld_bits2(unsigned cur, unsigned rb, unsigned wb) {
   const unsigned l = cur & 0x01010101u;                           /* L per record      */
-  return (((l << 7) | ((~l & 0x01010101u) << 6)) & rb)            /* rGG if L else rCG */
-         | (0x0A0A0A0Au & wb);                                    /* wG | P            */
+  const unsigned nl = ~l & 0x01010101u;                           /* L == CPU          */
+  return (((l << 7) | (nl << 6)) & rb)                            /* rGG if L else rCG */
+         | ((0x08080808u | (nl << 1)) & wb);                      /* wG, P if L == CPU */
 }
 
 /* The record bits an access of kind acc sets on the 4 records of shadow u32 cur,
@@ -183,8 +190,9 @@ static __device__ __forceinline__ void xpld_commit(unsigned needers, unsigned q,
     }
   }
   if (xpld_lane() == (unsigned)(__ffs(grp) - 1)) {
-    atomicOr(xpl_dctx.pool + q, xpld_bits2(cur, rb, wb)); /* no return value needed: RED */
-    if (wb) xpld_mark<TM>(q);
+    const unsigned bits = xpld_bits2(cur, rb, wb);
+    atomicOr(xpl_dctx.pool + q, bits); /* no return value needed: RED */
+    if (bits & XPLD_P4) xpld_mark<TM>(q);
   }
 }
 
@@ -211,9 +219,9 @@ static __device__ __noinline__ void xpld_remote(unsigned owner, unsigned long lo
         const unsigned long long gw = q * 4 + k;
         if (gw >= g0 && gw <= g1) bytes |= 0xFFu << (8 * k);
       }
-      const unsigned cur = K == XPL_ACC_W ? 0u : __ldcg(P + q);
+      const unsigned cur = __ldcg(P + q);
       const unsigned m = xpld_bits(cur, bytes, acc);
-      const bool need = K == XPL_ACC_W || (cur & m) != m;
+      const bool need = (cur & m) != m;
       const unsigned needers = __ballot_sync(__activemask(), need);
       if (need) {
         const unsigned grp = __match_any_sync(needers, ((unsigned long long)owner << 40) | q);
@@ -235,15 +243,14 @@ static __device__ __noinline__ void xpld_remote(unsigned owner, unsigned long lo
 }
 
 /* Test-before-set commit of one shadow u32 q by one lane: bits = the record
- * bits of the byte lanes rb (read) / wb (written) given the u32's current
- * value cur (cur unused and 0 for write-only call sites K == W: wG | P does not
- * depend on the record, so no load is needed and the RED is always issued). */
+ * bits of the byte lanes rb (read) / wb (written) given the u32's value cur at
+ * the hook (its L bits are the epoch's). */
 template <unsigned K, bool TM>
 static __device__ __forceinline__ void xpld_put(unsigned q, unsigned cur, unsigned rb, unsigned wb) {
   const unsigned bits = xpld_bits2(cur, rb, wb);
-  if (K == XPL_ACC_W || (cur & bits) != bits) {
+  if ((cur & bits) != bits) {
     atomicOr(xpl_dctx.pool + q, bits); /* no return value needed: RED */
-    if (wb) xpld_mark<TM>(q);
+    if (bits & XPLD_P4) xpld_mark<TM>(q);
   }
 }
 
@@ -276,10 +283,10 @@ static __device__ __forceinline__ void xpld_one(unsigned ones, unsigned long lon
   const unsigned q = (unsigned)(g0 >> 2);
   const unsigned bm = (0xFFFFFFFFu >> (24 - 8 * nb1)) << (8 * ((unsigned)g0 & 3u));
   const unsigned kind = K ? K : acc;
-  const unsigned cur = K == XPL_ACC_W ? 0u : xpl_dctx.pool[q];
+  const unsigned cur = xpl_dctx.pool[q];
   const unsigned rb = (kind & XPL_ACC_R) ? bm : 0u, wb = (kind & XPL_ACC_W) ? bm : 0u;
   const unsigned mine = xpld_bits2(cur, rb, wb);
-  const bool need = K == XPL_ACC_W || (cur & mine) != mine;
+  const bool need = (cur & mine) != mine;
   const unsigned needers = __ballot_sync(ones, need);
   if (!need) return;
   const unsigned grp = __match_any_sync(needers, q);
@@ -329,7 +336,7 @@ static __device__ __forceinline__ void xpl_dev_apply(unsigned long long g0,
   while (__any_sync(multis, more)) {
     unsigned cur = 0, m = 0, bytes = 0;
     if (more) {
-      cur = K == XPL_ACC_W ? 0u : xpl_dctx.pool[q];
+      cur = xpl_dctx.pool[q];
 #pragma unroll
       for (unsigned k = 0; k < 4; ++k) {
         const unsigned long long gw = q * 4 + k;
@@ -337,7 +344,7 @@ static __device__ __forceinline__ void xpl_dev_apply(unsigned long long g0,
       }
       m = xpld_bits(cur, bytes, acc);
     }
-    const bool need = more && (K == XPL_ACC_W || (cur & m) != m);
+    const bool need = more && (cur & m) != m;
     const unsigned needers = __ballot_sync(multis, need);
     if (need) xpld_commit<K, false, TM>(needers, (unsigned)q, cur, bytes, acc);
     more = more && q < ql;
@@ -432,10 +439,10 @@ static __device__ __forceinline__ void xpld_record_fast(unsigned long long g0, u
   const unsigned lane = xpld_lane();
   const unsigned q = (unsigned)(g0 >> 2);
   const unsigned bm = hit ? (0xFFFFFFFFu >> (24 - 8 * (unsigned)(g1 - g0))) << (8 * ((unsigned)g0 & 3u)) : 0u;
-  const unsigned cur = (K == XPL_ACC_W || !hit) ? 0u : xpl_dctx.pool[q];
+  const unsigned cur = hit ? xpl_dctx.pool[q] : 0u;
   const unsigned rb = (K & XPL_ACC_R) ? bm : 0u, wb = (K & XPL_ACC_W) ? bm : 0u;
   const unsigned mine = xpld_bits2(cur, rb, wb);
-  const bool need = hit && (K == XPL_ACC_W || (cur & mine) != mine);
+  const bool need = hit && (cur & mine) != mine;
   const unsigned needers = __ballot_sync(act, need);
   if (!needers) return; /* uniform: nothing missing (a re-touch) */
   const unsigned grp = __match_any_sync(act, need ? q : 0xFFFFFFFFu) & needers;
@@ -612,9 +619,9 @@ static __device__ __forceinline__ xpl_read_proxy<T> xpl_read_lat(const T& x) {
 
 /* traceW for latency-bound kernels (few threads, a few writes each, e.g. one
  * small block per tile of a wavefront): the same record, but the write's chunk
- * mark is stored without first testing it, so the hook issues only stores and
- * atomics and never waits on memory.  Do not use it where many warps write one
- * 2M-word region per epoch (every commit would store the same super-chunk byte). */
+ * mark is stored without first testing it.  Do not use it where many warps
+ * write one 2M-word region per epoch (every commit would store the same
+ * super-chunk byte). */
 template <class T>
 static __device__ __forceinline__ T& xpl_write_lat(T& x) {
   xpl_dev_record_k<XPL_ACC_W, false>(&x, sizeof(T), XPL_ACC_W);

@@ -237,7 +237,7 @@ __global__ void __launch_bounds__(256) range_kernel(const RangeDesc* __restrict_
         const uint32_t lb = in[c] & kL4;
         uint32_t m = 0;
         if (r.acc & XPL_ACC_R) m |= ((lb << 7) | ((~lb & kL4) << 6)) & bms[c];
-        if (r.acc & XPL_ACC_W) m |= 0x0A0A0A0Au & bms[c];
+        if (r.acc & XPL_ACC_W) m |= (0x08080808u | ((~lb & kL4) << 1)) & bms[c];  // P only where L = CPU
         if ((in[c] & m) == m) continue;
         const uint32_t q = (uint32_t)(vi * 4 + c);
         atomicOr(pool + q, m);
