@@ -39,28 +39,33 @@ constexpr uint32_t kP4 = 0x02020202u;
 // launch overlaps their tail.
 constexpr int kFoldThreads = 256;
 #ifndef XPL_FOLD_CTAS
-#define XPL_FOLD_CTAS (148 * 8)  // grid cap (A/B: profiles/r1_fold_grid_ab.txt)
+#define XPL_FOLD_CTAS (148 * 3)  // grid cap: one wave at 3 CTAs per SM (the register budget below)
 #endif
 
-__device__ __forceinline__ uint32_t fold_chunk(uint32_t* pool, uint64_t ch) {
-  uint4* w = reinterpret_cast<uint4*>(pool + ch * 32);
-  uint4 v[8];
-#pragma unroll
-  for (int k = 0; k < 8; ++k) v[k] = w[k];
+// P -> L over the 128-word chunks ch0 (if m0) and ch1 (if m1) of one lane: all
+// sixteen 16 B loads issued before the first store (one round trip for both).
+__device__ __forceinline__ void fold_two(uint32_t* pool, uint64_t ch0, bool m0, uint64_t ch1, bool m1) {
+  uint4* w0 = reinterpret_cast<uint4*>(pool + ch0 * 32);
+  uint4* w1 = reinterpret_cast<uint4*>(pool + ch1 * 32);
+  uint4 v[16];
 #pragma unroll
   for (int k = 0; k < 8; ++k) {
+    v[k] = m0 ? w0[k] : make_uint4(0, 0, 0, 0);
+    v[8 + k] = m1 ? w1[k] : make_uint4(0, 0, 0, 0);
+  }
+#pragma unroll
+  for (int k = 0; k < 16; ++k) {
     if ((v[k].x | v[k].y | v[k].z | v[k].w) & kP4) {
       v[k].x = (v[k].x & ~kP4) | ((v[k].x & kP4) >> 1);
       v[k].y = (v[k].y & ~kP4) | ((v[k].y & kP4) >> 1);
       v[k].z = (v[k].z & ~kP4) | ((v[k].z & kP4) >> 1);
       v[k].w = (v[k].w & ~kP4) | ((v[k].w & kP4) >> 1);
-      w[k] = v[k];
+      (k < 8 ? w0 : w1)[k & 7] = v[k];
     }
   }
-  return 1;
 }
 
-__global__ void __launch_bounds__(kFoldThreads) fold_kernel(uint32_t* __restrict__ pool,
+__global__ void __launch_bounds__(kFoldThreads, 3) fold_kernel(uint32_t* __restrict__ pool,
                                                             uint8_t* __restrict__ cmap,
                                                             uint8_t* __restrict__ smap,
                                                             uint64_t n_super,
@@ -83,11 +88,14 @@ __global__ void __launch_bounds__(kFoldThreads) fold_kernel(uint32_t* __restrict
       ms &= ms - 1;
       const uint64_t s = w + (k0 + j) * W;
       const uint64_t c0 = s * 128 + lane;
-      const uint8_t m0 = cmap[c0], m1 = cmap[c0 + 32], m2 = cmap[c0 + 64], m3 = cmap[c0 + 96];
-      if (m0) { folded += fold_chunk(pool, c0); cmap[c0] = 0; }
-      if (m1) { folded += fold_chunk(pool, c0 + 32); cmap[c0 + 32] = 0; }
-      if (m2) { folded += fold_chunk(pool, c0 + 64); cmap[c0 + 64] = 0; }
-      if (m3) { folded += fold_chunk(pool, c0 + 96); cmap[c0 + 96] = 0; }
+      const bool m0 = cmap[c0], m1 = cmap[c0 + 32], m2 = cmap[c0 + 64], m3 = cmap[c0 + 96];
+      if (m0 || m1) fold_two(pool, c0, m0, c0 + 32, m1);
+      if (m2 || m3) fold_two(pool, c0 + 64, m2, c0 + 96, m3);
+      folded += m0 + m1 + m2 + m3;
+      if (m0) cmap[c0] = 0;
+      if (m1) cmap[c0 + 32] = 0;
+      if (m2) cmap[c0 + 64] = 0;
+      if (m3) cmap[c0 + 96] = 0;
       if (lane == 0) smap[s] = 0;
     }
   }
