@@ -50,3 +50,30 @@ def test_lulesh_reduced_equals_plain_and_periodic():
     assert persistent(red[1]) == persistent(red[2])  # (already periodic from timestep 2 on)
     # the final diagnose: every allocation freed after a reset -> no access in the interval
     assert all(r["any_acc"] == 0 and r["live"] == 0 for r in red[6])
+
+
+def test_cfg5_partition_merge_equals_plain():
+    """cfg5's expectations are replayed partitioned by allocation (the force
+    temporary in word windows) and merged; on a small mesh the merged reports
+    must equal the plain replay of the whole program, every field."""
+    from xplgen import lulesh as L
+    from xplgen.rodinia import layout
+    s, steps = 6, 3
+    fw = 24 * s ** 3 * 2
+    cut = [0, (fw // 3 + 5) & ~1, (2 * fw // 3 + 1) & ~1, fw]  # (windows cut between 8-byte elements)
+    jobs = [(f"g{i}", g, None) for i, g in enumerate(G.CFG5_GROUPS)]
+    jobs += [(f"force{i}", (), {0: [(cut[i], cut[i + 1])]}) for i in range(3)]
+    jobs.append(("dvdx", (), {1: [(0, 3 * s ** 3 * 2)]}))
+    parts = []
+    for name, slots, tmp in jobs:
+        keep = {0, 1} | {2 + k for k in slots}
+        d = G.replay(G.reduced(G.cfg5_ops(slots, tmp, s=s, steps=steps)))
+        parts.append({"name": name, "tmp": tmp,
+                      "diagnoses": [[r for r in x if r["id"] in keep or (tmp and r["id"] >= 50)] for x in d]})
+    got = G.cfg5_merge(parts)
+    spec = L.lulesh_spec(s)
+    addrs, _, _ = layout(spec, 0, 0, 1 << 40)
+    tmps = [((1 << 44) + t * (1 << 36), (1 << 44) + t * (1 << 36) + (1 << 35)) for t in range(steps)]
+    plain = _strip(run_trace(list(L.lulesh_trace_iter(addrs, spec, s, steps, L.topology(s, 0x58504C05),
+                                                      G.PARAMS, tmps))))
+    assert got == plain

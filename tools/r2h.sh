@@ -9,3 +9,5 @@ XPL_DIST_BACKEND=gloo timeout 1200 python -m torch.distributed.run --nnodes=1 --
 timeout 900 ncu --set full --import-source on --clock-control none -k regex:k_integrate_stress --launch-skip 2 --launch-count 1 -o gpurun_out/${T}_ncu_stress python bench.py --step-only --steps 1 --warmup 0 --timesteps 3 > gpurun_out/${T}_ncu_stress.log 2>&1
 timeout 900 ncu --set full --import-source on --clock-control none -k regex:fold_kernel --launch-skip 40 --launch-count 1 -o gpurun_out/${T}_ncu_fold python bench.py --step-only --steps 1 --warmup 0 --timesteps 3 > gpurun_out/${T}_ncu_fold.log 2>&1
 timeout 900 ncu --set full --import-source on --clock-control none -k regex:diag_tile --launch-skip 2 --launch-count 1 -o gpurun_out/${T}_ncu_diag python bench.py --step-only --steps 1 --warmup 0 --timesteps 3 > gpurun_out/${T}_ncu_diag.log 2>&1
+timeout 600 python tools/hook_bench.py > gpurun_out/${T}_hook_bench.json 2> gpurun_out/${T}_hook_bench.err
+timeout 1800 python bench.py > gpurun_out/${T}_bench.json 2> gpurun_out/${T}_bench.err

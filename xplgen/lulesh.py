@@ -111,9 +111,12 @@ def lulesh_trace(addrs, spec, s, steps, topo, params, tmp_addrs, windows=None, r
     return ops, hooks
 
 
-def lulesh_trace_iter(addrs, spec, s, steps, topo, params, tmp_addrs, windows=None, reset=1, final=True):
+def lulesh_trace_iter(addrs, spec, s, steps, topo, params, tmp_addrs, windows=None, reset=1, final=True,
+                      tmp_windows=None):
     """lulesh_trace op by op (a generator: the full cfg4 trace, ~4e8 events per
-    timestep, never has to exist at once)."""
+    timestep, never has to exist at once).  Sampled form only: tmp_windows =
+    {0: [(w0, w1), ...], 1: [...]} keeps the events of those word windows of the
+    force (0) / gradient (1) temporaries too (else temporaries have none)."""
     ne, nn, nsym, nblk = sizes(s)
     dom, dtb = addrs[0], addrs[1]
     A = [addrs[2 + k] for k in range(48)]
@@ -141,8 +144,17 @@ def lulesh_trace_iter(addrs, spec, s, steps, topo, params, tmp_addrs, windows=No
     def rep(addr, n):  # one address read by n threads of a kernel
         return addr * np.ones(min(n, 1) if sampled else n, np.uint64)
 
-    def TMP(fn):  # events of a temporary (not sampled)
-        return np.zeros(0, np.uint64) if sampled else fn()
+    def TMP(fn, which=None, base=None):  # events of a temporary
+        if not sampled:
+            return fn()
+        if not tmp_windows or which not in tmp_windows:
+            return np.zeros(0, np.uint64)
+        a = np.asarray(fn(), np.uint64).reshape(-1)
+        w = (a - np.uint64(base)) >> np.uint64(2)  # first word of each (8-byte) event
+        keep = np.zeros(a.size, bool)
+        for w0, w1 in tmp_windows[which]:
+            keep |= (w + np.uint64(1) >= np.uint64(w0)) & (w < np.uint64(w1))
+        return a[keep]
 
     # ---- host initialisation ----
     h = _Ev()
@@ -197,7 +209,7 @@ def lulesh_trace_iter(addrs, spec, s, steps, topo, params, tmp_addrs, windows=No
         ev.add(I4(NODELIST, 8 * e[:, None] + np.arange(8)), 4, R)
         for k in (X, Y, Z):
             ev.add(D(k, nl), 8, R)
-        ev.add(TMP(lambda: tf + 8 * u(np.arange(24 * ne))), 8, W)
+        ev.add(TMP(lambda: tf + 8 * u(np.arange(24 * ne)), 0, tf), 8, W)
         kernels.append(ev)
         # 3 hourglass
         ev = _Ev()
@@ -211,7 +223,7 @@ def lulesh_trace_iter(addrs, spec, s, steps, topo, params, tmp_addrs, windows=No
         ev.add(I4(NODELIST, 8 * e[:, None] + np.arange(8)), 4, R)
         for k in (XD, YD, ZD):
             ev.add(D(k, nl), 8, R)
-        ev.add(TMP(lambda: tf + 8 * u(np.arange(24 * ne))), 8, RW)
+        ev.add(TMP(lambda: tf + 8 * u(np.arange(24 * ne)), 0, tf), 8, RW)
         kernels.append(ev)
         # 4 corner sums
         ev = _Ev()
@@ -220,7 +232,7 @@ def lulesh_trace_iter(addrs, spec, s, steps, topo, params, tmp_addrs, windows=No
         ev.add(I4(NODEELEMSTART, nidx), 4, R)
         ev.add(I4(NODEELEMSTART, nidx + 1), 4, R)
         ev.add(I4(CORNERLIST, np.arange(len(cl))), 4, R)
-        ev.add(TMP(lambda: tf + 8 * u(3 * cl[:, None] + np.arange(3))), 8, R)
+        ev.add(TMP(lambda: tf + 8 * u(3 * cl[:, None] + np.arange(3)), 0, tf), 8, R)
         for k in (FX, FY, FZ):
             ev.add(D(k, nidx), 8, W)
         kernels.append(ev)
@@ -281,13 +293,13 @@ def lulesh_trace_iter(addrs, spec, s, steps, topo, params, tmp_addrs, windows=No
             ev.add(ptr(k, ne), 8, R)
             ev.add(D(k, e), 8, W)
         ev.add(ptr(TMP_DVDX, ne), 8, R)
-        ev.add(TMP(lambda: tg + 8 * u(np.arange(3 * ne))), 8, W)
+        ev.add(TMP(lambda: tg + 8 * u(np.arange(3 * ne)), 1, tg), 8, W)
         kernels.append(ev)
         # 10 lagrange
         ev = _Ev()
         ev.add(numelem(grid_e), 4, R)
         ev.add(ptr(TMP_DVDX, ne), 8, R)
-        ev.add(TMP(lambda: tg + 8 * u(np.arange(3 * ne))), 8, R)
+        ev.add(TMP(lambda: tg + 8 * u(np.arange(3 * ne)), 1, tg), 8, R)
         ev.add(ptr(VNEW, ne), 8, R)
         ev.add(D(VNEW, e), 8, R)
         ev.add(ptr(VDOV, ne), 8, R)
