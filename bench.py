@@ -612,6 +612,7 @@ def main():
     clocks = clk.stop()
     st1 = ctx.stats()
     hooks, host_acc, epochs, n_diag, n_rows = acc[-1]
+    sharded_reports = c4.last_reports if world > 1 else None  # (the last timed step's reports)
     per_step = int(_allsum(torch, dist, hooks + host_acc))  # the logical program's accesses
     ms_max = _allmax(torch, dist, ms_total)
     value = per_step * args.steps / (ms_max / 1e3)
@@ -635,7 +636,6 @@ def main():
     # --- uninstrumented twin (whole-program slowdown) ---------------------------
     twin_ms, _ = timed_steps(torch, c4, None, args.steps, flush=flush_buf)
     twin_ms = _allmax(torch, dist, twin_ms)
-    sharded_reports = c4.last_reports if world > 1 else None
 
     # --- hook path: kernels alone, instrumented vs twin, events on their stream --
     c4.prepare()

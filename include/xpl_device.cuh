@@ -385,7 +385,7 @@ static __device__ __forceinline__ bool xpld_find(unsigned long long a, ulonglong
     if (lo > 0 && a < __ldg(&rows[lo - 1].end)) {
       ri = lo - 1;
       hit = true;
-      xpl_row_cache[slot] = ri;  /* benign race: any lane's row is a valid entry */
+      atomicExch(xpl_row_cache + slot, ri); /* (lanes may store different rows: any is valid) */
       be = __ldg(reinterpret_cast<const ulonglong2*>(rows + ri));
       ow = __ldg(reinterpret_cast<const ulonglong2*>(rows + ri) + 1);
     }
@@ -546,41 +546,12 @@ struct xpl_read_proxy {
   bool hit;
   __device__ __forceinline__ explicit xpl_read_proxy(const T& v) : x(v) {
 #ifndef XPL_OFF
-    unsigned* const xpl_row_cache = xpld_row_cache();
     const unsigned long long a = (unsigned long long)&v;
-    const xpl_dev_row* rows = xpl_dctx.rows;
-    const unsigned n = __ldg(xpl_dctx.n_rows);
-    const unsigned slot = ((threadIdx.z * blockDim.y + threadIdx.y) * blockDim.x + threadIdx.x) >> 5 & 31;
-    unsigned ri = xpl_row_cache[slot];
-    const unsigned rc = ri < n ? ri : 0;
-    ulonglong2 be = __ldg(reinterpret_cast<const ulonglong2*>(rows + rc));
-    ulonglong2 ow = __ldg(reinterpret_cast<const ulonglong2*>(rows + rc) + 1);
-    bool h = ri < n && be.x <= a && a < be.y;
-    if (!h) {
-      unsigned lo = 0, hi = n;
-      while (lo < hi) {
-        const unsigned mid = (lo + hi) >> 1;
-        if (__ldg(&rows[mid].base) <= a) lo = mid + 1;
-        else hi = mid;
-      }
-      if (lo > 0 && a < __ldg(&rows[lo - 1].end)) {
-        ri = lo - 1;
-        h = true;
-        xpl_row_cache[slot] = ri;
-        be = __ldg(reinterpret_cast<const ulonglong2*>(rows + ri));
-        ow = __ldg(reinterpret_cast<const ulonglong2*>(rows + ri) + 1);
-      }
-    }
+    ulonglong2 be, ow;
     unsigned long long g0 = 1, g1 = 0;
     unsigned owner = 0;
-    if (h) {
-      const unsigned long long w0 = (a - be.x) >> 2;
-      unsigned long long wl = (a + sizeof(T) - 1 - be.x) >> 2;
-      if (wl > ow.y - 1) wl = ow.y - 1;
-      owner = (unsigned)(ow.x >> 56);
-      g0 = (ow.x & XPLD_OFF_MASK) + w0;
-      g1 = (ow.x & XPLD_OFF_MASK) + wl;
-    }
+    const bool h = xpld_find(a, be, ow);
+    if (h) xpld_words(a, sizeof(T), be, ow, g0, g1, owner);
     if (__any_sync(__activemask(), owner != xpl_dctx.rank && h)) {  /* sharded: remote words now */
       if (owner != xpl_dctx.rank && h) {
         xpld_remote<XPL_ACC_R>(owner, g0, g1, XPL_ACC_R);
