@@ -27,7 +27,8 @@ class XplwRun(C.Structure):
                 ("diag_rows", vp), ("diag_cap", sz), ("n_diag", sz), ("dev_accesses", u64),
                 ("host_accesses", u64), ("copy_words", u64), ("epochs", u64), ("status", i32),
                 ("time_kernels", i32), ("kernel_ms", C.c_double), ("host_ms", C.c_double),
-                ("diag_no_reset", i32), ("keep_allocs", i32), ("rank", i32), ("world", i32)]
+                ("diag_no_reset", i32), ("keep_allocs", i32), ("rank", i32), ("world", i32),
+                ("kernel_ms_each", vp), ("kernel_cap", sz)]
 
 
 _w = xpl._work
@@ -113,6 +114,10 @@ class Run:
                  time_kernels=False, diag_reset=True, keep_allocs=False, rank=0, world=1):
         self.r = XplwRun()
         self.r.rank, self.r.world = rank, world
+        if time_kernels:  # each launch's event time too (LULESH)
+            self.kernel_each = (C.c_float * 8192)()
+            self.r.kernel_ms_each = C.cast(self.kernel_each, vp)
+            self.r.kernel_cap = 8192
         self.r.diag_no_reset = int(not diag_reset)
         self.r.keep_allocs = int(keep_allocs)
         self.r.time_kernels = int(time_kernels)

@@ -497,6 +497,7 @@ int xplw_lulesh(xplw_run* run, const xplw_arrays* arr, int s, int steps, unsigne
       float ms = 0.f;
       cudaEventElapsedTime(&ms, evs[i], evs[i + 1]);
       run->kernel_ms += ms;
+      if (run->kernel_ms_each && i / 2 < run->kernel_cap) run->kernel_ms_each[i / 2] = ms;
     }
     for (cudaEvent_t e : evs) cudaEventDestroy(e);
     evs.clear();

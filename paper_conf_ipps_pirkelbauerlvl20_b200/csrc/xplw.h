@@ -52,6 +52,8 @@ typedef struct {
                            *     frees + diagnose), for shadow dumps (LULESH)      */
   int rank, world;        /* world > 1: this process is rank `rank` of a sharded  *
                            * run (ctx sharded too); LULESH runs its slab only     */
+  float* kernel_ms_each;  /* time_kernels: each launch's event time, in order (or NULL) */
+  size_t kernel_cap;
 } xplw_run;
 
 /* Rodinia hotspot: rows x cols temperatures, `iters` 5-point stencil steps.
