@@ -130,3 +130,40 @@ def test_cfg3_sw16k_full_size():
     # CPU-written boundary row 0 and column 0 the last diagonals still read -- here
     # the whole-run check: every diagnose reports H's words and a G>G majority
     assert all(d[2]["words"] == (n + 1) * (mm + 1) for d in got)
+
+
+def test_cfg5_lulesh250_full_size():
+    """configs[4] (cfg5) at full size on one B200 -- LULESH-shaped 250^3 x 100
+    timesteps, 2.3e9 shadow words per timestep -- against the oracle's
+    partitioned replay (tests/golden/fullsize/cfg5.json, tools/golden_fullsize.py
+    cfg5): timesteps 1-2 every row, 3..100 equal to timestep 2 (periodic), the
+    final diagnose every row."""
+    import torch
+    from paper_conf_ipps_pirkelbauerlvl20_b200 import apps, xpl
+    from xplgen import lulesh as L
+    gold = _load("cfg5")
+    s, T = 250, 100
+    params = tuple(gold["meta"]["params"])
+    steps = gold["meta"]["steps"]
+    spec = L.lulesh_spec(s)
+    ar = apps.Arena(spec)
+    apps.lulesh_prepare(ar, s, L.topology(s, gold["meta"]["seed"]))
+    hc = torch.zeros(1, dtype=torch.int64, device="cuda")
+    st = torch.cuda.Stream()
+    with xpl.Context(pool_words=2_500_000_000, max_rows=64) as ctx:  # bench.py's cfg5 context
+        run = apps.Run(ctx, st.cuda_stream, params=params, out_cap=64 * (T + 2))
+        apps.lulesh(run, ar, s, T, hc)
+        got = [_strip(d) for d in run.reports()]
+    exp = gold["diagnoses"]
+    assert len(exp) == steps + 1 and len(got) == T + 1
+    for t in range(steps):
+        assert [r["id"] for r in got[t]] == [r["id"] for r in exp[t]]
+        for g, e in zip(got[t], exp[t]):
+            assert not _diff(g, e), (t, e["id"], _diff(g, e))
+    per = lambda d: [r for r in d if r["id"] < 50]
+    tmp = lambda d: [{f: v for f, v in r.items() if f != "id"} for r in d if r["id"] >= 50]
+    for t in range(steps, T):
+        assert per(got[t]) == per(exp[steps - 1]), t
+        assert tmp(got[t]) == tmp(exp[steps - 1]), t
+    for g, e in zip(got[T], exp[steps]):
+        assert not _diff(g, e), ("final", e["id"], _diff(g, e))
