@@ -14,7 +14,10 @@ cfg4: the golden holds the first 3 timesteps + the final diagnose (SURVEY §8(d)
       4..100 with timestep 3 (temporaries: new ids every timestep), the final
       diagnose with the golden final one; and the complete rows of `dom` (the
       Fig. 4 object) and `dt_block` of all 100 diagnoses against the oracle's
-      replay of the sampled twin (every event of those two allocations)."""
+      replay of the sampled twin (every event of those two allocations).
+cfg5: LULESH-shaped 250^3 x 100 timesteps on one GPU against the oracle's
+      replay partitioned by allocation (timesteps 1-2 + the final diagnose;
+      periodic from timestep 2 on)."""
 import json
 import os
 
@@ -126,9 +129,6 @@ def test_cfg3_sw16k_full_size():
         assert len(gd) == len(ed)
         for g, e in zip(gd, ed):
             assert not _diff(g, e), (t, e["id"], _diff(g, e))
-    # Fig. 7: the final interval's C>G reads of H are exactly the
-    # CPU-written boundary row 0 and column 0 the last diagonals still read -- here
-    # the whole-run check: every diagnose reports H's words and a G>G majority
     assert all(d[2]["words"] == (n + 1) * (mm + 1) for d in got)
 
 
