@@ -254,16 +254,6 @@ static __device__ __forceinline__ void xpld_put(unsigned q, unsigned cur, unsign
   }
 }
 
-/* OR, over the lanes of group mask gm, of the byte lanes each lane of `mask`
- * sets in v (a 0xFF-per-record byte mask): four ballots, one per byte lane. */
-static __device__ __forceinline__ unsigned xpld_group_bytes(unsigned mask, unsigned v, unsigned gm) {
-  unsigned u = 0;
-#pragma unroll
-  for (unsigned k = 0; k < 4; ++k)
-    if (__ballot_sync(mask, (v >> (8 * k)) & 1u) & gm) u |= 0xFFu << (8 * k);
-  return u;
-}
-
 /* The lanes of `ones` each access words [g0, g0+nb1] inside ONE shadow u32
  * (every aligned access of <= 4 words: ints, floats, doubles, ...):
  *  1. each lane loads its shadow u32 and tests whether a bit of its access is
