@@ -112,59 +112,90 @@ __global__ void __launch_bounds__(kFoldThreads, 3) fold_kernel(uint32_t* __restr
 // of written words and resets the scratch.  The scratch covers only the pool
 // words [fw0, fw0 + span) the batch touches (fw[w - fw0]).
 
+__device__ __forceinline__ void merge_firstw_rec(const uint64_t* __restrict__ recs, uint32_t i,
+                                                 uint32_t* __restrict__ fw, uint64_t fw0) {
+  const uint64_t r = recs[i];
+  if (!(rec_acc(r) & XPL_ACC_W)) return;
+  const uint64_t g0 = rec_g0(r), nw = rec_nw(r);
+  for (uint64_t w = g0; w < g0 + nw; ++w) atomicMin(fw + (w - fw0), i);
+}
+
+__device__ __forceinline__ void merge_apply_rec(const uint64_t* __restrict__ recs, uint32_t i,
+                                                const uint32_t* __restrict__ fw, uint64_t fw0, uint32_t* pool) {
+  const uint64_t r = recs[i];
+  const uint32_t acc = rec_acc(r);
+  const uint64_t g0 = rec_g0(r), g1 = g0 + rec_nw(r) - 1;
+  for (uint64_t q = g0 >> 2; q <= (g1 >> 2); ++q) {
+    const uint32_t cur = pool[q];  // L bits do not change during this pass
+    uint32_t m = 0;
+#pragma unroll
+    for (uint32_t k = 0; k < 4; ++k) {
+      const uint64_t w = q * 4 + k;
+      if (w < g0 || w > g1) continue;
+      uint32_t b = 0;
+      if (acc & XPL_ACC_R) {
+        const bool before = (fw == nullptr) || i <= fw[w - fw0];
+        b = before ? (((cur >> (8 * k)) & 1u) ? kRGC : kRCC) : kRCC;
+      }
+      if (acc & XPL_ACC_W) b |= kWC;
+      m |= b << (8 * k);
+    }
+    if ((cur & m) != m) atomicOr(pool + q, m);
+  }
+}
+
+__device__ __forceinline__ void merge_clear_rec(const uint64_t* __restrict__ recs, uint32_t i,
+                                                uint32_t* __restrict__ fw, uint64_t fw0, uint32_t* pool) {
+  const uint64_t r = recs[i];
+  if (!(rec_acc(r) & XPL_ACC_W)) return;
+  const uint64_t g0 = rec_g0(r), g1 = g0 + rec_nw(r) - 1;
+  for (uint64_t q = g0 >> 2; q <= (g1 >> 2); ++q) {
+    uint32_t lm = 0;
+#pragma unroll
+    for (uint32_t k = 0; k < 4; ++k) {
+      const uint64_t w = q * 4 + k;
+      if (w >= g0 && w <= g1) lm |= kL << (8 * k);
+    }
+    if (pool[q] & lm) atomicAnd(pool + q, ~lm);
+  }
+  if (fw)
+    for (uint64_t w = g0; w <= g1; ++w) fw[w - fw0] = 0xFFFFFFFFu;
+}
+
 __global__ void merge_firstw_kernel(const uint64_t* __restrict__ recs, uint32_t n,
                                     uint32_t* __restrict__ fw, uint64_t fw0) {
-  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
-    const uint64_t r = recs[i];
-    if (!(rec_acc(r) & XPL_ACC_W)) continue;
-    const uint64_t g0 = rec_g0(r), nw = rec_nw(r);
-    for (uint64_t w = g0; w < g0 + nw; ++w) atomicMin(fw + (w - fw0), i);
-  }
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
+    merge_firstw_rec(recs, i, fw, fw0);
 }
 
 __global__ void merge_apply_kernel(const uint64_t* __restrict__ recs, uint32_t n,
                                    const uint32_t* __restrict__ fw, uint64_t fw0, uint32_t* pool) {
-  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
-    const uint64_t r = recs[i];
-    const uint32_t acc = rec_acc(r);
-    const uint64_t g0 = rec_g0(r), g1 = g0 + rec_nw(r) - 1;
-    for (uint64_t q = g0 >> 2; q <= (g1 >> 2); ++q) {
-      const uint32_t cur = pool[q];  // L bits do not change during this kernel
-      uint32_t m = 0;
-#pragma unroll
-      for (uint32_t k = 0; k < 4; ++k) {
-        const uint64_t w = q * 4 + k;
-        if (w < g0 || w > g1) continue;
-        uint32_t b = 0;
-        if (acc & XPL_ACC_R) {
-          const bool before = (fw == nullptr) || i <= fw[w - fw0];
-          b = before ? (((cur >> (8 * k)) & 1u) ? kRGC : kRCC) : kRCC;
-        }
-        if (acc & XPL_ACC_W) b |= kWC;
-        m |= b << (8 * k);
-      }
-      if ((cur & m) != m) atomicOr(pool + q, m);
-    }
-  }
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
+    merge_apply_rec(recs, i, fw, fw0, pool);
 }
 
 __global__ void merge_clear_kernel(const uint64_t* __restrict__ recs, uint32_t n,
                                    uint32_t* __restrict__ fw, uint64_t fw0, uint32_t* pool) {
-  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
-    const uint64_t r = recs[i];
-    if (!(rec_acc(r) & XPL_ACC_W)) continue;
-    const uint64_t g0 = rec_g0(r), g1 = g0 + rec_nw(r) - 1;
-    for (uint64_t q = g0 >> 2; q <= (g1 >> 2); ++q) {
-      uint32_t lm = 0;
-#pragma unroll
-      for (uint32_t k = 0; k < 4; ++k) {
-        const uint64_t w = q * 4 + k;
-        if (w >= g0 && w <= g1) lm |= kL << (8 * k);
-      }
-      if (pool[q] & lm) atomicAnd(pool + q, ~lm);
-    }
-    if (fw)
-      for (uint64_t w = g0; w <= g1; ++w) fw[w - fw0] = 0xFFFFFFFFu;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
+    merge_clear_rec(recs, i, fw, fw0, pool);
+}
+
+// A small batch (a host segment of a few thousand records, the common case
+// between epochs): the three passes in one CTA, separated by CTA barriers
+// instead of kernel boundaries -- one launch instead of three.
+constexpr uint32_t kMergeSmall = 8192;
+__global__ void __launch_bounds__(1024) merge_small_kernel(const uint64_t* __restrict__ recs, uint32_t n,
+                                                           bool has_r, bool has_w, uint32_t* __restrict__ fw,
+                                                           uint64_t fw0, uint32_t* pool) {
+  const bool both = has_r && has_w;
+  if (both) {
+    for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) merge_firstw_rec(recs, i, fw, fw0);
+    __syncthreads();
+  }
+  for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) merge_apply_rec(recs, i, both ? fw : nullptr, fw0, pool);
+  if (has_w) {
+    __syncthreads();
+    for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) merge_clear_rec(recs, i, both ? fw : nullptr, fw0, pool);
   }
 }
 
@@ -1129,6 +1160,10 @@ void launch_fold(cudaStream_t s, bool pdl, uint32_t* pool, uint8_t* cmap, uint8_
 
 void launch_merge(cudaStream_t s, const uint64_t* recs, uint32_t n, bool has_r, bool has_w,
                   uint32_t* first_w, uint64_t fw0, uint32_t* pool) {
+  if (n <= kMergeSmall) {
+    merge_small_kernel<<<1, 1024, 0, s>>>(recs, n, has_r, has_w, first_w, fw0, pool);
+    return;
+  }
   const int g = grid_for(n, 256, 148 * 16);
   const bool both = has_r && has_w;
   if (both) merge_firstw_kernel<<<g, 256, 0, s>>>(recs, n, first_w, fw0);

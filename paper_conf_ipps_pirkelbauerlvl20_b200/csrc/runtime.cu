@@ -455,7 +455,7 @@ xpl_status flush_local(xpl_ctx* c) {
     launch_merge(c->cs, c->d_stage, (uint32_t)n, c->stage_has_r, c->stage_has_w, c->d_first_w, fw0,
                  (uint32_t*)c->d_pool);
     prof_end(c, pi);
-    c->st.kernel_launches += 1 + c->stage_has_w + (c->stage_has_r && c->stage_has_w);
+    c->st.kernel_launches += n <= 8192 ? 1 : 1 + c->stage_has_w + (c->stage_has_r && c->stage_has_w);
     c->st.merge_segments++;
   } else {
     // pieces go to a pinned buffer of their own, uploaded once
@@ -548,7 +548,7 @@ xpl_status flush_local(xpl_ctx* c) {
         launch_merge(c->cs, c->d_pieces + sg.start, (uint32_t)sg.n, sg.has_r, sg.has_w,
                      c->d_first_w, fw0, (uint32_t*)c->d_pool);
         prof_end(c, pi);
-        c->st.kernel_launches += 1 + sg.has_w + (sg.has_r && sg.has_w);
+        c->st.kernel_launches += sg.n <= 8192 ? 1 : 1 + sg.has_w + (sg.has_r && sg.has_w);
         c->st.merge_segments++;
       }
     }
