@@ -530,8 +530,24 @@ def sharded_tail(args, torch, dist, apps, xpl, rank, world, value, ms_max, per_s
         with xpl.Context(device=torch.cuda.current_device(), pool_words=1 << 28, max_rows=64) as ctx1:
             c1.prepare()
             one = c1.run(ctx1).reports()
-        strip = lambda ds: [[{f: v for f, v in r.items() if f != "base"} for r in d] for d in ds]
-        identical = strip(one) == strip(sharded_reports)
+        # (ids continue across the context's runs, bases are each program's own)
+        strip = lambda ds: [[{f: v for f, v in r.items() if f not in ("base", "id")} for r in d] for d in ds]
+        a, b = strip(one), strip(sharded_reports)
+        identical = a == b
+        if not identical:  # the first difference, for the record
+            for k, (da, db) in enumerate(zip(a, b)):
+                if da != db:
+                    for i, (ra, rb) in enumerate(zip(da, db)):
+                        if ra != rb:
+                            first_diff = {"diagnose": k, "row": i,
+                                          "fields": {f: (ra[f], rb[f]) for f in ra if ra[f] != rb[f]}}
+                            break
+                    else:
+                        first_diff = {"diagnose": k, "rows": (len(da), len(db))}
+                    break
+            else:
+                first_diff = {"diagnoses": (len(a), len(b))}
+            print(json.dumps({"identity_first_difference": first_diff}), file=sys.stderr, flush=True)
     roof = hook_roofline(args, hook_med, k_instr, k_twin, ms_max / args.steps, prof, peak, peak_src)
     line = {"metric": METRIC, "value": value, "unit": "accesses/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
