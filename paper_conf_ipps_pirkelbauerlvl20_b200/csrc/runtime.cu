@@ -110,6 +110,8 @@ struct xpl_ctx {
 
   // shadow memory table
   std::vector<Row> rows;               // by id
+  std::vector<uint64_t> active;        // ids of the rows a diagnose reports (live, or freed since the
+                                       // last reset), ascending: the walks below skip dropped rows
   std::map<uint64_t, uint64_t> live;   // base -> id
   uint32_t n_dead = 0;
   uint8_t* d_tab = nullptr;            // [u32 n | pad to 32 B | xpl_dev_row[max_rows]]
@@ -818,8 +820,8 @@ xpl_status xpl_page_summary(xpl_ctx* c, uint64_t P, xpl_page_report* out, size_t
   if (!c || !n_out || P == 0 || (cap && !out)) return XPL_ERR_INVALID_ARG;
   if (c->depth || c->world > 1) return XPL_ERR_STATE;  // (the page view is single-GPU)
   std::vector<const Row*> rows;
-  for (const Row& r : c->rows)
-    if (r.live) rows.push_back(&r);  // (c->rows is in id order)
+  for (uint64_t id : c->active)
+    if (c->rows[id].live) rows.push_back(&c->rows[id]);  // (active is in id order)
   *n_out = rows.size();
   if (cap < rows.size()) return XPL_ERR_INVALID_ARG;
   xpl_status st = flush(c);
@@ -1086,6 +1088,7 @@ static xpl_status register_row(xpl_ctx* c, const void* ptr, size_t bytes, xpl_al
   c->rows.push_back(r);
   if (c->rows.capacity() != cap_before) c->cache = nullptr;
   c->live[p] = r.id;
+  c->active.push_back(r.id);
   c->lrows[r.logical_id].push_back(r.id);
   c->table_dirty = true;
   c->cache = nullptr;
@@ -1576,7 +1579,10 @@ xpl_status xpl_shadow_dump(xpl_ctx* c, const void* base, uint64_t word0, uint64_
 // their shadow (D17); in sharded mode every rank drops every piece
 // (each rank keeps every owner's pool allocator in step).
 static void drop_dead(xpl_ctx* c) {
-  for (Row& r : c->rows) {
+  std::vector<uint64_t> keep;
+  for (uint64_t id : c->active) {
+    Row& r = c->rows[id];
+    if (r.live) keep.push_back(id);
     if (!r.live && !r.dropped) {
       r.dropped = true;
       c->pas[r.owner].release(r.off, r.span);
@@ -1588,6 +1594,7 @@ static void drop_dead(xpl_ctx* c) {
       }
     }
   }
+  c->active.swap(keep);
   c->n_dead = 0;
 }
 
@@ -1608,8 +1615,8 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
   const uint64_t B = p.block_words;
 
   std::vector<uint64_t> ids;  // live rows + rows freed since the last reset, id order (D23)
-  for (const Row& r : c->rows)
-    if ((r.live || !r.dropped) && r.owner == (uint32_t)c->rank) ids.push_back(r.id);
+  for (uint64_t id : c->active)
+    if (c->rows[id].owner == (uint32_t)c->rank) ids.push_back(id);
   *n_out = ids.size();
   if (cap < ids.size() || (!out && !pout && ids.size())) return XPL_ERR_INVALID_ARG;
 
@@ -1823,11 +1830,11 @@ xpl_status xpl_diagnose(xpl_ctx* c, const xpl_diag_params* params, const xpl_nam
   if (c->depth) return XPL_ERR_STATE;
   std::vector<uint64_t> lids;
   size_t n_own = 0;
-  for (const Row& r : c->rows)
-    if (r.live || !r.dropped) {
-      lids.push_back(r.logical_id);
-      if (r.owner == (uint32_t)c->rank) ++n_own;
-    }
+  for (uint64_t id : c->active) {
+    const Row& r = c->rows[id];
+    lids.push_back(r.logical_id);
+    if (r.owner == (uint32_t)c->rank) ++n_own;
+  }
   std::sort(lids.begin(), lids.end());
   lids.erase(std::unique(lids.begin(), lids.end()), lids.end());
   *n_out = lids.size();
