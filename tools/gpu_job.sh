@@ -11,6 +11,8 @@
 #   ncu:REGEX[:SKIP[:CMD]] ncu --set full of one launch of kernel REGEX (default command: bench.py --step-only)
 #   py:SCRIPT[:ARGS]       python SCRIPT ARGS > TAG_<name>.json
 #   sanitize:TOOL          compute-sanitizer --tool TOOL (memcheck|synccheck|racecheck) over tools/sanitize_driver.py
+#   bench2[:ARGS]          2 ranks on this one GPU over gloo (the sharded N>1 bench path): torchrun bench.py --gpus 2
+#   golden5                cfg5's oracle expectations on the box's host cores (tools/golden_fullsize.py cfg5)
 TAG=$1; shift
 mkdir -p gpurun_out
 echo "nproc=$(nproc) $(nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv,noheader)" > gpurun_out/${TAG}_box.txt
@@ -21,7 +23,8 @@ for step in "$@"; do
     build) make -s -C paper_conf_ipps_pirkelbauerlvl20_b200/csrc -j8 > gpurun_out/${TAG}_build.log 2>&1 ;;
     smoke) python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/${TAG}_smoke.log 2>&1
            echo "rc=$?" >> gpurun_out/${TAG}_smoke.log ;;
-    pytest) timeout 2400 python -m pytest tests -q -m gpu --durations=15 $args > gpurun_out/${TAG}_pytest.log 2>&1
+    pytest) timeout 2400 python -u -m pytest tests -q -m gpu --durations=15 --timeout=1200 --timeout-method=thread \
+              -p no:cacheprovider $args > gpurun_out/${TAG}_pytest.log 2>&1
             echo "pytest rc=$?" >> gpurun_out/${TAG}_pytest.log ;;
     bench) timeout 1800 python bench.py $args > gpurun_out/${TAG}_bench.json 2> gpurun_out/${TAG}_bench.err ;;
     launches) timeout 1200 ncu --metrics gpu__time_duration.sum --clock-control none -c 2000 --csv \
@@ -38,6 +41,13 @@ for step in "$@"; do
         timeout 1800 python $script ${a2//+/ } > gpurun_out/${TAG}_$name.json 2> gpurun_out/${TAG}_$name.err ;;
     sanitize) timeout 1500 compute-sanitizer --tool $rest --print-limit 50 python tools/sanitize_driver.py \
                 > gpurun_out/${TAG}_sanitize_$rest.log 2>&1; echo "rc=$?" >> gpurun_out/${TAG}_sanitize_$rest.log ;;
+    bench2) XPL_DIST_BACKEND=gloo timeout 1800 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 \
+              --master-addr 127.0.0.1 --master-port 29533 bench.py --gpus 2 $args \
+              > gpurun_out/${TAG}_bench2.json 2> gpurun_out/${TAG}_bench2.err ;;
+    golden5) mkdir -p gpurun_out/golden5
+             W=$(python -c "import os; m=os.sysconf('SC_PAGE_SIZE')*os.sysconf('SC_PHYS_PAGES')/2**30; print(max(1, min(os.cpu_count()-1, int(m//36))))")
+             echo "workers=$W" > gpurun_out/golden5/box.txt; free -g >> gpurun_out/golden5/box.txt
+             python tools/golden_fullsize.py cfg5 --workers $W --out gpurun_out/golden5 > gpurun_out/golden5/log.txt 2>&1 ;;
     *) echo "unknown step $step" >> gpurun_out/${TAG}_box.txt ;;
   esac
 done
