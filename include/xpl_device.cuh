@@ -384,16 +384,19 @@ static __device__ __forceinline__ bool xpld_find(unsigned long long a, ulonglong
 }
 
 /* Words [g0, g1] (in the owner's pool) of an access of `size` bytes at a in the
- * row (be, ow): clipped to the row (D1, D18). */
-static __device__ __forceinline__ void xpld_words(unsigned long long a, unsigned size, const ulonglong2& be,
-                                                  const ulonglong2& ow, unsigned long long& g0,
-                                                  unsigned long long& g1, unsigned& owner) {
-  const unsigned long long w0 = (a - be.x) >> 2;
-  unsigned long long wl = (a + size - 1 - be.x) >> 2;
-  if (wl > ow.y - 1) wl = ow.y - 1;
-  owner = (unsigned)(ow.x >> 56);
-  g0 = (ow.x & XPLD_OFF_MASK) + w0;
-  g1 = (ow.x & XPLD_OFF_MASK) + wl;
+ * row [base, end) whose shadow starts at pool word offo (owner rank in the top
+ * byte): clipped to the row (D1, D18; its last word is (end - 1 - base) / 4). */
+static __device__ __forceinline__ void xpld_words(unsigned long long a, unsigned size, unsigned long long base,
+                                                  unsigned long long end, unsigned long long offo,
+                                                  unsigned long long& g0, unsigned long long& g1,
+                                                  unsigned& owner) {
+  const unsigned long long w0 = (a - base) >> 2;
+  unsigned long long wl = (a + size - 1 - base) >> 2;
+  const unsigned long long wmax = (end - 1 - base) >> 2;
+  if (wl > wmax) wl = wmax;
+  owner = (unsigned)(offo >> 56);
+  g0 = (offo & XPLD_OFF_MASK) + w0;
+  g1 = (offo & XPLD_OFF_MASK) + wl;
 }
 
 /* Record words [g0, g1] of rank `owner`'s pool (g0 > g1: nothing).  All active
@@ -454,7 +457,7 @@ static __device__ __forceinline__ void xpl_dev_record_k(const void* p, unsigned 
   ulonglong2 be, ow;
   unsigned long long g0 = 1, g1 = 0;
   unsigned owner = xpl_dctx.rank;
-  if (xpld_find(a, be, ow) && size > 0) xpld_words(a, size, be, ow, g0, g1, owner);
+  if (xpld_find(a, be, ow) && size > 0) xpld_words(a, size, be.x, be.y, ow.x, g0, g1, owner);
   if (K != 0) xpld_record_fast<K, TM>(g0, g1, owner);
   else xpld_record_words<K, TM>(g0, g1, owner, acc);
 #else
@@ -471,10 +474,15 @@ static __device__ __forceinline__ void xpl_dev_record_k(const void* p, unsigned 
 template <class T>
 struct xpl_array {
   T* p;
-  ulonglong2 be, ow; /* the row of p; be = {0, 0}: none */
+  unsigned long long base = 0, end = 0, offo = 0; /* the row of p (end = 0: none) */
   __device__ __forceinline__ explicit xpl_array(T* ptr) : p(ptr) {
 #ifndef XPL_OFF
-    if (!xpld_find((unsigned long long)ptr, be, ow)) be = make_ulonglong2(0, 0);
+    ulonglong2 be, ow;
+    if (xpld_find((unsigned long long)ptr, be, ow)) {
+      base = be.x;
+      end = be.y;
+      offo = ow.x;
+    }
 #endif
   }
   template <unsigned K>
@@ -483,11 +491,11 @@ struct xpl_array {
     const unsigned long long a = (unsigned long long)(p + i);
     unsigned long long g0 = 1, g1 = 0;
     unsigned owner = xpl_dctx.rank;
-    if (a - be.x < be.y - be.x) {
-      xpld_words(a, sizeof(T), be, ow, g0, g1, owner);
+    if (a - base < end - base) {
+      xpld_words(a, sizeof(T), base, end, offo, g0, g1, owner);
     } else {
       ulonglong2 b2, o2;
-      if (xpld_find(a, b2, o2)) xpld_words(a, sizeof(T), b2, o2, g0, g1, owner);
+      if (xpld_find(a, b2, o2)) xpld_words(a, sizeof(T), b2.x, b2.y, o2.x, g0, g1, owner);
     }
     xpld_record_fast<K>(g0, g1, owner);
 #else
@@ -541,7 +549,7 @@ struct xpl_read_proxy {
     unsigned long long g0 = 1, g1 = 0;
     unsigned owner = 0;
     const bool h = xpld_find(a, be, ow);
-    if (h) xpld_words(a, sizeof(T), be, ow, g0, g1, owner);
+    if (h) xpld_words(a, sizeof(T), be.x, be.y, ow.x, g0, g1, owner);
     if (__any_sync(__activemask(), owner != xpl_dctx.rank && h)) {  /* sharded: remote words now */
       if (owner != xpl_dctx.rank && h) {
         xpld_remote<XPL_ACC_R>(owner, g0, g1, XPL_ACC_R);

@@ -94,6 +94,12 @@ struct Arr<false, T> {
   __device__ __forceinline__ T& rw(unsigned long long i) const { return p[i]; }
 };
 
+// Instrumented kernels: CTAs per SM the register budget is sized for (the hooks'
+// dependent loads want occupancy more than registers).
+#ifndef XPL_LULESH_MINB
+#define XPL_LULESH_MINB 3
+#endif
+
 // Hook calls are counted per thread (c) and added once per block (exact counts).
 template <bool I>
 __device__ __forceinline__ void count_hooks(unsigned long long* hc, unsigned c) {
@@ -120,7 +126,7 @@ __device__ __forceinline__ void count_hooks(unsigned long long* hc, unsigned c) 
 
 // 1. zero the nodal forces
 template <bool I>
-__global__ void k_zero_forces(Part P_, Dom* d, int nn, unsigned long long* hc) {
+__global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_zero_forces(Part P_, Dom* d, int nn, unsigned long long* hc) {
   const int n = P_.n0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   if (n < P_.n1 && n < nn) {
@@ -134,7 +140,7 @@ __global__ void k_zero_forces(Part P_, Dom* d, int nn, unsigned long long* hc) {
 
 // 2. stress integration: gather the 8 nodes, write 8 corner forces x 3
 template <bool I>
-__global__ void k_integrate_stress(Part P_, Dom* d, unsigned long long* hc) {
+__global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_integrate_stress(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
@@ -155,7 +161,7 @@ __global__ void k_integrate_stress(Part P_, Dom* d, unsigned long long* hc) {
 
 // 3. hourglass control: gather nodal velocities, add to the corner forces
 template <bool I>
-__global__ void k_hourglass(Part P_, Dom* d, unsigned long long* hc) {
+__global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_hourglass(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
@@ -177,7 +183,7 @@ __global__ void k_hourglass(Part P_, Dom* d, unsigned long long* hc) {
 
 // 4. sum the corner forces into the nodes through the node->corner lists
 template <bool I>
-__global__ void k_corner_sum(Part P_, Dom* d, int nn, unsigned long long* hc) {
+__global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_corner_sum(Part P_, Dom* d, int nn, unsigned long long* hc) {
   const int n = P_.n0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   if (n < P_.n1 && n < nn) {
@@ -201,7 +207,7 @@ __global__ void k_corner_sum(Part P_, Dom* d, int nn, unsigned long long* hc) {
 
 // 5. nodal accelerations
 template <bool I>
-__global__ void k_accel(Part P_, Dom* d, int nn, unsigned long long* hc) {
+__global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_accel(Part P_, Dom* d, int nn, unsigned long long* hc) {
   const int n = P_.n0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   if (n < P_.n1 && n < nn) {
@@ -217,7 +223,7 @@ __global__ void k_accel(Part P_, Dom* d, int nn, unsigned long long* hc) {
 
 // 6. symmetry plane: zero the accelerations of the plane's nodes
 template <bool I>
-__global__ void k_symm(Part P_, Dom* d, int ns, unsigned long long* hc) {
+__global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_symm(Part P_, Dom* d, int ns, unsigned long long* hc) {
   const int k = P_.s0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   if (k < P_.s1 && k < ns) {
@@ -231,7 +237,7 @@ __global__ void k_symm(Part P_, Dom* d, int ns, unsigned long long* hc) {
 
 // 7./8. velocity and position updates
 template <bool I>
-__global__ void k_velocity(Part P_, Dom* d, int nn, unsigned long long* hc) {
+__global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_velocity(Part P_, Dom* d, int nn, unsigned long long* hc) {
   const int n = P_.n0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   if (n < P_.n1 && n < nn) {
@@ -245,7 +251,7 @@ __global__ void k_velocity(Part P_, Dom* d, int nn, unsigned long long* hc) {
   count_hooks<I>(hc, c);
 }
 template <bool I>
-__global__ void k_position(Part P_, Dom* d, int nn, unsigned long long* hc) {
+__global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_position(Part P_, Dom* d, int nn, unsigned long long* hc) {
   const int n = P_.n0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   if (n < P_.n1 && n < nn) {
@@ -261,7 +267,7 @@ __global__ void k_position(Part P_, Dom* d, int nn, unsigned long long* hc) {
 
 // 9. element kinematics: gather positions and velocities, new volume, gradients
 template <bool I>
-__global__ void k_kinematics(Part P_, Dom* d, unsigned long long* hc) {
+__global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_kinematics(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
@@ -289,7 +295,7 @@ __global__ void k_kinematics(Part P_, Dom* d, unsigned long long* hc) {
 
 // 10. strain rate from the gradients
 template <bool I>
-__global__ void k_lagrange(Part P_, Dom* d, unsigned long long* hc) {
+__global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_lagrange(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
@@ -302,7 +308,7 @@ __global__ void k_lagrange(Part P_, Dom* d, unsigned long long* hc) {
 
 // 11./12. monotonic Q: gradients over the xi face neighbours, region limiter
 template <bool I>
-__global__ void k_monoq_grad(Part P_, Dom* d, unsigned long long* hc) {
+__global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_monoq_grad(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
@@ -314,7 +320,7 @@ __global__ void k_monoq_grad(Part P_, Dom* d, unsigned long long* hc) {
   count_hooks<I>(hc, c);
 }
 template <bool I>
-__global__ void k_monoq_region(Part P_, Dom* d, unsigned long long* hc) {
+__global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_monoq_region(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
@@ -327,7 +333,7 @@ __global__ void k_monoq_region(Part P_, Dom* d, unsigned long long* hc) {
 
 // 13. the four EOS stages (they read material parameters from the domain)
 template <bool I>
-__global__ void k_eos(Part P_, Dom* d, int stage, unsigned long long* hc) {
+__global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_eos(Part P_, Dom* d, int stage, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
@@ -359,7 +365,7 @@ __global__ void k_eos(Part P_, Dom* d, int stage, unsigned long long* hc) {
 
 // 14. volumes
 template <bool I>
-__global__ void k_update_volumes(Part P_, Dom* d, unsigned long long* hc) {
+__global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_update_volumes(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
@@ -371,7 +377,7 @@ __global__ void k_update_volumes(Part P_, Dom* d, unsigned long long* hc) {
 
 // 15./16. dt reductions: one minimum per 256-element block into dtb (GPU W, host R)
 template <bool I, bool COURANT>
-__global__ void __launch_bounds__(256) k_dt(Part P_, Dom* d, double* dtb, int nblk, unsigned long long* hc) {
+__global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_dt(Part P_, Dom* d, double* dtb, int nblk, unsigned long long* hc) {
   __shared__ double s_min[256];
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;

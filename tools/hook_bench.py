@@ -101,7 +101,7 @@ def main():
         ar = apps.Arena(spec)
         topo = L.topology(S, 0x58504C05)
         hc = torch.zeros(1, dtype=torch.int64, device="cuda")
-        res = {}
+        res, each = {}, {}
         with xpl.Context(pool_words=1 << 28, max_rows=64) as ctx:
             for c in (ctx, None, ctx, None):
                 apps.lulesh_prepare(ar, S, topo)
@@ -117,12 +117,16 @@ def main():
                 e1.record(rs if c is not None else st)
                 e1.synchronize()
                 torch.cuda.synchronize()
+                each["instr" if c is not None else "twin"] = list(run.kernel_each[:19 * a.lulesh_steps])
                 res["instr" if c is not None else "twin"] = {
                     "kernel_ms": run.r.kernel_ms, "total_ms": e0.elapsed_time(e1), "host_ms": run.r.host_ms,
                     "hooks": int(hc.item()), "epochs": run.r.epochs}
         st_ = a.lulesh_steps
+        import numpy as np
+        med = {k: np.median(np.array(v).reshape(st_, 19), axis=0) for k, v in each.items()}
         out["lulesh100"] = dict(res, steps=st_,
                                 hook_cost_ms_per_step=(res["instr"]["kernel_ms"] - res["twin"]["kernel_ms"]) / st_,
+                                hook_cost_ms_per_step_median=float(np.sum(med["instr"] - med["twin"])),
                                 kernel_slowdown=res["instr"]["kernel_ms"] / res["twin"]["kernel_ms"],
                                 hooks_per_step=res["instr"]["hooks"] / st_)
     print(json.dumps(out), flush=True)
