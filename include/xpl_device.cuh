@@ -474,30 +474,39 @@ static __device__ __forceinline__ void xpl_dev_record_k(const void* p, unsigned 
 template <class T>
 struct xpl_array {
   T* p;
-  unsigned long long base = 0, end = 0, offo = 0; /* the row of p (end = 0: none) */
+  /* element i of p (0 <= i < nel: whole elements inside the row holding p)
+   * covers pool words q0 + i * W .. q0 + i * W + W - 1 of rank `owner`; else
+   * (outside the row, or T not a multiple of 4 bytes / p not word-aligned in
+   * its row) the access takes the full lookup.  W = sizeof(T) / 4. */
+  unsigned long long q0 = 0, nel = 0;
+  unsigned owner = 0;
   __device__ __forceinline__ explicit xpl_array(T* ptr) : p(ptr) {
 #ifndef XPL_OFF
     ulonglong2 be, ow;
-    if (xpld_find((unsigned long long)ptr, be, ow)) {
-      base = be.x;
-      end = be.y;
-      offo = ow.x;
+    const unsigned long long a = (unsigned long long)ptr;
+    if (sizeof(T) % 4 == 0 && xpld_find(a, be, ow) && ((a - be.x) & 3) == 0) {
+      q0 = (ow.x & XPLD_OFF_MASK) + ((a - be.x) >> 2);
+      nel = (be.y - a) / sizeof(T);
+      owner = (unsigned)(ow.x >> 56);
     }
 #endif
   }
   template <unsigned K>
   __device__ __forceinline__ void rec(unsigned long long i) const {
 #ifndef XPL_OFF
-    const unsigned long long a = (unsigned long long)(p + i);
+    constexpr unsigned long long W = sizeof(T) / 4;
     unsigned long long g0 = 1, g1 = 0;
-    unsigned owner = xpl_dctx.rank;
-    if (a - base < end - base) {
-      xpld_words(a, sizeof(T), base, end, offo, g0, g1, owner);
+    unsigned own = owner;
+    if (i < nel) {
+      g0 = q0 + i * W;
+      g1 = g0 + (W - 1);
     } else {
+      const unsigned long long a = (unsigned long long)(p + i);
       ulonglong2 b2, o2;
-      if (xpld_find(a, b2, o2)) xpld_words(a, sizeof(T), b2.x, b2.y, o2.x, g0, g1, owner);
+      own = xpl_dctx.rank;
+      if (xpld_find(a, b2, o2)) xpld_words(a, sizeof(T), b2.x, b2.y, o2.x, g0, g1, own);
     }
-    xpld_record_fast<K>(g0, g1, owner);
+    xpld_record_fast<K>(g0, g1, own);
 #else
     (void)i;
 #endif
