@@ -17,9 +17,20 @@
 #include <unordered_map>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>  // (header-only NVTX 3: ranges cost nothing without a tool attached)
+
 #include "xpl_internal.h"
 
 using namespace xpl;
+
+namespace {
+// An NVTX range over one runtime call (nsight / ncu timelines show the
+// runtime's host work next to its kernels).
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+}  // namespace
 
 #define CK(x)                                      \
   do {                                             \
@@ -429,7 +440,11 @@ xpl_status route_flush(xpl_ctx* c) {
   return XPL_OK;
 }
 
-xpl_status flush(xpl_ctx* c) { return c->world > 1 ? route_flush(c) : flush_local(c); }
+xpl_status flush(xpl_ctx* c) {
+  if (c->world <= 1 && c->stage_n == 0) return XPL_OK;
+  NvtxRange nv("xpl host-record flush");
+  return c->world > 1 ? route_flush(c) : flush_local(c);
+}
 
 // Apply all staged host records on the runtime stream, in order.  Records of
 // more than kRangeWords words cut the batch and go through range_apply (runs of
@@ -1173,6 +1188,7 @@ xpl_status xpl_free(xpl_ctx* c, const void* ptr) {
 // streams are joined on rs first.
 xpl_status xpl_kernel_begin(xpl_ctx* c, void* stream) {
   if (!c) return XPL_ERR_INVALID_ARG;
+  NvtxRange nv("xpl_kernel_begin");
   cudaStream_t s = (cudaStream_t)stream;
   if (c->depth == 0) {
     xpl_status st = flush(c);
@@ -1204,6 +1220,7 @@ xpl_status xpl_kernel_begin(xpl_ctx* c, void* stream) {
 
 xpl_status xpl_kernel_end(xpl_ctx* c, void* stream) {
   if (!c) return XPL_ERR_INVALID_ARG;
+  NvtxRange nv("xpl_kernel_end");
   if (c->depth == 0) return XPL_ERR_STATE;
   cudaStream_t s = (cudaStream_t)stream;
   if (std::find(c->epoch_streams.begin(), c->epoch_streams.end(), s) == c->epoch_streams.end()) {
@@ -1604,6 +1621,7 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
                                 size_t n_names, xpl_alloc_report* out, xpl_partial* pout, size_t cap,
                                 size_t* n_out, int reset) {
   // (sharded mode: this rank analyses the pieces it owns)
+  NvtxRange nv("xpl_diagnose");
   if (!c || !n_out || (n_names && !names)) return XPL_ERR_INVALID_ARG;
   if (c->depth) return XPL_ERR_STATE;
   DiagParams p;
