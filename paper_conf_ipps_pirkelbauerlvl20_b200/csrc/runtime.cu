@@ -116,6 +116,7 @@ struct xpl_ctx {
   void* peer_pool[XPL_MAX_RANKS] = {};       // IPC-mapped pools / chunk maps of the other ranks
   void* peer_cmap[XPL_MAX_RANKS] = {};
   void* peer_smap[XPL_MAX_RANKS] = {};
+  bool ready = false;                        // xpl_init completed
   uint32_t* d_first_w = nullptr;  // merge scratch (first writer per word of a batch's span), grown lazily
   uint64_t first_w_cap = 0;
 
@@ -1002,6 +1003,7 @@ xpl_status xpl_init(const xpl_config* cfg, xpl_ctx** out) {
     if (c->comm->barrier(c->comm->user)) { xpl_finalize(c); return XPL_ERR_NCCL; }
   }
   memset(&c->st, 0, sizeof c->st);
+  c->ready = true;
   *out = c;
   return XPL_OK;
 #undef CKI
@@ -1011,8 +1013,9 @@ xpl_status xpl_finalize(xpl_ctx* c) {
   if (!c) return XPL_ERR_INVALID_ARG;
   if (c->cs) cudaStreamSynchronize(c->cs);
   if (c->rs) cudaStreamSynchronize(c->rs);
-  // (sharded: every rank finalises; no rank may unmap a pool a peer still writes)
-  if (c->world > 1 && c->comm && c->d_pool) c->comm->barrier(c->comm->user);
+  // (sharded: every rank finalises; no rank may unmap a pool a peer still writes --
+  // only once xpl_init completed, so a rank failing inside xpl_init does not wait)
+  if (c->world > 1 && c->comm && c->ready) c->comm->barrier(c->comm->user);
   for (int q = 0; q < XPL_MAX_RANKS; ++q)
     for (void* p : {c->peer_pool[q], c->peer_cmap[q], c->peer_smap[q]})
       if (p) cudaIpcCloseMemHandle(p);
@@ -1139,11 +1142,27 @@ xpl_status xpl_register_alloc(xpl_ctx* c, const void* ptr, size_t bytes, xpl_all
   const uint64_t lw = (bytes + 3) / 4;
   const auto pcs = shard_pieces(lid, lw, c->world);
   if (c->live.size() + pcs.size() > c->cfg.max_rows) return XPL_ERR_OOM;
-  for (const auto& pc : pcs) {  // (overlap of any piece = overlap of the whole range)
+  const size_t first_row = c->rows.size();
+  for (const auto& pc : pcs) {
     const uint64_t b0 = 4 * pc[0], b1 = std::min<uint64_t>(bytes, 4 * (pc[0] + pc[1]));
     xpl_status st = register_row(c, (const uint8_t*)ptr + b0, b1 - b0, kind, true, lid, pc[0], bytes,
                                  (uint32_t)pc[2]);
-    if (st) return st;  // (only the first piece can fail on overlap; OOM is fatal anyway)
+    if (st) {  // undo the pieces registered so far (every rank fails alike: same tables)
+      for (size_t id = first_row; id < c->rows.size(); ++id) {
+        Row& r = c->rows[id];
+        c->live.erase(r.base);
+        c->pas[r.owner].release(r.off, r.span);
+        r.live = false;
+        r.dropped = true;
+      }
+      c->active.erase(std::remove_if(c->active.begin(), c->active.end(),
+                                     [&](uint64_t id) { return id >= first_row; }),
+                      c->active.end());
+      c->lrows.erase(lid);
+      c->table_dirty = true;
+      c->cache = nullptr;
+      return st;
+    }
   }
   c->n_logical++;
   return XPL_OK;
