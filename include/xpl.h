@@ -200,13 +200,16 @@ typedef struct {
  * XPL_MAX_RANKS; the ranks' pools are mapped into each other (CUDA IPC) for the
  * hooks' remote atomics (every rank's pool_words must be equal). */
 xpl_status xpl_init(const xpl_config* cfg, xpl_ctx** out);
+/* Sharded mode: COLLECTIVE (no rank unmaps its pool while a peer may write it). */
 xpl_status xpl_finalize(xpl_ctx* ctx);
 
 /* The allocation wrappers.  register: ceil(bytes/4) zeroed records
  * (last writer = CPU, D3); OVERLAP if [ptr, ptr+bytes) intersects a live row;
  * STATE inside an open GPU epoch.  free: UNKNOWN_PTR unless ptr is a live
  * base; the row stops matching lookups now and is reported once more at the
- * next diagnose before its shadow is recycled (D17). */
+ * next diagnose before its shadow is recycled (D17).
+ * Sharded mode: both COLLECTIVE (same bytes / kind / order on every rank; free
+ * takes each rank's own base of the allocation). */
 xpl_status xpl_register_alloc(xpl_ctx* ctx, const void* ptr, size_t bytes, xpl_alloc_kind kind);
 xpl_status xpl_free(xpl_ctx* ctx, const void* ptr);
 
@@ -221,7 +224,8 @@ xpl_status xpl_free(xpl_ctx* ctx, const void* ptr);
  * runtime keeps using it for its next work (no cross-stream event for the next
  * epoch there).  Such a stream must stay valid until xpl_release_stream() names
  * it or xpl_finalize(); the legacy / per-thread default streams are never
- * adopted. */
+ * adopted.  Sharded mode: COLLECTIVE; end waits for this rank's epoch streams
+ * and for every rank (barrier) before the owner folds. */
 xpl_status xpl_kernel_begin(xpl_ctx* ctx, void* stream);
 xpl_status xpl_kernel_end(xpl_ctx* ctx, void* stream);
 
@@ -246,7 +250,9 @@ xpl_status xpl_record_host_ranges(xpl_ctx* ctx, const xpl_host_access* recs, siz
  * 1..3, size 0 or count 0. */
 xpl_status xpl_record_host_strided(xpl_ctx* ctx, const xpl_host_strided* recs, size_t n);
 
-/* The transfer wrappers (D7).  dst/src are the cudaMemcpy arguments. */
+/* The transfer wrappers (D7).  dst/src are the cudaMemcpy arguments.
+ * A range is clipped to the allocation holding its first byte (D18).  Sharded
+ * mode: COLLECTIVE; rank 0's call is the one recorded (D37). */
 xpl_status xpl_record_copy(xpl_ctx* ctx, const void* dst, const void* src, size_t bytes,
                            xpl_copy_dir dir);
 
@@ -256,7 +262,8 @@ xpl_status xpl_record_copy(xpl_ctx* ctx, const void* dst, const void* src, size_
  * reset != 0 the interval bits are cleared (the last writer is kept, D4) and
  * freed rows are dropped.  STATE inside an open epoch, or (like xpl_sync) after
  * a forbidden device-side split.  Blocks until done.
- * params NULL = defaults; names may be NULL when n_names == 0. */
+ * params NULL = defaults; names may be NULL when n_names == 0.  Sharded mode:
+ * COLLECTIVE; every rank gets the same reports (one per logical allocation). */
 xpl_status xpl_diagnose(xpl_ctx* ctx, const xpl_diag_params* params, const xpl_name* names,
                         size_t n_names, xpl_alloc_report* out, size_t cap, size_t* n_out,
                         int reset);
@@ -266,7 +273,8 @@ xpl_status xpl_diagnose(xpl_ctx* ctx, const xpl_diag_params* params, const xpl_n
  * logical words [word_offset, word_offset + ceil(bytes/4)) of the logical
  * allocation `logical_id` (logical size logical_bytes); its address range
  * [ptr, ptr+bytes) is registered like xpl_register_alloc.  Pieces of one logical
- * allocation must tile [0, ceil(logical_bytes/4)) exactly. */
+ * allocation must tile [0, ceil(logical_bytes/4)) exactly.  (Virtual shards of
+ * world-1 contexts; a sharded context cuts its pieces itself: STATE there.) */
 xpl_status xpl_register_alloc_piece(xpl_ctx* ctx, const void* ptr, size_t bytes,
                                     xpl_alloc_kind kind, uint64_t logical_id,
                                     uint64_t word_offset, uint64_t logical_bytes);
@@ -318,7 +326,8 @@ xpl_status xpl_get_device_ctx(xpl_ctx* ctx, struct xpl_dev_ctx* out);
 
 /* Per-word records of the live row whose base is `base`, words
  * [word0, word0+n), copied into the host array out[n] (access maps, Fig. 5/7/8/10;
- * also the sampled-parity hook of the tests).  Blocks until done. */
+ * also the sampled-parity hook of the tests).  Blocks until done.  Sharded mode:
+ * COLLECTIVE; `base` must be a piece this rank owns (INVALID_ARG otherwise). */
 xpl_status xpl_shadow_dump(xpl_ctx* ctx, const void* base, uint64_t word0, uint64_t n,
                            uint8_t* out);
 
@@ -359,7 +368,8 @@ typedef struct {
 /* The page view of every live row, in id order, into out[0..cap) (*n_out rows;
  * INVALID_ARG with *n_out = rows needed if cap is too small, or page_words == 0).
  * Reads the interval bits without changing them: call it before the resetting
- * diagnose of the interval.  STATE inside an open epoch.  Blocks until done. */
+ * diagnose of the interval.  STATE inside an open epoch, or in sharded mode.
+ * Blocks until done. */
 xpl_status xpl_page_summary(xpl_ctx* ctx, uint64_t page_words, xpl_page_report* out, size_t cap,
                             size_t* n_out);
 
@@ -424,7 +434,8 @@ xpl_status xpl_launch_log(xpl_ctx* ctx, xpl_launch_record* out, size_t cap, size
 const char* xpl_launch_name(xpl_ctx* ctx, uint32_t idx);
 
 /* Apply every staged host record now (normally done lazily at kernel_begin,
- * diagnose and when staging fills up).  Asynchronous. */
+ * diagnose and when staging fills up).  Asynchronous.  Sharded mode:
+ * COLLECTIVE (the records are routed to their owners). */
 xpl_status xpl_flush(xpl_ctx* ctx);
 /* Wait for all runtime work enqueued so far.  STATE if a device-side epoch split
  * (xpl_grid_epoch) ran in an epoch with several streams or with D2D / memset
