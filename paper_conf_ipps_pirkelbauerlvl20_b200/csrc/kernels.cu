@@ -82,7 +82,48 @@ __global__ void __launch_bounds__(kFoldThreads, 3) fold_kernel(uint32_t* __restr
   uint32_t folded = 0;
   for (uint64_t k0 = 0; w + k0 * W < n_super; k0 += 32) {
     const uint64_t sc = w + (k0 + lane) * W;
-    uint32_t ms = __ballot_sync(0xFFFFFFFFu, sc < n_super && smap[sc] != 0);
+    const bool marked = sc < n_super && smap[sc] != 0;
+    uint32_t ms = __ballot_sync(0xFFFFFFFFu, marked);
+    if (!ms) continue;
+    // Sparse super-chunks (<= 2 marked chunks: e.g. an anti-diagonal touches one
+    // word per row) are folded lane-per-super-chunk, all of the warp's at once:
+    // one 128 B read of the super's chunk bytes, then its one or two chunks.
+    bool dense = false;
+    if (marked) {
+      uint4 cm[8];
+      const uint4* cp = reinterpret_cast<const uint4*>(cmap + sc * 128);
+#pragma unroll
+      for (int k = 0; k < 8; ++k) cm[k] = cp[k];
+      uint32_t cnt = 0;  // (chunk bytes are 0 or 1)
+#pragma unroll
+      for (int k = 0; k < 8; ++k) cnt += __popc(cm[k].x) + __popc(cm[k].y) + __popc(cm[k].z) + __popc(cm[k].w);
+      dense = cnt > 2;
+      if (!dense) {
+        int ca = -1, cb = -1;
+#pragma unroll
+        for (int k = 0; k < 32; ++k) {
+          const uint32_t v = k % 4 == 0 ? cm[k / 4].x : k % 4 == 1 ? cm[k / 4].y : k % 4 == 2 ? cm[k / 4].z : cm[k / 4].w;
+          if (v) {
+            const int b0 = 4 * k + (__ffs(v) - 1) / 8;
+            const uint32_t rest = v & ~(0xFFu << (8 * ((__ffs(v) - 1) / 8)));
+            if (ca < 0) {
+              ca = b0;
+              if (rest) cb = 4 * k + (__ffs(rest) - 1) / 8;
+            } else if (cb < 0) {
+              cb = b0;
+            }
+          }
+        }
+        if (ca >= 0) {
+          fold_two(pool, sc * 128 + ca, true, sc * 128 + (cb >= 0 ? cb : ca), cb >= 0);
+          cmap[sc * 128 + ca] = 0;
+          if (cb >= 0) cmap[sc * 128 + cb] = 0;
+        }
+        folded += cnt;
+        smap[sc] = 0;
+      }
+    }
+    ms = __ballot_sync(0xFFFFFFFFu, marked && dense);
     while (ms) {
       const uint32_t j = __ffs(ms) - 1;
       ms &= ms - 1;
