@@ -13,6 +13,7 @@
 #   sanitize:TOOL          compute-sanitizer --tool TOOL (memcheck|synccheck|racecheck) over tools/sanitize_driver.py
 #   bench2[:ARGS]          2 ranks on this one GPU over gloo (the sharded N>1 bench path): torchrun bench.py --gpus 2
 #   golden5                cfg5's oracle expectations on the box's host cores (tools/golden_fullsize.py cfg5)
+#   hookab                 tools/hook_bench.py with libxplwork.so and with the A/B build libxplwork_ab.so
 TAG=$1; shift
 mkdir -p gpurun_out
 echo "nproc=$(nproc) $(nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv,noheader)" > gpurun_out/${TAG}_box.txt
@@ -48,6 +49,9 @@ for step in "$@"; do
              W=$(python -c "import os; m=os.sysconf('SC_PAGE_SIZE')*os.sysconf('SC_PHYS_PAGES')/2**30; print(max(1, min(os.cpu_count()-1, int(m//36))))")
              echo "workers=$W" > gpurun_out/golden5/box.txt; free -g >> gpurun_out/golden5/box.txt
              python tools/golden_fullsize.py cfg5 --workers $W --out gpurun_out/golden5 > gpurun_out/golden5/log.txt 2>&1 ;;
+    hookab) timeout 900 python tools/hook_bench.py --lulesh-steps 30 > gpurun_out/${TAG}_hook_a.json 2> gpurun_out/${TAG}_hook_a.err
+            XPL_WORK_PATH=paper_conf_ipps_pirkelbauerlvl20_b200/libxplwork_ab.so timeout 900 python tools/hook_bench.py \
+              --lulesh-steps 30 > gpurun_out/${TAG}_hook_b.json 2> gpurun_out/${TAG}_hook_b.err ;;
     *) echo "unknown step $step" >> gpurun_out/${TAG}_box.txt ;;
   esac
 done
