@@ -34,8 +34,12 @@
  *     super-chunk) in two byte maps with plain idempotent stores (test before
  *     store, no atomics), so closing the epoch costs O(chunks with P), not
  *     O(shadow).
- * A single-word access (the common case: an aligned scalar) takes a short path
- * with one ballot; multi-word accesses loop over the shadow u32s they cover.
+ * Paths: a compile-time-kind call site whose active lanes all access words
+ * inside one local shadow u32 (aligned scalars up to doubles) runs one
+ * straight-line warp-convergent sequence (xpld_record_fast); per-lane kinds
+ * and multi-u32 accesses take the general path (xpl_dev_apply), which loops
+ * over the shadow u32s an access covers; in sharded mode (xpl.h) words of
+ * another rank's pieces go to its peer-mapped pool (xpld_remote).
  * Device hooks never fail and never block.
  */
 #ifndef XPL_DEVICE_CUH
