@@ -45,6 +45,14 @@ SEED4 = 0x58504C05
 PARAMS = (50, 0, 256)  # threshold 50 %, whole-allocation blocks, min run 256 words (D16)
 WORKLOAD = "cfg4: LULESH-shaped 100^3 mesh x 100 timesteps (50 managed allocations + 2 temporaries/timestep, " \
            "19 instrumented launches/timestep, diagnose every timestep)"
+
+
+def workload(size, timesteps):
+    if size == S4 and timesteps == T4:
+        return WORKLOAD
+    name = "cfg5: " if size == 250 else ""
+    return (f"{name}LULESH-shaped {size}^3 mesh x {timesteps} timesteps (50 managed allocations + 2 "
+            "temporaries/timestep, 19 instrumented launches/timestep, diagnose every timestep)")
 METRIC = "recorded accesses/s (device hooks + host tracer) + diagnose GB/s; instrumented-kernel slowdown"
 # Distinct shadow words per epoch summed over one cfg4 timestep (tools/lulesh_words.py 100): the
 # unit count of the hook path's algorithmic bytes (1 B shadow read + <= 1 B written per word)
@@ -63,6 +71,8 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["xpl", "reference"], default="xpl")
     ap.add_argument("--timesteps", type=int, default=T4, help="cfg4 timesteps per step (default 100)")
+    ap.add_argument("--size", type=int, default=S4,
+                    help="LULESH mesh edge (default 100 = cfg4; 250 = cfg5, e.g. sharded: --gpus 8 --size 250)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-other-configs", action="store_true")
     ap.add_argument("--step-only", action="store_true",
@@ -322,13 +332,13 @@ def diag_at_scale(xpl, torch, words=1 << 31, reps=3):
 class Cfg4:
     """The cfg4 program's arrays, input and runs."""
 
-    def __init__(self, torch, apps, timesteps, rank=0, world=1):
+    def __init__(self, torch, apps, timesteps, rank=0, world=1, size=S4):
         from xplgen import lulesh as L
-        self.torch, self.apps, self.T = torch, apps, timesteps
+        self.torch, self.apps, self.T, self.S = torch, apps, timesteps, size
         self.rank, self.world = rank, world  # world > 1: the sharded program (this rank's slab)
-        self.spec = L.lulesh_spec(S4)
+        self.spec = L.lulesh_spec(size)
         self.ar = apps.Arena(self.spec)
-        self.topo = L.topology(S4, SEED4)
+        self.topo = L.topology(size, SEED4)
         self.host_topo = apps.lulesh_topology_host(self.topo)
         self.hc = torch.zeros(1, dtype=torch.int64, device="cuda")
         self.us = torch.cuda.Stream()
@@ -337,7 +347,7 @@ class Cfg4:
     def prepare(self, resident=True):
         self.hc.zero_()
         if resident:
-            self.apps.lulesh_prepare(self.ar, S4, self.topo)
+            self.apps.lulesh_prepare(self.ar, self.S, self.topo)
 
     def run(self, ctx, upload=False, time_kernels=False, params=PARAMS):
         """One step: the whole program.  upload: the topology H2D first (e2e)."""
@@ -345,7 +355,7 @@ class Cfg4:
             self.apps.lulesh_upload(self.ar, self.host_topo, self.us.cuda_stream)
         run = self.apps.Run(ctx, self.us.cuda_stream, params=params, out_cap=64 * (self.T + 2),
                             time_kernels=time_kernels, rank=self.rank, world=self.world)
-        self.apps.lulesh(run, self.ar, S4, self.T, self.hc)
+        self.apps.lulesh(run, self.ar, self.S, self.T, self.hc)
         return run
 
 
@@ -503,7 +513,8 @@ def other_configs(xpl, apps, torch, lulesh250_steps=100):
 
 def hook_roofline(args, hook_ms, k_instr, k_twin, ms_step, prof, peak, peak_src):
     hook_bytes = HOOK_BYTES_PER_WORD * CFG4_WORDS_PER_TIMESTEP
-    ach = hook_bytes / (hook_ms / 1e3) / 1e9 if hook_ms > 0 else None
+    # (the distinct-word count is the 100^3 mesh's; other sizes report the time only)
+    ach = hook_bytes / (hook_ms / 1e3) / 1e9 if hook_ms > 0 and args.size == S4 else None
     return {"kernel": "device hooks (a3), inlined in the 19 instrumented launches of each timestep",
             "bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s",
             "frac": (ach / peak) if ach else None, "traffic": None, "peak_source": peak_src,
@@ -526,8 +537,9 @@ def sharded_tail(args, torch, dist, apps, xpl, rank, world, value, ms_max, per_s
     program and checks every report (but `base`) is identical."""
     identical = None
     if rank == 0:
-        c1 = Cfg4(torch, apps, args.timesteps)
-        with xpl.Context(device=torch.cuda.current_device(), pool_words=1 << 28, max_rows=64) as ctx1:
+        c1 = Cfg4(torch, apps, args.timesteps, size=args.size)
+        pool = 1 << 28 if args.size <= S4 else 2_500_000_000
+        with xpl.Context(device=torch.cuda.current_device(), pool_words=pool, max_rows=64) as ctx1:
             c1.prepare()
             one = c1.run(ctx1).reports()
         # (ids continue across the context's runs, bases are each program's own)
@@ -552,7 +564,7 @@ def sharded_tail(args, torch, dist, apps, xpl, rank, world, value, ms_max, per_s
     line = {"metric": METRIC, "value": value, "unit": "accesses/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
-            "config": {"workload": WORKLOAD + f", sharded over {world} GPUs (one logical program: each rank "
+            "config": {"workload": workload(args.size, args.timesteps) + f", sharded over {world} GPUs (one logical program: each rank "
                                               "its slab of elements/nodes; shadow partitioned by word, host "
                                               "records routed all-to-all, remote hook atomics, partials combined)",
                        "timesteps": args.timesteps, "accesses_per_step": per_step, "epochs_per_step": epochs,
@@ -610,9 +622,10 @@ def main():
 
     # N > 1: the cfg4 program sharded over the ranks (each its slab; one logical
     # program, shadow partitioned by word over the GPUs, xpl.h sharded mode)
-    c4 = Cfg4(torch, apps, args.timesteps, rank, world)
+    c4 = Cfg4(torch, apps, args.timesteps, rank, world, args.size)
     comm = make_comm(xpl, torch, dist, rank, world, local, backend) if world > 1 else None
-    ctx = xpl.Context(device=local, pool_words=1 << 28, max_rows=256, comm=comm)
+    pool = 1 << 28 if args.size <= S4 else 2_500_000_000  # (cfg5: 2.3e9 shadow words per timestep)
+    ctx = xpl.Context(device=local, pool_words=pool, max_rows=256, comm=comm)
     flush_buf = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")  # > 126 MB L2
 
     clk = Clocks(local)
@@ -705,7 +718,8 @@ def main():
         "value": value, "unit": "accesses/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": ms_max / args.steps, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u8", "data": "synthetic",
-        "config": {"workload": WORKLOAD, "timesteps": args.timesteps, "accesses_per_step": per_step,
+        "config": {"workload": workload(args.size, args.timesteps), "timesteps": args.timesteps,
+                   "accesses_per_step": per_step,
                    "device_accesses": hooks, "host_accesses": host_acc, "epochs_per_step": epochs,
                    "diagnoses_per_step": n_diag,
                    "diag_params": {"threshold_pct": PARAMS[0], "block_words": PARAMS[1], "min_run": PARAMS[2]},
