@@ -229,8 +229,10 @@ def stream_microbench(xpl, torch, n=1 << 28, reps=5):
     """The hook path on a bandwidth-bound kernel with real data: y[i] = 2 x[i]
     over 1 GiB of 4-byte elements, every read traceR, every write traceW, in one
     epoch that first-touches every shadow word (the interval's REDs), against its
-    twin.  Algorithmic bytes = 8 B of data + 2 x 2 B of shadow per element (SURVEY
-    §8(d) a3: 1 B read + 1 B written per word on first touch); slowdown floor 1.5."""
+    twin -- with plain hooks (a row lookup per access) and through array handles
+    (the lookup hoisted out of the loop).  Algorithmic bytes = 8 B of data + 2 x 2 B
+    of shadow per element (1 B read + 1 B written per word on
+    first touch); slowdown floor 1.5."""
     peak, _ = peaks()
     st = torch.cuda.Stream()
     s = st.cuda_stream
@@ -244,34 +246,37 @@ def stream_microbench(xpl, torch, n=1 << 28, reps=5):
         e1.record(st)
         e1.synchronize()
         return e0.elapsed_time(e1)
-    twin = min(ev(lambda: xpl.stream_kernel(x.data_ptr(), y.data_ptr(), n, 4, False, s)) for _ in range(reps))
-    first, fold = [], []
+    twin = min(ev(lambda: xpl.stream_kernel(x.data_ptr(), y.data_ptr(), n, 4, 0, s)) for _ in range(reps))
+    data, shadow = 8 * n, 4 * n
+    out = {"n": n, "elem_bytes": 4, "twin_ms": twin, "slowdown_floor": (data + shadow) / data, "peak_gbs": peak,
+           "twin_gbs": data / (twin / 1e3) / 1e9}
     with xpl.Context(pool_words=2 * n + (1 << 20), max_rows=16) as ctx:
         ctx.register(x.data_ptr(), 4 * n, xpl.ALLOC_DEVICE)
         ctx.register(y.data_ptr(), 4 * n, xpl.ALLOC_DEVICE)
-        for _ in range(reps):
-            ctx.diagnose(*PARAMS, reset=True)  # a fresh interval: every shadow word is first-touched again
-            torch.cuda.synchronize()
-            ctx.kernel_begin(s)
-            e0, e1, e2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
-            e0.record(st)
-            xpl.stream_kernel(x.data_ptr(), y.data_ptr(), n, 4, True, s)
-            e1.record(st)
-            ctx.kernel_end(s)
-            ctx.join(s)
-            e2.record(st)
-            e2.synchronize()
-            first.append(e0.elapsed_time(e1))
-            fold.append(e1.elapsed_time(e2))
-    ms = min(first)
-    data, shadow = 8 * n, 4 * n
+        for mode, name in ((1, "plain"), (2, "handles")):
+            first, fold = [], []
+            for _ in range(reps):
+                ctx.diagnose(*PARAMS, reset=True)  # a fresh interval: every shadow word is first-touched again
+                torch.cuda.synchronize()
+                ctx.kernel_begin(s)
+                e0, e1, e2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+                e0.record(st)
+                xpl.stream_kernel(x.data_ptr(), y.data_ptr(), n, 4, mode, s)
+                e1.record(st)
+                ctx.kernel_end(s)
+                ctx.join(s)
+                e2.record(st)
+                e2.synchronize()
+                first.append(e0.elapsed_time(e1))
+                fold.append(e1.elapsed_time(e2))
+            ms = min(first)
+            out[name] = {"instr_ms": ms, "epoch_close_ms": min(fold), "slowdown": ms / twin,
+                         "achieved_gbs": (data + shadow) / (ms / 1e3) / 1e9,
+                         "frac": (data + shadow) / (ms / 1e3) / 1e9 / peak,
+                         "hooked_accesses_per_s": 2 * n / (ms / 1e3)}
     del x, y
     torch.cuda.empty_cache()
-    return {"n": n, "elem_bytes": 4, "twin_ms": twin, "instr_ms": ms, "epoch_close_ms": min(fold),
-            "slowdown": ms / twin, "slowdown_floor": (data + shadow) / data,
-            "achieved_gbs": (data + shadow) / (ms / 1e3) / 1e9, "peak_gbs": peak,
-            "frac": (data + shadow) / (ms / 1e3) / 1e9 / peak, "twin_gbs": data / (twin / 1e3) / 1e9,
-            "hooked_accesses_per_s": 2 * n / (ms / 1e3)}
+    return out
 
 
 def diag_at_scale(xpl, torch, words=1 << 31, reps=3):
@@ -747,8 +752,9 @@ def main():
         "diagnose_gbs": at_scale["reset"]["gbs"], "diagnose_frac": at_scale["reset"]["gbs"] / peak,
         "diagnose_gbs_no_reset": at_scale["no_reset"]["gbs"],
         "diagnose_gbs_in_step": (dg["bytes"] / (dg["ms"] / 1e3) / 1e9) if dg["ms"] else None,
-        "hook_frac_in_step": roof["frac"], "stream_hook_frac": smb["frac"],
-        "stream_slowdown": smb["slowdown"],
+        "hook_frac_in_step": roof["frac"], "stream_hook_frac": smb["plain"]["frac"],
+        "stream_slowdown": smb["plain"]["slowdown"], "stream_handles_slowdown": smb["handles"]["slowdown"],
+        "stream_handles_frac": smb["handles"]["frac"],
         "slowdown_whole_program": ms_total / twin_ms, "slowdown_kernels": k_instr / k_twin,
         "paper_slowdown_context": "Table III P:L431-443: 5x-20x, avg ~15x (Intel E5-2695 v4 + Pascal, CUDA 9.2)"}
     if rank == 0:

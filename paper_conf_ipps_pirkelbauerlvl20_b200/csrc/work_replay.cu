@@ -116,6 +116,37 @@ __global__ void __launch_bounds__(256) stream_kernel(const T* __restrict__ x, T*
   }
 }
 
+// The same streaming kernel through array handles (the lookups of x and y
+// hoisted out of the loop, as an instrumenting compiler would for a
+// loop-invariant base): same records.
+template <class T>
+__global__ void __launch_bounds__(256) stream_kernel_h(const T* __restrict__ x, T* __restrict__ y,
+                                                       unsigned long long n) {
+  const xpl_array<const T> hx(x);
+  const xpl_array<T> hy(y);
+  for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (unsigned long long)gridDim.x * blockDim.x) {
+    const T v = hx.read(i);
+    hy.write(i) = v + v;
+  }
+}
+
+struct T12 {  // a 12-byte element (3 words: handles of non-power-of-two sizes)
+  unsigned a, b, c;
+};
+
+// Accesses through one array handle made from `base` (addresses only): event i
+// is element idx[i] of the handle (any index, negative too: elements outside
+// the handle's row take the full lookup), with kind K.  The handle's parity test.
+template <class T, unsigned K>
+__global__ void handle_replay_kernel(unsigned long long base, const long long* __restrict__ idx,
+                                     unsigned long long n) {
+  const xpl_array<T> h(reinterpret_cast<T*>(base));
+  for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (unsigned long long)gridDim.x * blockDim.x)
+    h.template rec<K>((unsigned long long)idx[i]);
+}
+
 // A user kernel that really touches memory (managed memory for the UM-counter
 // check, NEXT-4): word k*stride of base for k < n/stride is read (write = 0) or
 // incremented (write = 1: read then write, hooked as RW), hooks on.
@@ -173,12 +204,18 @@ int xplw_touch_mem(void* base, unsigned long long n_words, unsigned long long st
   return cudaGetLastError() == cudaSuccess ? 0 : (int)XPL_ERR_CUDA;
 }
 
-// Launch the streaming kernel: elem = 4 or 8 bytes, instrumented (between
-// xpl_kernel_begin/_end) or the twin; one wave of 148 x 8 CTAs, grid-stride.
+// Launch the streaming kernel: elem = 4 or 8 bytes, instrumented (1: traceR /
+// traceW per element, 2: through array handles; between xpl_kernel_begin/_end)
+// or the twin (0); one wave of 148 x 8 CTAs, grid-stride.
 int xplw_stream(const void* x, void* y, unsigned long long n, int elem, int instrumented, void* stream) {
   cudaStream_t s = (cudaStream_t)stream;
   const unsigned g = 148 * 8;
-  if (elem == 4) {
+  if (instrumented == 2) {  // through array handles
+    if (elem == 4) stream_kernel_h<unsigned><<<g, 256, 0, s>>>((const unsigned*)x, (unsigned*)y, n);
+    else if (elem == 8)
+      stream_kernel_h<unsigned long long><<<g, 256, 0, s>>>((const unsigned long long*)x, (unsigned long long*)y, n);
+    else return (int)XPL_ERR_INVALID_ARG;
+  } else if (elem == 4) {
     if (instrumented) stream_kernel<unsigned, true><<<g, 256, 0, s>>>((const unsigned*)x, (unsigned*)y, n);
     else stream_kernel<unsigned, false><<<g, 256, 0, s>>>((const unsigned*)x, (unsigned*)y, n);
   } else if (elem == 8) {
@@ -189,6 +226,26 @@ int xplw_stream(const void* x, void* y, unsigned long long n, int elem, int inst
   } else {
     return (int)XPL_ERR_INVALID_ARG;
   }
+  return cudaGetLastError() == cudaSuccess ? 0 : (int)XPL_ERR_CUDA;
+}
+
+// Launch the handle replay: elem = 4, 8 or 12 bytes, kind = 1 R, 2 W, 3 RW.
+int xplw_handle_replay(unsigned long long base, int elem, const long long* d_idx, unsigned long long n,
+                       int kind, int grid, int block, void* stream) {
+  if (n == 0) return 0;
+  cudaStream_t s = (cudaStream_t)stream;
+#define XPLW_HR(T)                                                                                     \
+  switch (kind) {                                                                                     \
+    case 1: handle_replay_kernel<T, XPL_ACC_R><<<grid, block, 0, s>>>(base, d_idx, n); break;        \
+    case 2: handle_replay_kernel<T, XPL_ACC_W><<<grid, block, 0, s>>>(base, d_idx, n); break;        \
+    case 3: handle_replay_kernel<T, XPL_ACC_RW><<<grid, block, 0, s>>>(base, d_idx, n); break;       \
+    default: return (int)XPL_ERR_INVALID_ARG;                                                         \
+  }
+  if (elem == 4) { XPLW_HR(unsigned) }
+  else if (elem == 8) { XPLW_HR(unsigned long long) }
+  else if (elem == 12) { XPLW_HR(T12) }
+  else return (int)XPL_ERR_INVALID_ARG;
+#undef XPLW_HR
   return cudaGetLastError() == cudaSuccess ? 0 : (int)XPL_ERR_CUDA;
 }
 

@@ -194,6 +194,7 @@ if _work is not None:
     xplw_touch = _sig("xplw_touch", [u64, u64, u32, vp, u64], lib=_work)
     xplw_stream = _sig("xplw_stream", [vp, vp, u64, i32, i32, vp], lib=_work)
     xplw_replay_k = _sig("xplw_replay_k", [vp, vp, u64, i32, i32, i32, vp], lib=_work)
+    xplw_handle_replay = _sig("xplw_handle_replay", [u64, i32, vp, u64, i32, i32, i32, vp], lib=_work)
     # (optional so that A/B builds of the workload library without it still load)
     xplw_read_lat = (_sig("xplw_read_lat", [vp, u64, i32, i32, i32, vp], lib=_work)
                      if hasattr(_work, "xplw_read_lat") else None)
@@ -514,10 +515,19 @@ class Context:
         check("xplw_replay_split", xplw_replay_split(d_addr, d_size, d_acc, d_seg, nseg, grid, block, stream))
 
 
+def handle_replay(base, elem, d_idx, n, kind, grid=0, block=256, stream=0):
+    """Accesses through one array handle of `elem`-byte elements made from `base`:
+    element d_idx[i] (int64, any sign) with kind 1 R / 2 W / 3 RW (libxplwork)."""
+    if grid <= 0:
+        grid = max(1, min((n + block - 1) // block, 148 * 8))
+    check("xplw_handle_replay", xplw_handle_replay(base, elem, d_idx, n, kind, grid, block, stream))
+
+
 def stream_kernel(x_ptr, y_ptr, n, elem, instrumented, stream=0):
     """y[i] = 2 x[i] over n elements of `elem` bytes (4 or 8): the instrumented
-    streaming kernel (inside an epoch) or its twin (libxplwork.so)."""
-    check("xplw_stream", xplw_stream(x_ptr, y_ptr, n, elem, int(bool(instrumented)), stream))
+    streaming kernel (inside an epoch; instrumented = 1 plain hooks, 2 array
+    handles) or its twin (0) (libxplwork.so)."""
+    check("xplw_stream", xplw_stream(x_ptr, y_ptr, n, elem, int(instrumented), stream))
 
 
 def atomic_bench(buf_ptr, n_u32, mode, stream=0):

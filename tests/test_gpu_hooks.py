@@ -120,8 +120,9 @@ def test_random_traces_uniform_kind_launches(gpu, seed):
     compare(replay.run_trace(ops, uniform=True, grid=2, block=160, seed=seed), exp, "uniform shuffled")
 
 
+@pytest.mark.parametrize("mode", [1, 2])  # plain hooks / array handles
 @pytest.mark.parametrize("elem,n", [(4, 1000003), (8, 777777), (4, 31), (8, 1)])
-def test_stream_kernel(gpu, elem, n):
+def test_stream_kernel(gpu, elem, n, mode):
     torch, replay, xpl = gpu
     x = torch.arange(n * elem // 4, dtype=torch.int32, device="cuda")
     y = torch.zeros_like(x)
@@ -134,11 +135,11 @@ def test_stream_kernel(gpu, elem, n):
         got = []
         for rep in range(2):  # second epoch: every bit already set (re-touch)
             ctx.kernel_begin(s)
-            xpl.stream_kernel(xa, ya, n, elem, True, s)
+            xpl.stream_kernel(xa, ya, n, elem, mode, s)
             ctx.kernel_end(s)
         got.append(ctx.diagnose(50, 0, 256, reset=True))
         ctx.kernel_begin(s)
-        xpl.stream_kernel(xa, ya, n, elem, True, s)
+        xpl.stream_kernel(xa, ya, n, elem, mode, s)
         ctx.kernel_end(s)
         got.append(ctx.diagnose(50, 0, 256, reset=True))
     torch.cuda.synchronize()
@@ -151,3 +152,43 @@ def test_stream_kernel(gpu, elem, n):
            ("KB",), ev, ("KE",), ("KB",), ev, ("KE",), ("DIAG", 50, 0, 256, 1, ()),
            ("KB",), ev, ("KE",), ("DIAG", 50, 0, 256, 1, ())]
     compare(got, oracle_run(ops), "stream")
+
+
+@pytest.mark.parametrize("elem", [4, 8, 12])
+@pytest.mark.parametrize("shift", [0, 4, 2])
+def test_array_handles(gpu, elem, shift):
+    """xpl_array handles (the hoisted lookup): a handle made `shift` bytes into
+    an allocation (word-aligned or not), elements inside the row, past its end
+    (into the next allocation and into untracked memory), before its start
+    (negative indices) and straddling the row end -- each event recorded exactly
+    as the same access through xpl_read / xpl_write / xpl_rw."""
+    torch, replay, xpl = gpu
+    rng = np.random.default_rng(elem * 10 + shift)
+    a, b = 0x6000_0000, 0x6000_0000 + 4 * 1003 + 2  # b starts right after a's last (partial) word
+    na, nb = 4 * 1003 + 2, 4 * 500
+    base = a + shift
+    nel = (na - shift) // elem
+    ops = [("REG", a, na, MANAGED), ("REG", b, nb, MANAGED)]
+    with xpl.Context(pool_words=1 << 20) as ctx:
+        ctx.register(a, na, MANAGED)
+        ctx.register(b, nb, MANAGED)
+        s = torch.cuda.current_stream().cuda_stream
+        got = []
+        for ep in range(4):
+            idx = np.concatenate([np.arange(nel), rng.integers(-50, nel + 300, size=3000),
+                                  np.array([nel, nel - 1, -1, nel + 200])]).astype(np.int64)
+            if ep % 2:
+                idx = rng.permutation(idx)
+            kind = [1, 2, 3, 1][ep]
+            d = torch.from_numpy(idx).cuda()
+            ctx.kernel_begin(s)
+            xpl.handle_replay(base, elem, d.data_ptr(), idx.size, kind, stream=s)
+            ctx.kernel_end(s)
+            torch.cuda.synchronize()
+            addrs = (base + elem * idx).astype(np.uint64)
+            ops += [("KB",), ("DB", addrs, np.full(idx.size, elem, np.uint32), np.full(idx.size, kind, np.uint8)),
+                    ("KE",)]
+            if ep % 2:
+                got.append(ctx.diagnose(50, 0, 16, reset=True))
+                ops.append(("DIAG", 50, 0, 16, 1, ()))
+    compare(got, oracle_run(ops), "handles")
