@@ -231,7 +231,7 @@ static __device__ __noinline__ void xpld_remote(unsigned owner, unsigned long lo
         const unsigned grp = __match_any_sync(needers, ((unsigned long long)owner << 40) | q);
         const unsigned bits = __reduce_or_sync(grp, m);
         if (xpld_lane() == (unsigned)(__ffs(grp) - 1)) {
-          atomicOr(P + q, bits);
+          atomicOr_system(P + q, bits); /* (system scope: another GPU's memory over NVLink) */
           if (bits & XPLD_P4) {
             unsigned char* c = xpl_dctx.cmaps[owner] + (q >> 5);
             unsigned char* sm = xpl_dctx.smaps[owner] + (q >> 12);
