@@ -27,24 +27,39 @@ __device__ __forceinline__ T& WR(T& x) {
   else return x;
 }
 
+// H through an array handle (its row lookup hoisted out of the cell's four
+// accesses, as an instrumenting compiler would); the twin gets the pointer.
 template <bool I>
-__device__ __forceinline__ void sw_cell(const int* a, const int* b, int* H, int ld, int i, int j) {
+struct HArr : xpl_array<int> {
+  __device__ __forceinline__ explicit HArr(int* q) : xpl_array<int>(q) {}
+};
+template <>
+struct HArr<false> {
+  int* p;
+  __device__ __forceinline__ explicit HArr(int* q) : p(q) {}
+  __device__ __forceinline__ const int& read(long long i) const { return p[i]; }
+  __device__ __forceinline__ int& write(long long i) const { return p[i]; }
+};
+
+template <bool I>
+__device__ __forceinline__ void sw_cell(const int* a, const int* b, const HArr<I>& H, int ld, int i, int j) {
   const int s = RD<I>(a[i - 1]) == RD<I>(b[j - 1]) ? kMatch : kMismatch;
-  const int d = RD<I>(H[(i - 1) * ld + j - 1]) + s;
-  const int u = RD<I>(H[(i - 1) * ld + j]) - kGap;
-  const int l = RD<I>(H[i * ld + j - 1]) - kGap;
+  const int d = H.read((long long)(i - 1) * ld + j - 1) + s;
+  const int u = H.read((long long)(i - 1) * ld + j) - kGap;
+  const int l = H.read((long long)i * ld + j - 1) - kGap;
   int h = d > u ? d : u;
   h = h > l ? h : l;
-  WR<I>(H[i * ld + j]) = h > 0 ? h : 0;
+  H.write((long long)i * ld + j) = h > 0 ? h : 0;
 }
 
 // cfg1: one CTA, thread t owns row i = t + 1, sweeping the anti-diagonals.
 template <bool I>
 __global__ void sw_wavefront(const int* a, const int* b, int* H, int n, int m) {
   const int ld = m + 1, i = threadIdx.x + 1;
+  const HArr<I> Hh(H);
   for (int d = 2; d <= n + m; ++d) {
     const int j = d - i;
-    if (i <= n && j >= 1 && j <= m) sw_cell<I>(a, b, H, ld, i, j);
+    if (i <= n && j >= 1 && j <= m) sw_cell<I>(a, b, Hh, ld, i, j);
     __syncthreads();
   }
 }
@@ -56,9 +71,10 @@ __global__ void sw_wavefront(const int* a, const int* b, int* H, int n, int m) {
 template <bool I>
 __global__ void sw_wavefront_split(const int* a, const int* b, int* H, int n, int m) {
   const int ld = m + 1, i = threadIdx.x + 1;
+  const HArr<I> Hh(H);
   for (int d = 2; d <= n + m; ++d) {
     const int j = d - i;
-    if (i <= n && j >= 1 && j <= m) sw_cell<I>(a, b, H, ld, i, j);
+    if (i <= n && j >= 1 && j <= m) sw_cell<I>(a, b, Hh, ld, i, j);
     if constexpr (I) {
       if (d < n + m) xpl_grid_epoch();  // (the last diagonal's epoch closes at xpl_kernel_end)
     } else {
@@ -74,7 +90,8 @@ __global__ void __launch_bounds__(256) sw_diagonal(const int* a, const int* b, i
   const int i = max(1, d - m) + blockIdx.x * blockDim.x + threadIdx.x;
   const int j = d - i;
   if (i > n || j < 1) return;
-  sw_cell<I>(a, b, H, m + 1, i, j);
+  const HArr<I> Hh(H);
+  sw_cell<I>(a, b, Hh, m + 1, i, j);
 }
 
 template <bool I>
