@@ -200,6 +200,7 @@ def main():
     ap.add_argument("--workers", type=int, default=3)
     ap.add_argument("--part", type=int, default=-1)
     ap.add_argument("--no-merge", action="store_true")
+    ap.add_argument("--only", default="", help="cfg5: comma-separated part names to run (default: all missing)")
     a = ap.parse_args()
     if a.cfg in ("cfg5", "cfg5-part"):
         from xplgen import lulesh as L
@@ -215,7 +216,9 @@ def main():
             cfg5_part(name, slots, tmp, os.path.join(pdir, name + ".json"))
             return
         import subprocess
-        todo = [i for i, j in enumerate(jobs) if not os.path.exists(os.path.join(pdir, j[0] + ".json"))]
+        only = set(filter(None, a.only.split(",")))
+        todo = [i for i, j in enumerate(jobs) if not os.path.exists(os.path.join(pdir, j[0] + ".json"))
+                and (not only or j[0] in only)]
         todo.sort(key=lambda i: -(sum(L.slot_bytes(250, k) for k in jobs[i][1]) + (1 << 40 if jobs[i][2] else 0)))
         running = []
         while todo or running:
