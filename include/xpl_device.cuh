@@ -107,7 +107,9 @@ static __device__ __forceinline__ unsigned xpld_lane() {
 /* Mark the chunk (and super-chunk) of shadow u32 q as holding a pending GPU
  * write: plain idempotent byte stores, tested first (a stale cached 0 only
  * costs a redundant store).  Both bytes are loaded before either store, so
- * the two loads overlap.  Only first writes of a shadow u32 get here. */
+ * the two loads overlap.  Only first writes of a shadow u32 get here.  The
+ * first mark of a super-chunk also raises flags[2] ("the epoch close has
+ * work"), so the close of an epoch that set no pending write ends at once. */
 template <bool TESTED = true>
 static __device__ __forceinline__ void xpld_mark(unsigned q) {
   unsigned char* c = xpl_dctx.cmap + (q >> 5);
@@ -115,10 +117,14 @@ static __device__ __forceinline__ void xpld_mark(unsigned q) {
   if (TESTED) {
     const unsigned cv = *c, sv = *s;
     if (!cv) *c = 1;
-    if (!sv) *s = 1;
+    if (!sv) {
+      *s = 1;
+      xpl_dctx.flags[2] = 1u;
+    }
   } else {  /* latency variant: plain stores, nothing to wait for */
     *c = 1;
     *s = 1;
+    xpl_dctx.flags[2] = 1u;
   }
 }
 

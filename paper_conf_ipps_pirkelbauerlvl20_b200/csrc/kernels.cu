@@ -65,17 +65,9 @@ __device__ __forceinline__ void fold_two(uint32_t* pool, uint64_t ch0, bool m0, 
   }
 }
 
-__global__ void __launch_bounds__(kFoldThreads, 3) fold_kernel(uint32_t* __restrict__ pool,
-                                                            uint8_t* __restrict__ cmap,
-                                                            uint8_t* __restrict__ smap,
-                                                            uint64_t n_super,
-                                                            unsigned long long* stats,
-                                                            uint32_t* flags, int strict) {
-  asm volatile("griddepcontrol.wait;" ::: "memory");
-  if (blockIdx.x == 0 && threadIdx.x == 0) {  // a device-side split in an epoch that forbids it
-    if (strict && flags[0]) flags[1] = 1u;
-    flags[0] = 0u;
-  }
+__device__ __forceinline__ void fold_body(uint32_t* __restrict__ pool, uint8_t* __restrict__ cmap,
+                                          uint8_t* __restrict__ smap, uint64_t n_super,
+                                          unsigned long long* stats) {
   const uint32_t lane = threadIdx.x & 31;
   const uint64_t W = (uint64_t)gridDim.x * (kFoldThreads / 32);
   const uint64_t w = (uint64_t)blockIdx.x * (kFoldThreads / 32) + (threadIdx.x >> 5);
@@ -142,6 +134,33 @@ __global__ void __launch_bounds__(kFoldThreads, 3) fold_kernel(uint32_t* __restr
   }
   folded = __reduce_add_sync(0xFFFFFFFFu, folded);
   if (lane == 0 && folded) atomicAdd(stats + 3, (unsigned long long)folded);
+}
+
+__global__ void __launch_bounds__(kFoldThreads, 3) fold_kernel(uint32_t* __restrict__ pool,
+                                                            uint8_t* __restrict__ cmap,
+                                                            uint8_t* __restrict__ smap,
+                                                            uint64_t n_super,
+                                                            unsigned long long* stats,
+                                                            uint32_t* flags, int strict, int force) {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  if (blockIdx.x == 0 && threadIdx.x == 0) {  // a device-side split in an epoch that forbids it
+    if (strict && flags[0]) flags[1] = 1u;
+    flags[0] = 0u;
+  }
+  // flags[2]: some pending write was marked since the last close (hooks, range
+  // kernel); without one the close has nothing to fold.  The last CTA to finish
+  // clears it (flags[3] counts the finished CTAs).  (A sharded epoch's remote
+  // writers mark another rank's maps: there flags[2] is not used, force = 1.)
+  const bool work = force || *reinterpret_cast<volatile uint32_t*>(flags + 2) != 0;
+  __syncthreads();  // (every thread read the flag before any CTA can clear it below)
+  if (work) fold_body(pool, cmap, smap, n_super, stats);
+  if (threadIdx.x == 0) {
+    __threadfence();
+    if (atomicAdd(flags + 3, 1u) == gridDim.x - 1) {
+      flags[2] = 0u;
+      flags[3] = 0u;
+    }
+  }
 }
 
 // ---------------------------------------------------------------------------
@@ -258,7 +277,7 @@ __device__ __forceinline__ uint32_t cpu_range_op(uint32_t v, uint32_t bm, uint32
 
 __global__ void __launch_bounds__(256) range_kernel(const RangeDesc* __restrict__ rd, uint32_t nr,
                                                     uint64_t nvec, uint32_t* pool,
-                                                    uint8_t* cmap, uint8_t* smap) {
+                                                    uint8_t* cmap, uint8_t* smap, uint32_t* flags) {
   for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < nvec;
        v += (uint64_t)gridDim.x * blockDim.x) {
     uint32_t lo = 0, hi = nr;  // last range with vbase <= v
@@ -323,7 +342,10 @@ __global__ void __launch_bounds__(256) range_kernel(const RangeDesc* __restrict_
         atomicOr(pool + q, m);
         if (m & kP4) {
           if (!cmap[q >> 5]) cmap[q >> 5] = 1;
-          if (!smap[q >> 12]) smap[q >> 12] = 1;
+          if (!smap[q >> 12]) {
+            smap[q >> 12] = 1;
+            flags[2] = 1u;
+          }
         }
       }
     }
@@ -1185,7 +1207,7 @@ __global__ void __launch_bounds__(256) page_kernel(const PageRow* __restrict__ r
 }  // namespace
 
 void launch_fold(cudaStream_t s, bool pdl, uint32_t* pool, uint8_t* cmap, uint8_t* smap,
-                 uint64_t n_super, unsigned long long* stats, uint32_t* flags, int strict) {
+                 uint64_t n_super, unsigned long long* stats, uint32_t* flags, int strict, int force) {
   cudaLaunchConfig_t cfg = {};
   const uint64_t ctas = (n_super + 7) / 8;  // (one warp per super-chunk at most)
   cfg.gridDim = dim3((unsigned)(ctas == 0 ? 1 : ctas < XPL_FOLD_CTAS ? ctas : XPL_FOLD_CTAS));  // one wave
@@ -1196,7 +1218,7 @@ void launch_fold(cudaStream_t s, bool pdl, uint32_t* pool, uint8_t* cmap, uint8_
   at[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = at;
   cfg.numAttrs = pdl ? 1 : 0;
-  cudaLaunchKernelEx(&cfg, fold_kernel, pool, cmap, smap, n_super, stats, flags, strict);
+  cudaLaunchKernelEx(&cfg, fold_kernel, pool, cmap, smap, n_super, stats, flags, strict, force);
 }
 
 void launch_merge(cudaStream_t s, const uint64_t* recs, uint32_t n, bool has_r, bool has_w,
@@ -1213,9 +1235,9 @@ void launch_merge(cudaStream_t s, const uint64_t* recs, uint32_t n, bool has_r, 
 }
 
 void launch_range(cudaStream_t s, const RangeDesc* d_ranges, uint32_t nr, uint64_t nvec,
-                  uint32_t* pool, uint8_t* cmap, uint8_t* smap) {
+                  uint32_t* pool, uint8_t* cmap, uint8_t* smap, uint32_t* flags) {
   const int g = grid_for(nvec, 256, 148 * 8);
-  range_kernel<<<g, 256, 0, s>>>(d_ranges, nr, nvec, pool, cmap, smap);
+  range_kernel<<<g, 256, 0, s>>>(d_ranges, nr, nvec, pool, cmap, smap, flags);
 }
 
 void launch_diag(cudaStream_t s, const DiagRow* rows, uint32_t nrows, const uint32_t* tile_row,

@@ -552,7 +552,7 @@ xpl_status flush_local(xpl_ctx* c) {
         for (size_t i = sg.start; i < sg.start + sg.n; ++i) rw += c->h_ranges[i].nw;
         const int pi = prof_begin(c, XPL_K_RANGE, 2 * rw);
         launch_range(c->cs, c->d_ranges + sg.start, (uint32_t)sg.n, nvec, (uint32_t*)c->d_pool,
-                     c->d_cmap, c->d_smap);
+                     c->d_cmap, c->d_smap, c->d_misc);
         prof_end(c, pi);
         c->st.kernel_launches += 1;
         c->st.range_segments++;
@@ -627,7 +627,7 @@ xpl_status gpu_ranges(xpl_ctx* c, const RangeDesc* rd, size_t nr) {
   uint64_t rw = 0;
   for (size_t i = 0; i < nr; ++i) rw += rd[i].nw;
   const int pi = prof_begin(c, XPL_K_RANGE, 2 * rw);
-  launch_range(c->cs, c->d_ranges, (uint32_t)nr, v, (uint32_t*)c->d_pool, c->d_cmap, c->d_smap);
+  launch_range(c->cs, c->d_ranges, (uint32_t)nr, v, (uint32_t*)c->d_pool, c->d_cmap, c->d_smap, c->d_misc);
   if (c->depth) c->cs_in_epoch = true;
   c->st.kernel_launches += 1;
   prof_end(c, pi);
@@ -638,11 +638,15 @@ xpl_status gpu_ranges(xpl_ctx* c, const RangeDesc* rd, size_t nr) {
 // epoch's kernels on the same stream (programmatic stream serialization).
 // strict = the epoch had several streams or runtime range work of its own, so a
 // device-side split (xpl_grid_epoch) inside it is an error (its fold would race).
+// The fold skips its scan when no pending write was marked since the last close
+// (d_misc[2], raised by the hooks and the range kernel); in sharded mode other
+// ranks' writers mark this rank's maps without raising it, so the scan is forced.
 void fold(xpl_ctx* c, bool pdl, bool strict = false) {
   const int pi = prof_begin(c, XPL_K_FOLD, 0);
   // only super-chunks below the pool's high-water mark can be flagged
   launch_fold(c->cs, pdl && pi < 0, (uint32_t*)c->d_pool, c->d_cmap, c->d_smap,
-              (c->pas[c->rank].hwm + 16383) / 16384, c->d_stats, c->d_misc, strict ? 1 : 0);
+              (c->pas[c->rank].hwm + 16383) / 16384, c->d_stats, c->d_misc, strict ? 1 : 0,
+              c->world > 1 ? 1 : 0);
   c->folds_host++;
   c->st.kernel_launches += 1;
   prof_end(c, pi);

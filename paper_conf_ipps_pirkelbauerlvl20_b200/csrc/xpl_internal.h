@@ -98,11 +98,11 @@ struct DiagParams {
 
 // ---- launchers (kernels.cu) ----
 void launch_fold(cudaStream_t s, bool pdl, uint32_t* pool, uint8_t* cmap, uint8_t* smap,
-                 uint64_t n_super, unsigned long long* stats, uint32_t* flags, int strict);
+                 uint64_t n_super, unsigned long long* stats, uint32_t* flags, int strict, int force);
 void launch_merge(cudaStream_t s, const uint64_t* recs, uint32_t n, bool has_r, bool has_w,
                   uint32_t* first_w, uint64_t fw0, uint32_t* pool);
 void launch_range(cudaStream_t s, const RangeDesc* d_ranges, uint32_t nr, uint64_t nvec,
-                  uint32_t* pool, uint8_t* cmap, uint8_t* smap);
+                  uint32_t* pool, uint8_t* cmap, uint8_t* smap, uint32_t* flags);
 void launch_diag(cudaStream_t s, const DiagRow* rows, uint32_t nrows, const uint32_t* tile_row,
                  uint64_t ntiles, const StitchSeg* segs, uint32_t nseg, uint64_t nblocks,
                  const DiagParams& p, uint32_t* pool, unsigned long long* cnt, TileSum* tiles,
