@@ -459,10 +459,26 @@ static __device__ __forceinline__ void xpld_record_fast(unsigned long long g0, u
     xpld_put<K, TM>(q, cur, (K & XPL_ACC_R) ? gb : 0u, (K & XPL_ACC_W) ? gb : 0u);
 }
 
+/* A hooked read's own data load is issued after the hook (the hook returns the
+ * reference the caller loads through), so its latency would add to the hook's
+ * shadow load.  A prefetch of the data line at the start of the hook overlaps
+ * the two (the caller's load then hits L1).  A/B switch: XPL_HOOK_PREFETCH=0. */
+#ifndef XPL_HOOK_PREFETCH
+#define XPL_HOOK_PREFETCH 1
+#endif
+static __device__ __forceinline__ void xpld_prefetch(const void* p) {
+#if XPL_HOOK_PREFETCH
+  asm volatile("prefetch.L1 [%0];" ::"l"(p));
+#else
+  (void)p;
+#endif
+}
+
 template <unsigned K, bool TM = true>
 static __device__ __forceinline__ void xpl_dev_record_k(const void* p, unsigned size,
                                                         unsigned acc) {
 #ifndef XPL_OFF
+  if (K & XPL_ACC_R) xpld_prefetch(p);
   const unsigned long long a = (unsigned long long)p;
   ulonglong2 be, ow;
   unsigned long long g0 = 1, g1 = 0;
@@ -521,9 +537,26 @@ struct xpl_array {
     (void)i;
 #endif
   }
-  __device__ __forceinline__ const T& read(unsigned long long i) const { rec<XPL_ACC_R>(i); return p[i]; }
+  /* read: the element is loaded before the hook runs, so the data load and the
+   * hook's shadow load are in flight together (the value is returned) */
+  __device__ __forceinline__ T read(unsigned long long i) const {
+#if XPL_HOOK_PREFETCH
+    const T v = p[i];
+    rec<XPL_ACC_R>(i);
+    return v;
+#else
+    rec<XPL_ACC_R>(i);
+    return p[i];
+#endif
+  }
   __device__ __forceinline__ T& write(unsigned long long i) const { rec<XPL_ACC_W>(i); return p[i]; }
-  __device__ __forceinline__ T& rw(unsigned long long i) const { rec<XPL_ACC_RW>(i); return p[i]; }
+  __device__ __forceinline__ T& rw(unsigned long long i) const {
+#ifndef XPL_OFF
+    xpld_prefetch(p + i);
+#endif
+    rec<XPL_ACC_RW>(i);
+    return p[i];
+  }
 };
 
 /* Generic form: acc may differ from lane to lane. */

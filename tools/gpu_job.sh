@@ -10,6 +10,7 @@
 #   launches               ncu launch list (gpu__time_duration.sum) of a short bench run
 #   ncu:REGEX[:SKIP[:CMD]] ncu --set full of one launch of kernel REGEX (default command: bench.py --step-only)
 #   py:SCRIPT[:ARGS]       python SCRIPT ARGS > TAG_<name>.json
+#   pyab:SCRIPT[:ARGS]     the same with the A/B build libxplwork_ab.so > TAG_<name>_ab.json
 #   sanitize:TOOL          compute-sanitizer --tool TOOL (memcheck|synccheck|racecheck) over tools/sanitize_driver.py
 #   bench2[:ARGS]          2 ranks on this one GPU over gloo (the sharded N>1 bench path): torchrun bench.py --gpus 2
 #   golden5                cfg5's oracle expectations on the box's host cores (tools/golden_fullsize.py cfg5)
@@ -40,6 +41,10 @@ for step in "$@"; do
     py) script=${rest%%:*}; a2=${rest#*:}; [ "$a2" = "$rest" ] && a2=""
         name=$(basename "$script" .py)
         timeout 1800 python $script ${a2//+/ } > gpurun_out/${TAG}_$name.json 2> gpurun_out/${TAG}_$name.err ;;
+    pyab) script=${rest%%:*}; a2=${rest#*:}; [ "$a2" = "$rest" ] && a2=""
+          name=$(basename "$script" .py)
+          XPL_WORK_PATH=paper_conf_ipps_pirkelbauerlvl20_b200/libxplwork_ab.so timeout 1800 python $script ${a2//+/ } \
+            > gpurun_out/${TAG}_${name}_ab.json 2> gpurun_out/${TAG}_${name}_ab.err ;;
     sanitize) timeout 1500 compute-sanitizer --tool $rest --print-limit 50 python tools/sanitize_driver.py \
                 > gpurun_out/${TAG}_sanitize_$rest.log 2>&1; echo "rc=$?" >> gpurun_out/${TAG}_sanitize_$rest.log ;;
     bench2) XPL_DIST_BACKEND=gloo timeout 1800 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 \

@@ -48,11 +48,11 @@ def main():
             best = t if best is None else min(best, t)
         return best
 
-    for elem in (4, 8):
+    for elem, mode in ((4, 1), (8, 1), (4, 2), (8, 2)):  # mode 1: xpl_read/xpl_write, 2: array handles
         n = a.n if elem == 4 else a.n // 2
         x = torch.ones(n * elem // 4, dtype=torch.int32, device="cuda")
         y = torch.empty_like(x)
-        twin = ev_time(lambda: xpl.stream_kernel(x.data_ptr(), y.data_ptr(), n, elem, False, s), a.reps)
+        twin = ev_time(lambda: xpl.stream_kernel(x.data_ptr(), y.data_ptr(), n, elem, 0, s), a.reps)
         words = n * elem // 4
         with xpl.Context(pool_words=2 * words + (1 << 20), max_rows=16) as ctx:
             ctx.register(x.data_ptr(), n * elem, xpl.ALLOC_DEVICE)
@@ -64,7 +64,7 @@ def main():
                 ctx.kernel_begin(s)
                 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 e0.record(st)
-                xpl.stream_kernel(x.data_ptr(), y.data_ptr(), n, elem, True, s)
+                xpl.stream_kernel(x.data_ptr(), y.data_ptr(), n, elem, mode, s)
                 e1.record(st)
                 ctx.kernel_end(s)
                 ctx.join(s)
@@ -82,7 +82,7 @@ def main():
             torch.cuda.synchronize()
         data = 2 * n * elem
         shadow = 2 * 2 * words  # two arrays, 1 B read + 1 B written per word
-        out[f"stream{elem * 8}"] = {
+        out[f"stream{elem * 8}" + ("_handles" if mode == 2 else "")] = {
             "n": n, "elem_bytes": elem, "twin_ms": twin, "instr_ms_first_touch": ms_first,
             "instr_ms_retouch": ms_again,
             "slowdown_first": ms_first / twin, "slowdown_retouch": ms_again / twin,
