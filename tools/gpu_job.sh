@@ -50,10 +50,14 @@ for step in "$@"; do
     bench2) XPL_DIST_BACKEND=gloo timeout 1800 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 \
               --master-addr 127.0.0.1 --master-port 29533 bench.py --gpus 2 $args \
               > gpurun_out/${TAG}_bench2.json 2> gpurun_out/${TAG}_bench2.err ;;
-    golden5) mkdir -p gpurun_out/golden5
-             W=$(python -c "import os; m=os.sysconf('SC_PAGE_SIZE')*os.sysconf('SC_PHYS_PAGES')/2**30; print(max(1, min(os.cpu_count()-1, int(m//36))))")
+    golden5) mkdir -p gpurun_out/golden5/cfg5_parts
+             # (a part peaks near 30 GB of host memory: 40 GB of MemAvailable per worker)
+             W=$(python -c "import os; m=int(open('/proc/meminfo').read().split('MemAvailable:')[1].split()[0])/2**20; print(max(1, min(os.cpu_count()-1, int(m//40))))")
              echo "workers=$W" > gpurun_out/golden5/box.txt; free -g >> gpurun_out/golden5/box.txt
-             python tools/golden_fullsize.py cfg5 --workers $W --out gpurun_out/golden5 > gpurun_out/golden5/log.txt 2>&1 ;;
+             cp tests/golden/fullsize/cfg5_parts/*.json gpurun_out/golden5/cfg5_parts/ 2>/dev/null
+             timeout ${GOLDEN5_TIMEOUT:-5400} python tools/golden_fullsize.py cfg5 --workers $W --out gpurun_out/golden5 \
+               ${GOLDEN5_ONLY:+--only $GOLDEN5_ONLY --no-merge} > gpurun_out/golden5/log.txt 2>&1
+             echo "rc=$?" >> gpurun_out/golden5/log.txt ;;
     hookab) timeout 900 python tools/hook_bench.py --lulesh-steps 30 > gpurun_out/${TAG}_hook_a.json 2> gpurun_out/${TAG}_hook_a.err
             XPL_WORK_PATH=paper_conf_ipps_pirkelbauerlvl20_b200/libxplwork_ab.so timeout 900 python tools/hook_bench.py \
               --lulesh-steps 30 > gpurun_out/${TAG}_hook_b.json 2> gpurun_out/${TAG}_hook_b.err ;;
