@@ -109,22 +109,27 @@ static __device__ __forceinline__ unsigned xpld_lane() {
  * costs a redundant store).  Both bytes are loaded before either store, so
  * the two loads overlap.  Only first writes of a shadow u32 get here.  The
  * first mark of a super-chunk also raises flags[2] ("the epoch close has
- * work"), so the close of an epoch that set no pending write ends at once. */
+ * work"), so the close of an epoch that set no pending write ends at once.
+ * flags[2] is one word every marking lane of the grid would store to (a
+ * scattered writer, e.g. a wavefront's cells in 16K different rows, marks a
+ * new super-chunk per lane): it is tested first (its line stays in L1), so
+ * about one store per SM reaches L2 instead of one per lane; the latency
+ * variant raises it with a RED (no wait, combined at L2). */
 template <bool TESTED = true>
 static __device__ __forceinline__ void xpld_mark(unsigned q) {
   unsigned char* c = xpl_dctx.cmap + (q >> 5);
   unsigned char* s = xpl_dctx.smap + (q >> 12);
   if (TESTED) {
-    const unsigned cv = *c, sv = *s;
+    const unsigned cv = *c, sv = *s, fv = xpl_dctx.flags[2];
     if (!cv) *c = 1;
     if (!sv) {
       *s = 1;
-      xpl_dctx.flags[2] = 1u;
+      if (!fv) xpl_dctx.flags[2] = 1u;
     }
   } else {  /* latency variant: plain stores, nothing to wait for */
     *c = 1;
     *s = 1;
-    xpl_dctx.flags[2] = 1u;
+    atomicOr(xpl_dctx.flags + 2, 1u);
   }
 }
 

@@ -779,13 +779,30 @@ __device__ __forceinline__ void tile_loop(TileAcc& A, WarpRing& R, uint4* p4, ui
 // the uniform-step counts.  Runs: ballot fast paths for all-zero/all-one
 // 512-word steps, warp_runs() for mixed ones.  Reset fused.  The tile's counts
 // and run summaries go to tiles[t]; the stitch adds and combines them in order.
+// The stitch fused into the tile kernel (no block counts: p.block_words == 0):
+// the warp that finishes the last tile of a segment combines the segment, the
+// one that finishes its row's last segment combines the row and writes its
+// report (last-block-done: release fence + done counter, which that warp
+// resets to 0 for the next call).  Null seg_done = the separate stitch kernels.
+struct FusedStitch {
+  uint32_t* seg_done;               // per segment: tiles done
+  uint32_t* row_done;               // per row: segments done
+  void* segsum;                     // RunPair per segment
+  unsigned long long* segcnt;       // 9 counters per segment
+  unsigned long long* cnt;          // C_NCNT counters per row (partials)
+  xpl_alloc_report* out;
+  RowPartial* parts;
+};
+__device__ __noinline__ void fused_stitch(const DiagRow& row, uint32_t ri, uint64_t t, const DiagParams& p,
+                                          const TileSum* tiles, const FusedStitch& fs, uint32_t lane);
+
 #ifndef XPL_DIAG_MINB
 #define XPL_DIAG_MINB 4  // CTAs per SM the register budget is sized for (A/B: profiles/r1h_diag_variants.txt)
 #endif
 __global__ void __launch_bounds__(kDiagThreads, XPL_DIAG_MINB) diag_tile_kernel(
-    const DiagRow* __restrict__ rows, const uint32_t* __restrict__ tile_row, uint64_t ntiles,
+    const DiagRow* __restrict__ rows, uint32_t nrows, const uint32_t* __restrict__ tile_row, uint64_t ntiles,
     DiagParams p, uint32_t* __restrict__ pool, TileSum* __restrict__ tiles,
-    uint32_t* __restrict__ blk_cnt) {
+    uint32_t* __restrict__ blk_cnt, FusedStitch fs) {
   constexpr uint32_t kWarps = kDiagThreads / 32;
   __shared__ uint32_t s_uc[kWarps][9];
   extern __shared__ __align__(128) unsigned char s_dyn[];
@@ -798,7 +815,18 @@ __global__ void __launch_bounds__(kDiagThreads, XPL_DIAG_MINB) diag_tile_kernel(
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncwarp();
-  const uint32_t ri = tile_row[t];
+  uint32_t ri;
+  if (tile_row) {
+    ri = tile_row[t];
+  } else {  // the last row with tile0 <= t (rows in tile order, none empty)
+    uint32_t lo = 0, hi = nrows;
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (__ldg(&rows[mid].tile0) <= t) lo = mid;
+      else hi = mid;
+    }
+    ri = lo;
+  }
   const DiagRow row = rows[ri];
   const uint32_t tw = p.tile_words;
   const uint64_t ww0 = (t - row.tile0) * tw;  // row word
@@ -846,6 +874,7 @@ __global__ void __launch_bounds__(kDiagThreads, XPL_DIAG_MINB) diag_tile_kernel(
     ts->u = A.wu;
     ts->d = A.wd;
   }
+  if (fs.seg_done) fused_stitch(row, ri, t, p, tiles, fs, lane);
 }
 
 __device__ __forceinline__ void run_final(const RunSum64& s, uint64_t min_run, uint64_t* runs,
@@ -918,28 +947,11 @@ __global__ void stitch_seg_kernel(const StitchSeg* __restrict__ segs, uint32_t n
   }
 }
 
-// Stitch, level 2 + finalize: one warp per row combines its segment summaries,
-// then lane 0 turns the counters into the report row (flags P:L84-114, D8).
-__global__ void stitch_row_finalize_kernel(const DiagRow* __restrict__ rows, uint32_t nrows,
-                                           const RunPair* __restrict__ segsum, DiagParams p,
-                                           unsigned long long* __restrict__ cnt,
-                                           xpl_alloc_report* __restrict__ out,
-                                           RowPartial* __restrict__ parts,
-                                           const uint32_t* __restrict__ blk_cnt) {
-  const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const uint32_t lane = threadIdx.x & 31;
-  if (gw >= nrows) return;
-  const DiagRow r = rows[gw];
-  const uint64_t per = (r.nseg + 31) / 32;
-  const uint64_t s0 = r.seg0 + lane * per;
-  const uint64_t s1 = min(r.seg0 + r.nseg, s0 + per);
-  RunSum64 a = {0, 0, 0, 0, 0}, b = {0, 0, 0, 0, 0};
-  for (uint64_t s = s0; s < s1; ++s) {
-    a = rs_combine(a, segsum[s].u, p.min_run);
-    b = rs_combine(b, segsum[s].d, p.min_run);
-  }
-  warp_combine(a, b, lane, p.min_run);
-  if (lane != 0) return;
+// One report row from the row's combined run summaries and counters c (D8).
+__device__ __forceinline__ void row_finalize(const DiagRow& r, uint32_t gw, const RunSum64& a, const RunSum64& b,
+                                             const unsigned long long* c, const DiagParams& p,
+                                             xpl_alloc_report* __restrict__ out, RowPartial* __restrict__ parts,
+                                             const uint32_t* __restrict__ blk_cnt) {
   if (parts) {
     RowPartial& q = parts[gw];
     q.u[0] = a.len; q.u[1] = a.pre; q.u[2] = a.suf; q.u[3] = a.cnt; q.u[4] = a.sum;
@@ -947,7 +959,6 @@ __global__ void stitch_row_finalize_kernel(const DiagRow* __restrict__ rows, uin
     q.blk_first_g = (p.block_words && r.nblk) ? blk_cnt[r.blk0] : 0;
     q.blk_last_g = (p.block_words && r.nblk) ? blk_cnt[r.blk0 + r.nblk - 1] : 0;
   }
-  const unsigned long long* c = cnt + (uint64_t)gw * C_NCNT;
   xpl_alloc_report o;
   o.id = o.base = o.bytes = 0;
   o.words = r.words;
@@ -989,6 +1000,118 @@ __global__ void stitch_row_finalize_kernel(const DiagRow* __restrict__ rows, uin
   if (o.any_acc == 0) f |= XPL_PAT_UNUSED;
   o.flags = f;
   out[gw] = o;
+}
+
+// Stitch, level 2 + finalize: one warp per row combines its segment summaries,
+// then lane 0 turns the counters into the report row (flags P:L84-114, D8).
+__global__ void stitch_row_finalize_kernel(const DiagRow* __restrict__ rows, uint32_t nrows,
+                                           const RunPair* __restrict__ segsum, DiagParams p,
+                                           unsigned long long* __restrict__ cnt,
+                                           xpl_alloc_report* __restrict__ out,
+                                           RowPartial* __restrict__ parts,
+                                           const uint32_t* __restrict__ blk_cnt) {
+  const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint32_t lane = threadIdx.x & 31;
+  if (gw >= nrows) return;
+  const DiagRow r = rows[gw];
+  const uint64_t per = (r.nseg + 31) / 32;
+  const uint64_t s0 = r.seg0 + lane * per;
+  const uint64_t s1 = min(r.seg0 + r.nseg, s0 + per);
+  RunSum64 a = {0, 0, 0, 0, 0}, b = {0, 0, 0, 0, 0};
+  for (uint64_t s = s0; s < s1; ++s) {
+    a = rs_combine(a, segsum[s].u, p.min_run);
+    b = rs_combine(b, segsum[s].d, p.min_run);
+  }
+  warp_combine(a, b, lane, p.min_run);
+  if (lane == 0) row_finalize(r, gw, a, b, cnt + (uint64_t)gw * C_NCNT, p, out, parts, blk_cnt);
+}
+
+__device__ __forceinline__ RunSum64 rs64(const RunSum& u) { return RunSum64{u.len, u.pre, u.suf, u.cnt, u.sum}; }
+
+__device__ __noinline__ void fused_stitch(const DiagRow& row, uint32_t ri, uint64_t t, const DiagParams& p,
+                                          const TileSum* tiles, const FusedStitch& fs, uint32_t lane) {
+  const uint64_t k = (t - row.tile0) / kSegTiles;  // the tile's segment within its row
+  const uint64_t seg = row.seg0 + k;
+  const uint64_t st0 = row.tile0 + k * kSegTiles;
+  const uint32_t sn = (uint32_t)min(kSegTiles, row.ntiles - k * kSegTiles);
+  __threadfence();  // (release: this lane's TileSum stores before the count)
+  __syncwarp();
+  uint32_t last = 0;
+  if (lane == 0) last = atomicAdd(fs.seg_done + seg, 1u) == sn - 1;
+  if (!__shfl_sync(0xFFFFFFFFu, last, 0)) return;
+  __threadfence();  // (acquire: the segment's other TileSums)
+  // level 1: the segment's tiles in order (lanes take contiguous sub-ranges)
+  RunSum64 a = {0, 0, 0, 0, 0}, b = {0, 0, 0, 0, 0};
+  uint64_t c9[9] = {0, 0, 0, 0, 0, 0, 0, 0, 0};
+  {
+    const uint32_t per = (sn + 31) / 32;
+    const uint64_t t0 = st0 + lane * per, t1 = min(st0 + sn, t0 + per);
+    for (uint64_t u = t0; u < t1; ++u) {
+      const TileSum* ts = tiles + u;
+      RunSum uu, dd;
+      uu.len = __ldcg(&ts->u.len); uu.pre = __ldcg(&ts->u.pre); uu.suf = __ldcg(&ts->u.suf);
+      uu.cnt = __ldcg(&ts->u.cnt); uu.sum = __ldcg(&ts->u.sum);
+      dd.len = __ldcg(&ts->d.len); dd.pre = __ldcg(&ts->d.pre); dd.suf = __ldcg(&ts->d.suf);
+      dd.cnt = __ldcg(&ts->d.cnt); dd.sum = __ldcg(&ts->d.sum);
+      a = rs_combine(a, rs64(uu), p.min_run);
+      b = rs_combine(b, rs64(dd), p.min_run);
+#pragma unroll
+      for (int j = 0; j < 9; ++j) c9[j] += __ldcg(&ts->cnt[j]);
+    }
+  }
+  warp_combine(a, b, lane, p.min_run);
+#pragma unroll
+  for (int j = 0; j < 9; ++j)
+    for (uint32_t o = 16; o; o >>= 1) c9[j] += __shfl_down_sync(0xFFFFFFFFu, c9[j], o);
+  if (row.nseg == 1) {  // (the common case at small sizes: the segment is the row)
+    if (lane == 0) {
+      fs.seg_done[seg] = 0;
+      unsigned long long* c = fs.cnt + (uint64_t)ri * C_NCNT;
+      for (int j = 0; j < 9; ++j) c[j] = c9[j];
+      for (int j = 9; j < (int)C_NCNT; ++j) c[j] = 0;
+      row_finalize(row, ri, a, b, c, p, fs.out, fs.parts, nullptr);
+    }
+    return;
+  }
+  RunPair* const ss = reinterpret_cast<RunPair*>(fs.segsum);
+  if (lane == 0) {
+    ss[seg] = RunPair{a, b};
+    for (int j = 0; j < 9; ++j) fs.segcnt[seg * 9 + j] = c9[j];
+    fs.seg_done[seg] = 0;
+    __threadfence();
+    last = atomicAdd(fs.row_done + ri, 1u) == row.nseg - 1;
+  }
+  if (!__shfl_sync(0xFFFFFFFFu, last, 0)) return;
+  __threadfence();
+  // level 2: the row's segments in order
+  a = RunSum64{0, 0, 0, 0, 0};
+  b = RunSum64{0, 0, 0, 0, 0};
+#pragma unroll
+  for (int j = 0; j < 9; ++j) c9[j] = 0;
+  {
+    const uint64_t per = (row.nseg + 31) / 32;
+    const uint64_t s0 = row.seg0 + lane * per, s1 = min(row.seg0 + row.nseg, s0 + per);
+    for (uint64_t u = s0; u < s1; ++u) {
+      const uint64_t* q = reinterpret_cast<const uint64_t*>(ss + u);
+      const RunSum64 x = {__ldcg(q + 0), __ldcg(q + 1), __ldcg(q + 2), __ldcg(q + 3), __ldcg(q + 4)};
+      const RunSum64 y = {__ldcg(q + 5), __ldcg(q + 6), __ldcg(q + 7), __ldcg(q + 8), __ldcg(q + 9)};
+      a = rs_combine(a, x, p.min_run);
+      b = rs_combine(b, y, p.min_run);
+#pragma unroll
+      for (int j = 0; j < 9; ++j) c9[j] += __ldcg(fs.segcnt + u * 9 + j);
+    }
+  }
+  warp_combine(a, b, lane, p.min_run);
+#pragma unroll
+  for (int j = 0; j < 9; ++j)
+    for (uint32_t o = 16; o; o >>= 1) c9[j] += __shfl_down_sync(0xFFFFFFFFu, c9[j], o);
+  if (lane == 0) {
+    fs.row_done[ri] = 0;
+    unsigned long long* c = fs.cnt + (uint64_t)ri * C_NCNT;
+    for (int j = 0; j < 9; ++j) c[j] = c9[j];
+    for (int j = 9; j < (int)C_NCNT; ++j) c[j] = 0;
+    row_finalize(row, ri, a, b, c, p, fs.out, fs.parts, nullptr);
+  }
 }
 
 // Low-density blocks (Eq. P:L102, D11-D13): block flagged iff it has
@@ -1244,17 +1367,25 @@ void launch_diag(cudaStream_t s, const DiagRow* rows, uint32_t nrows, const uint
                  uint64_t ntiles, const StitchSeg* segs, uint32_t nseg, uint64_t nblocks,
                  const DiagParams& p, uint32_t* pool, unsigned long long* cnt, TileSum* tiles,
                  void* segsum, uint32_t* blk_cnt, xpl_alloc_report* out, RowPartial* parts,
-                 cudaEvent_t tile_ev0, cudaEvent_t tile_ev1) {
-  cudaMemsetAsync(cnt, 0, sizeof(unsigned long long) * C_NCNT * nrows, s);
-  if (p.block_words && nblocks) cudaMemsetAsync(blk_cnt, 0, sizeof(uint32_t) * nblocks, s);
+                 cudaEvent_t tile_ev0, cudaEvent_t tile_ev1, uint32_t* done, unsigned long long* segcnt) {
+  // fused: one launch (the stitch in the tile kernel's last warps); block
+  // counts (p.block_words) need the whole tile pass first: separate kernels
+  const bool fused = done != nullptr && p.block_words == 0;
+  FusedStitch fs = {};
+  if (fused) fs = FusedStitch{done, done + nseg, segsum, segcnt, cnt, out, parts};
+  if (!fused) {
+    cudaMemsetAsync(cnt, 0, sizeof(unsigned long long) * C_NCNT * nrows, s);
+    if (p.block_words && nblocks) cudaMemsetAsync(blk_cnt, 0, sizeof(uint32_t) * nblocks, s);
+  }
   if (tile_ev0) cudaEventRecord(tile_ev0, s);
   constexpr uint32_t kWarps = kDiagThreads / 32;
   // (per device; cheap next to a diagnose)
   cudaFuncSetAttribute(diag_tile_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kDiagSmem);
   if (ntiles)
     diag_tile_kernel<<<(unsigned)((ntiles + kWarps - 1) / kWarps), kDiagThreads, kDiagSmem, s>>>(
-        rows, tile_row, ntiles, p, pool, tiles, blk_cnt);
+        rows, nrows, fused ? nullptr : tile_row, ntiles, p, pool, tiles, blk_cnt, fs);
   if (tile_ev1) cudaEventRecord(tile_ev1, s);
+  if (fused) return;
   if (p.block_words && nblocks)
     block_eval_kernel<<<grid_for(nblocks, 256, 148 * 8), 256, 0, s>>>(rows, nrows, nblocks, blk_cnt,
                                                                     p.block_words, p.thr, cnt);

@@ -182,7 +182,10 @@ struct xpl_ctx {
   StitchSeg* h_segs = nullptr;
   StitchSeg* d_segs = nullptr;
   void* d_segsum = nullptr;
+  unsigned long long* d_segcnt = nullptr;  // fused stitch: 9 counters per segment
   size_t segs_cap = 0;
+  uint32_t* d_done = nullptr;  // fused stitch: segment + row done counters (kept zero)
+  size_t done_cap = 0;
   unsigned long long* d_cnt = nullptr;
   xpl_alloc_report* d_rep = nullptr;
   xpl_alloc_report* h_rep = nullptr;
@@ -1046,6 +1049,8 @@ xpl_status xpl_finalize(xpl_ctx* c) {
   cudaFreeHost(c->h_segs);
   cudaFree(c->d_segs);
   cudaFree(c->d_segsum);
+  cudaFree(c->d_segcnt);
+  cudaFree(c->d_done);
   cudaFree(c->d_cnt);
   cudaFree(c->d_rep);
   cudaFreeHost(c->h_rep);
@@ -1727,15 +1732,29 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
     cudaFreeHost(c->h_segs);
     cudaFree(c->d_segs);
     cudaFree(c->d_segsum);
+    cudaFree(c->d_segcnt);
     c->segs_cap = std::max<uint64_t>(nseg, 1024);
     CK(host_alloc(&c->h_segs, c->segs_cap));
     CK(cudaMalloc(&c->d_segs, sizeof(StitchSeg) * c->segs_cap));
     CK(cudaMalloc(&c->d_segsum, kRunPairBytes * c->segs_cap));
+    CK(cudaMalloc(&c->d_segcnt, sizeof(unsigned long long) * 9 * c->segs_cap));
   }
   if (nblocks > c->blk_cap) {
     cudaFree(c->d_blk);
     c->blk_cap = std::max<uint64_t>(nblocks, 1024);
     CK(cudaMalloc(&c->d_blk, sizeof(uint32_t) * c->blk_cap));
+  }
+  // fused stitch (one launch): no block counts, no empty row
+  bool fused = B == 0 && getenv("XPL_DIAG_UNFUSED") == nullptr;
+  for (uint64_t id : ids) fused = fused && c->rows[id].words > 0;
+  if (fused && nseg + nr > c->done_cap) {
+    if (c->d_done) {
+      CK(cudaStreamSynchronize(c->cs));
+      cudaFree(c->d_done);
+    }
+    c->done_cap = std::max<size_t>(nseg + nr, 4096);
+    CK(cudaMalloc(&c->d_done, sizeof(uint32_t) * c->done_cap));
+    CK(cudaMemsetAsync(c->d_done, 0, sizeof(uint32_t) * c->done_cap, c->cs));
   }
   uint64_t t = 0, b = 0, sgi = 0;
   for (size_t i = 0; i < nr; ++i) {
@@ -1753,29 +1772,33 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
     d.pad = 0;
     d.seg0 = sgi;
     d.nseg = (d.ntiles + kSegTiles - 1) / kSegTiles;
-    for (uint64_t k = 0; k < d.nseg; ++k) {
-      c->h_segs[sgi + k].t0 = t + k * kSegTiles;
-      c->h_segs[sgi + k].n = std::min<uint64_t>(kSegTiles, d.ntiles - k * kSegTiles);
-      c->h_segs[sgi + k].row = i;
+    if (!fused) {  // (the fused kernel finds a tile's row and segment itself)
+      for (uint64_t k = 0; k < d.nseg; ++k) {
+        c->h_segs[sgi + k].t0 = t + k * kSegTiles;
+        c->h_segs[sgi + k].n = std::min<uint64_t>(kSegTiles, d.ntiles - k * kSegTiles);
+        c->h_segs[sgi + k].row = i;
+      }
+      for (uint64_t k = 0; k < d.ntiles; ++k) c->h_tile_row[t + k] = (uint32_t)i;
     }
     sgi += d.nseg;
-    for (uint64_t k = 0; k < d.ntiles; ++k) c->h_tile_row[t + k] = (uint32_t)i;
     t += d.ntiles;
     b += d.nblk;
   }
   CK(cudaMemcpyAsync(c->d_drows, c->h_drows, sizeof(DiagRow) * nr, cudaMemcpyHostToDevice, c->cs));
-  CK(cudaMemcpyAsync(c->d_tile_row, c->h_tile_row, sizeof(uint32_t) * ntiles,
-                     cudaMemcpyHostToDevice, c->cs));
-  CK(cudaMemcpyAsync(c->d_segs, c->h_segs, sizeof(StitchSeg) * nseg, cudaMemcpyHostToDevice, c->cs));
+  if (!fused) {
+    CK(cudaMemcpyAsync(c->d_tile_row, c->h_tile_row, sizeof(uint32_t) * ntiles,
+                       cudaMemcpyHostToDevice, c->cs));
+    CK(cudaMemcpyAsync(c->d_segs, c->h_segs, sizeof(StitchSeg) * nseg, cudaMemcpyHostToDevice, c->cs));
+  }
   const uint64_t dbytes = total_words * (reset ? 2 : 1);
   const int pall = prof_begin(c, XPL_K_DIAGNOSE, dbytes);
   const int ptile = prof_begin(c, XPL_K_DIAG_TILE, dbytes, false);  // recorded by launch_diag
   launch_diag(c->cs, c->d_drows, (uint32_t)nr, c->d_tile_row, ntiles, c->d_segs, (uint32_t)nseg,
               nblocks, p, (uint32_t*)c->d_pool, c->d_cnt, c->d_tiles, c->d_segsum, c->d_blk, c->d_rep,
               pout ? c->d_rpart : nullptr, ptile >= 0 ? c->prof_pending[ptile].a : nullptr,
-              ptile >= 0 ? c->prof_pending[ptile].b : nullptr);
+              ptile >= 0 ? c->prof_pending[ptile].b : nullptr, fused ? c->d_done : nullptr, c->d_segcnt);
   CK(cudaGetLastError());
-  c->st.kernel_launches += 3 + (B && nblocks ? 1 : 0);
+  c->st.kernel_launches += fused ? 1 : 3 + (B && nblocks ? 1 : 0);
   CK(cudaMemcpyAsync(c->h_rep, c->d_rep, sizeof(xpl_alloc_report) * nr, cudaMemcpyDeviceToHost, c->cs));
   if (pout) {
     CK(cudaMemcpyAsync(c->h_rpart, c->d_rpart, sizeof(RowPartial) * nr, cudaMemcpyDeviceToHost, c->cs));

@@ -107,7 +107,9 @@ void launch_diag(cudaStream_t s, const DiagRow* rows, uint32_t nrows, const uint
                  uint64_t ntiles, const StitchSeg* segs, uint32_t nseg, uint64_t nblocks,
                  const DiagParams& p, uint32_t* pool, unsigned long long* cnt, TileSum* tiles,
                  void* segsum, uint32_t* blk_cnt, xpl_alloc_report* out, RowPartial* parts,
-                 cudaEvent_t tile_ev0, cudaEvent_t tile_ev1);
+                 cudaEvent_t tile_ev0, cudaEvent_t tile_ev1, uint32_t* done, unsigned long long* segcnt);
+// done: nseg + nrows zero u32s (segment / row done counters, left zero), or null
+// for the separate stitch kernels; segcnt: 9 u64 per segment.
 constexpr size_t kRunPairBytes = 80;  // sizeof(RunPair) in kernels.cu
 struct PageRow {  // one live row of a page pass (NEXT-3)
   uint64_t off, words, page0;  // pool word offset, words, first global page index

@@ -328,15 +328,69 @@ def test_uniform_stretches(gpu, seed):
     compare(replay.run_trace(ops, pool_words=1 << 22), oracle_run(ops), "stretches")
 
 
-@pytest.mark.parametrize("tile", ["2048", "4096", "16384"])
+@pytest.mark.parametrize("tile", ["2048", "4096", "16384", "2048u"])
 def test_tile_size_invariance(gpu, tile, monkeypatch):
     """The diagnose kernel's tile size (chosen per call from the call's size) must
     not change any report: the stretch and multi-tile traces under a forced tile
     size equal the oracle (which has no tiles)."""
     replay, _ = gpu
+    if tile.endswith("u"):  # the separate stitch kernels (not fused into the tile kernel)
+        tile = tile[:-1]
+        monkeypatch.setenv("XPL_DIAG_UNFUSED", "1")
     monkeypatch.setenv("XPL_DIAG_TILE_WORDS", tile)
     for ops in (stretch_trace(0x58504C50), big_trace(0x58504C51)):
         compare(replay.run_trace(ops, pool_words=1 << 24), oracle_run(ops), f"tile={tile}")
+
+
+def long_row_trace(seed, words=(5_000_003, 700_001, 3)):
+    """Rows of hundreds to thousands of tiles (the diagnose stitch's two levels:
+    segments of 128 tiles, then the row), sparse scattered GPU events, host
+    ranges and transfers cut at random words, runs crossing tile and segment
+    boundaries; three diagnose parameter sets, with and without reset."""
+    rng = np.random.default_rng(seed)
+    ops, allocs = [], []
+    b = 0x4000_0000
+    for i, w in enumerate(words):
+        ops.append(("REG", b, 4 * w - (i % 2), (MANAGED, DEVICE, MANAGED)[i]))
+        allocs.append((b, w))
+        b += ((4 * w + 65535) // 65536 + 1) * 65536
+    for rnd in range(3):
+        for base, w in allocs:
+            s = int(rng.integers(0, w))
+            e = min(w, s + int(rng.integers(1, 1 << 21)))
+            ops.append(("X", 0, base + 4 * s, 0x7000_0000, 4 * (e - s)))  # H2D of a stretch
+        ops.append(("KB",))
+        for base, w in allocs:
+            n = int(min(w, 60_000))
+            a = base + 4 * np.sort(rng.integers(0, w, size=n)).astype(np.uint64)
+            ops.append(("DB", a, np.full(n, 4, np.uint32), rng.integers(1, 4, size=n).astype(np.uint8)))
+        ops.append(("KE",))
+        base, w = allocs[rnd % len(allocs)]
+        s = int(rng.integers(0, w))
+        ops.append(("X", 1, 0x7000_0000, base + 4 * s, 4 * min(w - s, 300_000)))  # D2H
+        for params, reset in (((50, 0, 256), 0), ((50, 0, 1), rnd % 2), ((10, 0, 70_000), 0)):
+            ops.append(("DIAG", *params, reset, ()))
+    return ops
+
+
+_EXPECTED = {}
+
+
+@pytest.mark.parametrize("mode", ["fused", "unfused"])
+@pytest.mark.parametrize("tile", ["2048", "16384"])
+def test_diag_long_rows(gpu, mode, tile, monkeypatch):
+    """The diagnose stitch over rows of up to 2442 tiles (20 segments): the fused
+    one-launch path (last-warp-done segment and row combines inside the tile
+    kernel) and the separate stitch kernels (XPL_DIAG_UNFUSED) both equal the
+    oracle, under two forced tile sizes."""
+    replay, _ = gpu
+    monkeypatch.setenv("XPL_DIAG_TILE_WORDS", tile)
+    if mode == "unfused":
+        monkeypatch.setenv("XPL_DIAG_UNFUSED", "1")
+    ops = long_row_trace(0x58504C60)
+    if "long_row" not in _EXPECTED:  # (the oracle takes ~10 s here: once per module)
+        _EXPECTED["long_row"] = oracle_run(ops)
+    compare(replay.run_trace(ops, pool_words=1 << 23), _EXPECTED["long_row"], f"{mode} tile={tile}")
 
 
 @pytest.mark.parametrize("seed", range(6))
