@@ -792,6 +792,8 @@ struct FusedStitch {
   unsigned long long* cnt;          // C_NCNT counters per row (partials)
   xpl_alloc_report* out;
   RowPartial* parts;
+  const uint32_t* flags_in;         // d_misc[0..1], copied to flags_out by row 0's finalizer
+  uint32_t* flags_out;
 };
 __device__ __noinline__ void fused_stitch(const DiagRow& row, uint32_t ri, uint64_t t, const DiagParams& p,
                                           const TileSum* tiles, const FusedStitch& fs, uint32_t lane);
@@ -1026,6 +1028,12 @@ __global__ void stitch_row_finalize_kernel(const DiagRow* __restrict__ rows, uin
   if (lane == 0) row_finalize(r, gw, a, b, cnt + (uint64_t)gw * C_NCNT, p, out, parts, blk_cnt);
 }
 
+__device__ __forceinline__ void fused_flags(const FusedStitch& fs) {
+  if (!fs.flags_out) return;
+  fs.flags_out[0] = *reinterpret_cast<const volatile uint32_t*>(fs.flags_in);
+  fs.flags_out[1] = *reinterpret_cast<const volatile uint32_t*>(fs.flags_in + 1);
+}
+
 __device__ __forceinline__ RunSum64 rs64(const RunSum& u) { return RunSum64{u.len, u.pre, u.suf, u.cnt, u.sum}; }
 
 __device__ __noinline__ void fused_stitch(const DiagRow& row, uint32_t ri, uint64_t t, const DiagParams& p,
@@ -1070,6 +1078,7 @@ __device__ __noinline__ void fused_stitch(const DiagRow& row, uint32_t ri, uint6
       for (int j = 0; j < 9; ++j) c[j] = c9[j];
       for (int j = 9; j < (int)C_NCNT; ++j) c[j] = 0;
       row_finalize(row, ri, a, b, c, p, fs.out, fs.parts, nullptr);
+      if (ri == 0) fused_flags(fs);
     }
     return;
   }
@@ -1111,6 +1120,7 @@ __device__ __noinline__ void fused_stitch(const DiagRow& row, uint32_t ri, uint6
     for (int j = 0; j < 9; ++j) c[j] = c9[j];
     for (int j = 9; j < (int)C_NCNT; ++j) c[j] = 0;
     row_finalize(row, ri, a, b, c, p, fs.out, fs.parts, nullptr);
+    if (ri == 0) fused_flags(fs);
   }
 }
 
@@ -1367,12 +1377,13 @@ void launch_diag(cudaStream_t s, const DiagRow* rows, uint32_t nrows, const uint
                  uint64_t ntiles, const StitchSeg* segs, uint32_t nseg, uint64_t nblocks,
                  const DiagParams& p, uint32_t* pool, unsigned long long* cnt, TileSum* tiles,
                  void* segsum, uint32_t* blk_cnt, xpl_alloc_report* out, RowPartial* parts,
-                 cudaEvent_t tile_ev0, cudaEvent_t tile_ev1, uint32_t* done, unsigned long long* segcnt) {
+                 cudaEvent_t tile_ev0, cudaEvent_t tile_ev1, uint32_t* done, unsigned long long* segcnt,
+                 const uint32_t* flags_in, uint32_t* flags_out) {
   // fused: one launch (the stitch in the tile kernel's last warps); block
   // counts (p.block_words) need the whole tile pass first: separate kernels
   const bool fused = done != nullptr && p.block_words == 0;
   FusedStitch fs = {};
-  if (fused) fs = FusedStitch{done, done + nseg, segsum, segcnt, cnt, out, parts};
+  if (fused) fs = FusedStitch{done, done + nseg, segsum, segcnt, cnt, out, parts, flags_in, flags_out};
   if (!fused) {
     cudaMemsetAsync(cnt, 0, sizeof(unsigned long long) * C_NCNT * nrows, s);
     if (p.block_words && nblocks) cudaMemsetAsync(blk_cnt, 0, sizeof(uint32_t) * nblocks, s);

@@ -1793,20 +1793,25 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
   const uint64_t dbytes = total_words * (reset ? 2 : 1);
   const int pall = prof_begin(c, XPL_K_DIAGNOSE, dbytes);
   const int ptile = prof_begin(c, XPL_K_DIAG_TILE, dbytes, false);  // recorded by launch_diag
+  // fused: the kernel writes the report rows (and partials, counters, the
+  // epoch-split flags) straight into the pinned host buffers -- no copies back
   launch_diag(c->cs, c->d_drows, (uint32_t)nr, c->d_tile_row, ntiles, c->d_segs, (uint32_t)nseg,
-              nblocks, p, (uint32_t*)c->d_pool, c->d_cnt, c->d_tiles, c->d_segsum, c->d_blk, c->d_rep,
-              pout ? c->d_rpart : nullptr, ptile >= 0 ? c->prof_pending[ptile].a : nullptr,
-              ptile >= 0 ? c->prof_pending[ptile].b : nullptr, fused ? c->d_done : nullptr, c->d_segcnt);
+              nblocks, p, (uint32_t*)c->d_pool, fused ? c->h_cnt : c->d_cnt, c->d_tiles, c->d_segsum, c->d_blk,
+              fused ? c->h_rep : c->d_rep, pout ? (fused ? c->h_rpart : c->d_rpart) : nullptr,
+              ptile >= 0 ? c->prof_pending[ptile].a : nullptr, ptile >= 0 ? c->prof_pending[ptile].b : nullptr,
+              fused ? c->d_done : nullptr, c->d_segcnt, c->d_misc, fused ? c->h_misc : nullptr);
   CK(cudaGetLastError());
   c->st.kernel_launches += fused ? 1 : 3 + (B && nblocks ? 1 : 0);
-  CK(cudaMemcpyAsync(c->h_rep, c->d_rep, sizeof(xpl_alloc_report) * nr, cudaMemcpyDeviceToHost, c->cs));
-  if (pout) {
-    CK(cudaMemcpyAsync(c->h_rpart, c->d_rpart, sizeof(RowPartial) * nr, cudaMemcpyDeviceToHost, c->cs));
-    CK(cudaMemcpyAsync(c->h_cnt, c->d_cnt, sizeof(unsigned long long) * C_NCNT * nr,
-                       cudaMemcpyDeviceToHost, c->cs));
+  if (!fused) {
+    CK(cudaMemcpyAsync(c->h_rep, c->d_rep, sizeof(xpl_alloc_report) * nr, cudaMemcpyDeviceToHost, c->cs));
+    if (pout) {
+      CK(cudaMemcpyAsync(c->h_rpart, c->d_rpart, sizeof(RowPartial) * nr, cudaMemcpyDeviceToHost, c->cs));
+      CK(cudaMemcpyAsync(c->h_cnt, c->d_cnt, sizeof(unsigned long long) * C_NCNT * nr,
+                         cudaMemcpyDeviceToHost, c->cs));
+    }
+    CK(cudaMemcpyAsync(c->h_misc, c->d_misc, 8, cudaMemcpyDeviceToHost, c->cs));
   }
   prof_end(c, pall);
-  CK(cudaMemcpyAsync(c->h_misc, c->d_misc, 8, cudaMemcpyDeviceToHost, c->cs));
   CK(cudaStreamSynchronize(c->cs));
   s = split_error(c);
   if (s) return s;
