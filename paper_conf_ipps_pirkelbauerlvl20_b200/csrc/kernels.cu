@@ -180,28 +180,42 @@ __device__ __forceinline__ void merge_firstw_rec(const uint64_t* __restrict__ re
   for (uint64_t w = g0; w < g0 + nw; ++w) atomicMin(fw + (w - fw0), i);
 }
 
+// Record i's bits on shadow u32 q (one of the u32s its words [g0, g1] cover).
+__device__ __forceinline__ void merge_apply_q(uint32_t acc, uint64_t g0, uint64_t g1, uint32_t i, uint64_t q,
+                                              const uint32_t* __restrict__ fw, uint64_t fw0, uint32_t* pool) {
+  const uint32_t cur = pool[q];  // L bits do not change during this pass
+  uint32_t m = 0;
+#pragma unroll
+  for (uint32_t k = 0; k < 4; ++k) {
+    const uint64_t w = q * 4 + k;
+    if (w < g0 || w > g1) continue;
+    uint32_t b = 0;
+    if (acc & XPL_ACC_R) {
+      const bool before = (fw == nullptr) || i <= fw[w - fw0];
+      b = before ? (((cur >> (8 * k)) & 1u) ? kRGC : kRCC) : kRCC;
+    }
+    if (acc & XPL_ACC_W) b |= kWC;
+    m |= b << (8 * k);
+  }
+  if ((cur & m) != m) atomicOr(pool + q, m);
+}
+
 __device__ __forceinline__ void merge_apply_rec(const uint64_t* __restrict__ recs, uint32_t i,
                                                 const uint32_t* __restrict__ fw, uint64_t fw0, uint32_t* pool) {
   const uint64_t r = recs[i];
-  const uint32_t acc = rec_acc(r);
   const uint64_t g0 = rec_g0(r), g1 = g0 + rec_nw(r) - 1;
-  for (uint64_t q = g0 >> 2; q <= (g1 >> 2); ++q) {
-    const uint32_t cur = pool[q];  // L bits do not change during this pass
-    uint32_t m = 0;
+  for (uint64_t q = g0 >> 2; q <= (g1 >> 2); ++q) merge_apply_q(rec_acc(r), g0, g1, i, q, fw, fw0, pool);
+}
+
+// A written record's u32 q: clear L of its words (the CPU is now the last writer).
+__device__ __forceinline__ void merge_clear_q(uint64_t g0, uint64_t g1, uint64_t q, uint32_t* pool) {
+  uint32_t lm = 0;
 #pragma unroll
-    for (uint32_t k = 0; k < 4; ++k) {
-      const uint64_t w = q * 4 + k;
-      if (w < g0 || w > g1) continue;
-      uint32_t b = 0;
-      if (acc & XPL_ACC_R) {
-        const bool before = (fw == nullptr) || i <= fw[w - fw0];
-        b = before ? (((cur >> (8 * k)) & 1u) ? kRGC : kRCC) : kRCC;
-      }
-      if (acc & XPL_ACC_W) b |= kWC;
-      m |= b << (8 * k);
-    }
-    if ((cur & m) != m) atomicOr(pool + q, m);
+  for (uint32_t k = 0; k < 4; ++k) {
+    const uint64_t w = q * 4 + k;
+    if (w >= g0 && w <= g1) lm |= kL << (8 * k);
   }
+  if (pool[q] & lm) atomicAnd(pool + q, ~lm);
 }
 
 __device__ __forceinline__ void merge_clear_rec(const uint64_t* __restrict__ recs, uint32_t i,
@@ -209,15 +223,7 @@ __device__ __forceinline__ void merge_clear_rec(const uint64_t* __restrict__ rec
   const uint64_t r = recs[i];
   if (!(rec_acc(r) & XPL_ACC_W)) return;
   const uint64_t g0 = rec_g0(r), g1 = g0 + rec_nw(r) - 1;
-  for (uint64_t q = g0 >> 2; q <= (g1 >> 2); ++q) {
-    uint32_t lm = 0;
-#pragma unroll
-    for (uint32_t k = 0; k < 4; ++k) {
-      const uint64_t w = q * 4 + k;
-      if (w >= g0 && w <= g1) lm |= kL << (8 * k);
-    }
-    if (pool[q] & lm) atomicAnd(pool + q, ~lm);
-  }
+  for (uint64_t q = g0 >> 2; q <= (g1 >> 2); ++q) merge_clear_q(g0, g1, q, pool);
   if (fw)
     for (uint64_t w = g0; w <= g1; ++w) fw[w - fw0] = 0xFFFFFFFFu;
 }
@@ -242,20 +248,96 @@ __global__ void merge_clear_kernel(const uint64_t* __restrict__ recs, uint32_t n
 
 // A small batch (a host segment of a few thousand records, the common case
 // between epochs): the three passes in one CTA, separated by CTA barriers
-// instead of kernel boundaries -- one launch instead of three.
+// instead of kernel boundaries -- one launch instead of three.  The apply and
+// clear passes are spread over (record, shadow u32) items, not records: a
+// record of up to kPieceWords words covers up to 65 u32s, and one thread
+// walking them would chain as many dependent L2 round trips.  The items'
+// offsets are an exclusive scan of the records' u32 counts in shared memory;
+// an item finds its record by binary search.
 constexpr uint32_t kMergeSmall = 8192;
-__global__ void __launch_bounds__(1024) merge_small_kernel(const uint64_t* __restrict__ recs, uint32_t n,
-                                                           bool has_r, bool has_w, uint32_t* __restrict__ fw,
-                                                           uint64_t fw0, uint32_t* pool) {
+constexpr uint32_t kMergeThreads = 1024;
+constexpr uint32_t kMergePer = kMergeSmall / kMergeThreads;
+__global__ void __launch_bounds__(kMergeThreads) merge_small_kernel(const uint64_t* __restrict__ recs, uint32_t n,
+                                                                    bool has_r, bool has_w,
+                                                                    uint32_t* __restrict__ fw, uint64_t fw0,
+                                                                    uint32_t* pool) {
+  __shared__ uint32_t s_off[kMergeSmall + 1];  // exclusive scan of u32 counts; s_off[n] = items
+  __shared__ uint32_t s_warp[kMergeThreads / 32];
+  const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const bool both = has_r && has_w;
-  if (both) {
-    for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) merge_firstw_rec(recs, i, fw, fw0);
-    __syncthreads();
+  // scan: thread tid owns records [tid * kMergePer, +kMergePer)
+  uint32_t cnt[kMergePer], sum = 0;
+#pragma unroll
+  for (uint32_t k = 0; k < kMergePer; ++k) {
+    const uint32_t i = tid * kMergePer + k;
+    cnt[k] = 0;
+    if (i < n) {
+      const uint64_t r = recs[i];
+      const uint64_t g0 = rec_g0(r), g1 = g0 + rec_nw(r) - 1;
+      cnt[k] = (uint32_t)((g1 >> 2) - (g0 >> 2) + 1);
+      if (both) merge_firstw_rec(recs, i, fw, fw0);
+    }
+    sum += cnt[k];
   }
-  for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) merge_apply_rec(recs, i, both ? fw : nullptr, fw0, pool);
-  if (has_w) {
-    __syncthreads();
-    for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) merge_clear_rec(recs, i, both ? fw : nullptr, fw0, pool);
+  uint32_t incl = sum;
+#pragma unroll
+  for (uint32_t o = 1; o < 32; o <<= 1) {
+    const uint32_t v = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+    if (lane >= o) incl += v;
+  }
+  if (lane == 31) s_warp[wid] = incl;
+  __syncthreads();
+  if (wid == 0) {
+    uint32_t w = s_warp[lane], wi = w;
+#pragma unroll
+    for (uint32_t o = 1; o < 32; o <<= 1) {
+      const uint32_t v = __shfl_up_sync(0xFFFFFFFFu, wi, o);
+      if (lane >= o) wi += v;
+    }
+    s_warp[lane] = wi - w;  // exclusive over warps
+  }
+  __syncthreads();
+  uint32_t off = s_warp[wid] + incl - sum;
+#pragma unroll
+  for (uint32_t k = 0; k < kMergePer; ++k) {
+    const uint32_t i = tid * kMergePer + k;
+    if (i <= n) s_off[i] = off;  // (i == n: the total)
+    off += cnt[k];
+  }
+  if (tid == kMergeThreads - 1) s_off[n] = off;  // (the total; n == kMergeSmall has no owner above)
+  __syncthreads();  // (also orders pass 1's first writers before pass 2)
+  const uint32_t items = s_off[n];
+  auto rec_of = [&](uint32_t x) {  // the last record with s_off <= x
+    uint32_t lo = 0, hi = n;
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (s_off[mid] <= x) lo = mid;
+      else hi = mid;
+    }
+    return lo;
+  };
+  for (uint32_t x = tid; x < items; x += kMergeThreads) {
+    const uint32_t i = rec_of(x);
+    const uint64_t r = recs[i];
+    const uint64_t g0 = rec_g0(r), g1 = g0 + rec_nw(r) - 1;
+    merge_apply_q(rec_acc(r), g0, g1, i, (g0 >> 2) + (x - s_off[i]), both ? fw : nullptr, fw0, pool);
+  }
+  if (!has_w) return;
+  __syncthreads();
+  for (uint32_t x = tid; x < items; x += kMergeThreads) {
+    const uint32_t i = rec_of(x);
+    const uint64_t r = recs[i];
+    if (!(rec_acc(r) & XPL_ACC_W)) continue;
+    const uint64_t g0 = rec_g0(r), g1 = g0 + rec_nw(r) - 1;
+    merge_clear_q(g0, g1, (g0 >> 2) + (x - s_off[i]), pool);
+  }
+  if (both) {  // the first-writer scratch back to all-ones
+    for (uint32_t i = tid; i < n; i += kMergeThreads) {
+      const uint64_t r = recs[i];
+      if (!(rec_acc(r) & XPL_ACC_W)) continue;
+      const uint64_t g0 = rec_g0(r), g1 = g0 + rec_nw(r) - 1;
+      for (uint64_t w = g0; w <= g1; ++w) fw[w - fw0] = 0xFFFFFFFFu;
+    }
   }
 }
 
@@ -1357,7 +1439,7 @@ void launch_fold(cudaStream_t s, bool pdl, uint32_t* pool, uint8_t* cmap, uint8_
 void launch_merge(cudaStream_t s, const uint64_t* recs, uint32_t n, bool has_r, bool has_w,
                   uint32_t* first_w, uint64_t fw0, uint32_t* pool) {
   if (n <= kMergeSmall) {
-    merge_small_kernel<<<1, 1024, 0, s>>>(recs, n, has_r, has_w, first_w, fw0, pool);
+    merge_small_kernel<<<1, kMergeThreads, 0, s>>>(recs, n, has_r, has_w, first_w, fw0, pool);
     return;
   }
   const int g = grid_for(n, 256, 148 * 16);
