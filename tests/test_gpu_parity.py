@@ -376,6 +376,32 @@ def long_row_trace(seed, words=(5_000_003, 700_001, 3)):
 _EXPECTED = {}
 
 
+@pytest.mark.parametrize("n", [1, 1023, 8191, 8192, 8193])
+def test_merge_segment_sizes(gpu, n):
+    """Host segments of exactly n staged records around the single-CTA merge's
+    limit (8192 records): scattered non-abutting accesses of every kind, mixed
+    with ranges of up to 256 words (a piece's 65 shadow u32s), read before and
+    after writes of the same words; device epochs in between so L differs."""
+    replay, _ = gpu
+    rng = np.random.default_rng(0x58504C70 + n)
+    w = 40_000
+    base = 0x5000_0000
+    ops = [("REG", base, 4 * w, MANAGED), ("KB",),
+           ("DB", base + 4 * np.arange(0, w, 3, dtype=np.uint64), np.full(len(range(0, w, 3)), 4, np.uint32),
+            np.full(len(range(0, w, 3)), W, np.uint8)), ("KE",)]
+    for _ in range(2):
+        words = np.sort(rng.choice(w // 2, size=n, replace=False)) * 2  # (never abutting: no coalescing)
+        size = np.where(rng.random(n) < 0.05, 4 * rng.integers(2, 257, size=n), 4).astype(np.uint32)
+        words = np.minimum(words, w - size // 4)
+        perm = rng.permutation(n)
+        ops.append(("HB", base + 4 * words[perm].astype(np.uint64), size[perm],
+                    rng.integers(1, 4, size=n).astype(np.uint8)))
+        ops += [("KB",), ("DB", base + 4 * rng.integers(0, w, size=5000).astype(np.uint64),
+                          np.full(5000, 4, np.uint32), rng.integers(1, 4, size=5000).astype(np.uint8)), ("KE",)]
+        ops.append(("DIAG", 50, 0, 1, 0, ()))
+    compare(replay.run_trace(ops, pool_words=1 << 20), oracle_run(ops), f"n={n}")
+
+
 @pytest.mark.parametrize("mode", ["fused", "unfused"])
 @pytest.mark.parametrize("tile", ["2048", "16384"])
 def test_diag_long_rows(gpu, mode, tile, monkeypatch):
