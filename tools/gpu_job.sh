@@ -51,8 +51,8 @@ for step in "$@"; do
               --master-addr 127.0.0.1 --master-port 29533 bench.py --gpus 2 $args \
               > gpurun_out/${TAG}_bench2.json 2> gpurun_out/${TAG}_bench2.err ;;
     golden5) mkdir -p gpurun_out/golden5/cfg5_parts
-             # (a part peaks near 30 GB of host memory: 40 GB of MemAvailable per worker)
-             W=$(python -c "import os; m=int(open('/proc/meminfo').read().split('MemAvailable:')[1].split()[0])/2**20; print(max(1, min(os.cpu_count()-1, int(m//40))))")
+             # (a part peaks near 28 GB of host memory: GOLDEN5_GB (default 40) of MemAvailable per worker)
+             W=$(python -c "import os; m=int(open('/proc/meminfo').read().split('MemAvailable:')[1].split()[0])/2**20; print(max(1, min(os.cpu_count()-1, int(m//int(os.environ.get('GOLDEN5_GB', '40'))))))")
              echo "workers=$W" > gpurun_out/golden5/box.txt; free -g >> gpurun_out/golden5/box.txt
              cp tests/golden/fullsize/cfg5_parts/*.json gpurun_out/golden5/cfg5_parts/ 2>/dev/null
              timeout ${GOLDEN5_TIMEOUT:-5400} python tools/golden_fullsize.py cfg5 --workers $W --out gpurun_out/golden5 \
