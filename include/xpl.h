@@ -108,7 +108,8 @@ typedef struct {
  *    merged there in that order;
  *  - epochs are collective (all ranks' kernels between kernel_begin/_end form
  *    one GPU epoch); the close waits for every rank's kernels (barrier) before
- *    each owner folds its pool;
+ *    each owner folds its pool, and the next begin waits for every rank's
+ *    shadow work (folds, merges, resets) before any rank records again;
  *  - xpl_diagnose is collective: each owner analyses its pieces, the partials
  *    are exchanged (all-gather) and combined on every rank: every rank gets the
  *    same reports, equal to the unsharded run's (field `base`: the piece-0
@@ -225,7 +226,8 @@ xpl_status xpl_free(xpl_ctx* ctx, const void* ptr);
  * epoch there).  Such a stream must stay valid until xpl_release_stream() names
  * it or xpl_finalize(); the legacy / per-thread default streams are never
  * adopted.  Sharded mode: COLLECTIVE; end waits for this rank's epoch streams
- * and for every rank (barrier) before the owner folds. */
+ * and for every rank (barrier) before the owner folds; begin (outermost) waits
+ * for this rank's runtime stream and for every rank (barrier). */
 xpl_status xpl_kernel_begin(xpl_ctx* ctx, void* stream);
 xpl_status xpl_kernel_end(xpl_ctx* ctx, void* stream);
 

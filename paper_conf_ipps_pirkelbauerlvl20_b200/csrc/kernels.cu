@@ -861,15 +861,14 @@ __device__ __forceinline__ void tile_loop(TileAcc& A, WarpRing& R, uint4* p4, ui
 // the uniform-step counts.  Runs: ballot fast paths for all-zero/all-one
 // 512-word steps, warp_runs() for mixed ones.  Reset fused.  The tile's counts
 // and run summaries go to tiles[t]; the stitch adds and combines them in order.
-// The stitch fused into the tile kernel (no block counts: p.block_words == 0):
-// the warp that finishes the last tile of a segment combines the segment, the
-// one that finishes its row's last segment combines the row and writes its
-// report (last-block-done: release fence + done counter, which that warp
-// resets to 0 for the next call).  Null seg_done = the separate stitch kernels.
+// The stitch in one kernel launched right behind the tile kernel (programmatic
+// dependent launch; no block counts: p.block_words == 0): a warp per segment
+// combines its <= kSegTiles tiles; the warp that finishes its row's last
+// segment (last-warp-done: release fence + done counter, which that warp resets
+// to 0 for the next call) combines the row and writes its report.  Null
+// row_done = the separate stitch kernels.
 struct FusedStitch {
-  uint32_t* seg_done;               // per segment: tiles done
-  uint32_t* row_done;               // per row: segments done
-  void* segsum;                     // RunPair per segment
+  uint32_t* row_done;               // per row: segments done (kept zero between calls)
   unsigned long long* segcnt;       // 9 counters per segment
   unsigned long long* cnt;          // C_NCNT counters per row (partials)
   xpl_alloc_report* out;
@@ -877,16 +876,14 @@ struct FusedStitch {
   const uint32_t* flags_in;         // d_misc[0..1], copied to flags_out by row 0's finalizer
   uint32_t* flags_out;
 };
-__device__ __noinline__ void fused_stitch(const DiagRow& row, uint32_t ri, uint64_t t, const DiagParams& p,
-                                          const TileSum* tiles, const FusedStitch& fs, uint32_t lane);
 
 #ifndef XPL_DIAG_MINB
 #define XPL_DIAG_MINB 4  // CTAs per SM the register budget is sized for (A/B: profiles/r1h_diag_variants.txt)
 #endif
 __global__ void __launch_bounds__(kDiagThreads, XPL_DIAG_MINB) diag_tile_kernel(
-    const DiagRow* __restrict__ rows, uint32_t nrows, const uint32_t* __restrict__ tile_row, uint64_t ntiles,
+    const DiagRow* __restrict__ rows, const uint32_t* __restrict__ tile_row, uint64_t ntiles,
     DiagParams p, uint32_t* __restrict__ pool, TileSum* __restrict__ tiles,
-    uint32_t* __restrict__ blk_cnt, FusedStitch fs) {
+    uint32_t* __restrict__ blk_cnt) {
   constexpr uint32_t kWarps = kDiagThreads / 32;
   __shared__ uint32_t s_uc[kWarps][9];
   extern __shared__ __align__(128) unsigned char s_dyn[];
@@ -899,18 +896,7 @@ __global__ void __launch_bounds__(kDiagThreads, XPL_DIAG_MINB) diag_tile_kernel(
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncwarp();
-  uint32_t ri;
-  if (tile_row) {
-    ri = tile_row[t];
-  } else {  // the last row with tile0 <= t (rows in tile order, none empty)
-    uint32_t lo = 0, hi = nrows;
-    while (hi - lo > 1) {
-      const uint32_t mid = (lo + hi) >> 1;
-      if (__ldg(&rows[mid].tile0) <= t) lo = mid;
-      else hi = mid;
-    }
-    ri = lo;
-  }
+  const uint32_t ri = tile_row[t];
   const DiagRow row = rows[ri];
   const uint32_t tw = p.tile_words;
   const uint64_t ww0 = (t - row.tile0) * tw;  // row word
@@ -958,7 +944,6 @@ __global__ void __launch_bounds__(kDiagThreads, XPL_DIAG_MINB) diag_tile_kernel(
     ts->u = A.wu;
     ts->d = A.wd;
   }
-  if (fs.seg_done) fused_stitch(row, ri, t, p, tiles, fs, lane);
 }
 
 __device__ __forceinline__ void run_final(const RunSum64& s, uint64_t min_run, uint64_t* runs,
@@ -1118,68 +1103,50 @@ __device__ __forceinline__ void fused_flags(const FusedStitch& fs) {
 
 __device__ __forceinline__ RunSum64 rs64(const RunSum& u) { return RunSum64{u.len, u.pre, u.suf, u.cnt, u.sum}; }
 
-__device__ __noinline__ void fused_stitch(const DiagRow& row, uint32_t ri, uint64_t t, const DiagParams& p,
-                                          const TileSum* tiles, const FusedStitch& fs, uint32_t lane) {
-  const uint64_t k = (t - row.tile0) / kSegTiles;  // the tile's segment within its row
-  const uint64_t seg = row.seg0 + k;
-  const uint64_t st0 = row.tile0 + k * kSegTiles;
-  const uint32_t sn = (uint32_t)min(kSegTiles, row.ntiles - k * kSegTiles);
-  __threadfence();  // (release: this lane's TileSum stores before the count)
-  __syncwarp();
-  uint32_t last = 0;
-  if (lane == 0) last = atomicAdd(fs.seg_done + seg, 1u) == sn - 1;
-  if (!__shfl_sync(0xFFFFFFFFu, last, 0)) return;
-  __threadfence();  // (acquire: the segment's other TileSums)
+__global__ void __launch_bounds__(256) stitch_fused_kernel(const StitchSeg* __restrict__ segs, uint32_t nseg,
+                                                           const DiagRow* __restrict__ rows,
+                                                           const TileSum* __restrict__ tiles, DiagParams p,
+                                                           RunPair* __restrict__ ss, FusedStitch fs) {
+  asm volatile("griddepcontrol.wait;" ::: "memory");  // (the tile kernel's summaries are complete)
+  const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint32_t lane = threadIdx.x & 31;
+  if (gw >= nseg) return;
+  const StitchSeg sg = segs[gw];
+  const uint32_t ri = (uint32_t)sg.row;
+  const DiagRow row = rows[ri];
   // level 1: the segment's tiles in order (lanes take contiguous sub-ranges)
   RunSum64 a = {0, 0, 0, 0, 0}, b = {0, 0, 0, 0, 0};
   uint64_t c9[9] = {0, 0, 0, 0, 0, 0, 0, 0, 0};
   {
-    const uint32_t per = (sn + 31) / 32;
-    const uint64_t t0 = st0 + lane * per, t1 = min(st0 + sn, t0 + per);
+    const uint64_t per = (sg.n + 31) / 32;
+    const uint64_t t0 = sg.t0 + lane * per, t1 = min(sg.t0 + sg.n, t0 + per);
     for (uint64_t u = t0; u < t1; ++u) {
-      const TileSum* ts = tiles + u;
-      RunSum uu, dd;
-      uu.len = __ldcg(&ts->u.len); uu.pre = __ldcg(&ts->u.pre); uu.suf = __ldcg(&ts->u.suf);
-      uu.cnt = __ldcg(&ts->u.cnt); uu.sum = __ldcg(&ts->u.sum);
-      dd.len = __ldcg(&ts->d.len); dd.pre = __ldcg(&ts->d.pre); dd.suf = __ldcg(&ts->d.suf);
-      dd.cnt = __ldcg(&ts->d.cnt); dd.sum = __ldcg(&ts->d.sum);
+      const RunSum uu = tiles[u].u, dd = tiles[u].d;
       a = rs_combine(a, rs64(uu), p.min_run);
       b = rs_combine(b, rs64(dd), p.min_run);
 #pragma unroll
-      for (int j = 0; j < 9; ++j) c9[j] += __ldcg(&ts->cnt[j]);
+      for (int j = 0; j < 9; ++j) c9[j] += tiles[u].cnt[j];
     }
   }
   warp_combine(a, b, lane, p.min_run);
 #pragma unroll
   for (int j = 0; j < 9; ++j)
     for (uint32_t o = 16; o; o >>= 1) c9[j] += __shfl_down_sync(0xFFFFFFFFu, c9[j], o);
-  if (row.nseg == 1) {  // (the common case at small sizes: the segment is the row)
+  if (row.nseg > 1) {
+    uint32_t last = 0;
     if (lane == 0) {
-      fs.seg_done[seg] = 0;
-      unsigned long long* c = fs.cnt + (uint64_t)ri * C_NCNT;
-      for (int j = 0; j < 9; ++j) c[j] = c9[j];
-      for (int j = 9; j < (int)C_NCNT; ++j) c[j] = 0;
-      row_finalize(row, ri, a, b, c, p, fs.out, fs.parts, nullptr);
-      if (ri == 0) fused_flags(fs);
+      ss[gw] = RunPair{a, b};
+      for (int j = 0; j < 9; ++j) fs.segcnt[(uint64_t)gw * 9 + j] = c9[j];
+      __threadfence();  // (release: the segment's summary before the count)
+      last = atomicAdd(fs.row_done + ri, 1u) == row.nseg - 1;
     }
-    return;
-  }
-  RunPair* const ss = reinterpret_cast<RunPair*>(fs.segsum);
-  if (lane == 0) {
-    ss[seg] = RunPair{a, b};
-    for (int j = 0; j < 9; ++j) fs.segcnt[seg * 9 + j] = c9[j];
-    fs.seg_done[seg] = 0;
-    __threadfence();
-    last = atomicAdd(fs.row_done + ri, 1u) == row.nseg - 1;
-  }
-  if (!__shfl_sync(0xFFFFFFFFu, last, 0)) return;
-  __threadfence();
-  // level 2: the row's segments in order
-  a = RunSum64{0, 0, 0, 0, 0};
-  b = RunSum64{0, 0, 0, 0, 0};
+    if (!__shfl_sync(0xFFFFFFFFu, last, 0)) return;
+    __threadfence();  // (acquire: the row's other segment summaries)
+    // level 2: the row's segments in order
+    a = RunSum64{0, 0, 0, 0, 0};
+    b = RunSum64{0, 0, 0, 0, 0};
 #pragma unroll
-  for (int j = 0; j < 9; ++j) c9[j] = 0;
-  {
+    for (int j = 0; j < 9; ++j) c9[j] = 0;
     const uint64_t per = (row.nseg + 31) / 32;
     const uint64_t s0 = row.seg0 + lane * per, s1 = min(row.seg0 + row.nseg, s0 + per);
     for (uint64_t u = s0; u < s1; ++u) {
@@ -1191,13 +1158,13 @@ __device__ __noinline__ void fused_stitch(const DiagRow& row, uint32_t ri, uint6
 #pragma unroll
       for (int j = 0; j < 9; ++j) c9[j] += __ldcg(fs.segcnt + u * 9 + j);
     }
-  }
-  warp_combine(a, b, lane, p.min_run);
+    warp_combine(a, b, lane, p.min_run);
 #pragma unroll
-  for (int j = 0; j < 9; ++j)
-    for (uint32_t o = 16; o; o >>= 1) c9[j] += __shfl_down_sync(0xFFFFFFFFu, c9[j], o);
+    for (int j = 0; j < 9; ++j)
+      for (uint32_t o = 16; o; o >>= 1) c9[j] += __shfl_down_sync(0xFFFFFFFFu, c9[j], o);
+  }
   if (lane == 0) {
-    fs.row_done[ri] = 0;
+    if (row.nseg > 1) fs.row_done[ri] = 0;
     unsigned long long* c = fs.cnt + (uint64_t)ri * C_NCNT;
     for (int j = 0; j < 9; ++j) c[j] = c9[j];
     for (int j = 9; j < (int)C_NCNT; ++j) c[j] = 0;
@@ -1459,13 +1426,11 @@ void launch_diag(cudaStream_t s, const DiagRow* rows, uint32_t nrows, const uint
                  uint64_t ntiles, const StitchSeg* segs, uint32_t nseg, uint64_t nblocks,
                  const DiagParams& p, uint32_t* pool, unsigned long long* cnt, TileSum* tiles,
                  void* segsum, uint32_t* blk_cnt, xpl_alloc_report* out, RowPartial* parts,
-                 cudaEvent_t tile_ev0, cudaEvent_t tile_ev1, uint32_t* done, unsigned long long* segcnt,
+                 cudaEvent_t tile_ev0, cudaEvent_t tile_ev1, uint32_t* row_done, unsigned long long* segcnt,
                  const uint32_t* flags_in, uint32_t* flags_out) {
-  // fused: one launch (the stitch in the tile kernel's last warps); block
-  // counts (p.block_words) need the whole tile pass first: separate kernels
-  const bool fused = done != nullptr && p.block_words == 0;
-  FusedStitch fs = {};
-  if (fused) fs = FusedStitch{done, done + nseg, segsum, segcnt, cnt, out, parts, flags_in, flags_out};
+  // fused: tile kernel + one stitch kernel (PDL); block counts (p.block_words)
+  // need the block pass between them: separate kernels
+  const bool fused = row_done != nullptr && p.block_words == 0;
   if (!fused) {
     cudaMemsetAsync(cnt, 0, sizeof(unsigned long long) * C_NCNT * nrows, s);
     if (p.block_words && nblocks) cudaMemsetAsync(blk_cnt, 0, sizeof(uint32_t) * nblocks, s);
@@ -1476,9 +1441,22 @@ void launch_diag(cudaStream_t s, const DiagRow* rows, uint32_t nrows, const uint
   cudaFuncSetAttribute(diag_tile_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kDiagSmem);
   if (ntiles)
     diag_tile_kernel<<<(unsigned)((ntiles + kWarps - 1) / kWarps), kDiagThreads, kDiagSmem, s>>>(
-        rows, nrows, fused ? nullptr : tile_row, ntiles, p, pool, tiles, blk_cnt, fs);
+        rows, tile_row, ntiles, p, pool, tiles, blk_cnt);
   if (tile_ev1) cudaEventRecord(tile_ev1, s);
-  if (fused) return;
+  if (fused) {
+    const FusedStitch fs = {row_done, segcnt, cnt, out, parts, flags_in, flags_out};
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((nseg * 32 + 255) / 256);
+    cfg.blockDim = dim3(256);
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = tile_ev1 ? 0 : 1;  // (profiled: no overlap with the timed tile kernel)
+    cudaLaunchKernelEx(&cfg, stitch_fused_kernel, segs, nseg, rows, (const TileSum*)tiles, p, (RunPair*)segsum, fs);
+    return;
+  }
   if (p.block_words && nblocks)
     block_eval_kernel<<<grid_for(nblocks, 256, 148 * 8), 256, 0, s>>>(rows, nrows, nblocks, blk_cnt,
                                                                     p.block_words, p.thr, cnt);

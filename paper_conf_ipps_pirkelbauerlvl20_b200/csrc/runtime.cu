@@ -184,7 +184,7 @@ struct xpl_ctx {
   void* d_segsum = nullptr;
   unsigned long long* d_segcnt = nullptr;  // fused stitch: 9 counters per segment
   size_t segs_cap = 0;
-  uint32_t* d_done = nullptr;  // fused stitch: segment + row done counters (kept zero)
+  uint32_t* d_done = nullptr;  // fused stitch: row done counters (kept zero)
   size_t done_cap = 0;
   unsigned long long* d_cnt = nullptr;
   xpl_alloc_report* d_rep = nullptr;
@@ -1223,6 +1223,14 @@ xpl_status xpl_kernel_begin(xpl_ctx* c, void* stream) {
     if (st) return st;
     st = upload_table(c);
     if (st) return st;
+    if (c->world > 1) {
+      // sharded: every rank's shadow work before this epoch -- its fold of the
+      // last epoch, its merges of the routed host records, a diagnose's reset --
+      // has completed before any rank's kernels record into its pool again
+      // (a remote write landing before the owner's fold would be folded early)
+      CK(cudaStreamSynchronize(c->cs));
+      if (c->comm->barrier(c->comm->user)) return XPL_ERR_NCCL;
+    }
     c->ev_begin_valid = false;
     c->cs_in_epoch = false;
     c->epoch_streams.clear();
@@ -1744,15 +1752,15 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
     c->blk_cap = std::max<uint64_t>(nblocks, 1024);
     CK(cudaMalloc(&c->d_blk, sizeof(uint32_t) * c->blk_cap));
   }
-  // fused stitch (one launch): no block counts, no empty row
+  // fused stitch (tile kernel + one stitch kernel): no block counts, no empty row
   bool fused = B == 0 && getenv("XPL_DIAG_UNFUSED") == nullptr;
   for (uint64_t id : ids) fused = fused && c->rows[id].words > 0;
-  if (fused && nseg + nr > c->done_cap) {
+  if (fused && nr > c->done_cap) {
     if (c->d_done) {
       CK(cudaStreamSynchronize(c->cs));
       cudaFree(c->d_done);
     }
-    c->done_cap = std::max<size_t>(nseg + nr, 4096);
+    c->done_cap = std::max<size_t>(nr, 4096);
     CK(cudaMalloc(&c->d_done, sizeof(uint32_t) * c->done_cap));
     CK(cudaMemsetAsync(c->d_done, 0, sizeof(uint32_t) * c->done_cap, c->cs));
   }
@@ -1772,24 +1780,20 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
     d.pad = 0;
     d.seg0 = sgi;
     d.nseg = (d.ntiles + kSegTiles - 1) / kSegTiles;
-    if (!fused) {  // (the fused kernel finds a tile's row and segment itself)
-      for (uint64_t k = 0; k < d.nseg; ++k) {
-        c->h_segs[sgi + k].t0 = t + k * kSegTiles;
-        c->h_segs[sgi + k].n = std::min<uint64_t>(kSegTiles, d.ntiles - k * kSegTiles);
-        c->h_segs[sgi + k].row = i;
-      }
-      for (uint64_t k = 0; k < d.ntiles; ++k) c->h_tile_row[t + k] = (uint32_t)i;
+    for (uint64_t k = 0; k < d.nseg; ++k) {
+      c->h_segs[sgi + k].t0 = t + k * kSegTiles;
+      c->h_segs[sgi + k].n = std::min<uint64_t>(kSegTiles, d.ntiles - k * kSegTiles);
+      c->h_segs[sgi + k].row = i;
     }
+    for (uint64_t k = 0; k < d.ntiles; ++k) c->h_tile_row[t + k] = (uint32_t)i;
     sgi += d.nseg;
     t += d.ntiles;
     b += d.nblk;
   }
   CK(cudaMemcpyAsync(c->d_drows, c->h_drows, sizeof(DiagRow) * nr, cudaMemcpyHostToDevice, c->cs));
-  if (!fused) {
-    CK(cudaMemcpyAsync(c->d_tile_row, c->h_tile_row, sizeof(uint32_t) * ntiles,
-                       cudaMemcpyHostToDevice, c->cs));
-    CK(cudaMemcpyAsync(c->d_segs, c->h_segs, sizeof(StitchSeg) * nseg, cudaMemcpyHostToDevice, c->cs));
-  }
+  CK(cudaMemcpyAsync(c->d_tile_row, c->h_tile_row, sizeof(uint32_t) * ntiles,
+                     cudaMemcpyHostToDevice, c->cs));
+  CK(cudaMemcpyAsync(c->d_segs, c->h_segs, sizeof(StitchSeg) * nseg, cudaMemcpyHostToDevice, c->cs));
   const uint64_t dbytes = total_words * (reset ? 2 : 1);
   const int pall = prof_begin(c, XPL_K_DIAGNOSE, dbytes);
   const int ptile = prof_begin(c, XPL_K_DIAG_TILE, dbytes, false);  // recorded by launch_diag
@@ -1801,7 +1805,7 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
               ptile >= 0 ? c->prof_pending[ptile].a : nullptr, ptile >= 0 ? c->prof_pending[ptile].b : nullptr,
               fused ? c->d_done : nullptr, c->d_segcnt, c->d_misc, fused ? c->h_misc : nullptr);
   CK(cudaGetLastError());
-  c->st.kernel_launches += fused ? 1 : 3 + (B && nblocks ? 1 : 0);
+  c->st.kernel_launches += fused ? 2 : 3 + (B && nblocks ? 1 : 0);
   if (!fused) {
     CK(cudaMemcpyAsync(c->h_rep, c->d_rep, sizeof(xpl_alloc_report) * nr, cudaMemcpyDeviceToHost, c->cs));
     if (pout) {

@@ -107,12 +107,12 @@ void launch_diag(cudaStream_t s, const DiagRow* rows, uint32_t nrows, const uint
                  uint64_t ntiles, const StitchSeg* segs, uint32_t nseg, uint64_t nblocks,
                  const DiagParams& p, uint32_t* pool, unsigned long long* cnt, TileSum* tiles,
                  void* segsum, uint32_t* blk_cnt, xpl_alloc_report* out, RowPartial* parts,
-                 cudaEvent_t tile_ev0, cudaEvent_t tile_ev1, uint32_t* done, unsigned long long* segcnt,
+                 cudaEvent_t tile_ev0, cudaEvent_t tile_ev1, uint32_t* row_done, unsigned long long* segcnt,
                  const uint32_t* flags_in, uint32_t* flags_out);
-// done: nseg + nrows zero u32s (segment / row done counters, left zero), or null
-// for the separate stitch kernels; segcnt: 9 u64 per segment.  Fused, the
-// kernel may write out / parts / cnt and flags_out (<- flags_in[0..1]) straight
-// into pinned host memory (unified addressing): no copies back.
+// row_done: nrows zero u32s (row done counters, left zero), or null for the
+// separate stitch kernels; segcnt: 9 u64 per segment.  Fused, the stitch kernel
+// may write out / parts / cnt and flags_out (<- flags_in[0..1]) straight into
+// pinned host memory (unified addressing): no copies back.
 constexpr size_t kRunPairBytes = 80;  // sizeof(RunPair) in kernels.cu
 struct PageRow {  // one live row of a page pass (NEXT-3)
   uint64_t off, words, page0;  // pool word offset, words, first global page index
