@@ -120,12 +120,21 @@ static __device__ __forceinline__ void xpld_mark(unsigned q) {
   unsigned char* c = xpl_dctx.cmap + (q >> 5);
   unsigned char* s = xpl_dctx.smap + (q >> 12);
   if (TESTED) {
+#if XPL_MARK_FLAG_LAZY  /* A/B: the flag word loaded only on a super-chunk's first mark */
+    const unsigned cv = *c, sv = *s;
+    if (!cv) *c = 1;
+    if (!sv) {
+      *s = 1;
+      if (!xpl_dctx.flags[2]) xpl_dctx.flags[2] = 1u;
+    }
+#else
     const unsigned cv = *c, sv = *s, fv = xpl_dctx.flags[2];
     if (!cv) *c = 1;
     if (!sv) {
       *s = 1;
       if (!fv) xpl_dctx.flags[2] = 1u;
     }
+#endif
   } else {  /* latency variant: plain stores, nothing to wait for */
     *c = 1;
     *s = 1;

@@ -11,6 +11,7 @@
 #   ncu:REGEX[:SKIP[:CMD]] ncu --set full of one launch of kernel REGEX (default command: bench.py --step-only)
 #   py:SCRIPT[:ARGS]       python SCRIPT ARGS > TAG_<name>.json
 #   pyab:SCRIPT[:ARGS]     the same with the A/B build libxplwork_ab.so > TAG_<name>_ab.json
+#   pyw:LIB:SCRIPT[:ARGS]  the same with the work library LIB (an A/B build in the package dir)
 #   sanitize:TOOL          compute-sanitizer --tool TOOL (memcheck|synccheck|racecheck) over tools/sanitize_driver.py
 #   bench2[:ARGS]          2 ranks on this one GPU over gloo (the sharded N>1 bench path): torchrun bench.py --gpus 2
 #   golden5                cfg5's oracle expectations on the box's host cores (tools/golden_fullsize.py cfg5)
@@ -41,6 +42,10 @@ for step in "$@"; do
     py) script=${rest%%:*}; a2=${rest#*:}; [ "$a2" = "$rest" ] && a2=""
         name=$(basename "$script" .py)
         timeout 1800 python $script ${a2//+/ } > gpurun_out/${TAG}_$name.json 2> gpurun_out/${TAG}_$name.err ;;
+    pyw) lib=${rest%%:*}; r2=${rest#*:}; script=${r2%%:*}; a2=${r2#*:}; [ "$a2" = "$r2" ] && a2=""
+         name=$(basename "$script" .py)_$(basename "$lib" .so)
+         XPL_WORK_PATH=paper_conf_ipps_pirkelbauerlvl20_b200/$lib timeout 1800 python $script ${a2//+/ } \
+           > gpurun_out/${TAG}_$name.json 2> gpurun_out/${TAG}_$name.err ;;
     pyab) script=${rest%%:*}; a2=${rest#*:}; [ "$a2" = "$rest" ] && a2=""
           name=$(basename "$script" .py)
           XPL_WORK_PATH=paper_conf_ipps_pirkelbauerlvl20_b200/libxplwork_ab.so timeout 1800 python $script ${a2//+/ } \
