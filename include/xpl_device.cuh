@@ -463,6 +463,12 @@ static __device__ __forceinline__ void xpld_record_fast(unsigned long long g0, u
   const unsigned needers = __ballot_sync(act, need);
   if (!needers) return; /* uniform: nothing missing (a re-touch) */
   const unsigned grp = __match_any_sync(act, need ? q : 0xFFFFFFFFu) & needers;
+#if XPL_FAST_ALONE  /* A/B: scattered warps (every needer alone on its u32) commit at once */
+  if (__all_sync(act, !need || grp == (1u << lane))) {
+    if (need) xpld_put<K, TM>(q, cur, rb, wb);
+    return;
+  }
+#endif
   unsigned gb = 0;
 #pragma unroll
   for (unsigned k = 0; k < 4; ++k) {
