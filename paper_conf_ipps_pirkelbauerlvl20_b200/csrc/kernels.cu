@@ -1118,14 +1118,21 @@ __global__ void __launch_bounds__(256) stitch_fused_kernel(const StitchSeg* __re
   RunSum64 a = {0, 0, 0, 0, 0}, b = {0, 0, 0, 0, 0};
   uint64_t c9[9] = {0, 0, 0, 0, 0, 0, 0, 0, 0};
   {
+    // (kSegTiles / 32 tiles per lane: every load is issued before the first combine)
+    constexpr uint32_t kPer = (uint32_t)(kSegTiles / 32);
     const uint64_t per = (sg.n + 31) / 32;
     const uint64_t t0 = sg.t0 + lane * per, t1 = min(sg.t0 + sg.n, t0 + per);
-    for (uint64_t u = t0; u < t1; ++u) {
-      const RunSum uu = tiles[u].u, dd = tiles[u].d;
-      a = rs_combine(a, rs64(uu), p.min_run);
-      b = rs_combine(b, rs64(dd), p.min_run);
+    TileSum ts[kPer];
 #pragma unroll
-      for (int j = 0; j < 9; ++j) c9[j] += tiles[u].cnt[j];
+    for (uint32_t k = 0; k < kPer; ++k)
+      if (t0 + k < t1) ts[k] = tiles[t0 + k];
+#pragma unroll
+    for (uint32_t k = 0; k < kPer; ++k) {
+      if (t0 + k >= t1) break;
+      a = rs_combine(a, rs64(ts[k].u), p.min_run);
+      b = rs_combine(b, rs64(ts[k].d), p.min_run);
+#pragma unroll
+      for (int j = 0; j < 9; ++j) c9[j] += ts[k].cnt[j];
     }
   }
   warp_combine(a, b, lane, p.min_run);

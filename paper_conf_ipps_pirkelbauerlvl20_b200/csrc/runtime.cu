@@ -170,21 +170,20 @@ struct xpl_ctx {
   cudaEvent_t ranges_ev = nullptr;
 
   // diagnose buffers (grown on demand)
-  DiagRow* h_drows = nullptr;
-  DiagRow* d_drows = nullptr;
   size_t drows_cap = 0;
-  uint32_t* h_tile_row = nullptr;
-  uint32_t* d_tile_row = nullptr;
   TileSum* d_tiles = nullptr;
   size_t tiles_cap = 0;
   uint32_t* d_blk = nullptr;
   size_t blk_cap = 0;
-  StitchSeg* h_segs = nullptr;
-  StitchSeg* d_segs = nullptr;
   void* d_segsum = nullptr;
   unsigned long long* d_segcnt = nullptr;  // fused stitch: 9 counters per segment
   size_t segs_cap = 0;
   uint32_t* d_done = nullptr;  // fused stitch: row done counters (kept zero)
+  // one diagnose's upload (row table | tile -> row | segments): one pinned
+  // buffer, one device buffer, one copy
+  unsigned char* h_up = nullptr;
+  unsigned char* d_up = nullptr;
+  size_t up_cap = 0;
   size_t done_cap = 0;
   unsigned long long* d_cnt = nullptr;
   xpl_alloc_report* d_rep = nullptr;
@@ -1040,17 +1039,13 @@ xpl_status xpl_finalize(xpl_ctx* c) {
   cudaFree(c->d_stage);
   cudaFreeHost(c->h_ranges);
   cudaFree(c->d_ranges);
-  cudaFreeHost(c->h_drows);
-  cudaFree(c->d_drows);
-  cudaFreeHost(c->h_tile_row);
-  cudaFree(c->d_tile_row);
   cudaFree(c->d_tiles);
   cudaFree(c->d_blk);
-  cudaFreeHost(c->h_segs);
-  cudaFree(c->d_segs);
   cudaFree(c->d_segsum);
   cudaFree(c->d_segcnt);
   cudaFree(c->d_done);
+  cudaFreeHost(c->h_up);
+  cudaFree(c->d_up);
   cudaFree(c->d_cnt);
   cudaFree(c->d_rep);
   cudaFreeHost(c->h_rep);
@@ -1709,8 +1704,6 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
   }
   if (ntiles > 0x7FFFFFFFull) return XPL_ERR_OOM;
   if (nr > c->drows_cap) {
-    cudaFreeHost(c->h_drows);
-    cudaFree(c->d_drows);
     cudaFree(c->d_cnt);
     cudaFree(c->d_rep);
     cudaFreeHost(c->h_rep);
@@ -1718,8 +1711,6 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
     cudaFreeHost(c->h_rpart);
     cudaFreeHost(c->h_cnt);
     c->drows_cap = std::max<size_t>(nr, 256);
-    CK(host_alloc(&c->h_drows, c->drows_cap));
-    CK(cudaMalloc(&c->d_drows, sizeof(DiagRow) * c->drows_cap));
     CK(cudaMalloc(&c->d_cnt, sizeof(unsigned long long) * C_NCNT * c->drows_cap));
     CK(cudaMalloc(&c->d_rep, sizeof(xpl_alloc_report) * c->drows_cap));
     CK(host_alloc(&c->h_rep, c->drows_cap));
@@ -1728,22 +1719,14 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
     CK(host_alloc(&c->h_cnt, C_NCNT * c->drows_cap));
   }
   if (ntiles > c->tiles_cap) {
-    cudaFreeHost(c->h_tile_row);
-    cudaFree(c->d_tile_row);
     cudaFree(c->d_tiles);
     c->tiles_cap = std::max<uint64_t>(ntiles, 1024);
-    CK(host_alloc(&c->h_tile_row, c->tiles_cap));
-    CK(cudaMalloc(&c->d_tile_row, sizeof(uint32_t) * c->tiles_cap));
     CK(cudaMalloc(&c->d_tiles, sizeof(TileSum) * c->tiles_cap));
   }
   if (nseg > c->segs_cap) {
-    cudaFreeHost(c->h_segs);
-    cudaFree(c->d_segs);
     cudaFree(c->d_segsum);
     cudaFree(c->d_segcnt);
     c->segs_cap = std::max<uint64_t>(nseg, 1024);
-    CK(host_alloc(&c->h_segs, c->segs_cap));
-    CK(cudaMalloc(&c->d_segs, sizeof(StitchSeg) * c->segs_cap));
     CK(cudaMalloc(&c->d_segsum, kRunPairBytes * c->segs_cap));
     CK(cudaMalloc(&c->d_segcnt, sizeof(unsigned long long) * 9 * c->segs_cap));
   }
@@ -1752,6 +1735,25 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
     c->blk_cap = std::max<uint64_t>(nblocks, 1024);
     CK(cudaMalloc(&c->d_blk, sizeof(uint32_t) * c->blk_cap));
   }
+  auto al = [](size_t b) { return (b + 255) & ~(size_t)255; };
+  const size_t o_tr = al(sizeof(DiagRow) * nr), o_sg = o_tr + al(sizeof(uint32_t) * ntiles);
+  const size_t up_bytes = o_sg + sizeof(StitchSeg) * nseg;
+  if (up_bytes > c->up_cap) {
+    if (c->d_up) {
+      CK(cudaStreamSynchronize(c->cs));
+      cudaFreeHost(c->h_up);
+      cudaFree(c->d_up);
+    }
+    c->up_cap = std::max<size_t>(up_bytes + up_bytes / 2, 1 << 16);
+    CK(host_alloc(&c->h_up, c->up_cap));
+    CK(cudaMalloc(&c->d_up, c->up_cap));
+  }
+  DiagRow* const h_drows = reinterpret_cast<DiagRow*>(c->h_up);
+  uint32_t* const h_tile_row = reinterpret_cast<uint32_t*>(c->h_up + o_tr);
+  StitchSeg* const h_segs = reinterpret_cast<StitchSeg*>(c->h_up + o_sg);
+  const DiagRow* const d_drows = reinterpret_cast<const DiagRow*>(c->d_up);
+  const uint32_t* const d_tile_row = reinterpret_cast<const uint32_t*>(c->d_up + o_tr);
+  const StitchSeg* const d_segs = reinterpret_cast<const StitchSeg*>(c->d_up + o_sg);
   // fused stitch (tile kernel + one stitch kernel): no block counts, no empty row
   bool fused = B == 0 && getenv("XPL_DIAG_UNFUSED") == nullptr;
   for (uint64_t id : ids) fused = fused && c->rows[id].words > 0;
@@ -1767,7 +1769,7 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
   uint64_t t = 0, b = 0, sgi = 0;
   for (size_t i = 0; i < nr; ++i) {
     const Row& r = c->rows[ids[i]];
-    DiagRow& d = c->h_drows[i];
+    DiagRow& d = h_drows[i];
     d.off = r.off;
     d.words = r.words;
     d.tile0 = t;
@@ -1781,25 +1783,22 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
     d.seg0 = sgi;
     d.nseg = (d.ntiles + kSegTiles - 1) / kSegTiles;
     for (uint64_t k = 0; k < d.nseg; ++k) {
-      c->h_segs[sgi + k].t0 = t + k * kSegTiles;
-      c->h_segs[sgi + k].n = std::min<uint64_t>(kSegTiles, d.ntiles - k * kSegTiles);
-      c->h_segs[sgi + k].row = i;
+      h_segs[sgi + k].t0 = t + k * kSegTiles;
+      h_segs[sgi + k].n = std::min<uint64_t>(kSegTiles, d.ntiles - k * kSegTiles);
+      h_segs[sgi + k].row = i;
     }
-    for (uint64_t k = 0; k < d.ntiles; ++k) c->h_tile_row[t + k] = (uint32_t)i;
+    for (uint64_t k = 0; k < d.ntiles; ++k) h_tile_row[t + k] = (uint32_t)i;
     sgi += d.nseg;
     t += d.ntiles;
     b += d.nblk;
   }
-  CK(cudaMemcpyAsync(c->d_drows, c->h_drows, sizeof(DiagRow) * nr, cudaMemcpyHostToDevice, c->cs));
-  CK(cudaMemcpyAsync(c->d_tile_row, c->h_tile_row, sizeof(uint32_t) * ntiles,
-                     cudaMemcpyHostToDevice, c->cs));
-  CK(cudaMemcpyAsync(c->d_segs, c->h_segs, sizeof(StitchSeg) * nseg, cudaMemcpyHostToDevice, c->cs));
+  CK(cudaMemcpyAsync(c->d_up, c->h_up, up_bytes, cudaMemcpyHostToDevice, c->cs));
   const uint64_t dbytes = total_words * (reset ? 2 : 1);
   const int pall = prof_begin(c, XPL_K_DIAGNOSE, dbytes);
   const int ptile = prof_begin(c, XPL_K_DIAG_TILE, dbytes, false);  // recorded by launch_diag
   // fused: the kernel writes the report rows (and partials, counters, the
   // epoch-split flags) straight into the pinned host buffers -- no copies back
-  launch_diag(c->cs, c->d_drows, (uint32_t)nr, c->d_tile_row, ntiles, c->d_segs, (uint32_t)nseg,
+  launch_diag(c->cs, d_drows, (uint32_t)nr, d_tile_row, ntiles, d_segs, (uint32_t)nseg,
               nblocks, p, (uint32_t*)c->d_pool, fused ? c->h_cnt : c->d_cnt, c->d_tiles, c->d_segsum, c->d_blk,
               fused ? c->h_rep : c->d_rep, pout ? (fused ? c->h_rpart : c->d_rpart) : nullptr,
               ptile >= 0 ? c->prof_pending[ptile].a : nullptr, ptile >= 0 ? c->prof_pending[ptile].b : nullptr,
@@ -1843,7 +1842,7 @@ static xpl_status diagnose_impl(xpl_ctx* c, const xpl_diag_params* params, const
       out[i] = o;
     }
     if (pout) {
-      const DiagRow& d = c->h_drows[i];
+      const DiagRow& d = h_drows[i];
       const RowPartial& q = c->h_rpart[i];
       const unsigned long long* cn = c->h_cnt + (uint64_t)C_NCNT * i;
       xpl_partial o;
