@@ -532,7 +532,8 @@ def hook_roofline(args, hook_ms, k_instr, k_twin, ms_step, prof, peak, peak_src,
             "hook_ms_per_timestep": hook_ms,
             "timing": "CUDA events on the program's stream around each of the 1900 launches of a measurement "
                       "run in which every instrumented launch is paired with its twin (twin first on odd "
-                      "launches, second on even); per launch position the mean over the two orders of the "
+                      "launches, second on even; L2 flushed before each); per launch position the mean over "
+                      "the two orders of the "
                       "median over the timesteps of instrumented minus twin, summed over the 19 positions",
             "hook_ms_per_timestep_unpaired": hook_unpaired,
             "share_of_step": hook_ms * args.timesteps / ms_step,
@@ -696,9 +697,9 @@ def main():
     hook_unpaired = float(np.sum(np.median(ai, axis=0) - np.median(at, axis=0)))
     # paired (the headline's hook cost): one measurement run of the instrumented
     # program in which every launch also runs its twin right before or after it
-    # (alternating), both timed -- per launch position, the mean of the two
-    # orders' medians of (instrumented - twin): the unified-memory faults the
-    # first of a pair pays cancel between the orders
+    # (alternating), both timed, each after an L2 flush -- per launch position,
+    # the mean of the two orders' medians of (instrumented - twin): the
+    # unified-memory faults the first of a pair pays cancel between the orders
     c4.prepare()
     rp = c4.run(ctx, time_kernels=2)
     torch.cuda.synchronize()
