@@ -486,6 +486,11 @@ static __device__ __forceinline__ void xpld_record_fast(unsigned long long g0, u
 #ifndef XPL_HOOK_PREFETCH
 #define XPL_HOOK_PREFETCH 1
 #endif
+/* Array handles: the whole-warp consecutive-element path (xpl_array::rec_contig).
+ * A/B switch: XPL_HANDLE_CONTIG=0. */
+#ifndef XPL_HANDLE_CONTIG
+#define XPL_HANDLE_CONTIG 1
+#endif
 static __device__ __forceinline__ void xpld_prefetch(const void* p) {
 #if XPL_HOOK_PREFETCH
   asm volatile("prefetch.L1 [%0];" ::"l"(p));
@@ -537,10 +542,37 @@ struct xpl_array {
     }
 #endif
   }
+  /* A whole warp on 32 consecutive elements (i = i0 + lane: the streaming
+   * case, e.g. p[blockIdx.x * blockDim.x + threadIdx.x]) of 4- or 8-byte T,
+   * local, inside the row, the first element's words starting a shadow u32:
+   * every shadow u32 of the warp's span is covered by 4 / W whole lanes, so its
+   * record bits are known without grouping -- the group's first lane loads,
+   * tests and commits them (the same bits and test as the general path).
+   * Checked at run time (one 64-bit shuffle, one vote); false: not the case. */
+  template <unsigned K>
+  __device__ __forceinline__ bool rec_contig(unsigned long long i) const {
+    constexpr unsigned W = (unsigned)(sizeof(T) / 4);
+    if (__activemask() != 0xFFFFFFFFu) return false; /* (uniform) */
+    const unsigned lane = xpld_lane();
+    const unsigned long long b = i - lane;
+    const unsigned long long b0 = __shfl_sync(0xFFFFFFFFu, b, 0);
+    const bool ok = b == b0 && i < nel && owner == xpl_dctx.rank && ((q0 + b * W) & 3ull) == 0;
+    if (!__all_sync(0xFFFFFFFFu, ok)) return false;
+    if ((lane & (4 / W - 1)) == 0) {
+      const unsigned q = (unsigned)((q0 + i * W) >> 2);
+      xpld_put<K, true>(q, xpl_dctx.pool[q], (K & XPL_ACC_R) ? 0xFFFFFFFFu : 0u,
+                        (K & XPL_ACC_W) ? 0xFFFFFFFFu : 0u);
+    }
+    return true;
+  }
   template <unsigned K>
   __device__ __forceinline__ void rec(unsigned long long i) const {
 #ifndef XPL_OFF
     constexpr unsigned long long W = sizeof(T) / 4;
+#if XPL_HANDLE_CONTIG
+    if constexpr (sizeof(T) == 4 || sizeof(T) == 8)
+      if (rec_contig<K>(i)) return;
+#endif
     unsigned long long g0 = 1, g1 = 0;
     unsigned own = owner;
     if (i < nel) {
