@@ -91,6 +91,13 @@ static inline xpl_status xpl_device_bind(xpl_ctx* ctx) {
 /* Record byte layout ("processor of the last write ... whether a CPU or
  * GPU wrote ... whether a CPU or GPU read ... and whether the data originated on
  * the CPU or GPU"; seven bits + the pending bit P in the spare eighth). */
+/* The whole-warp consecutive-element path of the compile-time-kind hooks and
+ * the array handles (xpld_record_fast, xpl_array::rec_contig).  A/B switch:
+ * XPL_HANDLE_CONTIG=0. */
+#ifndef XPL_HANDLE_CONTIG
+#define XPL_HANDLE_CONTIG 1
+#endif
+
 #define XPLD_L 0x01u
 #define XPLD_P 0x02u
 #define XPLD_WG 0x08u
@@ -462,6 +469,22 @@ static __device__ __forceinline__ void xpld_record_fast(unsigned long long g0, u
   const bool need = hit && (cur & mine) != mine;
   const unsigned needers = __ballot_sync(act, need);
   if (!needers) return; /* uniform: nothing missing (a re-touch) */
+#if XPL_HANDLE_CONTIG
+  /* a whole warp on consecutive 4- or 8-byte elements starting a shadow u32
+   * (p[i0 + lane]): each u32 of the span is covered by 4 / W whole lanes --
+   * its first lane commits the u32's bits, no grouping (as xpl_array::rec_contig) */
+  if (act == 0xFFFFFFFFu) {
+    const unsigned w = (unsigned)(g1 - g0) + 1u;
+    const unsigned long long b = g0 - (unsigned long long)lane * w;
+    const unsigned long long b0 = __shfl_sync(0xFFFFFFFFu, b, 0);
+    const unsigned w0 = __shfl_sync(0xFFFFFFFFu, w, 0);
+    if (__all_sync(0xFFFFFFFFu, hit && b == b0 && w == w0 && w <= 2u && (b & 3ull) == 0)) {
+      if ((lane & (4u / w - 1u)) == 0)
+        xpld_put<K, TM>(q, cur, (K & XPL_ACC_R) ? 0xFFFFFFFFu : 0u, (K & XPL_ACC_W) ? 0xFFFFFFFFu : 0u);
+      return;
+    }
+  }
+#endif
   const unsigned grp = __match_any_sync(act, need ? q : 0xFFFFFFFFu) & needers;
 #if XPL_FAST_ALONE  /* A/B: scattered warps (every needer alone on its u32) commit at once */
   if (__all_sync(act, !need || grp == (1u << lane))) {
@@ -486,11 +509,7 @@ static __device__ __forceinline__ void xpld_record_fast(unsigned long long g0, u
 #ifndef XPL_HOOK_PREFETCH
 #define XPL_HOOK_PREFETCH 1
 #endif
-/* Array handles: the whole-warp consecutive-element path (xpl_array::rec_contig).
- * A/B switch: XPL_HANDLE_CONTIG=0. */
-#ifndef XPL_HANDLE_CONTIG
-#define XPL_HANDLE_CONTIG 1
-#endif
+
 static __device__ __forceinline__ void xpld_prefetch(const void* p) {
 #if XPL_HOOK_PREFETCH
   asm volatile("prefetch.L1 [%0];" ::"l"(p));
