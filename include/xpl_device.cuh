@@ -97,6 +97,12 @@ static inline xpl_status xpl_device_bind(xpl_ctx* ctx) {
 #ifndef XPL_HANDLE_CONTIG
 #define XPL_HANDLE_CONTIG 1
 #endif
+/* The same check on the plain hooks' path (after the lookup): measured neutral
+ * on streams and up to 10 % slower on gather kernels (profiles/r2z_contig_ab.txt),
+ * so off by default. */
+#ifndef XPL_PLAIN_CONTIG
+#define XPL_PLAIN_CONTIG 0
+#endif
 
 #define XPLD_L 0x01u
 #define XPLD_P 0x02u
@@ -469,7 +475,7 @@ static __device__ __forceinline__ void xpld_record_fast(unsigned long long g0, u
   const bool need = hit && (cur & mine) != mine;
   const unsigned needers = __ballot_sync(act, need);
   if (!needers) return; /* uniform: nothing missing (a re-touch) */
-#if XPL_HANDLE_CONTIG
+#if XPL_PLAIN_CONTIG
   /* a whole warp on consecutive 4- or 8-byte elements starting a shadow u32
    * (p[i0 + lane]): each u32 of the span is covered by 4 / W whole lanes --
    * its first lane commits the u32's bits, no grouping (as xpl_array::rec_contig) */
