@@ -636,6 +636,81 @@ struct xpl_array {
   }
 };
 
+/* A one-deep hook pipeline for an instrumented thread's straight-line code
+ * (one object per thread, e.g. a local at the top of the kernel):
+ * p.read(x) / p.write(x) / p.rw(x) record the same bits as xpl_read / _write /
+ * _rw, but a hook's commit (test before set, grouping, atomicOr) runs at the
+ * thread's NEXT hook, or when the object dies: its shadow load is in flight
+ * while the thread goes on to its next access, instead of stalling it (a GPU
+ * warp issues in order, so with immediate commits every hook costs one full
+ * memory latency; kernels with a dozen hooks per thread are latency-bound by
+ * them).  Record order inside an epoch does not matter (D5), so deferring the
+ * commit within the kernel changes nothing.  Accesses that are not local and
+ * inside one shadow u32 take the general path at once.  Commits group lanes by
+ * shadow u32 with per-lane kinds (a lane's pending access may come from another
+ * call site than its neighbours' after divergence).  Warp-synchronous like every
+ * hook: all lanes that made a hook must reach the next one (or the object's end)
+ * together with the lanes of their warp that are active there. */
+struct xpl_pipe {
+#ifndef XPL_OFF
+  unsigned pq = 0, pcur = 0, pbm = 0, pk = 0;  /* pending: shadow u32, its value, byte lanes, kind */
+#endif
+  __device__ __forceinline__ xpl_pipe() {}
+  xpl_pipe(const xpl_pipe&) = delete;
+  xpl_pipe& operator=(const xpl_pipe&) = delete;
+  __device__ __forceinline__ ~xpl_pipe() { complete(); }
+  __device__ __forceinline__ void complete() {
+#ifndef XPL_OFF
+    const unsigned act = __activemask();
+    const unsigned m = xpld_bits(pcur, pbm, pk);
+    const bool need = pk != 0 && (pcur & m) != m;
+    const unsigned needers = __ballot_sync(act, need);
+    if (need) xpld_commit<0, false, true>(needers, pq, pcur, pbm, pk);
+    pk = 0;
+#endif
+  }
+  template <unsigned K>
+  __device__ __forceinline__ void hook(const void* x, unsigned size) {
+#ifndef XPL_OFF
+    const unsigned long long a = (unsigned long long)x;
+    ulonglong2 be, ow;
+    unsigned long long g0 = 1, g1 = 0;
+    unsigned owner = xpl_dctx.rank;
+    if (xpld_find(a, be, ow) && size > 0) xpld_words(a, size, be.x, be.y, ow.x, g0, g1, owner);
+    const unsigned act = __activemask();
+    const bool hit = g0 <= g1;
+    const bool fast = !hit || (owner == xpl_dctx.rank && (g0 ^ g1) < 4ull);
+    if (__ballot_sync(act, !fast)) { /* uniform: the general path, now */
+      xpld_record_words<K>(g0, g1, owner, K);
+      return;
+    }
+    const unsigned q = (unsigned)(g0 >> 2);
+    const unsigned bm = hit ? (0xFFFFFFFFu >> (24 - 8 * (unsigned)(g1 - g0))) << (8 * ((unsigned)g0 & 3u)) : 0u;
+    const unsigned cur = hit ? xpl_dctx.pool[q] : 0u; /* in flight during the commit below */
+    complete();
+    pq = q;
+    pcur = cur;
+    pbm = bm;
+    pk = hit ? K : 0u;
+#endif
+  }
+  template <class T>
+  __device__ __forceinline__ const T& read(const T& x) {
+    hook<XPL_ACC_R>(&x, sizeof(T));
+    return x;
+  }
+  template <class T>
+  __device__ __forceinline__ T& write(T& x) {
+    hook<XPL_ACC_W>(&x, sizeof(T));
+    return x;
+  }
+  template <class T>
+  __device__ __forceinline__ T& rw(T& x) {
+    hook<XPL_ACC_RW>(&x, sizeof(T));
+    return x;
+  }
+};
+
 /* Generic form: acc may differ from lane to lane. */
 static __device__ __forceinline__ void xpl_dev_record(const void* p, unsigned size, unsigned acc) {
   xpl_dev_record_k<0>(p, size, acc);

@@ -114,9 +114,30 @@ __device__ __forceinline__ void count_hooks(unsigned long long* hc, unsigned c) 
 }
 
 // every traced access goes through one of these (and is counted)
+#ifndef XPL_LULESH_PIPE
+#define XPL_LULESH_PIPE 0
+#endif
+#if XPL_LULESH_PIPE
+// the plain hooks through a one-deep pipeline (xpl_pipe: each commit deferred
+// to the thread's next hook, so consecutive shadow loads overlap); A/B switch
+template <bool I>
+struct Pipe : xpl_pipe {};
+template <>
+struct Pipe<false> {
+  template <class T> __device__ __forceinline__ const T& read(const T& x) { return x; }
+  template <class T> __device__ __forceinline__ T& write(T& x) { return x; }
+  template <class T> __device__ __forceinline__ T& rw(T& x) { return x; }
+};
+#define R_(x) (++c, xp_.read(x))
+#define W_(x) (++c, xp_.write(x))
+#define RW_(x) (++c, xp_.rw(x))
+#define PIPE_DECL Pipe<I> xp_
+#else
 #define R_(x) (++c, RD<I>(x))
 #define W_(x) (++c, WR<I>(x))
 #define RW_(x) (++c, RW<I>(x))
+#define PIPE_DECL
+#endif
 #define PTR(T, slot) static_cast<T*>(R_(d->ptr[slot]))
 #define ARR(T, slot) Arr<I, T>(PTR(T, slot))
 #define RA_(h, i) (++c, (h).read(i))
@@ -129,6 +150,7 @@ template <bool I>
 __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_zero_forces(Part P_, Dom* d, int nn, unsigned long long* hc) {
   const int n = P_.n0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
+  PIPE_DECL;
   if (n < P_.n1 && n < nn) {
     double *fx = PTR(double, FX), *fy = PTR(double, FY), *fz = PTR(double, FZ);
     W_(fx[n]) = 0.0;
@@ -143,6 +165,7 @@ template <bool I>
 __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_integrate_stress(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
+  PIPE_DECL;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const auto nl = ARR(const int, NODELIST);
     const auto x = ARR(const double, X), y = ARR(const double, Y), z = ARR(const double, Z);
@@ -164,6 +187,7 @@ template <bool I>
 __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_hourglass(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
+  PIPE_DECL;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const auto nl = ARR(const int, NODELIST);
     const auto xd = ARR(const double, XD), yd = ARR(const double, YD), zd = ARR(const double, ZD);
@@ -186,6 +210,7 @@ template <bool I>
 __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_corner_sum(Part P_, Dom* d, int nn, unsigned long long* hc) {
   const int n = P_.n0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
+  PIPE_DECL;
   if (n < P_.n1 && n < nn) {
     const auto st = ARR(const int, NODEELEMSTART), cl = ARR(const int, CORNERLIST);
     const auto f = ARR(const double, TMP_FORCE);
@@ -210,6 +235,7 @@ template <bool I>
 __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_accel(Part P_, Dom* d, int nn, unsigned long long* hc) {
   const int n = P_.n0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
+  PIPE_DECL;
   if (n < P_.n1 && n < nn) {
     const double m = R_(PTR(const double, NODALMASS)[n]);
     const double ax = R_(PTR(const double, FX)[n]) / m, ay = R_(PTR(const double, FY)[n]) / m,
@@ -226,6 +252,7 @@ template <bool I>
 __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_symm(Part P_, Dom* d, int ns, unsigned long long* hc) {
   const int k = P_.s0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
+  PIPE_DECL;
   if (k < P_.s1 && k < ns) {
     const int n = R_(PTR(const int, SYMMX)[k]);
     W_(PTR(double, XDD)[n]) = 0.0;
@@ -240,6 +267,7 @@ template <bool I>
 __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_velocity(Part P_, Dom* d, int nn, unsigned long long* hc) {
   const int n = P_.n0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
+  PIPE_DECL;
   if (n < P_.n1 && n < nn) {
     const double dt = R_(d->dt);
     const double ax = R_(PTR(const double, XDD)[n]), ay = R_(PTR(const double, YDD)[n]),
@@ -254,6 +282,7 @@ template <bool I>
 __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_position(Part P_, Dom* d, int nn, unsigned long long* hc) {
   const int n = P_.n0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
+  PIPE_DECL;
   if (n < P_.n1 && n < nn) {
     const double dt = R_(d->dt);
     const double vx = R_(PTR(const double, XD)[n]), vy = R_(PTR(const double, YD)[n]),
@@ -270,6 +299,7 @@ template <bool I>
 __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_kinematics(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
+  PIPE_DECL;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const auto nl = ARR(const int, NODELIST);
     const auto x = ARR(const double, X), y = ARR(const double, Y), z = ARR(const double, Z);
@@ -298,6 +328,7 @@ template <bool I>
 __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_lagrange(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
+  PIPE_DECL;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const auto g = ARR(const double, TMP_DVDX);
     const double r = (RA_(g, 3 * e) + RA_(g, 3 * e + 1) + RA_(g, 3 * e + 2)) / (R_(PTR(const double, VNEW)[e]) + 1.0);
@@ -311,6 +342,7 @@ template <bool I>
 __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_monoq_grad(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
+  PIPE_DECL;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const double* vdov = PTR(const double, VDOV);
     const int m = R_(PTR(const int, LXIM)[e]), p = R_(PTR(const int, LXIP)[e]);
@@ -323,6 +355,7 @@ template <bool I>
 __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_monoq_region(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
+  PIPE_DECL;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const int bc = R_(PTR(const int, ELEMBC)[e]);
     const double r = (bc & 1 ? 0.5 : 1.0) * R_(PTR(const double, QL)[e]) * R_(PTR(const double, VDOV)[e]);
@@ -336,6 +369,7 @@ template <bool I>
 __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_eos(Part P_, Dom* d, int stage, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
+  PIPE_DECL;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const double t = R_(d->time);
     if (stage == 0) {  // energy
@@ -368,6 +402,7 @@ template <bool I>
 __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_update_volumes(Part P_, Dom* d, unsigned long long* hc) {
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
+  PIPE_DECL;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const double v = R_(PTR(const double, VNEW)[e]);
     W_(PTR(double, V)[e]) = v;
@@ -381,6 +416,7 @@ __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_dt(Part P_, Do
   __shared__ double s_min[256];
   const int e = P_.e0 + blockIdx.x * blockDim.x + threadIdx.x;
   unsigned c = 0;
+  PIPE_DECL;
   double v = 1e30;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     if (COURANT) {
