@@ -636,11 +636,11 @@ struct xpl_array {
   }
 };
 
-/* A one-deep hook pipeline for an instrumented thread's straight-line code
+/* A D-deep hook pipeline for an instrumented thread's straight-line code
  * (one object per thread, e.g. a local at the top of the kernel):
  * p.read(x) / p.write(x) / p.rw(x) record the same bits as xpl_read / _write /
- * _rw, but a hook's commit (test before set, grouping, atomicOr) runs at the
- * thread's NEXT hook, or when the object dies: its shadow load is in flight
+ * _rw, but a hook's commit (test before set, grouping, atomicOr) runs D hooks
+ * later, or when the object dies: its shadow load is in flight
  * while the thread goes on to its next access, instead of stalling it (a GPU
  * warp issues in order, so with immediate commits every hook costs one full
  * memory latency; kernels with a dozen hooks per thread are latency-bound by
@@ -651,24 +651,36 @@ struct xpl_array {
  * call site than its neighbours' after divergence).  Warp-synchronous like every
  * hook: all lanes that made a hook must reach the next one (or the object's end)
  * together with the lanes of their warp that are active there. */
+template <unsigned D = 4>
 struct xpl_pipe {
 #ifndef XPL_OFF
-  unsigned pq = 0, pcur = 0, pbm = 0, pk = 0;  /* pending: shadow u32, its value, byte lanes, kind */
+  /* pending, newest first: shadow u32, its value (load in flight), byte lanes, kind (0 = none) */
+  unsigned pq[D], pcur[D], pbm[D], pk[D];
 #endif
-  __device__ __forceinline__ xpl_pipe() {}
-  xpl_pipe(const xpl_pipe&) = delete;
-  xpl_pipe& operator=(const xpl_pipe&) = delete;
-  __device__ __forceinline__ ~xpl_pipe() { complete(); }
-  __device__ __forceinline__ void complete() {
+  __device__ __forceinline__ xpl_pipe() {
 #ifndef XPL_OFF
-    const unsigned act = __activemask();
-    const unsigned m = xpld_bits(pcur, pbm, pk);
-    const bool need = pk != 0 && (pcur & m) != m;
-    const unsigned needers = __ballot_sync(act, need);
-    if (need) xpld_commit<0, false, true>(needers, pq, pcur, pbm, pk);
-    pk = 0;
+#pragma unroll
+    for (unsigned j = 0; j < D; ++j) pq[j] = pcur[j] = pbm[j] = pk[j] = 0u;
 #endif
   }
+  xpl_pipe(const xpl_pipe&) = delete;
+  xpl_pipe& operator=(const xpl_pipe&) = delete;
+  __device__ __forceinline__ ~xpl_pipe() {
+#ifndef XPL_OFF
+#pragma unroll
+    for (unsigned j = D; j-- > 0;) commit(j);
+#endif
+  }
+#ifndef XPL_OFF
+  __device__ __forceinline__ void commit(unsigned j) {
+    const unsigned act = __activemask();
+    const unsigned m = xpld_bits(pcur[j], pbm[j], pk[j]);
+    const bool need = pk[j] != 0 && (pcur[j] & m) != m;
+    const unsigned needers = __ballot_sync(act, need);
+    if (need) xpld_commit<0, false, true>(needers, pq[j], pcur[j], pbm[j], pk[j]);
+    pk[j] = 0;
+  }
+#endif
   template <unsigned K>
   __device__ __forceinline__ void hook(const void* x, unsigned size) {
 #ifndef XPL_OFF
@@ -686,12 +698,19 @@ struct xpl_pipe {
     }
     const unsigned q = (unsigned)(g0 >> 2);
     const unsigned bm = hit ? (0xFFFFFFFFu >> (24 - 8 * (unsigned)(g1 - g0))) << (8 * ((unsigned)g0 & 3u)) : 0u;
-    const unsigned cur = hit ? xpl_dctx.pool[q] : 0u; /* in flight during the commit below */
-    complete();
-    pq = q;
-    pcur = cur;
-    pbm = bm;
-    pk = hit ? K : 0u;
+    const unsigned cur = hit ? xpl_dctx.pool[q] : 0u; /* in flight until this entry is the oldest */
+    commit(D - 1);
+#pragma unroll
+    for (unsigned j = D - 1; j > 0; --j) {
+      pq[j] = pq[j - 1];
+      pcur[j] = pcur[j - 1];
+      pbm[j] = pbm[j - 1];
+      pk[j] = pk[j - 1];
+    }
+    pq[0] = q;
+    pcur[0] = cur;
+    pbm[0] = bm;
+    pk[0] = hit ? K : 0u;
 #endif
   }
   template <class T>

@@ -118,10 +118,13 @@ __device__ __forceinline__ void count_hooks(unsigned long long* hc, unsigned c) 
 #define XPL_LULESH_PIPE 0
 #endif
 #if XPL_LULESH_PIPE
-// the plain hooks through a one-deep pipeline (xpl_pipe: each commit deferred
-// to the thread's next hook, so consecutive shadow loads overlap); A/B switch
+// the plain hooks through a hook pipeline (xpl_pipe: each commit deferred by
+// XPL_LULESH_PIPE_DEPTH hooks, so consecutive shadow loads overlap); A/B switch
+#ifndef XPL_LULESH_PIPE_DEPTH
+#define XPL_LULESH_PIPE_DEPTH 4
+#endif
 template <bool I>
-struct Pipe : xpl_pipe {};
+struct Pipe : xpl_pipe<XPL_LULESH_PIPE_DEPTH> {};
 template <>
 struct Pipe<false> {
   template <class T> __device__ __forceinline__ const T& read(const T& x) { return x; }
