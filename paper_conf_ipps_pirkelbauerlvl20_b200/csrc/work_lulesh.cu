@@ -115,13 +115,13 @@ __device__ __forceinline__ void count_hooks(unsigned long long* hc, unsigned c) 
 
 // every traced access goes through one of these (and is counted)
 #ifndef XPL_LULESH_PIPE
-#define XPL_LULESH_PIPE 0
+#define XPL_LULESH_PIPE 1  // (profiles/r2p_pipe_ab.txt: paired hook cost -25 % at depth 1)
 #endif
 #if XPL_LULESH_PIPE
 // the plain hooks through a hook pipeline (xpl_pipe: each commit deferred by
 // XPL_LULESH_PIPE_DEPTH hooks, so consecutive shadow loads overlap); A/B switch
 #ifndef XPL_LULESH_PIPE_DEPTH
-#define XPL_LULESH_PIPE_DEPTH 4
+#define XPL_LULESH_PIPE_DEPTH 1  // (depth 4 and 8 measured no better: the hooks are mostly issue-bound)
 #endif
 template <bool I>
 struct Pipe : xpl_pipe<XPL_LULESH_PIPE_DEPTH> {};
