@@ -155,10 +155,9 @@ __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_zero_forces(Pa
   unsigned c = 0;
   PIPE_DECL;
   if (n < P_.n1 && n < nn) {
-    double *fx = PTR(double, FX), *fy = PTR(double, FY), *fz = PTR(double, FZ);
-    W_(fx[n]) = 0.0;
-    W_(fy[n]) = 0.0;
-    W_(fz[n]) = 0.0;
+    WA_(ARR(double, FX), n) = 0.0;
+    WA_(ARR(double, FY), n) = 0.0;
+    WA_(ARR(double, FZ), n) = 0.0;
   }
   count_hooks<I>(hc, c);
 }
@@ -172,7 +171,7 @@ __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_integrate_stre
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const auto nl = ARR(const int, NODELIST);
     const auto x = ARR(const double, X), y = ARR(const double, Y), z = ARR(const double, Z);
-    const double sig = -(R_(PTR(const double, P)[e]) + R_(PTR(const double, Q)[e]));
+    const double sig = -(RA_(ARR(const double, P), e) + RA_(ARR(const double, Q), e));
     const auto f = ARR(double, TMP_FORCE);
     for (int k = 0; k < 8; ++k) {
       const int n = RA_(nl, 8 * e + k);
@@ -194,8 +193,8 @@ __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_hourglass(Part
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const auto nl = ARR(const int, NODELIST);
     const auto xd = ARR(const double, XD), yd = ARR(const double, YD), zd = ARR(const double, ZD);
-    const double coef = R_(PTR(const double, SS)[e]) * R_(PTR(const double, ELEMMASS)[e]) /
-                        (R_(PTR(const double, VOLO)[e]) * R_(PTR(const double, V)[e]) + 1.0);
+    const double coef = RA_(ARR(const double, SS), e) * RA_(ARR(const double, ELEMMASS), e) /
+                        (RA_(ARR(const double, VOLO), e) * RA_(ARR(const double, V), e) + 1.0);
     const auto f = ARR(double, TMP_FORCE);
     for (int k = 0; k < 8; ++k) {
       const int n = RA_(nl, 8 * e + k);
@@ -240,12 +239,12 @@ __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_accel(Part P_,
   unsigned c = 0;
   PIPE_DECL;
   if (n < P_.n1 && n < nn) {
-    const double m = R_(PTR(const double, NODALMASS)[n]);
-    const double ax = R_(PTR(const double, FX)[n]) / m, ay = R_(PTR(const double, FY)[n]) / m,
-                 az = R_(PTR(const double, FZ)[n]) / m;
-    W_(PTR(double, XDD)[n]) = ax;
-    W_(PTR(double, YDD)[n]) = ay;
-    W_(PTR(double, ZDD)[n]) = az;
+    const double m = RA_(ARR(const double, NODALMASS), n);
+    const double ax = RA_(ARR(const double, FX), n) / m, ay = RA_(ARR(const double, FY), n) / m,
+                 az = RA_(ARR(const double, FZ), n) / m;
+    WA_(ARR(double, XDD), n) = ax;
+    WA_(ARR(double, YDD), n) = ay;
+    WA_(ARR(double, ZDD), n) = az;
   }
   count_hooks<I>(hc, c);
 }
@@ -258,9 +257,9 @@ __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_symm(Part P_, 
   PIPE_DECL;
   if (k < P_.s1 && k < ns) {
     const int n = R_(PTR(const int, SYMMX)[k]);
-    W_(PTR(double, XDD)[n]) = 0.0;
-    W_(PTR(double, YDD)[n]) = 0.0;
-    W_(PTR(double, ZDD)[n]) = 0.0;
+    WA_(ARR(double, XDD), n) = 0.0;
+    WA_(ARR(double, YDD), n) = 0.0;
+    WA_(ARR(double, ZDD), n) = 0.0;
   }
   count_hooks<I>(hc, c);
 }
@@ -273,11 +272,11 @@ __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_velocity(Part 
   PIPE_DECL;
   if (n < P_.n1 && n < nn) {
     const double dt = R_(d->dt);
-    const double ax = R_(PTR(const double, XDD)[n]), ay = R_(PTR(const double, YDD)[n]),
-                 az = R_(PTR(const double, ZDD)[n]);
-    RW_(PTR(double, XD)[n]) += dt * ax;
-    RW_(PTR(double, YD)[n]) += dt * ay;
-    RW_(PTR(double, ZD)[n]) += dt * az;
+    const double ax = RA_(ARR(const double, XDD), n), ay = RA_(ARR(const double, YDD), n),
+                 az = RA_(ARR(const double, ZDD), n);
+    RWA_(ARR(double, XD), n) += dt * ax;
+    RWA_(ARR(double, YD), n) += dt * ay;
+    RWA_(ARR(double, ZD), n) += dt * az;
   }
   count_hooks<I>(hc, c);
 }
@@ -288,11 +287,11 @@ __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_position(Part 
   PIPE_DECL;
   if (n < P_.n1 && n < nn) {
     const double dt = R_(d->dt);
-    const double vx = R_(PTR(const double, XD)[n]), vy = R_(PTR(const double, YD)[n]),
-                 vz = R_(PTR(const double, ZD)[n]);
-    RW_(PTR(double, X)[n]) += dt * vx;
-    RW_(PTR(double, Y)[n]) += dt * vy;
-    RW_(PTR(double, Z)[n]) += dt * vz;
+    const double vx = RA_(ARR(const double, XD), n), vy = RA_(ARR(const double, YD), n),
+                 vz = RA_(ARR(const double, ZD), n);
+    RWA_(ARR(double, X), n) += dt * vx;
+    RWA_(ARR(double, Y), n) += dt * vy;
+    RWA_(ARR(double, Z), n) += dt * vz;
   }
   count_hooks<I>(hc, c);
 }
@@ -313,11 +312,11 @@ __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_kinematics(Par
       vol += RA_(x, n) * RA_(y, n) + RA_(z, n);
       dv += RA_(xd, n) + RA_(yd, n) + RA_(zd, n);
     }
-    const double vnew = vol / (R_(PTR(const double, VOLO)[e]) + 1.0);
-    const double vold = R_(PTR(const double, V)[e]);
-    W_(PTR(double, VNEW)[e]) = vnew;
-    W_(PTR(double, DELV)[e]) = vnew - vold;
-    W_(PTR(double, AREALG)[e]) = vol;
+    const double vnew = vol / (RA_(ARR(const double, VOLO), e) + 1.0);
+    const double vold = RA_(ARR(const double, V), e);
+    WA_(ARR(double, VNEW), e) = vnew;
+    WA_(ARR(double, DELV), e) = vnew - vold;
+    WA_(ARR(double, AREALG), e) = vol;
     const auto g = ARR(double, TMP_DVDX);
     WA_(g, 3 * e + 0) = dv;
     WA_(g, 3 * e + 1) = dv * 0.5;
@@ -334,8 +333,8 @@ __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_lagrange(Part 
   PIPE_DECL;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const auto g = ARR(const double, TMP_DVDX);
-    const double r = (RA_(g, 3 * e) + RA_(g, 3 * e + 1) + RA_(g, 3 * e + 2)) / (R_(PTR(const double, VNEW)[e]) + 1.0);
-    W_(PTR(double, VDOV)[e]) = r;
+    const double r = (RA_(g, 3 * e) + RA_(g, 3 * e + 1) + RA_(g, 3 * e + 2)) / (RA_(ARR(const double, VNEW), e) + 1.0);
+    WA_(ARR(double, VDOV), e) = r;
   }
   count_hooks<I>(hc, c);
 }
@@ -348,9 +347,9 @@ __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_monoq_grad(Par
   PIPE_DECL;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     const double* vdov = PTR(const double, VDOV);
-    const int m = R_(PTR(const int, LXIM)[e]), p = R_(PTR(const int, LXIP)[e]);
-    const double r = R_(vdov[p]) - R_(vdov[m]) + R_(PTR(const double, VNEW)[e]);
-    W_(PTR(double, QL)[e]) = r;
+    const int m = RA_(ARR(const int, LXIM), e), p = RA_(ARR(const int, LXIP), e);
+    const double r = R_(vdov[p]) - R_(vdov[m]) + RA_(ARR(const double, VNEW), e);
+    WA_(ARR(double, QL), e) = r;
   }
   count_hooks<I>(hc, c);
 }
@@ -360,9 +359,9 @@ __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_monoq_region(P
   unsigned c = 0;
   PIPE_DECL;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
-    const int bc = R_(PTR(const int, ELEMBC)[e]);
-    const double r = (bc & 1 ? 0.5 : 1.0) * R_(PTR(const double, QL)[e]) * R_(PTR(const double, VDOV)[e]);
-    W_(PTR(double, QQ)[e]) = r;
+    const int bc = RA_(ARR(const int, ELEMBC), e);
+    const double r = (bc & 1 ? 0.5 : 1.0) * RA_(ARR(const double, QL), e) * RA_(ARR(const double, VDOV), e);
+    WA_(ARR(double, QQ), e) = r;
   }
   count_hooks<I>(hc, c);
 }
@@ -377,24 +376,24 @@ __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_eos(Part P_, D
     const double t = R_(d->time);
     if (stage == 0) {  // energy
       const double w = R_(d->misc[0]) * 1e-6 + R_(d->misc[1]) * 1e-6 + R_(d->misc[2]);
-      const double de = R_(PTR(const double, DELV)[e]) *
-                        (R_(PTR(const double, P)[e]) + R_(PTR(const double, Q)[e]) +
-                         R_(PTR(const double, QQ)[e]) + R_(PTR(const double, QL)[e]));
-      RW_(PTR(double, E)[e]) += w - de;
+      const double de = RA_(ARR(const double, DELV), e) *
+                        (RA_(ARR(const double, P), e) + RA_(ARR(const double, Q), e) +
+                         RA_(ARR(const double, QQ), e) + RA_(ARR(const double, QL), e));
+      RWA_(ARR(double, E), e) += w - de;
     } else if (stage == 1) {  // pressure
       const double pmin = R_(d->misc[3]) * 1e-6 + R_(d->misc[4]);
-      const double r = pmin + R_(PTR(const double, E)[e]) / (R_(PTR(const double, VNEW)[e]) + t);
-      W_(PTR(double, P)[e]) = r;
+      const double r = pmin + RA_(ARR(const double, E), e) / (RA_(ARR(const double, VNEW), e) + t);
+      WA_(ARR(double, P), e) = r;
     } else if (stage == 2) {  // sound speed
       const double ss4o3 = R_(d->misc[5]) * 1e-6 + R_(d->misc[6]);
-      const double r = ss4o3 * (R_(PTR(const double, P)[e]) + R_(PTR(const double, E)[e])) /
-                       (R_(PTR(const double, VNEW)[e]) + 1.0);
-      W_(PTR(double, SS)[e]) = r;
+      const double r = ss4o3 * (RA_(ARR(const double, P), e) + RA_(ARR(const double, E), e)) /
+                       (RA_(ARR(const double, VNEW), e) + 1.0);
+      WA_(ARR(double, SS), e) = r;
     } else {  // artificial viscosity
       const double qstop = R_(d->misc[7]) * 1e-6 + R_(d->misc[8]) + R_(d->misc[9]);
-      const double r = qstop + R_(PTR(const double, QL)[e]) + R_(PTR(const double, QQ)[e]) +
-                       0.0 * R_(PTR(const double, P)[e]);
-      W_(PTR(double, Q)[e]) = r;
+      const double r = qstop + RA_(ARR(const double, QL), e) + RA_(ARR(const double, QQ), e) +
+                       0.0 * RA_(ARR(const double, P), e);
+      WA_(ARR(double, Q), e) = r;
     }
   }
   count_hooks<I>(hc, c);
@@ -407,8 +406,8 @@ __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_update_volumes
   unsigned c = 0;
   PIPE_DECL;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
-    const double v = R_(PTR(const double, VNEW)[e]);
-    W_(PTR(double, V)[e]) = v;
+    const double v = RA_(ARR(const double, VNEW), e);
+    WA_(ARR(double, V), e) = v;
   }
   count_hooks<I>(hc, c);
 }
@@ -423,11 +422,11 @@ __global__ void __launch_bounds__(256, I ? XPL_LULESH_MINB : 1) k_dt(Part P_, Do
   double v = 1e30;
   if (e < NE() && e < P_.e1) {  // (every thread reads numElem, as the twin counts)
     if (COURANT) {
-      const double ss = R_(PTR(const double, SS)[e]), vd = R_(PTR(const double, VDOV)[e]),
-                   ar = R_(PTR(const double, AREALG)[e]);
+      const double ss = RA_(ARR(const double, SS), e), vd = RA_(ARR(const double, VDOV), e),
+                   ar = RA_(ARR(const double, AREALG), e);
       v = ar / (ss * ss + vd * vd + 1.0);
     } else {
-      const double vd = R_(PTR(const double, VDOV)[e]);
+      const double vd = RA_(ARR(const double, VDOV), e);
       v = 1.0 / (vd * vd + 1e-3);
     }
   }
