@@ -773,7 +773,10 @@ def main():
         "diagnose_gbs": at_scale["reset"]["gbs"], "diagnose_frac": at_scale["reset"]["gbs"] / peak,
         "diagnose_gbs_no_reset": at_scale["no_reset"]["gbs"],
         "diagnose_gbs_in_step": (dg["bytes"] / (dg["ms"] / 1e3) / 1e9) if dg["ms"] else None,
-        "hook_frac_in_step": roof["frac"], "stream_hook_frac": smb["plain"]["frac"],
+        "hook_frac": roof["frac"],  # (paired, isolated: see roofline.timing)
+        "hook_ms_per_timestep": roof["hook_ms_per_timestep"],
+        "hook_ms_per_timestep_unpaired": roof.get("hook_ms_per_timestep_unpaired"),
+        "stream_hook_frac": smb["plain"]["frac"],
         "stream_slowdown": smb["plain"]["slowdown"], "stream_handles_slowdown": smb["handles"]["slowdown"],
         "stream_handles_frac": smb["handles"]["frac"],
         "slowdown_whole_program": ms_total / twin_ms, "slowdown_kernels": k_instr / k_twin,
